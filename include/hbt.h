@@ -1,0 +1,171 @@
+/* include/hbt.h — C ABI of the B200-native HB+-tree lookup library (libhbt.so).
+ *
+ * What it computes (Shahvarani & Jacobsen, SIGMOD'16; /root/reference/PAPER.md
+ * cited as P:<line>): batched point / lower-bound lookups of unsigned 32- or
+ * 64-bit keys in a B+-tree whose inner levels form the I-segment and whose
+ * leaves form the L-segment (Fig. 1), in two forms:
+ *   - IMPLICIT: breadth-first array, child j of node i of level m at
+ *     Offset[m+1] + i*F + j; inner node = F keys, last key MAX;
+ *     leaf = one 64-byte line of P = 64/(2S) (key, value) pairs.
+ *   - REGULAR: inner node = index entries + keys + child references, searched in
+ *     three accesses; big leaves of F lines sharing the pool index
+ *     of their last-level inner node.
+ * Empty key slots hold MAX = 2^n - 1.  Keys compare UNSIGNED
+ * (reading R2).  Values have the key's width (S covers "a key or a
+ * value").
+ *
+ * Result of a lookup of q: let Kd be the sorted
+ * distinct keys (duplicates in the input collapse to their LAST occurrence) and
+ * r = lower_bound(Kd, q).
+ *   found  = r < n' && Kd[r] == q
+ *   value  = found ? value of Kd[r] : 0
+ *   pos    = IMPLICIT: r (the dense L-segment slot) or HBT_POS_END if r == n';
+ *            REGULAR : the physical slot (v*F + j)*P + s of Kd[r] (big leaf v,
+ *            line j, slot s), or HBT_POS_END if r == n'.
+ *   pos_found[i] = pos | (found ? HBT_FOUND_BIT : 0)
+ *
+ * Ownership / memory: every pointer passed to hbt_bulk_build, hbt_search and
+ * hbt_bulk_update is a caller-owned DEVICE pointer (cudaMalloc / torch CUDA
+ * tensor on the current device).  hbt_search_host is the one entry point taking
+ * HOST pointers (pinned recommended).  A tree owns its device memory until
+ * hbt_destroy.
+ *
+ * Streams: `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ * stream).  hbt_bulk_build and hbt_bulk_update are host-synchronous on return;
+ * hbt_search is asynchronous on `stream`; hbt_search_host is synchronous.
+ * Concurrent hbt_search calls on one tree are allowed (read-only);
+ * hbt_bulk_update must not overlap any search on the same tree.
+ *
+ * Errors: every call returns an hbt_status; nothing throws across the ABI.  On
+ * error the tree is unchanged (for build, *out = NULL) and hbt_last_error()
+ * returns a thread-local message.  There is NO CPU fallback: without a CUDA
+ * device every compute entry point fails with HBT_ECUDA.
+ */
+#ifndef HBT_H
+#define HBT_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define HBT_API __attribute__((visibility("default")))
+#else
+#define HBT_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct hbt_tree hbt_tree;
+
+typedef enum {
+  HBT_OK = 0,
+  HBT_EINVAL = -1,        /* bad argument (NULL, host pointer where device expected, bad fanout/layout) */
+  HBT_ENOMEM = -2,        /* device allocation failed */
+  HBT_ECUDA = -3,         /* CUDA runtime error (message in hbt_last_error) */
+  HBT_ENCCL = -4,         /* NCCL error (sharded calls) */
+  HBT_EUNSUPPORTED = -5   /* valid but not supported by this build */
+} hbt_status;
+
+/* layout word: bit 0 = tree form, bits 4.. = key (= value) width */
+enum { HBT_IMPLICIT = 0x0, HBT_REGULAR = 0x1, HBT_KEY32 = 0x00, HBT_KEY64 = 0x10 };
+
+#define HBT_POS_END   0x7FFFFFFFFFFFFFFFull
+#define HBT_FOUND_BIT 0x8000000000000000ull
+
+/* Caller-owned device output arrays of length m: pos_found (uint64) and values
+ * (uint32 for HBT_KEY32, uint64 for HBT_KEY64). */
+typedef struct {
+  uint64_t* pos_found;
+  void* values;
+} hbt_out;
+
+/* A batch of updates: keys/values of the tree's width and one op
+ * byte per entry, 0 = UPSERT (insert or overwrite), 1 = DELETE (no-op if the key
+ * is absent).  The last op per key wins (reading R12).  Device pointers. */
+typedef struct {
+  const void* keys;
+  const void* values;
+  const uint8_t* ops;
+  uint64_t count;
+} hbt_batch;
+
+#define HBT_MAX_LEVELS 32
+
+typedef struct {
+  uint32_t layout;          /* HBT_IMPLICIT | HBT_REGULAR */
+  uint32_t width;           /* S in bytes: 4 or 8 */
+  uint32_t fanout;          /* F key slots per inner node */
+  uint32_t pairs_per_line;  /* P = 64 / (2S) */
+  uint64_t n_distinct;      /* n' live keys */
+  uint32_t height;          /* implicit: inner levels H; regular: upper levels U + 1 (last level) */
+  uint32_t smem_levels;     /* top levels the search kernel stages in shared memory */
+  uint64_t level_nodes[HBT_MAX_LEVELS]; /* implicit: nodes per inner level, root first;
+                                           regular: nodes per upper level, bottom first */
+  uint64_t leaf_lines;      /* implicit: L0 64-byte lines; regular: big-leaf pool size */
+  uint64_t chain_len;       /* regular: live big leaves; implicit: = leaf_lines */
+  uint64_t inner_bytes;     /* I-segment bytes on the device */
+  uint64_t leaf_bytes;      /* L-segment bytes on the device */
+} hbt_info_t;
+
+/* Segments copied out by hbt_export (for bitwise build parity in tests). */
+enum {
+  HBT_SEG_INNER = 0,       /* implicit: root-first node array, F keys of S bytes per node       */
+  HBT_SEG_LEAF = 1,        /* implicit: L0 lines of [P keys | P values];
+                              regular : pool x F lines of [P keys | P values]                    */
+  HBT_SEG_COUNT = 2,       /* regular: uint32 count per big leaf                                 */
+  HBT_SEG_LAST_KEYS = 3,   /* regular: pool x F separator keys of the last-level inner nodes      */
+  HBT_SEG_LAST_IDX = 4,    /* regular: pool x NI index entries of the last-level inner nodes      */
+  HBT_SEG_UPPER_KEYS = 5,  /* regular: upper pool x F keys                                        */
+  HBT_SEG_UPPER_IDX = 6,   /* regular: upper pool x NI index entries                              */
+  HBT_SEG_UPPER_REFS = 7,  /* regular: upper pool x F uint32 child references                     */
+  HBT_SEG_CHAIN = 8        /* regular: uint32 big-leaf pool indices in key order                  */
+};
+
+/* Build a tree from n (key, value) pairs.  keys/values: device
+ * arrays of n elements of width S (unsorted; duplicates allowed, last wins).
+ * fanout in {4, 8, 16, 32}; layout = HBT_IMPLICIT|HBT_REGULAR combined with
+ * HBT_KEY32|HBT_KEY64.  n = 0 builds the empty tree.  The inputs are copied;
+ * they may be freed after return.  Host-synchronous. */
+HBT_API int hbt_bulk_build(const void* keys, const void* values, uint64_t n, uint32_t fanout,
+                   uint32_t layout, void* stream, hbt_tree** out);
+
+/* Look up m queries (device array of width S) into out (device arrays, length
+ * m).  Asynchronous on `stream`.  m = 0 is a no-op. */
+HBT_API int hbt_search(const hbt_tree* t, const void* queries, uint64_t m, hbt_out out, void* stream);
+
+/* End-to-end lookup with HOST buffers: copies queries host->device, searches and
+ * copies results device->host, chunked so copies overlap the search (the
+ * paper's bucket pipelining + double buffering, re-done with CUDA
+ * streams).  Pinned host memory gives full PCIe/C2C bandwidth.  Synchronous;
+ * calls on one tree are serialised. */
+HBT_API int hbt_search_host(const hbt_tree* t, const void* host_queries, uint64_t m,
+                    uint64_t* host_pos_found, void* host_values, void* stream);
+
+/* Apply a batch of UPSERT/DELETE ops.  IMPLICIT: merge into the
+ * sorted pairs and rebuild.  REGULAR: per-big-leaf merge on the GPU,
+ * splits into new pool indices, removal of emptied leaves, then the upper
+ * levels are regrouped (reading R11).  Host-synchronous. */
+HBT_API int hbt_bulk_update(hbt_tree* t, const hbt_batch* batch, void* stream);
+
+HBT_API int hbt_destroy(hbt_tree* t);
+HBT_API int hbt_info(const hbt_tree* t, hbt_info_t* info);
+
+/* Copy one segment of the tree's device layout into host memory `dst` of
+ * `bytes` bytes (HBT_EINVAL if too small); *written receives the byte count. */
+HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t bytes, uint64_t* written);
+
+/* Override the shared-memory budget (bytes per CTA) and query tiling of the
+ * search kernel; 0 keeps the default.  For tuning and tests. */
+HBT_API int hbt_set_search_config(hbt_tree* t, uint32_t smem_bytes, uint32_t threads_per_cta,
+                          uint32_t ctas_per_sm);
+
+HBT_API const char* hbt_last_error(void);
+/* Library version string, e.g. "hbt 0.1 sm_100a". */
+HBT_API const char* hbt_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* HBT_H */

@@ -1,0 +1,212 @@
+"""paper_conf_sigmod_shahvaranij16_b200 — B200-native HB+-tree lookups.
+
+A thin ctypes binding of libhbt.so (include/hbt.h).  It only marshals
+arguments: every step of build, search and update runs in the library's CUDA
+kernels.  PyTorch provides device memory and streams.  There is no CPU
+fallback: importing this package without the built library raises, and every
+call on a machine without a CUDA device fails with HBTError.
+
+    import torch, paper_conf_sigmod_shahvaranij16_b200 as hbt
+    t = hbt.Tree(keys_u64_cuda, values_u64_cuda, fanout=16, layout="implicit")
+    pos_found, values = t.search(queries_u64_cuda)
+
+The result of a lookup (PAPER.md:190 node search): with Kd the
+sorted distinct keys (last duplicate wins) and r = lower_bound(Kd, q),
+found = r < n' and Kd[r] == q; pos = r for the implicit tree, the physical slot
+(v*F + j)*P + s for the regular tree, or END; pos_found = pos | found << 63.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libhbt.so")
+
+OK, EINVAL, ENOMEM, ECUDA, ENCCL, EUNSUPPORTED = 0, -1, -2, -3, -4, -5
+IMPLICIT, REGULAR, KEY32, KEY64 = 0x0, 0x1, 0x00, 0x10
+POS_END = 0x7FFFFFFFFFFFFFFF
+FOUND_BIT = 0x8000000000000000
+MAX_LEVELS = 32
+SEG_INNER, SEG_LEAF, SEG_COUNT, SEG_LAST_KEYS, SEG_LAST_IDX = 0, 1, 2, 3, 4
+SEG_UPPER_KEYS, SEG_UPPER_IDX, SEG_UPPER_REFS, SEG_CHAIN = 5, 6, 7, 8
+UPSERT, DELETE = 0, 1
+
+EXPORTED = ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
+            "hbt_info", "hbt_export", "hbt_set_search_config", "hbt_last_error", "hbt_version"]
+
+
+class HBTError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"hbt error {code}: {msg}")
+        self.code = code
+
+
+class _Out(C.Structure):
+    _fields_ = [("pos_found", C.c_void_p), ("values", C.c_void_p)]
+
+
+class _Batch(C.Structure):
+    _fields_ = [("keys", C.c_void_p), ("values", C.c_void_p), ("ops", C.c_void_p), ("count", C.c_uint64)]
+
+
+class _Info(C.Structure):
+    _fields_ = [("layout", C.c_uint32), ("width", C.c_uint32), ("fanout", C.c_uint32),
+                ("pairs_per_line", C.c_uint32), ("n_distinct", C.c_uint64), ("height", C.c_uint32),
+                ("smem_levels", C.c_uint32), ("level_nodes", C.c_uint64 * MAX_LEVELS),
+                ("leaf_lines", C.c_uint64), ("chain_len", C.c_uint64), ("inner_bytes", C.c_uint64),
+                ("leaf_bytes", C.c_uint64)]
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: build it with `make` or __graft_entry__.build() "
+                          "(there is no CPU fallback)")
+    L = C.CDLL(LIB_PATH)
+    vp, u64, u32 = C.c_void_p, C.c_uint64, C.c_uint32
+    L.hbt_bulk_build.argtypes = [vp, vp, u64, u32, u32, vp, C.POINTER(vp)]
+    L.hbt_search.argtypes = [vp, vp, u64, _Out, vp]
+    L.hbt_search_host.argtypes = [vp, vp, u64, vp, vp, vp]
+    L.hbt_bulk_update.argtypes = [vp, C.POINTER(_Batch), vp]
+    L.hbt_destroy.argtypes = [vp]
+    L.hbt_info.argtypes = [vp, C.POINTER(_Info)]
+    L.hbt_export.argtypes = [vp, u32, vp, u64, C.POINTER(u64)]
+    L.hbt_set_search_config.argtypes = [vp, u32, u32, u32]
+    L.hbt_last_error.restype = C.c_char_p
+    L.hbt_version.restype = C.c_char_p
+    for f in ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
+              "hbt_info", "hbt_export", "hbt_set_search_config"]:
+        getattr(L, f).restype = C.c_int
+    return L
+
+
+lib = _load()
+
+
+def _check(rc):
+    if rc != OK:
+        raise HBTError(rc, lib.hbt_last_error().decode(errors="replace"))
+
+
+def version() -> str:
+    return lib.hbt_version().decode()
+
+
+def _stream_ptr(stream):
+    import torch
+    s = torch.cuda.current_stream() if stream is None else stream
+    return C.c_void_p(s.cuda_stream)
+
+
+def _width(t) -> int:
+    w = t.element_size()
+    if w not in (4, 8):
+        raise ValueError("keys/values must be 32- or 64-bit integer tensors")
+    return w
+
+
+def _dtype(width):
+    import torch
+    return torch.int32 if width == 4 else torch.int64
+
+
+class Tree:
+    """A device-resident HB+-tree (implicit or regular layout)."""
+
+    def __init__(self, keys, values, fanout: int = 16, layout: str = "implicit", stream=None):
+        import torch
+        if keys.numel() and not (keys.is_cuda and values.is_cuda):
+            raise ValueError("keys/values must be CUDA tensors")
+        if keys.numel() != values.numel() or keys.element_size() != values.element_size():
+            raise ValueError("keys and values must have equal length and width")
+        self.width = _width(keys)
+        self.fanout = fanout
+        self.layout = layout
+        word = (REGULAR if layout == "regular" else IMPLICIT) | (KEY64 if self.width == 8 else KEY32)
+        keys = keys.contiguous()
+        values = values.contiguous()
+        h = C.c_void_p()
+        _check(lib.hbt_bulk_build(C.c_void_p(keys.data_ptr() if keys.numel() else 0),
+                                  C.c_void_p(values.data_ptr() if values.numel() else 0),
+                                  keys.numel(), fanout, word, _stream_ptr(stream), C.byref(h)))
+        self._h = h
+        self._torch = torch
+
+    # -- lifetime
+    def close(self):
+        if getattr(self, "_h", None) and self._h.value:
+            lib.hbt_destroy(self._h)
+            self._h = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    @property
+    def handle(self):
+        return self._h
+
+    # -- lookups
+    def search(self, queries, out_pos=None, out_vals=None, stream=None):
+        torch = self._torch
+        if queries.element_size() != self.width:
+            raise ValueError("query width differs from the tree's key width")
+        queries = queries.contiguous()
+        m = queries.numel()
+        if out_pos is None:
+            out_pos = torch.empty(m, dtype=torch.int64, device=queries.device)
+        if out_vals is None:
+            out_vals = torch.empty(m, dtype=_dtype(self.width), device=queries.device)
+        if m:
+            _check(lib.hbt_search(self._h, C.c_void_p(queries.data_ptr()), m,
+                                  _Out(out_pos.data_ptr(), out_vals.data_ptr()), _stream_ptr(stream)))
+        return out_pos, out_vals
+
+    def search_host(self, queries, out_pos, out_vals, stream=None):
+        """End-to-end lookups from/to HOST buffers (numpy arrays or pinned CPU tensors)."""
+        def ptr(a):
+            return a.ctypes.data if isinstance(a, np.ndarray) else a.data_ptr()
+        m = len(queries)
+        _check(lib.hbt_search_host(self._h, C.c_void_p(ptr(queries)), m, C.c_void_p(ptr(out_pos)),
+                                   C.c_void_p(ptr(out_vals)), _stream_ptr(stream)))
+        return out_pos, out_vals
+
+    # -- updates
+    def update(self, keys, values, ops, stream=None):
+        keys, values, ops = keys.contiguous(), values.contiguous(), ops.contiguous()
+        b = _Batch(keys.data_ptr() if keys.numel() else 0, values.data_ptr() if values.numel() else 0,
+                   ops.data_ptr() if ops.numel() else 0, keys.numel())
+        _check(lib.hbt_bulk_update(self._h, C.byref(b), _stream_ptr(stream)))
+
+    # -- introspection
+    def info(self) -> dict:
+        i = _Info()
+        _check(lib.hbt_info(self._h, C.byref(i)))
+        d = {f: getattr(i, f) for f, _ in _Info._fields_ if f != "level_nodes"}
+        nl = i.height if i.layout == IMPLICIT else max(i.height - 1, 0)
+        d["level_nodes"] = [i.level_nodes[k] for k in range(nl)]
+        return d
+
+    def export(self, segment: int) -> np.ndarray:
+        """Raw bytes of one device segment (uint8 numpy array)."""
+        need = C.c_uint64(0)
+        rc = lib.hbt_export(self._h, segment, C.c_void_p(1), 0, C.byref(need))
+        if rc != OK and need.value == 0:
+            _check(rc)
+        buf = np.empty(max(need.value, 1), np.uint8)
+        _check(lib.hbt_export(self._h, segment, C.c_void_p(buf.ctypes.data), buf.nbytes, C.byref(need)))
+        return buf[: need.value]
+
+    def set_search_config(self, smem_bytes: int = 0, threads_per_cta: int = 0, ctas_per_sm: int = 0):
+        _check(lib.hbt_set_search_config(self._h, smem_bytes, threads_per_cta, ctas_per_sm))
+
+
+def unpack(pos_found, values, width: int):
+    """Split device results into numpy (pos, found, value) with unsigned views."""
+    pf = pos_found.cpu().numpy().view(np.uint64)
+    vals = values.cpu().numpy().view(np.uint32 if width == 4 else np.uint64)
+    return pf, vals

@@ -1,0 +1,248 @@
+// api.cu — the C ABI of libhbt.so (include/hbt.h): argument validation,
+// handle ownership, dispatch to the implicit / regular paths, the chunked
+// host-buffer pipeline and error reporting.  Every compute step runs in this
+// library's CUDA kernels (or CUB device primitives for the build's sort); there
+// is no CPU fallback.
+#include <stdarg.h>
+#include <stdio.h>
+
+#include <string>
+
+#include "hbt_internal.cuh"
+
+namespace hbt {
+
+static thread_local std::string g_err;
+
+void set_error(const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+}
+
+static bool is_device_ptr(const void* p) {
+  if (!p) return false;
+  cudaPointerAttributes a;
+  cudaError_t e = cudaPointerGetAttributes(&a, p);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+static void free_tree(hbt_tree* t) {
+  if (!t) return;
+  cudaFree(t->d_inner);
+  cudaFree(t->d_leaf);
+  regular_free(t);
+  cudaFree(t->pipe.d_q);
+  cudaFree(t->pipe.d_pf);
+  cudaFree(t->pipe.d_v);
+  for (int i = 0; i < 2; ++i) {
+    if (t->pipe.s[i]) cudaStreamDestroy(t->pipe.s[i]);
+    if (t->pipe.ev[i]) cudaEventDestroy(t->pipe.ev[i]);
+  }
+  delete t;
+}
+
+static int device_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+  return t->form == HBT_REGULAR ? regular_search(t, q, m, pf, v, s) : implicit_search(t, q, m, pf, v, s);
+}
+
+}  // namespace hbt
+
+using namespace hbt;
+
+extern "C" {
+
+const char* hbt_last_error(void) { return g_err.c_str(); }
+
+const char* hbt_version(void) { return "hbt 0.1 (HB+-tree lookups, sm_100a)"; }
+
+int hbt_bulk_build(const void* keys, const void* values, uint64_t n, uint32_t fanout, uint32_t layout,
+                   void* stream, hbt_tree** out) {
+  g_err.clear();
+  if (!out) { set_error("out is NULL"); return HBT_EINVAL; }
+  *out = nullptr;
+  const uint32_t form = layout & 0x1;
+  const uint32_t wbits = layout & 0xF0;
+  if ((layout & ~0x11u) != 0 || (wbits != HBT_KEY32 && wbits != HBT_KEY64)) {
+    set_error("bad layout word 0x%x", layout);
+    return HBT_EINVAL;
+  }
+  if (fanout != 4 && fanout != 8 && fanout != 16 && fanout != 32) {
+    set_error("fanout must be 4, 8, 16 or 32 (got %u)", fanout);
+    return HBT_EINVAL;
+  }
+  if (n >= (1ull << 32)) { set_error("n must be < 2^32"); return HBT_EUNSUPPORTED; }
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) { set_error("no CUDA device: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
+  if (n > 0 && (!is_device_ptr(keys) || !is_device_ptr(values))) {
+    set_error("keys/values must be device pointers");
+    return HBT_EINVAL;
+  }
+  hbt_tree* t = new hbt_tree();
+  t->form = form;
+  t->width = wbits == HBT_KEY64 ? 8 : 4;
+  t->F = fanout;
+  t->P = 64 / (2 * t->width);
+  t->device = dev;
+  cudaDeviceGetAttribute(&t->num_sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaStream_t s = (cudaStream_t)stream;
+  int rc = form == HBT_REGULAR ? regular_build(t, keys, values, n, s) : implicit_build(t, keys, values, n, s);
+  if (rc != HBT_OK) {
+    free_tree(t);
+    return rc;
+  }
+  *out = t;
+  return HBT_OK;
+}
+
+int hbt_search(const hbt_tree* t, const void* queries, uint64_t m, hbt_out out, void* stream) {
+  if (!t) { set_error("tree is NULL"); return HBT_EINVAL; }
+  if (m == 0) return HBT_OK;
+  if (!is_device_ptr(queries) || !is_device_ptr(out.pos_found) || !is_device_ptr(out.values)) {
+    set_error("queries/out must be device pointers");
+    return HBT_EINVAL;
+  }
+  return device_search(t, queries, m, out.pos_found, out.values, (cudaStream_t)stream);
+}
+
+int hbt_search_host(const hbt_tree* t, const void* host_queries, uint64_t m, uint64_t* host_pos_found,
+                    void* host_values, void* stream) {
+  if (!t) { set_error("tree is NULL"); return HBT_EINVAL; }
+  if (m == 0) return HBT_OK;
+  if (!host_queries || !host_pos_found || !host_values) { set_error("NULL host buffer"); return HBT_EINVAL; }
+  HostPipe& p = t->pipe;
+  std::lock_guard<std::mutex> lock(p.mu);
+  const uint64_t S = t->width;
+  const uint64_t chunk = uint64_t(1) << 22;  // 4 Mi queries per bucket
+  if (!p.chunk) {
+    HBT_CUDA_TRY(cudaMalloc(&p.d_q, 2 * chunk * S));
+    HBT_CUDA_TRY(cudaMalloc(&p.d_pf, 2 * chunk * sizeof(uint64_t)));
+    HBT_CUDA_TRY(cudaMalloc(&p.d_v, 2 * chunk * S));
+    for (int i = 0; i < 2; ++i) {
+      HBT_CUDA_TRY(cudaStreamCreateWithFlags(&p.s[i], cudaStreamNonBlocking));
+      HBT_CUDA_TRY(cudaEventCreateWithFlags(&p.ev[i], cudaEventDisableTiming));
+    }
+    p.chunk = chunk;
+  }
+  // Order after the caller's stream.
+  cudaStream_t cs = (cudaStream_t)stream;
+  HBT_CUDA_TRY(cudaEventRecord(p.ev[0], cs));
+  for (int i = 0; i < 2; ++i) HBT_CUDA_TRY(cudaStreamWaitEvent(p.s[i], p.ev[0], 0));
+  // Buckets alternate between two (stream, buffer) pairs: bucket c+1's H2D copy
+  // overlaps bucket c's search and bucket c-1's D2H copy.
+  const char* hq = (const char*)host_queries;
+  char* hv = (char*)host_values;
+  uint64_t c = 0;
+  for (uint64_t off = 0; off < m; off += chunk, ++c) {
+    const uint64_t len = (m - off < chunk) ? (m - off) : chunk;
+    const int b = int(c & 1);
+    cudaStream_t s = p.s[b];
+    char* dq = (char*)p.d_q + b * chunk * S;
+    uint64_t* dpf = p.d_pf + b * chunk;
+    char* dv = (char*)p.d_v + b * chunk * S;
+    HBT_CUDA_TRY(cudaMemcpyAsync(dq, hq + off * S, len * S, cudaMemcpyHostToDevice, s));
+    int rc = device_search(t, dq, len, dpf, dv, s);
+    if (rc != HBT_OK) return rc;
+    HBT_CUDA_TRY(cudaMemcpyAsync(host_pos_found + off, dpf, len * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    HBT_CUDA_TRY(cudaMemcpyAsync(hv + off * S, dv, len * S, cudaMemcpyDeviceToHost, s));
+  }
+  for (int i = 0; i < 2; ++i) HBT_CUDA_TRY(cudaStreamSynchronize(p.s[i]));
+  return HBT_OK;
+}
+
+int hbt_bulk_update(hbt_tree* t, const hbt_batch* batch, void* stream) {
+  if (!t || !batch) { set_error("tree/batch is NULL"); return HBT_EINVAL; }
+  if (batch->count == 0) return HBT_OK;
+  if (!is_device_ptr(batch->keys) || !is_device_ptr(batch->values) || !is_device_ptr(batch->ops)) {
+    set_error("batch arrays must be device pointers");
+    return HBT_EINVAL;
+  }
+  cudaStream_t s = (cudaStream_t)stream;
+  return t->form == HBT_REGULAR ? regular_update(t, batch, s) : implicit_update(t, batch, s);
+}
+
+int hbt_destroy(hbt_tree* t) {
+  if (!t) return HBT_EINVAL;
+  cudaDeviceSynchronize();
+  free_tree(t);
+  return HBT_OK;
+}
+
+int hbt_info(const hbt_tree* t, hbt_info_t* info) {
+  if (!t || !info) { set_error("NULL argument"); return HBT_EINVAL; }
+  *info = hbt_info_t{};
+  info->layout = t->form;
+  info->width = t->width;
+  info->fanout = t->F;
+  info->pairs_per_line = t->P;
+  info->n_distinct = t->n;
+  if (t->form == HBT_IMPLICIT) {
+    info->height = t->H;
+    info->smem_levels = implicit_smem_levels(t, t->cfg.smem_budget);
+    for (uint32_t d = 0; d < t->H; ++d) info->level_nodes[d] = t->nodes[d];
+    info->leaf_lines = t->L0;
+    info->chain_len = t->L0;
+    info->inner_bytes = t->inner_bytes;
+    info->leaf_bytes = t->leaf_bytes;
+  } else {
+    const RegularState& r = t->r;
+    info->height = r.U + 1;
+    info->smem_levels = regular_smem_levels(t, t->cfg.smem_budget);
+    for (uint32_t u = 0; u < r.U; ++u) info->level_nodes[u] = r.unodes[u];
+    info->leaf_lines = r.pool;
+    info->chain_len = r.nchain;
+    const uint64_t nip = 32 / t->width;
+    info->inner_bytes = r.uoff[r.U] * (uint64_t(t->F) * (t->width + 4) + 32) + r.pool * (uint64_t(t->F) * t->width + nip * t->width);
+    info->leaf_bytes = r.pool * uint64_t(t->F) * 64;
+  }
+  return HBT_OK;
+}
+
+int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t bytes, uint64_t* written) {
+  if (!t || !dst) { set_error("NULL argument"); return HBT_EINVAL; }
+  const void* src = nullptr;
+  uint64_t len = 0;
+  const uint64_t S = t->width, F = t->F;
+  const RegularState& r = t->r;
+  const uint64_t nip = 32 / S;  // index entries padded to one 32 B sector
+  if (t->form == HBT_IMPLICIT) {
+    if (segment == HBT_SEG_INNER) { src = t->d_inner; len = t->inner_bytes; }
+    else if (segment == HBT_SEG_LEAF) { src = t->d_leaf; len = t->leaf_bytes; }
+    else { set_error("segment %u not in an implicit tree", segment); return HBT_EINVAL; }
+  } else {
+    switch (segment) {
+      case HBT_SEG_LEAF: src = r.d_leaf; len = r.pool * F * 64; break;
+      case HBT_SEG_COUNT: src = r.d_count; len = r.pool * 4; break;
+      case HBT_SEG_LAST_KEYS: src = r.d_lkeys; len = r.pool * F * S; break;
+      case HBT_SEG_LAST_IDX: src = r.d_lidx; len = r.pool * nip * S; break;
+      case HBT_SEG_UPPER_KEYS: src = r.d_ukeys; len = r.uoff[r.U] * F * S; break;
+      case HBT_SEG_UPPER_IDX: src = r.d_uidx; len = r.uoff[r.U] * nip * S; break;
+      case HBT_SEG_UPPER_REFS: src = r.d_urefs; len = r.uoff[r.U] * F * 4; break;
+      case HBT_SEG_CHAIN: src = r.d_chain; len = r.nchain * 4; break;
+      default: set_error("segment %u not in a regular tree", segment); return HBT_EINVAL;
+    }
+  }
+  if (written) *written = len;
+  if (bytes < len) { set_error("destination too small: need %llu bytes", (unsigned long long)len); return HBT_EINVAL; }
+  if (len) HBT_CUDA_TRY(cudaMemcpy(dst, src, len, cudaMemcpyDeviceToHost));
+  return HBT_OK;
+}
+
+int hbt_set_search_config(hbt_tree* t, uint32_t smem_bytes, uint32_t threads_per_cta, uint32_t ctas_per_sm) {
+  if (!t) return HBT_EINVAL;
+  if (smem_bytes > 227 * 1024) { set_error("smem budget above 227 KB"); return HBT_EINVAL; }
+  t->cfg.smem_budget = smem_bytes;
+  t->cfg.threads = threads_per_cta;
+  t->cfg.ctas_per_sm = ctas_per_sm;
+  return HBT_OK;
+}
+
+}  // extern "C"

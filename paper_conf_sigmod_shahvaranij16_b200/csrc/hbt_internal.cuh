@@ -1,0 +1,116 @@
+// hbt_internal.cuh — shared internals of libhbt.so (the CUDA path).
+// Nothing here is shared with oracle/ (test infrastructure); see DESIGN.md §4.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <mutex>
+#include <string>
+
+#include "../../include/hbt.h"
+
+namespace hbt {
+
+void set_error(const char* fmt, ...);
+
+#define HBT_CUDA_TRY(expr)                                                              \
+  do {                                                                                  \
+    cudaError_t _e = (expr);                                                            \
+    if (_e != cudaSuccess) {                                                            \
+      ::hbt::set_error("%s:%d %s: %s", __FILE__, __LINE__, #expr, cudaGetErrorString(_e)); \
+      return _e == cudaErrorMemoryAllocation ? HBT_ENOMEM : HBT_ECUDA;                  \
+    }                                                                                   \
+  } while (0)
+
+static inline uint64_t ceil_div_u64(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+
+// Level table passed by value to the search kernels (root-first, node units).
+struct LevelTable {
+  uint64_t offset[HBT_MAX_LEVELS + 1];
+  uint32_t H;   // inner levels
+  uint32_t SL;  // levels [0, SL) staged in shared memory
+};
+
+struct SearchConfig {
+  uint32_t smem_budget = 0;      // bytes per CTA for pinned levels (0 = default)
+  uint32_t threads = 0;          // threads per CTA (0 = default)
+  uint32_t ctas_per_sm = 0;      // 0 = occupancy-derived
+};
+
+// Regular-tree device state.  All pools are SoA arrays
+// indexed by pool index (node fragmentation).
+struct RegularState {
+  uint32_t kpl = 0, NI = 0, B = 0, b = 0;
+  uint64_t pool = 0, cap = 0;            // big leaves allocated / capacity
+  void* d_leaf = nullptr;                // cap x F lines x 64 B
+  uint32_t* d_count = nullptr;           // cap
+  void* d_lkeys = nullptr;               // cap x F keys (last-level inner node)
+  void* d_lidx = nullptr;                // cap x NIP index entries (padded to 32 B)
+  uint64_t nchain = 0;
+  uint32_t* d_chain = nullptr;           // cap
+  uint32_t U = 0;                        // upper levels
+  uint64_t unodes[HBT_MAX_LEVELS] = {};  // bottom-up
+  uint64_t uoff[HBT_MAX_LEVELS + 1] = {};
+  uint64_t ucap = 0;
+  void* d_ukeys = nullptr;               // ucap x F keys
+  void* d_uidx = nullptr;                // ucap x NIP
+  uint32_t* d_urefs = nullptr;           // ucap x F
+  void* d_umax = nullptr;                // scratch: max key per node of the level being built
+};
+
+struct HostPipe {
+  std::mutex mu;
+  void* d_q = nullptr;                   // 2 x chunk queries
+  uint64_t* d_pf = nullptr;              // 2 x chunk
+  void* d_v = nullptr;                   // 2 x chunk
+  uint64_t chunk = 0;
+  cudaStream_t s[2] = {nullptr, nullptr};
+  cudaEvent_t ev[2] = {nullptr, nullptr};
+};
+
+}  // namespace hbt
+
+struct hbt_tree {
+  uint32_t form = HBT_IMPLICIT;  // HBT_IMPLICIT | HBT_REGULAR
+  uint32_t width = 8;            // S
+  uint32_t F = 16;
+  uint32_t P = 4;                // 64 / (2S)
+  uint64_t n = 0;                // n' distinct keys
+  int device = 0;
+  int num_sms = 148;
+  // ---- implicit ----
+  uint32_t H = 0;
+  uint64_t nodes[HBT_MAX_LEVELS] = {};       // root-first
+  uint64_t offset[HBT_MAX_LEVELS + 1] = {};  // root-first, node units
+  void* d_inner = nullptr;
+  uint64_t inner_bytes = 0;
+  void* d_leaf = nullptr;
+  uint64_t L0 = 0;
+  uint64_t leaf_bytes = 0;
+  // ---- regular ----
+  hbt::RegularState r;
+  // ---- search ----
+  hbt::SearchConfig cfg;
+  mutable hbt::HostPipe pipe;
+};
+
+namespace hbt {
+// implicit_build.cu
+int implicit_build(hbt_tree* t, const void* keys, const void* values, uint64_t n, cudaStream_t s);
+int implicit_build_sorted(hbt_tree* t, const void* sk, const void* sv, uint64_t n_sorted_distinct,
+                          cudaStream_t s);
+// sort (stable) + dedupe-last-wins into fresh device arrays; *nd = distinct count
+int sort_dedupe(uint32_t width, const void* keys, const void* values, uint64_t n, void** out_k,
+                void** out_v, uint64_t* nd, cudaStream_t s);
+int implicit_update(hbt_tree* t, const hbt_batch* b, cudaStream_t s);
+// implicit_search.cu
+int implicit_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s);
+uint32_t implicit_smem_levels(const hbt_tree* t, uint32_t budget);
+// regular_*.cu
+int regular_build(hbt_tree* t, const void* keys, const void* values, uint64_t n, cudaStream_t s);
+int regular_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s);
+int regular_update(hbt_tree* t, const hbt_batch* b, cudaStream_t s);
+void regular_free(hbt_tree* t);
+uint32_t regular_smem_levels(const hbt_tree* t, uint32_t budget);
+}  // namespace hbt

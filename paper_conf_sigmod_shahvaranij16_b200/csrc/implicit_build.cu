@@ -1,0 +1,311 @@
+// implicit_build.cu — hbt_bulk_build / hbt_bulk_update for the IMPLICIT tree.
+//
+// Layout:
+//   L-segment: L0 = max(1, ceil(n'/P)) lines of 64 B = [P keys | P values],
+//              rank r at line r/P slot r%P, padding (MAX, 0)
+//   I-segment: inner levels root-first, node = F keys of S bytes (F*S-byte
+//              aligned), child i of node j at level d+1 index j*F + i;
+//              key slot i = max key of child i's subtree for i < cnt-1, else MAX
+//              (reading R3; slot F-1 always MAX).
+// The separators are gathered with the closed form
+//   sep(h, j, i) = Kd[min(n', (j*F + i + 1) * F^(h-1) * P) - 1]
+// from the sorted distinct key array (one kernel for all levels), so the build
+// is: CUB radix sort (stable) -> keep-last-of-run compaction -> pack -> gather.
+#include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_select.cuh>
+
+#include "hbt_internal.cuh"
+
+namespace hbt {
+namespace {
+
+template <typename K>
+__host__ __device__ constexpr K key_max() { return K(~K(0)); }
+
+template <typename K>
+__global__ void last_of_run_flags(const K* __restrict__ sk, uint64_t n, uint8_t* __restrict__ flags) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += uint64_t(gridDim.x) * blockDim.x)
+    flags[i] = (i + 1 == n) || (sk[i] != sk[i + 1]);
+}
+
+template <typename K>
+__global__ void pack_leaf_lines(const K* __restrict__ kd, const K* __restrict__ vd, uint64_t nd, uint64_t L0,
+                                K* __restrict__ leaf) {
+  constexpr uint32_t P = 64 / (2 * sizeof(K));
+  const uint64_t total = L0 * P;
+  for (uint64_t r = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; r < total; r += uint64_t(gridDim.x) * blockDim.x) {
+    const uint64_t line = r / P, s = r % P;
+    K* L = leaf + line * (2 * P);
+    L[s] = r < nd ? kd[r] : key_max<K>();
+    L[P + s] = r < nd ? vd[r] : K(0);
+  }
+}
+
+template <typename K>
+__global__ void gather_separators(const K* __restrict__ kd, uint64_t nd, const LevelTable lt, uint64_t L0,
+                                  uint32_t F, K* __restrict__ inner) {
+  constexpr uint32_t P = 64 / (2 * sizeof(K));
+  const uint32_t H = lt.H;
+  const uint64_t total = lt.offset[H] * F;
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < total; x += uint64_t(gridDim.x) * blockDim.x) {
+    const uint64_t node = x / F;
+    const uint32_t i = uint32_t(x % F);
+    uint32_t d = 0;
+    while (node >= lt.offset[d + 1]) ++d;
+    const uint64_t j = node - lt.offset[d];
+    const uint32_t h = H - d;  // height >= 1
+    const uint64_t below = (d + 1 < H) ? (lt.offset[d + 2] - lt.offset[d + 1]) : L0;
+    const uint64_t first = j * F;
+    const uint64_t cnt = (below - first < F) ? (below - first) : F;
+    K key = key_max<K>();
+    if (i + 1 < cnt) {
+      uint64_t span = P;  // ranks covered by one child: F^(h-1) * P
+      for (uint32_t e = 1; e < h; ++e) span *= F;
+      uint64_t end = (first + i + 1) * span;
+      if (end > nd) end = nd;
+      key = kd[end - 1];
+    }
+    inner[x] = key;
+  }
+}
+
+template <typename K>
+__global__ void unpack_leaf_lines(const K* __restrict__ leaf, uint64_t nd, K* __restrict__ kd, K* __restrict__ vd) {
+  constexpr uint32_t P = 64 / (2 * sizeof(K));
+  for (uint64_t r = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; r < nd; r += uint64_t(gridDim.x) * blockDim.x) {
+    const K* L = leaf + (r / P) * (2 * P);
+    kd[r] = L[r % P];
+    vd[r] = L[P + r % P];
+  }
+}
+
+// Update merge: concatenated (base ++ batch) sorted stably by key; the last
+// element of each key run decides (base entry: keep; UPSERT: keep with the
+// op's value; DELETE: drop).  Batch entries follow base entries in the
+// concatenation, so "last" = the batch's last op on the key (reading R12).
+template <typename K>
+__global__ void merge_flags(const K* __restrict__ sk, const uint32_t* __restrict__ sidx, uint64_t total,
+                            uint64_t n_base, const uint8_t* __restrict__ ops, uint8_t* __restrict__ flags) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < total; i += uint64_t(gridDim.x) * blockDim.x) {
+    const bool last = (i + 1 == total) || (sk[i] != sk[i + 1]);
+    const uint64_t src = sidx[i];
+    const bool del = src >= n_base && ops[src - n_base] != 0;
+    flags[i] = last && !del;
+  }
+}
+
+template <typename K>
+__global__ void merge_gather_values(const uint32_t* __restrict__ sidx, uint64_t total, uint64_t n_base,
+                                    const K* __restrict__ base_v, const K* __restrict__ batch_v,
+                                    K* __restrict__ out_v) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < total; i += uint64_t(gridDim.x) * blockDim.x) {
+    const uint64_t src = sidx[i];
+    out_v[i] = src < n_base ? base_v[src] : batch_v[src - n_base];
+  }
+}
+
+__global__ void iota_u32(uint32_t* p, uint64_t n) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += uint64_t(gridDim.x) * blockDim.x)
+    p[i] = uint32_t(i);
+}
+
+inline unsigned grid_for(uint64_t n) {
+  uint64_t g = (n + 255) / 256;
+  if (g > 148 * 64) g = 148 * 64;
+  return unsigned(g ? g : 1);
+}
+
+template <typename K>
+int sort_dedupe_t(const void* keys, const void* values, uint64_t n, void** out_k, void** out_v, uint64_t* nd,
+                  cudaStream_t s) {
+  *out_k = *out_v = nullptr;
+  *nd = 0;
+  if (n == 0) return HBT_OK;
+  K *sk = nullptr, *sv = nullptr, *kd = nullptr, *vd = nullptr;
+  uint8_t* flags = nullptr;
+  void* tmp = nullptr;
+  int64_t* d_nsel = nullptr;
+  size_t tb = 0, tb2 = 0;
+  int rc = HBT_OK;
+  auto fail = [&](int code) {
+    cudaFree(sk); cudaFree(sv); cudaFree(kd); cudaFree(vd); cudaFree(flags); cudaFree(tmp); cudaFree(d_nsel);
+    return code;
+  };
+#define TRY(x)                                                                          \
+  do {                                                                                  \
+    cudaError_t _e = (x);                                                               \
+    if (_e != cudaSuccess) {                                                            \
+      set_error("%s:%d %s: %s", __FILE__, __LINE__, #x, cudaGetErrorString(_e));         \
+      return fail(_e == cudaErrorMemoryAllocation ? HBT_ENOMEM : HBT_ECUDA);            \
+    }                                                                                   \
+  } while (0)
+  TRY(cudaMalloc(&sk, n * sizeof(K)));
+  TRY(cudaMalloc(&sv, n * sizeof(K)));
+  TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb, (const K*)keys, sk, (const K*)values, sv, n, 0,
+                                      int(8 * sizeof(K)), s));
+  TRY(cub::DeviceSelect::Flagged(nullptr, tb2, sk, flags, kd, d_nsel, int64_t(n), s));
+  if (tb2 > tb) tb = tb2;
+  TRY(cudaMalloc(&tmp, tb));
+  // Stable LSD radix sort: equal keys keep input order, so the last element of
+  // each run is the key's last occurrence (dedupe-last-wins, reading R4).
+  TRY(cub::DeviceRadixSort::SortPairs(tmp, tb, (const K*)keys, sk, (const K*)values, sv, n, 0,
+                                      int(8 * sizeof(K)), s));
+  TRY(cudaMalloc(&flags, n));
+  TRY(cudaMalloc(&d_nsel, sizeof(int64_t)));
+  last_of_run_flags<K><<<grid_for(n), 256, 0, s>>>(sk, n, flags);
+  TRY(cudaGetLastError());
+  TRY(cudaMalloc(&kd, n * sizeof(K)));
+  TRY(cudaMalloc(&vd, n * sizeof(K)));
+  TRY(cub::DeviceSelect::Flagged(tmp, tb, sk, flags, kd, d_nsel, int64_t(n), s));
+  TRY(cub::DeviceSelect::Flagged(tmp, tb, sv, flags, vd, d_nsel, int64_t(n), s));
+  int64_t h_nsel = 0;
+  TRY(cudaMemcpyAsync(&h_nsel, d_nsel, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  TRY(cudaStreamSynchronize(s));
+#undef TRY
+  cudaFree(sk); cudaFree(sv); cudaFree(flags); cudaFree(tmp); cudaFree(d_nsel);
+  *out_k = kd;
+  *out_v = vd;
+  *nd = uint64_t(h_nsel);
+  (void)rc;
+  return HBT_OK;
+}
+
+template <typename K>
+int build_sorted_t(hbt_tree* t, const K* kd, const K* vd, uint64_t nd, cudaStream_t s) {
+  const uint32_t P = 64 / (2 * sizeof(K));
+  const uint32_t F = t->F;
+  t->P = P;
+  t->n = nd;
+  t->L0 = nd == 0 ? 1 : ceil_div_u64(nd, P);
+  uint64_t c[HBT_MAX_LEVELS + 2];
+  uint32_t H = 0;
+  c[0] = t->L0;
+  while (c[H] > 1) {
+    if (H + 1 >= HBT_MAX_LEVELS) { set_error("tree too tall"); return HBT_EUNSUPPORTED; }
+    c[H + 1] = ceil_div_u64(c[H], F);
+    ++H;
+  }
+  t->H = H;
+  t->offset[0] = 0;
+  for (uint32_t d = 0; d < H; ++d) {
+    t->nodes[d] = c[H - d];
+    t->offset[d + 1] = t->offset[d] + t->nodes[d];
+  }
+  t->inner_bytes = t->offset[H] * F * sizeof(K);
+  t->leaf_bytes = t->L0 * 64;
+  HBT_CUDA_TRY(cudaMalloc(&t->d_leaf, t->leaf_bytes));
+  if (t->inner_bytes) HBT_CUDA_TRY(cudaMalloc(&t->d_inner, t->inner_bytes));
+  pack_leaf_lines<K><<<grid_for(t->L0 * P), 256, 0, s>>>(kd, vd, nd, t->L0, (K*)t->d_leaf);
+  HBT_CUDA_TRY(cudaGetLastError());
+  if (H) {
+    LevelTable lt{};
+    for (uint32_t d = 0; d <= H; ++d) lt.offset[d] = t->offset[d];
+    lt.H = H;
+    gather_separators<K><<<grid_for(t->offset[H] * F), 256, 0, s>>>(kd, nd, lt, t->L0, F, (K*)t->d_inner);
+    HBT_CUDA_TRY(cudaGetLastError());
+  }
+  HBT_CUDA_TRY(cudaStreamSynchronize(s));
+  return HBT_OK;
+}
+
+template <typename K>
+int implicit_update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
+  const uint64_t nb = t->n, m = b->count, total = nb + m;
+  if (total >= (1ull << 32)) { set_error("update: n + batch must be < 2^32"); return HBT_EUNSUPPORTED; }
+  K *ck = nullptr, *sk = nullptr, *base_v = nullptr, *mv = nullptr, *kd = nullptr, *vd = nullptr;
+  uint32_t *idx = nullptr, *sidx = nullptr;
+  uint8_t* flags = nullptr;
+  int64_t* d_nsel = nullptr;
+  void* tmp = nullptr;
+  size_t tb = 0, tb2 = 0;
+  auto cleanup = [&]() {
+    cudaFree(ck); cudaFree(sk); cudaFree(base_v); cudaFree(mv); cudaFree(kd); cudaFree(vd);
+    cudaFree(idx); cudaFree(sidx); cudaFree(flags); cudaFree(d_nsel); cudaFree(tmp);
+  };
+#define TRY(x)                                                                          \
+  do {                                                                                  \
+    cudaError_t _e = (x);                                                               \
+    if (_e != cudaSuccess) {                                                            \
+      set_error("%s:%d %s: %s", __FILE__, __LINE__, #x, cudaGetErrorString(_e));         \
+      cleanup();                                                                        \
+      return _e == cudaErrorMemoryAllocation ? HBT_ENOMEM : HBT_ECUDA;                  \
+    }                                                                                   \
+  } while (0)
+  TRY(cudaMalloc(&ck, total * sizeof(K)));
+  TRY(cudaMalloc(&sk, total * sizeof(K)));
+  TRY(cudaMalloc(&base_v, (nb ? nb : 1) * sizeof(K)));
+  TRY(cudaMalloc(&mv, total * sizeof(K)));
+  TRY(cudaMalloc(&idx, total * sizeof(uint32_t)));
+  TRY(cudaMalloc(&sidx, total * sizeof(uint32_t)));
+  TRY(cudaMalloc(&flags, total));
+  TRY(cudaMalloc(&d_nsel, sizeof(int64_t)));
+  if (nb) {
+    unpack_leaf_lines<K><<<grid_for(nb), 256, 0, s>>>((const K*)t->d_leaf, nb, ck, base_v);
+    TRY(cudaGetLastError());
+  }
+  TRY(cudaMemcpyAsync(ck + nb, b->keys, m * sizeof(K), cudaMemcpyDeviceToDevice, s));
+  iota_u32<<<grid_for(total), 256, 0, s>>>(idx, total);
+  TRY(cudaGetLastError());
+  TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb, ck, sk, idx, sidx, total, 0, int(8 * sizeof(K)), s));
+  TRY(cub::DeviceSelect::Flagged(nullptr, tb2, sk, flags, ck, d_nsel, int64_t(total), s));
+  if (tb2 > tb) tb = tb2;
+  TRY(cudaMalloc(&tmp, tb));
+  TRY(cub::DeviceRadixSort::SortPairs(tmp, tb, ck, sk, idx, sidx, total, 0, int(8 * sizeof(K)), s));
+  merge_flags<K><<<grid_for(total), 256, 0, s>>>(sk, sidx, total, nb, b->ops, flags);
+  TRY(cudaGetLastError());
+  merge_gather_values<K><<<grid_for(total), 256, 0, s>>>(sidx, total, nb, base_v, (const K*)b->values, mv);
+  TRY(cudaGetLastError());
+  TRY(cudaMalloc(&kd, total * sizeof(K)));
+  TRY(cudaMalloc(&vd, total * sizeof(K)));
+  TRY(cub::DeviceSelect::Flagged(tmp, tb, sk, flags, kd, d_nsel, int64_t(total), s));
+  TRY(cub::DeviceSelect::Flagged(tmp, tb, mv, flags, vd, d_nsel, int64_t(total), s));
+  int64_t h_nsel = 0;
+  TRY(cudaMemcpyAsync(&h_nsel, d_nsel, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  TRY(cudaStreamSynchronize(s));
+#undef TRY
+  // Rebuild into a fresh layout, then swap it in.
+  hbt_tree nt;
+  nt.form = t->form; nt.width = t->width; nt.F = t->F; nt.device = t->device; nt.num_sms = t->num_sms;
+  int rc = build_sorted_t<K>(&nt, kd, vd, uint64_t(h_nsel), s);
+  cleanup();
+  if (rc != HBT_OK) { cudaFree(nt.d_leaf); cudaFree(nt.d_inner); return rc; }
+  cudaFree(t->d_leaf);
+  cudaFree(t->d_inner);
+  t->n = nt.n; t->L0 = nt.L0; t->H = nt.H; t->P = nt.P;
+  for (int d = 0; d < HBT_MAX_LEVELS; ++d) t->nodes[d] = nt.nodes[d];
+  for (int d = 0; d <= HBT_MAX_LEVELS; ++d) t->offset[d] = nt.offset[d];
+  t->d_leaf = nt.d_leaf; t->leaf_bytes = nt.leaf_bytes;
+  t->d_inner = nt.d_inner; t->inner_bytes = nt.inner_bytes;
+  nt.d_leaf = nt.d_inner = nullptr;
+  return HBT_OK;
+}
+
+}  // namespace
+
+int sort_dedupe(uint32_t width, const void* keys, const void* values, uint64_t n, void** out_k, void** out_v,
+                uint64_t* nd, cudaStream_t s) {
+  return width == 4 ? sort_dedupe_t<uint32_t>(keys, values, n, out_k, out_v, nd, s)
+                    : sort_dedupe_t<uint64_t>(keys, values, n, out_k, out_v, nd, s);
+}
+
+int implicit_build_sorted(hbt_tree* t, const void* kd, const void* vd, uint64_t nd, cudaStream_t s) {
+  return t->width == 4 ? build_sorted_t<uint32_t>(t, (const uint32_t*)kd, (const uint32_t*)vd, nd, s)
+                       : build_sorted_t<uint64_t>(t, (const uint64_t*)kd, (const uint64_t*)vd, nd, s);
+}
+
+int implicit_build(hbt_tree* t, const void* keys, const void* values, uint64_t n, cudaStream_t s) {
+  void *kd = nullptr, *vd = nullptr;
+  uint64_t nd = 0;
+  int rc = sort_dedupe(t->width, keys, values, n, &kd, &vd, &nd, s);
+  if (rc != HBT_OK) return rc;
+  rc = implicit_build_sorted(t, kd, vd, nd, s);
+  cudaFree(kd);
+  cudaFree(vd);
+  return rc;
+}
+
+int implicit_update(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
+  return t->width == 4 ? implicit_update_t<uint32_t>(t, b, s) : implicit_update_t<uint64_t>(t, b, s);
+}
+
+}  // namespace hbt

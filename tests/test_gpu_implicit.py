@@ -1,0 +1,203 @@
+"""GPU parity of the IMPLICIT tree against the oracle (bit-exact pos|found and
+value; bitwise build arrays).  Calls go through the C ABI (libhbt.so)."""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from gpu_util import (END, GenLib, expected_implicit_bytes, from_dev, gpu_build, gpu_search, np_dtype,
+                      to_dev)
+from test_oracle_implicit import gen_keys, query_set
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def hbt():
+    import paper_conf_sigmod_shahvaranij16_b200 as m
+    assert torch.cuda.is_available(), "gpu tests need a CUDA device"
+    return m
+
+
+def sizes(F, P):
+    return sorted({0, 1, 2, P - 1, P, P + 1, F * P - 1, F * P, F * P + 1, F * F * P - 1, F * F * P + 1,
+                   F * F * F * P + 3, 5000})
+
+
+@pytest.mark.parametrize("width", [4, 8])
+@pytest.mark.parametrize("F", [4, 8, 16, 32])
+def test_edge_suite_parity(hbt, width, F):
+    P = 64 // (2 * width)
+    rng = np.random.default_rng(100 * F + width)
+    for n in sizes(F, P):
+        k, v = gen_keys(n, width, rng, dup=(n % 2 == 1), with_max=(n % 3 == 0))
+        o = oracle.ITree.from_pairs(k, v, F, width)
+        t = gpu_build(hbt, k, v, F, width)
+        info = t.info()
+        a = o.arrays()
+        assert info["n_distinct"] == a["n"] and info["height"] == a["H"]
+        assert info["level_nodes"] == a["nodes"]
+        inner, leaf = expected_implicit_bytes(o, width)
+        assert t.export(hbt.SEG_INNER).tobytes() == inner, (n, F, width)
+        assert t.export(hbt.SEG_LEAF).tobytes() == leaf, (n, F, width)
+        q = query_set(k, width, rng, 3000)
+        pf, val = gpu_search(t, q, width)
+        epf, ev = o.search(q)
+        assert np.array_equal(pf, epf), (n, F, width, np.nonzero(pf != epf)[0][:5])
+        assert np.array_equal(val, ev), (n, F, width)
+        t.close()
+
+
+@pytest.mark.parametrize("budget", [16, 4096, 100 * 1024, 200 * 1024])
+def test_smem_pinning_variants(hbt, budget):
+    """Results must not depend on how many top levels sit in shared memory."""
+    width, F = 8, 16
+    rng = np.random.default_rng(budget)
+    k, v = gen_keys(300000, width, rng)
+    o = oracle.ITree.from_pairs(k, v, F, width)
+    t = gpu_build(hbt, k, v, F, width)
+    t.set_search_config(smem_bytes=budget)
+    q = query_set(k[:5000], width, rng, 20000)
+    pf, val = gpu_search(t, q, width)
+    epf, ev = o.search(q)
+    assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+
+
+def test_c1_full(hbt):
+    """BASELINE configs[0]: implicit, 2^16 u32 keys, F = 8, 2^16 Knuth-shuffled queries
+    (PAPER.md:298), plus the c1 suite: 50 % hits, 25 % random u32, 25 % edges."""
+    c = gen.CONFIGS["c1"]
+    k, v = gen.workload_keys_values("c1")
+    q = gen.workload_queries("c1", k)
+    o = oracle.ITree.from_pairs(k, v, c["fanout"], c["width"])
+    t = gpu_build(hbt, k, v, c["fanout"], c["width"])
+    pf, val = gpu_search(t, q, c["width"])
+    epf, ev = o.search(q)
+    assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+    assert (pf >> np.uint64(63)).all()  # every query hits
+    rng = np.random.default_rng(1)
+    mx = 2**32 - 1
+    kk = k.astype(np.uint64)
+    edges = np.concatenate([[0, mx, kk.min(), kk.max()], kk[:4000] + 1, kk[4000:8000] - 1]).astype(np.uint64)
+    edges = np.clip(edges, 0, mx).astype(np.uint64)
+    suite = np.concatenate([kk[rng.integers(0, len(kk), 32768)],
+                            rng.integers(0, mx, 16384, dtype=np.uint64, endpoint=True), edges[:16384]])
+    pf, val = gpu_search(t, suite, 4)
+    epf, ev = o.search(suite)
+    assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+
+
+def test_c2_scaled_full_compare(hbt):
+    """configs[1] recipe at 1/32 scale: every output compared with the oracle."""
+    n, m = 1 << 18, 1 << 19
+    k, v = gen.workload_keys_values("c2", n)
+    q = gen.workload_queries("c2", k, m)
+    o = oracle.ITree.from_pairs(k, v, 16, 8)
+    t = gpu_build(hbt, k, v, 16, 8)
+    pf, val = gpu_search(t, q, 8)
+    epf, ev = o.search(q, nthreads=oracle.default_threads())
+    assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+
+
+def test_c2_full_size_bench_launch(hbt):
+    """configs[1] at full size (2^23 u64 keys, F = 16, 2^24 uniform hit queries)
+    through the same generator/launch path bench.py times: sampled outputs vs the
+    oracle, and for ALL outputs the properties that hold at any size
+    (found, value = V_u of the generator, pos = rank of K_u)."""
+    c = gen.CONFIGS["c2"]
+    n, m, w = c["n"], c["m"], 8
+    g = GenLib()
+    sk = gen.stream_seed(2, gen.STREAM_K)
+    sv = gen.stream_seed(2, gen.STREAM_V)
+    sq = gen.stream_seed(2, gen.STREAM_Q)
+    dk = g.mix_stream(n, w, sk)
+    dv = g.mix_stream(n, w, sv)
+    dq = g.uniform_queries(m, n, w, sq, sk)
+    t = hbt.Tree(dk, dv, fanout=16, layout="implicit")
+    pf, val = t.search(dq)
+    torch.cuda.synchronize()
+    pf = pf.cpu().numpy().view(np.uint64)
+    val = from_dev(val, w)
+    # all outputs: properties
+    k = gen.keys(n, w, sk)
+    v = gen.values(n, w, sv)
+    u = gen.uniform_indices(m, n, sq).astype(np.int64)
+    order = np.argsort(k, kind="stable")
+    rank = np.empty(n, np.int64)
+    rank[order] = np.arange(n)
+    assert (pf >> np.uint64(63)).all()
+    assert np.array_equal(val, v[u])
+    assert np.array_equal((pf & np.uint64(END)).astype(np.int64), rank[u])
+    # sample: the oracle tree, one by one
+    o = oracle.ITree.from_pairs(k, v, 16, 8)
+    idx = np.random.default_rng(0).integers(0, m, 1 << 18)
+    q = from_dev(dq, w)[idx]
+    epf, ev = o.search(q, nthreads=oracle.default_threads())
+    assert np.array_equal(pf[idx], epf) and np.array_equal(val[idx], ev)
+
+
+@pytest.mark.parametrize("width", [4, 8])
+def test_implicit_update_parity(hbt, width):
+    rng = np.random.default_rng(width)
+    for n in [0, 10, 4000]:
+        k, v = gen_keys(n, width, rng, dup=True)
+        o = oracle.ITree.from_pairs(k, v, 8, width)
+        t = gpu_build(hbt, k, v, 8, width)
+        for _ in range(3):
+            nops = 1500
+            mx = (1 << (8 * width)) - 1
+            live = k if len(k) else np.zeros(1, np.uint64)
+            ok = np.where(rng.random(nops) < 0.5, live[rng.integers(0, len(live), nops)],
+                          rng.integers(0, mx, nops, dtype=np.uint64, endpoint=True)).astype(np.uint64)
+            ov = rng.integers(0, mx, nops, dtype=np.uint64, endpoint=True)
+            op = (rng.random(nops) < 0.4).astype(np.uint8)
+            o = o.update(ok, ov, op)
+            t.update(to_dev(ok, width), to_dev(ov, width), torch.from_numpy(op).cuda())
+            inner, leaf = expected_implicit_bytes(o, width)
+            assert t.export(hbt.SEG_INNER).tobytes() == inner
+            assert t.export(hbt.SEG_LEAF).tobytes() == leaf
+            q = query_set(ok[:500], width, rng, 2000)
+            pf, val = gpu_search(t, q, width)
+            epf, ev = o.search(q)
+            assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+
+
+@pytest.mark.parametrize("pinned", [True, False])
+def test_search_host_pipeline(hbt, pinned):
+    """hbt_search_host: host buffers, chunked H2D / search / D2H over two streams."""
+    width, F = 8, 16
+    rng = np.random.default_rng(3)
+    k, v = gen_keys(100000, width, rng)
+    o = oracle.ITree.from_pairs(k, v, F, width)
+    t = gpu_build(hbt, k, v, F, width)
+    m = (1 << 22) + 12345  # more than one 4 Mi bucket, ragged tail
+    q = k[rng.integers(0, len(k), m)].astype(np.uint64)
+    q[::7] = rng.integers(0, 2**64 - 1, len(q[::7]), dtype=np.uint64, endpoint=True)
+    if pinned:
+        hq = torch.from_numpy(q.view(np.int64)).pin_memory()
+        hp = torch.empty(m, dtype=torch.int64).pin_memory()
+        hv = torch.empty(m, dtype=torch.int64).pin_memory()
+    else:
+        hq = q.copy()
+        hp = np.empty(m, np.uint64)
+        hv = np.empty(m, np.uint64)
+    t.search_host(hq, hp, hv)
+    pf = hp.numpy().view(np.uint64) if pinned else hp
+    val = hv.numpy().view(np.uint64) if pinned else hv
+    epf, ev = o.search(q, nthreads=oracle.default_threads())
+    assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+
+
+def test_device_generators_match_numpy():
+    g = GenLib()
+    for w in (4, 8):
+        s = gen.stream_seed(2, gen.STREAM_K)
+        assert np.array_equal(from_dev(g.mix_stream(100000, w, s, start=7), w),
+                              gen.keys(100000, w, s, start=7).astype(np.uint64))
+        sq = gen.stream_seed(2, gen.STREAM_Q)
+        keys = gen.keys(5000, w, s)
+        assert np.array_equal(from_dev(g.uniform_queries(50000, 5000, w, sq, s, start=3), w),
+                              gen.uniform_hit_queries(keys, 50000, sq, start=3).astype(np.uint64))
+    s = gen.stream_seed(4, gen.STREAM_K)
+    assert np.array_equal(from_dev(g.stratified_keys(1000, s, start=5), 8), gen.stratified_keys(1000, s, start=5))

@@ -1,0 +1,77 @@
+"""Roofline model for batched B+-tree lookups, used by bench.py.
+
+Algorithmic bytes per query (what the method must move):
+  I/O      2S + 8          (query in; value + pos|found out)
+  per inner level one node: implicit F*S rounded up to 32 B sectors;
+                            regular index sector 32 + key line 64 + ref sector 32
+                            (last level: 32 + 64)
+  leaf     key sector 32 + value sector 32 (the value sector only when found)
+Only bytes that miss the L2 count toward HBM.  The cache model is an ideal
+static cache: the L2 capacity holds the byte ranges with the highest access
+probability per byte (levels top-down for uniform queries; the Zipf pmf can
+be supplied per leaf line).  Levels pinned in shared memory cost nothing.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+
+def _sect(b):
+    return ((b + 31) // 32) * 32
+
+
+def implicit_tiers(info, hit_rate=1.0, smem_levels=None):
+    """List of (total_bytes, bytes_per_query) tiers of the implicit tree below the
+    shared-memory levels (uniform queries: every node of a level equally likely)."""
+    S, F = info["width"], info["fanout"]
+    SL = info["smem_levels"] if smem_levels is None else smem_levels
+    nb = _sect(F * S)
+    tiers = []
+    for d, nodes in enumerate(info["level_nodes"]):
+        if d < SL:
+            continue
+        tiers.append((nodes * nb, nb))
+    L0 = info["leaf_lines"]
+    tiers.append((L0 * 32, 32.0))             # key sector of the leaf line
+    tiers.append((L0 * 32, 32.0 * hit_rate))  # value sector (found only)
+    return tiers
+
+
+def regular_tiers(info, hit_rate=1.0, smem_levels=None):
+    S, F = info["width"], info["fanout"]
+    kpl = 64 // S
+    SL = info["smem_levels"] if smem_levels is None else smem_levels
+    per_upper = (32 if F > kpl else 0) + min(64, F * S) + 32
+    per_last = (32 if F > kpl else 0) + min(64, F * S)
+    levels = list(reversed(info["level_nodes"]))  # root first
+    tiers = []
+    node_bytes = (32 if F > kpl else 0) + F * S + 4 * F
+    for d, nodes in enumerate(levels):
+        if d < SL:
+            continue
+        tiers.append((nodes * node_bytes, per_upper))
+    pool = info["leaf_lines"]
+    tiers.append((pool * ((32 if F > kpl else 0) + F * S), per_last))
+    tiers.append((pool * F * 32, 32.0))
+    tiers.append((pool * F * 32, 32.0 * hit_rate))
+    return tiers
+
+
+def static_cache_bytes(tiers, capacity):
+    """Per-query bytes that miss an ideal static cache of `capacity` bytes."""
+    miss = 0.0
+    left = float(capacity)
+    for total, per_q in sorted(tiers, key=lambda t: -(t[1] / max(t[0], 1))):
+        cached = min(1.0, left / total) if total > 0 else 1.0
+        left = max(0.0, left - total)
+        miss += per_q * (1.0 - cached)
+    return miss
+
+
+def model(info, l2_bytes, hit_rate=1.0):
+    S = info["width"]
+    io = 2 * S + 8
+    tiers = implicit_tiers(info, hit_rate) if info["layout"] == 0 else regular_tiers(info, hit_rate)
+    hbm = io + static_cache_bytes(tiers, l2_bytes)
+    l2 = io + sum(t[1] for t in tiers)
+    return {"hbm_bytes_per_query": hbm, "l2_bytes_per_query": l2, "io_bytes_per_query": io}
