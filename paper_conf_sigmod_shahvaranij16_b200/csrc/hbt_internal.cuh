@@ -56,7 +56,9 @@ struct RegularState {
   void* d_ukeys = nullptr;               // ucap x F keys
   void* d_uidx = nullptr;                // ucap x NIP
   uint32_t* d_urefs = nullptr;           // ucap x F
-  void* d_umax = nullptr;                // scratch: max key per node of the level being built
+  uint32_t* d_seg_of_leaf = nullptr;     // pool-sized: leaf -> update segment (0xFFFFFFFF = none)
+  uint64_t seg_cap = 0;
+  uint32_t root_leaf = 0;                // chain[0] (the root when U == 0)
 };
 
 struct HostPipe {

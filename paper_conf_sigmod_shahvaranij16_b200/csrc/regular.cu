@@ -1,9 +1,1031 @@
-// regular.cu — placeholder until the regular tree lands.
+// regular.cu — the REGULAR (pointer) tree: build, search, batch update.
+//
+// Node formats (generalised to fanout F):
+//   upper inner node u (pool index, bottom-up, left to right):
+//       idx[u]  : NIP = 32/S index entries (one 32 B sector); entry t = the max key
+//                 of key line t ("I_s = K_8s"), entries >= NI are MAX
+//       keys[u] : F separator keys = max key of child i for i < cnt-1, else MAX
+//       refs[u] : F uint32 child references (pool indices)
+//   last-level inner node v and big leaf v share the pool index v:
+//       lidx[v], lkeys[v] : as above over the F lines of big leaf v
+//       leaf[v]           : F lines of 64 B = [P keys | P values], dense-packed
+//       count[v]          : entries in big leaf v (node fragmentation)
+//   chain : live big leaves in key order.
+// Search = three dependent accesses per upper level (index sector -> one 64 B
+// key line -> one reference), two at the last level, one leaf line;
+// the leaf's MAX padding needs no size except when the slot holds MAX.
+#include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_scan.cuh>
+#include <cub/device/device_select.cuh>
+
 #include "hbt_internal.cuh"
+
 namespace hbt {
-int regular_build(hbt_tree*, const void*, const void*, uint64_t, cudaStream_t) { set_error("regular tree not built yet"); return HBT_EUNSUPPORTED; }
-int regular_search(const hbt_tree*, const void*, uint64_t, uint64_t*, void*, cudaStream_t) { return HBT_EUNSUPPORTED; }
-int regular_update(hbt_tree*, const hbt_batch*, cudaStream_t) { return HBT_EUNSUPPORTED; }
-void regular_free(hbt_tree*) {}
-uint32_t regular_smem_levels(const hbt_tree*, uint32_t) { return 0; }
+namespace {
+
+constexpr uint64_t kEnd = HBT_POS_END;
+constexpr uint64_t kFound = HBT_FOUND_BIT;
+constexpr uint32_t kNoRef = 0xFFFFFFFFu;
+
+template <typename K>
+__host__ __device__ constexpr K key_max() { return K(~K(0)); }
+
+inline unsigned grid_for(uint64_t n) {
+  uint64_t g = (n + 255) / 256;
+  if (g > 148 * 64) g = 148 * 64;
+  return unsigned(g ? g : 1);
 }
+
+#define GRID_STRIDE(i, n) \
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < (n); i += uint64_t(gridDim.x) * blockDim.x)
+
+template <typename K>
+struct Geo {
+  static constexpr uint32_t S = sizeof(K);
+  static constexpr uint32_t P = 64 / (2 * S);
+  static constexpr uint32_t KPL = 64 / S;  // keys per 64 B key line
+  static constexpr uint32_t NIP = 32 / S;  // index entries per 32 B sector
+};
+
+// ---------------------------------------------------------------- build kernels
+
+template <typename K>
+__global__ void pack_big_leaves(const K* __restrict__ kd, const K* __restrict__ vd, uint64_t nd, uint64_t nb,
+                                uint32_t F, K* __restrict__ leaf, uint32_t* __restrict__ count) {
+  constexpr uint32_t P = Geo<K>::P;
+  const uint64_t B = uint64_t(F) * P;
+  GRID_STRIDE(x, nb * B) {
+    const uint64_t v = x / B, e = x % B;
+    const uint64_t lo = v * nd / nb, hi = (v + 1) * nd / nb;  // nd < 2^32: no overflow
+    K* line = leaf + (v * F + e / P) * (2 * P);
+    const bool real = e < hi - lo;
+    line[e % P] = real ? kd[lo + e] : key_max<K>();
+    line[P + e % P] = real ? vd[lo + e] : K(0);
+    if (e == 0) count[v] = uint32_t(hi - lo);
+  }
+}
+
+// Last-level inner node v from big leaf v: sep[j] = max of line j for j < lines-1.
+template <typename K>
+__global__ void derive_last_level(const K* __restrict__ leaf, const uint32_t* __restrict__ count, uint64_t pool,
+                                  uint32_t F, const uint8_t* __restrict__ dirty, K* __restrict__ lkeys,
+                                  K* __restrict__ lidx) {
+  constexpr uint32_t P = Geo<K>::P, KPL = Geo<K>::KPL, NIP = Geo<K>::NIP;
+  const uint32_t NI = F > KPL ? F / KPL : 1;
+  GRID_STRIDE(v, pool) {
+    if (dirty && !dirty[v]) continue;
+    const uint32_t c = count[v];
+    const uint32_t lines = c == 0 ? 1 : (c + P - 1) / P;
+    K* sep = lkeys + v * F;
+    for (uint32_t j = 0; j < F; ++j)
+      sep[j] = (j + 1 < lines) ? leaf[(v * F + j) * (2 * P) + (P - 1)] : key_max<K>();
+    for (uint32_t t = 0; t < NIP; ++t) {
+      uint32_t slot = t * KPL + KPL - 1;
+      if (slot > F - 1) slot = F - 1;
+      lidx[v * NIP + t] = t < NI ? sep[slot] : key_max<K>();
+    }
+  }
+}
+
+__global__ void iota_chain(uint32_t* chain, uint64_t n) {
+  GRID_STRIDE(i, n) chain[i] = uint32_t(i);
+}
+
+template <typename K>
+__global__ void chain_leaf_max(const K* __restrict__ leaf, const uint32_t* __restrict__ count,
+                               const uint32_t* __restrict__ chain, uint64_t nchain, uint32_t F, K* __restrict__ mx) {
+  constexpr uint32_t P = Geo<K>::P;
+  GRID_STRIDE(i, nchain) {
+    const uint64_t v = chain[i];
+    const uint32_t c = count[v];
+    mx[i] = c ? leaf[(v * F + (c - 1) / P) * (2 * P) + (c - 1) % P] : key_max<K>();
+  }
+}
+
+// One upper level: node j groups children [jF, jF+cnt) of the level below.
+template <typename K>
+__global__ void build_upper_level(const uint32_t* __restrict__ child_ids, uint64_t child_base, const K* __restrict__ child_max,
+                                  uint64_t cnt_below, uint64_t nodes, uint64_t node_base, uint32_t F,
+                                  K* __restrict__ ukeys, K* __restrict__ uidx, uint32_t* __restrict__ urefs,
+                                  K* __restrict__ out_max) {
+  constexpr uint32_t KPL = Geo<K>::KPL, NIP = Geo<K>::NIP;
+  const uint32_t NI = F > KPL ? F / KPL : 1;
+  GRID_STRIDE(j, nodes) {
+    const uint64_t first = j * F;
+    const uint64_t cnt = (cnt_below - first < F) ? cnt_below - first : F;
+    const uint64_t id = node_base + j;
+    K* keys = ukeys + id * F;
+    uint32_t* refs = urefs + id * F;
+    for (uint32_t i = 0; i < F; ++i) {
+      keys[i] = (i + 1 < cnt) ? child_max[first + i] : key_max<K>();
+      refs[i] = (i < cnt) ? (child_ids ? child_ids[first + i] : uint32_t(child_base + first + i)) : kNoRef;
+    }
+    for (uint32_t t = 0; t < NIP; ++t) {
+      uint32_t slot = t * KPL + KPL - 1;
+      if (slot > F - 1) slot = F - 1;
+      uidx[id * NIP + t] = t < NI ? keys[slot] : key_max<K>();
+    }
+    out_max[j] = child_max[first + cnt - 1];
+  }
+}
+
+// ---------------------------------------------------------------- search kernel
+
+struct RView {
+  const uint8_t* leaf;
+  const uint32_t* count;
+  const uint8_t* lkeys;
+  const uint8_t* lidx;
+  const uint8_t* ukeys;
+  const uint8_t* uidx;
+  const uint32_t* urefs;
+  uint64_t uoff[HBT_MAX_LEVELS + 1];
+  uint32_t U;
+  uint32_t SL;        // top upper levels staged in shared memory
+  uint32_t root_leaf; // big leaf when U == 0
+  uint64_t smem_first;  // pool index of the first staged upper node
+  uint64_t smem_nodes;
+};
+
+template <typename K, int N>
+__device__ __forceinline__ K pick(const K (&k)[N], uint32_t slot) {
+  K r = k[0];
+#pragma unroll
+  for (int t = 1; t < N; ++t) r = (slot == uint32_t(t)) ? k[t] : r;
+  return r;
+}
+
+template <typename K>
+union V16 {
+  uint4 u;
+  K k[16 / sizeof(K)];
+};
+
+template <typename K>
+__device__ __forceinline__ V16<K> ld16g(const uint8_t* p) {
+  V16<K> v;
+  v.u = __ldg(reinterpret_cast<const uint4*>(p));
+  return v;
+}
+template <typename K>
+__device__ __forceinline__ V16<K> ld16s(const uint8_t* p) {
+  V16<K> v;
+  v.u = *reinterpret_cast<const uint4*>(p);
+  return v;
+}
+
+__device__ __forceinline__ uint32_t ldcs(const uint32_t* p) { return __ldcs(p); }
+__device__ __forceinline__ uint64_t ldcs(const uint64_t* p) { return __ldcs(reinterpret_cast<const unsigned long long*>(p)); }
+__device__ __forceinline__ void stcs(uint32_t* p, uint32_t v) { __stcs(p, v); }
+__device__ __forceinline__ void stcs(uint64_t* p, uint64_t v) { __stcs(reinterpret_cast<unsigned long long*>(p), (unsigned long long)v); }
+
+// Group of G = 4 lanes per query; each lane holds 16 B of a 64 B key line / leaf
+// line; QPG queries in flight per group (8 groups x QPG = 32 queries per warp round).
+template <typename K, int F, int QPG, int THREADS>
+__global__ void __launch_bounds__(THREADS)
+regular_search_kernel(const RView rv, const K* __restrict__ queries, uint64_t m, uint64_t* __restrict__ out_pf,
+                      K* __restrict__ out_v) {
+  constexpr int G = 4, NG = 8, ROUND = NG * QPG;
+  constexpr uint32_t S = sizeof(K), P = Geo<K>::P, KPL = Geo<K>::KPL, NIP = Geo<K>::NIP;
+  constexpr uint32_t E16 = 16 / S;                       // entries per 16 B lane chunk
+  constexpr uint32_t NI = uint32_t(F) > KPL ? uint32_t(F) / KPL : 1;
+  constexpr uint32_t LINE = uint32_t(F) * S < 64 ? uint32_t(F) * S : 64;  // bytes of one key line
+  constexpr int KL = int(LINE / 16) ? int(LINE / 16) : 1;                 // lanes loading it
+  static_assert(ROUND <= 32, "tiling");
+  extern __shared__ __align__(16) uint8_t smem[];
+  // stage the top SL upper levels: keys | idx | refs (contiguous pool range)
+  const uint64_t NS = rv.smem_nodes;
+  uint8_t* s_keys = smem;
+  uint8_t* s_idx = smem + NS * F * S;
+  uint32_t* s_refs = reinterpret_cast<uint32_t*>(smem + NS * (F * S + NIP * S));
+  {
+    const uint4* a = reinterpret_cast<const uint4*>(rv.ukeys + rv.smem_first * F * S);
+    const uint4* b = reinterpret_cast<const uint4*>(rv.uidx + rv.smem_first * NIP * S);
+    const uint4* c = reinterpret_cast<const uint4*>(rv.urefs + rv.smem_first * F);
+    for (uint64_t i = threadIdx.x; i < NS * F * S / 16; i += THREADS) reinterpret_cast<uint4*>(s_keys)[i] = __ldg(a + i);
+    for (uint64_t i = threadIdx.x; i < NS * NIP * S / 16; i += THREADS) reinterpret_cast<uint4*>(s_idx)[i] = __ldg(b + i);
+    for (uint64_t i = threadIdx.x; i < NS * F * 4 / 16; i += THREADS) reinterpret_cast<uint4*>(s_refs)[i] = __ldg(c + i);
+  }
+  __syncthreads();
+
+  const int lane = threadIdx.x & 31;
+  const int g = lane / G, k = lane % G;
+  const unsigned gmask = 0xFu << (g * G);
+  const uint64_t warp = (uint64_t(blockIdx.x) * THREADS + threadIdx.x) >> 5;
+  const uint64_t nwarps = (uint64_t(gridDim.x) * THREADS) >> 5;
+  const uint64_t rounds = (m + ROUND - 1) / ROUND;
+  const uint32_t U = rv.U, SL = rv.SL;
+
+  for (uint64_t rd = warp; rd < rounds; rd += nwarps) {
+    const uint64_t my_i = rd * ROUND + uint64_t(k) * NG + g;
+    const bool my_ok = (k < QPG) && (my_i < m);
+    const K myq = my_ok ? ldcs(queries + my_i) : key_max<K>();
+    K q[QPG];
+    uint32_t cur[QPG];
+#pragma unroll
+    for (int j = 0; j < QPG; ++j) {
+      q[j] = __shfl_sync(0xffffffffu, myq, g * G + j);
+      cur[j] = U ? uint32_t(rv.uoff[U] - 1) : rv.root_leaf;
+    }
+    // ---- upper levels, root first
+    for (uint32_t l = 0; l < U; ++l) {
+      const bool sm = l < SL;
+      uint32_t t[QPG];
+      if constexpr (NI > 1) {  // (1) index sector: t = #{idx < q}
+        V16<K> iv[QPG];
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          if (k < 2) {
+            iv[j] = sm ? ld16s<K>(s_idx + (cur[j] - rv.smem_first) * NIP * S + k * 16)
+                       : ld16g<K>(rv.uidx + uint64_t(cur[j]) * NIP * S + k * 16);
+          } else {
+#pragma unroll
+            for (uint32_t e = 0; e < E16; ++e) iv[j].k[e] = key_max<K>();
+          }
+        }
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          uint32_t c = 0;
+#pragma unroll
+          for (uint32_t e = 0; e < E16; ++e) c += __popc(__ballot_sync(0xffffffffu, iv[j].k[e] < q[j]) & gmask);
+          t[j] = c;
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) t[j] = 0;
+      }
+      // (2) key line t
+      V16<K> kv[QPG];
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) {
+        if (k < KL) {
+          const uint64_t off = (uint64_t(cur[j]) * F + t[j] * KPL) * S + k * 16;
+          kv[j] = sm ? ld16s<K>(s_keys + (uint64_t(cur[j] - rv.smem_first) * F + t[j] * KPL) * S + k * 16)
+                     : ld16g<K>(rv.ukeys + off);
+        } else {
+#pragma unroll
+          for (uint32_t e = 0; e < E16; ++e) kv[j].k[e] = key_max<K>();
+        }
+      }
+      uint32_t slot[QPG];
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) {
+        uint32_t c = 0;
+#pragma unroll
+        for (uint32_t e = 0; e < E16; ++e) c += __popc(__ballot_sync(0xffffffffu, kv[j].k[e] < q[j]) & gmask);
+        slot[j] = t[j] * KPL + c;
+      }
+      // (3) child reference
+#pragma unroll
+      for (int j = 0; j < QPG; ++j)
+        cur[j] = sm ? s_refs[uint64_t(cur[j] - rv.smem_first) * F + slot[j]]
+                    : __ldg(rv.urefs + uint64_t(cur[j]) * F + slot[j]);
+    }
+    // ---- last level (shares pool index with the big leaf): index sector + key line -> line j
+    uint32_t lj[QPG];
+    {
+      uint32_t t[QPG];
+      if constexpr (NI > 1) {
+        V16<K> iv[QPG];
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          if (k < 2) iv[j] = ld16g<K>(rv.lidx + uint64_t(cur[j]) * NIP * S + k * 16);
+          else {
+#pragma unroll
+            for (uint32_t e = 0; e < E16; ++e) iv[j].k[e] = key_max<K>();
+          }
+        }
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          uint32_t c = 0;
+#pragma unroll
+          for (uint32_t e = 0; e < E16; ++e) c += __popc(__ballot_sync(0xffffffffu, iv[j].k[e] < q[j]) & gmask);
+          t[j] = c;
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) t[j] = 0;
+      }
+      V16<K> kv[QPG];
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) {
+        if (k < KL) kv[j] = ld16g<K>(rv.lkeys + (uint64_t(cur[j]) * F + t[j] * KPL) * S + k * 16);
+        else {
+#pragma unroll
+          for (uint32_t e = 0; e < E16; ++e) kv[j].k[e] = key_max<K>();
+        }
+      }
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) {
+        uint32_t c = 0;
+#pragma unroll
+        for (uint32_t e = 0; e < E16; ++e) c += __popc(__ballot_sync(0xffffffffu, kv[j].k[e] < q[j]) & gmask);
+        lj[j] = t[j] * KPL + c;
+      }
+    }
+    // ---- leaf line (v*F + j): lanes 0-1 keys, 2-3 values
+    V16<K> lv[QPG];
+#pragma unroll
+    for (int j = 0; j < QPG; ++j)
+      lv[j] = ld16g<K>(rv.leaf + (uint64_t(cur[j]) * F + lj[j]) * 64 + k * 16);
+    uint64_t my_pf = 0;
+    K my_v = 0;
+#pragma unroll
+    for (int j = 0; j < QPG; ++j) {
+      uint32_t s = 0;
+#pragma unroll
+      for (uint32_t e = 0; e < E16; ++e) s += __popc(__ballot_sync(0xffffffffu, (k < 2) && (lv[j].k[e] < q[j])) & gmask);
+      const uint32_t sc = s < P ? s : P - 1;
+      const K sel = pick(lv[j].k, sc % E16);
+      const int src = g * G + int(sc / E16);
+      const K key_s = __shfl_sync(0xffffffffu, sel, src);
+      const K val_s = __shfl_sync(0xffffffffu, sel, src + 2);
+      bool end = (s == P);
+      if (!end && key_s == key_max<K>()) {
+        // MAX slot: padding unless it is a counted entry ("must read the node size")
+        const int64_t in_line = int64_t(__ldg(rv.count + cur[j])) - int64_t(lj[j]) * P;
+        const int64_t lim = in_line < int64_t(P) ? in_line : int64_t(P);
+        end = int64_t(s) >= lim;
+      }
+      const bool found = !end && key_s == q[j];
+      if (j == k) {
+        my_pf = end ? kEnd : (((uint64_t(cur[j]) * F + lj[j]) * P + s) | (found ? kFound : 0ull));
+        my_v = found ? val_s : K(0);
+      }
+    }
+    if (my_ok) {
+      stcs(out_pf + my_i, my_pf);
+      stcs(out_v + my_i, my_v);
+    }
+  }
+}
+
+constexpr int kThreads = 512;
+constexpr int kQPG = 4;
+
+template <typename K>
+uint64_t upper_node_bytes(uint32_t F) { return uint64_t(F) * sizeof(K) + Geo<K>::NIP * sizeof(K) + 4ull * F; }
+
+template <typename K>
+uint32_t smem_levels_t(const hbt_tree* t, uint32_t budget) {
+  const RegularState& r = t->r;
+  uint32_t SL = 0;
+  while (SL < r.U) {
+    const uint64_t nodes = r.uoff[r.U] - r.uoff[r.U - SL - 1];
+    if (nodes * upper_node_bytes<K>(t->F) > budget) break;
+    ++SL;
+  }
+  return SL;
+}
+
+template <typename K, int F>
+int search_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+  const RegularState& r = t->r;
+  auto kern = regular_search_kernel<K, F, kQPG, kThreads>;
+  RView rv{};
+  rv.leaf = (const uint8_t*)r.d_leaf;
+  rv.count = r.d_count;
+  rv.lkeys = (const uint8_t*)r.d_lkeys;
+  rv.lidx = (const uint8_t*)r.d_lidx;
+  rv.ukeys = (const uint8_t*)r.d_ukeys;
+  rv.uidx = (const uint8_t*)r.d_uidx;
+  rv.urefs = r.d_urefs;
+  for (uint32_t u = 0; u <= r.U; ++u) rv.uoff[u] = r.uoff[u];
+  rv.U = r.U;
+  rv.root_leaf = r.root_leaf;
+  const uint32_t budget = t->cfg.smem_budget ? t->cfg.smem_budget : 100 * 1024;
+  rv.SL = smem_levels_t<K>(t, budget);
+  rv.smem_first = rv.SL ? r.uoff[r.U - rv.SL] : 0;
+  rv.smem_nodes = rv.SL ? r.uoff[r.U] - rv.smem_first : 0;
+  const size_t smem = rv.smem_nodes * upper_node_bytes<K>(F);
+  static bool attr = false;
+  if (!attr) {
+    HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    attr = true;
+  }
+  int occ = 0;
+  HBT_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, smem));
+  if (t->cfg.ctas_per_sm && int(t->cfg.ctas_per_sm) < occ) occ = int(t->cfg.ctas_per_sm);
+  if (occ < 1) occ = 1;
+  const uint64_t rounds = (m + 8 * kQPG - 1) / (8 * kQPG);
+  uint64_t grid = uint64_t(t->num_sms) * occ;
+  const uint64_t need = (rounds + kThreads / 32 - 1) / (kThreads / 32);
+  if (need < grid) grid = need ? need : 1;
+  kern<<<unsigned(grid), kThreads, smem, s>>>(rv, (const K*)q, m, pf, (K*)v);
+  HBT_CUDA_TRY(cudaGetLastError());
+  return HBT_OK;
+}
+
+template <typename K>
+int search_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+  switch (t->F) {
+    case 4: return search_launch<K, 4>(t, q, m, pf, v, s);
+    case 8: return search_launch<K, 8>(t, q, m, pf, v, s);
+    case 16: return search_launch<K, 16>(t, q, m, pf, v, s);
+    case 32: return search_launch<K, 32>(t, q, m, pf, v, s);
+  }
+  set_error("unsupported fanout");
+  return HBT_EINVAL;
+}
+
+// ---------------------------------------------------------------- state management
+
+template <typename K>
+int alloc_pool(hbt_tree* t, uint64_t cap) {
+  RegularState& r = t->r;
+  const uint64_t F = t->F, S = sizeof(K);
+  HBT_CUDA_TRY(cudaMalloc(&r.d_leaf, cap * F * 64));
+  HBT_CUDA_TRY(cudaMalloc(&r.d_count, cap * 4));
+  HBT_CUDA_TRY(cudaMalloc(&r.d_lkeys, cap * F * S));
+  HBT_CUDA_TRY(cudaMalloc(&r.d_lidx, cap * 32));
+  HBT_CUDA_TRY(cudaMalloc(&r.d_chain, cap * 4));
+  r.cap = cap;
+  return HBT_OK;
+}
+
+// grow the big-leaf pool arrays to hold `need` leaves (copying pool entries)
+template <typename K>
+int grow_pool(hbt_tree* t, uint64_t need, cudaStream_t s) {
+  RegularState& r = t->r;
+  if (need <= r.cap) return HBT_OK;
+  uint64_t cap = r.cap ? r.cap : 1;
+  while (cap < need) cap = cap + cap / 2 + 1;
+  const uint64_t F = t->F, S = sizeof(K);
+  void *leaf = nullptr, *lkeys = nullptr, *lidx = nullptr;
+  uint32_t *count = nullptr, *chain = nullptr;
+  HBT_CUDA_TRY(cudaMalloc(&leaf, cap * F * 64));
+  HBT_CUDA_TRY(cudaMalloc(&count, cap * 4));
+  HBT_CUDA_TRY(cudaMalloc(&lkeys, cap * F * S));
+  HBT_CUDA_TRY(cudaMalloc(&lidx, cap * 32));
+  HBT_CUDA_TRY(cudaMalloc(&chain, cap * 4));
+  HBT_CUDA_TRY(cudaMemcpyAsync(leaf, r.d_leaf, r.pool * F * 64, cudaMemcpyDeviceToDevice, s));
+  HBT_CUDA_TRY(cudaMemcpyAsync(count, r.d_count, r.pool * 4, cudaMemcpyDeviceToDevice, s));
+  HBT_CUDA_TRY(cudaMemcpyAsync(lkeys, r.d_lkeys, r.pool * F * S, cudaMemcpyDeviceToDevice, s));
+  HBT_CUDA_TRY(cudaMemcpyAsync(lidx, r.d_lidx, r.pool * 32, cudaMemcpyDeviceToDevice, s));
+  HBT_CUDA_TRY(cudaMemcpyAsync(chain, r.d_chain, r.nchain * 4, cudaMemcpyDeviceToDevice, s));
+  HBT_CUDA_TRY(cudaStreamSynchronize(s));
+  cudaFree(r.d_leaf); cudaFree(r.d_count); cudaFree(r.d_lkeys); cudaFree(r.d_lidx); cudaFree(r.d_chain);
+  r.d_leaf = leaf; r.d_count = count; r.d_lkeys = lkeys; r.d_lidx = lidx; r.d_chain = chain;
+  r.cap = cap;
+  return HBT_OK;
+}
+
+// Regroup every upper level from the chain (reading R11).
+template <typename K>
+int rebuild_upper(hbt_tree* t, cudaStream_t s) {
+  RegularState& r = t->r;
+  const uint32_t F = t->F;
+  uint64_t c = r.nchain, total = 0;
+  uint32_t U = 0;
+  uint64_t unodes[HBT_MAX_LEVELS];
+  while (c > 1) {
+    c = ceil_div_u64(c, F);
+    if (U >= HBT_MAX_LEVELS) { set_error("tree too tall"); return HBT_EUNSUPPORTED; }
+    unodes[U++] = c;
+    total += c;
+  }
+  if (total > r.ucap) {
+    cudaFree(r.d_ukeys); cudaFree(r.d_uidx); cudaFree(r.d_urefs);
+    r.d_ukeys = r.d_uidx = nullptr; r.d_urefs = nullptr; r.ucap = 0;
+    const uint64_t cap = total + total / 4 + 16;
+    HBT_CUDA_TRY(cudaMalloc(&r.d_ukeys, cap * F * sizeof(K)));
+    HBT_CUDA_TRY(cudaMalloc(&r.d_uidx, cap * 32));
+    HBT_CUDA_TRY(cudaMalloc(&r.d_urefs, cap * F * 4));
+    r.ucap = cap;
+  }
+  r.U = U;
+  r.uoff[0] = 0;
+  for (uint32_t u = 0; u < U; ++u) {
+    r.unodes[u] = unodes[u];
+    r.uoff[u + 1] = r.uoff[u] + unodes[u];
+  }
+  if (U == 0) return HBT_OK;
+  K *mx_a = nullptr, *mx_b = nullptr;
+  HBT_CUDA_TRY(cudaMalloc(&mx_a, r.nchain * sizeof(K)));
+  HBT_CUDA_TRY(cudaMalloc(&mx_b, (unodes[0] + 1) * sizeof(K)));
+  chain_leaf_max<K><<<grid_for(r.nchain), 256, 0, s>>>((const K*)r.d_leaf, r.d_count, r.d_chain, r.nchain, F, mx_a);
+  uint64_t below = r.nchain;
+  for (uint32_t u = 0; u < U; ++u) {
+    build_upper_level<K><<<grid_for(unodes[u]), 256, 0, s>>>(
+        u == 0 ? r.d_chain : nullptr, u == 0 ? 0 : r.uoff[u - 1], mx_a, below, unodes[u], r.uoff[u], F,
+        (K*)r.d_ukeys, (K*)r.d_uidx, r.d_urefs, mx_b);
+    K* tmp = mx_a; mx_a = mx_b; mx_b = tmp;
+    below = unodes[u];
+  }
+  cudaError_t e = cudaGetLastError();
+  cudaStreamSynchronize(s);
+  cudaFree(mx_a);
+  cudaFree(mx_b);
+  if (e != cudaSuccess) { set_error("rebuild_upper: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
+  return HBT_OK;
+}
+
+template <typename K>
+int build_t(hbt_tree* t, const void* keys, const void* values, uint64_t n, cudaStream_t s) {
+  RegularState& r = t->r;
+  const uint32_t F = t->F;
+  r.kpl = Geo<K>::KPL;
+  r.NI = F > r.kpl ? F / r.kpl : 1;
+  r.B = F * Geo<K>::P;
+  r.b = (3 * r.B) / 4;
+  void *kd = nullptr, *vd = nullptr;
+  uint64_t nd = 0;
+  int rc = sort_dedupe(sizeof(K), keys, values, n, &kd, &vd, &nd, s);
+  if (rc != HBT_OK) return rc;
+  const uint64_t nb = nd == 0 ? 1 : ceil_div_u64(nd, r.b);
+  rc = alloc_pool<K>(t, nb + nb / 8 + 16);
+  if (rc != HBT_OK) { cudaFree(kd); cudaFree(vd); return rc; }
+  r.pool = nb;
+  r.nchain = nb;
+  r.root_leaf = 0;
+  t->n = nd;
+  pack_big_leaves<K><<<grid_for(nb * r.B), 256, 0, s>>>((const K*)kd, (const K*)vd, nd, nb, F, (K*)r.d_leaf, r.d_count);
+  derive_last_level<K><<<grid_for(nb), 256, 0, s>>>((const K*)r.d_leaf, r.d_count, nb, F, nullptr, (K*)r.d_lkeys,
+                                                     (K*)r.d_lidx);
+  iota_chain<<<grid_for(nb), 256, 0, s>>>(r.d_chain, nb);
+  cudaError_t e = cudaGetLastError();
+  cudaStreamSynchronize(s);
+  cudaFree(kd);
+  cudaFree(vd);
+  if (e != cudaSuccess) { set_error("regular build: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
+  return rebuild_upper<K>(t, s);
+}
+
+// ---------------------------------------------------------------- update kernels
+
+// Scalar descent of one op key to its big leaf (stops above the last level).
+template <typename K>
+__global__ void locate_leaf(const K* __restrict__ keys, uint64_t m, const K* __restrict__ ukeys,
+                            const K* __restrict__ uidx, const uint32_t* __restrict__ urefs, uint64_t root,
+                            uint32_t U, uint32_t root_leaf, uint32_t F, uint32_t* __restrict__ leaf_of) {
+  constexpr uint32_t KPL = Geo<K>::KPL, NIP = Geo<K>::NIP;
+  const uint32_t NI = F > KPL ? F / KPL : 1;
+  GRID_STRIDE(x, m) {
+    const K q = keys[x];
+    uint64_t cur = U ? root : root_leaf;
+    for (uint32_t l = 0; l < U; ++l) {
+      uint32_t base = 0, len = F;
+      if (NI > 1) {
+        uint32_t t = 0;
+        for (uint32_t e = 0; e < NI; ++e) t += uidx[cur * NIP + e] < q;
+        base = t * KPL;
+        len = KPL;
+      }
+      uint32_t i = base;
+      for (uint32_t e = 0; e < len; ++e) i += ukeys[cur * F + base + e] < q;
+      cur = urefs[cur * F + i];
+    }
+    leaf_of[x] = uint32_t(cur);
+  }
+}
+
+__global__ void iota_u32(uint32_t* p, uint64_t n) { GRID_STRIDE(i, n) p[i] = uint32_t(i); }
+
+template <typename K>
+__global__ void last_of_run(const K* __restrict__ sk, uint64_t n, uint8_t* __restrict__ f) {
+  GRID_STRIDE(i, n) f[i] = (i + 1 == n) || (sk[i] != sk[i + 1]);
+}
+
+template <typename K>
+__global__ void gather_ops(const uint32_t* __restrict__ idx, uint64_t n, const K* __restrict__ bv,
+                           const uint8_t* __restrict__ bo, K* __restrict__ ov, uint8_t* __restrict__ oo) {
+  GRID_STRIDE(i, n) {
+    ov[i] = bv[idx[i]];
+    oo[i] = bo[idx[i]];
+  }
+}
+
+__global__ void segment_flags(const uint32_t* __restrict__ leaf_of, uint64_t m, uint32_t* __restrict__ start_flag) {
+  GRID_STRIDE(i, m) start_flag[i] = (i == 0 || leaf_of[i] != leaf_of[i - 1]) ? 1u : 0u;
+}
+
+// segment s = ops [seg_off[s], seg_off[s+1]) of leaf seg_leaf[s]
+__global__ void segment_tables(const uint32_t* __restrict__ leaf_of, const uint32_t* __restrict__ seg_incl, uint64_t m,
+                               uint32_t* __restrict__ seg_off, uint32_t* __restrict__ seg_leaf,
+                               uint32_t* __restrict__ seg_of_leaf) {
+  GRID_STRIDE(i, m) {
+    if (i == 0 || leaf_of[i] != leaf_of[i - 1]) {
+      const uint32_t sgi = seg_incl[i] - 1;
+      seg_off[sgi] = uint32_t(i);
+      seg_leaf[sgi] = leaf_of[i];
+      seg_of_leaf[leaf_of[i]] = sgi;
+    }
+    if (i + 1 == m) seg_off[seg_incl[i]] = uint32_t(m);
+  }
+}
+
+// Big-leaf entry e of leaf v (dense order): line e/P, slot e%P.
+template <typename K>
+__device__ __forceinline__ K leaf_key(const K* leaf, uint64_t v, uint32_t F, uint32_t e) {
+  constexpr uint32_t P = Geo<K>::P;
+  return leaf[(v * F + e / P) * (2 * P) + e % P];
+}
+
+// Per op: lower bound in its leaf, found?, inserted?, count delta.
+template <typename K>
+__global__ void op_classify(const K* __restrict__ ok, const uint8_t* __restrict__ oo, uint64_t m,
+                            const uint32_t* __restrict__ leaf_of, const uint32_t* __restrict__ seg_incl,
+                            const K* __restrict__ leaf, const uint32_t* __restrict__ count, uint32_t F,
+                            uint32_t* __restrict__ lb, uint32_t* __restrict__ ins, int* __restrict__ seg_delta) {
+  GRID_STRIDE(x, m) {
+    const uint64_t v = leaf_of[x];
+    const K q = ok[x];
+    uint32_t lo = 0, hi = count[v];
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi) / 2;
+      if (leaf_key(leaf, v, F, mid) < q) lo = mid + 1; else hi = mid;
+    }
+    const bool found = lo < count[v] && leaf_key(leaf, v, F, lo) == q;
+    lb[x] = lo;
+    const bool is_ins = oo[x] == 0 && !found;
+    const bool is_del = oo[x] != 0 && found;
+    ins[x] = is_ins ? 1u : 0u;
+    const int d = is_ins ? 1 : (is_del ? -1 : 0);
+    if (d) atomicAdd(seg_delta + (seg_incl[x] - 1), d);
+  }
+}
+
+__global__ void segment_counts(const uint32_t* __restrict__ seg_leaf, const int* __restrict__ seg_delta, uint64_t nseg,
+                               const uint32_t* __restrict__ count, uint32_t B, uint32_t* __restrict__ new_cnt,
+                               uint32_t* __restrict__ extra) {
+  GRID_STRIDE(s, nseg) {
+    const int64_t c = int64_t(count[seg_leaf[s]]) + seg_delta[s];
+    new_cnt[s] = uint32_t(c);
+    const uint64_t parts = c == 0 ? 0 : (uint64_t(c) + B - 1) / B;
+    extra[s] = parts > 1 ? uint32_t(parts - 1) : 0u;
+  }
+}
+
+// One warp per affected leaf: merge the leaf's entries with its ops and write
+// the result evenly split over ceil(c/B) leaves (the first keeps index v, the
+// others get new_base[s] + p - 1), padding every slot past each part's count.
+template <typename K, int MAXB>
+__global__ void merge_write(const uint32_t* __restrict__ seg_leaf, const uint32_t* __restrict__ seg_off, uint64_t nseg,
+                            const uint32_t* __restrict__ new_cnt, const uint32_t* __restrict__ new_base,
+                            const K* __restrict__ ok, const K* __restrict__ ov, const uint8_t* __restrict__ oo,
+                            const uint32_t* __restrict__ lb, const uint32_t* __restrict__ insx,
+                            K* __restrict__ leaf, uint32_t* __restrict__ count, uint8_t* __restrict__ dirty,
+                            uint32_t F) {
+  constexpr uint32_t P = Geo<K>::P;
+  constexpr int WARPS = 4;
+  __shared__ K s_k[WARPS][MAXB];
+  __shared__ K s_v[WARPS][MAXB];
+  __shared__ uint32_t s_del[WARPS][MAXB + 1];  // # deleted entries before index i
+  const int w = threadIdx.x / 32, lane = threadIdx.x & 31;
+  const uint32_t B = F * P;
+  for (uint64_t sg = blockIdx.x * uint64_t(WARPS) + w; sg < nseg; sg += uint64_t(gridDim.x) * WARPS) {
+    const uint64_t v = seg_leaf[sg];
+    const uint32_t c_old = count[v];
+    const uint32_t o0 = seg_off[sg], o1 = seg_off[sg + 1];
+    const uint32_t ins0 = insx[o0];
+    // stage old entries; resolve each against the ops (binary search in [o0, o1))
+    for (uint32_t i = lane; i < c_old; i += 32) {
+      const K key = leaf_key(leaf, v, F, i);
+      s_k[w][i] = key;
+      s_v[w][i] = leaf[(v * F + i / P) * (2 * P) + P + i % P];
+    }
+    __syncwarp();
+    // deleted flags + new values
+    for (uint32_t base = 0; base < c_old; base += 32) {
+      const uint32_t i = base + lane;
+      bool del = false;
+      if (i < c_old) {
+        const K key = s_k[w][i];
+        uint32_t lo = o0, hi = o1;
+        while (lo < hi) {
+          const uint32_t mid = (lo + hi) / 2;
+          if (ok[mid] < key) lo = mid + 1; else hi = mid;
+        }
+        if (lo < o1 && ok[lo] == key) {
+          if (oo[lo] != 0) del = true;
+          else s_v[w][i] = ov[lo];
+        }
+        s_del[w][i] = del;  // temporarily the flag
+      }
+    }
+    __syncwarp();
+    // exclusive prefix of deletions (chunked ballot scan)
+    uint32_t carry = 0;
+    for (uint32_t base = 0; base < c_old; base += 32) {
+      const uint32_t i = base + lane;
+      const bool f = i < c_old && s_del[w][i];
+      const unsigned bal = __ballot_sync(0xffffffffu, f);
+      const uint32_t before = carry + __popc(bal & ((1u << lane) - 1u));
+      __syncwarp();
+      if (i < c_old) s_del[w][i] = before;
+      carry += __popc(bal);
+      __syncwarp();
+    }
+    if (lane == 0) s_del[w][c_old] = carry;
+    __syncwarp();
+    const uint32_t c = new_cnt[sg];
+    const uint32_t parts = c == 0 ? 0 : (c + B - 1) / B;
+    auto dest = [&](uint32_t rnk, uint64_t& leaf_id, uint32_t& local) {
+      // part p holds merged ranks [floor(p c/k), floor((p+1) c/k))
+      uint32_t p = uint32_t((uint64_t(rnk + 1) * parts + c - 1) / c) - 1;
+      while (p + 1 < parts && uint64_t(p + 1) * c / parts <= rnk) ++p;
+      while (p > 0 && uint64_t(p) * c / parts > rnk) --p;
+      const uint32_t lo = uint32_t(uint64_t(p) * c / parts);
+      leaf_id = p == 0 ? v : uint64_t(new_base[sg]) + p - 1;
+      local = rnk - lo;
+    };
+    auto put = [&](uint64_t id, uint32_t e, K key, K val) {
+      K* line = leaf + (id * F + e / P) * (2 * P);
+      line[e % P] = key;
+      line[P + e % P] = val;
+    };
+    // surviving old entries
+    for (uint32_t i = lane; i < c_old; i += 32) {
+      const bool del = s_del[w][i + 1] != s_del[w][i];
+      if (del) continue;
+      const K key = s_k[w][i];
+      uint32_t lo = o0, hi = o1;  // first op >= key
+      while (lo < hi) {
+        const uint32_t mid = (lo + hi) / 2;
+        if (ok[mid] < key) lo = mid + 1; else hi = mid;
+      }
+      // inserted ops with key < entry key = inserted among [o0, lo)
+      const uint32_t ins_before = insx[lo] - ins0;
+      const uint32_t r2 = (i - s_del[w][i]) + ins_before;
+      uint64_t id; uint32_t local;
+      dest(r2, id, local);
+      put(id, local, key, s_v[w][i]);
+    }
+    // inserted ops
+    for (uint32_t j = o0 + lane; j < o1; j += 32) {
+      const uint32_t l = lb[j];
+      const bool found = l < c_old && s_k[w][l] == ok[j];
+      if (oo[j] != 0 || found) continue;
+      const uint32_t r2 = (l - s_del[w][l]) + (insx[j] - ins0);
+      uint64_t id; uint32_t local;
+      dest(r2, id, local);
+      put(id, local, ok[j], ov[j]);
+    }
+    // padding + counts of every destination leaf
+    const uint32_t np = parts ? parts : 1;
+    for (uint32_t p = 0; p < np; ++p) {
+      const uint64_t id = p == 0 ? v : uint64_t(new_base[sg]) + p - 1;
+      const uint32_t cnt = parts ? uint32_t(uint64_t(p + 1) * c / parts - uint64_t(p) * c / parts) : 0;
+      for (uint32_t e = cnt + lane; e < B; e += 32) put(id, e, key_max<K>(), K(0));
+      if (lane == 0) {
+        count[id] = cnt;
+        dirty[id] = 1;
+      }
+    }
+    __syncwarp();
+  }
+}
+
+// new chain: position i of the old chain expands to its parts (0 if emptied)
+__global__ void chain_parts(const uint32_t* __restrict__ chain, uint64_t nchain, const uint32_t* __restrict__ seg_of_leaf,
+                            const uint32_t* __restrict__ new_cnt, uint32_t B, uint32_t* __restrict__ parts) {
+  GRID_STRIDE(i, nchain) {
+    const uint32_t s = seg_of_leaf[chain[i]];
+    if (s == kNoRef) parts[i] = 1;
+    else parts[i] = new_cnt[s] == 0 ? 0 : (new_cnt[s] + B - 1) / B;
+  }
+}
+
+__global__ void chain_write(const uint32_t* __restrict__ chain, uint64_t nchain, const uint32_t* __restrict__ seg_of_leaf,
+                            const uint32_t* __restrict__ parts, const uint32_t* __restrict__ pos,
+                            const uint32_t* __restrict__ new_base, uint32_t* __restrict__ out) {
+  GRID_STRIDE(i, nchain) {
+    const uint32_t v = chain[i];
+    const uint32_t s = seg_of_leaf[v];
+    for (uint32_t p = 0; p < parts[i]; ++p) out[pos[i] + p] = p == 0 ? v : new_base[s] + p - 1;
+  }
+}
+
+__global__ void reset_seg_of_leaf(const uint32_t* __restrict__ seg_leaf, uint64_t nseg, uint32_t* __restrict__ seg_of_leaf) {
+  GRID_STRIDE(s, nseg) seg_of_leaf[seg_leaf[s]] = kNoRef;
+}
+
+__global__ void add_base(uint32_t* __restrict__ x, uint64_t n, uint64_t base) {
+  GRID_STRIDE(i, n) x[i] = uint32_t(x[i] + base);
+}
+
+template <typename K>
+__global__ void clear_leaf0(K* leaf, uint32_t* count, uint32_t* chain, uint32_t F, uint8_t* dirty) {
+  constexpr uint32_t P = Geo<K>::P;
+  for (uint32_t e = threadIdx.x; e < F * P; e += blockDim.x) {
+    leaf[(e / P) * (2 * P) + e % P] = key_max<K>();
+    leaf[(e / P) * (2 * P) + P + e % P] = K(0);
+  }
+  if (threadIdx.x == 0) { count[0] = 0; chain[0] = 0; dirty[0] = 1; }
+}
+
+__global__ void chain_count_sum(const uint32_t* __restrict__ chain, uint64_t nchain, const uint32_t* __restrict__ count,
+                                unsigned long long* __restrict__ sum) {
+  unsigned long long local = 0;
+  GRID_STRIDE(i, nchain) local += count[chain[i]];
+  if (local) atomicAdd(sum, local);
+}
+
+struct DevBuf {
+  void* p = nullptr;
+  ~DevBuf() { cudaFree(p); }
+  template <typename T> T* as() { return static_cast<T*>(p); }
+};
+
+template <typename K>
+int update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
+  RegularState& r = t->r;
+  const uint32_t F = t->F, B = r.B;
+  const uint64_t m0 = b->count;
+  if (m0 >= (1ull << 32)) { set_error("batch too large"); return HBT_EUNSUPPORTED; }
+  // 1. sort ops by key (stable), last op per key wins
+  DevBuf sk, sidx, idx, flags, tmp, dk, didx, dv, dop, nsel;
+  HBT_CUDA_TRY(cudaMalloc(&sk.p, m0 * sizeof(K)));
+  HBT_CUDA_TRY(cudaMalloc(&idx.p, m0 * 4));
+  HBT_CUDA_TRY(cudaMalloc(&sidx.p, m0 * 4));
+  HBT_CUDA_TRY(cudaMalloc(&flags.p, m0));
+  HBT_CUDA_TRY(cudaMalloc(&dk.p, m0 * sizeof(K)));
+  HBT_CUDA_TRY(cudaMalloc(&didx.p, m0 * 4));
+  HBT_CUDA_TRY(cudaMalloc(&dv.p, m0 * sizeof(K)));
+  HBT_CUDA_TRY(cudaMalloc(&dop.p, m0));
+  HBT_CUDA_TRY(cudaMalloc(&nsel.p, 8));
+  iota_u32<<<grid_for(m0), 256, 0, s>>>(idx.as<uint32_t>(), m0);
+  size_t tb = 0, tb2 = 0;
+  HBT_CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb, (const K*)b->keys, sk.as<K>(), idx.as<uint32_t>(),
+                                               sidx.as<uint32_t>(), m0, 0, int(8 * sizeof(K)), s));
+  HBT_CUDA_TRY(cub::DeviceSelect::Flagged(nullptr, tb2, sk.as<K>(), flags.as<uint8_t>(), dk.as<K>(),
+                                          nsel.as<int64_t>(), int64_t(m0), s));
+  if (tb2 > tb) tb = tb2;
+  HBT_CUDA_TRY(cudaMalloc(&tmp.p, tb));
+  HBT_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp.p, tb, (const K*)b->keys, sk.as<K>(), idx.as<uint32_t>(),
+                                               sidx.as<uint32_t>(), m0, 0, int(8 * sizeof(K)), s));
+  last_of_run<K><<<grid_for(m0), 256, 0, s>>>(sk.as<K>(), m0, flags.as<uint8_t>());
+  HBT_CUDA_TRY(cub::DeviceSelect::Flagged(tmp.p, tb, sk.as<K>(), flags.as<uint8_t>(), dk.as<K>(), nsel.as<int64_t>(),
+                                          int64_t(m0), s));
+  HBT_CUDA_TRY(cub::DeviceSelect::Flagged(tmp.p, tb, sidx.as<uint32_t>(), flags.as<uint8_t>(), didx.as<uint32_t>(),
+                                          nsel.as<int64_t>(), int64_t(m0), s));
+  int64_t hm = 0;
+  HBT_CUDA_TRY(cudaMemcpyAsync(&hm, nsel.p, 8, cudaMemcpyDeviceToHost, s));
+  HBT_CUDA_TRY(cudaStreamSynchronize(s));
+  const uint64_t m = uint64_t(hm);
+  gather_ops<K><<<grid_for(m), 256, 0, s>>>(didx.as<uint32_t>(), m, (const K*)b->values, b->ops, dv.as<K>(),
+                                            dop.as<uint8_t>());
+  // 2. locate each op's big leaf through the pre-update tree
+  DevBuf leaf_of, start, incl, seg_off, seg_leaf, seg_delta, lb, ins, insx, new_cnt, extra, new_base, dirty;
+  HBT_CUDA_TRY(cudaMalloc(&leaf_of.p, m * 4));
+  const uint32_t root_leaf = r.root_leaf;
+  locate_leaf<K><<<grid_for(m), 256, 0, s>>>(dk.as<K>(), m, (const K*)r.d_ukeys, (const K*)r.d_uidx, r.d_urefs,
+                                             r.U ? r.uoff[r.U] - 1 : 0, r.U, root_leaf, F, leaf_of.as<uint32_t>());
+  // 3. segments of ops per leaf (ops are in key order, so are their leaves)
+  HBT_CUDA_TRY(cudaMalloc(&start.p, m * 4));
+  HBT_CUDA_TRY(cudaMalloc(&incl.p, m * 4));
+  segment_flags<<<grid_for(m), 256, 0, s>>>(leaf_of.as<uint32_t>(), m, start.as<uint32_t>());
+  tb2 = 0;
+  HBT_CUDA_TRY(cub::DeviceScan::InclusiveSum(nullptr, tb2, start.as<uint32_t>(), incl.as<uint32_t>(), m, s));
+  DevBuf tmp2;
+  HBT_CUDA_TRY(cudaMalloc(&tmp2.p, tb2 + 256));
+  HBT_CUDA_TRY(cub::DeviceScan::InclusiveSum(tmp2.p, tb2, start.as<uint32_t>(), incl.as<uint32_t>(), m, s));
+  uint32_t nseg32 = 0;
+  HBT_CUDA_TRY(cudaMemcpyAsync(&nseg32, incl.as<uint32_t>() + (m - 1), 4, cudaMemcpyDeviceToHost, s));
+  HBT_CUDA_TRY(cudaStreamSynchronize(s));
+  const uint64_t nseg = nseg32;
+  HBT_CUDA_TRY(cudaMalloc(&seg_off.p, (nseg + 1) * 4));
+  HBT_CUDA_TRY(cudaMalloc(&seg_leaf.p, nseg * 4));
+  HBT_CUDA_TRY(cudaMalloc(&seg_delta.p, nseg * 4));
+  HBT_CUDA_TRY(cudaMemsetAsync(seg_delta.p, 0, nseg * 4, s));
+  segment_tables<<<grid_for(m), 256, 0, s>>>(leaf_of.as<uint32_t>(), incl.as<uint32_t>(), m, seg_off.as<uint32_t>(),
+                                             seg_leaf.as<uint32_t>(), r.d_seg_of_leaf);
+  // 4. classify ops against their leaf; new counts; new pool indices (key order)
+  HBT_CUDA_TRY(cudaMalloc(&lb.p, m * 4));
+  HBT_CUDA_TRY(cudaMalloc(&ins.p, (m + 1) * 4));
+  HBT_CUDA_TRY(cudaMalloc(&insx.p, (m + 1) * 4));
+  HBT_CUDA_TRY(cudaMemsetAsync(ins.p, 0, (m + 1) * 4, s));
+  op_classify<K><<<grid_for(m), 256, 0, s>>>(dk.as<K>(), dop.as<uint8_t>(), m, leaf_of.as<uint32_t>(),
+                                             incl.as<uint32_t>(), (const K*)r.d_leaf, r.d_count, F, lb.as<uint32_t>(),
+                                             ins.as<uint32_t>(), seg_delta.as<int>());
+  HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb2, ins.as<uint32_t>(), insx.as<uint32_t>(), m + 1, s));
+  DevBuf tmp3;
+  HBT_CUDA_TRY(cudaMalloc(&tmp3.p, tb2 + 256));
+  HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp3.p, tb2, ins.as<uint32_t>(), insx.as<uint32_t>(), m + 1, s));
+  HBT_CUDA_TRY(cudaMalloc(&new_cnt.p, nseg * 4));
+  HBT_CUDA_TRY(cudaMalloc(&extra.p, nseg * 4));
+  HBT_CUDA_TRY(cudaMalloc(&new_base.p, (nseg + 1) * 4));
+  segment_counts<<<grid_for(nseg), 256, 0, s>>>(seg_leaf.as<uint32_t>(), seg_delta.as<int>(), nseg, r.d_count, B,
+                                                new_cnt.as<uint32_t>(), extra.as<uint32_t>());
+  DevBuf tmp4;
+  HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb2, extra.as<uint32_t>(), new_base.as<uint32_t>(), nseg + 0, s));
+  HBT_CUDA_TRY(cudaMalloc(&tmp4.p, tb2 + 256));
+  HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp4.p, tb2, extra.as<uint32_t>(), new_base.as<uint32_t>(), nseg, s));
+  uint32_t last_base = 0, last_extra = 0;
+  HBT_CUDA_TRY(cudaMemcpyAsync(&last_base, new_base.as<uint32_t>() + nseg - 1, 4, cudaMemcpyDeviceToHost, s));
+  HBT_CUDA_TRY(cudaMemcpyAsync(&last_extra, extra.as<uint32_t>() + nseg - 1, 4, cudaMemcpyDeviceToHost, s));
+  HBT_CUDA_TRY(cudaStreamSynchronize(s));
+  const uint64_t n_new = uint64_t(last_base) + last_extra;
+  const uint64_t old_pool = r.pool;
+  if (old_pool + n_new >= (1ull << 32) - 1) { set_error("pool index overflow"); return HBT_EUNSUPPORTED; }
+  add_base<<<grid_for(nseg), 256, 0, s>>>(new_base.as<uint32_t>(), nseg, old_pool);
+  int rc = grow_pool<K>(t, old_pool + n_new, s);
+  if (rc != HBT_OK) return rc;
+  r.pool = old_pool + n_new;
+  HBT_CUDA_TRY(cudaMalloc(&dirty.p, r.pool));
+  HBT_CUDA_TRY(cudaMemsetAsync(dirty.p, 0, r.pool, s));
+  // 5. merge + split + pad, one warp per affected leaf
+  {
+    constexpr int MAXB = 32 * Geo<K>::P;  // F <= 32
+    const uint64_t blocks = (nseg + 3) / 4;
+    merge_write<K, MAXB><<<unsigned(blocks < 148 * 64 ? blocks : 148 * 64), 128, 0, s>>>(
+        seg_leaf.as<uint32_t>(), seg_off.as<uint32_t>(), nseg, new_cnt.as<uint32_t>(), new_base.as<uint32_t>(),
+        dk.as<K>(), dv.as<K>(), dop.as<uint8_t>(), lb.as<uint32_t>(), insx.as<uint32_t>(), (K*)r.d_leaf, r.d_count,
+        dirty.as<uint8_t>(), F);
+    HBT_CUDA_TRY(cudaGetLastError());
+  }
+  // 6. new chain (key order): every old position expands to its parts
+  DevBuf parts, ppos, nchain_buf;
+  HBT_CUDA_TRY(cudaMalloc(&parts.p, (r.nchain + 1) * 4));
+  HBT_CUDA_TRY(cudaMalloc(&ppos.p, (r.nchain + 1) * 4));
+  chain_parts<<<grid_for(r.nchain), 256, 0, s>>>(r.d_chain, r.nchain, r.d_seg_of_leaf, new_cnt.as<uint32_t>(), B,
+                                                 parts.as<uint32_t>());
+  DevBuf tmp5;
+  HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb2, parts.as<uint32_t>(), ppos.as<uint32_t>(), r.nchain, s));
+  HBT_CUDA_TRY(cudaMalloc(&tmp5.p, tb2 + 256));
+  HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp5.p, tb2, parts.as<uint32_t>(), ppos.as<uint32_t>(), r.nchain, s));
+  uint32_t lp = 0, lpart = 0;
+  HBT_CUDA_TRY(cudaMemcpyAsync(&lp, ppos.as<uint32_t>() + r.nchain - 1, 4, cudaMemcpyDeviceToHost, s));
+  HBT_CUDA_TRY(cudaMemcpyAsync(&lpart, parts.as<uint32_t>() + r.nchain - 1, 4, cudaMemcpyDeviceToHost, s));
+  HBT_CUDA_TRY(cudaStreamSynchronize(s));
+  const uint64_t new_nchain = uint64_t(lp) + lpart;
+  HBT_CUDA_TRY(cudaMalloc(&nchain_buf.p, (new_nchain + 1) * 4));
+  chain_write<<<grid_for(r.nchain), 256, 0, s>>>(r.d_chain, r.nchain, r.d_seg_of_leaf, parts.as<uint32_t>(),
+                                                 ppos.as<uint32_t>(), new_base.as<uint32_t>(), nchain_buf.as<uint32_t>());
+  reset_seg_of_leaf<<<grid_for(nseg), 256, 0, s>>>(seg_leaf.as<uint32_t>(), nseg, r.d_seg_of_leaf);
+  if (new_nchain == 0) {  // every key deleted: the empty tree (one empty leaf at index 0)
+    r.pool = 1;
+    clear_leaf0<K><<<1, 256, 0, s>>>((K*)r.d_leaf, r.d_count, r.d_chain, F, dirty.as<uint8_t>());
+    r.nchain = 1;
+  } else {
+    HBT_CUDA_TRY(cudaMemcpyAsync(r.d_chain, nchain_buf.p, new_nchain * 4, cudaMemcpyDeviceToDevice, s));
+    r.nchain = new_nchain;
+  }
+  // 7. refresh the last-level inner nodes of dirty leaves, then the upper levels
+  derive_last_level<K><<<grid_for(r.pool), 256, 0, s>>>((const K*)r.d_leaf, r.d_count, r.pool, F, dirty.as<uint8_t>(),
+                                                         (K*)r.d_lkeys, (K*)r.d_lidx);
+  HBT_CUDA_TRY(cudaGetLastError());
+  HBT_CUDA_TRY(cudaStreamSynchronize(s));
+  HBT_CUDA_TRY(cudaMemcpyAsync(&r.root_leaf, r.d_chain, 4, cudaMemcpyDeviceToHost, s));
+  HBT_CUDA_TRY(cudaStreamSynchronize(s));
+  rc = rebuild_upper<K>(t, s);
+  if (rc != HBT_OK) return rc;
+  // live key count n' = sum of the chain's counts
+  {
+    DevBuf sum;
+    HBT_CUDA_TRY(cudaMalloc(&sum.p, 8));
+    HBT_CUDA_TRY(cudaMemsetAsync(sum.p, 0, 8, s));
+    chain_count_sum<<<grid_for(r.nchain), 256, 0, s>>>(r.d_chain, r.nchain, r.d_count, sum.as<unsigned long long>());
+    uint64_t nn = 0;
+    HBT_CUDA_TRY(cudaMemcpyAsync(&nn, sum.p, 8, cudaMemcpyDeviceToHost, s));
+    HBT_CUDA_TRY(cudaStreamSynchronize(s));
+    t->n = nn;
+  }
+  return HBT_OK;
+}
+
+}  // namespace
+
+int regular_build(hbt_tree* t, const void* keys, const void* values, uint64_t n, cudaStream_t s) {
+  int rc = t->width == 4 ? build_t<uint32_t>(t, keys, values, n, s) : build_t<uint64_t>(t, keys, values, n, s);
+  if (rc != HBT_OK) return rc;
+  // pool-sized map leaf -> update segment (kept at "none" between updates)
+  HBT_CUDA_TRY(cudaMalloc(&t->r.d_seg_of_leaf, t->r.cap * 4));
+  HBT_CUDA_TRY(cudaMemset(t->r.d_seg_of_leaf, 0xFF, t->r.cap * 4));
+  t->r.seg_cap = t->r.cap;
+  return HBT_OK;
+}
+
+int regular_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+  if (m == 0) return HBT_OK;
+  return t->width == 4 ? search_t<uint32_t>(t, q, m, pf, v, s) : search_t<uint64_t>(t, q, m, pf, v, s);
+}
+
+int regular_update(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
+  RegularState& r = t->r;
+  // the leaf->segment map must cover the pool after growth: size it for the worst case
+  const uint64_t worst = r.pool + b->count + 1;
+  if (worst > r.seg_cap) {
+    uint32_t* nm = nullptr;
+    HBT_CUDA_TRY(cudaMalloc(&nm, worst * 4));
+    HBT_CUDA_TRY(cudaMemset(nm, 0xFF, worst * 4));
+    cudaFree(r.d_seg_of_leaf);
+    r.d_seg_of_leaf = nm;
+    r.seg_cap = worst;
+  }
+  return t->width == 4 ? update_t<uint32_t>(t, b, s) : update_t<uint64_t>(t, b, s);
+}
+
+void regular_free(hbt_tree* t) {
+  RegularState& r = t->r;
+  cudaFree(r.d_leaf); cudaFree(r.d_count); cudaFree(r.d_lkeys); cudaFree(r.d_lidx); cudaFree(r.d_chain);
+  cudaFree(r.d_ukeys); cudaFree(r.d_uidx); cudaFree(r.d_urefs); cudaFree(r.d_seg_of_leaf);
+  r = RegularState{};
+}
+
+uint32_t regular_smem_levels(const hbt_tree* t, uint32_t budget) {
+  if (!budget) budget = 100 * 1024;
+  return t->width == 4 ? smem_levels_t<uint32_t>(t, budget) : smem_levels_t<uint64_t>(t, budget);
+}
+
+}  // namespace hbt
