@@ -120,7 +120,9 @@ enum {
   HBT_SEG_UPPER_KEYS = 5,  /* regular: upper pool x F keys                                        */
   HBT_SEG_UPPER_IDX = 6,   /* regular: upper pool x NI index entries                              */
   HBT_SEG_UPPER_REFS = 7,  /* regular: upper pool x F uint32 child references                     */
-  HBT_SEG_CHAIN = 8        /* regular: uint32 big-leaf pool indices in key order                  */
+  HBT_SEG_CHAIN = 8,       /* regular: uint32 big-leaf pool indices in key order                  */
+  HBT_SEG_INNER_IDX = 9    /* implicit: per-node index sector (max key of each 32 B key sector,
+                              MAX-padded to max(16, F*S/32*S) bytes) for nodes wider than 32 B   */
 };
 
 /* Build a tree from n (key, value) pairs.  keys/values: device
@@ -156,10 +158,13 @@ HBT_API int hbt_info(const hbt_tree* t, hbt_info_t* info);
  * `bytes` bytes (HBT_EINVAL if too small); *written receives the byte count. */
 HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t bytes, uint64_t* written);
 
-/* Override the shared-memory budget (bytes per CTA) and query tiling of the
- * search kernel; 0 keeps the default.  For tuning and tests. */
+/* Override the search kernel's launch shape; 0 keeps the default.  smem_bytes:
+ * shared-memory budget per CTA for the pinned top levels (<= 227 KB);
+ * threads_per_cta: 256 or 512; ctas_per_sm: cap on resident CTAs per SM;
+ * queries_per_lane: 1 or 2 queries per lane per warp round (memory-level
+ * parallelism).  For tuning and tests; results never depend on it. */
 HBT_API int hbt_set_search_config(hbt_tree* t, uint32_t smem_bytes, uint32_t threads_per_cta,
-                          uint32_t ctas_per_sm);
+                                  uint32_t ctas_per_sm, uint32_t queries_per_lane);
 
 HBT_API const char* hbt_last_error(void);
 /* Library version string, e.g. "hbt 0.1 sm_100a". */

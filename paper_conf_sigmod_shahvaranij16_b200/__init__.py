@@ -31,7 +31,7 @@ POS_END = 0x7FFFFFFFFFFFFFFF
 FOUND_BIT = 0x8000000000000000
 MAX_LEVELS = 32
 SEG_INNER, SEG_LEAF, SEG_COUNT, SEG_LAST_KEYS, SEG_LAST_IDX = 0, 1, 2, 3, 4
-SEG_UPPER_KEYS, SEG_UPPER_IDX, SEG_UPPER_REFS, SEG_CHAIN = 5, 6, 7, 8
+SEG_UPPER_KEYS, SEG_UPPER_IDX, SEG_UPPER_REFS, SEG_CHAIN, SEG_INNER_IDX = 5, 6, 7, 8, 9
 UPSERT, DELETE = 0, 1
 
 EXPORTED = ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
@@ -73,7 +73,7 @@ def _load():
     L.hbt_destroy.argtypes = [vp]
     L.hbt_info.argtypes = [vp, C.POINTER(_Info)]
     L.hbt_export.argtypes = [vp, u32, vp, u64, C.POINTER(u64)]
-    L.hbt_set_search_config.argtypes = [vp, u32, u32, u32]
+    L.hbt_set_search_config.argtypes = [vp, u32, u32, u32, u32]
     L.hbt_last_error.restype = C.c_char_p
     L.hbt_version.restype = C.c_char_p
     for f in ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
@@ -201,8 +201,9 @@ class Tree:
         _check(lib.hbt_export(self._h, segment, C.c_void_p(buf.ctypes.data), buf.nbytes, C.byref(need)))
         return buf[: need.value]
 
-    def set_search_config(self, smem_bytes: int = 0, threads_per_cta: int = 0, ctas_per_sm: int = 0):
-        _check(lib.hbt_set_search_config(self._h, smem_bytes, threads_per_cta, ctas_per_sm))
+    def set_search_config(self, smem_bytes: int = 0, threads_per_cta: int = 0, ctas_per_sm: int = 0,
+                          queries_per_lane: int = 0):
+        _check(lib.hbt_set_search_config(self._h, smem_bytes, threads_per_cta, ctas_per_sm, queries_per_lane))
 
 
 def unpack(pos_found, values, width: int):

@@ -37,6 +37,7 @@ static bool is_device_ptr(const void* p) {
 static void free_tree(hbt_tree* t) {
   if (!t) return;
   cudaFree(t->d_inner);
+  cudaFree(t->d_inner_idx);
   cudaFree(t->d_leaf);
   regular_free(t);
   cudaFree(t->pipe.d_q);
@@ -190,7 +191,7 @@ int hbt_info(const hbt_tree* t, hbt_info_t* info) {
     for (uint32_t d = 0; d < t->H; ++d) info->level_nodes[d] = t->nodes[d];
     info->leaf_lines = t->L0;
     info->chain_len = t->L0;
-    info->inner_bytes = t->inner_bytes;
+    info->inner_bytes = t->inner_bytes + t->inner_idx_bytes;
     info->leaf_bytes = t->leaf_bytes;
   } else {
     const RegularState& r = t->r;
@@ -216,6 +217,7 @@ int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t bytes, u
   if (t->form == HBT_IMPLICIT) {
     if (segment == HBT_SEG_INNER) { src = t->d_inner; len = t->inner_bytes; }
     else if (segment == HBT_SEG_LEAF) { src = t->d_leaf; len = t->leaf_bytes; }
+    else if (segment == HBT_SEG_INNER_IDX) { src = t->d_inner_idx; len = t->inner_idx_bytes; }
     else { set_error("segment %u not in an implicit tree", segment); return HBT_EINVAL; }
   } else {
     switch (segment) {
@@ -236,12 +238,19 @@ int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t bytes, u
   return HBT_OK;
 }
 
-int hbt_set_search_config(hbt_tree* t, uint32_t smem_bytes, uint32_t threads_per_cta, uint32_t ctas_per_sm) {
+int hbt_set_search_config(hbt_tree* t, uint32_t smem_bytes, uint32_t threads_per_cta, uint32_t ctas_per_sm,
+                          uint32_t queries_per_lane) {
   if (!t) return HBT_EINVAL;
   if (smem_bytes > 227 * 1024) { set_error("smem budget above 227 KB"); return HBT_EINVAL; }
   t->cfg.smem_budget = smem_bytes;
   t->cfg.threads = threads_per_cta;
+  if (threads_per_cta && threads_per_cta != 256 && threads_per_cta != 512) {
+    set_error("threads_per_cta must be 256 or 512");
+    return HBT_EINVAL;
+  }
+  if (queries_per_lane > 2) { set_error("queries_per_lane must be 0, 1 or 2"); return HBT_EINVAL; }
   t->cfg.ctas_per_sm = ctas_per_sm;
+  t->cfg.qpl = queries_per_lane;
   return HBT_OK;
 }
 

@@ -36,6 +36,7 @@ struct SearchConfig {
   uint32_t smem_budget = 0;      // bytes per CTA for pinned levels (0 = default)
   uint32_t threads = 0;          // threads per CTA (0 = default)
   uint32_t ctas_per_sm = 0;      // 0 = occupancy-derived
+  uint32_t qpl = 0;              // queries per lane per warp round (0 = default)
 };
 
 // Regular-tree device state.  All pools are SoA arrays
@@ -87,6 +88,11 @@ struct hbt_tree {
   uint64_t offset[HBT_MAX_LEVELS + 1] = {};  // root-first, node units
   void* d_inner = nullptr;
   uint64_t inner_bytes = 0;
+  // derived per-node index sector ("I_s = K_8s" applied to implicit nodes
+  // wider than one 32 B sector): entry t = max key of sector t, MAX-padded
+  void* d_inner_idx = nullptr;
+  uint64_t inner_idx_bytes = 0;
+  uint32_t idx_stride = 0;  // bytes of index per node (0 = nodes fit one sector)
   void* d_leaf = nullptr;
   uint64_t L0 = 0;
   uint64_t leaf_bytes = 0;
@@ -109,6 +115,8 @@ int implicit_update(hbt_tree* t, const hbt_batch* b, cudaStream_t s);
 // implicit_search.cu
 int implicit_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s);
 uint32_t implicit_smem_levels(const hbt_tree* t, uint32_t budget);
+// index bytes per implicit node (0 when F*S <= 32)
+uint32_t implicit_idx_stride(uint32_t F, uint32_t S);
 // regular_*.cu
 int regular_build(hbt_tree* t, const void* keys, const void* values, uint64_t n, cudaStream_t s);
 int regular_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s);

@@ -69,6 +69,21 @@ __global__ void gather_separators(const K* __restrict__ kd, uint64_t nd, const L
   }
 }
 
+// Index sector of every inner node: entry t = node key t*KPS + KPS - 1 (the max
+// key of the node's t-th 32 B sector), entries >= NSEC are MAX.
+template <typename K>
+__global__ void derive_inner_index(const K* __restrict__ inner, uint64_t nodes, uint32_t F, uint32_t idx_entries,
+                                   K* __restrict__ idx) {
+  constexpr uint32_t KPS = 32 / sizeof(K);
+  const uint32_t nsec = F / KPS;
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < nodes * idx_entries;
+       x += uint64_t(gridDim.x) * blockDim.x) {
+    const uint64_t node = x / idx_entries;
+    const uint32_t t = uint32_t(x % idx_entries);
+    idx[x] = t < nsec ? inner[node * F + t * KPS + KPS - 1] : key_max<K>();
+  }
+}
+
 template <typename K>
 __global__ void unpack_leaf_lines(const K* __restrict__ leaf, uint64_t nd, K* __restrict__ kd, K* __restrict__ vd) {
   constexpr uint32_t P = 64 / (2 * sizeof(K));
@@ -203,6 +218,15 @@ int build_sorted_t(hbt_tree* t, const K* kd, const K* vd, uint64_t nd, cudaStrea
     lt.H = H;
     gather_separators<K><<<grid_for(t->offset[H] * F), 256, 0, s>>>(kd, nd, lt, t->L0, F, (K*)t->d_inner);
     HBT_CUDA_TRY(cudaGetLastError());
+    t->idx_stride = implicit_idx_stride(F, sizeof(K));
+    if (t->idx_stride) {
+      const uint32_t ie = t->idx_stride / sizeof(K);
+      t->inner_idx_bytes = t->offset[H] * t->idx_stride;
+      HBT_CUDA_TRY(cudaMalloc(&t->d_inner_idx, t->inner_idx_bytes));
+      derive_inner_index<K><<<grid_for(t->offset[H] * ie), 256, 0, s>>>((const K*)t->d_inner, t->offset[H], F, ie,
+                                                                         (K*)t->d_inner_idx);
+      HBT_CUDA_TRY(cudaGetLastError());
+    }
   }
   HBT_CUDA_TRY(cudaStreamSynchronize(s));
   return HBT_OK;
@@ -268,15 +292,17 @@ int implicit_update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   nt.form = t->form; nt.width = t->width; nt.F = t->F; nt.device = t->device; nt.num_sms = t->num_sms;
   int rc = build_sorted_t<K>(&nt, kd, vd, uint64_t(h_nsel), s);
   cleanup();
-  if (rc != HBT_OK) { cudaFree(nt.d_leaf); cudaFree(nt.d_inner); return rc; }
+  if (rc != HBT_OK) { cudaFree(nt.d_leaf); cudaFree(nt.d_inner); cudaFree(nt.d_inner_idx); return rc; }
   cudaFree(t->d_leaf);
   cudaFree(t->d_inner);
+  cudaFree(t->d_inner_idx);
   t->n = nt.n; t->L0 = nt.L0; t->H = nt.H; t->P = nt.P;
   for (int d = 0; d < HBT_MAX_LEVELS; ++d) t->nodes[d] = nt.nodes[d];
   for (int d = 0; d <= HBT_MAX_LEVELS; ++d) t->offset[d] = nt.offset[d];
   t->d_leaf = nt.d_leaf; t->leaf_bytes = nt.leaf_bytes;
   t->d_inner = nt.d_inner; t->inner_bytes = nt.inner_bytes;
-  nt.d_leaf = nt.d_inner = nullptr;
+  t->d_inner_idx = nt.d_inner_idx; t->inner_idx_bytes = nt.inner_idx_bytes; t->idx_stride = nt.idx_stride;
+  nt.d_leaf = nt.d_inner = nt.d_inner_idx = nullptr;
   return HBT_OK;
 }
 

@@ -1,19 +1,27 @@
 // implicit_search.cu — hbt_search for the IMPLICIT tree (the hot path).
 //
-// One lane GROUP of G = max(2, F*S/16) lanes searches one node: each lane loads
-// 16 B (8 B for 16-byte nodes) of the node with one vector load and the group
-// counts the node keys smaller than q with __ballot_sync + __popc:
-//   i = #{t : sep[t] < q} = the minimum i with q <= sep[i]   (PAPER.md:190,
-//       read with the "k is the minimum i" comments of P:520 / P:566; R1)
-// and descends to child node*F + i (Snippet 3's (nodeIndex+result)<<3,
-// P:689).  No shared flags and no barriers (Snippet 3 needs two __syncthreads
-// per level).  Each group keeps QPG queries in flight level-
-// synchronously (the GPU form of the paper's software pipelining, Alg. 2,
-// P:600-612), so a warp has 32 independent node loads outstanding per level.
-// The top SL levels are staged once per persistent CTA in shared memory (the
-// I-segment-in-fast-memory principle of P:178); deeper levels and the leaf line
-// come from L2/HBM with read-only loads; queries and results stream with
-// evict-first (.cs) accesses so they do not displace the tree from L2.
+// Node search = "the minimum i such that q <= sep[i]" = #{t : sep[t] < q}
+// (PAPER.md:190 read with the comments of Snippets 1/2, P:520 / P:566; reading
+// R1), then descend to child node*F + i (Snippet 3's
+// (nodeIndex+result)<<3).  Two phases per warp round of 32*QPL queries:
+//
+//  1. Shared-memory levels (the top SL levels, staged once per persistent CTA —
+//     the I-segment-in-fast-memory principle of P:178): ONE lane per query runs
+//     a branchless binary search over the node's F sorted keys (log2 F probes,
+//     each one LDS; the last key is MAX, so no size is needed).
+//  2. L2/HBM levels: a GROUP of G = 2 (4 for 256-byte nodes) lanes per query.
+//     A node wider than one 32 B sector is read through its index sector
+//     (entry t = max key of sector t, the paper's index line of P:134 applied
+//     to implicit nodes): t = popc(ballot(idx < q)), then ONLY key sector t is
+//     read: i = t*KPS + popc(ballot(key < q)).  So a level moves 64 B instead of
+//     F*S bytes, with 16 B vector loads, no divergence and no barriers (Snippet
+//     3 needs two __syncthreads per level).  Each group keeps QPG
+//     queries in flight level-synchronously (the GPU form of the software
+//     pipelining of Alg. 2).
+//  Leaf: the 64 B line [P keys | P values] is read by the group in one round
+//  trip; s = popc(ballot(key < q)); r = line*P + s; found = r < n' && key[s] == q.
+// Queries and results stream with evict-first (.cs) accesses so they do not
+// displace the tree from L2.
 #include "hbt_internal.cuh"
 
 namespace hbt {
@@ -25,39 +33,21 @@ constexpr uint64_t kFound = HBT_FOUND_BIT;
 template <typename K>
 __device__ __forceinline__ K key_max() { return K(~K(0)); }
 
-template <typename K, int BYTES>
-struct Chunk {
-  static constexpr int N = BYTES / int(sizeof(K));
-  K k[N];
+template <typename K>
+union V16 {
+  uint4 u;
+  K k[16 / sizeof(K)];
 };
 
-template <typename K, int BYTES>
-__device__ __forceinline__ void ld_global(Chunk<K, BYTES>& c, const uint8_t* p) {
-  if constexpr (BYTES == 8) {
-    uint2 v = __ldg(reinterpret_cast<const uint2*>(p));
-    memcpy(&c, &v, 8);
-  } else if constexpr (BYTES == 16) {
-    uint4 v = __ldg(reinterpret_cast<const uint4*>(p));
-    memcpy(&c, &v, 16);
-  } else {
-    static_assert(BYTES == 32, "chunk size");
-    uint4 v0 = __ldg(reinterpret_cast<const uint4*>(p));
-    uint4 v1 = __ldg(reinterpret_cast<const uint4*>(p) + 1);
-    memcpy(&c, &v0, 16);
-    memcpy(reinterpret_cast<uint8_t*>(&c) + 16, &v1, 16);
-  }
+template <typename K>
+__device__ __forceinline__ void ld16(V16<K>& v, const uint8_t* p) {
+  v.u = __ldg(reinterpret_cast<const uint4*>(p));
 }
 
-template <typename K, int BYTES>
-__device__ __forceinline__ void ld_shared(Chunk<K, BYTES>& c, const uint8_t* p) {
-  if constexpr (BYTES == 8) {
-    uint2 v = *reinterpret_cast<const uint2*>(p);
-    memcpy(&c, &v, 8);
-  } else {
-    static_assert(BYTES == 16, "chunk size");
-    uint4 v = *reinterpret_cast<const uint4*>(p);
-    memcpy(&c, &v, 16);
-  }
+template <typename K>
+__device__ __forceinline__ void fill_max(V16<K>& v) {
+#pragma unroll
+  for (int e = 0; e < int(16 / sizeof(K)); ++e) v.k[e] = key_max<K>();
 }
 
 __device__ __forceinline__ uint32_t ldcs(const uint32_t* p) { return __ldcs(p); }
@@ -69,30 +59,25 @@ __device__ __forceinline__ void stcs(uint64_t* p, uint64_t v) {
   __stcs(reinterpret_cast<unsigned long long*>(p), (unsigned long long)v);
 }
 
-template <typename K, int F, int QPG_>
+template <typename K, int F>
 struct Cfg {
   static constexpr int S = int(sizeof(K));
   static constexpr int NODE_BYTES = F * S;
-  static constexpr int G = NODE_BYTES / 16 < 2 ? 2 : NODE_BYTES / 16;  // lanes per group
-  static constexpr int LANE_BYTES = NODE_BYTES / G;                    // 8 or 16
-  static constexpr int NG = 32 / G;                                    // groups per warp
-  static constexpr int QPG = QPG_;                                     // queries in flight per group
-  static constexpr int ROUND = NG * QPG;                               // queries per warp round
-  static constexpr int P = 64 / (2 * S);                               // pairs per leaf line
-  static constexpr int LL = G < 4 ? G : 4;                             // lanes loading a leaf line
-  static constexpr int LB = 64 / LL;                                   // leaf bytes per lane
-  static constexpr int KEY_LANES = LL / 2;                             // lanes holding the key half
-  static constexpr int LK = LB / S;                                    // leaf entries per lane
-  static_assert(QPG <= G && ROUND <= 32, "tiling");
+  static constexpr int KPS = 32 / S;                                      // keys per 32 B sector
+  static constexpr int NSEC = NODE_BYTES >= 32 ? NODE_BYTES / 32 : 1;     // sectors per node
+  static constexpr bool HAS_IDX = NSEC > 1;
+  static constexpr int IDXB = HAS_IDX ? (NSEC * S > 16 ? NSEC * S : 16) : 0;  // index bytes per node
+  static constexpr int IL = IDXB / 16;                                    // lanes loading the index
+  static constexpr int SECB = NODE_BYTES < 32 ? NODE_BYTES : 32;          // bytes read after the index
+  static constexpr int SL_ = SECB / 16;                                   // lanes loading them
+  static constexpr int G = IL > 2 ? IL : 2;                               // lanes per query group
+  static constexpr int NG = 32 / G;                                       // groups per warp
+  static constexpr int P = 64 / (2 * S);                                  // pairs per leaf line
+  static constexpr int LL = G < 4 ? G : 4;                                // lanes loading a leaf line
+  static constexpr int LB = 64 / LL;                                      // leaf bytes per lane (32|16)
+  static constexpr int KEY_LANES = LL / 2;                                // lanes holding the keys
+  static constexpr int LK = LB / S;                                       // leaf entries per lane
 };
-
-template <typename K, int N>
-__device__ __forceinline__ uint32_t count_less(const K (&k)[N], K q, unsigned gmask) {
-  uint32_t c = 0;
-#pragma unroll
-  for (int t = 0; t < N; ++t) c += __popc(__ballot_sync(0xffffffffu, k[t] < q) & gmask);
-  return c;
-}
 
 template <typename K, int N>
 __device__ __forceinline__ K pick(const K (&k)[N], uint32_t slot) {
@@ -102,12 +87,23 @@ __device__ __forceinline__ K pick(const K (&k)[N], uint32_t slot) {
   return r;
 }
 
-template <typename K, int F, int QPG, int THREADS>
+template <typename K>
+__device__ __forceinline__ uint32_t count_less16(const V16<K>& v, K q, unsigned gmask) {
+  uint32_t c = 0;
+#pragma unroll
+  for (int e = 0; e < int(16 / sizeof(K)); ++e) c += __popc(__ballot_sync(0xffffffffu, v.k[e] < q) & gmask);
+  return c;
+}
+
+template <typename K, int F, int QPL, int THREADS>
 __global__ void __launch_bounds__(THREADS)
-implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ leaf,
-                       const K* __restrict__ queries, uint64_t m, uint64_t* __restrict__ out_pf,
-                       K* __restrict__ out_v, const LevelTable lt, uint64_t n) {
-  using C = Cfg<K, F, QPG>;
+implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ inner_idx,
+                       const uint8_t* __restrict__ leaf, const K* __restrict__ queries, uint64_t m,
+                       uint64_t* __restrict__ out_pf, K* __restrict__ out_v, const LevelTable lt, uint64_t n) {
+  using C = Cfg<K, F>;
+  constexpr int ROUND = 32 * QPL;        // queries per warp round (QPL per lane in phase 1)
+  constexpr int QPG = ROUND / C::NG;     // queries per group in phase 2
+  static_assert(QPG % C::G == 0, "every group lane stores QPG/G results");
   extern __shared__ __align__(16) uint8_t smem[];
   const uint32_t SL = lt.SL, H = lt.H;
   {  // stage the top SL levels (root-first, contiguous) once per persistent CTA
@@ -117,100 +113,143 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
     for (uint32_t i = threadIdx.x; i < vecs; i += THREADS) dst[i] = __ldg(src + i);
   }
   __syncthreads();
+  const K* s_keys = reinterpret_cast<const K*>(smem);
 
   const int lane = threadIdx.x & 31;
   const int g = lane / C::G, k = lane % C::G;
   const unsigned gmask = ((1u << C::G) - 1u) << (g * C::G);
   const uint64_t warp = (uint64_t(blockIdx.x) * THREADS + threadIdx.x) >> 5;
   const uint64_t nwarps = (uint64_t(gridDim.x) * THREADS) >> 5;
-  const uint64_t rounds = (m + C::ROUND - 1) / C::ROUND;
+  const uint64_t rounds = (m + ROUND - 1) / ROUND;
 
   for (uint64_t rd = warp; rd < rounds; rd += nwarps) {
-    // Query j of group g is query base + j*NG + g: lane (g, k<QPG) loads query
-    // k of its group, so the warp's load and store are one coalesced segment.
-    const uint64_t my_i = rd * C::ROUND + uint64_t(k) * C::NG + g;
-    const bool my_ok = (k < QPG) && (my_i < m);
-    const K myq = my_ok ? ldcs(queries + my_i) : key_max<K>();
+    const uint64_t base = rd * ROUND;
+    // ---- phase 1: one lane per query; coalesced query loads
+    K myq[QPL];
+    uint32_t mynode[QPL];
+#pragma unroll
+    for (int u = 0; u < QPL; ++u) {
+      const uint64_t i = base + uint64_t(u) * 32 + lane;
+      myq[u] = i < m ? ldcs(queries + i) : key_max<K>();
+      mynode[u] = 0;
+    }
+    for (uint32_t d = 0; d < SL; ++d) {
+      const K* lvl = s_keys + lt.offset[d] * F;
+      uint32_t pos[QPL];
+#pragma unroll
+      for (int u = 0; u < QPL; ++u) pos[u] = 0;
+#pragma unroll
+      for (int step = F / 2; step >= 1; step /= 2) {
+#pragma unroll
+        for (int u = 0; u < QPL; ++u)
+          pos[u] += (lvl[mynode[u] * F + pos[u] + step - 1] < myq[u]) ? uint32_t(step) : 0u;
+      }
+#pragma unroll
+      for (int u = 0; u < QPL; ++u) mynode[u] = mynode[u] * F + pos[u];
+    }
+    // ---- phase 2: lane groups; slot j of group g is round query j*NG + g,
+    //      owned in phase 1 by lane (j*NG)%32 + g, slot (j*NG)/32
     K q[QPG];
     uint32_t node[QPG];
 #pragma unroll
     for (int j = 0; j < QPG; ++j) {
-      q[j] = __shfl_sync(0xffffffffu, myq, g * C::G + j);
-      node[j] = 0;
+      const int src = (j * C::NG) % 32 + g;
+      q[j] = __shfl_sync(0xffffffffu, myq[(j * C::NG) / 32], src);
+      node[j] = __shfl_sync(0xffffffffu, mynode[(j * C::NG) / 32], src);
     }
-    // ---- inner levels pinned in shared memory
-    for (uint32_t d = 0; d < SL; ++d) {
-      const uint8_t* lvl = smem + uint32_t(lt.offset[d]) * C::NODE_BYTES + k * C::LANE_BYTES;
-      Chunk<K, C::LANE_BYTES> c[QPG];
-#pragma unroll
-      for (int j = 0; j < QPG; ++j) ld_shared(c[j], lvl + node[j] * C::NODE_BYTES);
-#pragma unroll
-      for (int j = 0; j < QPG; ++j) node[j] = node[j] * F + count_less(c[j].k, q[j], gmask);
-    }
-    // ---- inner levels in L2 / HBM
     for (uint32_t d = SL; d < H; ++d) {
-      const uint8_t* lvl = inner + lt.offset[d] * C::NODE_BYTES + k * C::LANE_BYTES;
-      Chunk<K, C::LANE_BYTES> c[QPG];
+      const uint8_t* lvl = inner + lt.offset[d] * C::NODE_BYTES;
+      uint32_t sec[QPG];
+      if constexpr (C::HAS_IDX) {
+        const uint8_t* lidx = inner_idx + lt.offset[d] * C::IDXB;
+        V16<K> iv[QPG];
 #pragma unroll
-      for (int j = 0; j < QPG; ++j) ld_global(c[j], lvl + uint64_t(node[j]) * C::NODE_BYTES);
+        for (int j = 0; j < QPG; ++j) {
+          if (k < C::IL) ld16(iv[j], lidx + uint64_t(node[j]) * C::IDXB + k * 16);
+          else fill_max(iv[j]);
+        }
 #pragma unroll
-      for (int j = 0; j < QPG; ++j) node[j] = node[j] * F + count_less(c[j].k, q[j], gmask);
+        for (int j = 0; j < QPG; ++j) sec[j] = count_less16(iv[j], q[j], gmask);
+      } else {
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) sec[j] = 0;
+      }
+      V16<K> kv[QPG];
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) {
+        if (k < C::SL_) ld16(kv[j], lvl + uint64_t(node[j]) * C::NODE_BYTES + sec[j] * 32 + k * 16);
+        else fill_max(kv[j]);
+      }
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) node[j] = node[j] * F + sec[j] * C::KPS + count_less16(kv[j], q[j], gmask);
     }
     // ---- leaf line: lanes [0, KEY_LANES) hold the P keys, [KEY_LANES, LL) the P values
-    Chunk<K, C::LB> lc[QPG];
+    K lk[QPG][C::LK];
 #pragma unroll
     for (int j = 0; j < QPG; ++j) {
       if (k < C::LL) {
-        ld_global(lc[j], leaf + uint64_t(node[j]) * 64 + k * C::LB);
+        const uint8_t* p = leaf + uint64_t(node[j]) * 64 + k * C::LB;
+#pragma unroll
+        for (int h = 0; h < C::LB / 16; ++h) {
+          V16<K> v;
+          ld16(v, p + h * 16);
+#pragma unroll
+          for (int e = 0; e < 16 / C::S; ++e) lk[j][h * (16 / C::S) + e] = v.k[e];
+        }
       } else {
 #pragma unroll
-        for (int t = 0; t < C::LK; ++t) lc[j].k[t] = key_max<K>();
+        for (int e = 0; e < C::LK; ++e) lk[j][e] = key_max<K>();
       }
     }
-    uint64_t my_pf = 0;
-    K my_v = 0;
+    uint64_t my_pf[QPG / C::G];
+    K my_v[QPG / C::G];
 #pragma unroll
     for (int j = 0; j < QPG; ++j) {
       uint32_t s = 0;
 #pragma unroll
-      for (int t = 0; t < C::LK; ++t)
-        s += __popc(__ballot_sync(0xffffffffu, (k < C::KEY_LANES) && (lc[j].k[t] < q[j])) & gmask);
+      for (int e = 0; e < C::LK; ++e)
+        s += __popc(__ballot_sync(0xffffffffu, (k < C::KEY_LANES) && (lk[j][e] < q[j])) & gmask);
       const uint32_t sc = s < uint32_t(C::P) ? s : uint32_t(C::P - 1);
-      const K sel = pick(lc[j].k, sc % C::LK);
+      const K sel = pick(lk[j], sc % C::LK);
       const int src = g * C::G + int(sc / C::LK);
       const K key_s = __shfl_sync(0xffffffffu, sel, src);
       const K val_s = __shfl_sync(0xffffffffu, sel, src + C::KEY_LANES);
       const uint64_t r = uint64_t(node[j]) * C::P + s;
       const bool found = (s < uint32_t(C::P)) && (r < n) && (key_s == q[j]);
-      if (j == k) {
-        my_pf = (r < n ? r : kEnd) | (found ? kFound : 0ull);
-        my_v = found ? val_s : K(0);
+      if (j % C::G == k) {
+        my_pf[j / C::G] = (r < n ? r : kEnd) | (found ? kFound : 0ull);
+        my_v[j / C::G] = found ? val_s : K(0);
       }
     }
-    if (my_ok) {
-      stcs(out_pf + my_i, my_pf);
-      stcs(out_v + my_i, my_v);
+    // lane (g, k) stores slots j = k + G*t: round queries (k + G*t)*NG + g
+#pragma unroll
+    for (int t = 0; t < QPG / C::G; ++t) {
+      const uint64_t i = base + uint64_t(k + C::G * t) * C::NG + g;
+      if (i < m) {
+        stcs(out_pf + i, my_pf[t]);
+        stcs(out_v + i, my_v[t]);
+      }
     }
   }
 }
 
-constexpr int kThreads = 512;
-
 template <typename K, int F>
 struct Launch {
-  static constexpr int G = Cfg<K, F, 1>::G;
-  static constexpr int QPG = G < 8 ? G : 8;
-  using C = Cfg<K, F, QPG>;
+  using C = Cfg<K, F>;
 
-  static auto kernel() { return implicit_search_kernel<K, F, QPG, kThreads>; }
+  static uint32_t smem_levels(const hbt_tree* t, uint32_t budget) {
+    uint32_t SL = 0;
+    while (SL < t->H && t->offset[SL + 1] * uint64_t(C::NODE_BYTES) <= budget) ++SL;
+    return SL;
+  }
 
-  static int run(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
-    auto kern = kernel();
+  template <int QPL, int THREADS>
+  static int run_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+    auto kern = implicit_search_kernel<K, F, QPL, THREADS>;
     LevelTable lt{};
     for (uint32_t d = 0; d <= t->H; ++d) lt.offset[d] = t->offset[d];
     lt.H = t->H;
-    const uint32_t budget = t->cfg.smem_budget ? t->cfg.smem_budget : default_budget();
-    lt.SL = smem_levels(t, budget);
+    lt.SL = smem_levels(t, t->cfg.smem_budget ? t->cfg.smem_budget : 100 * 1024);
     const size_t smem = size_t(lt.offset[lt.SL]) * C::NODE_BYTES;
     static bool attr_set = false;  // per instantiation
     if (!attr_set) {
@@ -218,29 +257,24 @@ struct Launch {
       attr_set = true;
     }
     int occ = 0;
-    HBT_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, smem));
+    HBT_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, THREADS, smem));
     if (t->cfg.ctas_per_sm && int(t->cfg.ctas_per_sm) < occ) occ = int(t->cfg.ctas_per_sm);
     if (occ < 1) occ = 1;
-    const uint64_t rounds = (m + C::ROUND - 1) / C::ROUND;
-    const uint64_t warps_per_cta = kThreads / 32;
+    const uint64_t rounds = (m + 32 * QPL - 1) / (32 * QPL);
     uint64_t grid = uint64_t(t->num_sms) * occ;
-    const uint64_t need = (rounds + warps_per_cta - 1) / warps_per_cta;
+    const uint64_t need = (rounds + THREADS / 32 - 1) / (THREADS / 32);
     if (need < grid) grid = need ? need : 1;
-    kern<<<unsigned(grid), kThreads, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_leaf,
-                                                (const K*)q, m, pf, (K*)v, lt, t->n);
+    kern<<<unsigned(grid), THREADS, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
+                                               (const uint8_t*)t->d_leaf, (const K*)q, m, pf, (K*)v, lt, t->n);
     HBT_CUDA_TRY(cudaGetLastError());
     return HBT_OK;
   }
 
-  static uint32_t default_budget() {
-    // Two resident CTAs per SM share the 228 KB carve-out.
-    return 100 * 1024;
-  }
-
-  static uint32_t smem_levels(const hbt_tree* t, uint32_t budget) {
-    uint32_t SL = 0;
-    while (SL < t->H && t->offset[SL + 1] * uint64_t(C::NODE_BYTES) <= budget) ++SL;
-    return SL;
+  static int run(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+    const uint32_t qpl = t->cfg.qpl ? t->cfg.qpl : 1;
+    const uint32_t th = t->cfg.threads ? t->cfg.threads : 512;
+    if (qpl == 2) return th == 256 ? run_t<2, 256>(t, q, m, pf, v, s) : run_t<2, 512>(t, q, m, pf, v, s);
+    return th == 256 ? run_t<1, 256>(t, q, m, pf, v, s) : run_t<1, 512>(t, q, m, pf, v, s);
   }
 };
 
@@ -268,6 +302,13 @@ uint32_t smem_levels_f(const hbt_tree* t, uint32_t budget) {
 }
 
 }  // namespace
+
+uint32_t implicit_idx_stride(uint32_t F, uint32_t S) {
+  const uint32_t node = F * S;
+  if (node <= 32) return 0;
+  const uint32_t b = (node / 32) * S;
+  return b > 16 ? b : 16;
+}
 
 int implicit_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
   if (m == 0) return HBT_OK;

@@ -41,6 +41,7 @@ def test_edge_suite_parity(hbt, width, F):
         inner, leaf = expected_implicit_bytes(o, width)
         assert t.export(hbt.SEG_INNER).tobytes() == inner, (n, F, width)
         assert t.export(hbt.SEG_LEAF).tobytes() == leaf, (n, F, width)
+        assert t.export(hbt.SEG_INNER_IDX).tobytes() == expected_index_bytes(o, width), (n, F, width)
         q = query_set(k, width, rng, 3000)
         pf, val = gpu_search(t, q, width)
         epf, ev = o.search(q)
@@ -49,16 +50,36 @@ def test_edge_suite_parity(hbt, width, F):
         t.close()
 
 
-@pytest.mark.parametrize("budget", [16, 4096, 100 * 1024, 200 * 1024])
-def test_smem_pinning_variants(hbt, budget):
-    """Results must not depend on how many top levels sit in shared memory."""
-    width, F = 8, 16
-    rng = np.random.default_rng(budget)
+def expected_index_bytes(o, width):
+    """Per-node index sector derived from the oracle's nodes: entry t = the max
+    key of the node's t-th 32 B sector (PAPER.md:134's I_s applied to implicit
+    nodes), MAX-padded to max(16, NSEC*S) bytes; empty when F*S <= 32."""
+    a = o.arrays()
+    F = a["F"]
+    node_bytes = F * width
+    if node_bytes <= 32 or a["H"] == 0:
+        return b""
+    kps = 32 // width
+    nsec = node_bytes // 32
+    ent = max(16, nsec * width) // width
+    inner = a["inner"]
+    idx = np.full((inner.shape[0], ent), (1 << (8 * width)) - 1, dtype=np.uint64)
+    idx[:, :nsec] = inner[:, kps - 1::kps][:, :nsec]
+    return idx.astype(np_dtype(width)).tobytes()
+
+
+@pytest.mark.parametrize("width,F", [(8, 16), (4, 8), (8, 32), (4, 32)])
+@pytest.mark.parametrize("budget,threads,qpl", [(16, 0, 0), (4096, 256, 2), (100 * 1024, 512, 1),
+                                                (200 * 1024, 512, 2), (64 * 1024, 256, 1)])
+def test_launch_shape_variants(hbt, width, F, budget, threads, qpl):
+    """Results must not depend on how many top levels sit in shared memory, the
+    CTA size or the queries in flight per lane."""
+    rng = np.random.default_rng(budget + threads + qpl + F)
     k, v = gen_keys(300000, width, rng)
     o = oracle.ITree.from_pairs(k, v, F, width)
     t = gpu_build(hbt, k, v, F, width)
-    t.set_search_config(smem_bytes=budget)
-    q = query_set(k[:5000], width, rng, 20000)
+    t.set_search_config(smem_bytes=budget, threads_per_cta=threads, queries_per_lane=qpl)
+    q = query_set(k[:5000], width, rng, 20011)
     pf, val = gpu_search(t, q, width)
     epf, ev = o.search(q)
     assert np.array_equal(pf, epf) and np.array_equal(val, ev)
