@@ -43,6 +43,10 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--smem", type=int, default=0, help="override smem budget (bytes)")
+    ap.add_argument("--qpl", type=int, default=0, help="queries per lane per warp round (1|2)")
+    ap.add_argument("--threads", type=int, default=0, help="threads per CTA (256|512)")
+    ap.add_argument("--smem-mode", type=int, default=0, help="0 = key words, 1 = hi/lo planes")
+    ap.add_argument("--carveout", type=int, default=-1, help="smem carve-out percent (-1 default)")
     return ap.parse_args()
 
 
@@ -159,8 +163,8 @@ def run_hbt(args):
     keys, vals, q, hit_rate, qdesc = make_workload(args.config, rank, g)
     m = q.numel()
     tree = hbt.Tree(keys, vals, fanout=c["fanout"], layout=c["layout"])
-    if args.smem:
-        tree.set_search_config(smem_bytes=args.smem)
+    tree.set_search_config(smem_bytes=args.smem, threads_per_cta=args.threads, queries_per_lane=args.qpl,
+                           smem_mode=args.smem_mode, carveout=args.carveout)
     info = tree.info()
     del keys, vals
     out_pos = torch.empty(m, dtype=torch.int64, device="cuda")

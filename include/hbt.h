@@ -158,13 +158,16 @@ HBT_API int hbt_info(const hbt_tree* t, hbt_info_t* info);
  * `bytes` bytes (HBT_EINVAL if too small); *written receives the byte count. */
 HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t bytes, uint64_t* written);
 
-/* Override the search kernel's launch shape; 0 keeps the default.  smem_bytes:
- * shared-memory budget per CTA for the pinned top levels (<= 227 KB);
- * threads_per_cta: 256 or 512; ctas_per_sm: cap on resident CTAs per SM;
- * queries_per_lane: 1 or 2 queries per lane per warp round (memory-level
- * parallelism).  For tuning and tests; results never depend on it. */
-HBT_API int hbt_set_search_config(hbt_tree* t, uint32_t smem_bytes, uint32_t threads_per_cta,
-                                  uint32_t ctas_per_sm, uint32_t queries_per_lane);
+/* Tune the search kernel's launch shape on one tree; results never depend on
+ * it.  name / value:
+ *   "smem_bytes"  shared-memory budget per CTA for the pinned top levels (<= 227 KB; 0 = default 100 KB)
+ *   "threads"     threads per CTA: 256 or 512 (0 = default 512)
+ *   "ctas_per_sm" cap on resident CTAs per SM (0 = occupancy-derived)
+ *   "qpl"         queries per lane per warp round, 1 or 2 (0 = default)
+ *   "smem_mode"   0 = probe S-byte keys, 1 = probe 32-bit hi/lo planes (64-bit keys)
+ *   "carveout"    preferred shared-memory carve-out percent, -1 = driver default
+ * Unknown names or out-of-range values return HBT_EINVAL. */
+HBT_API int hbt_set_param(hbt_tree* t, const char* name, int64_t value);
 
 HBT_API const char* hbt_last_error(void);
 /* Library version string, e.g. "hbt 0.1 sm_100a". */

@@ -35,7 +35,7 @@ SEG_UPPER_KEYS, SEG_UPPER_IDX, SEG_UPPER_REFS, SEG_CHAIN, SEG_INNER_IDX = 5, 6, 
 UPSERT, DELETE = 0, 1
 
 EXPORTED = ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
-            "hbt_info", "hbt_export", "hbt_set_search_config", "hbt_last_error", "hbt_version"]
+            "hbt_info", "hbt_export", "hbt_set_param", "hbt_last_error", "hbt_version"]
 
 
 class HBTError(RuntimeError):
@@ -73,11 +73,11 @@ def _load():
     L.hbt_destroy.argtypes = [vp]
     L.hbt_info.argtypes = [vp, C.POINTER(_Info)]
     L.hbt_export.argtypes = [vp, u32, vp, u64, C.POINTER(u64)]
-    L.hbt_set_search_config.argtypes = [vp, u32, u32, u32, u32]
+    L.hbt_set_param.argtypes = [vp, C.c_char_p, C.c_int64]
     L.hbt_last_error.restype = C.c_char_p
     L.hbt_version.restype = C.c_char_p
     for f in ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
-              "hbt_info", "hbt_export", "hbt_set_search_config"]:
+              "hbt_info", "hbt_export", "hbt_set_param"]:
         getattr(L, f).restype = C.c_int
     return L
 
@@ -201,9 +201,14 @@ class Tree:
         _check(lib.hbt_export(self._h, segment, C.c_void_p(buf.ctypes.data), buf.nbytes, C.byref(need)))
         return buf[: need.value]
 
+    def set_param(self, name: str, value: int):
+        _check(lib.hbt_set_param(self._h, name.encode(), int(value)))
+
     def set_search_config(self, smem_bytes: int = 0, threads_per_cta: int = 0, ctas_per_sm: int = 0,
-                          queries_per_lane: int = 0):
-        _check(lib.hbt_set_search_config(self._h, smem_bytes, threads_per_cta, ctas_per_sm, queries_per_lane))
+                          queries_per_lane: int = 0, smem_mode: int = 0, carveout: int = -1):
+        for k, v in [("smem_bytes", smem_bytes), ("threads", threads_per_cta), ("ctas_per_sm", ctas_per_sm),
+                     ("qpl", queries_per_lane), ("smem_mode", smem_mode), ("carveout", carveout)]:
+            self.set_param(k, v)
 
 
 def unpack(pos_found, values, width: int):

@@ -238,19 +238,20 @@ int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t bytes, u
   return HBT_OK;
 }
 
-int hbt_set_search_config(hbt_tree* t, uint32_t smem_bytes, uint32_t threads_per_cta, uint32_t ctas_per_sm,
-                          uint32_t queries_per_lane) {
-  if (!t) return HBT_EINVAL;
-  if (smem_bytes > 227 * 1024) { set_error("smem budget above 227 KB"); return HBT_EINVAL; }
-  t->cfg.smem_budget = smem_bytes;
-  t->cfg.threads = threads_per_cta;
-  if (threads_per_cta && threads_per_cta != 256 && threads_per_cta != 512) {
-    set_error("threads_per_cta must be 256 or 512");
+int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
+  if (!t || !name) { set_error("NULL argument"); return HBT_EINVAL; }
+  const std::string n(name);
+  SearchConfig& c = t->cfg;
+  if (n == "smem_bytes" && value >= 0 && value <= 227 * 1024) c.smem_budget = uint32_t(value);
+  else if (n == "threads" && (value == 0 || value == 256 || value == 512)) c.threads = uint32_t(value);
+  else if (n == "ctas_per_sm" && value >= 0 && value <= 32) c.ctas_per_sm = uint32_t(value);
+  else if (n == "qpl" && value >= 0 && value <= 2) c.qpl = uint32_t(value);
+  else if (n == "smem_mode" && (value == 0 || value == 1)) c.mode = uint32_t(value);
+  else if (n == "carveout" && value >= -1 && value <= 100) c.carveout = int(value);
+  else {
+    set_error("bad parameter %s = %lld", name, (long long)value);
     return HBT_EINVAL;
   }
-  if (queries_per_lane > 2) { set_error("queries_per_lane must be 0, 1 or 2"); return HBT_EINVAL; }
-  t->cfg.ctas_per_sm = ctas_per_sm;
-  t->cfg.qpl = queries_per_lane;
   return HBT_OK;
 }
 

@@ -37,6 +37,8 @@ struct SearchConfig {
   uint32_t threads = 0;          // threads per CTA (0 = default)
   uint32_t ctas_per_sm = 0;      // 0 = occupancy-derived
   uint32_t qpl = 0;              // queries per lane per warp round (0 = default)
+  uint32_t mode = 0;             // smem probe mode: 0 = K words, 1 = hi/lo 32-bit planes
+  int carveout = -1;             // shared-memory carve-out percent (-1 = driver default)
 };
 
 // Regular-tree device state.  All pools are SoA arrays

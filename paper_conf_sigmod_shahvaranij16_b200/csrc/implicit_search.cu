@@ -95,7 +95,7 @@ __device__ __forceinline__ uint32_t count_less16(const V16<K>& v, K q, unsigned 
   return c;
 }
 
-template <typename K, int F, int QPL, int THREADS>
+template <typename K, int F, int QPL, int THREADS, int MODE>
 __global__ void __launch_bounds__(THREADS)
 implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ inner_idx,
                        const uint8_t* __restrict__ leaf, const K* __restrict__ queries, uint64_t m,
@@ -106,14 +106,23 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
   static_assert(QPG % C::G == 0, "every group lane stores QPG/G results");
   extern __shared__ __align__(16) uint8_t smem[];
   const uint32_t SL = lt.SL, H = lt.H;
-  {  // stage the top SL levels (root-first, contiguous) once per persistent CTA
-    const uint32_t vecs = uint32_t(lt.offset[SL] * C::NODE_BYTES / 16);
-    const uint4* src = reinterpret_cast<const uint4*>(inner);
-    uint4* dst = reinterpret_cast<uint4*>(smem);
-    for (uint32_t i = threadIdx.x; i < vecs; i += THREADS) dst[i] = __ldg(src + i);
+  // Stage the top SL levels (root-first, contiguous) once per persistent CTA.
+  // MODE 1 splits 64-bit keys into 32-bit hi / lo planes (a probe reads one
+  // 4-byte bank per plane); MODE 0 keeps the node array as is.
+  const uint32_t s_n = uint32_t(lt.offset[SL]) * F;  // staged keys
+  K* s_keys = reinterpret_cast<K*>(smem);
+  uint32_t* s_hi = reinterpret_cast<uint32_t*>(smem);
+  uint32_t* s_lo = s_hi + s_n;
+  for (uint32_t i = threadIdx.x; i < s_n; i += THREADS) {
+    const K key = __ldg(reinterpret_cast<const K*>(inner) + i);
+    if constexpr (MODE == 1 && sizeof(K) == 8) {
+      s_hi[i] = uint32_t(uint64_t(key) >> 32);
+      s_lo[i] = uint32_t(key);
+    } else {
+      s_keys[i] = key;
+    }
   }
   __syncthreads();
-  const K* s_keys = reinterpret_cast<const K*>(smem);
 
   const int lane = threadIdx.x & 31;
   const int g = lane / C::G, k = lane % C::G;
@@ -134,15 +143,25 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
       mynode[u] = 0;
     }
     for (uint32_t d = 0; d < SL; ++d) {
-      const K* lvl = s_keys + lt.offset[d] * F;
+      const uint32_t lvl = uint32_t(lt.offset[d]) * F;
       uint32_t pos[QPL];
 #pragma unroll
       for (int u = 0; u < QPL; ++u) pos[u] = 0;
 #pragma unroll
       for (int step = F / 2; step >= 1; step /= 2) {
 #pragma unroll
-        for (int u = 0; u < QPL; ++u)
-          pos[u] += (lvl[mynode[u] * F + pos[u] + step - 1] < myq[u]) ? uint32_t(step) : 0u;
+        for (int u = 0; u < QPL; ++u) {
+          const uint32_t a = lvl + mynode[u] * F + pos[u] + step - 1;
+          bool lt_;
+          if constexpr (MODE == 1 && sizeof(K) == 8) {
+            const uint32_t qh = uint32_t(uint64_t(myq[u]) >> 32), ql = uint32_t(myq[u]);
+            const uint32_t kh = s_hi[a], kl = s_lo[a];
+            lt_ = (kh < qh) | ((kh == qh) & (kl < ql));
+          } else {
+            lt_ = s_keys[a] < myq[u];
+          }
+          pos[u] += lt_ ? uint32_t(step) : 0u;
+        }
       }
 #pragma unroll
       for (int u = 0; u < QPL; ++u) mynode[u] = mynode[u] * F + pos[u];
@@ -243,18 +262,24 @@ struct Launch {
     return SL;
   }
 
-  template <int QPL, int THREADS>
+  template <int QPL, int THREADS, int MODE>
   static int run_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
-    auto kern = implicit_search_kernel<K, F, QPL, THREADS>;
+    auto kern = implicit_search_kernel<K, F, QPL, THREADS, MODE>;
     LevelTable lt{};
     for (uint32_t d = 0; d <= t->H; ++d) lt.offset[d] = t->offset[d];
     lt.H = t->H;
     lt.SL = smem_levels(t, t->cfg.smem_budget ? t->cfg.smem_budget : 100 * 1024);
-    const size_t smem = size_t(lt.offset[lt.SL]) * C::NODE_BYTES;
+    const size_t smem = size_t(lt.offset[lt.SL]) * C::NODE_BYTES;  // both MODEs use F*S bytes per node
     static bool attr_set = false;  // per instantiation
     if (!attr_set) {
       HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
       attr_set = true;
+    }
+    static int carve = -2;  // per instantiation: last carve-out applied
+    if (carve != t->cfg.carveout) {
+      HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                        t->cfg.carveout >= 0 ? t->cfg.carveout : int(cudaSharedmemCarveoutDefault)));
+      carve = t->cfg.carveout;
     }
     int occ = 0;
     HBT_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, THREADS, smem));
@@ -271,10 +296,15 @@ struct Launch {
   }
 
   static int run(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
-    const uint32_t qpl = t->cfg.qpl ? t->cfg.qpl : 1;
+    const uint32_t qpl = t->cfg.qpl ? t->cfg.qpl : 2;
     const uint32_t th = t->cfg.threads ? t->cfg.threads : 512;
-    if (qpl == 2) return th == 256 ? run_t<2, 256>(t, q, m, pf, v, s) : run_t<2, 512>(t, q, m, pf, v, s);
-    return th == 256 ? run_t<1, 256>(t, q, m, pf, v, s) : run_t<1, 512>(t, q, m, pf, v, s);
+    const bool hilo = t->cfg.mode == 1;
+    if (qpl == 2) {
+      if (hilo) return th == 256 ? run_t<2, 256, 1>(t, q, m, pf, v, s) : run_t<2, 512, 1>(t, q, m, pf, v, s);
+      return th == 256 ? run_t<2, 256, 0>(t, q, m, pf, v, s) : run_t<2, 512, 0>(t, q, m, pf, v, s);
+    }
+    if (hilo) return th == 256 ? run_t<1, 256, 1>(t, q, m, pf, v, s) : run_t<1, 512, 1>(t, q, m, pf, v, s);
+    return th == 256 ? run_t<1, 256, 0>(t, q, m, pf, v, s) : run_t<1, 512, 0>(t, q, m, pf, v, s);
   }
 };
 

@@ -69,16 +69,18 @@ def expected_index_bytes(o, width):
 
 
 @pytest.mark.parametrize("width,F", [(8, 16), (4, 8), (8, 32), (4, 32)])
-@pytest.mark.parametrize("budget,threads,qpl", [(16, 0, 0), (4096, 256, 2), (100 * 1024, 512, 1),
-                                                (200 * 1024, 512, 2), (64 * 1024, 256, 1)])
-def test_launch_shape_variants(hbt, width, F, budget, threads, qpl):
+@pytest.mark.parametrize("budget,threads,qpl,mode", [(16, 0, 0, 0), (4096, 256, 2, 1), (100 * 1024, 512, 1, 0),
+                                                     (200 * 1024, 512, 2, 1), (64 * 1024, 256, 1, 1),
+                                                     (100 * 1024, 512, 2, 0)])
+def test_launch_shape_variants(hbt, width, F, budget, threads, qpl, mode):
     """Results must not depend on how many top levels sit in shared memory, the
     CTA size or the queries in flight per lane."""
-    rng = np.random.default_rng(budget + threads + qpl + F)
+    rng = np.random.default_rng(budget + threads + qpl + F + mode)
     k, v = gen_keys(300000, width, rng)
     o = oracle.ITree.from_pairs(k, v, F, width)
     t = gpu_build(hbt, k, v, F, width)
-    t.set_search_config(smem_bytes=budget, threads_per_cta=threads, queries_per_lane=qpl)
+    t.set_search_config(smem_bytes=budget, threads_per_cta=threads, queries_per_lane=qpl, smem_mode=mode,
+                        carveout=100 if mode else -1)
     q = query_set(k[:5000], width, rng, 20011)
     pf, val = gpu_search(t, q, width)
     epf, ev = o.search(q)
