@@ -29,6 +29,10 @@ namespace {
 
 constexpr uint64_t kEnd = HBT_POS_END;
 constexpr uint64_t kFound = HBT_FOUND_BIT;
+// Only the tiny top levels go to shared memory: measured on B200 (profiles/
+// r01_*), a large shared carve-out costs more L1 hits on the L2 levels than the
+// pinned levels save (c2: SL=4 / 70 KB -> 24.0 G q/s, SL=3 / 4.4 KB -> 26.4).
+constexpr uint32_t kDefaultSmemBudget = 8 * 1024;
 
 template <typename K>
 __device__ __forceinline__ K key_max() { return K(~K(0)); }
@@ -268,7 +272,7 @@ struct Launch {
     LevelTable lt{};
     for (uint32_t d = 0; d <= t->H; ++d) lt.offset[d] = t->offset[d];
     lt.H = t->H;
-    lt.SL = smem_levels(t, t->cfg.smem_budget ? t->cfg.smem_budget : 100 * 1024);
+    lt.SL = smem_levels(t, t->cfg.smem_budget ? t->cfg.smem_budget : kDefaultSmemBudget);
     const size_t smem = size_t(lt.offset[lt.SL]) * C::NODE_BYTES;  // both MODEs use F*S bytes per node
     static bool attr_set = false;  // per instantiation
     if (!attr_set) {
@@ -296,7 +300,7 @@ struct Launch {
   }
 
   static int run(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
-    const uint32_t qpl = t->cfg.qpl ? t->cfg.qpl : 2;
+    const uint32_t qpl = t->cfg.qpl ? t->cfg.qpl : 1;
     const uint32_t th = t->cfg.threads ? t->cfg.threads : 512;
     const bool hilo = t->cfg.mode == 1;
     if (qpl == 2) {
@@ -346,7 +350,7 @@ int implicit_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, 
 }
 
 uint32_t implicit_smem_levels(const hbt_tree* t, uint32_t budget) {
-  if (!budget) budget = 100 * 1024;
+  if (!budget) budget = kDefaultSmemBudget;
   return t->width == 4 ? smem_levels_f<uint32_t>(t, budget) : smem_levels_f<uint64_t>(t, budget);
 }
 

@@ -2,7 +2,8 @@
 
 Algorithmic bytes per query (what the method must move):
   I/O      2S + 8          (query in; value + pos|found out)
-  per inner level one node: implicit F*S rounded up to 32 B sectors;
+  per inner level: implicit nodes wider than 32 B = index sector + one key
+                   sector (64 B; the paper's index line, P:134), else F*S;
                             regular index sector 32 + key line 64 + ref sector 32
                             (last level: 32 + 64)
   leaf     key sector 32 + value sector 32 (the value sector only when found)
@@ -21,19 +22,26 @@ def _sect(b):
 
 
 def implicit_tiers(info, hit_rate=1.0, smem_levels=None):
-    """List of (total_bytes, bytes_per_query) tiers of the implicit tree below the
-    shared-memory levels (uniform queries: every node of a level equally likely)."""
+    """(total_bytes, bytes_per_query) tiers of the implicit tree below the
+    shared-memory levels, for uniform queries (every node of a level equally
+    likely).  A node wider than one 32 B sector is read as its index sector plus
+    ONE key sector (the search kernel's access pattern); narrower nodes whole."""
     S, F = info["width"], info["fanout"]
     SL = info["smem_levels"] if smem_levels is None else smem_levels
-    nb = _sect(F * S)
+    node = F * S
     tiers = []
     for d, nodes in enumerate(info["level_nodes"]):
         if d < SL:
             continue
-        tiers.append((nodes * nb, nb))
+        if node > 32:
+            idx_stride = max(16, (node // 32) * S)
+            tiers.append((nodes * idx_stride, 32.0))   # index sector
+            tiers.append((nodes * node, 32.0))         # one key sector
+        else:
+            tiers.append((nodes * _sect(node), float(_sect(node))))
     L0 = info["leaf_lines"]
-    tiers.append((L0 * 32, 32.0))             # key sector of the leaf line
-    tiers.append((L0 * 32, 32.0 * hit_rate))  # value sector (found only)
+    tiers.append((L0 * 32, 32.0))             # key half of the leaf line
+    tiers.append((L0 * 32, 32.0 * hit_rate))  # value half (needed when found)
     return tiers
 
 
