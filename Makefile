@@ -4,6 +4,7 @@ ARCH      := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS   := -O3 -std=c++17 $(ARCH) -lineinfo -Xcompiler -fPIC -Xcompiler -fvisibility=hidden \
              --expt-relaxed-constexpr -diag-suppress 177 -cudart static
 PKG       := paper_conf_sigmod_shahvaranij16_b200
+NCCL_HOME ?= $(shell python -c "import nvidia.nccl, os; print(os.path.dirname(nvidia.nccl.__file__) if nvidia.nccl.__file__ else list(nvidia.nccl.__path__)[0])" 2>/dev/null)
 CSRC      := $(wildcard $(PKG)/csrc/*.cu)
 HDRS      := $(wildcard $(PKG)/csrc/*.cuh) include/hbt.h
 OBJDIR    := build/obj
@@ -13,10 +14,11 @@ all: $(PKG)/libhbt.so gen/libhbtgen.so oracle/liboracle.so tools/libhbtprobe.so
 
 $(OBJDIR)/%.o: $(PKG)/csrc/%.cu $(HDRS)
 	@mkdir -p $(OBJDIR)
-	$(NVCC) $(NVFLAGS) -Xcompiler -DHBT_BUILDING -c $< -o $@
+	$(NVCC) $(NVFLAGS) -I$(NCCL_HOME)/include -Xcompiler -DHBT_BUILDING -c $< -o $@
 
 $(PKG)/libhbt.so: $(OBJS)
-	$(NVCC) $(ARCH) -shared -cudart static -o $@ $(OBJS)
+	$(NVCC) $(ARCH) -shared -cudart static -o $@ $(OBJS) -L$(NCCL_HOME)/lib -l:libnccl.so.2 \
+	  -Xlinker -rpath -Xlinker $(NCCL_HOME)/lib
 
 gen/libhbtgen.so: gen/gen.cu
 	$(NVCC) -O3 -std=c++17 $(ARCH) -Xcompiler -fPIC -shared -cudart static -o $@ $<

@@ -169,6 +169,39 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  * Unknown names or out-of-range values return HBT_EINVAL. */
 HBT_API int hbt_set_param(hbt_tree* t, const char* name, int64_t value);
 
+/* ---- key-range sharding over G GPUs (one process per GPU), SURVEY §8(e) ----
+ * Shard g holds a contiguous key range; shards are numbered in key order (the
+ * keys of shard g are all larger than those of every non-empty shard < g; keys
+ * may be unsorted within a shard).  A query goes to owner(q) = #(shard_max < q)
+ * over the non-empty shards (the max-separator rule of the node search applied
+ * above the shard roots), is searched there, and its result comes back to the
+ * rank that asked; pos is GLOBAL: the shard's first global rank + local rank.
+ * Implicit trees only. */
+typedef struct hbt_comm hbt_comm;
+
+/* ncclGetUniqueId into a 128-byte buffer (rank 0; broadcast it to all ranks). */
+HBT_API int hbt_comm_unique_id(void* id128);
+/* ncclCommInitRank over nranks processes (one GPU each, current device). */
+HBT_API int hbt_comm_init(int nranks, int rank, const void* id128, hbt_comm** out);
+HBT_API int hbt_comm_destroy(hbt_comm* c);
+/* Collective: every rank builds its shard from its local (device) pairs, then the
+ * ranks all-gather (n', min, max).  HBT_EINVAL if shard ranges overlap. */
+HBT_API int hbt_bulk_build_sharded(hbt_comm* c, const void* keys_local, const void* values_local,
+                                   uint64_t n_local, uint32_t fanout, uint32_t layout, void* stream,
+                                   hbt_tree** out);
+/* Collective: every rank searches its local batch; queries and results cross
+ * NVLink by NCCL send/recv (an all-to-all).  Host-synchronous on the count
+ * exchange (one small D2H per batch). */
+HBT_API int hbt_search_sharded(const hbt_tree* t, const void* queries_local, uint64_t m_local,
+                               hbt_out out_local, void* stream);
+/* Single-process shard group on ONE device (tests, capacity planning): mark G
+ * implicit trees built from key-ordered disjoint ranges as shards 0..G-1 ... */
+HBT_API int hbt_shard_local_init(hbt_tree* const* shards, int G);
+/* ... and run the sharded search for G query batches with the same route /
+ * search / unpermute kernels, the exchange being device-to-device copies. */
+HBT_API int hbt_search_sharded_local(hbt_tree* const* shards, int G, const void* const* queries,
+                                     const uint64_t* m, const hbt_out* outs, void* stream);
+
 HBT_API const char* hbt_last_error(void);
 /* Library version string, e.g. "hbt 0.1 sm_100a". */
 HBT_API const char* hbt_version(void);

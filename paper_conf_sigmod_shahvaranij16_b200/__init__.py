@@ -35,7 +35,9 @@ SEG_UPPER_KEYS, SEG_UPPER_IDX, SEG_UPPER_REFS, SEG_CHAIN, SEG_INNER_IDX = 5, 6, 
 UPSERT, DELETE = 0, 1
 
 EXPORTED = ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
-            "hbt_info", "hbt_export", "hbt_set_param", "hbt_last_error", "hbt_version"]
+            "hbt_info", "hbt_export", "hbt_set_param", "hbt_last_error", "hbt_version",
+            "hbt_comm_unique_id", "hbt_comm_init", "hbt_comm_destroy", "hbt_bulk_build_sharded",
+            "hbt_search_sharded", "hbt_shard_local_init", "hbt_search_sharded_local"]
 
 
 class HBTError(RuntimeError):
@@ -74,10 +76,20 @@ def _load():
     L.hbt_info.argtypes = [vp, C.POINTER(_Info)]
     L.hbt_export.argtypes = [vp, u32, vp, u64, C.POINTER(u64)]
     L.hbt_set_param.argtypes = [vp, C.c_char_p, C.c_int64]
+    L.hbt_comm_unique_id.argtypes = [vp]
+    L.hbt_comm_init.argtypes = [C.c_int, C.c_int, vp, C.POINTER(vp)]
+    L.hbt_comm_destroy.argtypes = [vp]
+    L.hbt_bulk_build_sharded.argtypes = [vp, vp, vp, u64, u32, u32, vp, C.POINTER(vp)]
+    L.hbt_search_sharded.argtypes = [vp, vp, u64, _Out, vp]
+    L.hbt_shard_local_init.argtypes = [C.POINTER(vp), C.c_int]
+    L.hbt_search_sharded_local.argtypes = [C.POINTER(vp), C.c_int, C.POINTER(vp), C.POINTER(u64),
+                                           C.POINTER(_Out), vp]
     L.hbt_last_error.restype = C.c_char_p
     L.hbt_version.restype = C.c_char_p
     for f in ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
-              "hbt_info", "hbt_export", "hbt_set_param"]:
+              "hbt_info", "hbt_export", "hbt_set_param", "hbt_comm_unique_id", "hbt_comm_init",
+              "hbt_comm_destroy", "hbt_bulk_build_sharded", "hbt_search_sharded", "hbt_shard_local_init",
+              "hbt_search_sharded_local"]:
         getattr(L, f).restype = C.c_int
     return L
 
@@ -114,6 +126,13 @@ def _dtype(width):
 
 class Tree:
     """A device-resident HB+-tree (implicit or regular layout)."""
+
+    @classmethod
+    def _adopt(cls, handle, width, fanout, layout):
+        import torch
+        t = cls.__new__(cls)
+        t._h, t.width, t.fanout, t.layout, t._torch = handle, width, fanout, layout, torch
+        return t
 
     def __init__(self, keys, values, fanout: int = 16, layout: str = "implicit", stream=None):
         import torch
@@ -209,6 +228,110 @@ class Tree:
         for k, v in [("smem_bytes", smem_bytes), ("threads", threads_per_cta), ("ctas_per_sm", ctas_per_sm),
                      ("qpl", queries_per_lane), ("smem_mode", smem_mode), ("carveout", carveout)]:
             self.set_param(k, v)
+
+
+# ---------------------------------------------------------------- sharding
+
+
+def unique_id() -> bytes:
+    """ncclGetUniqueId (call on one rank and broadcast the 128 bytes)."""
+    buf = C.create_string_buffer(128)
+    _check(lib.hbt_comm_unique_id(buf))
+    return buf.raw
+
+
+def shard_plan(n_total: int, world: int, rank: int):
+    """Contiguous key-index range [lo, hi) of shard `rank` when n_total generated
+    keys (stratified, i.e. sorted by index, c4) are split over `world` ranks."""
+    return rank * n_total // world, (rank + 1) * n_total // world
+
+
+def broadcast_unique_id(group=None) -> bytes:
+    """Rank 0 creates the NCCL id; every rank receives it (torch.distributed,
+    any backend)."""
+    import torch.distributed as dist
+    obj = [unique_id() if dist.get_rank(group) == 0 else None]
+    dist.broadcast_object_list(obj, src=0, group=group)
+    return obj[0]
+
+
+class Comm:
+    """An NCCL communicator owned by libhbt (one process per GPU)."""
+
+    def __init__(self, nranks: int, rank: int, uid: bytes):
+        h = C.c_void_p()
+        _check(lib.hbt_comm_init(nranks, rank, C.c_char_p(uid), C.byref(h)))
+        self._h, self.nranks, self.rank = h, nranks, rank
+
+    @classmethod
+    def from_torch(cls, group=None):
+        import torch.distributed as dist
+        uid = broadcast_unique_id(group)
+        return cls(dist.get_world_size(group), dist.get_rank(group), uid)
+
+    def close(self):
+        if getattr(self, "_h", None) and self._h.value:
+            lib.hbt_comm_destroy(self._h)
+            self._h = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class ShardedTree(Tree):
+    """This rank's shard of a key-range-sharded implicit tree (collective calls)."""
+
+    def __init__(self, comm: Comm, keys, values, fanout: int = 16, stream=None):
+        import torch
+        self.width = _width(keys)
+        self.fanout, self.layout, self._torch, self.comm = fanout, "implicit", torch, comm
+        word = IMPLICIT | (KEY64 if self.width == 8 else KEY32)
+        keys, values = keys.contiguous(), values.contiguous()
+        h = C.c_void_p()
+        _check(lib.hbt_bulk_build_sharded(comm._h, C.c_void_p(keys.data_ptr() if keys.numel() else 0),
+                                          C.c_void_p(values.data_ptr() if values.numel() else 0), keys.numel(),
+                                          fanout, word, _stream_ptr(stream), C.byref(h)))
+        self._h = h
+
+    def search(self, queries, out_pos=None, out_vals=None, stream=None):
+        torch = self._torch
+        queries = queries.contiguous()
+        m = queries.numel()
+        if out_pos is None:
+            out_pos = torch.empty(m, dtype=torch.int64, device="cuda")
+        if out_vals is None:
+            out_vals = torch.empty(m, dtype=_dtype(self.width), device="cuda")
+        _check(lib.hbt_search_sharded(self._h, C.c_void_p(queries.data_ptr() if m else 0), m,
+                                      _Out(out_pos.data_ptr() if m else 0, out_vals.data_ptr() if m else 0),
+                                      _stream_ptr(stream)))
+        return out_pos, out_vals
+
+
+class LocalShardGroup:
+    """G implicit trees on ONE device used as a key-range shard group: the same
+    route / search / unpermute kernels as ShardedTree, the exchange being
+    device-to-device copies."""
+
+    def __init__(self, trees):
+        self.trees = list(trees)
+        G = len(self.trees)
+        self._arr = (C.c_void_p * G)(*[t.handle.value for t in self.trees])
+        _check(lib.hbt_shard_local_init(self._arr, G))
+
+    def search(self, queries, stream=None):
+        torch = self.trees[0]._torch
+        G = len(self.trees)
+        qs = [q.contiguous() for q in queries]
+        outs = [(torch.empty(q.numel(), dtype=torch.int64, device="cuda"),
+                 torch.empty(q.numel(), dtype=_dtype(self.trees[0].width), device="cuda")) for q in qs]
+        qa = (C.c_void_p * G)(*[q.data_ptr() if q.numel() else 0 for q in qs])
+        ma = (C.c_uint64 * G)(*[q.numel() for q in qs])
+        oa = (_Out * G)(*[_Out(p.data_ptr() if p.numel() else 0, v.data_ptr() if v.numel() else 0) for p, v in outs])
+        _check(lib.hbt_search_sharded_local(self._arr, G, qa, ma, oa, _stream_ptr(stream)))
+        return outs
 
 
 def unpack(pos_found, values, width: int):

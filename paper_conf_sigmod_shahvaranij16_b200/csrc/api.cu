@@ -40,6 +40,7 @@ static void free_tree(hbt_tree* t) {
   cudaFree(t->d_inner_idx);
   cudaFree(t->d_leaf);
   regular_free(t);
+  shard_free(t);
   cudaFree(t->pipe.d_q);
   cudaFree(t->pipe.d_pf);
   cudaFree(t->pipe.d_v);

@@ -74,6 +74,30 @@ struct HostPipe {
   cudaEvent_t ev[2] = {nullptr, nullptr};
 };
 
+// Key-range shard metadata (sharded.cu): shard g holds global ranks
+// [base[g], base[g] + count[g]) with largest key max[g].
+struct ShardMeta {
+  int G = 0;
+  int rank = 0;
+  ::hbt_comm* comm = nullptr;  // NULL for single-process (virtual) shard groups
+  uint64_t count[64] = {};
+  uint64_t base[64] = {};
+  uint64_t max[64] = {};
+};
+
+// Per-tree scratch of the sharded search (grown on demand).
+struct Scratch {
+  uint8_t* dest = nullptr; uint64_t dest_cap = 0;
+  uint8_t* send_q = nullptr; uint64_t send_cap = 0;      // elements of S bytes
+  uint32_t* origin = nullptr; uint64_t origin_cap = 0;
+  uint8_t* recv_q = nullptr; uint64_t recv_cap = 0;
+  uint64_t* res_pf = nullptr; uint64_t res_pf_cap = 0;   // receive order
+  uint8_t* res_v = nullptr; uint64_t res_v_cap = 0;
+  uint64_t* back_pf = nullptr; uint64_t back_pf_cap = 0; // send order
+  uint8_t* back_v = nullptr; uint64_t back_v_cap = 0;
+  unsigned long long* counts = nullptr;                  // 2 x 64
+};
+
 }  // namespace hbt
 
 struct hbt_tree {
@@ -100,6 +124,9 @@ struct hbt_tree {
   uint64_t leaf_bytes = 0;
   // ---- regular ----
   hbt::RegularState r;
+  // ---- key-range sharding ----
+  hbt::ShardMeta shard;
+  hbt::Scratch shard_scratch;
   // ---- search ----
   hbt::SearchConfig cfg;
   mutable hbt::HostPipe pipe;
@@ -116,6 +143,10 @@ int sort_dedupe(uint32_t width, const void* keys, const void* values, uint64_t n
 int implicit_update(hbt_tree* t, const hbt_batch* b, cudaStream_t s);
 // implicit_search.cu
 int implicit_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s);
+// same, reporting global positions base + rank (sharded trees)
+int implicit_search_base(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
+                         cudaStream_t s);
+void shard_free(hbt_tree* t);
 uint32_t implicit_smem_levels(const hbt_tree* t, uint32_t budget);
 // index bytes per implicit node (0 when F*S <= 32)
 uint32_t implicit_idx_stride(uint32_t F, uint32_t S);

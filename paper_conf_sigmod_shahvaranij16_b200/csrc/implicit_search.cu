@@ -103,7 +103,8 @@ template <typename K, int F, int QPL, int THREADS, int MODE>
 __global__ void __launch_bounds__(THREADS)
 implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ inner_idx,
                        const uint8_t* __restrict__ leaf, const K* __restrict__ queries, uint64_t m,
-                       uint64_t* __restrict__ out_pf, K* __restrict__ out_v, const LevelTable lt, uint64_t n) {
+                       uint64_t* __restrict__ out_pf, K* __restrict__ out_v, const LevelTable lt, uint64_t n,
+                       uint64_t pos_base) {
   using C = Cfg<K, F>;
   constexpr int ROUND = 32 * QPL;        // queries per warp round (QPL per lane in phase 1)
   constexpr int QPG = ROUND / C::NG;     // queries per group in phase 2
@@ -240,7 +241,7 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
       const uint64_t r = uint64_t(node[j]) * C::P + s;
       const bool found = (s < uint32_t(C::P)) && (r < n) && (key_s == q[j]);
       if (j % C::G == k) {
-        my_pf[j / C::G] = (r < n ? r : kEnd) | (found ? kFound : 0ull);
+        my_pf[j / C::G] = (r < n ? r + pos_base : kEnd) | (found ? kFound : 0ull);
         my_v[j / C::G] = found ? val_s : K(0);
       }
     }
@@ -267,7 +268,8 @@ struct Launch {
   }
 
   template <int QPL, int THREADS, int MODE>
-  static int run_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+  static int run_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t base,
+                   cudaStream_t s) {
     auto kern = implicit_search_kernel<K, F, QPL, THREADS, MODE>;
     LevelTable lt{};
     for (uint32_t d = 0; d <= t->H; ++d) lt.offset[d] = t->offset[d];
@@ -294,31 +296,31 @@ struct Launch {
     const uint64_t need = (rounds + THREADS / 32 - 1) / (THREADS / 32);
     if (need < grid) grid = need ? need : 1;
     kern<<<unsigned(grid), THREADS, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
-                                               (const uint8_t*)t->d_leaf, (const K*)q, m, pf, (K*)v, lt, t->n);
+                                               (const uint8_t*)t->d_leaf, (const K*)q, m, pf, (K*)v, lt, t->n, base);
     HBT_CUDA_TRY(cudaGetLastError());
     return HBT_OK;
   }
 
-  static int run(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+  static int run(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t b, cudaStream_t s) {
     const uint32_t qpl = t->cfg.qpl ? t->cfg.qpl : 1;
     const uint32_t th = t->cfg.threads ? t->cfg.threads : 512;
     const bool hilo = t->cfg.mode == 1;
     if (qpl == 2) {
-      if (hilo) return th == 256 ? run_t<2, 256, 1>(t, q, m, pf, v, s) : run_t<2, 512, 1>(t, q, m, pf, v, s);
-      return th == 256 ? run_t<2, 256, 0>(t, q, m, pf, v, s) : run_t<2, 512, 0>(t, q, m, pf, v, s);
+      if (hilo) return th == 256 ? run_t<2, 256, 1>(t, q, m, pf, v, b, s) : run_t<2, 512, 1>(t, q, m, pf, v, b, s);
+      return th == 256 ? run_t<2, 256, 0>(t, q, m, pf, v, b, s) : run_t<2, 512, 0>(t, q, m, pf, v, b, s);
     }
-    if (hilo) return th == 256 ? run_t<1, 256, 1>(t, q, m, pf, v, s) : run_t<1, 512, 1>(t, q, m, pf, v, s);
-    return th == 256 ? run_t<1, 256, 0>(t, q, m, pf, v, s) : run_t<1, 512, 0>(t, q, m, pf, v, s);
+    if (hilo) return th == 256 ? run_t<1, 256, 1>(t, q, m, pf, v, b, s) : run_t<1, 512, 1>(t, q, m, pf, v, b, s);
+    return th == 256 ? run_t<1, 256, 0>(t, q, m, pf, v, b, s) : run_t<1, 512, 0>(t, q, m, pf, v, b, s);
   }
 };
 
 template <typename K>
-int dispatch_f(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+int dispatch_f(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t b, cudaStream_t s) {
   switch (t->F) {
-    case 4: return Launch<K, 4>::run(t, q, m, pf, v, s);
-    case 8: return Launch<K, 8>::run(t, q, m, pf, v, s);
-    case 16: return Launch<K, 16>::run(t, q, m, pf, v, s);
-    case 32: return Launch<K, 32>::run(t, q, m, pf, v, s);
+    case 4: return Launch<K, 4>::run(t, q, m, pf, v, b, s);
+    case 8: return Launch<K, 8>::run(t, q, m, pf, v, b, s);
+    case 16: return Launch<K, 16>::run(t, q, m, pf, v, b, s);
+    case 32: return Launch<K, 32>::run(t, q, m, pf, v, b, s);
   }
   set_error("unsupported fanout %u", t->F);
   return HBT_EINVAL;
@@ -344,9 +346,14 @@ uint32_t implicit_idx_stride(uint32_t F, uint32_t S) {
   return b > 16 ? b : 16;
 }
 
-int implicit_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+int implicit_search_base(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t base,
+                         cudaStream_t s) {
   if (m == 0) return HBT_OK;
-  return t->width == 4 ? dispatch_f<uint32_t>(t, q, m, pf, v, s) : dispatch_f<uint64_t>(t, q, m, pf, v, s);
+  return t->width == 4 ? dispatch_f<uint32_t>(t, q, m, pf, v, base, s) : dispatch_f<uint64_t>(t, q, m, pf, v, base, s);
+}
+
+int implicit_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+  return implicit_search_base(t, q, m, pf, v, 0, s);
 }
 
 uint32_t implicit_smem_levels(const hbt_tree* t, uint32_t budget) {

@@ -1,0 +1,93 @@
+"""GPU parity of the key-range-sharded search.
+
+* Virtual shard groups on one B200 (hbt_search_sharded_local): G shards built
+  from key-ordered disjoint ranges, empty shards included; every shard's query
+  batch (hits anywhere, misses, edges, keys beyond every shard) must equal the
+  UNSHARDED oracle bit for bit (global pos = rank).
+* The NCCL path (hbt_comm_init + hbt_bulk_build_sharded + hbt_search_sharded)
+  with one rank on one GPU.
+"""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from gpu_util import from_dev, to_dev
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def hbt():
+    import paper_conf_sigmod_shahvaranij16_b200 as m
+    assert torch.cuda.is_available(), "gpu tests need a CUDA device"
+    return m
+
+
+def split_points(n, G, empty):
+    cuts = [g * n // G for g in range(G + 1)]
+    spans = [(cuts[g], cuts[g + 1]) for g in range(G)]
+    for g in empty:  # make shard g empty, give its keys to a neighbour
+        lo, hi = spans[g]
+        spans[g] = (lo, lo)
+        if g + 1 < G:
+            spans[g + 1] = (lo, spans[g + 1][1])
+        else:
+            spans[g - 1] = (spans[g - 1][0], hi)
+    return spans
+
+
+def queries(allk, rng, m):
+    n = len(allk)
+    return np.concatenate([allk[rng.integers(0, n, m // 2)],
+                           rng.integers(0, 2**64 - 1, m // 2, dtype=np.uint64, endpoint=True),
+                           np.array([0, 2**64 - 1, allk[0], allk[-1], allk[-1] + 1, allk[0] - 1], np.uint64)])
+
+
+@pytest.mark.parametrize("G,empty", [(1, []), (2, []), (3, [1]), (5, [0, 4]), (8, []), (8, [2, 3])])
+def test_virtual_shards_match_unsharded_oracle(hbt, G, empty):
+    n = 200000
+    allk = gen.stratified_keys(n, gen.stream_seed(4, gen.STREAM_K))
+    allv = gen.values(n, 8, gen.stream_seed(4, gen.STREAM_V))
+    full = oracle.ITree.from_pairs(allk, allv, 16, 8)
+    spans = split_points(n, G, empty)
+    trees = []
+    for lo, hi in spans:
+        k, v = allk[lo:hi], allv[lo:hi]
+        perm = np.random.default_rng(lo).permutation(len(k))  # unsorted within the shard is fine
+        trees.append(hbt.Tree(to_dev(k[perm], 8), to_dev(v[perm], 8), fanout=16))
+    grp = hbt.LocalShardGroup(trees)
+    rng = np.random.default_rng(G)
+    qs = [queries(allk, rng, 4000 + 1000 * g) for g in range(G)]
+    outs = grp.search([to_dev(q, 8) for q in qs])
+    torch.cuda.synchronize()
+    for q, (pf, v) in zip(qs, outs):
+        epf, ev = full.search(q)
+        assert np.array_equal(pf.cpu().numpy().view(np.uint64), epf)
+        assert np.array_equal(from_dev(v, 8), ev)
+
+
+def test_virtual_shards_reject_overlap(hbt):
+    k = np.arange(1, 1001, dtype=np.uint64)
+    a = hbt.Tree(to_dev(k[:600], 8), to_dev(k[:600], 8), fanout=8)
+    b = hbt.Tree(to_dev(k[500:], 8), to_dev(k[500:], 8), fanout=8)
+    with pytest.raises(hbt.HBTError):
+        hbt.LocalShardGroup([a, b])
+
+
+def test_nccl_path_one_rank(hbt):
+    uid = hbt.unique_id()
+    comm = hbt.Comm(1, 0, uid)
+    n = 100000
+    allk = gen.stratified_keys(n, 7)
+    allv = gen.values(n, 8, 9)
+    t = hbt.ShardedTree(comm, to_dev(allk, 8), to_dev(allv, 8), fanout=16)
+    q = queries(allk, np.random.default_rng(0), 50000)
+    pf, v = t.search(to_dev(q, 8))
+    torch.cuda.synchronize()
+    epf, ev = oracle.ITree.from_pairs(allk, allv, 16, 8).search(q)
+    assert np.array_equal(pf.cpu().numpy().view(np.uint64), epf)
+    assert np.array_equal(from_dev(v, 8), ev)
+    t.close()
+    comm.close()
