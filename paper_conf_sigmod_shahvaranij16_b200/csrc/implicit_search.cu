@@ -29,10 +29,10 @@ namespace {
 
 constexpr uint64_t kEnd = HBT_POS_END;
 constexpr uint64_t kFound = HBT_FOUND_BIT;
-// Only the tiny top levels go to shared memory: measured on B200 (profiles/
-// r01_*), a large shared carve-out costs more L1 hits on the L2 levels than the
-// pinned levels save (c2: SL=4 / 70 KB -> 24.0 G q/s, SL=3 / 4.4 KB -> 26.4).
-constexpr uint32_t kDefaultSmemBudget = 8 * 1024;
+// Pinned-level budget per CTA (measured on B200, profiles/r01_sweep_v*.log): with
+// the padded node stride, c2's 4 top levels (74 KB) beat 3 levels (29.3 -> 31.5
+// G q/s); the carve-out is left to the driver so the L2 levels keep L1 hits.
+constexpr uint32_t kDefaultSmemBudget = 100 * 1024;
 
 template <typename K>
 __device__ __forceinline__ K key_max() { return K(~K(0)); }
@@ -111,20 +111,23 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
   static_assert(QPG % C::G == 0, "every group lane stores QPG/G results");
   extern __shared__ __align__(16) uint8_t smem[];
   const uint32_t SL = lt.SL, H = lt.H;
-  // Stage the top SL levels (root-first, contiguous) once per persistent CTA.
-  // MODE 1 splits 64-bit keys into 32-bit hi / lo planes (a probe reads one
-  // 4-byte bank per plane); MODE 0 keeps the node array as is.
-  const uint32_t s_n = uint32_t(lt.offset[SL]) * F;  // staged keys
+  // Stage the top SL levels (root-first, contiguous) once per persistent CTA
+  // with a padded node stride of F+1 keys: with a 128 B stride, key i of every
+  // node would sit in the same bank and the lanes' probes into different nodes
+  // would serialise.  MODE 1 splits 64-bit keys into 32-bit hi / lo planes.
+  constexpr uint32_t FP = F + 1;
+  const uint32_t s_nodes = uint32_t(lt.offset[SL]);
   K* s_keys = reinterpret_cast<K*>(smem);
   uint32_t* s_hi = reinterpret_cast<uint32_t*>(smem);
-  uint32_t* s_lo = s_hi + s_n;
-  for (uint32_t i = threadIdx.x; i < s_n; i += THREADS) {
+  uint32_t* s_lo = s_hi + s_nodes * FP;
+  for (uint32_t i = threadIdx.x; i < s_nodes * F; i += THREADS) {
     const K key = __ldg(reinterpret_cast<const K*>(inner) + i);
+    const uint32_t a = (i / F) * FP + i % F;
     if constexpr (MODE == 1 && sizeof(K) == 8) {
-      s_hi[i] = uint32_t(uint64_t(key) >> 32);
-      s_lo[i] = uint32_t(key);
+      s_hi[a] = uint32_t(uint64_t(key) >> 32);
+      s_lo[a] = uint32_t(key);
     } else {
-      s_keys[i] = key;
+      s_keys[a] = key;
     }
   }
   __syncthreads();
@@ -148,7 +151,7 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
       mynode[u] = 0;
     }
     for (uint32_t d = 0; d < SL; ++d) {
-      const uint32_t lvl = uint32_t(lt.offset[d]) * F;
+      const uint32_t lvl = uint32_t(lt.offset[d]) * FP;
       uint32_t pos[QPL];
 #pragma unroll
       for (int u = 0; u < QPL; ++u) pos[u] = 0;
@@ -156,7 +159,7 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
       for (int step = F / 2; step >= 1; step /= 2) {
 #pragma unroll
         for (int u = 0; u < QPL; ++u) {
-          const uint32_t a = lvl + mynode[u] * F + pos[u] + step - 1;
+          const uint32_t a = lvl + mynode[u] * FP + pos[u] + step - 1;
           bool lt_;
           if constexpr (MODE == 1 && sizeof(K) == 8) {
             const uint32_t qh = uint32_t(uint64_t(myq[u]) >> 32), ql = uint32_t(myq[u]);
@@ -263,7 +266,7 @@ struct Launch {
 
   static uint32_t smem_levels(const hbt_tree* t, uint32_t budget) {
     uint32_t SL = 0;
-    while (SL < t->H && t->offset[SL + 1] * uint64_t(C::NODE_BYTES) <= budget) ++SL;
+    while (SL < t->H && t->offset[SL + 1] * uint64_t(C::NODE_BYTES + C::S) <= budget) ++SL;
     return SL;
   }
 
@@ -275,7 +278,7 @@ struct Launch {
     for (uint32_t d = 0; d <= t->H; ++d) lt.offset[d] = t->offset[d];
     lt.H = t->H;
     lt.SL = smem_levels(t, t->cfg.smem_budget ? t->cfg.smem_budget : kDefaultSmemBudget);
-    const size_t smem = size_t(lt.offset[lt.SL]) * C::NODE_BYTES;  // both MODEs use F*S bytes per node
+    const size_t smem = size_t(lt.offset[lt.SL]) * (C::NODE_BYTES + C::S);  // (F+1)*S bytes per staged node
     static bool attr_set = false;  // per instantiation
     if (!attr_set) {
       HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
