@@ -77,10 +77,6 @@ struct Cfg {
   static constexpr int G = IL > 2 ? IL : 2;                               // lanes per query group
   static constexpr int NG = 32 / G;                                       // groups per warp
   static constexpr int P = 64 / (2 * S);                                  // pairs per leaf line
-  static constexpr int LL = G < 4 ? G : 4;                                // lanes loading a leaf line
-  static constexpr int LB = 64 / LL;                                      // leaf bytes per lane (32|16)
-  static constexpr int KEY_LANES = LL / 2;                                // lanes holding the keys
-  static constexpr int LK = LB / S;                                       // leaf entries per lane
 };
 
 template <typename K, int N>
@@ -210,37 +206,31 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
 #pragma unroll
       for (int j = 0; j < QPG; ++j) node[j] = node[j] * F + sec[j] * C::KPS + count_less16(kv[j], q[j], gmask);
     }
-    // ---- leaf line: lanes [0, KEY_LANES) hold the P keys, [KEY_LANES, LL) the P values
-    K lk[QPG][C::LK];
+    // ---- leaf line [P keys | P values]: lanes 0 and 1 of the group each load one
+    //      16 B half of the key sector and of the value sector, so every load
+    //      instruction touches exactly one 32 B sector per group.
+    constexpr int E16 = 16 / C::S;
+    V16<K> lkey[QPG], lval[QPG];
 #pragma unroll
     for (int j = 0; j < QPG; ++j) {
-      if (k < C::LL) {
-        const uint8_t* p = leaf + uint64_t(node[j]) * 64 + k * C::LB;
-#pragma unroll
-        for (int h = 0; h < C::LB / 16; ++h) {
-          V16<K> v;
-          ld16(v, p + h * 16);
-#pragma unroll
-          for (int e = 0; e < 16 / C::S; ++e) lk[j][h * (16 / C::S) + e] = v.k[e];
-        }
+      if (k < 2) {
+        const uint8_t* p = leaf + uint64_t(node[j]) * 64 + k * 16;
+        ld16(lkey[j], p);
+        ld16(lval[j], p + 32);
       } else {
-#pragma unroll
-        for (int e = 0; e < C::LK; ++e) lk[j][e] = key_max<K>();
+        fill_max(lkey[j]);
+        fill_max(lval[j]);
       }
     }
     uint64_t my_pf[QPG / C::G];
     K my_v[QPG / C::G];
 #pragma unroll
     for (int j = 0; j < QPG; ++j) {
-      uint32_t s = 0;
-#pragma unroll
-      for (int e = 0; e < C::LK; ++e)
-        s += __popc(__ballot_sync(0xffffffffu, (k < C::KEY_LANES) && (lk[j][e] < q[j])) & gmask);
+      const uint32_t s = count_less16(lkey[j], q[j], gmask);  // lanes >= 2 hold MAX
       const uint32_t sc = s < uint32_t(C::P) ? s : uint32_t(C::P - 1);
-      const K sel = pick(lk[j], sc % C::LK);
-      const int src = g * C::G + int(sc / C::LK);
-      const K key_s = __shfl_sync(0xffffffffu, sel, src);
-      const K val_s = __shfl_sync(0xffffffffu, sel, src + C::KEY_LANES);
+      const int src = g * C::G + int(sc / E16);
+      const K key_s = __shfl_sync(0xffffffffu, pick(lkey[j].k, sc % E16), src);
+      const K val_s = __shfl_sync(0xffffffffu, pick(lval[j].k, sc % E16), src);
       const uint64_t r = uint64_t(node[j]) * C::P + s;
       const bool found = (s < uint32_t(C::P)) && (r < n) && (key_s == q[j]);
       if (j % C::G == k) {
