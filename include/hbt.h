@@ -161,7 +161,7 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
 /* Tune the search kernel's launch shape on one tree; results never depend on
  * it.  name / value:
  *   "smem_bytes"  shared-memory budget per CTA for the pinned top levels (<= 227 KB; 0 = default 100 KB)
- *   "threads"     threads per CTA: 256 or 512 (0 = default 512)
+ *   "threads"     threads per CTA: 256, 512 or 1024 (0 = default: implicit 1024, regular 512)
  *   "ctas_per_sm" cap on resident CTAs per SM (0 = occupancy-derived)
  *   "qpl"         queries per lane per warp round, 1 or 2 (0 = default)
  *   "smem_mode"   0 = probe S-byte keys, 1 = probe 32-bit hi/lo planes (64-bit keys)

@@ -244,7 +244,7 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   const std::string n(name);
   SearchConfig& c = t->cfg;
   if (n == "smem_bytes" && value >= 0 && value <= 227 * 1024) c.smem_budget = uint32_t(value);
-  else if (n == "threads" && (value == 0 || value == 256 || value == 512)) c.threads = uint32_t(value);
+  else if (n == "threads" && (value == 0 || value == 256 || value == 512 || value == 1024)) c.threads = uint32_t(value);
   else if (n == "ctas_per_sm" && value >= 0 && value <= 32) c.ctas_per_sm = uint32_t(value);
   else if (n == "qpl" && value >= 0 && value <= 2) c.qpl = uint32_t(value);
   else if (n == "smem_mode" && (value == 0 || value == 1)) c.mode = uint32_t(value);

@@ -296,13 +296,17 @@ struct Launch {
 
   static int run(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t b, cudaStream_t s) {
     const uint32_t qpl = t->cfg.qpl ? t->cfg.qpl : 1;
-    const uint32_t th = t->cfg.threads ? t->cfg.threads : 512;
+    const uint32_t th = t->cfg.threads ? t->cfg.threads : 1024;
     const bool hilo = t->cfg.mode == 1;
+    if (hilo) {
+      if (qpl == 2) return th == 256 ? run_t<2, 256, 1>(t, q, m, pf, v, b, s) : run_t<2, 512, 1>(t, q, m, pf, v, b, s);
+      return th == 256 ? run_t<1, 256, 1>(t, q, m, pf, v, b, s) : run_t<1, 512, 1>(t, q, m, pf, v, b, s);
+    }
     if (qpl == 2) {
-      if (hilo) return th == 256 ? run_t<2, 256, 1>(t, q, m, pf, v, b, s) : run_t<2, 512, 1>(t, q, m, pf, v, b, s);
+      if (th == 1024) return run_t<2, 1024, 0>(t, q, m, pf, v, b, s);
       return th == 256 ? run_t<2, 256, 0>(t, q, m, pf, v, b, s) : run_t<2, 512, 0>(t, q, m, pf, v, b, s);
     }
-    if (hilo) return th == 256 ? run_t<1, 256, 1>(t, q, m, pf, v, b, s) : run_t<1, 512, 1>(t, q, m, pf, v, b, s);
+    if (th == 1024) return run_t<1, 1024, 0>(t, q, m, pf, v, b, s);
     return th == 256 ? run_t<1, 256, 0>(t, q, m, pf, v, b, s) : run_t<1, 512, 0>(t, q, m, pf, v, b, s);
   }
 };
