@@ -45,7 +45,7 @@ def parse():
     ap.add_argument("--smem", type=int, default=0, help="override smem budget (bytes)")
     ap.add_argument("--qpl", type=int, default=0, help="queries per lane per warp round (1|2)")
     ap.add_argument("--threads", type=int, default=0, help="threads per CTA (256|512)")
-    ap.add_argument("--smem-mode", type=int, default=0, help="0 = key words, 1 = hi/lo planes")
+    ap.add_argument("--smem-mode", type=int, default=None, help="2 = directory (default), 0 = staged levels, 1 = hi/lo")
     ap.add_argument("--carveout", type=int, default=-1, help="smem carve-out percent (-1 default)")
     return ap.parse_args()
 

@@ -164,7 +164,8 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *   "threads"     threads per CTA: 256, 512 or 1024 (0 = default: implicit 1024, regular 512)
  *   "ctas_per_sm" cap on resident CTAs per SM (0 = occupancy-derived)
  *   "qpl"         queries per lane per warp round, 1 or 2 (0 = default)
- *   "smem_mode"   0 = probe S-byte keys, 1 = probe 32-bit hi/lo planes (64-bit keys)
+ *   "smem_mode"   implicit top levels: 2 = level-T directory + one lower bound (default),
+ *                 0 = per-level binary search of staged nodes, 1 = the same on 32-bit hi/lo planes
  *   "carveout"    preferred shared-memory carve-out percent, -1 = driver default
  * Unknown names or out-of-range values return HBT_EINVAL. */
 HBT_API int hbt_set_param(hbt_tree* t, const char* name, int64_t value);

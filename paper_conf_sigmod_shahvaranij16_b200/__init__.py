@@ -224,10 +224,11 @@ class Tree:
         _check(lib.hbt_set_param(self._h, name.encode(), int(value)))
 
     def set_search_config(self, smem_bytes: int = 0, threads_per_cta: int = 0, ctas_per_sm: int = 0,
-                          queries_per_lane: int = 0, smem_mode: int = 0, carveout: int = -1):
+                          queries_per_lane: int = 0, smem_mode=None, carveout: int = -1):
         for k, v in [("smem_bytes", smem_bytes), ("threads", threads_per_cta), ("ctas_per_sm", ctas_per_sm),
                      ("qpl", queries_per_lane), ("smem_mode", smem_mode), ("carveout", carveout)]:
-            self.set_param(k, v)
+            if v is not None:
+                self.set_param(k, v)
 
 
 # ---------------------------------------------------------------- sharding

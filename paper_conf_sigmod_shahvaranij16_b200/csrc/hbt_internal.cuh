@@ -29,7 +29,9 @@ static inline uint64_t ceil_div_u64(uint64_t a, uint64_t b) { return (a + b - 1)
 struct LevelTable {
   uint64_t offset[HBT_MAX_LEVELS + 1];
   uint32_t H;   // inner levels
-  uint32_t SL;  // levels [0, SL) staged in shared memory
+  uint32_t SL;  // levels [0, SL) searched in shared memory (mode 2: = the directory level T)
+  uint32_t dcount;  // mode 2: nodes at level T
+  uint32_t dbits;   // mode 2: directory prefix bits
 };
 
 struct SearchConfig {
@@ -37,7 +39,7 @@ struct SearchConfig {
   uint32_t threads = 0;          // threads per CTA (0 = default)
   uint32_t ctas_per_sm = 0;      // 0 = occupancy-derived
   uint32_t qpl = 0;              // queries per lane per warp round (0 = default)
-  uint32_t mode = 0;             // smem probe mode: 0 = K words, 1 = hi/lo 32-bit planes
+  uint32_t mode = 2;             // top-level mode: 0 = staged levels (K words), 1 = hi/lo planes, 2 = directory
   int carveout = -1;             // shared-memory carve-out percent (-1 = driver default)
 };
 
@@ -119,6 +121,14 @@ struct hbt_tree {
   void* d_inner_idx = nullptr;
   uint64_t inner_idx_bytes = 0;
   uint32_t idx_stride = 0;  // bytes of index per node (0 = nodes fit one sector)
+  // Level-T directory (search mode 2): d_dir = [M_T: count_T keys | dir: 2^dir_bits x (u16 lo, u16 hi)]
+  // M_T[j] = max key below level-T node j (MAX for the last node); dir[p] = the
+  // range of level-T nodes that queries with key prefix p can reach.
+  void* d_dir = nullptr;
+  uint64_t dir_bytes = 0;
+  uint32_t dir_T = 0;       // target level (H = leaf lines)
+  uint32_t dir_count = 0;   // nodes at level T
+  uint32_t dir_bits = 0;
   void* d_leaf = nullptr;
   uint64_t L0 = 0;
   uint64_t leaf_bytes = 0;

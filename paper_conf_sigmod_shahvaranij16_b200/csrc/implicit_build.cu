@@ -84,6 +84,52 @@ __global__ void derive_inner_index(const K* __restrict__ inner, uint64_t nodes, 
   }
 }
 
+// Directory (search mode 2).  The descent through levels 0..T-1 reaches the
+// FIRST level-T node whose subtree max key is >= q (or the last node): at every
+// level the child picked is #{sep < q} with sep = child max keys and the last
+// slot MAX (R1, R3).  So node_T(q) = lower_bound(M_T, q) with M_T[j] = the max
+// key below node j and M_T[last] = MAX.  dir[p] = [node_T(p << shift),
+// node_T(((p + 1) << shift) - 1)] bounds that lower bound for every q of prefix p
+// (node_T is monotone in q), so the search = one dir lookup + a binary search of
+// M_T restricted to that range.  Exact for any key distribution.
+template <typename K>
+__global__ void build_dir_max(const K* __restrict__ leaf, uint64_t nd, uint64_t count, uint64_t span,
+                              K* __restrict__ M) {
+  constexpr uint32_t P = 64 / (2 * sizeof(K));
+  for (uint64_t j = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; j < count; j += uint64_t(gridDim.x) * blockDim.x) {
+    if (j + 1 == count || nd == 0) {
+      M[j] = key_max<K>();
+    } else {
+      uint64_t end = (j + 1) * span;
+      if (end > nd) end = nd;
+      const uint64_t r = end - 1;
+      M[j] = leaf[(r / P) * (2 * P) + r % P];
+    }
+  }
+}
+
+template <typename K>
+__device__ __forceinline__ uint32_t lower_bound_dev(const K* M, uint32_t count, K q) {
+  uint32_t lo = 0, hi = count - 1;  // M[count-1] = MAX >= q
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (M[mid] < q) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
+template <typename K>
+__global__ void build_dir_table(const K* __restrict__ M, uint32_t count, uint32_t bits, uint32_t* __restrict__ dir) {
+  const uint32_t shift = 8 * sizeof(K) - bits;
+  for (uint64_t p = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; p < (1ull << bits); p += uint64_t(gridDim.x) * blockDim.x) {
+    const K first = K(K(p) << shift);
+    const K last = K(first | K((K(1) << shift) - 1));
+    const uint32_t lo = lower_bound_dev(M, count, first);
+    const uint32_t hi = lower_bound_dev(M, count, last);
+    dir[p] = lo | (hi << 16);
+  }
+}
+
 template <typename K>
 __global__ void unpack_leaf_lines(const K* __restrict__ leaf, uint64_t nd, K* __restrict__ kd, K* __restrict__ vd) {
   constexpr uint32_t P = 64 / (2 * sizeof(K));
@@ -216,6 +262,7 @@ int build_sorted_t(hbt_tree* t, const K* kd, const K* vd, uint64_t nd, cudaStrea
     LevelTable lt{};
     for (uint32_t d = 0; d <= H; ++d) lt.offset[d] = t->offset[d];
     lt.H = H;
+    lt.SL = 0;
     gather_separators<K><<<grid_for(t->offset[H] * F), 256, 0, s>>>(kd, nd, lt, t->L0, F, (K*)t->d_inner);
     HBT_CUDA_TRY(cudaGetLastError());
     t->idx_stride = implicit_idx_stride(F, sizeof(K));
@@ -227,6 +274,30 @@ int build_sorted_t(hbt_tree* t, const K* kd, const K* vd, uint64_t nd, cudaStrea
                                                                          (K*)t->d_inner_idx);
       HBT_CUDA_TRY(cudaGetLastError());
     }
+  }
+  // level-T directory: T = the deepest level whose max-key array fits 64 KB
+  {
+    uint32_t T = 0;
+    for (uint32_t d = 0; d <= H; ++d) {
+      const uint64_t cnt = d < H ? t->nodes[d] : t->L0;
+      if (cnt * sizeof(K) <= 64 * 1024 && cnt <= 65535) T = d;
+    }
+    const uint64_t cnt = T < H ? t->nodes[T] : t->L0;
+    uint64_t span = P;  // ranks below one level-T node: P * F^(H-T)
+    for (uint32_t e = T; e < H; ++e) span *= F;
+    uint32_t bits = 1;
+    while ((1ull << bits) < 4 * cnt && bits < 13) ++bits;
+    t->dir_T = T;
+    t->dir_count = uint32_t(cnt);
+    t->dir_bits = bits;
+    t->dir_bytes = cnt * sizeof(K) + (4ull << bits);
+    HBT_CUDA_TRY(cudaMalloc(&t->d_dir, t->dir_bytes));
+    K* M = (K*)t->d_dir;
+    uint32_t* dir = (uint32_t*)((uint8_t*)t->d_dir + cnt * sizeof(K));
+    build_dir_max<K><<<grid_for(cnt), 256, 0, s>>>((const K*)t->d_leaf, nd, cnt, span, M);
+    HBT_CUDA_TRY(cudaGetLastError());
+    build_dir_table<K><<<grid_for(1ull << bits), 256, 0, s>>>(M, uint32_t(cnt), bits, dir);
+    HBT_CUDA_TRY(cudaGetLastError());
   }
   HBT_CUDA_TRY(cudaStreamSynchronize(s));
   return HBT_OK;
@@ -292,17 +363,23 @@ int implicit_update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   nt.form = t->form; nt.width = t->width; nt.F = t->F; nt.device = t->device; nt.num_sms = t->num_sms;
   int rc = build_sorted_t<K>(&nt, kd, vd, uint64_t(h_nsel), s);
   cleanup();
-  if (rc != HBT_OK) { cudaFree(nt.d_leaf); cudaFree(nt.d_inner); cudaFree(nt.d_inner_idx); return rc; }
+  if (rc != HBT_OK) {
+    cudaFree(nt.d_leaf); cudaFree(nt.d_inner); cudaFree(nt.d_inner_idx); cudaFree(nt.d_dir);
+    return rc;
+  }
   cudaFree(t->d_leaf);
   cudaFree(t->d_inner);
   cudaFree(t->d_inner_idx);
+  cudaFree(t->d_dir);
   t->n = nt.n; t->L0 = nt.L0; t->H = nt.H; t->P = nt.P;
   for (int d = 0; d < HBT_MAX_LEVELS; ++d) t->nodes[d] = nt.nodes[d];
   for (int d = 0; d <= HBT_MAX_LEVELS; ++d) t->offset[d] = nt.offset[d];
   t->d_leaf = nt.d_leaf; t->leaf_bytes = nt.leaf_bytes;
   t->d_inner = nt.d_inner; t->inner_bytes = nt.inner_bytes;
   t->d_inner_idx = nt.d_inner_idx; t->inner_idx_bytes = nt.inner_idx_bytes; t->idx_stride = nt.idx_stride;
-  nt.d_leaf = nt.d_inner = nt.d_inner_idx = nullptr;
+  t->d_dir = nt.d_dir; t->dir_bytes = nt.dir_bytes; t->dir_T = nt.dir_T; t->dir_count = nt.dir_count;
+  t->dir_bits = nt.dir_bits;
+  nt.d_leaf = nt.d_inner = nt.d_inner_idx = nt.d_dir = nullptr;
   return HBT_OK;
 }
 

@@ -98,7 +98,7 @@ __device__ __forceinline__ uint32_t count_less16(const V16<K>& v, K q, unsigned 
 template <typename K, int F, int QPL, int THREADS, int MODE>
 __global__ void __launch_bounds__(THREADS)
 implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ inner_idx,
-                       const uint8_t* __restrict__ leaf, const K* __restrict__ queries, uint64_t m,
+                       const uint8_t* __restrict__ leaf, const uint32_t* __restrict__ dirbuf, const K* __restrict__ queries, uint64_t m,
                        uint64_t* __restrict__ out_pf, K* __restrict__ out_v, const LevelTable lt, uint64_t n,
                        uint64_t pos_base) {
   using C = Cfg<K, F>;
@@ -112,21 +112,28 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
   // node would sit in the same bank and the lanes' probes into different nodes
   // would serialise.  MODE 1 splits 64-bit keys into 32-bit hi / lo planes.
   constexpr uint32_t FP = F + 1;
-  const uint32_t s_nodes = uint32_t(lt.offset[SL]);
+  const uint32_t s_nodes = MODE == 2 ? 0u : uint32_t(lt.offset[SL]);
   K* s_keys = reinterpret_cast<K*>(smem);
   uint32_t* s_hi = reinterpret_cast<uint32_t*>(smem);
   uint32_t* s_lo = s_hi + s_nodes * FP;
-  for (uint32_t i = threadIdx.x; i < s_nodes * F; i += THREADS) {
-    const K key = __ldg(reinterpret_cast<const K*>(inner) + i);
-    const uint32_t a = (i / F) * FP + i % F;
-    if constexpr (MODE == 1 && sizeof(K) == 8) {
-      s_hi[a] = uint32_t(uint64_t(key) >> 32);
-      s_lo[a] = uint32_t(key);
-    } else {
-      s_keys[a] = key;
+  if constexpr (MODE == 2) {
+    // directory: [M_T (dcount keys) | 2^dbits x (u16 lo, u16 hi)]
+    const uint32_t words = (lt.dcount * uint32_t(sizeof(K)) + (4u << lt.dbits)) / 4;
+    for (uint32_t i = threadIdx.x; i < words; i += THREADS) s_hi[i] = __ldg(dirbuf + i);
+  } else {
+    for (uint32_t i = threadIdx.x; i < s_nodes * F; i += THREADS) {
+      const K key = __ldg(reinterpret_cast<const K*>(inner) + i);
+      const uint32_t a = (i / F) * FP + i % F;
+      if constexpr (MODE == 1 && sizeof(K) == 8) {
+        s_hi[a] = uint32_t(uint64_t(key) >> 32);
+        s_lo[a] = uint32_t(key);
+      } else {
+        s_keys[a] = key;
+      }
     }
   }
   __syncthreads();
+  const uint32_t* s_dir = reinterpret_cast<const uint32_t*>(smem + lt.dcount * sizeof(K));
 
   const int lane = threadIdx.x & 31;
   const int g = lane / C::G, k = lane % C::G;
@@ -146,6 +153,19 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
       myq[u] = i < m ? ldcs(queries + i) : key_max<K>();
       mynode[u] = 0;
     }
+    if constexpr (MODE == 2) {
+      // level-T node = lower_bound(M_T, q), narrowed by the prefix directory
+#pragma unroll
+      for (int u = 0; u < QPL; ++u) {
+        const uint32_t e = s_dir[uint32_t(myq[u] >> (8 * sizeof(K) - lt.dbits))];
+        uint32_t lo = e & 0xFFFFu, hi = e >> 16;
+        while (lo < hi) {
+          const uint32_t mid = (lo + hi) >> 1;
+          if (s_keys[mid] < myq[u]) lo = mid + 1; else hi = mid;
+        }
+        mynode[u] = lo;
+      }
+    } else {
     for (uint32_t d = 0; d < SL; ++d) {
       const uint32_t lvl = uint32_t(lt.offset[d]) * FP;
       uint32_t pos[QPL];
@@ -169,6 +189,7 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
       }
 #pragma unroll
       for (int u = 0; u < QPL; ++u) mynode[u] = mynode[u] * F + pos[u];
+    }
     }
     // ---- phase 2: lane groups; slot j of group g is round query j*NG + g,
     //      owned in phase 1 by lane (j*NG)%32 + g, slot (j*NG)/32
@@ -267,8 +288,18 @@ struct Launch {
     LevelTable lt{};
     for (uint32_t d = 0; d <= t->H; ++d) lt.offset[d] = t->offset[d];
     lt.H = t->H;
-    lt.SL = smem_levels(t, t->cfg.smem_budget ? t->cfg.smem_budget : kDefaultSmemBudget);
-    const size_t smem = size_t(lt.offset[lt.SL]) * (C::NODE_BYTES + C::S);  // (F+1)*S bytes per staged node
+    size_t smem;
+    if (MODE == 2) {
+      lt.SL = t->dir_T;
+      lt.dcount = t->dir_count;
+      lt.dbits = t->dir_bits;
+      smem = t->dir_bytes;
+    } else {
+      lt.SL = smem_levels(t, t->cfg.smem_budget ? t->cfg.smem_budget : kDefaultSmemBudget);
+      lt.dcount = 0;
+      lt.dbits = 0;
+      smem = size_t(lt.offset[lt.SL]) * (C::NODE_BYTES + C::S);  // (F+1)*S bytes per staged node
+    }
     static bool attr_set = false;  // per instantiation
     if (!attr_set) {
       HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
@@ -289,7 +320,7 @@ struct Launch {
     const uint64_t need = (rounds + THREADS / 32 - 1) / (THREADS / 32);
     if (need < grid) grid = need ? need : 1;
     kern<<<unsigned(grid), THREADS, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
-                                               (const uint8_t*)t->d_leaf, (const K*)q, m, pf, (K*)v, lt, t->n, base);
+                                               (const uint8_t*)t->d_leaf, (const uint32_t*)t->d_dir, (const K*)q, m, pf, (K*)v, lt, t->n, base);
     HBT_CUDA_TRY(cudaGetLastError());
     return HBT_OK;
   }
@@ -297,6 +328,10 @@ struct Launch {
   static int run(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t b, cudaStream_t s) {
     const uint32_t qpl = t->cfg.qpl ? t->cfg.qpl : 1;
     const uint32_t th = t->cfg.threads ? t->cfg.threads : 1024;
+    if (t->cfg.mode == 2) {
+      if (th == 512) return run_t<1, 512, 2>(t, q, m, pf, v, b, s);
+      return qpl == 2 ? run_t<2, 1024, 2>(t, q, m, pf, v, b, s) : run_t<1, 1024, 2>(t, q, m, pf, v, b, s);
+    }
     const bool hilo = t->cfg.mode == 1;
     if (hilo) {
       if (qpl == 2) return th == 256 ? run_t<2, 256, 1>(t, q, m, pf, v, b, s) : run_t<2, 512, 1>(t, q, m, pf, v, b, s);

@@ -43,10 +43,12 @@ def test_edge_suite_parity(hbt, width, F):
         assert t.export(hbt.SEG_LEAF).tobytes() == leaf, (n, F, width)
         assert t.export(hbt.SEG_INNER_IDX).tobytes() == expected_index_bytes(o, width), (n, F, width)
         q = query_set(k, width, rng, 3000)
-        pf, val = gpu_search(t, q, width)
         epf, ev = o.search(q)
-        assert np.array_equal(pf, epf), (n, F, width, np.nonzero(pf != epf)[0][:5])
-        assert np.array_equal(val, ev), (n, F, width)
+        for mode in (0, 2):  # staged levels / level-T directory
+            t.set_search_config(smem_mode=mode)
+            pf, val = gpu_search(t, q, width)
+            assert np.array_equal(pf, epf), (mode, n, F, width, np.nonzero(pf != epf)[0][:5])
+            assert np.array_equal(val, ev), (mode, n, F, width)
         t.close()
 
 
@@ -71,7 +73,8 @@ def expected_index_bytes(o, width):
 @pytest.mark.parametrize("width,F", [(8, 16), (4, 8), (8, 32), (4, 32)])
 @pytest.mark.parametrize("budget,threads,qpl,mode", [(16, 0, 0, 0), (4096, 256, 2, 1), (100 * 1024, 512, 1, 0),
                                                      (200 * 1024, 512, 2, 1), (64 * 1024, 256, 1, 1),
-                                                     (100 * 1024, 512, 2, 0)])
+                                                     (100 * 1024, 512, 2, 0), (0, 1024, 1, 2), (0, 512, 1, 2),
+                                                     (0, 1024, 2, 2), (0, 1024, 1, 0)])
 def test_launch_shape_variants(hbt, width, F, budget, threads, qpl, mode):
     """Results must not depend on how many top levels sit in shared memory, the
     CTA size or the queries in flight per lane."""
@@ -80,7 +83,7 @@ def test_launch_shape_variants(hbt, width, F, budget, threads, qpl, mode):
     o = oracle.ITree.from_pairs(k, v, F, width)
     t = gpu_build(hbt, k, v, F, width)
     t.set_search_config(smem_bytes=budget, threads_per_cta=threads, queries_per_lane=qpl, smem_mode=mode,
-                        carveout=100 if mode else -1)
+                        carveout=100 if mode == 1 else -1)
     q = query_set(k[:5000], width, rng, 20011)
     pf, val = gpu_search(t, q, width)
     epf, ev = o.search(q)
