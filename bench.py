@@ -1,18 +1,21 @@
 #!/usr/bin/env python
 """bench.py — batched HB+-tree lookups on B200 (one JSON line on rank 0).
 
-Workload (BASELINE.json configs[1], the metric's 1-GPU configuration): implicit
-tree, 2^23 uint64 keys, fanout 16, 2^24 uniform hit queries per GPU.  A "step"
-is one hbt_search over the whole batch (all hot-path rows: node search through
-every level, leaf search, result write).  Inputs are seeded synthetic
-(gen/); queries (128 MiB) + results (256 MiB) per step exceed the
-126 MB L2, so no explicit flush is done between steps.
+Default workload = BASELINE.json configs[1] (c2), the metric's 1-GPU config:
+implicit tree, 2^23 uint64 keys, fanout 16, 2^24 uniform hit queries per GPU.
+A "step" is one hbt_search over the whole batch (every hot-path row: the
+top-level directory / node search through every level, the leaf search and
+the result write).  Inputs are seeded synthetic (gen/) generated
+on the device; queries + results per step exceed the 126 MB L2, so no L2 flush
+is done between steps.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2|c1|c5|c3]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c1|c2|c3|c4|c5]
   python bench.py --impl reference ...   # the CPU oracle arm (rank 0 only)
 
-Multi-GPU (torchrun): every rank holds a replica and searches its own 2^24
-queries (weak scaling, no collective on the data path).
+Multi-GPU (torchrun, one process per GPU): c1/c2/c3/c5 run one replica per
+rank, each searching its own batch (weak scaling, no collective on the data
+path); c4 is the key-range-sharded tree (2^31 keys split over
+the ranks, 2^28 queries in total, NCCL all-to-all of queries and results).
 """
 from __future__ import annotations
 
@@ -32,6 +35,8 @@ sys.path.insert(0, ROOT)
 import gen  # noqa: E402
 from tools import roofline  # noqa: E402
 
+NVLINK_GBS = 770.0  # measured peer copy per direction (B200_PROFILING.md), for c4's a2a term
+
 
 def parse():
     ap = argparse.ArgumentParser()
@@ -39,12 +44,12 @@ def parse():
     ap.add_argument("--steps", type=int, default=400)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="hbt", choices=["hbt", "reference"])
-    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c5"])
+    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c4", "c5"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--smem", type=int, default=0, help="override smem budget (bytes)")
     ap.add_argument("--qpl", type=int, default=0, help="queries per lane per warp round (1|2)")
-    ap.add_argument("--threads", type=int, default=0, help="threads per CTA (256|512)")
+    ap.add_argument("--threads", type=int, default=0, help="threads per CTA (256|512|1024)")
     ap.add_argument("--smem-mode", type=int, default=None, help="2 = directory (default), 0 = staged levels, 1 = hi/lo")
     ap.add_argument("--carveout", type=int, default=-1, help="smem carve-out percent (-1 default)")
     return ap.parse_args()
@@ -118,67 +123,80 @@ def probe_l2_gbs(chunk):
         return None
 
 
-def make_workload(cfg_name, rank, dev_gen):
-    """Device keys/values and this rank's queries, plus host copies needed later."""
-    import torch
-    c = gen.CONFIGS[cfg_name]
-    n, m, w = c["n"], c["m"], c["width"]
-    sk = gen.stream_seed(c["cfg"], gen.STREAM_K)
-    sv = gen.stream_seed(c["cfg"], gen.STREAM_V)
-    sq = gen.stream_seed(c["cfg"], gen.STREAM_Q)
-    keys = dev_gen.mix_stream(n, w, sk)
-    vals = dev_gen.mix_stream(n, w, sv)
-    hit_rate = 1.0
-    if c["queries"] in ("uniform",):
-        q = dev_gen.uniform_queries(m, n, w, sq, sk, start=rank * m)
-        qdesc = "uniform hits with replacement"
-    elif c["queries"] == "shuffle":
-        hk = gen.keys(n, w, sk)
-        q = torch.from_numpy(gen.workload_queries(cfg_name, hk).view(np.int32 if w == 4 else np.int64)).cuda()
-        qdesc = "Knuth shuffle of the keys (PAPER.md:298)"
-    elif c["queries"] == "zipf":
-        hk = gen.keys(n, w, sk)
-        r = gen.zipf_ranks(m, n, c["theta"], sq, start=rank * m)
-        q = torch.from_numpy(hk[r - 1].view(np.int64)).cuda()
-        qdesc = f"Zipf({c['theta']}) over key ranks, scrambled"
-    else:
-        raise SystemExit(f"config {cfg_name} not wired into bench.py yet")
-    return keys, vals, q, hit_rate, qdesc
+# --------------------------------------------------------------------------- workloads
 
 
-def run_hbt(args):
+class Work:
+    """One rank's share of a configuration, ready to time."""
+
+    def __init__(self, **kw):
+        self.__dict__.update(kw)
+
+
+def make_work(cfg_name, rank, world, args):
     import torch
-    import torch.distributed as dist
 
     import paper_conf_sigmod_shahvaranij16_b200 as hbt
     from gen.device import GenLib
 
-    rank, world, local = dist_env()
-    torch.cuda.set_device(local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    c = gen.CONFIGS[args.config]
-    w = c["width"]
     g = GenLib()
-    keys, vals, q, hit_rate, qdesc = make_workload(args.config, rank, g)
-    m = q.numel()
-    tree = hbt.Tree(keys, vals, fanout=c["fanout"], layout=c["layout"])
+    c = gen.CONFIGS[cfg_name]
+    n, m, w, F = c["n"], c["m"], c["width"], c["fanout"]
+    sk = gen.stream_seed(c["cfg"], gen.STREAM_K)
+    sv = gen.stream_seed(c["cfg"], gen.STREAM_V)
+    sq = gen.stream_seed(c["cfg"], gen.STREAM_Q)
+    sdt = torch.int32 if w == 4 else torch.int64
+    extra = {}
+    hit_rate = 1.0
+    if cfg_name == "c4":
+        lo, hi = hbt.shard_plan(n, world, rank)
+        keys = g.stratified_keys(hi - lo, sk, start=lo)
+        vals = g.mix_stream(hi - lo, w, sv, start=lo)
+        m_local = m // world
+        q = g.stratified_queries(m_local, n, sq, sk, start=rank * m_local)
+        comm = hbt.Comm.from_torch() if world > 1 else hbt.Comm(1, 0, hbt.unique_id())
+        tree = hbt.ShardedTree(comm, keys, vals, fanout=F)
+        qdesc = f"uniform hits over all {n} keys, {m_local} per rank, routed to their owner shard"
+        extra["comm"] = comm
+        m = m_local
+    else:
+        keys = g.mix_stream(n, w, sk)
+        vals = g.mix_stream(n, w, sv)
+        if c["queries"] == "uniform":
+            q = g.uniform_queries(m, n, w, sq, sk, start=rank * m)
+            qdesc = "uniform hits with replacement"
+        elif c["queries"] == "uniform_ins":
+            bk, bv, bo, n_ins = gen.update_batch(cfg_name, n)
+            q = g.uniform_queries(m, n + n_ins, w, sq, sk, start=rank * m)
+            hit_rate = n / (n + n_ins)
+            qdesc = f"uniform over key indices [0, n + {n_ins}) (misses = not-yet-inserted keys)"
+            extra["batch"] = (torch.from_numpy(bk.view(np.int64)).cuda(), torch.from_numpy(bv.view(np.int64)).cuda(),
+                              torch.from_numpy(bo).cuda())
+        elif c["queries"] == "shuffle":
+            hk = gen.keys(n, w, sk)
+            q = torch.from_numpy(gen.workload_queries(cfg_name, hk).view(np.int32 if w == 4 else np.int64)).cuda()
+            qdesc = "Knuth shuffle of the keys (PAPER.md:298)"
+        elif c["queries"] == "zipf":
+            hk = gen.keys(n, w, sk)
+            r = gen.zipf_ranks(m, n, c["theta"], sq, start=rank * m)
+            q = torch.from_numpy(hk[r - 1].view(np.int64)).cuda()
+            qdesc = f"Zipf({c['theta']}) over key ranks, scrambled through the key order"
+        else:
+            raise SystemExit(cfg_name)
+        tree = hbt.Tree(keys, vals, fanout=F, layout=c["layout"])
+    del keys, vals
     tree.set_search_config(smem_bytes=args.smem, threads_per_cta=args.threads, queries_per_lane=args.qpl,
                            smem_mode=args.smem_mode, carveout=args.carveout)
-    info = tree.info()
-    del keys, vals
     out_pos = torch.empty(m, dtype=torch.int64, device="cuda")
-    out_val = torch.empty(m, dtype=q.dtype, device="cuda")
-    torch.cuda.synchronize()
+    out_val = torch.empty(m, dtype=sdt, device="cuda")
+    return Work(c=c, name=cfg_name, tree=tree, q=q, m=m, w=w, hit_rate=hit_rate, qdesc=qdesc, extra=extra,
+                out_pos=out_pos, out_val=out_val, info=tree.info())
 
-    l2_probe = probe_l2_gbs(min(128, ((c["fanout"] * w + 31) // 32) * 32)) if rank == 0 else None
 
-    for _ in range(max(args.warmup, 3)):
-        tree.search(q, out_pos, out_val)
-    torch.cuda.synchronize()
-
-    sampler = ClockSampler(local)
-    sampler.start()
+def time_search(work, steps, world):
+    """K launches of the step, CUDA events on the launching stream, max over ranks."""
+    import torch
+    import torch.distributed as dist
     stream = torch.cuda.current_stream()
     ev0 = torch.cuda.Event(enable_timing=True)
     ev1 = torch.cuda.Event(enable_timing=True)
@@ -186,44 +204,106 @@ def run_hbt(args):
         dist.barrier()
     torch.cuda.synchronize()
     ev0.record(stream)
-    for _ in range(args.steps):
-        tree.search(q, out_pos, out_val)
+    for _ in range(steps):
+        work.tree.search(work.q, work.out_pos, work.out_val)
     ev1.record(stream)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    clocks = sampler.stop()
-    ms = ev0.elapsed_time(ev1)
-    t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    t = torch.tensor([ev0.elapsed_time(ev1)], dtype=torch.float64, device="cuda")
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms_max = float(t.item())
-    ms_step = ms_max / args.steps
-    qps = world * m / (ms_step * 1e-3)
+    return float(t.item()) / steps
 
-    # ---- end to end through the public API with pinned HOST buffers
-    hq = q.cpu().pin_memory()
+
+def time_e2e(work, steps, world):
+    """Same metric through the public API with pinned HOST buffers (H2D + D2H inside)."""
+    import torch
+    import torch.distributed as dist
+    m, w = work.m, work.w
+    hq = work.q.cpu().pin_memory()
     hp = torch.empty(m, dtype=torch.int64).pin_memory()
-    hv = torch.empty(m, dtype=q.dtype).pin_memory()
-    tree.search_host(hq, hp, hv)  # warm the pipeline buffers
+    hv = torch.empty(m, dtype=work.q.dtype).pin_memory()
+    sharded = work.name == "c4"
+
+    def one():
+        if sharded:  # H2D, collective search, D2H on the current stream
+            dq = hq.to("cuda", non_blocking=True)
+            p, v = work.tree.search(dq)
+            hp.copy_(p, non_blocking=True)
+            hv.copy_(v, non_blocking=True)
+            torch.cuda.synchronize()
+        else:
+            work.tree.search_host(hq, hp, hv)
+
+    one()
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    for _ in range(args.e2e_steps):
-        tree.search_host(hq, hp, hv)
-    e2e_s = time.perf_counter() - t0
-    te = torch.tensor([e2e_s], dtype=torch.float64, device="cuda")
+    for _ in range(steps):
+        one()
+    el = time.perf_counter() - t0
+    te = torch.tensor([el], dtype=torch.float64, device="cuda")
     if world > 1:
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
-    e2e_qps = world * m * args.e2e_steps / float(te.item())
-    chunks = -(-m // (1 << 22))
+    qps = world * m * steps / float(te.item())
+    api = ("H2D + hbt_search_sharded + D2H (pinned host buffers)" if sharded else
+           "hbt_search_host (pinned host buffers, 4 Mi-query buckets double-buffered over 2 streams)")
+    return {"value": round(qps / 1e6, 2), "unit": "M queries/s", "h2d_bytes_per_step": m * w,
+            "d2h_bytes_per_step": m * (8 + w), "api": api,
+            "gpu_launches_per_step": (4 if sharded else -(-m // (1 << 22)))}
 
-    # ---- roofline of the (only) kernel of the step
+
+def run_hbt(args):
+    import torch
+    import torch.distributed as dist
+
+    rank, world, local = dist_env()
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    work = make_work(args.config, rank, world, args)
+    c, m, w, info = work.c, work.m, work.w, work.info
+    torch.cuda.synchronize()
+    node_b = ((c["fanout"] * w + 31) // 32) * 32
+    l2_probe = probe_l2_gbs(32 if node_b > 32 else node_b) if rank == 0 else None
+
+    for _ in range(max(args.warmup, 3)):
+        work.tree.search(work.q, work.out_pos, work.out_val)
+    torch.cuda.synchronize()
+    sampler = ClockSampler(local)
+    sampler.start()
+    ms_step = time_search(work, args.steps, world)
+    clocks = sampler.stop()
+    qps = world * m / (ms_step * 1e-3)
+    launches_per_step = 4 if args.config == "c4" else 1
+
+    after = None
+    if "batch" in work.extra:  # c3: the 1 % bulk update, timed once, then search again
+        bk, bv, bo = work.extra["batch"]
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        work.tree.update(bk, bv, bo)
+        torch.cuda.synchronize()
+        upd_s = time.perf_counter() - t0
+        for _ in range(3):
+            work.tree.search(work.q, work.out_pos, work.out_val)
+        ms_after = time_search(work, args.steps, world)
+        after = {"update_ops": int(bk.numel()), "update_ms": round(upd_s * 1e3, 3),
+                 "update_ops_per_s": round(bk.numel() / upd_s, 1),
+                 "search_after_update": {"value": round(world * m / (ms_after * 1e-3) / 1e6, 2),
+                                         "unit": "M queries/s", "ms_per_step": round(ms_after, 4)},
+                 "n_distinct_after": work.tree.info()["n_distinct"]}
+
+    e2e = time_e2e(work, args.e2e_steps, world)
+
+    # ---- roofline of the step's dominant kernel (the search)
     l2_size = torch.cuda.get_device_properties(local).L2_cache_size
-    mdl = roofline.model(info, l2_size, hit_rate)
+    mdl = roofline.model(info, l2_size, work.hit_rate)
     peak, peak_src = measured_peaks()
-    achieved = mdl["hbm_bytes_per_query"] * m / (ms_step * 1e-3) / 1e9
+    t_kernel = ms_step * 1e-3
+    achieved = mdl["hbm_bytes_per_query"] * m / t_kernel / 1e9
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
@@ -231,10 +311,16 @@ def run_hbt(args):
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
             "frac": round(achieved / peak, 4), "traffic": traffic,
             "bytes_per_query_model": round(mdl["hbm_bytes_per_query"], 2), "peak_source": peak_src,
-            "model": "ideal static L2 cache of %d B (SURVEY §8d)" % l2_size}
+            "model": "ideal static L2 cache of %d B (SURVEY §8d)%s" % (
+                l2_size, "; Zipf modelled as uniform (upper bound on bytes)" if args.config == "c5" else "")}
+    if args.config == "c4" and world > 1:
+        a2a_b = (world - 1) / world * (w + 8 + w)
+        t_roof = mdl["hbm_bytes_per_query"] / (peak * 1e9) + a2a_b / (NVLINK_GBS * 1e9)
+        roof["a2a_bytes_per_query"] = round(a2a_b, 2)
+        roof["frac_with_nvlink"] = round((m / t_kernel) * t_roof, 4)
     l2_roof = None
     if l2_probe:
-        l2_ach = mdl["l2_bytes_per_query"] * m / (ms_step * 1e-3) / 1e9
+        l2_ach = mdl["l2_bytes_per_query"] * m / t_kernel / 1e9
         l2_roof = {"bound": "l2", "achieved": round(l2_ach, 1), "peak": round(l2_probe, 1), "unit": "GB/s",
                    "frac": round(l2_ach / l2_probe, 4), "bytes_per_query_model": mdl["l2_bytes_per_query"],
                    "peak_source": "in-run random-read probe, 32 MB buffer (tools/probe.cu)"}
@@ -245,58 +331,68 @@ def run_hbt(args):
 
     if world > 1:
         dist.barrier()
+    if rank == 0:
+        line = {
+            "metric": "lookups/sec (M queries/s)",
+            "value": round(qps / 1e6, 2),
+            "unit": "M queries/s",
+            "n_gpus": world,
+            "steps": args.steps,
+            "warmup": max(args.warmup, 3),
+            "ms_per_step": round(ms_step, 4),
+            "higher_is_better": True,
+            "scaling": "weak",
+            "vs_baseline": None,
+            "dtype": "u64" if w == 8 else "u32",
+            "data": "synthetic (seeded counter-based generators, gen/)",
+            "config": {"workload": f"{args.config}: {c['layout']} tree, n={c['n']} keys (u{8 * w}), fanout "
+                                   f"{c['fanout']}, m={m} queries/GPU ({work.qdesc})",
+                       "n_keys": c["n"], "queries_per_gpu": m, "fanout": c["fanout"], "layout": c["layout"],
+                       "key_bits": 8 * w,
+                       "parallelism": (f"key-range sharded x{world}" if args.config == "c4" else
+                                       (f"replicated x{world}" if world > 1 else "single")),
+                       "l2_policy": "inputs larger than L2 (queries+results %d MiB/step/GPU > 126 MB L2)"
+                                    % (m * (2 * w + 8) >> 20),
+                       "tree": {k: info[k] for k in ("height", "smem_levels", "level_nodes", "leaf_lines",
+                                                     "chain_len", "inner_bytes", "leaf_bytes", "n_distinct")}},
+            "e2e": e2e,
+            "gpu_launches": args.steps * launches_per_step,
+            "roofline": roof,
+            "roofline_l2": l2_roof,
+            "clocks": clocks,
+            "cpu_baseline": cpu,
+            "context": "paper: up to 240 M queries/s (HB+ implicit, GTX 780 + Xeon E5-2665, PAPER.md:9,57)",
+        }
+        if after:
+            line["update"] = after
+        print(json.dumps(line), flush=True)
+    if world > 1:
         dist.destroy_process_group()
-    if rank != 0:
-        return
-    line = {
-        "metric": "lookups/sec (M queries/s)",
-        "value": round(qps / 1e6, 2),
-        "unit": "M queries/s",
-        "n_gpus": world,
-        "steps": args.steps,
-        "warmup": max(args.warmup, 3),
-        "ms_per_step": round(ms_step, 4),
-        "higher_is_better": True,
-        "scaling": "weak",
-        "vs_baseline": None,
-        "dtype": "u64" if w == 8 else "u32",
-        "data": "synthetic (seeded counter-based generators, gen/)",
-        "config": {"workload": f"{args.config}: {c['layout']} tree, n={c['n']} keys (u{8 * w}), fanout {c['fanout']}, "
-                               f"m={m} queries/GPU ({qdesc})",
-                   "n_keys": c["n"], "queries_per_gpu": m, "fanout": c["fanout"], "layout": c["layout"],
-                   "key_bits": 8 * w, "parallelism": f"replicated x{world}" if world > 1 else "single",
-                   "l2_policy": "inputs larger than L2 (queries+results %d MiB/step > L2)" % (m * (2 * w + 8) >> 20),
-                   "tree": {"height": info["height"], "smem_levels": info["smem_levels"],
-                            "level_nodes": info["level_nodes"], "leaf_lines": info["leaf_lines"],
-                            "inner_bytes": info["inner_bytes"], "leaf_bytes": info["leaf_bytes"]}},
-        "e2e": {"value": round(e2e_qps / 1e6, 2), "unit": "M queries/s", "h2d_bytes_per_step": m * w,
-                "d2h_bytes_per_step": m * (8 + w), "api": "hbt_search_host (pinned host buffers, 4 Mi-query buckets "
-                "double-buffered over 2 streams)", "gpu_launches_per_step": chunks},
-        "gpu_launches": args.steps,
-        "roofline": roof,
-        "roofline_l2": l2_roof,
-        "clocks": clocks,
-        "cpu_baseline": cpu,
-        "context": "paper: up to 240 M queries/s (HB+ implicit, GTX 780 + Xeon E5-2665, PAPER.md:9,57)",
-    }
-    print(json.dumps(line), flush=True)
+
+
+def _oracle_workload(cfg_name, m):
+    """Host copy of the config's keys/values and an m-query sample (same generators)."""
+    c = gen.CONFIGS[cfg_name]
+    k, v = gen.workload_keys_values(cfg_name)
+    if cfg_name == "c3":
+        _, _, _, n_ins = gen.update_batch(cfg_name, len(k))
+        return c, k, v, gen.workload_queries(cfg_name, k, m, n_ins=n_ins)
+    if cfg_name == "c1":
+        return c, k, v, gen.workload_queries(cfg_name, k)
+    return c, k, v, gen.workload_queries(cfg_name, k, m)
 
 
 def cpu_baseline(cfg_name, target_s=8.0):
     """The oracle as it stands, on this host's cores, over a bounded sample."""
     import oracle
-    c = gen.CONFIGS[cfg_name]
-    n, w = c["n"], c["width"]
-    k, v = gen.workload_keys_values(cfg_name)
+    if cfg_name == "c4":
+        return {"value": None, "unit": "M queries/s", "cores": oracle.default_threads(), "kind": "oracle",
+                "sample": "not run: the 2^31-key oracle tree needs ~80 GB of host RAM and minutes to build"}
+    c, k, v, q = _oracle_workload(cfg_name, 1 << 20)
     t0 = time.perf_counter()
-    if c["layout"] == "implicit":
-        tree = oracle.ITree.from_pairs(k, v, c["fanout"], w)
-    else:
-        tree = oracle.RTree.from_pairs(k, v, c["fanout"], w)
+    tree = (oracle.ITree if c["layout"] == "implicit" else oracle.RTree).from_pairs(k, v, c["fanout"], c["width"])
     build_s = time.perf_counter() - t0
     cores = oracle.default_threads()
-    m = 1 << 20
-    q = gen.workload_queries(cfg_name, k, m) if cfg_name != "c1" else gen.workload_queries(cfg_name, k)
     tree.search(q[: 1 << 16], nthreads=cores)
     t0 = time.perf_counter()
     reps = 0
@@ -318,28 +414,27 @@ def run_reference(args):
     if rank != 0:
         return
     import oracle
-    c = gen.CONFIGS[args.config]
-    w = c["width"]
-    k, v = gen.workload_keys_values(args.config)
-    tree = (oracle.ITree if c["layout"] == "implicit" else oracle.RTree).from_pairs(k, v, c["fanout"], w)
+    cfg = args.config if args.config != "c4" else "c2"
+    c, k, v, q = _oracle_workload(cfg, 1 << 20)
+    tree = (oracle.ITree if c["layout"] == "implicit" else oracle.RTree).from_pairs(k, v, c["fanout"], c["width"])
     cores = oracle.default_threads()
-    m = 1 << 20
-    q = gen.workload_queries(args.config, k, m)
-    for _ in range(args.warmup):
+    for _ in range(max(args.warmup, 1)):
         tree.search(q, nthreads=cores)
+    steps = max(1, min(args.steps, 200))
     t0 = time.perf_counter()
-    for _ in range(args.steps):
+    for _ in range(steps):
         tree.search(q, nthreads=cores)
     el = time.perf_counter() - t0
-    qps = args.steps * len(q) / el
+    qps = steps * len(q) / el
     val = round(qps / 1e6, 3)
     line = {
         "impl": "reference", "metric": "lookups/sec (M queries/s)", "value": val, "unit": "M queries/s",
-        "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(el / args.steps * 1e3, 3),
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64" if w == 8 else "u32",
-        "data": "synthetic", "config": {"workload": f"{args.config} (oracle, {len(q)}-query sample per step)"},
+        "n_gpus": world, "steps": steps, "warmup": args.warmup, "ms_per_step": round(el / steps * 1e3, 3),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64" if c["width"] == 8 else "u32",
+        "data": "synthetic", "config": {"workload": f"{cfg} (oracle tree search on {cores} host threads, "
+                                                     f"{len(q)}-query sample per step)"},
         "cpu_baseline": {"value": val, "unit": "M queries/s", "cores": cores, "kind": "oracle",
-                         "sample": f"{len(q)} queries of {args.config} per step"},
+                         "sample": f"{len(q)} queries of {cfg} per step, {steps} steps"},
         "e2e": {"value": val, "unit": "M queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)

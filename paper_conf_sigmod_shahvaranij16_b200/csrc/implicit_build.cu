@@ -176,6 +176,29 @@ inline unsigned grid_for(uint64_t n) {
   return unsigned(g ? g : 1);
 }
 
+// 1 if keys[] is strictly increasing (already sorted and distinct), else 0.
+template <typename K>
+__global__ void strictly_increasing(const K* __restrict__ k, uint64_t n, int* __restrict__ bad) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i + 1 < n; i += uint64_t(gridDim.x) * blockDim.x)
+    if (!(k[i] < k[i + 1])) { *bad = 1; return; }
+}
+
+template <typename K>
+int is_sorted_distinct(const void* keys, uint64_t n, bool* out, cudaStream_t s) {
+  *out = false;
+  int* d = nullptr;
+  HBT_CUDA_TRY(cudaMalloc(&d, sizeof(int)));
+  cudaMemsetAsync(d, 0, sizeof(int), s);
+  strictly_increasing<K><<<grid_for(n), 256, 0, s>>>((const K*)keys, n, d);
+  int h = 1;
+  cudaMemcpyAsync(&h, d, sizeof(int), cudaMemcpyDeviceToHost, s);
+  cudaError_t e = cudaStreamSynchronize(s);
+  cudaFree(d);
+  if (e != cudaSuccess) { set_error("sorted check: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
+  *out = (h == 0);
+  return HBT_OK;
+}
+
 template <typename K>
 int sort_dedupe_t(const void* keys, const void* values, uint64_t n, void** out_k, void** out_v, uint64_t* nd,
                   cudaStream_t s) {
@@ -397,9 +420,17 @@ int implicit_build_sorted(hbt_tree* t, const void* kd, const void* vd, uint64_t 
 }
 
 int implicit_build(hbt_tree* t, const void* keys, const void* values, uint64_t n, cudaStream_t s) {
+  // Presorted distinct input (e.g. c4's stratified keys): build straight from it
+  // (no sort workspace: 2^31 u64 pairs would otherwise need ~100 GB of temporaries).
+  bool sorted = false;
+  int rc = n ? (t->width == 4 ? is_sorted_distinct<uint32_t>(keys, n, &sorted, s)
+                              : is_sorted_distinct<uint64_t>(keys, n, &sorted, s))
+             : HBT_OK;
+  if (rc != HBT_OK) return rc;
+  if (sorted) return implicit_build_sorted(t, keys, values, n, s);
   void *kd = nullptr, *vd = nullptr;
   uint64_t nd = 0;
-  int rc = sort_dedupe(t->width, keys, values, n, &kd, &vd, &nd, s);
+  rc = sort_dedupe(t->width, keys, values, n, &kd, &vd, &nd, s);
   if (rc != HBT_OK) return rc;
   rc = implicit_build_sorted(t, kd, vd, nd, s);
   cudaFree(kd);

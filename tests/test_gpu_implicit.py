@@ -227,3 +227,25 @@ def test_device_generators_match_numpy():
                               gen.uniform_hit_queries(keys, 50000, sq, start=3).astype(np.uint64))
     s = gen.stream_seed(4, gen.STREAM_K)
     assert np.array_equal(from_dev(g.stratified_keys(1000, s, start=5), 8), gen.stratified_keys(1000, s, start=5))
+
+
+@pytest.mark.parametrize("width", [4, 8])
+def test_presorted_input_fast_path(hbt, width):
+    """Strictly increasing input skips the sort (c4's stratified keys); a sorted
+    input with a duplicate must still take the sort + dedupe path."""
+    rng = np.random.default_rng(width)
+    k, v = gen_keys(50000, width, rng)
+    Kd, Vd = oracle.dedupe(k, v)
+    o = oracle.ITree(Kd, Vd, 16, width)
+    t = gpu_build(hbt, Kd, Vd, 16, width)
+    inner, leaf = expected_implicit_bytes(o, width)
+    assert t.export(hbt.SEG_INNER).tobytes() == inner and t.export(hbt.SEG_LEAF).tobytes() == leaf
+    q = query_set(Kd[:3000], width, rng, 3000)
+    pf, val = gpu_search(t, q, width)
+    epf, ev = o.search(q)
+    assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+    kd2 = np.insert(Kd, 100, Kd[100])  # sorted, not distinct: last occurrence wins
+    vd2 = np.insert(Vd, 101, np.uint64(7))
+    o2 = oracle.ITree.from_pairs(kd2, vd2, 16, width)
+    t2 = gpu_build(hbt, kd2, vd2, 16, width)
+    assert t2.export(hbt.SEG_LEAF).tobytes() == expected_implicit_bytes(o2, width)[1]
