@@ -52,6 +52,7 @@ def parse():
     ap.add_argument("--threads", type=int, default=0, help="threads per CTA (256|512|1024)")
     ap.add_argument("--smem-mode", type=int, default=None, help="2 = directory (default), 0 = staged levels, 1 = hi/lo")
     ap.add_argument("--carveout", type=int, default=-1, help="smem carve-out percent (-1 default)")
+    ap.add_argument("--l2-persist", type=int, default=None, help="bytes of I-segment in a persisting L2 window")
     return ap.parse_args()
 
 
@@ -187,6 +188,8 @@ def make_work(cfg_name, rank, world, args):
     del keys, vals
     tree.set_search_config(smem_bytes=args.smem, threads_per_cta=args.threads, queries_per_lane=args.qpl,
                            smem_mode=args.smem_mode, carveout=args.carveout)
+    if args.l2_persist is not None and c["layout"] == "implicit":
+        tree.set_param("l2_persist", args.l2_persist)
     out_pos = torch.empty(m, dtype=torch.int64, device="cuda")
     out_val = torch.empty(m, dtype=sdt, device="cuda")
     return Work(c=c, name=cfg_name, tree=tree, q=q, m=m, w=w, hit_rate=hit_rate, qdesc=qdesc, extra=extra,

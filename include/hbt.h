@@ -167,6 +167,8 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *   "smem_mode"   implicit top levels: 2 = level-T directory + one lower bound (default),
  *                 0 = per-level binary search of staged nodes, 1 = the same on 32-bit hi/lo planes
  *   "carveout"    preferred shared-memory carve-out percent, -1 = driver default
+ *   "l2_persist"  implicit: keep up to this many bytes of the I-segment (+ index) in a
+ *                 persisting L2 access-policy window (sets the device persisting-L2 limit), 0 = off
  * Unknown names or out-of-range values return HBT_EINVAL. */
 HBT_API int hbt_set_param(hbt_tree* t, const char* name, int64_t value);
 

@@ -36,8 +36,7 @@ static bool is_device_ptr(const void* p) {
 
 static void free_tree(hbt_tree* t) {
   if (!t) return;
-  cudaFree(t->d_inner);
-  cudaFree(t->d_inner_idx);
+  cudaFree(t->d_inner);  // also holds d_inner_idx
   cudaFree(t->d_dir);
   cudaFree(t->d_leaf);
   regular_free(t);
@@ -250,6 +249,7 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "qpl" && value >= 0 && value <= 2) c.qpl = uint32_t(value);
   else if (n == "smem_mode" && value >= 0 && value <= 2) c.mode = uint32_t(value);
   else if (n == "carveout" && value >= -1 && value <= 100) c.carveout = int(value);
+  else if (n == "l2_persist" && value >= 0) c.l2_persist = uint64_t(value);
   else {
     set_error("bad parameter %s = %lld", name, (long long)value);
     return HBT_EINVAL;

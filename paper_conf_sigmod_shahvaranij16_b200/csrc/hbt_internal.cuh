@@ -41,6 +41,7 @@ struct SearchConfig {
   uint32_t qpl = 0;              // queries per lane per warp round (0 = default)
   uint32_t mode = 2;             // top-level mode: 0 = staged levels (K words), 1 = hi/lo planes, 2 = directory
   int carveout = -1;             // shared-memory carve-out percent (-1 = driver default)
+  uint64_t l2_persist = 0;       // bytes of the I-segment to keep in a persisting L2 window (0 = off)
 };
 
 // Regular-tree device state.  All pools are SoA arrays

@@ -278,7 +278,13 @@ int build_sorted_t(hbt_tree* t, const K* kd, const K* vd, uint64_t nd, cudaStrea
   t->inner_bytes = t->offset[H] * F * sizeof(K);
   t->leaf_bytes = t->L0 * 64;
   HBT_CUDA_TRY(cudaMalloc(&t->d_leaf, t->leaf_bytes));
-  if (t->inner_bytes) HBT_CUDA_TRY(cudaMalloc(&t->d_inner, t->inner_bytes));
+  // I-segment and its derived index share ONE allocation so that a single L2
+  // access-policy window can cover both (search: "l2_persist").
+  t->idx_stride = H ? implicit_idx_stride(F, sizeof(K)) : 0;
+  t->inner_idx_bytes = t->offset[H] * t->idx_stride;
+  const uint64_t inner_al = (t->inner_bytes + 255) & ~uint64_t(255);
+  if (t->inner_bytes) HBT_CUDA_TRY(cudaMalloc(&t->d_inner, inner_al + t->inner_idx_bytes));
+  t->d_inner_idx = t->inner_idx_bytes ? (uint8_t*)t->d_inner + inner_al : nullptr;
   pack_leaf_lines<K><<<grid_for(t->L0 * P), 256, 0, s>>>(kd, vd, nd, t->L0, (K*)t->d_leaf);
   HBT_CUDA_TRY(cudaGetLastError());
   if (H) {
@@ -288,11 +294,8 @@ int build_sorted_t(hbt_tree* t, const K* kd, const K* vd, uint64_t nd, cudaStrea
     lt.SL = 0;
     gather_separators<K><<<grid_for(t->offset[H] * F), 256, 0, s>>>(kd, nd, lt, t->L0, F, (K*)t->d_inner);
     HBT_CUDA_TRY(cudaGetLastError());
-    t->idx_stride = implicit_idx_stride(F, sizeof(K));
     if (t->idx_stride) {
       const uint32_t ie = t->idx_stride / sizeof(K);
-      t->inner_idx_bytes = t->offset[H] * t->idx_stride;
-      HBT_CUDA_TRY(cudaMalloc(&t->d_inner_idx, t->inner_idx_bytes));
       derive_inner_index<K><<<grid_for(t->offset[H] * ie), 256, 0, s>>>((const K*)t->d_inner, t->offset[H], F, ie,
                                                                          (K*)t->d_inner_idx);
       HBT_CUDA_TRY(cudaGetLastError());
@@ -387,12 +390,11 @@ int implicit_update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   int rc = build_sorted_t<K>(&nt, kd, vd, uint64_t(h_nsel), s);
   cleanup();
   if (rc != HBT_OK) {
-    cudaFree(nt.d_leaf); cudaFree(nt.d_inner); cudaFree(nt.d_inner_idx); cudaFree(nt.d_dir);
+    cudaFree(nt.d_leaf); cudaFree(nt.d_inner); cudaFree(nt.d_dir);
     return rc;
   }
   cudaFree(t->d_leaf);
-  cudaFree(t->d_inner);
-  cudaFree(t->d_inner_idx);
+  cudaFree(t->d_inner);  // also holds the derived index
   cudaFree(t->d_dir);
   t->n = nt.n; t->L0 = nt.L0; t->H = nt.H; t->P = nt.P;
   for (int d = 0; d < HBT_MAX_LEVELS; ++d) t->nodes[d] = nt.nodes[d];

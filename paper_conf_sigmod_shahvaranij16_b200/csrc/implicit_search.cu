@@ -22,6 +22,8 @@
 //  trip; s = popc(ballot(key < q)); r = line*P + s; found = r < n' && key[s] == q.
 // Queries and results stream with evict-first (.cs) accesses so they do not
 // displace the tree from L2.
+#include <algorithm>
+
 #include "hbt_internal.cuh"
 
 namespace hbt {
@@ -319,8 +321,34 @@ struct Launch {
     uint64_t grid = uint64_t(t->num_sms) * occ;
     const uint64_t need = (rounds + THREADS / 32 - 1) / (THREADS / 32);
     if (need < grid) grid = need ? need : 1;
-    kern<<<unsigned(grid), THREADS, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
-                                               (const uint8_t*)t->d_leaf, (const uint32_t*)t->d_dir, (const K*)q, m, pf, (K*)v, lt, t->n, base);
+    cudaLaunchConfig_t lc = {};
+    lc.gridDim = dim3(unsigned(grid));
+    lc.blockDim = dim3(THREADS);
+    lc.dynamicSmemBytes = smem;
+    lc.stream = s;
+    cudaLaunchAttribute attr[1];
+    lc.attrs = attr;
+    lc.numAttrs = 0;
+    if (t->cfg.l2_persist && t->d_inner) {
+      // Keep the inner levels resident against the leaf / query / result streams.
+      static uint64_t limit_set = 0;
+      const uint64_t win = std::min<uint64_t>(t->cfg.l2_persist,
+                                              ((t->inner_bytes + 255) & ~uint64_t(255)) + t->inner_idx_bytes);
+      if (limit_set < win) {
+        HBT_CUDA_TRY(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, win));
+        limit_set = win;
+      }
+      attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
+      attr[0].val.accessPolicyWindow.base_ptr = t->d_inner;
+      attr[0].val.accessPolicyWindow.num_bytes = win;
+      attr[0].val.accessPolicyWindow.hitRatio = 1.0f;
+      attr[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+      attr[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+      lc.numAttrs = 1;
+    }
+    HBT_CUDA_TRY(cudaLaunchKernelEx(&lc, kern, (const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
+                                    (const uint8_t*)t->d_leaf, (const uint32_t*)t->d_dir, (const K*)q, m, pf,
+                                    (K*)v, lt, t->n, base));
     HBT_CUDA_TRY(cudaGetLastError());
     return HBT_OK;
   }
