@@ -53,6 +53,7 @@ def parse():
     ap.add_argument("--smem-mode", type=int, default=None, help="2 = directory (default), 0 = staged levels, 1 = hi/lo")
     ap.add_argument("--carveout", type=int, default=-1, help="smem carve-out percent (-1 default)")
     ap.add_argument("--l2-persist", type=int, default=None, help="bytes of I-segment in a persisting L2 window")
+    ap.add_argument("--l2-levels", type=int, default=None, help="L2 budget for index+sector levels (bytes)")
     return ap.parse_args()
 
 
@@ -190,6 +191,8 @@ def make_work(cfg_name, rank, world, args):
                            smem_mode=args.smem_mode, carveout=args.carveout)
     if args.l2_persist is not None and c["layout"] == "implicit":
         tree.set_param("l2_persist", args.l2_persist)
+    if args.l2_levels is not None and c["layout"] == "implicit":
+        tree.set_param("l2_levels_bytes", args.l2_levels)
     out_pos = torch.empty(m, dtype=torch.int64, device="cuda")
     out_val = torch.empty(m, dtype=sdt, device="cuda")
     return Work(c=c, name=cfg_name, tree=tree, q=q, m=m, w=w, hit_rate=hit_rate, qdesc=qdesc, extra=extra,

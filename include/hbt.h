@@ -169,6 +169,9 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *   "carveout"    preferred shared-memory carve-out percent, -1 = driver default
  *   "l2_persist"  implicit: keep up to this many bytes of the I-segment (+ index) in a
  *                 persisting L2 access-policy window (sets the device persisting-L2 limit), 0 = off
+ *   "l2_levels_bytes" implicit: inner levels below the shared-memory top are read as index
+ *                 sector + one key sector while their cumulative bytes fit this L2 budget,
+ *                 as whole nodes beyond it (0 = default 32 MB; 1 = every level whole)
  * Unknown names or out-of-range values return HBT_EINVAL. */
 HBT_API int hbt_set_param(hbt_tree* t, const char* name, int64_t value);
 

@@ -250,6 +250,7 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "smem_mode" && value >= 0 && value <= 2) c.mode = uint32_t(value);
   else if (n == "carveout" && value >= -1 && value <= 100) c.carveout = int(value);
   else if (n == "l2_persist" && value >= 0) c.l2_persist = uint64_t(value);
+  else if (n == "l2_levels_bytes" && value >= 0) c.l2_levels_bytes = uint64_t(value);
   else {
     set_error("bad parameter %s = %lld", name, (long long)value);
     return HBT_EINVAL;

@@ -32,6 +32,7 @@ struct LevelTable {
   uint32_t SL;  // levels [0, SL) searched in shared memory (mode 2: = the directory level T)
   uint32_t dcount;  // mode 2: nodes at level T
   uint32_t dbits;   // mode 2: directory prefix bits
+  uint32_t full_mask;  // bit d: read level d's nodes whole (not index + sector)
 };
 
 struct SearchConfig {
@@ -42,6 +43,7 @@ struct SearchConfig {
   uint32_t mode = 2;             // top-level mode: 0 = staged levels (K words), 1 = hi/lo planes, 2 = directory
   int carveout = -1;             // shared-memory carve-out percent (-1 = driver default)
   uint64_t l2_persist = 0;       // bytes of the I-segment to keep in a persisting L2 window (0 = off)
+  uint64_t l2_levels_bytes = 0;  // L2-resident budget for index+sector levels (0 = default 32 MB)
 };
 
 // Regular-tree device state.  All pools are SoA arrays

@@ -205,6 +205,32 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
     }
     for (uint32_t d = SL; d < H; ++d) {
       const uint8_t* lvl = inner + lt.offset[d] * C::NODE_BYTES;
+      if constexpr (C::HAS_IDX) {
+        if ((lt.full_mask >> d) & 1u) {
+          // Level beyond the L2-resident budget: a miss costs a whole DRAM line
+          // anyway, so read the full node in ONE round trip (each of the G lanes
+          // loads NODE_BYTES/G contiguous bytes) instead of index + sector.
+          constexpr int NCH = C::NODE_BYTES / C::G / 16;
+          V16<K> fv[QPG][NCH];
+#pragma unroll
+          for (int j = 0; j < QPG; ++j)
+#pragma unroll
+            for (int h = 0; h < NCH; ++h)
+              ld16(fv[j][h], lvl + uint64_t(node[j]) * C::NODE_BYTES + (k * NCH + h) * 16);
+#pragma unroll
+          for (int j = 0; j < QPG; ++j) {
+            uint32_t c = 0;
+#pragma unroll
+            for (int h = 0; h < NCH; ++h)
+#pragma unroll
+              for (int e = 0; e < 16 / C::S; ++e) c += (fv[j][h].k[e] < q[j]) ? 1u : 0u;
+#pragma unroll
+            for (int x = 1; x < C::G; x <<= 1) c += __shfl_xor_sync(0xffffffffu, c, x);
+            node[j] = node[j] * F + c;
+          }
+          continue;
+        }
+      }
       uint32_t sec[QPG];
       if constexpr (C::HAS_IDX) {
         const uint8_t* lidx = inner_idx + lt.offset[d] * C::IDXB;
@@ -290,6 +316,9 @@ struct Launch {
     LevelTable lt{};
     for (uint32_t d = 0; d <= t->H; ++d) lt.offset[d] = t->offset[d];
     lt.H = t->H;
+    // Levels whose cumulative footprint (from the first global level down) exceeds
+    // the L2-resident budget are read as whole nodes (see the kernel).
+    lt.full_mask = 0;
     size_t smem;
     if (MODE == 2) {
       lt.SL = t->dir_T;
@@ -312,6 +341,14 @@ struct Launch {
       HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout,
                                         t->cfg.carveout >= 0 ? t->cfg.carveout : int(cudaSharedmemCarveoutDefault)));
       carve = t->cfg.carveout;
+    }
+    {
+      uint64_t cum = 0;
+      const uint64_t budget = t->cfg.l2_levels_bytes ? t->cfg.l2_levels_bytes : (32ull << 20);
+      for (uint32_t d = lt.SL; d < t->H; ++d) {
+        cum += t->nodes[d] * uint64_t(C::NODE_BYTES + C::IDXB);
+        if (C::HAS_IDX && cum > budget && d < 32) lt.full_mask |= 1u << d;
+      }
     }
     int occ = 0;
     HBT_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, THREADS, smem));
@@ -355,7 +392,8 @@ struct Launch {
 
   static int run(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t b, cudaStream_t s) {
     const uint32_t qpl = t->cfg.qpl ? t->cfg.qpl : 1;
-    const uint32_t th = t->cfg.threads ? t->cfg.threads : 1024;
+    // 256-byte nodes (u64, F = 32) need more registers than a 1024-thread CTA allows
+    const uint32_t th = t->cfg.threads ? t->cfg.threads : (C::NODE_BYTES > 128 ? 512 : 1024);
     if (t->cfg.mode == 2) {
       if (th == 512) return run_t<1, 512, 2>(t, q, m, pf, v, b, s);
       return qpl == 2 ? run_t<2, 1024, 2>(t, q, m, pf, v, b, s) : run_t<1, 1024, 2>(t, q, m, pf, v, b, s);

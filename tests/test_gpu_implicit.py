@@ -44,8 +44,9 @@ def test_edge_suite_parity(hbt, width, F):
         assert t.export(hbt.SEG_INNER_IDX).tobytes() == expected_index_bytes(o, width), (n, F, width)
         q = query_set(k, width, rng, 3000)
         epf, ev = o.search(q)
-        for mode in (0, 2):  # staged levels / level-T directory
+        for mode, l2b in ((0, 0), (2, 0), (2, 1), (0, 1)):  # staged levels / directory x index+sector / whole nodes
             t.set_search_config(smem_mode=mode)
+            t.set_param("l2_levels_bytes", l2b)
             pf, val = gpu_search(t, q, width)
             assert np.array_equal(pf, epf), (mode, n, F, width, np.nonzero(pf != epf)[0][:5])
             assert np.array_equal(val, ev), (mode, n, F, width)

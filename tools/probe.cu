@@ -43,6 +43,16 @@ __global__ void __launch_bounds__(512) l2_random_read(const uint4* __restrict__ 
 
 // Returns achieved GB/s for the given chunk size (32, 64 or 128 B) over a
 // `bytes`-sized buffer (keep it below L2 for an L2 figure), or <0 on error.
+PROBE_API int probe_set_l2_fetch(int bytes) {
+  return int(cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, size_t(bytes)));
+}
+
+PROBE_API int probe_get_l2_fetch(void) {
+  size_t v = 0;
+  cudaDeviceGetLimit(&v, cudaLimitMaxL2FetchGranularity);
+  return int(v);
+}
+
 PROBE_API double probe_random_read_gbs(uint64_t bytes, int chunk, int reps) {
   uint4* buf = nullptr;
   uint4* sink = nullptr;
