@@ -67,6 +67,11 @@ struct RegularState {
   uint32_t* d_seg_of_leaf = nullptr;     // pool-sized: leaf -> update segment (0xFFFFFFFF = none)
   uint64_t seg_cap = 0;
   uint32_t root_leaf = 0;                // chain[0] (the root when U == 0)
+  // directory over root-first level T (search mode 2), rebuilt with the upper levels:
+  // d_dir = [M_T: dir_count keys | 2^dir_bits x (u16 lo, u16 hi)]
+  void* d_dir = nullptr;
+  uint64_t dir_bytes = 0, dir_cap = 0;
+  uint32_t dir_T = 0, dir_count = 0, dir_bits = 0;
 };
 
 struct HostPipe {

@@ -129,6 +129,51 @@ __global__ void build_upper_level(const uint32_t* __restrict__ child_ids, uint64
   }
 }
 
+// Directory over root-first level T (search mode 2; same argument as the
+// implicit tree's, implicit_build.cu): the descent through levels 0..T-1
+// reaches the FIRST level-T node whose max key is >= q (the last node
+// otherwise), so node_T(q) = lower_bound(M_T, q) with M_T[j] = max key below
+// level-T node j and M_T[last] = MAX.  Level-T nodes sit in key order at pool
+// indices uoff + j (upper levels are regrouped in chain order), and node j
+// covers chain leaves [j*span, (j+1)*span) with span = F^(U-T).
+template <typename K>
+__global__ void reg_dir_max(const K* __restrict__ leaf, const uint32_t* __restrict__ count,
+                            const uint32_t* __restrict__ chain, uint64_t nchain, uint32_t F, uint64_t nodes,
+                            uint64_t span, K* __restrict__ M) {
+  constexpr uint32_t P = Geo<K>::P;
+  GRID_STRIDE(j, nodes) {
+    if (j + 1 == nodes) {
+      M[j] = key_max<K>();
+    } else {
+      uint64_t e = (j + 1) * span;
+      if (e > nchain) e = nchain;
+      const uint64_t v = chain[e - 1];
+      const uint32_t c = count[v];
+      M[j] = c ? leaf[(v * F + (c - 1) / P) * (2 * P) + (c - 1) % P] : key_max<K>();
+    }
+  }
+}
+
+template <typename K>
+__device__ __forceinline__ uint32_t lower_bound_u(const K* M, uint32_t n, K q) {
+  uint32_t lo = 0, hi = n - 1;
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (M[mid] < q) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
+template <typename K>
+__global__ void reg_dir_table(const K* __restrict__ M, uint32_t n, uint32_t bits, uint32_t* __restrict__ dir) {
+  const uint32_t shift = 8 * sizeof(K) - bits;
+  GRID_STRIDE(p, (1ull << bits)) {
+    const K first = K(K(p) << shift);
+    const K last = K(first | K((K(1) << shift) - 1));
+    dir[p] = lower_bound_u(M, n, first) | (lower_bound_u(M, n, last) << 16);
+  }
+}
+
 // ---------------------------------------------------------------- search kernel
 
 struct RView {
@@ -360,6 +405,167 @@ regular_search_kernel(const RView rv, const K* __restrict__ queries, uint64_t m,
   }
 }
 
+// Search v2 (mode 2, default).  Phase 1: ONE lane per query finds its node at
+// root-first level T through the directory + a lower bound over M_T (shared
+// memory).  Phase 2: groups of G = 2 lanes per query, 2*QPL queries in flight
+// per group: per upper level index sector -> ONE 64 B key line -> one
+// reference; last level index -> key line -> line j of big leaf v;
+// leaf key sector + value sector.  Every load instruction touches one 32 B
+// sector per group; no barriers, no divergence except the MAX slow path.
+struct RDir {
+  uint32_t T, count, bits;
+  uint64_t T_base;  // pool index of level T's first node (T < U), unused when T == U
+};
+
+template <typename K, int F, int QPL, int THREADS>
+__global__ void __launch_bounds__(THREADS)
+regular_search_v2(const RView rv, const RDir rd, const uint32_t* __restrict__ dirbuf,
+                  const uint32_t* __restrict__ chain, const K* __restrict__ queries, uint64_t m,
+                  uint64_t* __restrict__ out_pf, K* __restrict__ out_v) {
+  constexpr int G = 2, NG = 16, ROUND = 32 * QPL, QPG = ROUND / NG;
+  constexpr uint32_t S = sizeof(K), P = Geo<K>::P, KPL = Geo<K>::KPL;
+  constexpr uint32_t E16 = 16 / S;
+  constexpr uint32_t NI = uint32_t(F) > KPL ? uint32_t(F) / KPL : 1;
+  constexpr uint32_t LINE = uint32_t(F) * S < 64 ? uint32_t(F) * S : 64;  // bytes of one key line
+  constexpr int LCH = int(LINE / 16);                                      // 16 B chunks in it (1..4)
+  extern __shared__ __align__(16) uint8_t smem[];
+  {
+    const uint32_t words = (rd.count * S + (4u << rd.bits)) / 4;
+    uint32_t* w = reinterpret_cast<uint32_t*>(smem);
+    for (uint32_t i = threadIdx.x; i < words; i += THREADS) w[i] = __ldg(dirbuf + i);
+  }
+  __syncthreads();
+  const K* s_M = reinterpret_cast<const K*>(smem);
+  const uint32_t* s_dir = reinterpret_cast<const uint32_t*>(smem + rd.count * S);
+
+  const int lane = threadIdx.x & 31;
+  const int g = lane / G, k = lane % G;
+  const unsigned gmask = 3u << (g * G);
+  const uint64_t warp = (uint64_t(blockIdx.x) * THREADS + threadIdx.x) >> 5;
+  const uint64_t nwarps = (uint64_t(gridDim.x) * THREADS) >> 5;
+  const uint64_t rounds = (m + ROUND - 1) / ROUND;
+  const uint32_t U = rv.U;
+
+  for (uint64_t r0 = warp; r0 < rounds; r0 += nwarps) {
+    const uint64_t base = r0 * ROUND;
+    K myq[QPL];
+    uint32_t myj[QPL];
+#pragma unroll
+    for (int u = 0; u < QPL; ++u) {
+      const uint64_t i = base + uint64_t(u) * 32 + lane;
+      myq[u] = i < m ? ldcs(queries + i) : key_max<K>();
+      const uint32_t e = s_dir[uint32_t(myq[u] >> (8 * S - rd.bits))];
+      uint32_t lo = e & 0xFFFFu, hi = e >> 16;
+      while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (s_M[mid] < myq[u]) lo = mid + 1; else hi = mid;
+      }
+      myj[u] = lo;
+    }
+    K q[QPG];
+    uint32_t cur[QPG];
+#pragma unroll
+    for (int j = 0; j < QPG; ++j) {
+      const int src = (j * NG) % 32 + g;
+      q[j] = __shfl_sync(0xffffffffu, myq[(j * NG) / 32], src);
+      const uint32_t pj = __shfl_sync(0xffffffffu, myj[(j * NG) / 32], src);
+      cur[j] = rd.T < U ? uint32_t(rd.T_base + pj) : __ldg(chain + pj);
+    }
+    // ---- upper levels T .. U-1 (root-first), then the last level
+    for (uint32_t d = rd.T; d <= U; ++d) {
+      const bool last = d == U;
+      const uint8_t* idxb = last ? rv.lidx : rv.uidx;
+      const uint8_t* keyb = last ? rv.lkeys : rv.ukeys;
+      uint32_t t[QPG];
+      if constexpr (NI > 1) {
+        V16<K> iv[QPG];
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) iv[j] = ld16g<K>(idxb + uint64_t(cur[j]) * 32 + k * 16);
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          uint32_t c = 0;
+#pragma unroll
+          for (uint32_t e = 0; e < E16; ++e) c += __popc(__ballot_sync(0xffffffffu, iv[j].k[e] < q[j]) & gmask);
+          t[j] = c;
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) t[j] = 0;
+      }
+      // one key line: lane k holds 16 B chunks k and k + 2
+      V16<K> kv[QPG][2];
+#pragma unroll
+      for (int j = 0; j < QPG; ++j)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int ch = k + 2 * h;
+          if (ch < LCH) kv[j][h] = ld16g<K>(keyb + (uint64_t(cur[j]) * F + t[j] * KPL) * S + ch * 16);
+          else {
+#pragma unroll
+            for (uint32_t e = 0; e < E16; ++e) kv[j][h].k[e] = key_max<K>();
+          }
+        }
+      uint32_t slot[QPG];
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) {
+        uint32_t c = 0;
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+#pragma unroll
+          for (uint32_t e = 0; e < E16; ++e) c += __popc(__ballot_sync(0xffffffffu, kv[j][h].k[e] < q[j]) & gmask);
+        slot[j] = t[j] * KPL + c;
+      }
+      if (last) {
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) t[j] = slot[j];  // line j of big leaf cur
+        // ---- leaf line (cur*F + line): key sector + value sector, 16 B per lane each
+        V16<K> lk[QPG], lvv[QPG];
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          const uint8_t* p = rv.leaf + (uint64_t(cur[j]) * F + t[j]) * 64 + k * 16;
+          lk[j] = ld16g<K>(p);
+          lvv[j] = ld16g<K>(p + 32);
+        }
+        uint64_t my_pf[QPG / G];
+        K my_v[QPG / G];
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          uint32_t s = 0;
+#pragma unroll
+          for (uint32_t e = 0; e < E16; ++e) s += __popc(__ballot_sync(0xffffffffu, lk[j].k[e] < q[j]) & gmask);
+          const uint32_t sc = s < P ? s : P - 1;
+          const int src = g * G + int(sc / E16);
+          const K key_s = __shfl_sync(0xffffffffu, pick(lk[j].k, sc % E16), src);
+          const K val_s = __shfl_sync(0xffffffffu, pick(lvv[j].k, sc % E16), src);
+          bool end = (s == P);
+          if (!end && key_s == key_max<K>()) {
+            // MAX slot: padding unless it is a counted entry ("must read the node size")
+            const int64_t in_line = int64_t(__ldg(rv.count + cur[j])) - int64_t(t[j]) * P;
+            const int64_t lim = in_line < int64_t(P) ? in_line : int64_t(P);
+            end = int64_t(s) >= lim;
+          }
+          const bool found = !end && key_s == q[j];
+          if (j % G == k) {
+            my_pf[j / G] = end ? kEnd : (((uint64_t(cur[j]) * F + t[j]) * P + s) | (found ? kFound : 0ull));
+            my_v[j / G] = found ? val_s : K(0);
+          }
+        }
+#pragma unroll
+        for (int tt = 0; tt < QPG / G; ++tt) {
+          const uint64_t i = base + uint64_t(k + G * tt) * NG + g;
+          if (i < m) {
+            stcs(out_pf + i, my_pf[tt]);
+            stcs(out_v + i, my_v[tt]);
+          }
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) cur[j] = __ldg(rv.urefs + uint64_t(cur[j]) * F + slot[j]);
+      }
+    }
+  }
+}
+
 constexpr int kThreads = 512;
 constexpr int kQPG = 4;
 
@@ -379,7 +585,7 @@ uint32_t smem_levels_t(const hbt_tree* t, uint32_t budget) {
 }
 
 template <typename K, int F>
-int search_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+int search_v1_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
   const RegularState& r = t->r;
   auto kern = regular_search_kernel<K, F, kQPG, kThreads>;
   RView rv{};
@@ -414,6 +620,57 @@ int search_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, vo
   kern<<<unsigned(grid), kThreads, smem, s>>>(rv, (const K*)q, m, pf, (K*)v);
   HBT_CUDA_TRY(cudaGetLastError());
   return HBT_OK;
+}
+
+template <typename K, int F, int QPL, int THREADS>
+int search_v2_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+  const RegularState& r = t->r;
+  auto kern = regular_search_v2<K, F, QPL, THREADS>;
+  RView rv{};
+  rv.leaf = (const uint8_t*)r.d_leaf;
+  rv.count = r.d_count;
+  rv.lkeys = (const uint8_t*)r.d_lkeys;
+  rv.lidx = (const uint8_t*)r.d_lidx;
+  rv.ukeys = (const uint8_t*)r.d_ukeys;
+  rv.uidx = (const uint8_t*)r.d_uidx;
+  rv.urefs = r.d_urefs;
+  for (uint32_t u = 0; u <= r.U; ++u) rv.uoff[u] = r.uoff[u];
+  rv.U = r.U;
+  RDir rd{};
+  rd.T = r.dir_T;
+  rd.count = r.dir_count;
+  rd.bits = r.dir_bits;
+  rd.T_base = r.dir_T < r.U ? r.uoff[r.U - 1 - r.dir_T] : 0;
+  const size_t smem = r.dir_bytes;
+  static bool attr = false;
+  if (!attr) {
+    HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    attr = true;
+  }
+  int occ = 0;
+  HBT_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, THREADS, smem));
+  if (t->cfg.ctas_per_sm && int(t->cfg.ctas_per_sm) < occ) occ = int(t->cfg.ctas_per_sm);
+  if (occ < 1) occ = 1;
+  const uint64_t rounds = (m + 32 * QPL - 1) / (32 * QPL);
+  uint64_t grid = uint64_t(t->num_sms) * occ;
+  const uint64_t need = (rounds + THREADS / 32 - 1) / (THREADS / 32);
+  if (need < grid) grid = need ? need : 1;
+  kern<<<unsigned(grid), THREADS, smem, s>>>(rv, rd, (const uint32_t*)r.d_dir, r.d_chain, (const K*)q, m, pf, (K*)v);
+  HBT_CUDA_TRY(cudaGetLastError());
+  return HBT_OK;
+}
+
+template <typename K, int F>
+int search_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+  if (t->cfg.mode == 2) {
+    const uint32_t th = t->cfg.threads ? t->cfg.threads : 1024;
+    const uint32_t qpl = t->cfg.qpl ? t->cfg.qpl : 1;
+    if (qpl == 2) return th == 512 ? search_v2_launch<K, F, 2, 512>(t, q, m, pf, v, s)
+                                   : search_v2_launch<K, F, 2, 1024>(t, q, m, pf, v, s);
+    return th == 512 ? search_v2_launch<K, F, 1, 512>(t, q, m, pf, v, s)
+                     : search_v2_launch<K, F, 1, 1024>(t, q, m, pf, v, s);
+  }
+  return search_v1_launch<K, F>(t, q, m, pf, v, s);
 }
 
 template <typename K>
@@ -521,6 +778,42 @@ int rebuild_upper(hbt_tree* t, cudaStream_t s) {
 }
 
 template <typename K>
+int rebuild_dir(hbt_tree* t, cudaStream_t s) {
+  RegularState& r = t->r;
+  const uint32_t F = t->F;
+  // root-first level d: d < U -> upper level U-1-d, d == U -> the last level (big leaves)
+  auto count_at = [&](uint32_t d) -> uint64_t { return d < r.U ? r.unodes[r.U - 1 - d] : r.nchain; };
+  uint32_t T = 0;
+  for (uint32_t d = 0; d <= r.U; ++d)
+    if (count_at(d) * sizeof(K) <= 64 * 1024 && count_at(d) <= 65535) T = d;
+  const uint64_t cnt = count_at(T);
+  uint64_t span = 1;
+  for (uint32_t e = T; e < r.U; ++e) span *= F;
+  uint32_t bits = 1;
+  while ((1ull << bits) < 4 * cnt && bits < 13) ++bits;
+  const uint64_t bytes = cnt * sizeof(K) + (4ull << bits);
+  if (bytes > r.dir_cap) {
+    cudaFree(r.d_dir);
+    r.d_dir = nullptr;
+    r.dir_cap = 0;
+    const uint64_t cap = 64 * 1024 + (4ull << 13);  // the largest M_T (64 KB) + directory (32 KB)
+    HBT_CUDA_TRY(cudaMalloc(&r.d_dir, cap));
+    r.dir_cap = cap;
+  }
+  r.dir_T = T;
+  r.dir_count = uint32_t(cnt);
+  r.dir_bits = bits;
+  r.dir_bytes = bytes;
+  K* M = (K*)r.d_dir;
+  uint32_t* dir = (uint32_t*)((uint8_t*)r.d_dir + cnt * sizeof(K));
+  reg_dir_max<K><<<grid_for(cnt), 256, 0, s>>>((const K*)r.d_leaf, r.d_count, r.d_chain, r.nchain, F, cnt, span, M);
+  reg_dir_table<K><<<grid_for(1ull << bits), 256, 0, s>>>(M, uint32_t(cnt), bits, dir);
+  HBT_CUDA_TRY(cudaGetLastError());
+  HBT_CUDA_TRY(cudaStreamSynchronize(s));
+  return HBT_OK;
+}
+
+template <typename K>
 int build_t(hbt_tree* t, const void* keys, const void* values, uint64_t n, cudaStream_t s) {
   RegularState& r = t->r;
   const uint32_t F = t->F;
@@ -548,7 +841,8 @@ int build_t(hbt_tree* t, const void* keys, const void* values, uint64_t n, cudaS
   cudaFree(kd);
   cudaFree(vd);
   if (e != cudaSuccess) { set_error("regular build: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
-  return rebuild_upper<K>(t, s);
+  int rc2 = rebuild_upper<K>(t, s);
+  return rc2 != HBT_OK ? rc2 : rebuild_dir<K>(t, s);
 }
 
 // ---------------------------------------------------------------- update kernels
@@ -970,6 +1264,8 @@ int update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   HBT_CUDA_TRY(cudaStreamSynchronize(s));
   rc = rebuild_upper<K>(t, s);
   if (rc != HBT_OK) return rc;
+  rc = rebuild_dir<K>(t, s);
+  if (rc != HBT_OK) return rc;
   // live key count n' = sum of the chain's counts
   {
     DevBuf sum;
@@ -1019,7 +1315,7 @@ int regular_update(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
 void regular_free(hbt_tree* t) {
   RegularState& r = t->r;
   cudaFree(r.d_leaf); cudaFree(r.d_count); cudaFree(r.d_lkeys); cudaFree(r.d_lidx); cudaFree(r.d_chain);
-  cudaFree(r.d_ukeys); cudaFree(r.d_uidx); cudaFree(r.d_urefs); cudaFree(r.d_seg_of_leaf);
+  cudaFree(r.d_ukeys); cudaFree(r.d_uidx); cudaFree(r.d_urefs); cudaFree(r.d_seg_of_leaf); cudaFree(r.d_dir);
   r = RegularState{};
 }
 

@@ -59,10 +59,12 @@ def test_regular_edge_suite_parity(hbt, width, F):
         t = gpu_build(hbt, k, v, F, width, layout="regular")
         check_arrays(hbt, t, o, width)
         q = query_set(k, width, rng, 3000)
-        pf, val = gpu_search(t, q, width)
         epf, ev = o.search(q)
-        assert np.array_equal(pf, epf), (n, F, width, np.nonzero(pf != epf)[0][:5])
-        assert np.array_equal(val, ev), (n, F, width)
+        for mode, th, qpl in ((2, 0, 0), (0, 0, 0), (2, 512, 2)):  # directory v2 / staged v1 / shapes
+            t.set_search_config(smem_mode=mode, threads_per_cta=th, queries_per_lane=qpl)
+            pf, val = gpu_search(t, q, width)
+            assert np.array_equal(pf, epf), (mode, n, F, width, np.nonzero(pf != epf)[0][:5])
+            assert np.array_equal(val, ev), (mode, n, F, width)
         t.close()
 
 
@@ -99,10 +101,12 @@ def test_regular_update_parity(hbt, width, F):
                     live.discard(a_)
             check_arrays(hbt, t, o, width)
             q = query_set(ok[:300], width, rng, 3000)
-            pf, val = gpu_search(t, q, width)
             epf, ev = o.search(q)
-            assert np.array_equal(pf, epf), (trial, batch)
-            assert np.array_equal(val, ev), (trial, batch)
+            for mode in (2, 0):
+                t.set_search_config(smem_mode=mode)
+                pf, val = gpu_search(t, q, width)
+                assert np.array_equal(pf, epf), (mode, trial, batch)
+                assert np.array_equal(val, ev), (mode, trial, batch)
         assert t.info()["n_distinct"] == 0
 
 
