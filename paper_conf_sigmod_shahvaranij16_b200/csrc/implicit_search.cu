@@ -144,6 +144,17 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
   const uint64_t nwarps = (uint64_t(gridDim.x) * THREADS) >> 5;
   const uint64_t rounds = (m + ROUND - 1) / ROUND;
 
+  // MODE 2 pipelines the query stream across rounds: the next round's queries
+  // are loaded while this round walks the tree (their HBM latency was the
+  // largest single stall, profiles/r01_c2_v11_*).
+  K nextq[QPL];
+  if constexpr (MODE == 2) {
+#pragma unroll
+    for (int u = 0; u < QPL; ++u) {
+      const uint64_t i = warp * ROUND + uint64_t(u) * 32 + lane;
+      nextq[u] = (warp < rounds && i < m) ? ldcs(queries + i) : key_max<K>();
+    }
+  }
   for (uint64_t rd = warp; rd < rounds; rd += nwarps) {
     const uint64_t base = rd * ROUND;
     // ---- phase 1: one lane per query; coalesced query loads
@@ -151,8 +162,14 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
     uint32_t mynode[QPL];
 #pragma unroll
     for (int u = 0; u < QPL; ++u) {
-      const uint64_t i = base + uint64_t(u) * 32 + lane;
-      myq[u] = i < m ? ldcs(queries + i) : key_max<K>();
+      if constexpr (MODE == 2) {
+        myq[u] = nextq[u];
+        const uint64_t i = (rd + nwarps) * ROUND + uint64_t(u) * 32 + lane;
+        nextq[u] = (rd + nwarps < rounds && i < m) ? ldcs(queries + i) : key_max<K>();
+      } else {
+        const uint64_t i = base + uint64_t(u) * 32 + lane;
+        myq[u] = i < m ? ldcs(queries + i) : key_max<K>();
+      }
       mynode[u] = 0;
     }
     if constexpr (MODE == 2) {
