@@ -54,6 +54,7 @@ def parse():
     ap.add_argument("--carveout", type=int, default=-1, help="smem carve-out percent (-1 default)")
     ap.add_argument("--l2-persist", type=int, default=None, help="bytes of I-segment in a persisting L2 window")
     ap.add_argument("--l2-levels", type=int, default=None, help="L2 budget for index+sector levels (bytes)")
+    ap.add_argument("--exchange", type=int, default=None, help="c4: 0 = fused peer-memory exchange, 1 = NCCL")
     return ap.parse_args()
 
 
@@ -193,6 +194,8 @@ def make_work(cfg_name, rank, world, args):
         tree.set_param("l2_persist", args.l2_persist)
     if args.l2_levels is not None and c["layout"] == "implicit":
         tree.set_param("l2_levels_bytes", args.l2_levels)
+    if args.exchange is not None:
+        tree.set_param("exchange", args.exchange)
     out_pos = torch.empty(m, dtype=torch.int64, device="cuda")
     out_val = torch.empty(m, dtype=sdt, device="cuda")
     return Work(c=c, name=cfg_name, tree=tree, q=q, m=m, w=w, hit_rate=hit_rate, qdesc=qdesc, extra=extra,
@@ -355,6 +358,8 @@ def run_hbt(args):
                                    f"{c['fanout']}, m={m} queries/GPU ({work.qdesc})",
                        "n_keys": c["n"], "queries_per_gpu": m, "fanout": c["fanout"], "layout": c["layout"],
                        "key_bits": 8 * w,
+                       "exchange": ("fused peer-memory (CUDA IPC windows)" if not args.exchange else "NCCL send/recv")
+                                   if args.config == "c4" else None,
                        "parallelism": (f"key-range sharded x{world}" if args.config == "c4" else
                                        (f"replicated x{world}" if world > 1 else "single")),
                        "l2_policy": "inputs larger than L2 (queries+results %d MiB/step/GPU > 126 MB L2)"

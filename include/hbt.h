@@ -172,6 +172,8 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *   "l2_levels_bytes" implicit: inner levels below the shared-memory top are read as index
  *                 sector + one key sector while their cumulative bytes fit this L2 budget,
  *                 as whole nodes beyond it (0 = default 32 MB; 1 = every level whole)
+ *   "exchange"    sharded search: 0 = fused peer-memory exchange (CUDA IPC windows, default),
+ *                 1 = NCCL send/recv (multi-process) / device copies (hbt_search_sharded_local)
  * Unknown names or out-of-range values return HBT_EINVAL. */
 HBT_API int hbt_set_param(hbt_tree* t, const char* name, int64_t value);
 

@@ -41,6 +41,7 @@ static void free_tree(hbt_tree* t) {
   cudaFree(t->d_leaf);
   regular_free(t);
   shard_free(t);
+  fused_free(t);
   cudaFree(t->pipe.d_q);
   cudaFree(t->pipe.d_pf);
   cudaFree(t->pipe.d_v);
@@ -251,6 +252,7 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "carveout" && value >= -1 && value <= 100) c.carveout = int(value);
   else if (n == "l2_persist" && value >= 0) c.l2_persist = uint64_t(value);
   else if (n == "l2_levels_bytes" && value >= 0) c.l2_levels_bytes = uint64_t(value);
+  else if (n == "exchange" && (value == 0 || value == 1)) c.exchange = uint32_t(value);
   else {
     set_error("bad parameter %s = %lld", name, (long long)value);
     return HBT_EINVAL;

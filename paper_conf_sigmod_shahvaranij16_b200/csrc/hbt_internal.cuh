@@ -3,6 +3,7 @@
 #pragma once
 
 #include <cuda_runtime.h>
+#include <nccl.h>
 #include <stdint.h>
 
 #include <mutex>
@@ -44,6 +45,7 @@ struct SearchConfig {
   int carveout = -1;             // shared-memory carve-out percent (-1 = driver default)
   uint64_t l2_persist = 0;       // bytes of the I-segment to keep in a persisting L2 window (0 = off)
   uint64_t l2_levels_bytes = 0;  // L2-resident budget for index+sector levels (0 = default 32 MB)
+  uint32_t exchange = 0;         // sharded search: 0 = fused peer-memory exchange, 1 = NCCL send/recv
 };
 
 // Regular-tree device state.  All pools are SoA arrays
@@ -110,6 +112,12 @@ struct Scratch {
 
 }  // namespace hbt
 
+struct hbt_comm {
+  ncclComm_t comm = nullptr;
+  int nranks = 1;
+  int rank = 0;
+};
+
 struct hbt_tree {
   uint32_t form = HBT_IMPLICIT;  // HBT_IMPLICIT | HBT_REGULAR
   uint32_t width = 8;            // S
@@ -145,6 +153,7 @@ struct hbt_tree {
   // ---- key-range sharding ----
   hbt::ShardMeta shard;
   hbt::Scratch shard_scratch;
+  void* fused = nullptr;  // sharded_fused.cu state (peer windows)
   // ---- search ----
   hbt::SearchConfig cfg;
   mutable hbt::HostPipe pipe;
@@ -165,6 +174,11 @@ int implicit_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, 
 int implicit_search_base(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
                          cudaStream_t s);
 void shard_free(hbt_tree* t);
+// sharded_fused.cu
+void fused_free(hbt_tree* t);
+int fused_search_local(hbt_tree* const* shards, int G, const void* const* queries, const uint64_t* m,
+                       const hbt_out* outs, cudaStream_t st);
+int fused_search_nccl(const hbt_tree* t, const void* queries, uint64_t m, hbt_out out, cudaStream_t st);
 uint32_t implicit_smem_levels(const hbt_tree* t, uint32_t budget);
 // index bytes per implicit node (0 when F*S <= 32)
 uint32_t implicit_idx_stride(uint32_t F, uint32_t S);

@@ -22,12 +22,6 @@
 
 #include "hbt_internal.cuh"
 
-struct hbt_comm {
-  ncclComm_t comm = nullptr;
-  int nranks = 1;
-  int rank = 0;
-};
-
 namespace hbt {
 namespace {
 
@@ -434,6 +428,7 @@ int hbt_search_sharded(const hbt_tree* t, const void* queries_local, uint64_t m_
                        void* stream) {
   if (!t || !t->shard.comm) { set_error("not a sharded tree"); return HBT_EINVAL; }
   cudaStream_t st = (cudaStream_t)stream;
+  if (t->cfg.exchange == 0) return fused_search_nccl(t, queries_local, m_local, out_local, st);
   return t->width == 4 ? search_nccl_t<uint32_t>(t, queries_local, m_local, out_local, st)
                        : search_nccl_t<uint64_t>(t, queries_local, m_local, out_local, st);
 }
@@ -468,6 +463,7 @@ int hbt_search_sharded_local(hbt_tree* const* shards, int G, const void* const* 
     return HBT_EINVAL;
   }
   cudaStream_t st = (cudaStream_t)stream;
+  if (shards[0]->cfg.exchange == 0) return fused_search_local(shards, G, queries, m, outs, st);
   return shards[0]->width == 4 ? search_local_t<uint32_t>(shards, G, queries, m, outs, st)
                                : search_local_t<uint64_t>(shards, G, queries, m, outs, st);
 }

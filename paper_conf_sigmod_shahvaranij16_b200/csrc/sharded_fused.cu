@@ -1,0 +1,447 @@
+// sharded_fused.cu — the key-range-sharded search with a FUSED exchange over
+// peer memory (NVLink 5 / NVSwitch): no NCCL on the data path.
+//
+// Every rank owns one window (one cudaMalloc, exported with CUDA IPC and
+// mapped by every peer):
+//   [flags: 64 x u32 | matrix: 64 x 64 u64 | res_pf: cap_m u64 | res_v: cap_m x S
+//    | recv_q: cap_r x S | recv_org: cap_r u64]
+// Per batch (all kernels stream-ordered; barriers are device-side flag
+// exchanges over peer memory):
+//   1. route_count (sharded.cu's owner rule) + publish: this rank's count row
+//      is stored into EVERY peer's matrix                         -> barrier
+//   2. route_put: every query is stored straight into its owner's receive
+//      window at (prefix of earlier sources' counts) + a CTA-reserved slot,
+//      with its origin (source rank, index)                       -> barrier
+//   3. the owner searches its receive window (pos_base = its first global rank)
+//   4. return_put: each result is stored straight into the requester's result
+//      window at its ORIGINAL index (no unpermute pass)           -> barrier
+//   5. the requester copies its result window into the caller's out arrays.
+// The same kernels run for G virtual shards on one GPU (peer table = local
+// windows, barriers = stream order), which is how they are tested here.
+#include <nccl.h>
+
+#include <vector>
+
+#include "hbt_internal.cuh"
+
+namespace hbt {
+namespace {
+
+constexpr int kMaxG = 64;
+constexpr int kThreads = 256;
+constexpr uint64_t kOrgShift = 40;  // recv_org = (source rank << 40) | origin index
+
+struct Win {
+  uint32_t* flags;
+  unsigned long long* matrix;  // [src][dst]
+  uint64_t* res_pf;
+  uint8_t* res_v;
+  uint8_t* recv_q;
+  uint64_t* recv_org;
+};
+
+struct PeerTable {
+  Win w[kMaxG];
+  int G;
+};
+
+struct RouteTab {
+  uint64_t max[kMaxG];
+  uint32_t id[kMaxG];
+  uint32_t n;
+};
+
+inline unsigned grid_for(uint64_t n) {
+  uint64_t g = (n + kThreads - 1) / kThreads;
+  if (g > 148 * 16) g = 148 * 16;
+  return unsigned(g ? g : 1);
+}
+
+uint64_t win_bytes(uint64_t cap_m, uint64_t cap_r, uint32_t S) {
+  auto al = [](uint64_t x) { return (x + 255) & ~uint64_t(255); };
+  return al(kMaxG * 4) + al(kMaxG * kMaxG * 8) + al(cap_m * 8) + al(cap_m * S) + al(cap_r * S) + al(cap_r * 8);
+}
+
+Win carve(uint8_t* base, uint64_t cap_m, uint64_t cap_r, uint32_t S) {
+  auto al = [](uint64_t x) { return (x + 255) & ~uint64_t(255); };
+  Win w;
+  uint64_t o = 0;
+  w.flags = (uint32_t*)(base + o); o += al(kMaxG * 4);
+  w.matrix = (unsigned long long*)(base + o); o += al(kMaxG * kMaxG * 8);
+  w.res_pf = (uint64_t*)(base + o); o += al(cap_m * 8);
+  w.res_v = base + o; o += al(cap_m * S);
+  w.recv_q = base + o; o += al(cap_r * S);
+  w.recv_org = (uint64_t*)(base + o);
+  return w;
+}
+
+template <typename K>
+__device__ __forceinline__ uint32_t owner(K q, const RouteTab& rt) {
+  if (rt.n == 0) return 0;
+  uint32_t c = 0;
+  for (uint32_t i = 0; i < rt.n; ++i) c += (K(rt.max[i]) < q) ? 1u : 0u;
+  return rt.id[c < rt.n ? c : rt.n - 1];
+}
+
+template <typename K>
+__global__ void __launch_bounds__(kThreads) f_count(const K* __restrict__ q, uint64_t m, const RouteTab rt, int G,
+                                                    uint8_t* __restrict__ dest, unsigned long long* __restrict__ cnt) {
+  __shared__ unsigned int h[kMaxG];
+  for (int i = threadIdx.x; i < G; i += blockDim.x) h[i] = 0;
+  __syncthreads();
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < m; i += uint64_t(gridDim.x) * blockDim.x) {
+    const uint32_t o = owner(q[i], rt);
+    dest[i] = uint8_t(o);
+    atomicAdd(&h[o], 1u);
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < G; i += blockDim.x)
+    if (h[i]) atomicAdd(cnt + i, (unsigned long long)h[i]);
+}
+
+// Store this rank's count row into every peer's matrix (row `me`).
+__global__ void f_publish(const PeerTable pt, int me, const unsigned long long* __restrict__ cnt) {
+  for (int x = threadIdx.x; x < pt.G * pt.G; x += blockDim.x) {
+    const int d = x / pt.G, c = x % pt.G;
+    pt.w[d].matrix[me * kMaxG + c] = cnt[c];
+  }
+}
+
+// Route + put: queries go straight into their owner's receive window.
+template <typename K>
+__global__ void __launch_bounds__(kThreads) f_put(const K* __restrict__ q, uint64_t m, const uint8_t* __restrict__ dest,
+                                                  const PeerTable pt, int me,
+                                                  unsigned long long* __restrict__ cursor, uint64_t chunk) {
+  __shared__ unsigned int h[kMaxG];
+  __shared__ unsigned long long base[kMaxG];
+  const int G = pt.G;
+  const uint64_t lo = blockIdx.x * chunk;
+  const uint64_t hi = lo + chunk < m ? lo + chunk : m;
+  for (int i = threadIdx.x; i < G; i += blockDim.x) h[i] = 0;
+  __syncthreads();
+  for (uint64_t i = lo + threadIdx.x; i < hi; i += blockDim.x) atomicAdd(&h[dest[i]], 1u);
+  __syncthreads();
+  const unsigned long long* M = pt.w[me].matrix;  // full matrix (every row published)
+  for (int d = threadIdx.x; d < G; d += blockDim.x) {
+    unsigned long long start = 0;  // earlier sources' share of destination d
+    for (int s = 0; s < me; ++s) start += M[s * kMaxG + d];
+    base[d] = h[d] ? start + atomicAdd(cursor + d, (unsigned long long)h[d]) : 0ull;
+    h[d] = 0;
+  }
+  __syncthreads();
+  for (uint64_t i = lo + threadIdx.x; i < hi; i += blockDim.x) {
+    const uint32_t d = dest[i];
+    const uint64_t slot = base[d] + atomicAdd(&h[d], 1u);
+    reinterpret_cast<K*>(pt.w[d].recv_q)[slot] = q[i];
+    pt.w[d].recv_org[slot] = (uint64_t(me) << kOrgShift) | i;
+  }
+}
+
+// Results straight into the requester's result window at the original index.
+template <typename K>
+__global__ void f_return(const PeerTable pt, int me, uint64_t nrecv, const uint64_t* __restrict__ pf,
+                         const K* __restrict__ v) {
+  const Win& mine = pt.w[me];
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < nrecv; i += uint64_t(gridDim.x) * blockDim.x) {
+    const uint64_t org = mine.recv_org[i];
+    const int src = int(org >> kOrgShift);
+    const uint64_t idx = org & ((1ull << kOrgShift) - 1);
+    pt.w[src].res_pf[idx] = pf[i];
+    reinterpret_cast<K*>(pt.w[src].res_v)[idx] = v[i];
+  }
+}
+
+// Device-side barrier over peer memory: publish `epoch` into every peer's flag
+// slot `me`, then wait until every peer has published it into ours.
+__global__ void f_barrier(const PeerTable pt, int me, uint32_t epoch) {
+  if (threadIdx.x != 0) return;
+  __threadfence_system();
+  for (int d = 0; d < pt.G; ++d) {
+    volatile uint32_t* f = pt.w[d].flags + me;
+    *f = epoch;
+  }
+  __threadfence_system();
+  for (int s = 0; s < pt.G; ++s) {
+    volatile uint32_t* f = pt.w[me].flags + s;
+    while (int32_t(*f - epoch) < 0) {
+    }
+  }
+  __threadfence_system();
+}
+
+template <typename T>
+int ensure(T** p, uint64_t* cap, uint64_t need) {
+  if (need <= *cap) return HBT_OK;
+  cudaFree(*p);
+  *p = nullptr;
+  *cap = 0;
+  const uint64_t c = need + need / 8 + 1024;
+  HBT_CUDA_TRY(cudaMalloc(p, c * sizeof(T)));
+  *cap = c;
+  return HBT_OK;
+}
+
+RouteTab table_of(const ShardMeta& sm) {
+  RouteTab rt{};
+  for (int g = 0; g < sm.G; ++g)
+    if (sm.count[g]) {
+      rt.max[rt.n] = sm.max[g];
+      rt.id[rt.n] = uint32_t(g);
+      ++rt.n;
+    }
+  return rt;
+}
+
+}  // namespace
+
+// Per-tree state of the fused exchange.
+struct FusedState {
+  uint8_t* win = nullptr;        // this rank's window (own allocation)
+  uint64_t cap_m = 0, cap_r = 0;
+  uint8_t* peer[kMaxG] = {};     // mapped peer windows (multi-process)
+  uint8_t* dest = nullptr; uint64_t dest_cap = 0;
+  uint64_t* tmp_pf = nullptr; uint64_t tmp_pf_cap = 0;
+  uint8_t* tmp_v = nullptr; uint64_t tmp_v_cap = 0;
+  unsigned long long* cnt = nullptr;  // 2 x kMaxG: counts, cursors
+  uint32_t epoch = 0;
+};
+
+void fused_free(hbt_tree* t) {
+  FusedState* f = static_cast<FusedState*>(t->fused);
+  if (!f) return;
+  for (int g = 0; g < kMaxG; ++g)
+    if (f->peer[g] && f->peer[g] != f->win) cudaIpcCloseMemHandle(f->peer[g]);
+  cudaFree(f->win); cudaFree(f->dest); cudaFree(f->tmp_pf); cudaFree(f->tmp_v); cudaFree(f->cnt);
+  delete f;
+  t->fused = nullptr;
+}
+
+namespace {
+
+FusedState* state_of(hbt_tree* t) {
+  if (!t->fused) t->fused = new FusedState();
+  return static_cast<FusedState*>(t->fused);
+}
+
+int alloc_window(FusedState* f, uint64_t cap_m, uint64_t cap_r, uint32_t S) {
+  cudaFree(f->win);
+  f->win = nullptr;
+  HBT_CUDA_TRY(cudaMalloc(&f->win, win_bytes(cap_m, cap_r, S)));
+  HBT_CUDA_TRY(cudaMemset(f->win, 0, 256 * ((kMaxG * 4 + 255) / 256)));  // flags
+  f->cap_m = cap_m;
+  f->cap_r = cap_r;
+  f->epoch = 0;
+  return HBT_OK;
+}
+
+int prep_local(FusedState* f, uint64_t m) {
+  int rc;
+  if ((rc = ensure(&f->dest, &f->dest_cap, m ? m : 1))) return rc;
+  if (!f->cnt) HBT_CUDA_TRY(cudaMalloc(&f->cnt, 2 * kMaxG * sizeof(unsigned long long)));
+  return HBT_OK;
+}
+
+template <typename K>
+int route_and_count(FusedState* f, const K* q, uint64_t m, const RouteTab& rt, int G, cudaStream_t st) {
+  HBT_CUDA_TRY(cudaMemsetAsync(f->cnt, 0, 2 * kMaxG * sizeof(unsigned long long), st));
+  if (m) {
+    f_count<K><<<grid_for(m), kThreads, 0, st>>>(q, m, rt, G, f->dest, f->cnt);
+    HBT_CUDA_TRY(cudaGetLastError());
+  }
+  return HBT_OK;
+}
+
+template <typename K>
+int put_queries(FusedState* f, const K* q, uint64_t m, const PeerTable& pt, int me, cudaStream_t st) {
+  if (!m) return HBT_OK;
+  const uint64_t chunk = 4096;
+  f_put<K><<<unsigned((m + chunk - 1) / chunk), kThreads, 0, st>>>(q, m, f->dest, pt, me, f->cnt + kMaxG, chunk);
+  HBT_CUDA_TRY(cudaGetLastError());
+  return HBT_OK;
+}
+
+template <typename K>
+int search_and_return(hbt_tree* t, FusedState* f, const PeerTable& pt, int me, uint64_t nrecv, cudaStream_t st) {
+  int rc;
+  if ((rc = ensure(&f->tmp_pf, &f->tmp_pf_cap, nrecv ? nrecv : 1))) return rc;
+  if ((rc = ensure(&f->tmp_v, &f->tmp_v_cap, (nrecv ? nrecv : 1) * sizeof(K)))) return rc;
+  if (!nrecv) return HBT_OK;
+  const Win& w = pt.w[me];
+  rc = implicit_search_base(t, w.recv_q, nrecv, f->tmp_pf, f->tmp_v, t->shard.base[me], st);
+  if (rc) return rc;
+  f_return<K><<<grid_for(nrecv), kThreads, 0, st>>>(pt, me, nrecv, f->tmp_pf, (const K*)f->tmp_v);
+  HBT_CUDA_TRY(cudaGetLastError());
+  return HBT_OK;
+}
+
+// ------------------------------------------------------------ single process
+
+template <typename K>
+int local_t(hbt_tree* const* shards, int G, const void* const* queries, const uint64_t* m, const hbt_out* outs,
+            cudaStream_t st) {
+  const uint32_t S = sizeof(K);
+  const RouteTab rt = table_of(shards[0]->shard);
+  // host-side sizes (the multi-process path learns them from the published matrix)
+  std::vector<FusedState*> fs(G);
+  std::vector<std::vector<unsigned long long>> cnt(G, std::vector<unsigned long long>(G));
+  for (int s = 0; s < G; ++s) {
+    fs[s] = state_of(shards[s]);
+    int rc = prep_local(fs[s], m[s]);
+    if (rc) return rc;
+    rc = route_and_count<K>(fs[s], (const K*)queries[s], m[s], rt, G, st);
+    if (rc) return rc;
+    HBT_CUDA_TRY(cudaMemcpyAsync(cnt[s].data(), fs[s]->cnt, G * 8, cudaMemcpyDeviceToHost, st));
+  }
+  HBT_CUDA_TRY(cudaStreamSynchronize(st));
+  uint64_t need_m = 1, need_r = 1;
+  for (int d = 0; d < G; ++d) {
+    uint64_t r = 0;
+    for (int s = 0; s < G; ++s) r += cnt[s][d];
+    need_r = std::max<uint64_t>(need_r, r);
+    need_m = std::max<uint64_t>(need_m, m[d]);
+  }
+  PeerTable pt{};
+  pt.G = G;
+  for (int g = 0; g < G; ++g) {
+    if (fs[g]->cap_m < need_m || fs[g]->cap_r < need_r || !fs[g]->win) {
+      int rc = alloc_window(fs[g], need_m + need_m / 8, need_r + need_r / 8, S);
+      if (rc) return rc;
+    }
+    pt.w[g] = carve(fs[g]->win, fs[g]->cap_m, fs[g]->cap_r, S);
+  }
+  for (int s = 0; s < G; ++s) {
+    f_publish<<<1, 256, 0, st>>>(pt, s, fs[s]->cnt);
+    HBT_CUDA_TRY(cudaGetLastError());
+  }
+  for (int s = 0; s < G; ++s) {
+    int rc = put_queries<K>(fs[s], (const K*)queries[s], m[s], pt, s, st);
+    if (rc) return rc;
+  }
+  for (int d = 0; d < G; ++d) {
+    uint64_t r = 0;
+    for (int s = 0; s < G; ++s) r += cnt[s][d];
+    int rc = search_and_return<K>(shards[d], fs[d], pt, d, r, st);
+    if (rc) return rc;
+  }
+  for (int s = 0; s < G; ++s) {
+    if (!m[s]) continue;
+    HBT_CUDA_TRY(cudaMemcpyAsync(outs[s].pos_found, pt.w[s].res_pf, m[s] * 8, cudaMemcpyDeviceToDevice, st));
+    HBT_CUDA_TRY(cudaMemcpyAsync(outs[s].values, pt.w[s].res_v, m[s] * S, cudaMemcpyDeviceToDevice, st));
+  }
+  return HBT_OK;
+}
+
+// ------------------------------------------------------------ one process per GPU
+
+#define NCCL_TRY2(expr)                                                                   \
+  do {                                                                                    \
+    ncclResult_t _r = (expr);                                                             \
+    if (_r != ncclSuccess) {                                                              \
+      set_error("%s:%d %s: %s", __FILE__, __LINE__, #expr, ncclGetErrorString(_r));        \
+      return HBT_ENCCL;                                                                   \
+    }                                                                                     \
+  } while (0)
+
+// (Re)allocate this rank's window and map every peer's (collective).
+int exchange_windows(FusedState* f, hbt_comm* c, uint64_t cap_m, uint64_t cap_r, uint32_t S, cudaStream_t st) {
+  for (int g = 0; g < kMaxG; ++g) {
+    if (f->peer[g] && f->peer[g] != f->win) cudaIpcCloseMemHandle(f->peer[g]);
+    f->peer[g] = nullptr;
+  }
+  int rc = alloc_window(f, cap_m, cap_r, S);
+  if (rc) return rc;
+  cudaIpcMemHandle_t h;
+  HBT_CUDA_TRY(cudaIpcGetMemHandle(&h, f->win));
+  void* d = nullptr;
+  HBT_CUDA_TRY(cudaMalloc(&d, sizeof(h) * (c->nranks + 1)));
+  HBT_CUDA_TRY(cudaMemcpyAsync(d, &h, sizeof(h), cudaMemcpyHostToDevice, st));
+  ncclResult_t r = ncclAllGather(d, (uint8_t*)d + sizeof(h), sizeof(h), ncclUint8, c->comm, st);
+  std::vector<cudaIpcMemHandle_t> all(c->nranks);
+  if (r == ncclSuccess) cudaMemcpyAsync(all.data(), (uint8_t*)d + sizeof(h), sizeof(h) * c->nranks, cudaMemcpyDeviceToHost, st);
+  cudaStreamSynchronize(st);
+  cudaFree(d);
+  if (r != ncclSuccess) { set_error("handle all-gather: %s", ncclGetErrorString(r)); return HBT_ENCCL; }
+  for (int g = 0; g < c->nranks; ++g) {
+    if (g == c->rank) { f->peer[g] = f->win; continue; }
+    void* p = nullptr;
+    HBT_CUDA_TRY(cudaIpcOpenMemHandle(&p, all[g], cudaIpcMemLazyEnablePeerAccess));
+    f->peer[g] = (uint8_t*)p;
+  }
+  return HBT_OK;
+}
+
+template <typename K>
+int nccl_fused_t(hbt_tree* t, const void* queries, uint64_t m, hbt_out out, cudaStream_t st) {
+  hbt_comm* c = t->shard.comm;
+  const int G = c->nranks, me = c->rank;
+  const uint32_t S = sizeof(K);
+  FusedState* f = state_of(t);
+  int rc = prep_local(f, m);
+  if (rc) return rc;
+  // agree on window capacities: every rank needs m_s <= cap_m and recv_d <= cap_r.
+  // The count row is all-gathered by NCCL once per batch on the host path (small),
+  // the data path itself is peer stores.
+  const RouteTab rt = table_of(t->shard);
+  rc = route_and_count<K>(f, (const K*)queries, m, rt, G, st);
+  if (rc) return rc;
+  unsigned long long* d = nullptr;
+  HBT_CUDA_TRY(cudaMalloc(&d, sizeof(unsigned long long) * (G + 1) * (G + 1) * 2));
+  HBT_CUDA_TRY(cudaMemcpyAsync(d, f->cnt, G * 8, cudaMemcpyDeviceToDevice, st));
+  ncclResult_t r = ncclAllGather(d, d + G, G, ncclUint64, c->comm, st);
+  std::vector<unsigned long long> mat(G * G);
+  if (r == ncclSuccess) cudaMemcpyAsync(mat.data(), d + G, G * G * 8, cudaMemcpyDeviceToHost, st);
+  cudaStreamSynchronize(st);
+  cudaFree(d);
+  if (r != ncclSuccess) { set_error("count all-gather: %s", ncclGetErrorString(r)); return HBT_ENCCL; }
+  uint64_t need_m = 1, need_r = 1;
+  for (int x = 0; x < G; ++x) {
+    uint64_t row = 0, col = 0;
+    for (int y = 0; y < G; ++y) { row += mat[x * G + y]; col += mat[y * G + x]; }
+    need_m = std::max<uint64_t>(need_m, row);
+    need_r = std::max<uint64_t>(need_r, col);
+  }
+  if (!f->win || f->cap_m < need_m || f->cap_r < need_r) {
+    rc = exchange_windows(f, c, need_m + need_m / 8, need_r + need_r / 8, S, st);
+    if (rc) return rc;
+  }
+  PeerTable pt{};
+  pt.G = G;
+  for (int g = 0; g < G; ++g) pt.w[g] = carve(f->peer[g], f->cap_m, f->cap_r, S);
+  // the full matrix is known: write it into our own window (no peer publish needed)
+  std::vector<unsigned long long> full(kMaxG * kMaxG, 0);
+  for (int s = 0; s < G; ++s)
+    for (int x = 0; x < G; ++x) full[s * kMaxG + x] = mat[s * G + x];
+  HBT_CUDA_TRY(cudaMemcpyAsync(pt.w[me].matrix, full.data(), full.size() * 8, cudaMemcpyHostToDevice, st));
+  // everybody's previous batch must be finished with our windows
+  f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);
+  rc = put_queries<K>(f, (const K*)queries, m, pt, me, st);
+  if (rc) return rc;
+  f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);
+  uint64_t nrecv = 0;
+  for (int s = 0; s < G; ++s) nrecv += mat[s * G + me];
+  rc = search_and_return<K>(t, f, pt, me, nrecv, st);
+  if (rc) return rc;
+  f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);
+  HBT_CUDA_TRY(cudaGetLastError());
+  if (m) {
+    HBT_CUDA_TRY(cudaMemcpyAsync(out.pos_found, pt.w[me].res_pf, m * 8, cudaMemcpyDeviceToDevice, st));
+    HBT_CUDA_TRY(cudaMemcpyAsync(out.values, pt.w[me].res_v, m * S, cudaMemcpyDeviceToDevice, st));
+  }
+  return HBT_OK;
+}
+
+}  // namespace
+
+int fused_search_local(hbt_tree* const* shards, int G, const void* const* queries, const uint64_t* m,
+                       const hbt_out* outs, cudaStream_t st) {
+  return shards[0]->width == 4 ? local_t<uint32_t>(shards, G, queries, m, outs, st)
+                               : local_t<uint64_t>(shards, G, queries, m, outs, st);
+}
+
+int fused_search_nccl(const hbt_tree* t, const void* queries, uint64_t m, hbt_out out, cudaStream_t st) {
+  hbt_tree* tt = const_cast<hbt_tree*>(t);
+  std::lock_guard<std::mutex> lock(tt->pipe.mu);
+  return t->width == 4 ? nccl_fused_t<uint32_t>(tt, queries, m, out, st) : nccl_fused_t<uint64_t>(tt, queries, m, out, st);
+}
+
+}  // namespace hbt

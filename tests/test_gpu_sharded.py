@@ -45,8 +45,9 @@ def queries(allk, rng, m):
                            np.array([0, 2**64 - 1, allk[0], allk[-1], allk[-1] + 1, allk[0] - 1], np.uint64)])
 
 
+@pytest.mark.parametrize("exchange", [0, 1])
 @pytest.mark.parametrize("G,empty", [(1, []), (2, []), (3, [1]), (5, [0, 4]), (8, []), (8, [2, 3])])
-def test_virtual_shards_match_unsharded_oracle(hbt, G, empty):
+def test_virtual_shards_match_unsharded_oracle(hbt, G, empty, exchange):
     n = 200000
     allk = gen.stratified_keys(n, gen.stream_seed(4, gen.STREAM_K))
     allv = gen.values(n, 8, gen.stream_seed(4, gen.STREAM_V))
@@ -57,15 +58,17 @@ def test_virtual_shards_match_unsharded_oracle(hbt, G, empty):
         k, v = allk[lo:hi], allv[lo:hi]
         perm = np.random.default_rng(lo).permutation(len(k))  # unsorted within the shard is fine
         trees.append(hbt.Tree(to_dev(k[perm], 8), to_dev(v[perm], 8), fanout=16))
+        trees[-1].set_param("exchange", exchange)
     grp = hbt.LocalShardGroup(trees)
     rng = np.random.default_rng(G)
-    qs = [queries(allk, rng, 4000 + 1000 * g) for g in range(G)]
-    outs = grp.search([to_dev(q, 8) for q in qs])
-    torch.cuda.synchronize()
-    for q, (pf, v) in zip(qs, outs):
-        epf, ev = full.search(q)
-        assert np.array_equal(pf.cpu().numpy().view(np.uint64), epf)
-        assert np.array_equal(from_dev(v, 8), ev)
+    for rep in range(2):  # second batch: larger, forces the windows to grow
+        qs = [queries(allk, rng, (4000 + 1000 * g) * (1 + 3 * rep)) for g in range(G)]
+        outs = grp.search([to_dev(q, 8) for q in qs])
+        torch.cuda.synchronize()
+        for q, (pf, v) in zip(qs, outs):
+            epf, ev = full.search(q)
+            assert np.array_equal(pf.cpu().numpy().view(np.uint64), epf)
+            assert np.array_equal(from_dev(v, 8), ev)
 
 
 def test_virtual_shards_reject_overlap(hbt):
@@ -76,18 +79,24 @@ def test_virtual_shards_reject_overlap(hbt):
         hbt.LocalShardGroup([a, b])
 
 
-def test_nccl_path_one_rank(hbt):
+@pytest.mark.parametrize("exchange", [0, 1])
+def test_nccl_path_one_rank(hbt, exchange):
+    """One rank over the real communicator: exchange 0 = fused peer-memory path
+    (IPC window export/all-gather, device barriers), 1 = NCCL send/recv."""
     uid = hbt.unique_id()
     comm = hbt.Comm(1, 0, uid)
     n = 100000
     allk = gen.stratified_keys(n, 7)
     allv = gen.values(n, 8, 9)
     t = hbt.ShardedTree(comm, to_dev(allk, 8), to_dev(allv, 8), fanout=16)
-    q = queries(allk, np.random.default_rng(0), 50000)
-    pf, v = t.search(to_dev(q, 8))
-    torch.cuda.synchronize()
-    epf, ev = oracle.ITree.from_pairs(allk, allv, 16, 8).search(q)
-    assert np.array_equal(pf.cpu().numpy().view(np.uint64), epf)
-    assert np.array_equal(from_dev(v, 8), ev)
+    t.set_param("exchange", exchange)
+    o = oracle.ITree.from_pairs(allk, allv, 16, 8)
+    for rep in range(3):
+        q = queries(allk, np.random.default_rng(rep), 20000 * (1 + rep))
+        pf, v = t.search(to_dev(q, 8))
+        torch.cuda.synchronize()
+        epf, ev = o.search(q)
+        assert np.array_equal(pf.cpu().numpy().view(np.uint64), epf)
+        assert np.array_equal(from_dev(v, 8), ev)
     t.close()
     comm.close()
