@@ -81,6 +81,9 @@ def lib():
         L.orc_rtree_update.restype = C.c_int
         L.orc_rtree_update.argtypes = [C.POINTER(_RTree), u64p, u64p, C.POINTER(C.c_uint8), C.c_uint64]
         L.orc_lower_bound.argtypes = [u64p, u64p, C.c_uint64, u64p, C.c_uint64, u64p, u64p, C.c_int]
+        u32p = C.POINTER(C.c_uint32)
+        L.orc_itree_range.argtypes = [C.POINTER(_ITree), u64p, u64p, C.c_uint64, C.c_uint32, u64p, u64p, u32p]
+        L.orc_rtree_range.argtypes = [C.POINTER(_RTree), u64p, u64p, C.c_uint64, C.c_uint32, u64p, u64p, u32p]
         _lib = L
     return _lib
 
@@ -120,6 +123,16 @@ def lower_bound(Kd, Vd, q, nthreads: int = 1):
     return pf, vals
 
 
+def _range(fn, ptr, lo, hi, k):
+    lo, hi = _as_u64(lo), _as_u64(hi)
+    m = len(lo)
+    ok = np.empty(m * k, np.uint64)
+    ov = np.empty(m * k, np.uint64)
+    oc = np.empty(m, np.uint32)
+    fn(ptr, _p64(lo), _p64(hi), m, k, _p64(ok), _p64(ov), oc.ctypes.data_as(C.POINTER(C.c_uint32)))
+    return ok.reshape(m, k), ov.reshape(m, k), oc
+
+
 class ITree:
     """Implicit tree: build from sorted distinct (Kd, Vd)."""
 
@@ -150,6 +163,10 @@ class ITree:
         vals = np.empty(len(q), np.uint64)
         lib().orc_itree_search(self._p, _p64(q), len(q), _p64(pf), _p64(vals), nthreads)
         return pf, vals
+
+    def range(self, lo, hi, k):
+        """Up to k pairs with lo <= key <= hi per query."""
+        return _range(lib().orc_itree_range, self._p, lo, hi, k)
 
     def update(self, keys, vals, ops):
         k, v = _as_u64(keys), _as_u64(vals)
@@ -197,6 +214,10 @@ class RTree:
         vals = np.empty(len(q), np.uint64)
         lib().orc_rtree_search(self._p, _p64(q), len(q), _p64(pf), _p64(vals), nthreads)
         return pf, vals
+
+    def range(self, lo, hi, k):
+        """Up to k pairs with lo <= key <= hi per query, through the chain."""
+        return _range(lib().orc_rtree_range, self._p, lo, hi, k)
 
     def update(self, keys, vals, ops):
         k, v = _as_u64(keys), _as_u64(vals)

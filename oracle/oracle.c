@@ -486,3 +486,61 @@ int orc_rtree_update(orc_rtree* t, const uint64_t* ok, const uint64_t* ov,
   free(dk); free(dv); free(dop);
   return 0;
 }
+
+/* ===========================================================================
+ * Range scan.  Implicit: the leaves are contiguous in key order,
+ * so after the descent the scan walks ranks r, r+1, ... of the L-segment.
+ * Regular: the scan walks the big leaf's entries, then the next big leaves in
+ * key order (the chain; the paper's linked leaves).
+ * ========================================================================= */
+void orc_itree_range(const orc_itree* t, const uint64_t* lo, const uint64_t* hi, uint64_t m, uint32_t k,
+                     uint64_t* out_keys, uint64_t* out_vals, uint32_t* out_count) {
+  uint64_t* pf = (uint64_t*)malloc((m ? m : 1) * sizeof(uint64_t));
+  uint64_t* vv = (uint64_t*)malloc((m ? m : 1) * sizeof(uint64_t));
+  orc_itree_search(t, lo, m, pf, vv, 1);
+  for (uint64_t x = 0; x < m; ++x) {
+    uint64_t r = pf[x] & ORC_END;
+    uint32_t c = 0;
+    for (uint32_t i = 0; i < k; ++i) {
+      out_keys[x * k + i] = t->kmax;
+      out_vals[x * k + i] = 0;
+    }
+    while (r != ORC_END && r < t->n && c < k && t->lkeys[r] <= hi[x]) {
+      out_keys[x * k + c] = t->lkeys[r];
+      out_vals[x * k + c] = t->lvals[r];
+      ++c;
+      ++r;
+    }
+    out_count[x] = c;
+  }
+  free(pf);
+  free(vv);
+}
+
+void orc_rtree_range(const orc_rtree* t, const uint64_t* lo, const uint64_t* hi, uint64_t m, uint32_t k,
+                     uint64_t* out_keys, uint64_t* out_vals, uint32_t* out_count) {
+  const uint64_t FP = (uint64_t)t->F * t->P;
+  for (uint64_t x = 0; x < m; ++x) {
+    for (uint32_t i = 0; i < k; ++i) {
+      out_keys[x * k + i] = t->kmax;
+      out_vals[x * k + i] = 0;
+    }
+    uint32_t c = 0;
+    /* the first entry >= lo: descend to its big leaf, then scan forward */
+    uint64_t v = rt_find_leaf(t, lo[x]);
+    uint64_t ci = 0;
+    while (t->chain[ci] != v) ++ci;   /* position of v in key order */
+    uint64_t e = 0;
+    while (e < t->lcount[v] && t->lkeys[v * FP + e] < lo[x]) ++e;
+    while (c < k && ci < t->nchain) {
+      v = t->chain[ci];
+      if (e >= t->lcount[v]) { ++ci; e = 0; continue; }
+      if (t->lkeys[v * FP + e] > hi[x]) break;
+      out_keys[x * k + c] = t->lkeys[v * FP + e];
+      out_vals[x * k + c] = t->lvals[v * FP + e];
+      ++c;
+      ++e;
+    }
+    out_count[x] = c;
+  }
+}

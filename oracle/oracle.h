@@ -74,6 +74,15 @@ void orc_rtree_search(const orc_rtree* t, const uint64_t* q, uint64_t m,
 int orc_rtree_update(orc_rtree* t, const uint64_t* ok, const uint64_t* ov,
                      const uint8_t* op, uint64_t nops);
 
+/* Range scan ("search for the first key in the range and then traverse
+ * leaf nodes until the last key is found"): for query i, the first up-to-k
+ * pairs with lo[i] <= key <= hi[i] in key order.  out_keys/out_vals are m x k
+ * row-major; unused slots are (MAX, 0); out_count[i] = pairs written. */
+void orc_itree_range(const orc_itree* t, const uint64_t* lo, const uint64_t* hi, uint64_t m, uint32_t k,
+                     uint64_t* out_keys, uint64_t* out_vals, uint32_t* out_count);
+void orc_rtree_range(const orc_rtree* t, const uint64_t* lo, const uint64_t* hi, uint64_t m, uint32_t k,
+                     uint64_t* out_keys, uint64_t* out_vals, uint32_t* out_count);
+
 /* plain definition: lower_bound over sorted distinct keys */
 void orc_lower_bound(const uint64_t* Kd, const uint64_t* Vd, uint64_t n,
                      const uint64_t* q, uint64_t m, uint64_t* pos_found, uint64_t* vals,

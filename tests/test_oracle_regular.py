@@ -202,3 +202,44 @@ def test_regular_split_appends_pool_indices_in_key_order():
     assert a["chain"].tolist() == [0, 3, 1, 2, 4]
     assert a["pool"] == 5
     assert a["lcount"].tolist() == [8, 10, 8, 9, 9]
+
+
+@pytest.mark.parametrize("layout", ["implicit", "regular"])
+@pytest.mark.parametrize("width", [4, 8])
+def test_range_scan_matches_sorted_slices(layout, width):
+    """Range scan = the first up-to-k sorted keys in [lo, hi]: pinned by
+    numpy.searchsorted + slicing of the sorted key array (and a dict for values),
+    also after updates that split / remove leaves (regular: chain traversal)."""
+    rng = np.random.default_rng(width + (layout == "regular"))
+    mx = kmax(width)
+    k, v = gen_keys(3000, width, rng, dup=True)
+    T = oracle.ITree if layout == "implicit" else oracle.RTree
+    t = T.from_pairs(k, v, 4, width)
+    d = dict(zip(k.tolist(), v.tolist()))
+    if layout == "regular":  # make the chain non-trivial: splits and removals
+        ins = rng.integers(0, mx, 2000, dtype=np.uint64, endpoint=True)
+        dels = k[:1000]
+        ok = np.concatenate([ins, dels])
+        ov = rng.integers(0, mx, len(ok), dtype=np.uint64, endpoint=True)
+        op = np.concatenate([np.zeros(len(ins), np.uint8), np.ones(len(dels), np.uint8)])
+        t.update(ok, ov, op)
+        for a_, b_, o_ in zip(ok.tolist(), ov.tolist(), op.tolist()):
+            if o_ == 0:
+                d[a_] = b_
+            else:
+                d.pop(a_, None)
+    Kd = np.array(sorted(d), np.uint64)
+    lo = query_set(Kd[:200], width, rng, 300)
+    span = rng.integers(0, mx // 200, len(lo), dtype=np.uint64)
+    hi = np.minimum(lo.astype(object) + span.astype(object), mx).astype(np.uint64)
+    hi[:10] = mx
+    for kk in (1, 5, 32):
+        ok_, ov_, oc = t.range(lo, hi, kk)
+        for x in range(len(lo)):
+            a = int(np.searchsorted(Kd, lo[x], side="left"))
+            b = int(np.searchsorted(Kd, hi[x], side="right"))
+            want = Kd[a:min(b, a + kk)]
+            assert oc[x] == len(want), (x, kk)
+            assert ok_[x, : len(want)].tolist() == want.tolist()
+            assert ov_[x, : len(want)].tolist() == [d[int(z)] for z in want.tolist()]
+            assert (ok_[x, len(want):] == mx).all() and (ov_[x, len(want):] == 0).all()
