@@ -145,6 +145,16 @@ HBT_API int hbt_search(const hbt_tree* t, const void* queries, uint64_t m, hbt_o
 HBT_API int hbt_search_host(const hbt_tree* t, const void* host_queries, uint64_t m,
                     uint64_t* host_pos_found, void* host_values, void* stream);
 
+/* Range scan (the range-query experiment of P:392): for each of the m
+ * queries, the first up-to-k pairs with lo[i] <= key <= hi[i] in key order.
+ * lo/hi: device arrays (width S, length m).  out_keys/out_values: device arrays
+ * of m*k elements (row i = query i; slots past the count are (MAX, 0));
+ * out_count: device uint32[m].  k in [1, 4096].  Asynchronous on `stream`.
+ * IMPLICIT scans consecutive ranks of the contiguous L-segment; REGULAR scans
+ * the big leaf, then the next big leaves in key order. */
+HBT_API int hbt_range(const hbt_tree* t, const void* lo, const void* hi, uint64_t m, uint32_t k,
+                      void* out_keys, void* out_values, uint32_t* out_count, void* stream);
+
 /* Apply a batch of UPSERT/DELETE ops.  IMPLICIT: merge into the
  * sorted pairs and rebuild.  REGULAR: per-big-leaf merge on the GPU,
  * splits into new pool indices, removal of emptied leaves, then the upper

@@ -36,7 +36,7 @@ UPSERT, DELETE = 0, 1
 
 EXPORTED = ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
             "hbt_info", "hbt_export", "hbt_set_param", "hbt_last_error", "hbt_version",
-            "hbt_comm_unique_id", "hbt_comm_init", "hbt_comm_destroy", "hbt_bulk_build_sharded",
+            "hbt_range", "hbt_comm_unique_id", "hbt_comm_init", "hbt_comm_destroy", "hbt_bulk_build_sharded",
             "hbt_search_sharded", "hbt_shard_local_init", "hbt_search_sharded_local"]
 
 
@@ -76,6 +76,7 @@ def _load():
     L.hbt_info.argtypes = [vp, C.POINTER(_Info)]
     L.hbt_export.argtypes = [vp, u32, vp, u64, C.POINTER(u64)]
     L.hbt_set_param.argtypes = [vp, C.c_char_p, C.c_int64]
+    L.hbt_range.argtypes = [vp, vp, vp, u64, u32, vp, vp, vp, vp]
     L.hbt_comm_unique_id.argtypes = [vp]
     L.hbt_comm_init.argtypes = [C.c_int, C.c_int, vp, C.POINTER(vp)]
     L.hbt_comm_destroy.argtypes = [vp]
@@ -87,7 +88,7 @@ def _load():
     L.hbt_last_error.restype = C.c_char_p
     L.hbt_version.restype = C.c_char_p
     for f in ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
-              "hbt_info", "hbt_export", "hbt_set_param", "hbt_comm_unique_id", "hbt_comm_init",
+              "hbt_info", "hbt_export", "hbt_set_param", "hbt_range", "hbt_comm_unique_id", "hbt_comm_init",
               "hbt_comm_destroy", "hbt_bulk_build_sharded", "hbt_search_sharded", "hbt_shard_local_init",
               "hbt_search_sharded_local"]:
         getattr(L, f).restype = C.c_int
@@ -193,6 +194,22 @@ class Tree:
         _check(lib.hbt_search_host(self._h, C.c_void_p(ptr(queries)), m, C.c_void_p(ptr(out_pos)),
                                    C.c_void_p(ptr(out_vals)), _stream_ptr(stream)))
         return out_pos, out_vals
+
+    def range(self, lo, hi, k: int, stream=None):
+        """Up to k pairs with lo <= key <= hi per query.
+        Returns (keys [m, k], values [m, k], count [m] int32)."""
+        torch = self._torch
+        lo, hi = lo.contiguous(), hi.contiguous()
+        m = lo.numel()
+        dt = _dtype(self.width)
+        ok = torch.empty((m, k), dtype=dt, device=lo.device)
+        ov = torch.empty((m, k), dtype=dt, device=lo.device)
+        oc = torch.empty(m, dtype=torch.int32, device=lo.device)
+        if m:
+            _check(lib.hbt_range(self._h, C.c_void_p(lo.data_ptr()), C.c_void_p(hi.data_ptr()), m, k,
+                                 C.c_void_p(ok.data_ptr()), C.c_void_p(ov.data_ptr()), C.c_void_p(oc.data_ptr()),
+                                 _stream_ptr(stream)))
+        return ok, ov, oc
 
     # -- updates
     def update(self, keys, values, ops, stream=None):

@@ -42,6 +42,7 @@ static void free_tree(hbt_tree* t) {
   regular_free(t);
   shard_free(t);
   fused_free(t);
+  range_free(t);
   cudaFree(t->pipe.d_q);
   cudaFree(t->pipe.d_pf);
   cudaFree(t->pipe.d_v);
@@ -159,6 +160,19 @@ int hbt_search_host(const hbt_tree* t, const void* host_queries, uint64_t m, uin
   }
   for (int i = 0; i < 2; ++i) HBT_CUDA_TRY(cudaStreamSynchronize(p.s[i]));
   return HBT_OK;
+}
+
+int hbt_range(const hbt_tree* t, const void* lo, const void* hi, uint64_t m, uint32_t k, void* out_keys,
+              void* out_values, uint32_t* out_count, void* stream) {
+  if (!t) { set_error("tree is NULL"); return HBT_EINVAL; }
+  if (m == 0) return HBT_OK;
+  if (k == 0 || k > 4096) { set_error("k must be in [1, 4096]"); return HBT_EINVAL; }
+  if (!is_device_ptr(lo) || !is_device_ptr(hi) || !is_device_ptr(out_keys) || !is_device_ptr(out_values) ||
+      !is_device_ptr(out_count)) {
+    set_error("range arrays must be device pointers");
+    return HBT_EINVAL;
+  }
+  return range_scan(t, lo, hi, m, k, out_keys, out_values, out_count, (cudaStream_t)stream);
 }
 
 int hbt_bulk_update(hbt_tree* t, const hbt_batch* batch, void* stream) {

@@ -74,6 +74,8 @@ struct RegularState {
   void* d_dir = nullptr;
   uint64_t dir_bytes = 0, dir_cap = 0;
   uint32_t dir_T = 0, dir_count = 0, dir_bits = 0;
+  uint32_t* d_chainpos = nullptr;        // pool-sized: big leaf -> position in the chain (range scans)
+  uint64_t chainpos_cap = 0;
 };
 
 struct HostPipe {
@@ -154,6 +156,10 @@ struct hbt_tree {
   hbt::ShardMeta shard;
   hbt::Scratch shard_scratch;
   void* fused = nullptr;  // sharded_fused.cu state (peer windows)
+  // range-scan scratch (lower bounds of the range starts)
+  uint64_t* d_rpf = nullptr;
+  void* d_rv = nullptr;
+  uint64_t rcap = 0;
   // ---- search ----
   hbt::SearchConfig cfg;
   mutable hbt::HostPipe pipe;
@@ -174,6 +180,10 @@ int implicit_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, 
 int implicit_search_base(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
                          cudaStream_t s);
 void shard_free(hbt_tree* t);
+// range.cu
+void range_free(hbt_tree* t);
+int range_scan(const hbt_tree* t, const void* lo, const void* hi, uint64_t m, uint32_t k, void* ok, void* ov,
+               uint32_t* oc, cudaStream_t s);
 // sharded_fused.cu
 void fused_free(hbt_tree* t);
 int fused_search_local(hbt_tree* const* shards, int G, const void* const* queries, const uint64_t* m,

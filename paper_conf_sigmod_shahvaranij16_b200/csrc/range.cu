@@ -1,0 +1,164 @@
+// range.cu — hbt_range: range scans ("search for the first key in
+// the range and then traverse leaf nodes until the last key is found"; the
+// paper's range-query experiment, returns 1..32 keys per query).
+//
+// Step 1 is the tree's own lower-bound search of the range start (the hot
+// path).  Step 2: one warp per query walks forward 32 entries at a time —
+// implicit: consecutive ranks of the contiguous L-segment ("leaf nodes
+// are arranged sequentially"); regular: the entries of big leaf v, then the next
+// big leaf in key order (the chain, the paper's linked leaves).  Keys are sorted,
+// so the entries <= hi form a prefix of each chunk: popc(ballot(key <= hi)).
+#include "hbt_internal.cuh"
+
+namespace hbt {
+namespace {
+
+constexpr uint64_t kEnd = HBT_POS_END;
+
+template <typename K>
+__device__ __forceinline__ K key_max() { return K(~K(0)); }
+
+template <typename K>
+__global__ void range_implicit(const K* __restrict__ leaf, uint64_t n, const uint64_t* __restrict__ pf,
+                               const K* __restrict__ hi, uint64_t m, uint32_t k, K* __restrict__ ok,
+                               K* __restrict__ ov, uint32_t* __restrict__ oc) {
+  constexpr uint32_t P = 64 / (2 * sizeof(K));
+  const int lane = threadIdx.x & 31;
+  const uint64_t w0 = (blockIdx.x * uint64_t(blockDim.x) + threadIdx.x) >> 5;
+  const uint64_t nw = (uint64_t(gridDim.x) * blockDim.x) >> 5;
+  for (uint64_t x = w0; x < m; x += nw) {
+    const uint64_t r0 = pf[x] & kEnd;
+    const K h = hi[x];
+    uint32_t c = 0;
+    bool done = (r0 == kEnd);
+    for (uint32_t base = 0; base < k; base += 32) {
+      const uint32_t i = base + lane;
+      bool valid = false;
+      K key = key_max<K>(), val = K(0);
+      if (!done && i < k) {
+        const uint64_t r = r0 + i;
+        if (r < n) {
+          key = leaf[(r / P) * (2 * P) + r % P];
+          val = leaf[(r / P) * (2 * P) + P + r % P];
+          valid = key <= h;
+        }
+      }
+      const unsigned b = __ballot_sync(0xffffffffu, valid);
+      if (i < k) {
+        ok[x * k + i] = valid ? key : key_max<K>();
+        ov[x * k + i] = valid ? val : K(0);
+      }
+      c += __popc(b);
+      if (b != 0xffffffffu) done = true;
+    }
+    if (lane == 0) oc[x] = c;
+  }
+}
+
+template <typename K>
+__global__ void range_regular(const K* __restrict__ leaf, const uint32_t* __restrict__ count,
+                              const uint32_t* __restrict__ chain, const uint32_t* __restrict__ chainpos,
+                              uint64_t nchain, uint32_t F, const uint64_t* __restrict__ pf,
+                              const K* __restrict__ hi, uint64_t m, uint32_t k, K* __restrict__ ok,
+                              K* __restrict__ ov, uint32_t* __restrict__ oc) {
+  constexpr uint32_t P = 64 / (2 * sizeof(K));
+  const uint64_t FP = uint64_t(F) * P;
+  const int lane = threadIdx.x & 31;
+  const uint64_t w0 = (blockIdx.x * uint64_t(blockDim.x) + threadIdx.x) >> 5;
+  const uint64_t nw = (uint64_t(gridDim.x) * blockDim.x) >> 5;
+  for (uint64_t x = w0; x < m; x += nw) {
+    const uint64_t pos = pf[x] & kEnd;
+    const K h = hi[x];
+    for (uint32_t i = lane; i < k; i += 32) {
+      ok[x * k + i] = key_max<K>();
+      ov[x * k + i] = K(0);
+    }
+    uint32_t c = 0;
+    if (pos != kEnd) {
+      uint64_t v = pos / FP;
+      uint32_t e = uint32_t(pos % FP);  // dense packing: line j slot s = entry j*P + s
+      uint64_t ci = chainpos[v];
+      while (c < k) {
+        const uint32_t cnt = count[v];
+        const uint32_t take0 = cnt - e < 32u ? cnt - e : 32u;
+        const uint32_t take = take0 < k - c ? take0 : k - c;
+        bool valid = false;
+        K key = key_max<K>(), val = K(0);
+        if (uint32_t(lane) < take) {
+          const uint32_t en = e + lane;
+          key = leaf[(v * F + en / P) * (2 * P) + en % P];
+          val = leaf[(v * F + en / P) * (2 * P) + P + en % P];
+          valid = key <= h;
+        }
+        const unsigned b = __ballot_sync(0xffffffffu, valid);
+        if (valid) {
+          ok[x * k + c + lane] = key;
+          ov[x * k + c + lane] = val;
+        }
+        const uint32_t got = __popc(b);
+        c += got;
+        if (got < take) break;       // passed hi
+        e += take;
+        if (e >= cnt) {              // next big leaf in key order
+          if (++ci >= nchain) break;
+          v = chain[ci];
+          e = 0;
+        }
+      }
+    }
+    if (lane == 0) oc[x] = c;
+  }
+}
+
+inline unsigned warps_grid(uint64_t m) {
+  uint64_t g = (m + 7) / 8;  // 8 warps per 256-thread block
+  if (g > 148 * 32) g = 148 * 32;
+  return unsigned(g ? g : 1);
+}
+
+template <typename K>
+int range_t(hbt_tree* t, const void* lo, const void* hi, uint64_t m, uint32_t k, void* ok, void* ov, uint32_t* oc,
+            cudaStream_t s) {
+  if (m > t->rcap) {
+    cudaFree(t->d_rpf);
+    cudaFree(t->d_rv);
+    t->d_rpf = nullptr;
+    t->d_rv = nullptr;
+    t->rcap = 0;
+    HBT_CUDA_TRY(cudaMalloc(&t->d_rpf, m * 8));
+    HBT_CUDA_TRY(cudaMalloc(&t->d_rv, m * sizeof(K)));
+    t->rcap = m;
+  }
+  int rc = t->form == HBT_REGULAR ? regular_search(t, lo, m, t->d_rpf, t->d_rv, s)
+                                  : implicit_search(t, lo, m, t->d_rpf, t->d_rv, s);
+  if (rc) return rc;
+  if (t->form == HBT_REGULAR) {
+    const RegularState& r = t->r;
+    range_regular<K><<<warps_grid(m), 256, 0, s>>>((const K*)r.d_leaf, r.d_count, r.d_chain, r.d_chainpos, r.nchain,
+                                                   t->F, t->d_rpf, (const K*)hi, m, k, (K*)ok, (K*)ov, oc);
+  } else {
+    range_implicit<K><<<warps_grid(m), 256, 0, s>>>((const K*)t->d_leaf, t->n, t->d_rpf, (const K*)hi, m, k, (K*)ok,
+                                                    (K*)ov, oc);
+  }
+  HBT_CUDA_TRY(cudaGetLastError());
+  return HBT_OK;
+}
+
+}  // namespace
+
+void range_free(hbt_tree* t) {
+  cudaFree(t->d_rpf);
+  cudaFree(t->d_rv);
+  t->d_rpf = nullptr;
+  t->d_rv = nullptr;
+  t->rcap = 0;
+}
+
+int range_scan(const hbt_tree* tc, const void* lo, const void* hi, uint64_t m, uint32_t k, void* ok, void* ov,
+               uint32_t* oc, cudaStream_t s) {
+  hbt_tree* t = const_cast<hbt_tree*>(tc);
+  std::lock_guard<std::mutex> lock(t->pipe.mu);
+  return t->width == 4 ? range_t<uint32_t>(t, lo, hi, m, k, ok, ov, oc, s) : range_t<uint64_t>(t, lo, hi, m, k, ok, ov, oc, s);
+}
+
+}  // namespace hbt

@@ -777,9 +777,21 @@ int rebuild_upper(hbt_tree* t, cudaStream_t s) {
   return HBT_OK;
 }
 
+__global__ void chain_positions(const uint32_t* __restrict__ chain, uint64_t nchain, uint32_t* __restrict__ pos) {
+  GRID_STRIDE(i, nchain) pos[chain[i]] = uint32_t(i);
+}
+
 template <typename K>
 int rebuild_dir(hbt_tree* t, cudaStream_t s) {
   RegularState& r = t->r;
+  if (r.chainpos_cap < r.cap) {
+    cudaFree(r.d_chainpos);
+    r.d_chainpos = nullptr;
+    r.chainpos_cap = 0;
+    HBT_CUDA_TRY(cudaMalloc(&r.d_chainpos, r.cap * 4));
+    r.chainpos_cap = r.cap;
+  }
+  chain_positions<<<grid_for(r.nchain), 256, 0, s>>>(r.d_chain, r.nchain, r.d_chainpos);
   const uint32_t F = t->F;
   // root-first level d: d < U -> upper level U-1-d, d == U -> the last level (big leaves)
   auto count_at = [&](uint32_t d) -> uint64_t { return d < r.U ? r.unodes[r.U - 1 - d] : r.nchain; };
@@ -1316,6 +1328,7 @@ void regular_free(hbt_tree* t) {
   RegularState& r = t->r;
   cudaFree(r.d_leaf); cudaFree(r.d_count); cudaFree(r.d_lkeys); cudaFree(r.d_lidx); cudaFree(r.d_chain);
   cudaFree(r.d_ukeys); cudaFree(r.d_uidx); cudaFree(r.d_urefs); cudaFree(r.d_seg_of_leaf); cudaFree(r.d_dir);
+  cudaFree(r.d_chainpos);
   r = RegularState{};
 }
 
