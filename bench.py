@@ -55,6 +55,8 @@ def parse():
     ap.add_argument("--l2-persist", type=int, default=None, help="bytes of I-segment in a persisting L2 window")
     ap.add_argument("--l2-levels", type=int, default=None, help="L2 budget for index+sector levels (bytes)")
     ap.add_argument("--exchange", type=int, default=None, help="c4: 0 = fused peer-memory exchange, 1 = NCCL")
+    ap.add_argument("--range-k", type=int, default=0,
+                    help="time range scans returning k keys per query (PAPER.md:392) instead of point lookups")
     return ap.parse_args()
 
 
@@ -198,8 +200,20 @@ def make_work(cfg_name, rank, world, args):
         tree.set_param("exchange", args.exchange)
     out_pos = torch.empty(m, dtype=torch.int64, device="cuda")
     out_val = torch.empty(m, dtype=sdt, device="cuda")
+    hi = None
+    if args.range_k:
+        hi = torch.full_like(q, -1)  # MAX: every range returns k keys unless the tree ends
+        qdesc += f"; range scans of {args.range_k} keys from each query key"
     return Work(c=c, name=cfg_name, tree=tree, q=q, m=m, w=w, hit_rate=hit_rate, qdesc=qdesc, extra=extra,
-                out_pos=out_pos, out_val=out_val, info=tree.info())
+                out_pos=out_pos, out_val=out_val, info=tree.info(), range_k=args.range_k, hi=hi)
+
+
+def step(work):
+    """One step: the whole batch through the hot path."""
+    if work.range_k:
+        work.tree.range(work.q, work.hi, work.range_k)
+    else:
+        work.tree.search(work.q, work.out_pos, work.out_val)
 
 
 def time_search(work, steps, world):
@@ -214,7 +228,7 @@ def time_search(work, steps, world):
     torch.cuda.synchronize()
     ev0.record(stream)
     for _ in range(steps):
-        work.tree.search(work.q, work.out_pos, work.out_val)
+        step(work)
     ev1.record(stream)
     torch.cuda.synchronize()
     if world > 1:
@@ -279,14 +293,14 @@ def run_hbt(args):
     l2_probe = probe_l2_gbs(32 if node_b > 32 else node_b) if rank == 0 else None
 
     for _ in range(max(args.warmup, 3)):
-        work.tree.search(work.q, work.out_pos, work.out_val)
+        step(work)
     torch.cuda.synchronize()
     sampler = ClockSampler(local)
     sampler.start()
     ms_step = time_search(work, args.steps, world)
     clocks = sampler.stop()
     qps = world * m / (ms_step * 1e-3)
-    launches_per_step = 4 if args.config == "c4" else 1
+    launches_per_step = 4 if args.config == "c4" else (2 if args.range_k else 1)
 
     after = None
     if "batch" in work.extra:  # c3: the 1 % bulk update, timed once, then search again
@@ -305,11 +319,16 @@ def run_hbt(args):
                                          "unit": "M queries/s", "ms_per_step": round(ms_after, 4)},
                  "n_distinct_after": work.tree.info()["n_distinct"]}
 
-    e2e = time_e2e(work, args.e2e_steps, world)
+    e2e = time_e2e(work, args.e2e_steps, world) if not args.range_k else None
 
     # ---- roofline of the step's dominant kernel (the search)
     l2_size = torch.cuda.get_device_properties(local).L2_cache_size
     mdl = roofline.model(info, l2_size, work.hit_rate)
+    if args.range_k:  # + the further leaf lines walked and the k pairs written (+ count)
+        P = 64 // (2 * w)
+        extra_b = ((args.range_k - 1 + P - 1) // P) * 64 + args.range_k * 2 * w + 4
+        mdl["hbm_bytes_per_query"] += extra_b
+        mdl["l2_bytes_per_query"] += extra_b
     peak, peak_src = measured_peaks()
     t_kernel = ms_step * 1e-3
     achieved = mdl["hbm_bytes_per_query"] * m / t_kernel / 1e9

@@ -18,21 +18,26 @@ constexpr uint64_t kEnd = HBT_POS_END;
 template <typename K>
 __device__ __forceinline__ K key_max() { return K(~K(0)); }
 
+// L lanes per query (L = next power of two >= min(k, 32)), 32/L queries per warp;
+// every sub-group walks its own query, chunk by chunk, until done or k reached.
 template <typename K>
 __global__ void range_implicit(const K* __restrict__ leaf, uint64_t n, const uint64_t* __restrict__ pf,
-                               const K* __restrict__ hi, uint64_t m, uint32_t k, K* __restrict__ ok,
+                               const K* __restrict__ hi, uint64_t m, uint32_t k, uint32_t L, K* __restrict__ ok,
                                K* __restrict__ ov, uint32_t* __restrict__ oc) {
   constexpr uint32_t P = 64 / (2 * sizeof(K));
-  const int lane = threadIdx.x & 31;
+  const uint32_t lane = threadIdx.x & 31, sub = lane % L, grp = lane / L, QW = 32 / L;
+  const unsigned gmask = (L == 32 ? 0xffffffffu : ((1u << L) - 1u)) << (grp * L);
   const uint64_t w0 = (blockIdx.x * uint64_t(blockDim.x) + threadIdx.x) >> 5;
   const uint64_t nw = (uint64_t(gridDim.x) * blockDim.x) >> 5;
-  for (uint64_t x = w0; x < m; x += nw) {
-    const uint64_t r0 = pf[x] & kEnd;
-    const K h = hi[x];
+  for (uint64_t xb = w0 * QW; xb < m; xb += nw * QW) {
+    const uint64_t x = xb + grp;
+    const bool live = x < m;
+    const uint64_t r0 = live ? (pf[x] & kEnd) : kEnd;
+    const K h = live ? hi[x] : K(0);
     uint32_t c = 0;
     bool done = (r0 == kEnd);
-    for (uint32_t base = 0; base < k; base += 32) {
-      const uint32_t i = base + lane;
+    for (uint32_t base = 0; base < k; base += L) {
+      const uint32_t i = base + sub;
       bool valid = false;
       K key = key_max<K>(), val = K(0);
       if (!done && i < k) {
@@ -43,15 +48,15 @@ __global__ void range_implicit(const K* __restrict__ leaf, uint64_t n, const uin
           valid = key <= h;
         }
       }
-      const unsigned b = __ballot_sync(0xffffffffu, valid);
-      if (i < k) {
+      const unsigned b = __ballot_sync(0xffffffffu, valid) & gmask;
+      if (live && i < k) {
         ok[x * k + i] = valid ? key : key_max<K>();
         ov[x * k + i] = valid ? val : K(0);
       }
       c += __popc(b);
-      if (b != 0xffffffffu) done = true;
+      if (b != gmask) done = true;
     }
-    if (lane == 0) oc[x] = c;
+    if (live && sub == 0) oc[x] = c;
   }
 }
 
@@ -59,59 +64,67 @@ template <typename K>
 __global__ void range_regular(const K* __restrict__ leaf, const uint32_t* __restrict__ count,
                               const uint32_t* __restrict__ chain, const uint32_t* __restrict__ chainpos,
                               uint64_t nchain, uint32_t F, const uint64_t* __restrict__ pf,
-                              const K* __restrict__ hi, uint64_t m, uint32_t k, K* __restrict__ ok,
+                              const K* __restrict__ hi, uint64_t m, uint32_t k, uint32_t L, K* __restrict__ ok,
                               K* __restrict__ ov, uint32_t* __restrict__ oc) {
   constexpr uint32_t P = 64 / (2 * sizeof(K));
   const uint64_t FP = uint64_t(F) * P;
-  const int lane = threadIdx.x & 31;
+  const uint32_t lane = threadIdx.x & 31, sub = lane % L, grp = lane / L, QW = 32 / L;
+  const unsigned gmask = (L == 32 ? 0xffffffffu : ((1u << L) - 1u)) << (grp * L);
   const uint64_t w0 = (blockIdx.x * uint64_t(blockDim.x) + threadIdx.x) >> 5;
   const uint64_t nw = (uint64_t(gridDim.x) * blockDim.x) >> 5;
-  for (uint64_t x = w0; x < m; x += nw) {
-    const uint64_t pos = pf[x] & kEnd;
-    const K h = hi[x];
-    for (uint32_t i = lane; i < k; i += 32) {
-      ok[x * k + i] = key_max<K>();
-      ov[x * k + i] = K(0);
-    }
+  for (uint64_t xb = w0 * QW; xb < m; xb += nw * QW) {
+    const uint64_t x = xb + grp;
+    const bool live = x < m;
+    const uint64_t pos = live ? (pf[x] & kEnd) : kEnd;
+    const K h = live ? hi[x] : K(0);
+    if (live)
+      for (uint32_t i = sub; i < k; i += L) {
+        ok[x * k + i] = key_max<K>();
+        ov[x * k + i] = K(0);
+      }
     uint32_t c = 0;
-    if (pos != kEnd) {
-      uint64_t v = pos / FP;
-      uint32_t e = uint32_t(pos % FP);  // dense packing: line j slot s = entry j*P + s
-      uint64_t ci = chainpos[v];
-      while (c < k) {
+    bool active = pos != kEnd;
+    uint64_t v = active ? pos / FP : 0, ci = active ? chainpos[v] : 0;
+    uint32_t e = active ? uint32_t(pos % FP) : 0;  // dense packing: line j slot s = entry j*P + s
+    while (__any_sync(0xffffffffu, active)) {
+      uint32_t take = 0;
+      bool valid = false;
+      K key = key_max<K>(), val = K(0);
+      if (active) {
         const uint32_t cnt = count[v];
-        const uint32_t take0 = cnt - e < 32u ? cnt - e : 32u;
-        const uint32_t take = take0 < k - c ? take0 : k - c;
-        bool valid = false;
-        K key = key_max<K>(), val = K(0);
-        if (uint32_t(lane) < take) {
-          const uint32_t en = e + lane;
+        const uint32_t take0 = cnt - e < L ? cnt - e : L;
+        take = take0 < k - c ? take0 : k - c;
+        if (sub < take) {
+          const uint32_t en = e + sub;
           key = leaf[(v * F + en / P) * (2 * P) + en % P];
           val = leaf[(v * F + en / P) * (2 * P) + P + en % P];
           valid = key <= h;
         }
-        const unsigned b = __ballot_sync(0xffffffffu, valid);
+      }
+      const unsigned b = __ballot_sync(0xffffffffu, valid) & gmask;
+      if (active) {
         if (valid) {
-          ok[x * k + c + lane] = key;
-          ov[x * k + c + lane] = val;
+          ok[x * k + c + sub] = key;
+          ov[x * k + c + sub] = val;
         }
         const uint32_t got = __popc(b);
         c += got;
-        if (got < take) break;       // passed hi
         e += take;
-        if (e >= cnt) {              // next big leaf in key order
-          if (++ci >= nchain) break;
-          v = chain[ci];
-          e = 0;
+        if (got < take || c >= k) {
+          active = false;                    // passed hi, or k reached
+        } else if (e >= count[v]) {          // next big leaf in key order
+          if (++ci >= nchain) active = false;
+          else { v = chain[ci]; e = 0; }
         }
       }
     }
-    if (lane == 0) oc[x] = c;
+    if (live && sub == 0) oc[x] = c;
   }
 }
 
-inline unsigned warps_grid(uint64_t m) {
-  uint64_t g = (m + 7) / 8;  // 8 warps per 256-thread block
+inline unsigned warps_grid(uint64_t m, uint32_t L) {
+  const uint64_t warps = (m + 32 / L - 1) / (32 / L);
+  uint64_t g = (warps + 7) / 8;  // 8 warps per 256-thread block
   if (g > 148 * 32) g = 148 * 32;
   return unsigned(g ? g : 1);
 }
@@ -132,13 +145,16 @@ int range_t(hbt_tree* t, const void* lo, const void* hi, uint64_t m, uint32_t k,
   int rc = t->form == HBT_REGULAR ? regular_search(t, lo, m, t->d_rpf, t->d_rv, s)
                                   : implicit_search(t, lo, m, t->d_rpf, t->d_rv, s);
   if (rc) return rc;
+  uint32_t L = 1;
+  while (L < k && L < 32) L <<= 1;
   if (t->form == HBT_REGULAR) {
     const RegularState& r = t->r;
-    range_regular<K><<<warps_grid(m), 256, 0, s>>>((const K*)r.d_leaf, r.d_count, r.d_chain, r.d_chainpos, r.nchain,
-                                                   t->F, t->d_rpf, (const K*)hi, m, k, (K*)ok, (K*)ov, oc);
+    range_regular<K><<<warps_grid(m, L), 256, 0, s>>>((const K*)r.d_leaf, r.d_count, r.d_chain, r.d_chainpos,
+                                                      r.nchain, t->F, t->d_rpf, (const K*)hi, m, k, L, (K*)ok,
+                                                      (K*)ov, oc);
   } else {
-    range_implicit<K><<<warps_grid(m), 256, 0, s>>>((const K*)t->d_leaf, t->n, t->d_rpf, (const K*)hi, m, k, (K*)ok,
-                                                    (K*)ov, oc);
+    range_implicit<K><<<warps_grid(m, L), 256, 0, s>>>((const K*)t->d_leaf, t->n, t->d_rpf, (const K*)hi, m, k, L,
+                                                       (K*)ok, (K*)ov, oc);
   }
   HBT_CUDA_TRY(cudaGetLastError());
   return HBT_OK;
