@@ -174,8 +174,11 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *   "threads"     threads per CTA: 256, 512 or 1024 (0 = default: implicit 1024, regular 512)
  *   "ctas_per_sm" cap on resident CTAs per SM (0 = occupancy-derived)
  *   "qpl"         queries per lane per warp round, 1 or 2 (0 = default)
- *   "smem_mode"   implicit top levels: 2 = level-T directory + one lower bound (default),
- *                 0 = per-level binary search of staged nodes, 1 = the same on 32-bit hi/lo planes
+ *   "smem_mode"   implicit top levels: 2 = level-T directory + one lower bound, staged in shared
+ *                 memory (default), 3 = the same read in place from L2 (used automatically for
+ *                 batches <= "small_batch"), 0 = per-level binary search of staged nodes,
+ *                 1 = the same on 32-bit hi/lo planes
+ *   "small_batch" mode 2: batches of at most this many queries use mode 3 (default 65536)
  *   "carveout"    preferred shared-memory carve-out percent, -1 = driver default
  *   "l2_persist"  implicit: keep up to this many bytes of the I-segment (+ index) in a
  *                 persisting L2 access-policy window (sets the device persisting-L2 limit), 0 = off

@@ -203,7 +203,7 @@ int hbt_info(const hbt_tree* t, hbt_info_t* info) {
   info->n_distinct = t->n;
   if (t->form == HBT_IMPLICIT) {
     info->height = t->H;
-    info->smem_levels = t->cfg.mode == 2 ? t->dir_T : implicit_smem_levels(t, t->cfg.smem_budget);
+    info->smem_levels = t->cfg.mode >= 2 ? t->dir_T : implicit_smem_levels(t, t->cfg.smem_budget);
     for (uint32_t d = 0; d < t->H; ++d) info->level_nodes[d] = t->nodes[d];
     info->leaf_lines = t->L0;
     info->chain_len = t->L0;
@@ -262,7 +262,8 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "threads" && (value == 0 || value == 256 || value == 512 || value == 1024)) c.threads = uint32_t(value);
   else if (n == "ctas_per_sm" && value >= 0 && value <= 32) c.ctas_per_sm = uint32_t(value);
   else if (n == "qpl" && value >= 0 && value <= 2) c.qpl = uint32_t(value);
-  else if (n == "smem_mode" && value >= 0 && value <= 2) c.mode = uint32_t(value);
+  else if (n == "smem_mode" && value >= 0 && value <= 3) c.mode = uint32_t(value);
+  else if (n == "small_batch" && value >= 0) c.small_batch = uint64_t(value);
   else if (n == "carveout" && value >= -1 && value <= 100) c.carveout = int(value);
   else if (n == "l2_persist" && value >= 0) c.l2_persist = uint64_t(value);
   else if (n == "l2_levels_bytes" && value >= 0) c.l2_levels_bytes = uint64_t(value);

@@ -46,6 +46,7 @@ struct SearchConfig {
   uint64_t l2_persist = 0;       // bytes of the I-segment to keep in a persisting L2 window (0 = off)
   uint64_t l2_levels_bytes = 0;  // L2-resident budget for index+sector levels (0 = default 32 MB)
   uint32_t exchange = 0;         // sharded search: 0 = fused peer-memory exchange, 1 = NCCL send/recv
+  uint64_t small_batch = 1u << 16;  // mode 2: batches up to this size read the directory in place (mode 3)
 };
 
 // Regular-tree device state.  All pools are SoA arrays

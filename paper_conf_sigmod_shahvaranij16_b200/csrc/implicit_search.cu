@@ -114,7 +114,7 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
   // node would sit in the same bank and the lanes' probes into different nodes
   // would serialise.  MODE 1 splits 64-bit keys into 32-bit hi / lo planes.
   constexpr uint32_t FP = F + 1;
-  const uint32_t s_nodes = MODE == 2 ? 0u : uint32_t(lt.offset[SL]);
+  const uint32_t s_nodes = MODE >= 2 ? 0u : uint32_t(lt.offset[SL]);
   K* s_keys = reinterpret_cast<K*>(smem);
   uint32_t* s_hi = reinterpret_cast<uint32_t*>(smem);
   uint32_t* s_lo = s_hi + s_nodes * FP;
@@ -122,6 +122,9 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
     // directory: [M_T (dcount keys) | 2^dbits x (u16 lo, u16 hi)]
     const uint32_t words = (lt.dcount * uint32_t(sizeof(K)) + (4u << lt.dbits)) / 4;
     for (uint32_t i = threadIdx.x; i < words; i += THREADS) s_hi[i] = __ldg(dirbuf + i);
+  } else if constexpr (MODE == 3) {
+    // small batches: the directory is read from L2 in place (staging 96 KB per
+    // CTA would dominate a launch that serves only a few warp rounds)
   } else {
     for (uint32_t i = threadIdx.x; i < s_nodes * F; i += THREADS) {
       const K key = __ldg(reinterpret_cast<const K*>(inner) + i);
@@ -135,7 +138,10 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
     }
   }
   __syncthreads();
-  const uint32_t* s_dir = reinterpret_cast<const uint32_t*>(smem + lt.dcount * sizeof(K));
+  const K* d_M = MODE == 3 ? reinterpret_cast<const K*>(dirbuf) : s_keys;
+  const uint32_t* d_dir = MODE == 3 ? reinterpret_cast<const uint32_t*>(reinterpret_cast<const uint8_t*>(dirbuf) +
+                                                                         lt.dcount * sizeof(K))
+                                    : reinterpret_cast<const uint32_t*>(smem + lt.dcount * sizeof(K));
 
   const int lane = threadIdx.x & 31;
   const int g = lane / C::G, k = lane % C::G;
@@ -148,7 +154,7 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
   // are loaded while this round walks the tree (their HBM latency was the
   // largest single stall, profiles/r01_c2_v11_*).
   K nextq[QPL];
-  if constexpr (MODE == 2) {
+  if constexpr (MODE >= 2) {
 #pragma unroll
     for (int u = 0; u < QPL; ++u) {
       const uint64_t i = warp * ROUND + uint64_t(u) * 32 + lane;
@@ -162,7 +168,7 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
     uint32_t mynode[QPL];
 #pragma unroll
     for (int u = 0; u < QPL; ++u) {
-      if constexpr (MODE == 2) {
+      if constexpr (MODE >= 2) {
         myq[u] = nextq[u];
         const uint64_t i = (rd + nwarps) * ROUND + uint64_t(u) * 32 + lane;
         nextq[u] = (rd + nwarps < rounds && i < m) ? ldcs(queries + i) : key_max<K>();
@@ -172,15 +178,15 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
       }
       mynode[u] = 0;
     }
-    if constexpr (MODE == 2) {
+    if constexpr (MODE >= 2) {
       // level-T node = lower_bound(M_T, q), narrowed by the prefix directory
 #pragma unroll
       for (int u = 0; u < QPL; ++u) {
-        const uint32_t e = s_dir[uint32_t(myq[u] >> (8 * sizeof(K) - lt.dbits))];
+        const uint32_t e = d_dir[uint32_t(myq[u] >> (8 * sizeof(K) - lt.dbits))];
         uint32_t lo = e & 0xFFFFu, hi = e >> 16;
         while (lo < hi) {
           const uint32_t mid = (lo + hi) >> 1;
-          if (s_keys[mid] < myq[u]) lo = mid + 1; else hi = mid;
+          if (d_M[mid] < myq[u]) lo = mid + 1; else hi = mid;
         }
         mynode[u] = lo;
       }
@@ -337,11 +343,11 @@ struct Launch {
     // the L2-resident budget are read as whole nodes (see the kernel).
     lt.full_mask = 0;
     size_t smem;
-    if (MODE == 2) {
+    if (MODE >= 2) {
       lt.SL = t->dir_T;
       lt.dcount = t->dir_count;
       lt.dbits = t->dir_bits;
-      smem = t->dir_bytes;
+      smem = MODE == 2 ? t->dir_bytes : 0;
     } else {
       lt.SL = smem_levels(t, t->cfg.smem_budget ? t->cfg.smem_budget : kDefaultSmemBudget);
       lt.dcount = 0;
@@ -367,8 +373,16 @@ struct Launch {
         if (C::HAS_IDX && cum > budget && d < 32) lt.full_mask |= 1u << d;
       }
     }
+    // occupancy of this instantiation for this smem size (cached: the query costs
+    // microseconds, which dominate small batches)
+    static size_t occ_smem = ~size_t(0);
+    static int occ_cached = 0;
     int occ = 0;
-    HBT_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, THREADS, smem));
+    if (occ_smem != smem) {
+      HBT_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_cached, kern, THREADS, smem));
+      occ_smem = smem;
+    }
+    occ = occ_cached;
     if (t->cfg.ctas_per_sm && int(t->cfg.ctas_per_sm) < occ) occ = int(t->cfg.ctas_per_sm);
     if (occ < 1) occ = 1;
     const uint64_t rounds = (m + 32 * QPL - 1) / (32 * QPL);
@@ -411,6 +425,8 @@ struct Launch {
     const uint32_t qpl = t->cfg.qpl ? t->cfg.qpl : 1;
     // 256-byte nodes (u64, F = 32) need more registers than a 1024-thread CTA allows
     const uint32_t th = t->cfg.threads ? t->cfg.threads : (C::NODE_BYTES > 128 ? 512 : 1024);
+    // small batches read the directory in place (no 96 KB staging per CTA)
+    if (t->cfg.mode == 3 || (t->cfg.mode == 2 && m <= t->cfg.small_batch)) return run_t<1, 1024, 3>(t, q, m, pf, v, b, s);
     if (t->cfg.mode == 2) {
       if (th == 512) return run_t<1, 512, 2>(t, q, m, pf, v, b, s);
       return qpl == 2 ? run_t<2, 1024, 2>(t, q, m, pf, v, b, s) : run_t<1, 1024, 2>(t, q, m, pf, v, b, s);

@@ -647,8 +647,13 @@ int search_v2_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf,
     HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
     attr = true;
   }
-  int occ = 0;
-  HBT_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, THREADS, smem));
+  static size_t occ_smem = ~size_t(0);
+  static int occ_cached = 0;
+  if (occ_smem != smem) {
+    HBT_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_cached, kern, THREADS, smem));
+    occ_smem = smem;
+  }
+  int occ = occ_cached;
   if (t->cfg.ctas_per_sm && int(t->cfg.ctas_per_sm) < occ) occ = int(t->cfg.ctas_per_sm);
   if (occ < 1) occ = 1;
   const uint64_t rounds = (m + 32 * QPL - 1) / (32 * QPL);
