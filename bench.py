@@ -336,8 +336,14 @@ def run_hbt(args):
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
         traffic = json.load(open(tp)).get(args.config)
+    traffic_bytes = traffic.get("dram_bytes_per_launch") if isinstance(traffic, dict) else None
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-            "frac": round(achieved / peak, 4), "traffic": traffic,
+            "frac": round(achieved / peak, 4), "traffic": traffic_bytes,
+            "traffic_source": traffic.get("source") if isinstance(traffic, dict) else None,
+            # measured DRAM bytes of one launch (ncu, steady state) over this run's launch time:
+            # how busy HBM actually is (random 32 B sector misses move whole DRAM lines)
+            "traffic_gbs": round(traffic_bytes / t_kernel / 1e9, 1) if traffic_bytes and not args.range_k else None,
+            "traffic_frac": round(traffic_bytes / t_kernel / 1e9 / peak, 4) if traffic_bytes and not args.range_k else None,
             "bytes_per_query_model": round(mdl["hbm_bytes_per_query"], 2), "peak_source": peak_src,
             "model": "ideal static L2 cache of %d B (SURVEY §8d)%s" % (
                 l2_size, "; Zipf modelled as uniform (upper bound on bytes)" if args.config == "c5" else "")}
