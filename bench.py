@@ -334,7 +334,7 @@ def run_hbt(args):
     achieved = mdl["hbm_bytes_per_query"] * m / t_kernel / 1e9
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tp):
+    if os.path.exists(tp) and not (args.config == "c4" and world > 1):  # measured on one GPU
         traffic = json.load(open(tp)).get(args.config)
     traffic_bytes = traffic.get("dram_bytes_per_launch") if isinstance(traffic, dict) else None
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
