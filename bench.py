@@ -192,7 +192,7 @@ def make_work(cfg_name, rank, world, args):
     del keys, vals
     tree.set_search_config(smem_bytes=args.smem, threads_per_cta=args.threads, queries_per_lane=args.qpl,
                            smem_mode=args.smem_mode, carveout=args.carveout)
-    if args.l2_persist is not None and c["layout"] == "implicit":
+    if args.l2_persist is not None:
         tree.set_param("l2_persist", args.l2_persist)
     if args.l2_levels is not None and c["layout"] == "implicit":
         tree.set_param("l2_levels_bytes", args.l2_levels)

@@ -18,6 +18,8 @@
 #include <cub/device/device_scan.cuh>
 #include <cub/device/device_select.cuh>
 
+#include <algorithm>
+
 #include "hbt_internal.cuh"
 
 namespace hbt {
@@ -660,8 +662,32 @@ int search_v2_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf,
   uint64_t grid = uint64_t(t->num_sms) * occ;
   const uint64_t need = (rounds + THREADS / 32 - 1) / (THREADS / 32);
   if (need < grid) grid = need ? need : 1;
-  kern<<<unsigned(grid), THREADS, smem, s>>>(rv, rd, (const uint32_t*)r.d_dir, r.d_chain, (const K*)q, m, pf, (K*)v);
-  HBT_CUDA_TRY(cudaGetLastError());
+  cudaLaunchConfig_t lc = {};
+  lc.gridDim = dim3(unsigned(grid));
+  lc.blockDim = dim3(THREADS);
+  lc.dynamicSmemBytes = smem;
+  lc.stream = s;
+  cudaLaunchAttribute la[1];
+  lc.attrs = la;
+  lc.numAttrs = 0;
+  if (t->cfg.l2_persist) {
+    // keep the last level's index sectors (one 32 B sector per big leaf) resident
+    static uint64_t limit_set = 0;
+    const uint64_t win = std::min<uint64_t>(t->cfg.l2_persist, r.pool * 32);
+    if (limit_set < win) {
+      HBT_CUDA_TRY(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, win));
+      limit_set = win;
+    }
+    la[0].id = cudaLaunchAttributeAccessPolicyWindow;
+    la[0].val.accessPolicyWindow.base_ptr = r.d_lidx;
+    la[0].val.accessPolicyWindow.num_bytes = win;
+    la[0].val.accessPolicyWindow.hitRatio = 1.0f;
+    la[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    la[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    lc.numAttrs = 1;
+  }
+  HBT_CUDA_TRY(cudaLaunchKernelEx(&lc, kern, rv, rd, (const uint32_t*)r.d_dir, (const uint32_t*)r.d_chain, (const K*)q,
+                                  m, pf, (K*)v));
   return HBT_OK;
 }
 
