@@ -189,6 +189,39 @@ def zipf_ranks(m: int, n: int, theta: float, seed: int, start: int = 0):
     return out
 
 
+def skew_values(kind: str, m: int, width: int, seed: int, n_ranks: int = 1 << 20, start: int = 0):
+    """Query VALUES drawn from the paper's skewed distributions on [0, 1] and
+    mapped linearly to [0, MAX] (reading R15/R20 in DESIGN.md):
+      normal  N(mu = 0.5, sigma^2 = 0.125) (Box-Muller), clipped to [0, 1]
+      gamma   Gamma(k = 3, theta = 3) = -3 ln(u1 u2 u3), divided by 30, clipped to [0, 1]
+      zipf    Zipf(alpha = 2) rank r in [1, n_ranks] -> (r - 1) / n_ranks  (clustered at 0)
+      uniform u
+    Counter-based: sample j draws unit_doubles(3j + t, seed) for t = 0, 1, 2."""
+    j = np.arange(start, start + m, dtype=np.uint64) * np.uint64(3)
+    u1 = unit_doubles(j, seed)
+    u2 = unit_doubles(j + np.uint64(1), seed)
+    u3 = unit_doubles(j + np.uint64(2), seed)
+    if kind == "normal":
+        x = 0.5 + np.sqrt(0.125) * np.sqrt(-2.0 * np.log1p(-u1)) * np.cos(2.0 * np.pi * u2)
+    elif kind == "gamma":
+        x = -3.0 * (np.log1p(-u1) + np.log1p(-u2) + np.log1p(-u3)) / 30.0
+    elif kind == "zipf":
+        x = (zipf_ranks(m, n_ranks, 2.0, seed, start) - 1).astype(np.float64) / n_ranks
+    elif kind == "uniform":
+        x = u1
+    else:
+        raise ValueError(kind)
+    x = np.clip(x, 0.0, 1.0)
+    mx = float((1 << (8 * width)) - 1)
+    # x * MAX in float64, then exact integer conversion (values >= 2^63 via the high half)
+    v = x * mx
+    with np.errstate(over="ignore", invalid="ignore"):
+        out = np.where(v >= 2.0 ** 63, (np.minimum(v, 2.0 ** 64 - 4096.0) - 2.0 ** 63).astype(np.uint64)
+                       + np.uint64(1 << 63), np.minimum(v, 2.0 ** 63 - 1).astype(np.uint64))
+    out = np.where(x >= 1.0, np.uint64((1 << (8 * width)) - 1), out)  # x = 1 maps to MAX exactly
+    return out.astype(dtype_of(width))
+
+
 def stratified_keys(n: int, seed: int, start: int = 0):
     """c4: K_i = (i << 33) | (mix64(i ^ seed) & (2^33-1)); sorted and distinct for i < 2^31."""
     i = np.arange(start, start + n, dtype=np.uint64)

@@ -23,6 +23,26 @@ void set_error(const char* fmt, ...) {
   g_err = buf;
 }
 
+cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t s) {
+  static thread_local int configured = -1;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (configured != dev) {
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+      uint64_t keep = 4ull << 30;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+    }
+    configured = dev;
+  }
+  *p = nullptr;
+  return cudaMallocAsync(p, bytes ? bytes : 1, s);
+}
+
+void scratch_free(void* p, cudaStream_t s) {
+  if (p) cudaFreeAsync(p, s);
+}
+
 static bool is_device_ptr(const void* p) {
   if (!p) return false;
   cudaPointerAttributes a;

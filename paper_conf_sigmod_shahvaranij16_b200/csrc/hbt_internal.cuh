@@ -26,6 +26,13 @@ void set_error(const char* fmt, ...);
 
 static inline uint64_t ceil_div_u64(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
 
+// Scratch of builds and updates comes from the device's stream-ordered pool
+// (cudaMallocAsync): after the first use, repeated updates allocate without
+// cudaMalloc / cudaFree (which synchronise the device).  The pool keeps up to
+// 4 GiB between calls (api.cu sets the release threshold once).
+cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t s);
+void scratch_free(void* p, cudaStream_t s);
+
 // Level table passed by value to the search kernels (root-first, node units).
 struct LevelTable {
   uint64_t offset[HBT_MAX_LEVELS + 1];

@@ -212,7 +212,8 @@ int sort_dedupe_t(const void* keys, const void* values, uint64_t n, void** out_k
   size_t tb = 0, tb2 = 0;
   int rc = HBT_OK;
   auto fail = [&](int code) {
-    cudaFree(sk); cudaFree(sv); cudaFree(kd); cudaFree(vd); cudaFree(flags); cudaFree(tmp); cudaFree(d_nsel);
+    scratch_free(sk, s); scratch_free(sv, s); scratch_free(kd, s); scratch_free(vd, s); scratch_free(flags, s);
+    scratch_free(tmp, s); scratch_free(d_nsel, s);
     return code;
   };
 #define TRY(x)                                                                          \
@@ -223,30 +224,30 @@ int sort_dedupe_t(const void* keys, const void* values, uint64_t n, void** out_k
       return fail(_e == cudaErrorMemoryAllocation ? HBT_ENOMEM : HBT_ECUDA);            \
     }                                                                                   \
   } while (0)
-  TRY(cudaMalloc(&sk, n * sizeof(K)));
-  TRY(cudaMalloc(&sv, n * sizeof(K)));
+  TRY(scratch_alloc((void**)&sk, n * sizeof(K), s));
+  TRY(scratch_alloc((void**)&sv, n * sizeof(K), s));
   TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb, (const K*)keys, sk, (const K*)values, sv, n, 0,
                                       int(8 * sizeof(K)), s));
   TRY(cub::DeviceSelect::Flagged(nullptr, tb2, sk, flags, kd, d_nsel, int64_t(n), s));
   if (tb2 > tb) tb = tb2;
-  TRY(cudaMalloc(&tmp, tb));
+  TRY(scratch_alloc((void**)&tmp, tb, s));
   // Stable LSD radix sort: equal keys keep input order, so the last element of
   // each run is the key's last occurrence (dedupe-last-wins, reading R4).
   TRY(cub::DeviceRadixSort::SortPairs(tmp, tb, (const K*)keys, sk, (const K*)values, sv, n, 0,
                                       int(8 * sizeof(K)), s));
-  TRY(cudaMalloc(&flags, n));
-  TRY(cudaMalloc(&d_nsel, sizeof(int64_t)));
+  TRY(scratch_alloc((void**)&flags, n, s));
+  TRY(scratch_alloc((void**)&d_nsel, sizeof(int64_t), s));
   last_of_run_flags<K><<<grid_for(n), 256, 0, s>>>(sk, n, flags);
   TRY(cudaGetLastError());
-  TRY(cudaMalloc(&kd, n * sizeof(K)));
-  TRY(cudaMalloc(&vd, n * sizeof(K)));
+  TRY(scratch_alloc((void**)&kd, n * sizeof(K), s));
+  TRY(scratch_alloc((void**)&vd, n * sizeof(K), s));
   TRY(cub::DeviceSelect::Flagged(tmp, tb, sk, flags, kd, d_nsel, int64_t(n), s));
   TRY(cub::DeviceSelect::Flagged(tmp, tb, sv, flags, vd, d_nsel, int64_t(n), s));
   int64_t h_nsel = 0;
   TRY(cudaMemcpyAsync(&h_nsel, d_nsel, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
   TRY(cudaStreamSynchronize(s));
 #undef TRY
-  cudaFree(sk); cudaFree(sv); cudaFree(flags); cudaFree(tmp); cudaFree(d_nsel);
+  scratch_free(sk, s); scratch_free(sv, s); scratch_free(flags, s); scratch_free(tmp, s); scratch_free(d_nsel, s);
   *out_k = kd;
   *out_v = vd;
   *nd = uint64_t(h_nsel);
@@ -340,8 +341,9 @@ int implicit_update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   void* tmp = nullptr;
   size_t tb = 0, tb2 = 0;
   auto cleanup = [&]() {
-    cudaFree(ck); cudaFree(sk); cudaFree(base_v); cudaFree(mv); cudaFree(kd); cudaFree(vd);
-    cudaFree(idx); cudaFree(sidx); cudaFree(flags); cudaFree(d_nsel); cudaFree(tmp);
+    scratch_free(ck, s); scratch_free(sk, s); scratch_free(base_v, s); scratch_free(mv, s); scratch_free(kd, s);
+    scratch_free(vd, s); scratch_free(idx, s); scratch_free(sidx, s); scratch_free(flags, s); scratch_free(d_nsel, s);
+    scratch_free(tmp, s);
   };
 #define TRY(x)                                                                          \
   do {                                                                                  \
@@ -352,14 +354,14 @@ int implicit_update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
       return _e == cudaErrorMemoryAllocation ? HBT_ENOMEM : HBT_ECUDA;                  \
     }                                                                                   \
   } while (0)
-  TRY(cudaMalloc(&ck, total * sizeof(K)));
-  TRY(cudaMalloc(&sk, total * sizeof(K)));
-  TRY(cudaMalloc(&base_v, (nb ? nb : 1) * sizeof(K)));
-  TRY(cudaMalloc(&mv, total * sizeof(K)));
-  TRY(cudaMalloc(&idx, total * sizeof(uint32_t)));
-  TRY(cudaMalloc(&sidx, total * sizeof(uint32_t)));
-  TRY(cudaMalloc(&flags, total));
-  TRY(cudaMalloc(&d_nsel, sizeof(int64_t)));
+  TRY(scratch_alloc((void**)&ck, total * sizeof(K), s));
+  TRY(scratch_alloc((void**)&sk, total * sizeof(K), s));
+  TRY(scratch_alloc((void**)&base_v, (nb ? nb : 1) * sizeof(K), s));
+  TRY(scratch_alloc((void**)&mv, total * sizeof(K), s));
+  TRY(scratch_alloc((void**)&idx, total * sizeof(uint32_t), s));
+  TRY(scratch_alloc((void**)&sidx, total * sizeof(uint32_t), s));
+  TRY(scratch_alloc((void**)&flags, total, s));
+  TRY(scratch_alloc((void**)&d_nsel, sizeof(int64_t), s));
   if (nb) {
     unpack_leaf_lines<K><<<grid_for(nb), 256, 0, s>>>((const K*)t->d_leaf, nb, ck, base_v);
     TRY(cudaGetLastError());
@@ -370,14 +372,14 @@ int implicit_update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb, ck, sk, idx, sidx, total, 0, int(8 * sizeof(K)), s));
   TRY(cub::DeviceSelect::Flagged(nullptr, tb2, sk, flags, ck, d_nsel, int64_t(total), s));
   if (tb2 > tb) tb = tb2;
-  TRY(cudaMalloc(&tmp, tb));
+  TRY(scratch_alloc((void**)&tmp, tb, s));
   TRY(cub::DeviceRadixSort::SortPairs(tmp, tb, ck, sk, idx, sidx, total, 0, int(8 * sizeof(K)), s));
   merge_flags<K><<<grid_for(total), 256, 0, s>>>(sk, sidx, total, nb, b->ops, flags);
   TRY(cudaGetLastError());
   merge_gather_values<K><<<grid_for(total), 256, 0, s>>>(sidx, total, nb, base_v, (const K*)b->values, mv);
   TRY(cudaGetLastError());
-  TRY(cudaMalloc(&kd, total * sizeof(K)));
-  TRY(cudaMalloc(&vd, total * sizeof(K)));
+  TRY(scratch_alloc((void**)&kd, total * sizeof(K), s));
+  TRY(scratch_alloc((void**)&vd, total * sizeof(K), s));
   TRY(cub::DeviceSelect::Flagged(tmp, tb, sk, flags, kd, d_nsel, int64_t(total), s));
   TRY(cub::DeviceSelect::Flagged(tmp, tb, mv, flags, vd, d_nsel, int64_t(total), s));
   int64_t h_nsel = 0;
@@ -435,8 +437,9 @@ int implicit_build(hbt_tree* t, const void* keys, const void* values, uint64_t n
   rc = sort_dedupe(t->width, keys, values, n, &kd, &vd, &nd, s);
   if (rc != HBT_OK) return rc;
   rc = implicit_build_sorted(t, kd, vd, nd, s);
-  cudaFree(kd);
-  cudaFree(vd);
+  scratch_free(kd, s);
+  scratch_free(vd, s);
+  cudaStreamSynchronize(s);
   return rc;
 }
 

@@ -789,8 +789,8 @@ int rebuild_upper(hbt_tree* t, cudaStream_t s) {
   }
   if (U == 0) return HBT_OK;
   K *mx_a = nullptr, *mx_b = nullptr;
-  HBT_CUDA_TRY(cudaMalloc(&mx_a, r.nchain * sizeof(K)));
-  HBT_CUDA_TRY(cudaMalloc(&mx_b, (unodes[0] + 1) * sizeof(K)));
+  HBT_CUDA_TRY(scratch_alloc((void**)&mx_a, r.nchain * sizeof(K), s));
+  HBT_CUDA_TRY(scratch_alloc((void**)&mx_b, (unodes[0] + 1) * sizeof(K), s));
   chain_leaf_max<K><<<grid_for(r.nchain), 256, 0, s>>>((const K*)r.d_leaf, r.d_count, r.d_chain, r.nchain, F, mx_a);
   uint64_t below = r.nchain;
   for (uint32_t u = 0; u < U; ++u) {
@@ -801,9 +801,9 @@ int rebuild_upper(hbt_tree* t, cudaStream_t s) {
     below = unodes[u];
   }
   cudaError_t e = cudaGetLastError();
+  scratch_free(mx_a, s);
+  scratch_free(mx_b, s);
   cudaStreamSynchronize(s);
-  cudaFree(mx_a);
-  cudaFree(mx_b);
   if (e != cudaSuccess) { set_error("rebuild_upper: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
   return HBT_OK;
 }
@@ -870,7 +870,7 @@ int build_t(hbt_tree* t, const void* keys, const void* values, uint64_t n, cudaS
   if (rc != HBT_OK) return rc;
   const uint64_t nb = nd == 0 ? 1 : ceil_div_u64(nd, r.b);
   rc = alloc_pool<K>(t, nb + nb / 8 + 16);
-  if (rc != HBT_OK) { cudaFree(kd); cudaFree(vd); return rc; }
+  if (rc != HBT_OK) { scratch_free(kd, s); scratch_free(vd, s); return rc; }
   r.pool = nb;
   r.nchain = nb;
   r.root_leaf = 0;
@@ -880,9 +880,9 @@ int build_t(hbt_tree* t, const void* keys, const void* values, uint64_t n, cudaS
                                                      (K*)r.d_lidx);
   iota_chain<<<grid_for(nb), 256, 0, s>>>(r.d_chain, nb);
   cudaError_t e = cudaGetLastError();
+  scratch_free(kd, s);
+  scratch_free(vd, s);
   cudaStreamSynchronize(s);
-  cudaFree(kd);
-  cudaFree(vd);
   if (e != cudaSuccess) { set_error("regular build: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
   int rc2 = rebuild_upper<K>(t, s);
   return rc2 != HBT_OK ? rc2 : rebuild_dir<K>(t, s);
@@ -1158,9 +1158,11 @@ __global__ void chain_count_sum(const uint32_t* __restrict__ chain, uint64_t nch
   if (local) atomicAdd(sum, local);
 }
 
+// Update scratch from the stream-ordered pool (freed on the update's stream).
 struct DevBuf {
   void* p = nullptr;
-  ~DevBuf() { cudaFree(p); }
+  cudaStream_t s = nullptr;
+  ~DevBuf() { scratch_free(p, s); }
   template <typename T> T* as() { return static_cast<T*>(p); }
 };
 
@@ -1172,15 +1174,24 @@ int update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   if (m0 >= (1ull << 32)) { set_error("batch too large"); return HBT_EUNSUPPORTED; }
   // 1. sort ops by key (stable), last op per key wins
   DevBuf sk, sidx, idx, flags, tmp, dk, didx, dv, dop, nsel;
-  HBT_CUDA_TRY(cudaMalloc(&sk.p, m0 * sizeof(K)));
-  HBT_CUDA_TRY(cudaMalloc(&idx.p, m0 * 4));
-  HBT_CUDA_TRY(cudaMalloc(&sidx.p, m0 * 4));
-  HBT_CUDA_TRY(cudaMalloc(&flags.p, m0));
-  HBT_CUDA_TRY(cudaMalloc(&dk.p, m0 * sizeof(K)));
-  HBT_CUDA_TRY(cudaMalloc(&didx.p, m0 * 4));
-  HBT_CUDA_TRY(cudaMalloc(&dv.p, m0 * sizeof(K)));
-  HBT_CUDA_TRY(cudaMalloc(&dop.p, m0));
-  HBT_CUDA_TRY(cudaMalloc(&nsel.p, 8));
+  sk.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&sk.p, m0 * sizeof(K), s));
+  idx.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&idx.p, m0 * 4, s));
+  sidx.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&sidx.p, m0 * 4, s));
+  flags.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&flags.p, m0, s));
+  dk.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&dk.p, m0 * sizeof(K), s));
+  didx.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&didx.p, m0 * 4, s));
+  dv.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&dv.p, m0 * sizeof(K), s));
+  dop.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&dop.p, m0, s));
+  nsel.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&nsel.p, 8, s));
   iota_u32<<<grid_for(m0), 256, 0, s>>>(idx.as<uint32_t>(), m0);
   size_t tb = 0, tb2 = 0;
   HBT_CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb, (const K*)b->keys, sk.as<K>(), idx.as<uint32_t>(),
@@ -1188,7 +1199,8 @@ int update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   HBT_CUDA_TRY(cub::DeviceSelect::Flagged(nullptr, tb2, sk.as<K>(), flags.as<uint8_t>(), dk.as<K>(),
                                           nsel.as<int64_t>(), int64_t(m0), s));
   if (tb2 > tb) tb = tb2;
-  HBT_CUDA_TRY(cudaMalloc(&tmp.p, tb));
+  tmp.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&tmp.p, tb, s));
   HBT_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp.p, tb, (const K*)b->keys, sk.as<K>(), idx.as<uint32_t>(),
                                                sidx.as<uint32_t>(), m0, 0, int(8 * sizeof(K)), s));
   last_of_run<K><<<grid_for(m0), 256, 0, s>>>(sk.as<K>(), m0, flags.as<uint8_t>());
@@ -1204,49 +1216,64 @@ int update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
                                             dop.as<uint8_t>());
   // 2. locate each op's big leaf through the pre-update tree
   DevBuf leaf_of, start, incl, seg_off, seg_leaf, seg_delta, lb, ins, insx, new_cnt, extra, new_base, dirty;
-  HBT_CUDA_TRY(cudaMalloc(&leaf_of.p, m * 4));
+  leaf_of.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&leaf_of.p, m * 4, s));
   const uint32_t root_leaf = r.root_leaf;
   locate_leaf<K><<<grid_for(m), 256, 0, s>>>(dk.as<K>(), m, (const K*)r.d_ukeys, (const K*)r.d_uidx, r.d_urefs,
                                              r.U ? r.uoff[r.U] - 1 : 0, r.U, root_leaf, F, leaf_of.as<uint32_t>());
   // 3. segments of ops per leaf (ops are in key order, so are their leaves)
-  HBT_CUDA_TRY(cudaMalloc(&start.p, m * 4));
-  HBT_CUDA_TRY(cudaMalloc(&incl.p, m * 4));
+  start.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&start.p, m * 4, s));
+  incl.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&incl.p, m * 4, s));
   segment_flags<<<grid_for(m), 256, 0, s>>>(leaf_of.as<uint32_t>(), m, start.as<uint32_t>());
   tb2 = 0;
   HBT_CUDA_TRY(cub::DeviceScan::InclusiveSum(nullptr, tb2, start.as<uint32_t>(), incl.as<uint32_t>(), m, s));
   DevBuf tmp2;
-  HBT_CUDA_TRY(cudaMalloc(&tmp2.p, tb2 + 256));
+  tmp2.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&tmp2.p, tb2 + 256, s));
   HBT_CUDA_TRY(cub::DeviceScan::InclusiveSum(tmp2.p, tb2, start.as<uint32_t>(), incl.as<uint32_t>(), m, s));
   uint32_t nseg32 = 0;
   HBT_CUDA_TRY(cudaMemcpyAsync(&nseg32, incl.as<uint32_t>() + (m - 1), 4, cudaMemcpyDeviceToHost, s));
   HBT_CUDA_TRY(cudaStreamSynchronize(s));
   const uint64_t nseg = nseg32;
-  HBT_CUDA_TRY(cudaMalloc(&seg_off.p, (nseg + 1) * 4));
-  HBT_CUDA_TRY(cudaMalloc(&seg_leaf.p, nseg * 4));
-  HBT_CUDA_TRY(cudaMalloc(&seg_delta.p, nseg * 4));
+  seg_off.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&seg_off.p, (nseg + 1) * 4, s));
+  seg_leaf.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&seg_leaf.p, nseg * 4, s));
+  seg_delta.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&seg_delta.p, nseg * 4, s));
   HBT_CUDA_TRY(cudaMemsetAsync(seg_delta.p, 0, nseg * 4, s));
   segment_tables<<<grid_for(m), 256, 0, s>>>(leaf_of.as<uint32_t>(), incl.as<uint32_t>(), m, seg_off.as<uint32_t>(),
                                              seg_leaf.as<uint32_t>(), r.d_seg_of_leaf);
   // 4. classify ops against their leaf; new counts; new pool indices (key order)
-  HBT_CUDA_TRY(cudaMalloc(&lb.p, m * 4));
-  HBT_CUDA_TRY(cudaMalloc(&ins.p, (m + 1) * 4));
-  HBT_CUDA_TRY(cudaMalloc(&insx.p, (m + 1) * 4));
+  lb.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&lb.p, m * 4, s));
+  ins.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&ins.p, (m + 1) * 4, s));
+  insx.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&insx.p, (m + 1) * 4, s));
   HBT_CUDA_TRY(cudaMemsetAsync(ins.p, 0, (m + 1) * 4, s));
   op_classify<K><<<grid_for(m), 256, 0, s>>>(dk.as<K>(), dop.as<uint8_t>(), m, leaf_of.as<uint32_t>(),
                                              incl.as<uint32_t>(), (const K*)r.d_leaf, r.d_count, F, lb.as<uint32_t>(),
                                              ins.as<uint32_t>(), seg_delta.as<int>());
   HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb2, ins.as<uint32_t>(), insx.as<uint32_t>(), m + 1, s));
   DevBuf tmp3;
-  HBT_CUDA_TRY(cudaMalloc(&tmp3.p, tb2 + 256));
+  tmp3.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&tmp3.p, tb2 + 256, s));
   HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp3.p, tb2, ins.as<uint32_t>(), insx.as<uint32_t>(), m + 1, s));
-  HBT_CUDA_TRY(cudaMalloc(&new_cnt.p, nseg * 4));
-  HBT_CUDA_TRY(cudaMalloc(&extra.p, nseg * 4));
-  HBT_CUDA_TRY(cudaMalloc(&new_base.p, (nseg + 1) * 4));
+  new_cnt.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&new_cnt.p, nseg * 4, s));
+  extra.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&extra.p, nseg * 4, s));
+  new_base.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&new_base.p, (nseg + 1) * 4, s));
   segment_counts<<<grid_for(nseg), 256, 0, s>>>(seg_leaf.as<uint32_t>(), seg_delta.as<int>(), nseg, r.d_count, B,
                                                 new_cnt.as<uint32_t>(), extra.as<uint32_t>());
   DevBuf tmp4;
   HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb2, extra.as<uint32_t>(), new_base.as<uint32_t>(), nseg + 0, s));
-  HBT_CUDA_TRY(cudaMalloc(&tmp4.p, tb2 + 256));
+  tmp4.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&tmp4.p, tb2 + 256, s));
   HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp4.p, tb2, extra.as<uint32_t>(), new_base.as<uint32_t>(), nseg, s));
   uint32_t last_base = 0, last_extra = 0;
   HBT_CUDA_TRY(cudaMemcpyAsync(&last_base, new_base.as<uint32_t>() + nseg - 1, 4, cudaMemcpyDeviceToHost, s));
@@ -1259,7 +1286,8 @@ int update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   int rc = grow_pool<K>(t, old_pool + n_new, s);
   if (rc != HBT_OK) return rc;
   r.pool = old_pool + n_new;
-  HBT_CUDA_TRY(cudaMalloc(&dirty.p, r.pool));
+  dirty.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&dirty.p, r.pool, s));
   HBT_CUDA_TRY(cudaMemsetAsync(dirty.p, 0, r.pool, s));
   // 5. merge + split + pad, one warp per affected leaf
   {
@@ -1273,20 +1301,24 @@ int update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   }
   // 6. new chain (key order): every old position expands to its parts
   DevBuf parts, ppos, nchain_buf;
-  HBT_CUDA_TRY(cudaMalloc(&parts.p, (r.nchain + 1) * 4));
-  HBT_CUDA_TRY(cudaMalloc(&ppos.p, (r.nchain + 1) * 4));
+  parts.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&parts.p, (r.nchain + 1) * 4, s));
+  ppos.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&ppos.p, (r.nchain + 1) * 4, s));
   chain_parts<<<grid_for(r.nchain), 256, 0, s>>>(r.d_chain, r.nchain, r.d_seg_of_leaf, new_cnt.as<uint32_t>(), B,
                                                  parts.as<uint32_t>());
   DevBuf tmp5;
   HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb2, parts.as<uint32_t>(), ppos.as<uint32_t>(), r.nchain, s));
-  HBT_CUDA_TRY(cudaMalloc(&tmp5.p, tb2 + 256));
+  tmp5.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&tmp5.p, tb2 + 256, s));
   HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp5.p, tb2, parts.as<uint32_t>(), ppos.as<uint32_t>(), r.nchain, s));
   uint32_t lp = 0, lpart = 0;
   HBT_CUDA_TRY(cudaMemcpyAsync(&lp, ppos.as<uint32_t>() + r.nchain - 1, 4, cudaMemcpyDeviceToHost, s));
   HBT_CUDA_TRY(cudaMemcpyAsync(&lpart, parts.as<uint32_t>() + r.nchain - 1, 4, cudaMemcpyDeviceToHost, s));
   HBT_CUDA_TRY(cudaStreamSynchronize(s));
   const uint64_t new_nchain = uint64_t(lp) + lpart;
-  HBT_CUDA_TRY(cudaMalloc(&nchain_buf.p, (new_nchain + 1) * 4));
+  nchain_buf.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&nchain_buf.p, (new_nchain + 1) * 4, s));
   chain_write<<<grid_for(r.nchain), 256, 0, s>>>(r.d_chain, r.nchain, r.d_seg_of_leaf, parts.as<uint32_t>(),
                                                  ppos.as<uint32_t>(), new_base.as<uint32_t>(), nchain_buf.as<uint32_t>());
   reset_seg_of_leaf<<<grid_for(nseg), 256, 0, s>>>(seg_leaf.as<uint32_t>(), nseg, r.d_seg_of_leaf);
@@ -1312,7 +1344,8 @@ int update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   // live key count n' = sum of the chain's counts
   {
     DevBuf sum;
-    HBT_CUDA_TRY(cudaMalloc(&sum.p, 8));
+    sum.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&sum.p, 8, s));
     HBT_CUDA_TRY(cudaMemsetAsync(sum.p, 0, 8, s));
     chain_count_sum<<<grid_for(r.nchain), 256, 0, s>>>(r.d_chain, r.nchain, r.d_count, sum.as<unsigned long long>());
     uint64_t nn = 0;

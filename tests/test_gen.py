@@ -79,3 +79,18 @@ def test_update_batch_shape():
     ins = bk[bo == 0].tolist()
     dels = bk[bo == 1].tolist()
     assert not (set(ins) & base) and set(dels) <= base and len(set(dels)) == len(dels)
+
+
+def test_skew_values_moments():
+    """The paper's skewed query distributions before the [0, MAX] mapping."""
+    m = 200000
+    mx = float(2**64 - 1)
+    x = gen.skew_values("normal", m, 8, 5).astype(np.float64) / mx
+    assert abs(x.mean() - 0.5) < 0.01 and abs(x.std() - 0.304) < 0.01  # sigma 0.354 clipped to [0, 1]: 0.304
+    g = gen.skew_values("gamma", m, 8, 6).astype(np.float64) / mx
+    assert abs(g.mean() - 9.0 / 30.0) < 0.01                          # E[Gamma(3,3)] = 9
+    z = gen.skew_values("zipf", m, 8, 7, n_ranks=1 << 20).astype(np.float64) / mx
+    assert (z == 0).mean() > 0.55                                     # rank 1 has p = 1/zeta(2) = 0.61
+    u = gen.skew_values("uniform", m, 4, 8)
+    assert u.dtype == np.uint32 and abs(u.astype(np.float64).mean() / (2**32 - 1) - 0.5) < 0.01
+    assert np.array_equal(gen.skew_values("normal", 100, 8, 5), gen.skew_values("normal", 100, 8, 5))

@@ -250,3 +250,21 @@ def test_presorted_input_fast_path(hbt, width):
     o2 = oracle.ITree.from_pairs(kd2, vd2, 16, width)
     t2 = gpu_build(hbt, kd2, vd2, 16, width)
     assert t2.export(hbt.SEG_LEAF).tobytes() == expected_implicit_bytes(o2, width)[1]
+
+
+@pytest.mark.parametrize("kind", ["normal", "gamma", "zipf", "uniform"])
+def test_skewed_query_values(hbt, kind):
+    """The paper's skew experiment: query values from Normal / Gamma /
+    clustered Zipf on [0, 1] mapped to [0, MAX] — mostly misses, concentrated in
+    a part of the key space; both tree forms vs the oracle."""
+    import gen as g
+    rng = np.random.default_rng(1)
+    k, v = gen_keys(200000, 8, rng)
+    q = g.skew_values(kind, 50000, 8, 99).astype(np.uint64)
+    for layout in ("implicit", "regular"):
+        T = oracle.ITree if layout == "implicit" else oracle.RTree
+        o = T.from_pairs(k, v, 16, 8)
+        t = gpu_build(hbt, k, v, 16, 8, layout=layout)
+        pf, val = gpu_search(t, q, 8)
+        epf, ev = o.search(q)
+        assert np.array_equal(pf, epf) and np.array_equal(val, ev)
