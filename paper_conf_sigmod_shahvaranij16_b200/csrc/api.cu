@@ -58,6 +58,8 @@ static void free_tree(hbt_tree* t) {
   if (!t) return;
   cudaFree(t->d_inner);  // also holds d_inner_idx
   cudaFree(t->d_dir);
+  cudaFree(t->d_sdir);
+  cudaFree(t->d_sdir_full);
   cudaFree(t->d_leaf);
   regular_free(t);
   shard_free(t);
@@ -282,7 +284,7 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "threads" && (value == 0 || value == 256 || value == 512 || value == 1024)) c.threads = uint32_t(value);
   else if (n == "ctas_per_sm" && value >= 0 && value <= 32) c.ctas_per_sm = uint32_t(value);
   else if (n == "qpl" && value >= 0 && value <= 2) c.qpl = uint32_t(value);
-  else if (n == "smem_mode" && value >= 0 && value <= 3) c.mode = uint32_t(value);
+  else if (n == "smem_mode" && value >= 0 && value <= 4) c.mode = uint32_t(value);
   else if (n == "small_batch" && value >= 0) c.small_batch = uint64_t(value);
   else if (n == "carveout" && value >= -1 && value <= 100) c.carveout = int(value);
   else if (n == "l2_persist" && value >= 0) c.l2_persist = uint64_t(value);

@@ -38,8 +38,8 @@ struct LevelTable {
   uint64_t offset[HBT_MAX_LEVELS + 1];
   uint32_t H;   // inner levels
   uint32_t SL;  // levels [0, SL) searched in shared memory (mode 2: = the directory level T)
-  uint32_t dcount;  // mode 2: nodes at level T
-  uint32_t dbits;   // mode 2: directory prefix bits
+  uint32_t dcount;  // mode 2/3: nodes at level T; mode 4: sectors at level T
+  uint32_t dbits;   // mode 2/3/4: directory prefix bits
   uint32_t full_mask;  // bit d: read level d's nodes whole (not index + sector)
 };
 
@@ -155,6 +155,13 @@ struct hbt_tree {
   uint32_t dir_T = 0;       // target level (H = leaf lines)
   uint32_t dir_count = 0;   // nodes at level T
   uint32_t dir_bits = 0;
+  // Sector directory (search mode 4): over the key SECTORS of level T.
+  // d_sdir = [hi 32 bits of Msec (sdir_count u32) | 2^sdir_bits x (u16 lo, u16 hi)];
+  // d_sdir_full = Msec at full width (tie fallback when the high words are equal).
+  void* d_sdir = nullptr;
+  void* d_sdir_full = nullptr;
+  uint64_t sdir_bytes = 0;
+  uint32_t sdir_count = 0, sdir_bits = 0;
   void* d_leaf = nullptr;
   uint64_t L0 = 0;
   uint64_t leaf_bytes = 0;

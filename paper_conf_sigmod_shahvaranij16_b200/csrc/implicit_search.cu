@@ -100,7 +100,8 @@ __device__ __forceinline__ uint32_t count_less16(const V16<K>& v, K q, unsigned 
 template <typename K, int F, int QPL, int THREADS, int MODE>
 __global__ void __launch_bounds__(THREADS)
 implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ inner_idx,
-                       const uint8_t* __restrict__ leaf, const uint32_t* __restrict__ dirbuf, const K* __restrict__ queries, uint64_t m,
+                       const uint8_t* __restrict__ leaf, const uint32_t* __restrict__ dirbuf,
+                       const K* __restrict__ sfull, const K* __restrict__ queries, uint64_t m,
                        uint64_t* __restrict__ out_pf, K* __restrict__ out_v, const LevelTable lt, uint64_t n,
                        uint64_t pos_base) {
   using C = Cfg<K, F>;
@@ -121,6 +122,10 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
   if constexpr (MODE == 2) {
     // directory: [M_T (dcount keys) | 2^dbits x (u16 lo, u16 hi)]
     const uint32_t words = (lt.dcount * uint32_t(sizeof(K)) + (4u << lt.dbits)) / 4;
+    for (uint32_t i = threadIdx.x; i < words; i += THREADS) s_hi[i] = __ldg(dirbuf + i);
+  } else if constexpr (MODE == 4) {
+    // sector directory: [hi words of Msec (dcount u32) | 2^dbits x (u16 lo, u16 hi)]
+    const uint32_t words = lt.dcount + (1u << lt.dbits);
     for (uint32_t i = threadIdx.x; i < words; i += THREADS) s_hi[i] = __ldg(dirbuf + i);
   } else if constexpr (MODE == 3) {
     // small batches: the directory is read from L2 in place (staging 96 KB per
@@ -166,8 +171,10 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
     // ---- phase 1: one lane per query; coalesced query loads
     K myq[QPL];
     uint32_t mynode[QPL];
+    uint32_t mysec[QPL];
 #pragma unroll
     for (int u = 0; u < QPL; ++u) {
+      mysec[u] = 0;
       if constexpr (MODE >= 2) {
         myq[u] = nextq[u];
         const uint64_t i = (rd + nwarps) * ROUND + uint64_t(u) * 32 + lane;
@@ -178,7 +185,27 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
       }
       mynode[u] = 0;
     }
-    if constexpr (MODE >= 2) {
+    if constexpr (MODE == 4) {
+      // (level-T node, key sector) = lower_bound(Msec, q) over 32-bit high words;
+      // equal high words fall back to the full key (global, L2-resident)
+      constexpr uint32_t NSEC = C::NSEC;
+      const uint32_t* s_sdir = s_hi + lt.dcount;
+#pragma unroll
+      for (int u = 0; u < QPL; ++u) {
+        const uint32_t qh = uint32_t(uint64_t(myq[u]) >> (8 * sizeof(K) - 32));
+        const uint32_t e = s_sdir[uint32_t(myq[u] >> (8 * sizeof(K) - lt.dbits))];
+        uint32_t lo = e & 0xFFFFu, hi = e >> 16;
+        while (lo < hi) {
+          const uint32_t mid = (lo + hi) >> 1;
+          const uint32_t mh = s_hi[mid];
+          bool lt_ = mh < qh;
+          if (sizeof(K) == 8 && mh == qh) lt_ = __ldg(sfull + mid) < myq[u];
+          if (lt_) lo = mid + 1; else hi = mid;
+        }
+        mynode[u] = lo / NSEC;
+        mysec[u] = lo % NSEC;
+      }
+    } else if constexpr (MODE >= 2) {
       // level-T node = lower_bound(M_T, q), narrowed by the prefix directory
 #pragma unroll
       for (int u = 0; u < QPL; ++u) {
@@ -220,16 +247,19 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
     //      owned in phase 1 by lane (j*NG)%32 + g, slot (j*NG)/32
     K q[QPG];
     uint32_t node[QPG];
+    uint32_t sec0[QPG];
 #pragma unroll
     for (int j = 0; j < QPG; ++j) {
       const int src = (j * C::NG) % 32 + g;
       q[j] = __shfl_sync(0xffffffffu, myq[(j * C::NG) / 32], src);
       node[j] = __shfl_sync(0xffffffffu, mynode[(j * C::NG) / 32], src);
+      sec0[j] = MODE == 4 ? __shfl_sync(0xffffffffu, mysec[(j * C::NG) / 32], src) : 0u;
     }
     for (uint32_t d = SL; d < H; ++d) {
       const uint8_t* lvl = inner + lt.offset[d] * C::NODE_BYTES;
+      const bool sec_known = MODE == 4 && d == SL;  // mode 4: the sector directory chose it
       if constexpr (C::HAS_IDX) {
-        if ((lt.full_mask >> d) & 1u) {
+        if (!sec_known && ((lt.full_mask >> d) & 1u)) {
           // Level beyond the L2-resident budget: a miss costs a whole DRAM line
           // anyway, so read the full node in ONE round trip (each of the G lanes
           // loads NODE_BYTES/G contiguous bytes) instead of index + sector.
@@ -255,7 +285,10 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
         }
       }
       uint32_t sec[QPG];
-      if constexpr (C::HAS_IDX) {
+      if (C::HAS_IDX && sec_known) {
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) sec[j] = sec0[j];
+      } else if constexpr (C::HAS_IDX) {
         const uint8_t* lidx = inner_idx + lt.offset[d] * C::IDXB;
         V16<K> iv[QPG];
 #pragma unroll
@@ -343,7 +376,12 @@ struct Launch {
     // the L2-resident budget are read as whole nodes (see the kernel).
     lt.full_mask = 0;
     size_t smem;
-    if (MODE >= 2) {
+    if (MODE == 4) {
+      lt.SL = t->dir_T;
+      lt.dcount = t->sdir_count;
+      lt.dbits = t->sdir_bits;
+      smem = t->sdir_bytes;
+    } else if (MODE >= 2) {
       lt.SL = t->dir_T;
       lt.dcount = t->dir_count;
       lt.dbits = t->dir_bits;
@@ -415,8 +453,9 @@ struct Launch {
       lc.numAttrs = 1;
     }
     HBT_CUDA_TRY(cudaLaunchKernelEx(&lc, kern, (const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
-                                    (const uint8_t*)t->d_leaf, (const uint32_t*)t->d_dir, (const K*)q, m, pf,
-                                    (K*)v, lt, t->n, base));
+                                    (const uint8_t*)t->d_leaf,
+                                    (const uint32_t*)(MODE == 4 ? t->d_sdir : t->d_dir),
+                                    (const K*)t->d_sdir_full, (const K*)q, m, pf, (K*)v, lt, t->n, base));
     HBT_CUDA_TRY(cudaGetLastError());
     return HBT_OK;
   }
@@ -427,6 +466,8 @@ struct Launch {
     const uint32_t th = t->cfg.threads ? t->cfg.threads : (C::NODE_BYTES > 128 ? 512 : 1024);
     // small batches read the directory in place (no 96 KB staging per CTA)
     if (t->cfg.mode == 3 || (t->cfg.mode == 2 && m <= t->cfg.small_batch)) return run_t<1, 1024, 3>(t, q, m, pf, v, b, s);
+    if (t->cfg.mode == 4 && t->d_sdir)
+      return th == 512 ? run_t<1, 512, 4>(t, q, m, pf, v, b, s) : run_t<1, 1024, 4>(t, q, m, pf, v, b, s);
     if (t->cfg.mode == 2) {
       if (th == 512) return run_t<1, 512, 2>(t, q, m, pf, v, b, s);
       return qpl == 2 ? run_t<2, 1024, 2>(t, q, m, pf, v, b, s) : run_t<1, 1024, 2>(t, q, m, pf, v, b, s);

@@ -44,7 +44,7 @@ def test_edge_suite_parity(hbt, width, F):
         assert t.export(hbt.SEG_INNER_IDX).tobytes() == expected_index_bytes(o, width), (n, F, width)
         q = query_set(k, width, rng, 3000)
         epf, ev = o.search(q)
-        for mode, l2b in ((0, 0), (2, 0), (2, 1), (0, 1), (3, 0)):  # staged / directory / in-place x read modes
+        for mode, l2b in ((0, 0), (2, 0), (2, 1), (0, 1), (3, 0), (4, 0), (4, 1)):  # top-level modes x read modes
             t.set_search_config(smem_mode=mode)
             t.set_param("l2_levels_bytes", l2b)
             pf, val = gpu_search(t, q, width)
