@@ -200,10 +200,20 @@ HBT_API int hbt_set_param(hbt_tree* t, const char* name, int64_t value);
  * Implicit trees only. */
 typedef struct hbt_comm hbt_comm;
 
+/* Host all-gather used by communicators created with hbt_comm_init_host:
+ * gather `bytes` from every rank's `send` into `recv` (nranks * bytes, rank
+ * order); return 0 on success. */
+typedef int (*hbt_allgather_fn)(const void* send, void* recv, uint64_t bytes, void* ctx);
+
 /* ncclGetUniqueId into a 128-byte buffer (rank 0; broadcast it to all ranks). */
 HBT_API int hbt_comm_unique_id(void* id128);
 /* ncclCommInitRank over nranks processes (one GPU each, current device). */
 HBT_API int hbt_comm_init(int nranks, int rank, const void* id128, hbt_comm** out);
+/* A communicator WITHOUT NCCL: the few small host-side exchanges of the sharded
+ * calls (shard ranges, per-batch counts, IPC window handles) go through the
+ * caller's all-gather callback; the data path is the fused peer-memory exchange
+ * (exchange = 0).  Works with any number of ranks per GPU. */
+HBT_API int hbt_comm_init_host(int nranks, int rank, hbt_allgather_fn fn, void* ctx, hbt_comm** out);
 HBT_API int hbt_comm_destroy(hbt_comm* c);
 /* Collective: every rank builds its shard from its local (device) pairs, then the
  * ranks all-gather (n', min, max).  HBT_EINVAL if shard ranges overlap. */

@@ -36,7 +36,7 @@ UPSERT, DELETE = 0, 1
 
 EXPORTED = ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
             "hbt_info", "hbt_export", "hbt_set_param", "hbt_last_error", "hbt_version",
-            "hbt_range", "hbt_comm_unique_id", "hbt_comm_init", "hbt_comm_destroy", "hbt_bulk_build_sharded",
+            "hbt_range", "hbt_comm_unique_id", "hbt_comm_init", "hbt_comm_init_host", "hbt_comm_destroy", "hbt_bulk_build_sharded",
             "hbt_search_sharded", "hbt_shard_local_init", "hbt_search_sharded_local"]
 
 
@@ -62,6 +62,9 @@ class _Info(C.Structure):
                 ("leaf_bytes", C.c_uint64)]
 
 
+ALLGATHER_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_void_p, C.c_uint64, C.c_void_p)
+
+
 def _load():
     if not os.path.exists(LIB_PATH):
         raise ImportError(f"{LIB_PATH} is missing: build it with `make` or __graft_entry__.build() "
@@ -79,6 +82,7 @@ def _load():
     L.hbt_range.argtypes = [vp, vp, vp, u64, u32, vp, vp, vp, vp]
     L.hbt_comm_unique_id.argtypes = [vp]
     L.hbt_comm_init.argtypes = [C.c_int, C.c_int, vp, C.POINTER(vp)]
+    L.hbt_comm_init_host.argtypes = [C.c_int, C.c_int, ALLGATHER_FN, vp, C.POINTER(vp)]
     L.hbt_comm_destroy.argtypes = [vp]
     L.hbt_bulk_build_sharded.argtypes = [vp, vp, vp, u64, u32, u32, vp, C.POINTER(vp)]
     L.hbt_search_sharded.argtypes = [vp, vp, u64, _Out, vp]
@@ -89,6 +93,7 @@ def _load():
     L.hbt_version.restype = C.c_char_p
     for f in ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
               "hbt_info", "hbt_export", "hbt_set_param", "hbt_range", "hbt_comm_unique_id", "hbt_comm_init",
+              "hbt_comm_init_host",
               "hbt_comm_destroy", "hbt_bulk_build_sharded", "hbt_search_sharded", "hbt_shard_local_init",
               "hbt_search_sharded_local"]:
         getattr(L, f).restype = C.c_int
@@ -286,6 +291,32 @@ class Comm:
         import torch.distributed as dist
         uid = broadcast_unique_id(group)
         return cls(dist.get_world_size(group), dist.get_rank(group), uid)
+
+    @classmethod
+    def from_torch_host(cls, group=None):
+        """A communicator without NCCL: the library's small host-side exchanges go
+        through torch.distributed (any backend, e.g. gloo) all-gathers; the data
+        path is the fused peer-memory exchange.  Allows several ranks per GPU."""
+        import torch
+        import torch.distributed as dist
+        world, rank = dist.get_world_size(group), dist.get_rank(group)
+
+        def allgather(send, recv, nbytes, ctx):
+            try:
+                mine = torch.frombuffer(bytearray(C.string_at(send, nbytes)), dtype=torch.uint8)
+                out = [torch.empty(nbytes, dtype=torch.uint8) for _ in range(world)]
+                dist.all_gather(out, mine, group=group)
+                C.memmove(recv, torch.cat(out).numpy().tobytes(), nbytes * world)
+                return 0
+            except Exception:
+                return 1
+
+        self = cls.__new__(cls)
+        self._fn = ALLGATHER_FN(allgather)  # keep the callback alive
+        h = C.c_void_p()
+        _check(lib.hbt_comm_init_host(world, rank, self._fn, None, C.byref(h)))
+        self._h, self.nranks, self.rank = h, world, rank
+        return self
 
     def close(self):
         if getattr(self, "_h", None) and self._h.value:

@@ -123,10 +123,18 @@ struct Scratch {
 }  // namespace hbt
 
 struct hbt_comm {
-  ncclComm_t comm = nullptr;
+  ncclComm_t comm = nullptr;          // NULL for a host-callback communicator
   int nranks = 1;
   int rank = 0;
+  hbt_allgather_fn host_allgather = nullptr;  // host all-gather (hbt_comm_init_host)
+  void* host_ctx = nullptr;
 };
+
+namespace hbt {
+// All-gather `bytes` of host memory from every rank into recv (rank order),
+// through the host callback if the communicator has one, else through NCCL.
+int comm_allgather_host(hbt_comm* c, const void* send, void* recv, uint64_t bytes, cudaStream_t st);
+}  // namespace hbt
 
 struct hbt_tree {
   uint32_t form = HBT_IMPLICIT;  // HBT_IMPLICIT | HBT_REGULAR

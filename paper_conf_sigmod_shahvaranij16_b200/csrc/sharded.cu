@@ -346,6 +346,26 @@ int search_nccl_t(const hbt_tree* tc, const void* queries, uint64_t m, hbt_out o
 
 }  // namespace
 
+int comm_allgather_host(hbt_comm* c, const void* send, void* recv, uint64_t bytes, cudaStream_t st) {
+  if (c->host_allgather) {
+    if (c->host_allgather(send, recv, bytes, c->host_ctx) != 0) {
+      set_error("host all-gather callback failed");
+      return HBT_ENCCL;
+    }
+    return HBT_OK;
+  }
+  uint8_t* d = nullptr;
+  HBT_CUDA_TRY(cudaMalloc(&d, bytes * (c->nranks + 1)));
+  cudaMemcpyAsync(d, send, bytes, cudaMemcpyHostToDevice, st);
+  ncclResult_t r = ncclAllGather(d, d + bytes, bytes, ncclUint8, c->comm, st);
+  if (r == ncclSuccess) cudaMemcpyAsync(recv, d + bytes, bytes * c->nranks, cudaMemcpyDeviceToHost, st);
+  cudaError_t e = cudaStreamSynchronize(st);
+  cudaFree(d);
+  if (r != ncclSuccess) { set_error("ncclAllGather: %s", ncclGetErrorString(r)); return HBT_ENCCL; }
+  if (e != cudaSuccess) { set_error("all-gather: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
+  return HBT_OK;
+}
+
 void shard_free(hbt_tree* t) { free_scratch(t->shard_scratch); }
 
 }  // namespace hbt
@@ -382,6 +402,20 @@ int hbt_comm_init(int nranks, int rank, const void* id128, hbt_comm** out) {
   return HBT_OK;
 }
 
+int hbt_comm_init_host(int nranks, int rank, hbt_allgather_fn fn, void* ctx, hbt_comm** out) {
+  if (!out || !fn || nranks < 1 || nranks > kMaxShards || rank < 0 || rank >= nranks) {
+    set_error("bad communicator arguments");
+    return HBT_EINVAL;
+  }
+  hbt_comm* c = new hbt_comm();
+  c->nranks = nranks;
+  c->rank = rank;
+  c->host_allgather = fn;
+  c->host_ctx = ctx;
+  *out = c;
+  return HBT_OK;
+}
+
 int hbt_comm_destroy(hbt_comm* c) {
   if (!c) return HBT_EINVAL;
   if (c->comm) ncclCommDestroy(c->comm);
@@ -400,21 +434,13 @@ int hbt_bulk_build_sharded(hbt_comm* c, const void* keys_local, const void* valu
   uint64_t mn = 0, mx = 0;
   if ((rc = first_last_keys(t, &mn, &mx))) { hbt_destroy(t); *out = nullptr; return rc; }
   // all-gather (n', min, max) of every shard
-  uint64_t* d = nullptr;
   cudaStream_t st = (cudaStream_t)stream;
-  if (cudaMalloc(&d, 4 * 3 * G * 8) != cudaSuccess) { hbt_destroy(t); *out = nullptr; set_error("alloc"); return HBT_ENOMEM; }
   uint64_t mine[3] = {t->n, mn, mx};
   std::vector<uint64_t> all(3 * G);
-  cudaMemcpyAsync(d, mine, 24, cudaMemcpyHostToDevice, st);
-  ncclResult_t r = ncclAllGather(d, d + 3, 3, ncclUint64, c->comm, st);
-  if (r == ncclSuccess) cudaMemcpyAsync(all.data(), d + 3, 3 * G * 8, cudaMemcpyDeviceToHost, st);
-  cudaStreamSynchronize(st);
-  cudaFree(d);
-  if (r != ncclSuccess) {
-    set_error("ncclAllGather: %s", ncclGetErrorString(r));
+  if ((rc = comm_allgather_host(c, mine, all.data(), sizeof(mine), st))) {
     hbt_destroy(t);
     *out = nullptr;
-    return HBT_ENCCL;
+    return rc;
   }
   std::vector<uint64_t> cn(G), mnv(G), mxv(G);
   for (int g = 0; g < G; ++g) { cn[g] = all[3 * g]; mnv[g] = all[3 * g + 1]; mxv[g] = all[3 * g + 2]; }
@@ -429,6 +455,7 @@ int hbt_search_sharded(const hbt_tree* t, const void* queries_local, uint64_t m_
   if (!t || !t->shard.comm) { set_error("not a sharded tree"); return HBT_EINVAL; }
   cudaStream_t st = (cudaStream_t)stream;
   if (t->cfg.exchange == 0) return fused_search_nccl(t, queries_local, m_local, out_local, st);
+  if (!t->shard.comm->comm) { set_error("exchange=1 needs an NCCL communicator"); return HBT_EUNSUPPORTED; }
   return t->width == 4 ? search_nccl_t<uint32_t>(t, queries_local, m_local, out_local, st)
                        : search_nccl_t<uint64_t>(t, queries_local, m_local, out_local, st);
 }

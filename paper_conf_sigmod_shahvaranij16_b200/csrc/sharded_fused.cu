@@ -352,15 +352,9 @@ int exchange_windows(FusedState* f, hbt_comm* c, uint64_t cap_m, uint64_t cap_r,
   if (rc) return rc;
   cudaIpcMemHandle_t h;
   HBT_CUDA_TRY(cudaIpcGetMemHandle(&h, f->win));
-  void* d = nullptr;
-  HBT_CUDA_TRY(cudaMalloc(&d, sizeof(h) * (c->nranks + 1)));
-  HBT_CUDA_TRY(cudaMemcpyAsync(d, &h, sizeof(h), cudaMemcpyHostToDevice, st));
-  ncclResult_t r = ncclAllGather(d, (uint8_t*)d + sizeof(h), sizeof(h), ncclUint8, c->comm, st);
   std::vector<cudaIpcMemHandle_t> all(c->nranks);
-  if (r == ncclSuccess) cudaMemcpyAsync(all.data(), (uint8_t*)d + sizeof(h), sizeof(h) * c->nranks, cudaMemcpyDeviceToHost, st);
-  cudaStreamSynchronize(st);
-  cudaFree(d);
-  if (r != ncclSuccess) { set_error("handle all-gather: %s", ncclGetErrorString(r)); return HBT_ENCCL; }
+  rc = comm_allgather_host(c, &h, all.data(), sizeof(h), st);
+  if (rc) return rc;
   for (int g = 0; g < c->nranks; ++g) {
     if (g == c->rank) { f->peer[g] = f->win; continue; }
     void* p = nullptr;
@@ -384,15 +378,11 @@ int nccl_fused_t(hbt_tree* t, const void* queries, uint64_t m, hbt_out out, cuda
   const RouteTab rt = table_of(t->shard);
   rc = route_and_count<K>(f, (const K*)queries, m, rt, G, st);
   if (rc) return rc;
-  unsigned long long* d = nullptr;
-  HBT_CUDA_TRY(cudaMalloc(&d, sizeof(unsigned long long) * (G + 1) * (G + 1) * 2));
-  HBT_CUDA_TRY(cudaMemcpyAsync(d, f->cnt, G * 8, cudaMemcpyDeviceToDevice, st));
-  ncclResult_t r = ncclAllGather(d, d + G, G, ncclUint64, c->comm, st);
-  std::vector<unsigned long long> mat(G * G);
-  if (r == ncclSuccess) cudaMemcpyAsync(mat.data(), d + G, G * G * 8, cudaMemcpyDeviceToHost, st);
-  cudaStreamSynchronize(st);
-  cudaFree(d);
-  if (r != ncclSuccess) { set_error("count all-gather: %s", ncclGetErrorString(r)); return HBT_ENCCL; }
+  std::vector<unsigned long long> mine(G), mat(G * G);
+  HBT_CUDA_TRY(cudaMemcpyAsync(mine.data(), f->cnt, G * 8, cudaMemcpyDeviceToHost, st));
+  HBT_CUDA_TRY(cudaStreamSynchronize(st));
+  rc = comm_allgather_host(c, mine.data(), mat.data(), G * 8, st);
+  if (rc) return rc;
   uint64_t need_m = 1, need_r = 1;
   for (int x = 0; x < G; ++x) {
     uint64_t row = 0, col = 0;

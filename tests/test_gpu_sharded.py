@@ -100,3 +100,24 @@ def test_nccl_path_one_rank(hbt, exchange):
         assert np.array_equal(from_dev(v, 8), ev)
     t.close()
     comm.close()
+
+
+def test_fused_exchange_two_processes_one_gpu():
+    """Two ranks (processes) on one GPU through the host-callback communicator:
+    CUDA IPC windows, device flag barriers and peer stores (exchange = 0), each
+    rank's results vs the unsharded oracle (tools/two_rank_one_gpu.py)."""
+    import os
+    import socket
+    import subprocess
+    import sys
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nproc-per-node", "2",
+                        "--master-addr", "127.0.0.1", "--master-port", str(port),
+                        os.path.join(root, "tools", "two_rank_one_gpu.py"), "0"],
+                       capture_output=True, text=True, timeout=600, cwd=root)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+    assert r.stdout.count("ok=True") == 2, r.stdout[-2000:]

@@ -120,3 +120,39 @@ def test_shard_plan_covers_range():
         spans = [hbt.shard_plan(n, w, r) for r in range(w)]
         assert spans[0][0] == 0 and spans[-1][1] == n
         assert all(spans[i][1] == spans[i + 1][0] for i in range(w - 1))
+
+
+def _host_comm_worker(rank, world, port, q):
+    import ctypes as C
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import paper_conf_sigmod_shahvaranij16_b200 as hbt
+        comm = hbt.Comm.from_torch_host()
+        # drive the callback the library calls, through its C function pointer
+        send = (C.c_uint64 * 3)(100 + rank, 2**64 - 1 - rank, 7)
+        recv = (C.c_uint64 * (3 * world))()
+        rc = comm._fn(C.cast(send, C.c_void_p), C.cast(recv, C.c_void_p), C.sizeof(send), None)
+        want = [x for r in range(world) for x in (100 + r, 2**64 - 1 - r, 7)]
+        ok = rc == 0 and list(recv) == want and comm.nranks == world and comm.rank == rank
+        comm.close()
+        q.put((rank, ok))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_host_allgather_communicator_two_ranks_gloo():
+    """hbt_comm_init_host + the torch.distributed all-gather callback that carries
+    the sharded calls' host-side exchanges when NCCL is not used (exchange = 0)."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_host_comm_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=300) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert all(ok for _, ok in res), res

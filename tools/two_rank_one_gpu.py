@@ -1,0 +1,54 @@
+"""Two processes on ONE GPU running the sharded search through the real
+communicator: exercises CUDA IPC window export/import, the device-side flag
+barriers and the peer-store exchange (exchange=0) or NCCL send/recv (1), and
+checks every rank's results against the unsharded oracle.  Launch with
+torchrun --nproc-per-node 2 (gloo for the host-side plumbing)."""
+import os
+import sys
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import gen  # noqa: E402
+import oracle  # noqa: E402  (test tool: checks the results)
+import paper_conf_sigmod_shahvaranij16_b200 as hbt  # noqa: E402
+
+
+def main():
+    exchange = int(sys.argv[1]) if len(sys.argv) > 1 else 0
+    dist.init_process_group("gloo")
+    rank, world = dist.get_rank(), dist.get_world_size()
+    torch.cuda.set_device(0)
+    comm = hbt.Comm.from_torch_host() if exchange == 0 else hbt.Comm.from_torch()
+    n = 200000
+    allk = gen.stratified_keys(n, 7)
+    allv = gen.values(n, 8, 9)
+    lo, hi = hbt.shard_plan(n, world, rank)
+    k = torch.from_numpy(allk[lo:hi].view(np.int64)).cuda()
+    v = torch.from_numpy(allv[lo:hi].view(np.int64)).cuda()
+    t = hbt.ShardedTree(comm, k, v, fanout=16)
+    t.set_param("exchange", exchange)
+    full = oracle.ITree.from_pairs(allk, allv, 16, 8)
+    ok = True
+    for rep in range(3):
+        rng = np.random.default_rng(100 * rank + rep)
+        q = np.concatenate([allk[rng.integers(0, n, 30000 * (rep + 1))],
+                            rng.integers(0, 2**64 - 1, 5000, dtype=np.uint64, endpoint=True)])
+        pf, vals = t.search(torch.from_numpy(q.view(np.int64)).cuda())
+        torch.cuda.synchronize()
+        epf, ev = full.search(q)
+        ok &= np.array_equal(pf.cpu().numpy().view(np.uint64), epf)
+        ok &= np.array_equal(vals.cpu().numpy().view(np.uint64), ev)
+    print(f"rank {rank} exchange {exchange} ok={ok}", flush=True)
+    t.close()
+    comm.close()
+    dist.destroy_process_group()
+    sys.exit(0 if ok else 1)
+
+
+if __name__ == "__main__":
+    main()
