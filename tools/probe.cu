@@ -89,3 +89,290 @@ PROBE_API double probe_random_read_gbs(uint64_t bytes, int chunk, int reps) {
   const double total = double(grid) * threads * iters * 8 * 16;  // bytes read
   return total / (best_ms * 1e-3) / 1e9;
 }
+
+// Die-affinity experiment: the SMs are split into two halves by `map` applied
+// to %smid (0 = no split, 1 = smid < nsm/2, 2 = smid & 1, 3 = (smid >> 1) & 1,
+// 4 = (smid >> 2) & 1, 5 = (smid >> 3) & 1); each half reads random chunks of
+// its own half of the buffer only.  If L2 capacity for all-SM random reads is
+// lost to cross-die duplication, the right split restores it.
+__device__ __forceinline__ uint32_t smid() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+  return r;
+}
+
+template <int CHUNK, int UNROLL>
+__global__ void __launch_bounds__(512) l2_random_read_aff(const uint4* __restrict__ buf, uint64_t nchunks,
+                                                          uint64_t iters, uint64_t seed, int map, uint32_t nsm,
+                                                          const uint8_t* __restrict__ die, uint4* __restrict__ sink) {
+  constexpr int G = CHUNK / 16;
+  const int lane = threadIdx.x & 31;
+  const uint64_t gid = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) / G;
+  const int k = lane % G;
+  const uint32_t s = smid();
+  uint32_t half = 0;
+  switch (map) {
+    case 1: half = s >= nsm / 2; break;
+    case 2: half = s & 1; break;
+    case 3: half = (s >> 1) & 1; break;
+    case 4: half = (s >> 2) & 1; break;
+    case 5: half = (s >> 3) & 1; break;
+    case 6: half = die[s]; break;
+    default: half = 0;
+  }
+  const uint64_t span = map ? nchunks / 2 : nchunks;
+  const uint64_t off = uint64_t(half) * span;
+  uint4 acc = make_uint4(0, 0, 0, 0);
+  uint64_t state = mix64(gid ^ seed);
+  for (uint64_t it = 0; it < iters; ++it) {
+    uint4 v[UNROLL];
+#pragma unroll
+    for (int u = 0; u < UNROLL; ++u) {
+      state = mix64(state);
+      const uint64_t c = off + __umul64hi(state, span);
+      v[u] = __ldg(buf + c * G + k);
+    }
+#pragma unroll
+    for (int u = 0; u < UNROLL; ++u) {
+      acc.x ^= v[u].x; acc.y ^= v[u].y; acc.z ^= v[u].z; acc.w ^= v[u].w;
+    }
+  }
+  if ((acc.x ^ acc.y ^ acc.z ^ acc.w) == 0x12345678u) sink[threadIdx.x] = acc;
+}
+
+PROBE_API double probe_random_read_aff_gbs(uint64_t bytes, int chunk, int map, int reps, const uint8_t* die_host) {
+  uint4* buf = nullptr;
+  uint8_t* die = nullptr;
+  cudaMalloc(&die, 1024);
+  cudaMemset(die, 0, 1024);
+  if (die_host) cudaMemcpy(die, die_host, 256, cudaMemcpyHostToDevice);
+  uint4* sink = nullptr;
+  if (cudaMalloc(&buf, bytes) != cudaSuccess) return -1;
+  cudaMalloc(&sink, 512 * sizeof(uint4));
+  cudaMemset(buf, 1, bytes);
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const uint64_t nchunks = bytes / chunk;
+  const uint64_t iters = 256;
+  const unsigned grid = sms * 4;
+  const unsigned threads = 512;
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  float best_ms = 1e30f;
+  for (int r = 0; r < reps + 1; ++r) {
+    cudaEventRecord(a);
+    if (chunk == 32) l2_random_read_aff<32, 8><<<grid, threads>>>(buf, nchunks, iters, r, map, sms, die, sink);
+    else l2_random_read_aff<64, 8><<<grid, threads>>>(buf, nchunks, iters, r, map, sms, die, sink);
+    cudaEventRecord(b);
+    cudaEventSynchronize(b);
+    float ms = 0;
+    cudaEventElapsedTime(&ms, a, b);
+    if (r > 0 && ms < best_ms) best_ms = ms;
+  }
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  cudaFree(buf);
+  cudaFree(sink);
+  cudaFree(die);
+  if (cudaGetLastError() != cudaSuccess) return -2;
+  const double total = double(grid) * threads * iters * 8 * 16;
+  return total / (best_ms * 1e-3) / 1e9;
+}
+
+// SM -> die discovery: one CTA per SM, one thread, times a dependent L2 hit to
+// each of NA addresses (warm); lines homed on the far die's L2 take longer.
+constexpr int kNA = 64;
+__global__ void sm_latency(const uint64_t* __restrict__ buf, uint64_t stride_words, uint32_t* __restrict__ out,
+                           uint32_t* __restrict__ sm_of_cta) {
+  if (threadIdx.x) return;
+  const uint32_t s = smid();
+  sm_of_cta[blockIdx.x] = s;
+  uint64_t x = 0;
+  for (int rep = 0; rep < 2; ++rep) {
+    for (int a = 0; a < kNA; ++a) {
+      const uint64_t* p = buf + uint64_t(a) * stride_words + (x & 1);
+      const long long t0 = clock64();
+      uint64_t v;
+      asm volatile("ld.global.cg.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+      x += v;
+      const long long t1 = clock64() + (long long)(x & 0);  // depends on v
+      if (rep == 1) out[blockIdx.x * kNA + a] = uint32_t(t1 - t0);
+    }
+  }
+  if (x == 12345) out[0] = 0;
+}
+
+PROBE_API int probe_sm_latency(uint32_t* host_lat, uint32_t* host_sm, int nctas) {
+  uint64_t* buf = nullptr;
+  uint32_t *lat = nullptr, *sm = nullptr;
+  const uint64_t stride_words = 4096 / 8 + 4;  // 4 KB + 32 B apart
+  cudaMalloc(&buf, kNA * stride_words * 8 + 64);
+  cudaMemset(buf, 0, kNA * stride_words * 8 + 64);
+  cudaMalloc(&lat, sizeof(uint32_t) * kNA * nctas);
+  cudaMalloc(&sm, sizeof(uint32_t) * nctas);
+  sm_latency<<<nctas, 32>>>(buf, stride_words, lat, sm);
+  cudaMemcpy(host_lat, lat, sizeof(uint32_t) * kNA * nctas, cudaMemcpyDeviceToHost);
+  cudaMemcpy(host_sm, sm, sizeof(uint32_t) * nctas, cudaMemcpyDeviceToHost);
+  cudaFree(buf);
+  cudaFree(lat);
+  cudaFree(sm);
+  return int(cudaGetLastError());
+}
+
+// Address -> home-die discovery: every CTA (one per SM) times a dependent L2 hit
+// to each of na addresses `stride` bytes apart (second pass, warm).
+__global__ void addr_latency(const uint8_t* __restrict__ buf, uint64_t stride, int na, uint16_t* __restrict__ out,
+                             uint32_t* __restrict__ sm_of_cta) {
+  if (threadIdx.x) return;
+  sm_of_cta[blockIdx.x] = smid();
+  uint64_t x = 0;
+  for (int rep = 0; rep < 2; ++rep) {
+    for (int a = 0; a < na; ++a) {
+      const uint64_t* p = reinterpret_cast<const uint64_t*>(buf + uint64_t(a) * stride) + (x & 1);
+      const long long t0 = clock64();
+      uint64_t v;
+      asm volatile("ld.global.cg.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+      x += v;
+      const long long t1 = clock64() + (long long)(x & 0);
+      if (rep == 1) out[uint64_t(blockIdx.x) * na + a] = uint16_t(min(t1 - t0, 65535ll));
+    }
+  }
+  if (x == 12345) out[0] = 0;
+}
+
+PROBE_API int probe_addr_latency(uint16_t* host_lat, uint32_t* host_sm, int nctas, uint64_t stride, int na) {
+  uint8_t* buf = nullptr;
+  uint16_t* lat = nullptr;
+  uint32_t* sm = nullptr;
+  cudaMalloc(&buf, stride * na + 64);
+  cudaMemset(buf, 0, stride * na + 64);
+  cudaMalloc(&lat, sizeof(uint16_t) * na * nctas);
+  cudaMalloc(&sm, sizeof(uint32_t) * nctas);
+  addr_latency<<<nctas, 32>>>(buf, stride, na, lat, sm);
+  cudaMemcpy(host_lat, lat, sizeof(uint16_t) * na * nctas, cudaMemcpyDeviceToHost);
+  cudaMemcpy(host_sm, sm, sizeof(uint32_t) * nctas, cudaMemcpyDeviceToHost);
+  cudaFree(buf);
+  cudaFree(lat);
+  cudaFree(sm);
+  return int(cudaGetLastError());
+}
+
+// Home die of every 256 B chunk of a buffer: each CTA (thread 0) touches its
+// chunks once (miss) and times a second, L2-hit access; the latency compared
+// with the CTA's own die says near (same die) or far.
+__global__ void chunk_home(const uint8_t* __restrict__ buf, uint64_t nchunks, const uint8_t* __restrict__ die,
+                           uint8_t* __restrict__ home, uint32_t thresh) {
+  if (threadIdx.x) return;
+  const uint32_t d = die[smid()];
+  uint64_t x = 0;
+  for (uint64_t c = blockIdx.x; c < nchunks; c += gridDim.x) {
+    const uint64_t* p = reinterpret_cast<const uint64_t*>(buf + c * 256);
+    uint64_t v;
+    asm volatile("ld.global.cg.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    x += v;
+    const uint64_t* p2 = p + (x & 1);
+    const long long t0 = clock64();
+    asm volatile("ld.global.cg.u64 %0, [%1];" : "=l"(v) : "l"(p2) : "memory");
+    x += v;
+    const long long t1 = clock64() + (long long)(x & 0);
+    const bool near = uint32_t(t1 - t0) < thresh;
+    home[c] = uint8_t(near ? d : 1 - d);
+  }
+  if (x == 12345) home[0] = 7;
+}
+
+template <int UNROLL>
+__global__ void __launch_bounds__(512) l2_random_read_home(const uint4* __restrict__ buf, uint64_t nchunks,
+                                                           const uint32_t* __restrict__ homebits, int mode,
+                                                           uint64_t iters, uint64_t seed, const uint8_t* __restrict__ die,
+                                                           uint4* __restrict__ sink) {
+  extern __shared__ uint32_t sbits[];
+  const uint32_t nw = uint32_t((nchunks + 31) / 32);
+  for (uint32_t i = threadIdx.x; i < nw; i += blockDim.x) sbits[i] = homebits[i];
+  __syncthreads();
+  const uint64_t gid = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) / 2;
+  const int k = threadIdx.x & 1;
+  const uint32_t want = mode == 1 ? die[smid()] : 1u - die[smid()];
+  uint4 acc = make_uint4(0, 0, 0, 0);
+  uint64_t state = mix64(gid ^ seed);
+  for (uint64_t it = 0; it < iters; ++it) {
+    uint4 v[UNROLL];
+#pragma unroll
+    for (int u = 0; u < UNROLL; ++u) {
+      uint64_t c;
+      for (;;) {  // both lanes of the pair draw the same sequence
+        state = mix64(state);
+        c = __umul64hi(state, nchunks);
+        if (mode == 0 || ((sbits[c >> 5] >> (c & 31)) & 1u) == want) break;
+      }
+      const uint32_t sec = uint32_t(state) & 7u;
+      v[u] = __ldg(buf + c * 16 + sec * 2 + k);
+    }
+#pragma unroll
+    for (int u = 0; u < UNROLL; ++u) {
+      acc.x ^= v[u].x; acc.y ^= v[u].y; acc.z ^= v[u].z; acc.w ^= v[u].w;
+    }
+  }
+  if ((acc.x ^ acc.y ^ acc.z ^ acc.w) == 0x12345678u) sink[threadIdx.x] = acc;
+}
+
+// mode 0: both SM groups read random sectors of the whole buffer;
+// mode 1: each group reads only chunks homed on its own die;
+// mode 2: each group reads only chunks homed on the OTHER die.
+PROBE_API double probe_affinity_read_gbs(uint64_t bytes, int mode, const uint8_t* die_host, uint32_t thresh,
+                                         double* frac_home0) {
+  uint8_t *buf = nullptr, *die = nullptr, *home = nullptr;
+  uint4* sink = nullptr;
+  const uint64_t nchunks = bytes / 256;
+  if (cudaMalloc(&buf, bytes) != cudaSuccess) return -1;
+  cudaMemset(buf, 1, bytes);
+  cudaMalloc(&die, 256);
+  cudaMemcpy(die, die_host, 256, cudaMemcpyHostToDevice);
+  cudaMalloc(&home, nchunks);
+  cudaMalloc(&sink, 512 * sizeof(uint4));
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  chunk_home<<<sms, 32>>>(buf, nchunks, die, home, thresh);
+  uint8_t* h = new uint8_t[nchunks];
+  cudaMemcpy(h, home, nchunks, cudaMemcpyDeviceToHost);
+  const uint64_t nw = (nchunks + 31) / 32;
+  uint32_t* hb = new uint32_t[nw]();
+  uint64_t n0 = 0;
+  for (uint64_t c = 0; c < nchunks; ++c) {
+    n0 += h[c] == 0;
+    if (h[c] == 1) hb[c >> 5] |= 1u << (c & 31);
+  }
+  *frac_home0 = double(n0) / double(nchunks);
+  uint32_t* dl = nullptr;
+  cudaMalloc(&dl, nw * 4);
+  cudaMemcpy(dl, hb, nw * 4, cudaMemcpyHostToDevice);
+  if (nw * 4 > 200 * 1024) return -3;
+  cudaFuncSetAttribute(l2_random_read_home<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024);
+  const uint64_t iters = 256;
+  const unsigned grid = sms, threads = 512;
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  float best_ms = 1e30f;
+  for (int r = 0; r < 3; ++r) {
+    cudaEventRecord(a);
+    l2_random_read_home<8><<<grid, threads, nw * 4>>>((const uint4*)buf, nchunks, dl, mode, iters, r, die, sink);
+    cudaEventRecord(b);
+    cudaEventSynchronize(b);
+    float ms = 0;
+    cudaEventElapsedTime(&ms, a, b);
+    if (r > 0 && ms < best_ms) best_ms = ms;
+  }
+  delete[] h;
+  delete[] hb;
+  cudaFree(buf);
+  cudaFree(die);
+  cudaFree(home);
+  cudaFree(sink);
+  cudaFree(dl);
+  if (cudaGetLastError() != cudaSuccess) return -2;
+  return double(grid) * threads * iters * 8 * 16 / (best_ms * 1e-3) / 1e9;
+}
