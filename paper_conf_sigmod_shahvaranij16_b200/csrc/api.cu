@@ -65,6 +65,7 @@ static void free_tree(hbt_tree* t) {
   shard_free(t);
   fused_free(t);
   range_free(t);
+  bucket_free(t);
   cudaFree(t->pipe.d_q);
   cudaFree(t->pipe.d_pf);
   cudaFree(t->pipe.d_v);
@@ -76,6 +77,7 @@ static void free_tree(hbt_tree* t) {
 }
 
 static int device_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+  if (bucketed_enabled(t, m)) return bucketed_search(t, q, m, pf, v, s);
   return t->form == HBT_REGULAR ? regular_search(t, q, m, pf, v, s) : implicit_search(t, q, m, pf, v, s);
 }
 
@@ -205,6 +207,7 @@ int hbt_bulk_update(hbt_tree* t, const hbt_batch* batch, void* stream) {
     return HBT_EINVAL;
   }
   cudaStream_t s = (cudaStream_t)stream;
+  t->bk.valid = false;  // bucket splitters follow the tree
   return t->form == HBT_REGULAR ? regular_update(t, batch, s) : implicit_update(t, batch, s);
 }
 
@@ -290,6 +293,8 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "l2_persist" && value >= 0) c.l2_persist = uint64_t(value);
   else if (n == "l2_levels_bytes" && value >= 0) c.l2_levels_bytes = uint64_t(value);
   else if (n == "exchange" && (value == 0 || value == 1)) c.exchange = uint32_t(value);
+  else if (n == "bucket" && value >= 0 && value <= 2) c.bucket = uint32_t(value);
+  else if (n == "bucket_slice" && value >= 0) { c.bucket_slice = uint64_t(value); t->bk.valid = false; }
   else {
     set_error("bad parameter %s = %lld", name, (long long)value);
     return HBT_EINVAL;

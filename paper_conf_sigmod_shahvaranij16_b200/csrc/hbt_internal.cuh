@@ -54,6 +54,17 @@ struct SearchConfig {
   uint64_t l2_levels_bytes = 0;  // L2-resident budget for index+sector levels (0 = default 32 MB)
   uint32_t exchange = 0;         // sharded search: 0 = fused peer-memory exchange, 1 = NCCL send/recv
   uint64_t small_batch = 1u << 16;  // mode 2: batches up to this size read the directory in place (mode 3)
+  uint32_t bucket = 2;           // query bucketing (bucketed.cu): 0 = off, 1 = on, 2 = auto
+  uint64_t bucket_slice = 0;     // tree bytes per bucket (0 = default 16 MB)
+};
+
+// Query-bucketing state (bucketed.cu): B splitter keys and a prefix directory,
+// derived from the tree on first use and after every update.
+struct BucketState {
+  bool valid = false;
+  uint32_t B = 0;
+  void* d_sp = nullptr;          // B keys
+  uint32_t* d_dir = nullptr;     // 2^12 x (u16 lo, u16 hi)
 };
 
 // Regular-tree device state.  All pools are SoA arrays
@@ -186,6 +197,7 @@ struct hbt_tree {
   // ---- search ----
   hbt::SearchConfig cfg;
   mutable hbt::HostPipe pipe;
+  mutable hbt::BucketState bk;
 };
 
 namespace hbt {
@@ -221,4 +233,8 @@ int regular_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, v
 int regular_update(hbt_tree* t, const hbt_batch* b, cudaStream_t s);
 void regular_free(hbt_tree* t);
 uint32_t regular_smem_levels(const hbt_tree* t, uint32_t budget);
+// bucketed.cu
+bool bucketed_enabled(const hbt_tree* t, uint64_t m);
+int bucketed_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s);
+void bucket_free(hbt_tree* t);
 }  // namespace hbt

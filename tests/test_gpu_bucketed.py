@@ -1,0 +1,116 @@
+"""GPU parity of the BUCKETED search (csrc/bucketed.cu): queries partitioned by
+key range before the tree walk and gathered back to query order.  Every output
+must equal the oracle's bit for bit, for both tree forms, every bucket count
+from 2 to the 1024 cap, empty / tiny trees, misses, 0 and MAX, and after
+updates (the splitters are re-derived from the updated tree)."""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from gpu_util import gpu_build, gpu_search, to_dev
+from test_oracle_implicit import gen_keys, kmax, query_set
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def hbt():
+    import paper_conf_sigmod_shahvaranij16_b200 as m
+    assert torch.cuda.is_available(), "gpu tests need a CUDA device"
+    return m
+
+
+def _oracle(layout, k, v, F, width):
+    return (oracle.ITree if layout == "implicit" else oracle.RTree).from_pairs(k, v, F, width)
+
+
+@pytest.mark.parametrize("layout", ["implicit", "regular"])
+@pytest.mark.parametrize("width,F", [(4, 8), (8, 16), (8, 32), (4, 32)])
+def test_bucketed_edge_suite(hbt, layout, width, F):
+    P = 64 // (2 * width)
+    rng = np.random.default_rng(900 + 10 * F + width)
+    for n in sorted({0, 1, 2, P + 1, F * P + 1, 5 * F * P + 3, 30011}):
+        k, v = gen_keys(n, width, rng, dup=(n % 2 == 1), with_max=(n % 3 == 0))
+        o = _oracle(layout, k, v, F, width)
+        t = gpu_build(hbt, k, v, F, width, layout=layout)
+        q = query_set(k, width, rng, 5000)
+        q = np.concatenate([q, np.array([0, kmax(width)] * 50, dtype=np.uint64)])
+        epf, ev = o.search(q)
+        t.set_param("bucket", 1)
+        for slice_bytes in (1, 4096, 1 << 16):  # 1 B: one bucket per unit up to the 1024 cap
+            t.set_param("bucket_slice", slice_bytes)
+            pf, val = gpu_search(t, q, width)
+            assert np.array_equal(pf, epf), (layout, n, F, width, slice_bytes, np.nonzero(pf != epf)[0][:5])
+            assert np.array_equal(val, ev), (layout, n, F, width, slice_bytes)
+        t.close()
+
+
+@pytest.mark.parametrize("layout,F", [("implicit", 16), ("regular", 32)])
+def test_bucketed_scaled_workload(hbt, layout, F):
+    """c2 / c3 recipes at reduced size, several bucket counts, every output vs the oracle."""
+    cfg = "c2" if layout == "implicit" else "c3"
+    n, m = 1 << 19, 1 << 20
+    k, v = gen.workload_keys_values(cfg, n)
+    q = gen.workload_queries(cfg, k, m) if cfg == "c2" else gen.workload_queries(cfg, k, m, n_ins=n // 100)
+    o = _oracle(layout, k, v, F, 8)
+    epf, ev = o.search(q, nthreads=oracle.default_threads())
+    t = gpu_build(hbt, k, v, F, 8, layout=layout)
+    t.set_param("bucket", 1)
+    for slice_bytes in (1 << 16, 1 << 20, 1 << 22):
+        t.set_param("bucket_slice", slice_bytes)
+        pf, val = gpu_search(t, q, 8)
+        assert np.array_equal(pf, epf) and np.array_equal(val, ev), (layout, slice_bytes)
+    t.set_param("bucket", 0)
+    pf, val = gpu_search(t, q, 8)
+    assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+    t.close()
+
+
+@pytest.mark.parametrize("layout", ["implicit", "regular"])
+def test_bucketed_after_update(hbt, layout):
+    """The splitters follow the tree: search, update (keys move between buckets,
+    regular leaves split / empty), search again."""
+    width, F = 8, 8
+    rng = np.random.default_rng(4242)
+    n = 20000
+    k, v = gen_keys(n, width, rng, dup=True)
+    o = _oracle(layout, k, v, F, width)
+    t = gpu_build(hbt, k, v, F, width, layout=layout)
+    t.set_param("bucket", 1)
+    t.set_param("bucket_slice", 2048)
+    q = query_set(k, width, rng, 4000)
+    pf, val = gpu_search(t, q, width)
+    epf, ev = o.search(q)
+    assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+    for trial in range(3):
+        mu = 6000
+        src = np.concatenate([k[rng.integers(0, len(k), mu // 2)],
+                              rng.integers(0, kmax(width), mu - mu // 2, dtype=np.uint64)]).astype(np.uint64)
+        bv = rng.integers(0, kmax(width), mu, dtype=np.uint64)
+        bo = rng.integers(0, 2, mu).astype(np.uint8)
+        o = o.update(src, bv, bo) or o  # ITree.update returns the rebuilt tree
+        t.update(to_dev(src, width), to_dev(bv, width), torch.from_numpy(bo).cuda())
+        q = query_set(np.concatenate([k, src]), width, rng, 4000)
+        pf, val = gpu_search(t, q, width)
+        epf, ev = o.search(q)
+        assert np.array_equal(pf, epf) and np.array_equal(val, ev), (layout, trial)
+    t.close()
+
+
+def test_bucketed_host_pipeline(hbt):
+    """hbt_search_host runs the bucketed path per 4 Mi-query chunk."""
+    n, m = 1 << 16, (1 << 22) + 12345
+    k, v = gen.workload_keys_values("c2", n)
+    q = gen.workload_queries("c2", k, m)
+    o = _oracle("implicit", k, v, 16, 8)
+    t = gpu_build(hbt, k, v, 16, 8)
+    t.set_param("bucket", 1)
+    t.set_param("bucket_slice", 1 << 14)
+    pf = np.empty(m, np.uint64)
+    val = np.empty(m, np.uint64)
+    t.search_host(q.copy(), pf, val)
+    epf, ev = o.search(q, nthreads=oracle.default_threads())
+    assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+    t.close()
