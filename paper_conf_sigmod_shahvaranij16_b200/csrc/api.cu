@@ -295,6 +295,8 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "exchange" && (value == 0 || value == 1)) c.exchange = uint32_t(value);
   else if (n == "bucket" && value >= 0 && value <= 2) c.bucket = uint32_t(value);
   else if (n == "bucket_slice" && value >= 0) { c.bucket_slice = uint64_t(value); t->bk.valid = false; }
+  else if (n == "bucket_items" && (value == 0 || value == 1)) { c.bucket_items = uint32_t(value); t->bk.valid = false; }
+  else if (n == "bucket_cap" && value >= 0 && value < (1 << 20)) { c.bucket_cap = uint32_t(value); t->bk.valid = false; }
   else {
     set_error("bad parameter %s = %lld", name, (long long)value);
     return HBT_EINVAL;

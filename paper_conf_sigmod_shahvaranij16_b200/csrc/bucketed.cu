@@ -84,6 +84,43 @@ __global__ void bk_splitters_regular(const uint8_t* __restrict__ leaf, const uin
   sp[b] = load_key<K>(leaf + (uint64_t(v) * F + e / P) * 64 + (e % P) * sizeof(K));
 }
 
+// Item directory (implicit): M[j] = max key below level node j = the key of rank
+// min(n, (j+1) * span * P) - 1 (span = leaf lines per node; dense L-segment).
+template <typename K>
+__global__ void bk_level_max(const uint8_t* __restrict__ leaf, uint64_t n, uint32_t P, uint64_t span,
+                             uint64_t nunits, K* __restrict__ M) {
+  for (uint64_t j = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; j < nunits; j += uint64_t(gridDim.x) * blockDim.x) {
+    if (n == 0) { M[j] = kmax<K>(); continue; }
+    const uint64_t r = std::min<uint64_t>(n, (j + 1) * span * P) - 1;
+    M[j] = load_key<K>(leaf + (r / P) * 64 + (r % P) * sizeof(K));
+  }
+}
+
+// Item directory (regular): M[c * NI + t] = true max key of key line t of the
+// last-level node of chain leaf c = the key of entry min(count, (t+1)*KPL*P) - 1
+// (KPL separators per 64 B key line, each covering one leaf line of P entries);
+// key lines past the leaf's last entry repeat the leaf max (keeps M sorted).
+template <typename K>
+__global__ void bk_keyline_max(const uint8_t* __restrict__ leaf, const uint32_t* __restrict__ count,
+                               const uint32_t* __restrict__ chain, uint64_t nchain, uint32_t F, uint32_t P,
+                               uint32_t NI, uint32_t KPL, K* __restrict__ M) {
+  const uint64_t total = nchain * NI;
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < total; x += uint64_t(gridDim.x) * blockDim.x) {
+    const uint32_t v = chain[x / NI], t = uint32_t(x % NI);
+    const uint32_t cnt = count[v];
+    if (cnt == 0) { M[x] = kmax<K>(); continue; }
+    const uint32_t e = std::min<uint32_t>(cnt, (t + 1) * KPL * P) - 1;
+    M[x] = load_key<K>(leaf + (uint64_t(v) * F + e / P) * 64 + (e % P) * sizeof(K));
+  }
+}
+
+__global__ void bk_bstart(const uint32_t* __restrict__ gb, uint64_t chunks, uint32_t B, uint64_t m,
+                          uint64_t* __restrict__ bstart) {
+  const uint32_t b = blockIdx.x * blockDim.x + threadIdx.x;
+  if (b < B) bstart[b] = gb[uint64_t(b) * chunks];
+  if (b == B) bstart[b] = m;
+}
+
 template <typename K>
 __device__ __forceinline__ uint32_t lower_bound_in(const K* sp, uint32_t lo, uint32_t hi, K q) {
   while (lo < hi) {
@@ -115,13 +152,14 @@ __device__ __forceinline__ uint32_t bucket_of(K q, const K* s_sp, const uint32_t
 
 // Exclusive scan of s_in[0, B) into s_out (B <= 2 * kThreads) by one CTA; s_tmp
 // holds kThreads partial sums.  Ends with a barrier.
+template <int TH = kThreads>
 __device__ __forceinline__ void block_exclusive_scan(const uint32_t* s_in, uint32_t* s_out, uint32_t B,
                                                      uint32_t* s_tmp) {
   const uint32_t t = threadIdx.x;
   const uint32_t a = 2 * t < B ? s_in[2 * t] : 0u, b = 2 * t + 1 < B ? s_in[2 * t + 1] : 0u;
   s_tmp[t] = a + b;
   __syncthreads();
-  for (uint32_t off = 1; off < kThreads; off <<= 1) {
+  for (uint32_t off = 1; off < TH; off <<= 1) {
     const uint32_t x = t >= off ? s_tmp[t - off] : 0u;
     __syncthreads();
     s_tmp[t] += x;
@@ -173,15 +211,16 @@ __global__ void __launch_bounds__(kThreads) bk_count(const K* __restrict__ q, ui
 // Per-chunk bucket layout shared by the scatter and the gather: s_cnt (this
 // chunk's count per bucket), s_lb (their exclusive scan = the bucket's start in
 // the chunk's bucket-sorted order), s_gb (the run's first global slot).
+template <int TH = kThreads>
 __device__ __forceinline__ void chunk_layout(const uint32_t* __restrict__ tab, const uint32_t* __restrict__ gb,
                                              uint32_t B, uint64_t chunks, uint64_t c, uint32_t* s_cnt,
                                              uint32_t* s_lb, uint32_t* s_gb, uint32_t* s_tmp) {
-  for (uint32_t b = threadIdx.x; b < B; b += kThreads) {
+  for (uint32_t b = threadIdx.x; b < B; b += TH) {
     s_cnt[b] = tab[uint64_t(b) * chunks + c];
     s_gb[b] = gb[uint64_t(b) * chunks + c];
   }
   __syncthreads();
-  block_exclusive_scan(s_cnt, s_lb, B, s_tmp);
+  block_exclusive_scan<TH>(s_cnt, s_lb, B, s_tmp);
 }
 
 // Pass 2: each chunk's queries are ordered by bucket in shared memory, then
@@ -320,6 +359,68 @@ __global__ void __launch_bounds__(kThreads, 2) bk_gather(const uint16_t* __restr
   }
 }
 
+// Pass 4 for 16 B result records (the item-directory searches): one pass, the
+// chunk's record runs into shared memory, then {pos|found, value} in query
+// order.  (Measured: splitting the chunk into two halves for two CTAs per SM
+// makes each half's stores partial sectors and costs DRAM read-modify-writes,
+// 0.77 -> 0.88 ms on c3.)
+constexpr int kGThreads = 1024;
+template <typename K>
+__global__ void __launch_bounds__(kGThreads) bk_gather_rec(const uint16_t* __restrict__ linv, uint64_t m,
+                                                           const uint32_t* __restrict__ tab,
+                                                           const uint32_t* __restrict__ gb, uint32_t B,
+                                                           uint64_t chunks, const ulonglong2* __restrict__ rec,
+                                                           uint64_t* __restrict__ out_pf, K* __restrict__ out_v) {
+  constexpr int PT = int(kChunk) / kGThreads;
+  extern __shared__ __align__(16) uint8_t smem[];
+  ulonglong2* s_rec = reinterpret_cast<ulonglong2*>(smem);
+  uint16_t* s_b = reinterpret_cast<uint16_t*>(s_rec + kChunk);
+  uint32_t* s_cnt = reinterpret_cast<uint32_t*>(s_b + kChunk);
+  uint32_t* s_lb = s_cnt + kMaxBuckets;
+  uint32_t* s_gb = s_lb + kMaxBuckets;
+  uint32_t* s_tmp = s_gb + kMaxBuckets;
+  for (uint64_t c = blockIdx.x; c < chunks; c += gridDim.x) {
+    const uint64_t lo = c * kChunk;
+    const uint32_t nc = uint32_t(m - lo < kChunk ? m - lo : kChunk);
+    chunk_layout<kGThreads>(tab, gb, B, chunks, c, s_cnt, s_lb, s_gb, s_tmp);
+    for (uint32_t b = threadIdx.x; b < B; b += kGThreads)
+      for (uint32_t k = 0, n = s_cnt[b], p = s_lb[b]; k < n; ++k) s_b[p + k] = uint16_t(b);
+    __syncthreads();
+#pragma unroll 1
+    for (int h = 0; h < PT; h += 4) {
+      ulonglong2 x[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t t = uint32_t(h + j) * kGThreads + threadIdx.x;
+        if (t < nc) {
+          const uint32_t b = s_b[t];
+          x[j] = __ldcs(rec + s_gb[b] + (t - s_lb[b]));
+        }
+      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t t = uint32_t(h + j) * kGThreads + threadIdx.x;
+        if (t < nc) s_rec[t] = x[j];
+      }
+    }
+    __syncthreads();
+    const unsigned short* li = reinterpret_cast<const unsigned short*>(linv) + lo;
+#pragma unroll
+    for (int j = 0; j < PT; ++j) {
+      const uint32_t t = uint32_t(j) * kGThreads + threadIdx.x;
+      if (t < nc) {
+        const ulonglong2 r = s_rec[__ldcs(li + t)];
+        __stcs(reinterpret_cast<unsigned long long*>(out_pf) + lo + t, r.x);
+        if constexpr (sizeof(K) == 8)
+          __stcs(reinterpret_cast<unsigned long long*>(out_v) + lo + t, r.y);
+        else
+          __stcs(reinterpret_cast<unsigned int*>(out_v) + lo + t, (unsigned int)r.y);
+      }
+    }
+    __syncthreads();
+  }
+}
+
 uint64_t tree_bytes(const hbt_tree* t) {
   if (t->form == HBT_IMPLICIT) return t->inner_bytes + t->inner_idx_bytes + t->leaf_bytes;
   const RegularState& r = t->r;
@@ -330,12 +431,23 @@ uint64_t tree_bytes(const hbt_tree* t) {
 // Number of buckets: one per `slice` bytes of tree, at most one per unit and
 // kMaxBuckets.
 uint32_t pick_buckets(const hbt_tree* t) {
-  const uint64_t slice = t->cfg.bucket_slice ? t->cfg.bucket_slice : (16ull << 20);
+  // default 1 MB slices: with the 1024-bucket cap, large trees get the most
+  // buckets, which keeps the item directory in shared memory (measured on c3:
+  // 16 MB slices 15.0 G q/s, 1 MB 18.6 before the prefix table)
+  const uint64_t slice = t->cfg.bucket_slice ? t->cfg.bucket_slice : (1ull << 20);
   const uint64_t units = t->form == HBT_IMPLICIT ? t->L0 : t->r.nchain;
   uint64_t B = (tree_bytes(t) + slice - 1) / slice;
   B = std::min<uint64_t>(B, kMaxBuckets);
   B = std::min<uint64_t>(B, units);
   return uint32_t(std::max<uint64_t>(B, 1));
+}
+
+// Shared-memory entries of the item directory (keys; the regular tree also
+// stages one u32 chain id per NI entries): ~150 KB per CTA beside the bucket starts.
+uint64_t item_cap(const hbt_tree* t, uint32_t B) {
+  const uint64_t budget = 150 * 1024 - (uint64_t(B) + 1) * 8;
+  const uint64_t per = t->width + (t->form == HBT_REGULAR ? 4 : 0);
+  return budget / per;
 }
 
 template <typename K>
@@ -356,6 +468,54 @@ int prepare_splitters(const hbt_tree* t, cudaStream_t s) {
   HBT_CUDA_TRY(cudaGetLastError());
   bk_directory<K><<<(1u << kDirBits) / 256, 256, 0, s>>>((const K*)bs.d_sp, B, bs.d_dir);
   HBT_CUDA_TRY(cudaGetLastError());
+  // Item directory: the deepest unit level whose range for two buckets fits the
+  // shared-memory capacity.
+  bs.items = false;
+  if (t->cfg.bucket_items) {
+    const uint64_t cap = item_cap(t, B);
+    uint64_t nunits = 0;
+    if (t->form == HBT_IMPLICIT) {
+      uint64_t span = 1;
+      for (int d = int(t->H); d >= 0; --d) {
+        const uint64_t units = d == int(t->H) ? t->L0 : t->nodes[d];
+        if (2 * ((t->L0 / B) / span + 2) <= cap) {
+          bs.level = uint32_t(d);
+          bs.span = span;
+          nunits = units;
+          bs.items = true;
+          break;
+        }
+        span *= t->F;
+      }
+    } else {
+      const uint32_t KPL = 64 / sizeof(K);
+      const uint32_t NI = t->F > KPL ? t->F / KPL : 1;
+      if (2 * ((t->r.nchain / B) + 2) * NI <= cap) {
+        bs.span = NI;
+        nunits = t->r.nchain * NI;
+        bs.items = true;
+      }
+    }
+    if (bs.items) {
+      const uint64_t bytes = std::max<uint64_t>(nunits, 1) * sizeof(K);
+      if (bs.M_cap < bytes) {
+        cudaFree(bs.d_M);
+        bs.d_M = nullptr;
+        bs.M_cap = 0;
+        HBT_CUDA_TRY(cudaMalloc(&bs.d_M, bytes));
+        bs.M_cap = bytes;
+      }
+      bs.nunits = nunits;
+      if (t->form == HBT_IMPLICIT)
+        bk_level_max<K><<<t->num_sms * 4, 256, 0, s>>>((const uint8_t*)t->d_leaf, t->n, t->P, bs.span, nunits,
+                                                        (K*)bs.d_M);
+      else
+        bk_keyline_max<K><<<t->num_sms * 4, 256, 0, s>>>((const uint8_t*)t->r.d_leaf, t->r.d_count, t->r.d_chain,
+                                                          t->r.nchain, t->F, t->P, uint32_t(bs.span),
+                                                          uint32_t(64 / sizeof(K)), (K*)bs.d_M);
+      HBT_CUDA_TRY(cudaGetLastError());
+    }
+  }
   bs.B = B;
   bs.valid = true;
   return HBT_OK;
@@ -375,9 +535,11 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
                                              ntab, s));
   // scratch (stream-ordered pool): qs, pf_s, v_s, bq, linv, tab, gb, scan temp
   auto al = [](uint64_t x) { return (x + 255) & ~uint64_t(255); };
-  const uint64_t o_pf = al(m * sizeof(K)), o_v = o_pf + al(m * 8), o_bq = o_v + al(m * sizeof(K)),
+  // pf_s + v_s (plain search) or 16 B records (item directory: o_pf .. o_pf + 16 m)
+  const uint64_t o_pf = al(m * sizeof(K)), o_v = o_pf + al(m * 8), o_bq = o_v + al(m * 8),
                  o_li = o_bq + al(m * 2), o_tab = o_li + al(m * 2), o_gb = o_tab + al(ntab * 4),
-                 o_tmp = o_gb + al(ntab * 4), total = o_tmp + al(scan_bytes);
+                 o_bs = o_gb + al(ntab * 4), o_tmp = o_bs + al((uint64_t(B) + 1) * 8),
+                 total = o_tmp + al(scan_bytes);
   void* buf = nullptr;
   HBT_CUDA_TRY(scratch_alloc(&buf, total, s));
   uint8_t* base = static_cast<uint8_t*>(buf);
@@ -393,6 +555,7 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
     const size_t smem_count = (1u << kDirBits) * 4 + kMaxBuckets * 4 + kMaxBuckets * sizeof(K);
     const size_t smem_scatter = kChunk * (sizeof(K) + 2) + kMaxBuckets * 4 * 4 + kThreads * 4;
     const size_t smem_gather = kChunk * (8 + 2) + kMaxBuckets * 4 * 3 + kThreads * 4;
+    const size_t smem_gather_rec = kChunk * (16 + 2) + kMaxBuckets * 4 * 3 + kGThreads * 4;
     static bool attr = false;
     if (!attr) {
       const int lim = 120 * 1024;
@@ -402,6 +565,8 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
       cudaFuncSetAttribute(bk_scatter<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
       cudaFuncSetAttribute(bk_gather<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
       cudaFuncSetAttribute(bk_gather<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
+      cudaFuncSetAttribute(bk_gather_rec<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+      cudaFuncSetAttribute(bk_gather_rec<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
       attr = true;
     }
     const unsigned grid = unsigned(std::min<uint64_t>(chunks, uint64_t(t->num_sms) * 2));
@@ -417,9 +582,31 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
       rc = HBT_ECUDA;
       break;
     }
-    rc = search(t, qs, m, pf_s, v_s, s);
+    if (bs.items) {
+      uint64_t* bstart = reinterpret_cast<uint64_t*>(base + o_bs);
+      bk_bstart<<<(B + 256) / 256, 256, 0, s>>>(gb, chunks, B, m, bstart);
+      ItemDir d;
+      d.M = bs.d_M;
+      d.chain = t->form == HBT_REGULAR ? t->r.d_chain : nullptr;
+      d.bstart = bstart;
+      d.B = B;
+      d.U = t->form == HBT_IMPLICIT ? t->L0 : t->r.nchain;
+      d.level = bs.level;
+      d.span = bs.span;
+      d.nunits = bs.nunits;
+      d.cap = t->cfg.bucket_cap ? std::min<uint32_t>(t->cfg.bucket_cap, uint32_t(item_cap(t, B)))
+                                : uint32_t(item_cap(t, B));
+      rc = t->form == HBT_IMPLICIT ? implicit_search_items(t, qs, m, pf_s, v_s, d, s)
+                                   : regular_search_items(t, qs, m, pf_s, v_s, d, s);
+    } else {
+      rc = search(t, qs, m, pf_s, v_s, s);
+    }
     if (rc != HBT_OK) break;
-    bk_gather<K><<<grid, kThreads, smem_gather, s>>>(linv, m, tab, gb, B, chunks, pf_s, v_s, pf, (K*)v);
+    if (bs.items)
+      bk_gather_rec<K><<<unsigned(std::min<uint64_t>(chunks, t->num_sms)), kGThreads, smem_gather_rec, s>>>(
+          linv, m, tab, gb, B, chunks, reinterpret_cast<const ulonglong2*>(pf_s), pf, (K*)v);
+    else
+      bk_gather<K><<<grid, kThreads, smem_gather, s>>>(linv, m, tab, gb, B, chunks, pf_s, v_s, pf, (K*)v);
     if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) {
       set_error("bucket gather failed to launch: %s", cudaGetErrorString(e));
       rc = HBT_ECUDA;
@@ -454,6 +641,7 @@ int bucketed_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, 
 void bucket_free(hbt_tree* t) {
   cudaFree(t->bk.d_sp);
   cudaFree(t->bk.d_dir);
+  cudaFree(t->bk.d_M);
   t->bk = BucketState{};
 }
 

@@ -55,7 +55,30 @@ struct SearchConfig {
   uint32_t exchange = 0;         // sharded search: 0 = fused peer-memory exchange, 1 = NCCL send/recv
   uint64_t small_batch = 1u << 16;  // mode 2: batches up to this size read the directory in place (mode 3)
   uint32_t bucket = 2;           // query bucketing (bucketed.cu): 0 = off, 1 = on, 2 = auto
-  uint64_t bucket_slice = 0;     // tree bytes per bucket (0 = default 16 MB)
+  uint64_t bucket_slice = 0;     // tree bytes per bucket (0 = default 1 MB)
+  uint32_t bucket_items = 1;     // bucketed search: bucket-local shared-memory directory (ItemDir)
+  uint32_t bucket_cap = 0;       // item directory: shared-memory entries (0 = derived; tests force the fallback)
+};
+
+// Bucket-local directory of the bucketed search (bucketed.cu): after the
+// partition, the queries of a work item (kItem consecutive bucketed queries)
+// fall in the key range of a few consecutive buckets, so the item stages the
+// maxima of that range's UNITS into shared memory and finds each query's unit
+// by one lower bound there, skipping every level above it.
+//   implicit: unit = node of level `level` (level H = leaf lines), M[j] = max
+//             key below node j; the search continues at that level.
+//   regular:  unit = key line t of the last-level node of chain leaf c
+//             (entry c*span + t), M = its true max key; chain[c] = the leaf.
+struct ItemDir {
+  const void* M = nullptr;
+  const uint32_t* chain = nullptr;  // regular: chain ids
+  const uint64_t* bstart = nullptr; // B + 1 bucket starts in the bucketed order (bstart[B] = m)
+  uint32_t B = 0;
+  uint64_t U = 0;      // splitter units (implicit: leaf lines, regular: chain leaves)
+  uint32_t level = 0;  // implicit: level of the directory units
+  uint64_t span = 1;   // implicit: leaf lines per unit; regular: entries per chain leaf
+  uint64_t nunits = 0; // entries of M
+  uint32_t cap = 0;    // shared-memory entries (larger ranges search M in global memory)
 };
 
 // Query-bucketing state (bucketed.cu): B splitter keys and a prefix directory,
@@ -65,6 +88,11 @@ struct BucketState {
   uint32_t B = 0;
   void* d_sp = nullptr;          // B keys
   uint32_t* d_dir = nullptr;     // 2^12 x (u16 lo, u16 hi)
+  void* d_M = nullptr;           // item-directory unit maxima (ItemDir::M)
+  uint64_t M_cap = 0;            // bytes allocated
+  uint32_t level = 0;            // implicit: directory level
+  uint64_t span = 1, nunits = 0;
+  bool items = false;            // the item directory is in use
 };
 
 // Regular-tree device state.  All pools are SoA arrays
@@ -233,6 +261,12 @@ int regular_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, v
 int regular_update(hbt_tree* t, const hbt_batch* b, cudaStream_t s);
 void regular_free(hbt_tree* t);
 uint32_t regular_smem_levels(const hbt_tree* t, uint32_t budget);
+// Item-directory searches write 16 B records {pos|found, value (zero-extended)}
+// at pf (v is unused): rec[i] = (pf[2i], pf[2i+1]).
+int implicit_search_items(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v,
+                          const ItemDir& d, cudaStream_t s);
+int regular_search_items(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v,
+                         const ItemDir& d, cudaStream_t s);
 // bucketed.cu
 bool bucketed_enabled(const hbt_tree* t, uint64_t m);
 int bucketed_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s);

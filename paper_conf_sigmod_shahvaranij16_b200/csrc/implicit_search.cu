@@ -25,6 +25,7 @@
 #include <algorithm>
 
 #include "hbt_internal.cuh"
+#include "item_dir.cuh"
 
 namespace hbt {
 namespace {
@@ -95,6 +96,123 @@ __device__ __forceinline__ uint32_t count_less16(const V16<K>& v, K q, unsigned 
 #pragma unroll
   for (int e = 0; e < int(16 / sizeof(K)); ++e) c += __popc(__ballot_sync(0xffffffffu, v.k[e] < q) & gmask);
   return c;
+}
+
+// Phase 2 of a warp round: levels [d0, H) by lane groups, the leaf line, and the
+// results of the round (slot j of group g = round query j*NG + g, stored at
+// base + j*NG + g).  sec_known: the sector of level d0 is already in sec0.
+template <typename K, int F, int QPG, bool REC = false>
+__device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ inner,
+                                                  const uint8_t* __restrict__ inner_idx,
+                                                  const uint8_t* __restrict__ leaf, const LevelTable& lt,
+                                                  uint32_t d0, bool sec_known_d0, K (&q)[QPG], uint32_t (&node)[QPG],
+                                                  const uint32_t (&sec0)[QPG], int g, int k, unsigned gmask,
+                                                  uint64_t base, uint64_t m, uint64_t n, uint64_t pos_base,
+                                                  uint64_t* __restrict__ out_pf, K* __restrict__ out_v) {
+  using C = Cfg<K, F>;
+  const uint32_t H = lt.H;
+  for (uint32_t d = d0; d < H; ++d) {
+    const uint8_t* lvl = inner + lt.offset[d] * C::NODE_BYTES;
+    const bool sec_known = sec_known_d0 && d == d0;  // mode 4: the sector directory chose it
+    if constexpr (C::HAS_IDX) {
+      if (!sec_known && ((lt.full_mask >> d) & 1u)) {
+        // Level beyond the L2-resident budget: a miss costs a whole DRAM line
+        // anyway, so read the full node in ONE round trip (each of the G lanes
+        // loads NODE_BYTES/G contiguous bytes) instead of index + sector.
+        constexpr int NCH = C::NODE_BYTES / C::G / 16;
+        V16<K> fv[QPG][NCH];
+#pragma unroll
+        for (int j = 0; j < QPG; ++j)
+#pragma unroll
+          for (int h = 0; h < NCH; ++h)
+            ld16(fv[j][h], lvl + uint64_t(node[j]) * C::NODE_BYTES + (k * NCH + h) * 16);
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          uint32_t c = 0;
+#pragma unroll
+          for (int h = 0; h < NCH; ++h)
+#pragma unroll
+            for (int e = 0; e < 16 / C::S; ++e) c += (fv[j][h].k[e] < q[j]) ? 1u : 0u;
+#pragma unroll
+          for (int x = 1; x < C::G; x <<= 1) c += __shfl_xor_sync(0xffffffffu, c, x);
+          node[j] = node[j] * F + c;
+        }
+        continue;
+      }
+    }
+    uint32_t sec[QPG];
+    if (C::HAS_IDX && sec_known) {
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) sec[j] = sec0[j];
+    } else if constexpr (C::HAS_IDX) {
+      const uint8_t* lidx = inner_idx + lt.offset[d] * C::IDXB;
+      V16<K> iv[QPG];
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) {
+        if (k < C::IL) ld16(iv[j], lidx + uint64_t(node[j]) * C::IDXB + k * 16);
+        else fill_max(iv[j]);
+      }
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) sec[j] = count_less16(iv[j], q[j], gmask);
+    } else {
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) sec[j] = 0;
+    }
+    V16<K> kv[QPG];
+#pragma unroll
+    for (int j = 0; j < QPG; ++j) {
+      if (k < C::SL_) ld16(kv[j], lvl + uint64_t(node[j]) * C::NODE_BYTES + sec[j] * 32 + k * 16);
+      else fill_max(kv[j]);
+    }
+#pragma unroll
+    for (int j = 0; j < QPG; ++j) node[j] = node[j] * F + sec[j] * C::KPS + count_less16(kv[j], q[j], gmask);
+  }
+  // ---- leaf line [P keys | P values]: lanes 0 and 1 of the group each load one
+  //      16 B half of the key sector and of the value sector, so every load
+  //      instruction touches exactly one 32 B sector per group.
+  constexpr int E16 = 16 / C::S;
+  V16<K> lkey[QPG], lval[QPG];
+#pragma unroll
+  for (int j = 0; j < QPG; ++j) {
+    if (k < 2) {
+      const uint8_t* p = leaf + uint64_t(node[j]) * 64 + k * 16;
+      ld16(lkey[j], p);
+      ld16(lval[j], p + 32);
+    } else {
+      fill_max(lkey[j]);
+      fill_max(lval[j]);
+    }
+  }
+  uint64_t my_pf[QPG / C::G];
+  K my_v[QPG / C::G];
+#pragma unroll
+  for (int j = 0; j < QPG; ++j) {
+    const uint32_t s = count_less16(lkey[j], q[j], gmask);  // lanes >= 2 hold MAX
+    const uint32_t sc = s < uint32_t(C::P) ? s : uint32_t(C::P - 1);
+    const int src = g * C::G + int(sc / E16);
+    const K key_s = __shfl_sync(0xffffffffu, pick(lkey[j].k, sc % E16), src);
+    const K val_s = __shfl_sync(0xffffffffu, pick(lval[j].k, sc % E16), src);
+    const uint64_t r = uint64_t(node[j]) * C::P + s;
+    const bool found = (s < uint32_t(C::P)) && (r < n) && (key_s == q[j]);
+    if (j % C::G == k) {
+      my_pf[j / C::G] = (r < n ? r + pos_base : kEnd) | (found ? kFound : 0ull);
+      my_v[j / C::G] = found ? val_s : K(0);
+    }
+  }
+  // lane (g, k) stores slots j = k + G*t: round queries (k + G*t)*NG + g
+#pragma unroll
+  for (int t = 0; t < QPG / C::G; ++t) {
+    const uint64_t i = base + uint64_t(k + C::G * t) * C::NG + g;
+    if (i < m) {
+      if constexpr (REC) {
+        // 16 B record {pos|found, value} (bucketed search: the gather reads records)
+        __stcs(reinterpret_cast<ulonglong2*>(out_pf) + i, make_ulonglong2(my_pf[t], (unsigned long long)my_v[t]));
+      } else {
+        stcs(out_pf + i, my_pf[t]);
+        stcs(out_v + i, my_v[t]);
+      }
+    }
+  }
 }
 
 template <typename K, int F, int QPL, int THREADS, int MODE>
@@ -255,103 +373,111 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
       node[j] = __shfl_sync(0xffffffffu, mynode[(j * C::NG) / 32], src);
       sec0[j] = MODE == 4 ? __shfl_sync(0xffffffffu, mysec[(j * C::NG) / 32], src) : 0u;
     }
-    for (uint32_t d = SL; d < H; ++d) {
-      const uint8_t* lvl = inner + lt.offset[d] * C::NODE_BYTES;
-      const bool sec_known = MODE == 4 && d == SL;  // mode 4: the sector directory chose it
-      if constexpr (C::HAS_IDX) {
-        if (!sec_known && ((lt.full_mask >> d) & 1u)) {
-          // Level beyond the L2-resident budget: a miss costs a whole DRAM line
-          // anyway, so read the full node in ONE round trip (each of the G lanes
-          // loads NODE_BYTES/G contiguous bytes) instead of index + sector.
-          constexpr int NCH = C::NODE_BYTES / C::G / 16;
-          V16<K> fv[QPG][NCH];
+    descend_and_store<K, F, QPG>(inner, inner_idx, leaf, lt, SL, MODE == 4, q, node, sec0, g, k, gmask, base, m, n,
+                                 pos_base, out_pf, out_v);
+  }
+}
+
+
+// Bucketed search with a bucket-local directory (bucketed.cu, ItemDir).  One
+// persistent CTA works through items of kItemRounds * THREADS consecutive
+// bucketed queries.  Per item: the item's first and last queries give its bucket
+// range [b0, b1] (binary search over the staged bucket starts), hence a
+// contiguous range of level-`level` nodes [u0, u1] that contains every query's
+// node at that level: all nodes before u0 end at or below splitter b0-1 < q and
+// q <= splitter b1 <= max of node u1.  The maxima of [u0, u1] are staged in
+// shared memory; a query's node is u0 + lower_bound(maxima, q) (clamped to u1,
+// which only binds past the last key), exactly the node the root-first descent
+// reaches (every level picks the first child whose subtree max is >= q,
+// DESIGN.md R1/R3).  The rest of the walk is descend_and_store from that level.
+constexpr int kItemRounds = 16;
+
+// Cooperative copy of cnt keys into shared memory, four loads in flight per thread.
+template <typename K>
+__device__ __forceinline__ void stage_keys(K* dst, const K* __restrict__ src, uint32_t cnt, uint32_t threads) {
+  for (uint32_t i = threadIdx.x; i < cnt; i += 4 * threads) {
+    K x[4];
 #pragma unroll
-          for (int j = 0; j < QPG; ++j)
+    for (int u = 0; u < 4; ++u) x[u] = i + u * threads < cnt ? __ldg(src + i + u * threads) : K(0);
 #pragma unroll
-            for (int h = 0; h < NCH; ++h)
-              ld16(fv[j][h], lvl + uint64_t(node[j]) * C::NODE_BYTES + (k * NCH + h) * 16);
-#pragma unroll
-          for (int j = 0; j < QPG; ++j) {
-            uint32_t c = 0;
-#pragma unroll
-            for (int h = 0; h < NCH; ++h)
-#pragma unroll
-              for (int e = 0; e < 16 / C::S; ++e) c += (fv[j][h].k[e] < q[j]) ? 1u : 0u;
-#pragma unroll
-            for (int x = 1; x < C::G; x <<= 1) c += __shfl_xor_sync(0xffffffffu, c, x);
-            node[j] = node[j] * F + c;
-          }
-          continue;
-        }
+    for (int u = 0; u < 4; ++u)
+      if (i + u * threads < cnt) dst[i + u * threads] = x[u];
+  }
+}
+
+template <typename K, int F, int THREADS>
+__global__ void __launch_bounds__(THREADS)
+implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ inner_idx,
+                             const uint8_t* __restrict__ leaf, const ItemDir d, const K* __restrict__ queries,
+                             uint64_t m, uint64_t* __restrict__ out_pf, K* __restrict__ out_v, const LevelTable lt,
+                             uint64_t n) {
+  using C = Cfg<K, F>;
+  constexpr int QPG = 32 / C::NG;
+  constexpr uint64_t W = uint64_t(THREADS) * kItemRounds;
+  extern __shared__ __align__(16) uint8_t smem[];
+  uint64_t* s_bstart = reinterpret_cast<uint64_t*>(smem);
+  K* s_M = reinterpret_cast<K*>(s_bstart + d.B + 1);
+  uint32_t* s_T = reinterpret_cast<uint32_t*>(s_M + d.cap);
+  __shared__ uint64_t s_range[2];
+  const K* gM = static_cast<const K*>(d.M);
+  for (uint32_t i = threadIdx.x; i <= d.B; i += THREADS) s_bstart[i] = d.bstart[i];
+  __syncthreads();
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int g = lane / C::G, k = lane % C::G;
+  const unsigned gmask = ((1u << C::G) - 1u) << (g * C::G);
+  const uint64_t items = (m + W - 1) / W;
+  for (uint64_t it = blockIdx.x; it < items; it += gridDim.x) {
+    const uint64_t p0 = it * W, p1 = (p0 + W < m ? p0 + W : m) - 1;
+    if (threadIdx.x < 2) {
+      const uint64_t p = threadIdx.x ? p1 : p0;
+      uint32_t lo = 0, hi = d.B;  // largest b with bstart[b] <= p
+      while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (s_bstart[mid] <= p) lo = mid; else hi = mid;
       }
-      uint32_t sec[QPG];
-      if (C::HAS_IDX && sec_known) {
-#pragma unroll
-        for (int j = 0; j < QPG; ++j) sec[j] = sec0[j];
-      } else if constexpr (C::HAS_IDX) {
-        const uint8_t* lidx = inner_idx + lt.offset[d] * C::IDXB;
-        V16<K> iv[QPG];
-#pragma unroll
-        for (int j = 0; j < QPG; ++j) {
-          if (k < C::IL) ld16(iv[j], lidx + uint64_t(node[j]) * C::IDXB + k * 16);
-          else fill_max(iv[j]);
-        }
-#pragma unroll
-        for (int j = 0; j < QPG; ++j) sec[j] = count_less16(iv[j], q[j], gmask);
-      } else {
-#pragma unroll
-        for (int j = 0; j < QPG; ++j) sec[j] = 0;
+      const uint64_t lu = threadIdx.x ? ((uint64_t(lo) + 1) * d.U) / d.B - 1 : (uint64_t(lo) * d.U) / d.B;
+      s_range[threadIdx.x] = lu / d.span;
+    }
+    __syncthreads();
+    const uint64_t u0 = s_range[0], u1 = s_range[1];
+    const uint32_t cnt = uint32_t(u1 - u0 + 1);
+    const bool in_smem = cnt <= d.cap;
+    if (in_smem) stage_keys(s_M, gM + u0, cnt, THREADS);
+    __syncthreads();
+    PrefixTab<K> pt{};
+    if (in_smem) pt = build_prefix(s_M, cnt, s_T, THREADS);
+    __syncthreads();
+    const K* M = in_smem ? s_M : gM + u0;
+    // the next round's queries are loaded while this round walks the tree
+    K nextq;
+    {
+      const uint64_t i = p0 + uint64_t(wid) * 32 + lane;
+      nextq = i <= p1 ? ldcs(queries + i) : key_max<K>();
+    }
+#pragma unroll 1
+    for (int r = 0; r < kItemRounds; ++r) {
+      const uint64_t base = p0 + (uint64_t(r) * (THREADS / 32) + wid) * 32;
+      if (base > p1) break;
+      const K myq = nextq;
+      {
+        const uint64_t i = base + (THREADS / 32) * 32 + lane;
+        nextq = (r + 1 < kItemRounds && i <= p1) ? ldcs(queries + i) : key_max<K>();
       }
-      V16<K> kv[QPG];
+      const uint32_t lo = in_smem ? prefix_lower_bound(s_M, cnt, s_T, pt, myq) : lb_range(M, 0, cnt, myq);
+      const uint32_t mynode = uint32_t(u0) + (lo < cnt ? lo : cnt - 1);
+      K q[QPG];
+      uint32_t node[QPG], sec0[QPG];
 #pragma unroll
       for (int j = 0; j < QPG; ++j) {
-        if (k < C::SL_) ld16(kv[j], lvl + uint64_t(node[j]) * C::NODE_BYTES + sec[j] * 32 + k * 16);
-        else fill_max(kv[j]);
+        const int src = (j * C::NG) % 32 + g;
+        q[j] = __shfl_sync(0xffffffffu, myq, src);
+        node[j] = __shfl_sync(0xffffffffu, mynode, src);
+        sec0[j] = 0;
       }
-#pragma unroll
-      for (int j = 0; j < QPG; ++j) node[j] = node[j] * F + sec[j] * C::KPS + count_less16(kv[j], q[j], gmask);
+      descend_and_store<K, F, QPG, true>(inner, inner_idx, leaf, lt, d.level, false, q, node, sec0, g, k, gmask,
+                                         base, p1 + 1, n, 0, out_pf, out_v);
     }
-    // ---- leaf line [P keys | P values]: lanes 0 and 1 of the group each load one
-    //      16 B half of the key sector and of the value sector, so every load
-    //      instruction touches exactly one 32 B sector per group.
-    constexpr int E16 = 16 / C::S;
-    V16<K> lkey[QPG], lval[QPG];
-#pragma unroll
-    for (int j = 0; j < QPG; ++j) {
-      if (k < 2) {
-        const uint8_t* p = leaf + uint64_t(node[j]) * 64 + k * 16;
-        ld16(lkey[j], p);
-        ld16(lval[j], p + 32);
-      } else {
-        fill_max(lkey[j]);
-        fill_max(lval[j]);
-      }
-    }
-    uint64_t my_pf[QPG / C::G];
-    K my_v[QPG / C::G];
-#pragma unroll
-    for (int j = 0; j < QPG; ++j) {
-      const uint32_t s = count_less16(lkey[j], q[j], gmask);  // lanes >= 2 hold MAX
-      const uint32_t sc = s < uint32_t(C::P) ? s : uint32_t(C::P - 1);
-      const int src = g * C::G + int(sc / E16);
-      const K key_s = __shfl_sync(0xffffffffu, pick(lkey[j].k, sc % E16), src);
-      const K val_s = __shfl_sync(0xffffffffu, pick(lval[j].k, sc % E16), src);
-      const uint64_t r = uint64_t(node[j]) * C::P + s;
-      const bool found = (s < uint32_t(C::P)) && (r < n) && (key_s == q[j]);
-      if (j % C::G == k) {
-        my_pf[j / C::G] = (r < n ? r + pos_base : kEnd) | (found ? kFound : 0ull);
-        my_v[j / C::G] = found ? val_s : K(0);
-      }
-    }
-    // lane (g, k) stores slots j = k + G*t: round queries (k + G*t)*NG + g
-#pragma unroll
-    for (int t = 0; t < QPG / C::G; ++t) {
-      const uint64_t i = base + uint64_t(k + C::G * t) * C::NG + g;
-      if (i < m) {
-        stcs(out_pf + i, my_pf[t]);
-        stcs(out_v + i, my_v[t]);
-      }
-    }
+    __syncthreads();
   }
 }
 
@@ -460,6 +586,38 @@ struct Launch {
     return HBT_OK;
   }
 
+
+  static int run_items(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, const ItemDir& d,
+                       cudaStream_t s) {
+    constexpr int TH = C::NODE_BYTES > 128 ? 512 : 1024;
+    auto kern = implicit_search_items_kernel<K, F, TH>;
+    LevelTable lt{};
+    for (uint32_t x = 0; x <= t->H; ++x) lt.offset[x] = t->offset[x];
+    lt.H = t->H;
+    lt.SL = d.level;
+    {
+      uint64_t cum = 0;
+      const uint64_t budget = t->cfg.l2_levels_bytes ? t->cfg.l2_levels_bytes : (32ull << 20);
+      for (uint32_t x = d.level; x < t->H; ++x) {
+        cum += t->nodes[x] * uint64_t(C::NODE_BYTES + C::IDXB);
+        if (C::HAS_IDX && cum > budget && x < 32) lt.full_mask |= 1u << x;
+      }
+    }
+    const size_t smem = (d.B + 1) * 8 + size_t(d.cap) * C::S + ((1u << kPrefixBits) + 1) * 4;
+    static bool attr_set = false;
+    if (!attr_set) {
+      HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
+      attr_set = true;
+    }
+    uint64_t grid = t->num_sms;
+    const uint64_t items = (m + uint64_t(TH) * kItemRounds - 1) / (uint64_t(TH) * kItemRounds);
+    if (items < grid) grid = items ? items : 1;
+    kern<<<unsigned(grid), TH, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
+                                          (const uint8_t*)t->d_leaf, d, (const K*)q, m, pf, (K*)v, lt, t->n);
+    HBT_CUDA_TRY(cudaGetLastError());
+    return HBT_OK;
+  }
+
   static int run(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t b, cudaStream_t s) {
     const uint32_t qpl = t->cfg.qpl ? t->cfg.qpl : 1;
     // 256-byte nodes (u64, F = 32) need more registers than a 1024-thread CTA allows
@@ -522,6 +680,23 @@ int implicit_search_base(const hbt_tree* t, const void* q, uint64_t m, uint64_t*
                          cudaStream_t s) {
   if (m == 0) return HBT_OK;
   return t->width == 4 ? dispatch_f<uint32_t>(t, q, m, pf, v, base, s) : dispatch_f<uint64_t>(t, q, m, pf, v, base, s);
+}
+
+int implicit_search_items(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, const ItemDir& d,
+                          cudaStream_t s) {
+  if (m == 0) return HBT_OK;
+  auto go = [&](auto tag) -> int {
+    using K = decltype(tag);
+    switch (t->F) {
+      case 4: return Launch<K, 4>::run_items(t, q, m, pf, v, d, s);
+      case 8: return Launch<K, 8>::run_items(t, q, m, pf, v, d, s);
+      case 16: return Launch<K, 16>::run_items(t, q, m, pf, v, d, s);
+      case 32: return Launch<K, 32>::run_items(t, q, m, pf, v, d, s);
+    }
+    set_error("unsupported fanout %u", t->F);
+    return HBT_EINVAL;
+  };
+  return t->width == 4 ? go(uint32_t{}) : go(uint64_t{});
 }
 
 int implicit_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {

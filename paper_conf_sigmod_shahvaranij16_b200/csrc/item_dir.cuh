@@ -1,0 +1,60 @@
+// item_dir.cuh — the per-item prefix table of the bucket-local directory
+// (ItemDir, bucketed.cu).  After a work item has staged the sorted maxima
+// s_M[0, cnt) of its unit range, one table of 2^kPrefixBits + 1 lower bounds
+// over evenly spaced keys of [s_M[0], s_M[cnt-1]] narrows every query's lower
+// bound to a short slice, so a query costs one table read plus a few probes
+// instead of log2(cnt) bank-conflicted probes (ncu, profiles/r01_items_*: the
+// LSU pipe was 86-88 % busy, 60-70 % of it shared-memory bank conflicts).
+#pragma once
+
+#include <stdint.h>
+
+namespace hbt {
+
+constexpr uint32_t kPrefixBits = 10;
+
+template <typename K>
+__device__ __forceinline__ uint32_t lb_range(const K* s, uint32_t lo, uint32_t hi, K q) {
+  uint32_t len = hi - lo;
+  while (len > 0) {
+    const uint32_t half = len >> 1;
+    if (s[lo + half] < q) { lo += half + 1; len -= half + 1; } else { len = half; }
+  }
+  return lo;
+}
+
+template <typename K>
+struct PrefixTab {
+  K lo, span;
+  uint32_t sh;
+};
+
+// Builds s_T[p] = #{s_M < lo + p * 2^sh} for p in [0, 2^kPrefixBits] (cnt past
+// the range); (span >> sh) < 2^kPrefixBits.  Caller synchronises before use.
+template <typename K>
+__device__ __forceinline__ PrefixTab<K> build_prefix(const K* s_M, uint32_t cnt, uint32_t* s_T, uint32_t threads) {
+  PrefixTab<K> pt;
+  pt.lo = s_M[0];
+  pt.span = K(s_M[cnt - 1] - pt.lo);
+  const uint32_t bits = pt.span ? uint32_t(8 * sizeof(K)) - uint32_t(sizeof(K) == 8 ? __clzll((long long)pt.span)
+                                                                                    : __clz(int(pt.span)))
+                                : 0u;
+  pt.sh = bits > kPrefixBits ? bits - kPrefixBits : 0u;
+  const K pmax = K(pt.span >> pt.sh);
+  for (uint32_t p = threadIdx.x; p <= (1u << kPrefixBits); p += threads)
+    s_T[p] = K(p) > pmax ? cnt : lb_range(s_M, 0, cnt, K(pt.lo + (K(p) << pt.sh)));
+  return pt;
+}
+
+// lower_bound(s_M[0, cnt), q) through the table.
+template <typename K>
+__device__ __forceinline__ uint32_t prefix_lower_bound(const K* s_M, uint32_t cnt, const uint32_t* s_T,
+                                                       const PrefixTab<K>& pt, K q) {
+  if (q <= pt.lo) return 0;
+  const K d = K(q - pt.lo);
+  if (d > pt.span) return cnt;
+  const uint32_t p = uint32_t(d >> pt.sh);
+  return lb_range(s_M, s_T[p], s_T[p + 1], q);
+}
+
+}  // namespace hbt

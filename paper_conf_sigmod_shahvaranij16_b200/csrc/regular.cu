@@ -21,6 +21,7 @@
 #include <algorithm>
 
 #include "hbt_internal.cuh"
+#include "item_dir.cuh"
 
 namespace hbt {
 namespace {
@@ -568,6 +569,172 @@ regular_search_v2(const RView rv, const RDir rd, const uint32_t* __restrict__ di
   }
 }
 
+
+// Bucketed search with a bucket-local directory (bucketed.cu, ItemDir): per item
+// of kItemRounds * THREADS consecutive bucketed queries, the true maxima of the
+// key lines of the chain leaves [c0, c1] its buckets cover (and their chain
+// ids) are staged in shared memory.  A query's (chain leaf c, key line t) =
+// lower_bound over them: the root-first descent reaches the first big leaf whose
+// max is >= q (every upper separator is its child's max, the last one MAX, R11)
+// and in it the first key line whose index entry is >= q, and an index entry
+// equals the key line's true max except on the leaf's last used line (MAX),
+// where both rules stop anyway.  Then: key line t of last-level node v (one
+// 64 B access) -> slot j -> leaf line (v*F + j): two dependent accesses instead
+// of three per level.
+constexpr int kItemRounds = 16;
+
+// Cooperative copy of cnt elements into shared memory, four loads in flight per thread.
+template <typename T>
+__device__ __forceinline__ void stage4(T* dst, const T* __restrict__ src, uint32_t cnt, uint32_t threads) {
+  for (uint32_t i = threadIdx.x; i < cnt; i += 4 * threads) {
+    T x[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) x[u] = i + u * threads < cnt ? __ldg(src + i + u * threads) : T(0);
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (i + u * threads < cnt) dst[i + u * threads] = x[u];
+  }
+}
+
+template <typename K, int F, int THREADS>
+__global__ void __launch_bounds__(THREADS)
+regular_search_items_kernel(const RView rv, const ItemDir d, const K* __restrict__ queries, uint64_t m,
+                            uint64_t* __restrict__ out_pf, K* __restrict__ out_v) {
+  constexpr int G = 2, NG = 16, QPG = 32 / NG;
+  constexpr uint32_t S = sizeof(K), P = Geo<K>::P, KPL = Geo<K>::KPL;
+  constexpr uint32_t E16 = 16 / S;
+  constexpr uint32_t LINE = uint32_t(F) * S < 64 ? uint32_t(F) * S : 64;
+  constexpr int LCH = int(LINE / 16);
+  constexpr uint64_t W = uint64_t(THREADS) * kItemRounds;
+  extern __shared__ __align__(16) uint8_t smem[];
+  uint64_t* s_bstart = reinterpret_cast<uint64_t*>(smem);
+  K* s_M = reinterpret_cast<K*>(s_bstart + d.B + 1);
+  uint32_t* s_chain = reinterpret_cast<uint32_t*>(s_M + d.cap);
+  uint32_t* s_T = s_chain + d.cap;
+  __shared__ uint64_t s_range[2];
+  const K* gM = static_cast<const K*>(d.M);
+  const uint32_t NI = uint32_t(d.span);
+  for (uint32_t i = threadIdx.x; i <= d.B; i += THREADS) s_bstart[i] = d.bstart[i];
+  __syncthreads();
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int g = lane / G, k = lane % G;
+  const unsigned gmask = 3u << (g * G);
+  const uint64_t items = (m + W - 1) / W;
+  for (uint64_t it = blockIdx.x; it < items; it += gridDim.x) {
+    const uint64_t p0 = it * W, p1 = (p0 + W < m ? p0 + W : m) - 1;
+    if (threadIdx.x < 2) {
+      const uint64_t p = threadIdx.x ? p1 : p0;
+      uint32_t lo = 0, hi = d.B;  // largest b with bstart[b] <= p
+      while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (s_bstart[mid] <= p) lo = mid; else hi = mid;
+      }
+      s_range[threadIdx.x] = threadIdx.x ? ((uint64_t(lo) + 1) * d.U) / d.B - 1 : (uint64_t(lo) * d.U) / d.B;
+    }
+    __syncthreads();
+    const uint64_t c0 = s_range[0], c1 = s_range[1];
+    const uint32_t cnt = uint32_t((c1 - c0 + 1) * NI);
+    const bool in_smem = cnt <= d.cap;
+    if (in_smem) {
+      stage4(s_M, gM + c0 * NI, cnt, THREADS);
+      stage4(s_chain, d.chain + c0, uint32_t(c1 - c0 + 1), THREADS);
+    }
+    __syncthreads();
+    PrefixTab<K> pt{};
+    if (in_smem) pt = build_prefix(s_M, cnt, s_T, THREADS);
+    __syncthreads();
+    const K* M = in_smem ? s_M : gM + c0 * NI;
+    // the next round's queries are loaded while this round walks the tree
+    K nextq;
+    {
+      const uint64_t i = p0 + uint64_t(wid) * 32 + lane;
+      nextq = i <= p1 ? ldcs(queries + i) : key_max<K>();
+    }
+#pragma unroll 1
+    for (int r = 0; r < kItemRounds; ++r) {
+      const uint64_t base = p0 + (uint64_t(r) * (THREADS / 32) + wid) * 32;
+      if (base > p1) break;
+      const K myq = nextq;
+      {
+        const uint64_t i = base + (THREADS / 32) * 32 + lane;
+        nextq = (r + 1 < kItemRounds && i <= p1) ? ldcs(queries + i) : key_max<K>();
+      }
+      const uint32_t lo = in_smem ? prefix_lower_bound(s_M, cnt, s_T, pt, myq) : lb_range(M, 0, cnt, myq);
+      const uint32_t e = lo < cnt ? lo : cnt - 1;
+      const uint32_t myv = in_smem ? s_chain[e / NI] : __ldg(d.chain + c0 + e / NI);
+      const uint32_t myt = e % NI;
+      K q[QPG];
+      uint32_t cur[QPG], t[QPG];
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) {
+        const int src = (j * NG) % 32 + g;
+        q[j] = __shfl_sync(0xffffffffu, myq, src);
+        cur[j] = __shfl_sync(0xffffffffu, myv, src);
+        t[j] = __shfl_sync(0xffffffffu, myt, src);
+      }
+      // key line t of last-level node cur: lane k holds 16 B chunks k and k + 2
+      V16<K> kv[QPG][2];
+#pragma unroll
+      for (int j = 0; j < QPG; ++j)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int ch = k + 2 * h;
+          if (ch < LCH) kv[j][h] = ld16g<K>(rv.lkeys + (uint64_t(cur[j]) * F + t[j] * KPL) * S + ch * 16);
+          else {
+#pragma unroll
+            for (uint32_t x = 0; x < E16; ++x) kv[j][h].k[x] = key_max<K>();
+          }
+        }
+      uint32_t line[QPG];
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) {
+        uint32_t c = 0;
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+#pragma unroll
+          for (uint32_t x = 0; x < E16; ++x) c += __popc(__ballot_sync(0xffffffffu, kv[j][h].k[x] < q[j]) & gmask);
+        line[j] = t[j] * KPL + c;
+      }
+      // leaf line (cur*F + line): key sector + value sector, 16 B per lane each
+      V16<K> lk[QPG], lvv[QPG];
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) {
+        const uint8_t* p = rv.leaf + (uint64_t(cur[j]) * F + line[j]) * 64 + k * 16;
+        lk[j] = ld16g<K>(p);
+        lvv[j] = ld16g<K>(p + 32);
+      }
+      uint64_t my_pf = 0;
+      K my_v = 0;
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) {
+        uint32_t sl = 0;
+#pragma unroll
+        for (uint32_t x = 0; x < E16; ++x) sl += __popc(__ballot_sync(0xffffffffu, lk[j].k[x] < q[j]) & gmask);
+        const uint32_t sc = sl < P ? sl : P - 1;
+        const int src = g * G + int(sc / E16);
+        const K key_s = __shfl_sync(0xffffffffu, pick(lk[j].k, sc % E16), src);
+        const K val_s = __shfl_sync(0xffffffffu, pick(lvv[j].k, sc % E16), src);
+        bool end = (sl == P);
+        if (!end && key_s == key_max<K>()) {
+          // MAX slot: padding unless it is a counted entry ("must read the node size")
+          const int64_t in_line = int64_t(__ldg(rv.count + cur[j])) - int64_t(line[j]) * P;
+          const int64_t lim = in_line < int64_t(P) ? in_line : int64_t(P);
+          end = int64_t(sl) >= lim;
+        }
+        const bool found = !end && key_s == q[j];
+        if (j == k) {
+          my_pf = end ? kEnd : (((uint64_t(cur[j]) * F + line[j]) * P + sl) | (found ? kFound : 0ull));
+          my_v = found ? val_s : K(0);
+        }
+      }
+      const uint64_t o = base + uint64_t(k) * NG + g;
+      if (o <= p1)  // 16 B record {pos|found, value}: the bucket gather reads records
+        __stcs(reinterpret_cast<ulonglong2*>(out_pf) + o, make_ulonglong2(my_pf, (unsigned long long)my_v));
+    }
+    __syncthreads();
+  }
+}
+
 constexpr int kThreads = 512;
 constexpr int kQPG = 4;
 
@@ -688,6 +855,33 @@ int search_v2_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf,
   }
   HBT_CUDA_TRY(cudaLaunchKernelEx(&lc, kern, rv, rd, (const uint32_t*)r.d_dir, (const uint32_t*)r.d_chain, (const K*)q,
                                   m, pf, (K*)v));
+  return HBT_OK;
+}
+
+
+template <typename K, int F>
+int search_items_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, const ItemDir& d,
+                        cudaStream_t s) {
+  constexpr int TH = 1024;
+  const RegularState& r = t->r;
+  auto kern = regular_search_items_kernel<K, F, TH>;
+  RView rv{};
+  rv.leaf = (const uint8_t*)r.d_leaf;
+  rv.count = r.d_count;
+  rv.lkeys = (const uint8_t*)r.d_lkeys;
+  rv.lidx = (const uint8_t*)r.d_lidx;
+  rv.U = r.U;
+  const size_t smem = (d.B + 1) * 8 + size_t(d.cap) * (sizeof(K) + 4) + ((1u << kPrefixBits) + 1) * 4;
+  static bool attr = false;
+  if (!attr) {
+    HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
+    attr = true;
+  }
+  uint64_t grid = t->num_sms;
+  const uint64_t items = (m + uint64_t(TH) * kItemRounds - 1) / (uint64_t(TH) * kItemRounds);
+  if (items < grid) grid = items ? items : 1;
+  kern<<<unsigned(grid), TH, smem, s>>>(rv, d, (const K*)q, m, pf, (K*)v);
+  HBT_CUDA_TRY(cudaGetLastError());
   return HBT_OK;
 }
 
@@ -1366,6 +1560,23 @@ int regular_build(hbt_tree* t, const void* keys, const void* values, uint64_t n,
   HBT_CUDA_TRY(cudaMemset(t->r.d_seg_of_leaf, 0xFF, t->r.cap * 4));
   t->r.seg_cap = t->r.cap;
   return HBT_OK;
+}
+
+int regular_search_items(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, const ItemDir& d,
+                         cudaStream_t s) {
+  if (m == 0) return HBT_OK;
+  auto go = [&](auto tag) -> int {
+    using K = decltype(tag);
+    switch (t->F) {
+      case 4: return search_items_launch<K, 4>(t, q, m, pf, v, d, s);
+      case 8: return search_items_launch<K, 8>(t, q, m, pf, v, d, s);
+      case 16: return search_items_launch<K, 16>(t, q, m, pf, v, d, s);
+      case 32: return search_items_launch<K, 32>(t, q, m, pf, v, d, s);
+    }
+    set_error("unsupported fanout %u", t->F);
+    return HBT_EINVAL;
+  };
+  return t->width == 4 ? go(uint32_t{}) : go(uint64_t{});
 }
 
 int regular_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {

@@ -26,9 +26,13 @@ def _oracle(layout, k, v, F, width):
     return (oracle.ITree if layout == "implicit" else oracle.RTree).from_pairs(k, v, F, width)
 
 
+ITEM_MODES = [(0, 0), (1, 0), (1, 7)]  # (bucket_items, bucket_cap): plain search, smem directory, global fallback
+
+
 @pytest.mark.parametrize("layout", ["implicit", "regular"])
 @pytest.mark.parametrize("width,F", [(4, 8), (8, 16), (8, 32), (4, 32)])
-def test_bucketed_edge_suite(hbt, layout, width, F):
+@pytest.mark.parametrize("items,cap", ITEM_MODES)
+def test_bucketed_edge_suite(hbt, layout, width, F, items, cap):
     P = 64 // (2 * width)
     rng = np.random.default_rng(900 + 10 * F + width)
     for n in sorted({0, 1, 2, P + 1, F * P + 1, 5 * F * P + 3, 30011}):
@@ -39,16 +43,20 @@ def test_bucketed_edge_suite(hbt, layout, width, F):
         q = np.concatenate([q, np.array([0, kmax(width)] * 50, dtype=np.uint64)])
         epf, ev = o.search(q)
         t.set_param("bucket", 1)
+        t.set_param("bucket_items", items)
+        t.set_param("bucket_cap", cap)
         for slice_bytes in (1, 4096, 1 << 16):  # 1 B: one bucket per unit up to the 1024 cap
             t.set_param("bucket_slice", slice_bytes)
             pf, val = gpu_search(t, q, width)
-            assert np.array_equal(pf, epf), (layout, n, F, width, slice_bytes, np.nonzero(pf != epf)[0][:5])
-            assert np.array_equal(val, ev), (layout, n, F, width, slice_bytes)
+            assert np.array_equal(pf, epf), (layout, n, F, width, slice_bytes, items, cap,
+                                             np.nonzero(pf != epf)[0][:5])
+            assert np.array_equal(val, ev), (layout, n, F, width, slice_bytes, items, cap)
         t.close()
 
 
 @pytest.mark.parametrize("layout,F", [("implicit", 16), ("regular", 32)])
-def test_bucketed_scaled_workload(hbt, layout, F):
+@pytest.mark.parametrize("items,cap", ITEM_MODES)
+def test_bucketed_scaled_workload(hbt, layout, F, items, cap):
     """c2 / c3 recipes at reduced size, several bucket counts, every output vs the oracle."""
     cfg = "c2" if layout == "implicit" else "c3"
     n, m = 1 << 19, 1 << 20
@@ -58,6 +66,8 @@ def test_bucketed_scaled_workload(hbt, layout, F):
     epf, ev = o.search(q, nthreads=oracle.default_threads())
     t = gpu_build(hbt, k, v, F, 8, layout=layout)
     t.set_param("bucket", 1)
+    t.set_param("bucket_items", items)
+    t.set_param("bucket_cap", cap)
     for slice_bytes in (1 << 16, 1 << 20, 1 << 22):
         t.set_param("bucket_slice", slice_bytes)
         pf, val = gpu_search(t, q, 8)
@@ -69,7 +79,8 @@ def test_bucketed_scaled_workload(hbt, layout, F):
 
 
 @pytest.mark.parametrize("layout", ["implicit", "regular"])
-def test_bucketed_after_update(hbt, layout):
+@pytest.mark.parametrize("items,cap", ITEM_MODES)
+def test_bucketed_after_update(hbt, layout, items, cap):
     """The splitters follow the tree: search, update (keys move between buckets,
     regular leaves split / empty), search again."""
     width, F = 8, 8
@@ -79,6 +90,8 @@ def test_bucketed_after_update(hbt, layout):
     o = _oracle(layout, k, v, F, width)
     t = gpu_build(hbt, k, v, F, width, layout=layout)
     t.set_param("bucket", 1)
+    t.set_param("bucket_items", items)
+    t.set_param("bucket_cap", cap)
     t.set_param("bucket_slice", 2048)
     q = query_set(k, width, rng, 4000)
     pf, val = gpu_search(t, q, width)

@@ -1,6 +1,6 @@
 # Per-kernel device time and DRAM bytes of the bucketed pipeline (steady state, single pass).
 mkdir -p gpurun_out
-for spec in "c3 16777216" "c5 16777216"; do
+for spec in ${SPECS:-"c3 16777216" "c5 16777216"}; do
   set -- $spec
   timeout 900 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,lts__t_sector_hit_rate.pct,gpu__time_duration.sum \
     --cache-control none --clock-control none -k regex:"bk_|search" -s 12 -c 10 --csv \
