@@ -363,43 +363,82 @@ def run_hbt(args):
 
     e2e = time_e2e(work, args.e2e_steps, world) if not args.range_k else None
 
-    # ---- roofline of the step's dominant kernel (the search)
+    # ---- roofline of the step's dominant kernel.  Unbucketed: the step IS one search
+    # launch.  Bucketed (regular trees beyond the L2, csrc/bucketed.cu): the step is
+    # count / scan / scatter / search / gather; the library's phase events (CUDA events
+    # on the launching stream) give the tree-search kernel's own duration.
+    import paper_conf_sigmod_shahvaranij16_b200 as hbt
+    phases = None
+    if hasattr(work.tree, "last_phases") and not args.range_k:
+        try:
+            work.tree.set_param("phase_timing", 1)
+            acc = {}
+            reps = 5
+            for _ in range(reps):
+                step(work)
+                for k_, v_ in work.tree.last_phases().items():
+                    acc[k_] = acc.get(k_, 0.0) + v_
+            work.tree.set_param("phase_timing", 0)
+            phases = {k_: (round(v_ / reps, 4) if k_ != "launches" else int(v_ / reps)) for k_, v_ in acc.items()}
+        except hbt.HBTError:
+            phases = None
     l2_size = torch.cuda.get_device_properties(local).L2_cache_size
-    mdl = roofline.model(info, l2_size, work.hit_rate)
+    if phases:
+        mdl = roofline.model_bucketed(info, m)
+        t_kernel = phases["search"] * 1e-3
+        kernel = ("regular_search_items_kernel" if c["layout"] == "regular" else "implicit_search_items_kernel")
+        launches_per_step = phases["launches"]
+        model_desc = "bucketed search: query + 16 B record + distinct tree lines per pass (tools/roofline.py)"
+    else:
+        mdl = roofline.model(info, l2_size, work.hit_rate)
+        t_kernel = ms_step * 1e-3
+        kernel = ("regular_search_v2" if c["layout"] == "regular" else "implicit_search_kernel")
+        model_desc = "ideal static L2 cache of %d B (SURVEY §8d)%s" % (
+            l2_size, "; Zipf modelled as uniform (upper bound on bytes)" if args.config == "c5" else "")
     if args.range_k:  # + the further leaf lines walked and the k pairs written (+ count)
         P = 64 // (2 * w)
         extra_b = ((args.range_k - 1 + P - 1) // P) * 64 + args.range_k * 2 * w + 4
         mdl["hbm_bytes_per_query"] += extra_b
         mdl["l2_bytes_per_query"] += extra_b
+        kernel = "range_scan_kernel"
     peak, peak_src = measured_peaks()
-    t_kernel = ms_step * 1e-3
-    achieved = mdl["hbm_bytes_per_query"] * m / t_kernel / 1e9
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp) and not (args.config == "c4" and world > 1):  # measured on one GPU
         traffic = json.load(open(tp)).get(args.config)
-    traffic_bytes = traffic.get("dram_bytes_per_launch") if isinstance(traffic, dict) else None
-    roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-            "frac": round(achieved / peak, 4), "traffic": traffic_bytes,
-            "traffic_source": traffic.get("source") if isinstance(traffic, dict) else None,
-            # measured DRAM bytes of one launch (ncu, steady state) over this run's launch time:
-            # how busy HBM actually is (random 32 B sector misses move whole DRAM lines)
-            "traffic_gbs": round(traffic_bytes / t_kernel / 1e9, 1) if traffic_bytes and not args.range_k else None,
-            "traffic_frac": round(traffic_bytes / t_kernel / 1e9 / peak, 4) if traffic_bytes and not args.range_k else None,
-            "bytes_per_query_model": round(mdl["hbm_bytes_per_query"], 2), "peak_source": peak_src,
-            "model": "ideal static L2 cache of %d B (SURVEY §8d)%s" % (
-                l2_size, "; Zipf modelled as uniform (upper bound on bytes)" if args.config == "c5" else "")}
+    traffic_bytes = traffic.get("dram_bytes_per_launch") if isinstance(traffic, dict) and not args.range_k else None
+    hbm_ach = mdl["hbm_bytes_per_query"] * m / t_kernel / 1e9
+    roof_hbm = {"bound": "hbm", "achieved": round(hbm_ach, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(hbm_ach / peak, 4), "traffic": traffic_bytes,
+                "traffic_source": traffic.get("source") if isinstance(traffic, dict) else None,
+                # measured DRAM bytes of one launch (ncu, steady state) over this run's launch time
+                "traffic_gbs": round(traffic_bytes / t_kernel / 1e9, 1) if traffic_bytes else None,
+                "traffic_frac": round(traffic_bytes / t_kernel / 1e9 / peak, 4) if traffic_bytes else None,
+                "bytes_per_query_model": round(mdl["hbm_bytes_per_query"], 2), "peak_source": peak_src,
+                "model": model_desc}
     if args.config == "c4" and world > 1:
         a2a_b = (world - 1) / world * (w + 8 + w)
         t_roof = mdl["hbm_bytes_per_query"] / (peak * 1e9) + a2a_b / (NVLINK_GBS * 1e9)
-        roof["a2a_bytes_per_query"] = round(a2a_b, 2)
-        roof["frac_with_nvlink"] = round((m / t_kernel) * t_roof, 4)
-    l2_roof = None
+        roof_hbm["a2a_bytes_per_query"] = round(a2a_b, 2)
+        roof_hbm["frac_with_nvlink"] = round((m / t_kernel) * t_roof, 4)
+    roof_l2 = None
     if l2_probe:
         l2_ach = mdl["l2_bytes_per_query"] * m / t_kernel / 1e9
-        l2_roof = {"bound": "l2", "achieved": round(l2_ach, 1), "peak": round(l2_probe, 1), "unit": "GB/s",
-                   "frac": round(l2_ach / l2_probe, 4), "bytes_per_query_model": mdl["l2_bytes_per_query"],
-                   "peak_source": "in-run random-read probe, 32 MB buffer (tools/probe.cu)"}
+        roof_l2 = {"bound": "l2", "achieved": round(l2_ach, 1), "peak": round(l2_probe, 1), "unit": "GB/s",
+                   "frac": round(l2_ach / l2_probe, 4), "bytes_per_query_model": round(mdl["l2_bytes_per_query"], 2),
+                   "peak_source": "measured in this run: all-SM random 32 B reads of a 32 MB L2-resident buffer "
+                                  "(tools/probe.cu; SURVEY §8d BW_L2)"}
+    # roof time = max(B_HBM / BW_HBM, B_L2 / BW_L2); the binding term is the
+    # kernel's roofline, its frac = roof time / measured kernel time.
+    roof = dict(roof_l2 if roof_l2 and roof_l2["frac"] > roof_hbm["frac"] else roof_hbm)
+    roof["traffic"] = traffic_bytes
+    roof["kernel"] = kernel
+    roof["kernel_ms"] = round(t_kernel * 1e3, 4)
+    roof["frac_hbm"] = roof_hbm["frac"]
+    roof["frac_l2"] = roof_l2["frac"] if roof_l2 else None
+
+    if phases and e2e:  # each 4 Mi-query chunk of hbt_search_host runs the bucketed pipeline
+        e2e["gpu_launches_per_step"] *= phases["launches"]
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -436,7 +475,9 @@ def run_hbt(args):
             "e2e": e2e,
             "gpu_launches": args.steps * launches_per_step,
             "roofline": roof,
-            "roofline_l2": l2_roof,
+            "roofline_hbm": roof_hbm,
+            "roofline_l2": roof_l2,
+            "phases_ms": phases,
             "clocks": clocks,
             "cpu_baseline": cpu,
             "context": "paper: up to 240 M queries/s (HB+ implicit, GTX 780 + Xeon E5-2665, PAPER.md:9,57)",

@@ -187,8 +187,33 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *                 as whole nodes beyond it (0 = default 32 MB; 1 = every level whole)
  *   "exchange"    sharded search: 0 = fused peer-memory exchange (CUDA IPC windows, default),
  *                 1 = NCCL send/recv (multi-process) / device copies (hbt_search_sharded_local)
+ *   "bucket"      query bucketing before the tree walk (north_star "queries bucketed per batch"):
+ *                 0 = off, 1 = on, 2 = auto (default: regular trees larger than 8x the L2 and
+ *                 batches of >= 4 Mi queries).  The batch is partitioned into B key-range
+ *                 buckets, searched bucket after bucket, and the results are gathered back
+ *                 to query order; outputs are identical to the unbucketed search.
+ *   "bucket_slice" tree bytes per bucket (0 = default 1 MB; B <= 1024)
+ *   "bucket_items" bucketed search through a bucket-local shared-memory directory (1, default)
+ *                 or the normal search kernel on the bucketed queries (0)
+ *   "bucket_cap"  item-directory shared-memory entries (0 = derived; small values force the
+ *                 global-memory fallback, for tests)
+ *   "phase_timing" 1 = record CUDA events around the phases of each bucketed search (read
+ *                 them with hbt_last_phases), 0 = off (default)
  * Unknown names or out-of-range values return HBT_EINVAL. */
 HBT_API int hbt_set_param(hbt_tree* t, const char* name, int64_t value);
+
+/* Device time of the phases of the tree's last BUCKETED search (hbt_search with
+ * "bucket" in effect and "phase_timing" = 1), in milliseconds, measured with
+ * CUDA events recorded on the search's stream:
+ *   ms[0] bucket count   ms[1] scan   ms[2] scatter   ms[3] tree search   ms[4] gather
+ * `launches` = kernel launches of that search.  Synchronises on the last event.
+ * HBT_EINVAL if no timed bucketed search has run on this tree. */
+typedef struct {
+  uint32_t phases;    /* valid entries of ms (5) */
+  uint32_t launches;  /* kernels launched by the search */
+  float ms[8];
+} hbt_phase_times;
+HBT_API int hbt_last_phases(const hbt_tree* t, hbt_phase_times* out);
 
 /* ---- key-range sharding over G GPUs (one process per GPU), SURVEY §8(e) ----
  * Shard g holds a contiguous key range; shards are numbered in key order (the

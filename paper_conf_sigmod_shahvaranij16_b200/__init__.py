@@ -37,7 +37,7 @@ UPSERT, DELETE = 0, 1
 EXPORTED = ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
             "hbt_info", "hbt_export", "hbt_set_param", "hbt_last_error", "hbt_version",
             "hbt_range", "hbt_comm_unique_id", "hbt_comm_init", "hbt_comm_init_host", "hbt_comm_destroy", "hbt_bulk_build_sharded",
-            "hbt_search_sharded", "hbt_shard_local_init", "hbt_search_sharded_local"]
+            "hbt_search_sharded", "hbt_shard_local_init", "hbt_search_sharded_local", "hbt_last_phases"]
 
 
 class HBTError(RuntimeError):
@@ -52,6 +52,10 @@ class _Out(C.Structure):
 
 class _Batch(C.Structure):
     _fields_ = [("keys", C.c_void_p), ("values", C.c_void_p), ("ops", C.c_void_p), ("count", C.c_uint64)]
+
+
+class _Phases(C.Structure):
+    _fields_ = [("phases", C.c_uint32), ("launches", C.c_uint32), ("ms", C.c_float * 8)]
 
 
 class _Info(C.Structure):
@@ -89,13 +93,14 @@ def _load():
     L.hbt_shard_local_init.argtypes = [C.POINTER(vp), C.c_int]
     L.hbt_search_sharded_local.argtypes = [C.POINTER(vp), C.c_int, C.POINTER(vp), C.POINTER(u64),
                                            C.POINTER(_Out), vp]
+    L.hbt_last_phases.argtypes = [vp, vp]
     L.hbt_last_error.restype = C.c_char_p
     L.hbt_version.restype = C.c_char_p
     for f in ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
               "hbt_info", "hbt_export", "hbt_set_param", "hbt_range", "hbt_comm_unique_id", "hbt_comm_init",
               "hbt_comm_init_host",
               "hbt_comm_destroy", "hbt_bulk_build_sharded", "hbt_search_sharded", "hbt_shard_local_init",
-              "hbt_search_sharded_local"]:
+              "hbt_search_sharded_local", "hbt_last_phases"]:
         getattr(L, f).restype = C.c_int
     return L
 
@@ -244,6 +249,16 @@ class Tree:
 
     def set_param(self, name: str, value: int):
         _check(lib.hbt_set_param(self._h, name.encode(), int(value)))
+
+    PHASES = ("count", "scan", "scatter", "search", "gather")
+
+    def last_phases(self) -> dict:
+        """Device ms of each phase of the last bucketed search (needs set_param("phase_timing", 1))."""
+        p = _Phases()
+        _check(lib.hbt_last_phases(self._h, C.byref(p)))
+        d = {self.PHASES[i]: float(p.ms[i]) for i in range(p.phases)}
+        d["launches"] = int(p.launches)
+        return d
 
     def set_search_config(self, smem_bytes: int = 0, threads_per_cta: int = 0, ctas_per_sm: int = 0,
                           queries_per_lane: int = 0, smem_mode=None, carveout: int = -1):

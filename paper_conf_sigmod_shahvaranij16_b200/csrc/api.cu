@@ -279,6 +279,18 @@ int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t bytes, u
   return HBT_OK;
 }
 
+int hbt_last_phases(const hbt_tree* t, hbt_phase_times* out) {
+  if (!t || !out) { set_error("NULL argument"); return HBT_EINVAL; }
+  const BucketState& bs = t->bk;
+  if (!bs.timed) { set_error("no timed bucketed search on this tree"); return HBT_EINVAL; }
+  *out = hbt_phase_times{};
+  HBT_CUDA_TRY(cudaEventSynchronize(bs.ev[5]));
+  out->phases = 5;
+  out->launches = bs.launches;
+  for (int i = 0; i < 5; ++i) HBT_CUDA_TRY(cudaEventElapsedTime(&out->ms[i], bs.ev[i], bs.ev[i + 1]));
+  return HBT_OK;
+}
+
 int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   if (!t || !name) { set_error("NULL argument"); return HBT_EINVAL; }
   const std::string n(name);
@@ -297,6 +309,7 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "bucket_slice" && value >= 0) { c.bucket_slice = uint64_t(value); t->bk.valid = false; }
   else if (n == "bucket_items" && (value == 0 || value == 1)) { c.bucket_items = uint32_t(value); t->bk.valid = false; }
   else if (n == "bucket_cap" && value >= 0 && value < (1 << 20)) { c.bucket_cap = uint32_t(value); t->bk.valid = false; }
+  else if (n == "phase_timing" && (value == 0 || value == 1)) c.phase_timing = uint32_t(value);
   else {
     set_error("bad parameter %s = %lld", name, (long long)value);
     return HBT_EINVAL;

@@ -551,6 +551,13 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
   uint32_t* tab = reinterpret_cast<uint32_t*>(base + o_tab);
   uint32_t* gb = reinterpret_cast<uint32_t*>(base + o_gb);
   rc = HBT_OK;
+  BucketState& bw = t->bk;
+  const bool timing = t->cfg.phase_timing != 0;
+  if (timing && !bw.ev[0])
+    for (auto& e : bw.ev) HBT_CUDA_TRY(cudaEventCreate(&e));
+  auto mark = [&](int i) {
+    if (timing) cudaEventRecord(bw.ev[i], s);
+  };
   do {
     const size_t smem_count = (1u << kDirBits) * 4 + kMaxBuckets * 4 + kMaxBuckets * sizeof(K);
     const size_t smem_scatter = kChunk * (sizeof(K) + 2) + kMaxBuckets * 4 * 4 + kThreads * 4;
@@ -570,18 +577,22 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
       attr = true;
     }
     const unsigned grid = unsigned(std::min<uint64_t>(chunks, uint64_t(t->num_sms) * 2));
+    mark(0);
     bk_count<K><<<grid, kThreads, smem_count, s>>>((const K*)q, m, (const K*)bs.d_sp, bs.d_dir, B, chunks, bq, tab);
+    mark(1);
     if (cub::DeviceScan::ExclusiveSum(base + o_tmp, scan_bytes, tab, gb, ntab, s) != cudaSuccess) {
       set_error("bucket scan failed");
       rc = HBT_ECUDA;
       break;
     }
+    mark(2);
     bk_scatter<K><<<grid, kThreads, smem_scatter, s>>>((const K*)q, m, bq, tab, gb, B, chunks, qs, linv);
     if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) {
       set_error("bucketing kernels failed to launch: %s", cudaGetErrorString(e));
       rc = HBT_ECUDA;
       break;
     }
+    mark(3);
     if (bs.items) {
       uint64_t* bstart = reinterpret_cast<uint64_t*>(base + o_bs);
       bk_bstart<<<(B + 256) / 256, 256, 0, s>>>(gb, chunks, B, m, bstart);
@@ -602,6 +613,7 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
       rc = search(t, qs, m, pf_s, v_s, s);
     }
     if (rc != HBT_OK) break;
+    mark(4);
     if (bs.items)
       bk_gather_rec<K><<<unsigned(std::min<uint64_t>(chunks, t->num_sms)), kGThreads, smem_gather_rec, s>>>(
           linv, m, tab, gb, B, chunks, reinterpret_cast<const ulonglong2*>(pf_s), pf, (K*)v);
@@ -612,6 +624,10 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
       rc = HBT_ECUDA;
       break;
     }
+    mark(5);
+    // count, CUB scan (2), scatter, [bucket starts,] search, gather
+    bw.launches = bs.items ? 7u : 6u;
+    bw.timed = timing;
   } while (0);
   scratch_free(buf, s);
   return rc;
@@ -639,6 +655,8 @@ int bucketed_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, 
 }
 
 void bucket_free(hbt_tree* t) {
+  for (auto& e : t->bk.ev)
+    if (e) cudaEventDestroy(e);
   cudaFree(t->bk.d_sp);
   cudaFree(t->bk.d_dir);
   cudaFree(t->bk.d_M);

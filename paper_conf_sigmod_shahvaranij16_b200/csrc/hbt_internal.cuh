@@ -58,6 +58,7 @@ struct SearchConfig {
   uint64_t bucket_slice = 0;     // tree bytes per bucket (0 = default 1 MB)
   uint32_t bucket_items = 1;     // bucketed search: bucket-local shared-memory directory (ItemDir)
   uint32_t bucket_cap = 0;       // item directory: shared-memory entries (0 = derived; tests force the fallback)
+  uint32_t phase_timing = 0;     // bucketed search: CUDA events around each phase (hbt_last_phases)
 };
 
 // Bucket-local directory of the bucketed search (bucketed.cu): after the
@@ -93,6 +94,9 @@ struct BucketState {
   uint32_t level = 0;            // implicit: directory level
   uint64_t span = 1, nunits = 0;
   bool items = false;            // the item directory is in use
+  cudaEvent_t ev[6] = {};        // phase boundaries of the last timed bucketed search
+  bool timed = false;
+  uint32_t launches = 0;
 };
 
 // Regular-tree device state.  All pools are SoA arrays

@@ -83,3 +83,45 @@ def model(info, l2_bytes, hit_rate=1.0):
     hbm = io + static_cache_bytes(tiers, l2_bytes)
     l2 = io + sum(t[1] for t in tiers)
     return {"hbm_bytes_per_query": hbm, "l2_bytes_per_query": l2, "io_bytes_per_query": io}
+
+
+def _touched(units, m):
+    """Expected distinct units touched by m uniform accesses over `units` units."""
+    if units <= 0:
+        return 0.0
+    return units * (1.0 - np.exp(-float(m) / units))
+
+
+def model_bucketed(info, m, level=None):
+    """Algorithmic bytes per query of the BUCKETED tree search kernel (csrc/bucketed.cu,
+    item directory): the query in (S), the 16 B result record out, and the tree lines
+    below the shared-memory directory, each fetched from HBM once per pass when the
+    queries of a bucket share it (uniform queries: distinct lines touched = U (1 - e^(-m/U))).
+    regular: one 64 B key line of a last-level node + one 64 B leaf line per query;
+    implicit: the levels from `level` down (index sector + key sector, or the whole
+    node when wider than the L2 budget) + the 64 B leaf line.  The staged directory
+    maxima (S per unit) are read once per pass."""
+    S, F, n = info["width"], info["fanout"], info["n_distinct"]
+    P = 64 // (2 * S)
+    io = S + 16
+    if info["layout"] == 1:  # regular
+        kpl = 64 // S
+        ni = F // kpl if F > kpl else 1
+        key_lines = max(1.0, n / (kpl * P))
+        leaf_lines = max(1.0, n / P)
+        dram = (_touched(key_lines, m) * 64 + _touched(leaf_lines, m) * 64
+                + info["chain_len"] * (ni * S + 4)) / m
+        l2 = 64 + 64
+    else:
+        L0 = info["leaf_lines"]
+        lv = info["height"] if level is None else level
+        nodes = info["level_nodes"]
+        dram = _touched(L0, m) * 64 / m
+        l2 = 64
+        for d in range(lv, info["height"]):
+            node_b = F * S
+            dram += _touched(nodes[d], m) * node_b / m
+            l2 += 64 if node_b > 32 else _sect(node_b)
+        units = L0 if lv >= info["height"] else nodes[lv]
+        dram += units * S / m
+    return {"hbm_bytes_per_query": io + dram, "l2_bytes_per_query": io + l2, "io_bytes_per_query": io}

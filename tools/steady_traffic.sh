@@ -1,5 +1,5 @@
 # single-pass (no replay) DRAM bytes per launch of the search kernel, steady state, per config
-for spec in "c2 implicit_search" "c1 implicit_search" "c5 implicit_search" "c3 regular_search" "c4 implicit_search"; do
+for spec in "c2 implicit_search" "c1 implicit_search" "c5 implicit_search" "c3 regular_search_items" "c4 implicit_search"; do
   set -- $spec
   timeout 900 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,lts__t_sector_hit_rate.pct,gpu__time_duration.sum \
     --cache-control none --clock-control none -k regex:$2 -s 6 -c 2 --csv \
