@@ -9,7 +9,7 @@ import torch
 
 import gen
 import oracle
-from gpu_util import gpu_build, gpu_search, to_dev
+from gpu_util import GenLib, from_dev, gpu_build, gpu_search, to_dev
 from test_oracle_implicit import gen_keys, kmax, query_set
 
 pytestmark = pytest.mark.gpu
@@ -126,4 +126,53 @@ def test_bucketed_host_pipeline(hbt):
     t.search_host(q.copy(), pf, val)
     epf, ev = o.search(q, nthreads=oracle.default_threads())
     assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+    t.close()
+
+
+def _full_c3_tree(hbt):
+    c = gen.CONFIGS["c3"]
+    n, m, w = c["n"], c["m"], 8
+    g = GenLib()
+    sk = gen.stream_seed(c["cfg"], gen.STREAM_K)
+    sv = gen.stream_seed(c["cfg"], gen.STREAM_V)
+    sq = gen.stream_seed(c["cfg"], gen.STREAM_Q)
+    _, _, _, n_ins = gen.update_batch("c3", n)
+    t = hbt.Tree(g.mix_stream(n, w, sk), g.mix_stream(n, w, sv), fanout=c["fanout"], layout="regular")
+    dq = g.uniform_queries(m, n + n_ins, w, sq, sk)
+    return c, n, m, n_ins, sk, sv, sq, t, dq
+
+
+def test_c3_full_size_bench_launch(hbt):
+    """configs[2] at full size (2^27 u64 keys, F = 32, 2^26 queries) through the bench's
+    launch path: auto bucketing with the item directory (asserted via the phase timer),
+    before and after the 1 % bulk update.  ALL outputs: found iff the query index is a
+    built key, value = V_u; a 2^18 sample: pos|found and value equal the oracle's."""
+    c, n, m, n_ins, sk, sv, sq, t, dq = _full_c3_tree(hbt)
+    t.set_param("phase_timing", 1)
+    pf, val = t.search(dq)
+    torch.cuda.synchronize()
+    assert t.last_phases()["launches"] == 7  # count, scan x2, scatter, starts, item search, gather
+    pf = pf.cpu().numpy().view(np.uint64)
+    val = from_dev(val, 8)
+    u = gen.uniform_indices(m, n + n_ins, sq).astype(np.int64)
+    hit = u < n
+    v = gen.values(n, 8, sv)
+    assert np.array_equal((pf >> np.uint64(63)).astype(bool), hit)
+    assert np.array_equal(val[hit], v[u[hit]]) and not val[~hit].any()
+    k = gen.keys(n, 8, sk)
+    o = oracle.RTree.from_pairs(k, v, c["fanout"], 8)
+    idx = np.random.default_rng(5).integers(0, m, 1 << 18)
+    q = from_dev(dq, 8)[idx]
+    epf, ev = o.search(q, nthreads=oracle.default_threads())
+    assert np.array_equal(pf[idx], epf) and np.array_equal(val[idx], ev)
+    # the bench's 1 % update, then search again (splitters and item directory re-derived)
+    bk, bv, bo, _ = gen.update_batch("c3", n)
+    o.update(bk, bv, bo)
+    t.update(to_dev(bk, 8), to_dev(bv, 8), torch.from_numpy(bo).cuda())
+    pf, val = t.search(dq)
+    torch.cuda.synchronize()
+    pf = pf.cpu().numpy().view(np.uint64)
+    val = from_dev(val, 8)
+    epf, ev = o.search(q, nthreads=oracle.default_threads())
+    assert np.array_equal(pf[idx], epf) and np.array_equal(val[idx], ev)
     t.close()

@@ -268,3 +268,34 @@ def test_skewed_query_values(hbt, kind):
         pf, val = gpu_search(t, q, 8)
         epf, ev = o.search(q)
         assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+
+
+def test_c5_full_size_bench_launch(hbt):
+    """configs[4] at full size on one GPU (2^27 u64 keys, F = 16, 2^26 Zipf(0.99)
+    queries scrambled through the key order) through the bench's launch path.
+    ALL outputs: found, value = V_{r-1}, pos = rank of K_{r-1}; a 2^18 sample vs the oracle."""
+    c = gen.CONFIGS["c5"]
+    n, m, w = c["n"], c["m"], 8
+    g = GenLib()
+    sk = gen.stream_seed(c["cfg"], gen.STREAM_K)
+    sv = gen.stream_seed(c["cfg"], gen.STREAM_V)
+    sq = gen.stream_seed(c["cfg"], gen.STREAM_Q)
+    t = hbt.Tree(g.mix_stream(n, w, sk), g.mix_stream(n, w, sv), fanout=16, layout="implicit")
+    k = gen.keys(n, w, sk)
+    r = gen.zipf_ranks(m, n, c["theta"], sq)
+    q = k[r - 1]
+    pf, val = t.search(torch.from_numpy(q.view(np.int64)).cuda())
+    torch.cuda.synchronize()
+    pf = pf.cpu().numpy().view(np.uint64)
+    val = from_dev(val, w)
+    v = gen.values(n, w, sv)
+    rank = np.empty(n, np.int64)
+    rank[np.argsort(k, kind="stable")] = np.arange(n)
+    assert (pf >> np.uint64(63)).all()
+    assert np.array_equal(val, v[r - 1])
+    assert np.array_equal((pf & np.uint64(END)).astype(np.int64), rank[r - 1])
+    o = oracle.ITree.from_pairs(k, v, 16, w)
+    idx = np.random.default_rng(7).integers(0, m, 1 << 18)
+    epf, ev = o.search(q[idx], nthreads=oracle.default_threads())
+    assert np.array_equal(pf[idx], epf) and np.array_equal(val[idx], ev)
+    t.close()
