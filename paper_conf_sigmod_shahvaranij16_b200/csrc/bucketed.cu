@@ -150,29 +150,57 @@ __device__ __forceinline__ uint32_t bucket_of(K q, const K* s_sp, const uint32_t
   return lower_bound_in(s_sp, e & 0xFFFFu, e >> 16, q);
 }
 
-// Exclusive scan of s_in[0, B) into s_out (B <= 2 * kThreads) by one CTA; s_tmp
-// holds kThreads partial sums.  Ends with a barrier.
+// Exclusive scan of s_in[0, B) into s_out (B <= 2 * TH) by one CTA of TH threads:
+// two elements per thread, a shuffle scan per warp, the warp totals (s_tmp) scanned
+// by warp 0.  Ends with a barrier.
 template <int TH = kThreads>
 __device__ __forceinline__ void block_exclusive_scan(const uint32_t* s_in, uint32_t* s_out, uint32_t B,
                                                      uint32_t* s_tmp) {
-  const uint32_t t = threadIdx.x;
+  const uint32_t t = threadIdx.x, lane = t & 31, wid = t >> 5;
   const uint32_t a = 2 * t < B ? s_in[2 * t] : 0u, b = 2 * t + 1 < B ? s_in[2 * t + 1] : 0u;
-  s_tmp[t] = a + b;
-  __syncthreads();
-  for (uint32_t off = 1; off < TH; off <<= 1) {
-    const uint32_t x = t >= off ? s_tmp[t - off] : 0u;
-    __syncthreads();
-    s_tmp[t] += x;
-    __syncthreads();
+  uint32_t x = a + b;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= uint32_t(o)) x += y;
   }
-  const uint32_t ex = s_tmp[t] - (a + b);
+  if (lane == 31) s_tmp[wid] = x;
+  __syncthreads();
+  if (wid == 0) {
+    uint32_t w = lane < uint32_t(TH / 32) ? s_tmp[lane] : 0u;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, w, o);
+      if (lane >= uint32_t(o)) w += y;
+    }
+    if (lane < uint32_t(TH / 32)) s_tmp[lane] = w;
+  }
+  __syncthreads();
+  const uint32_t ex = x - (a + b) + (wid ? s_tmp[wid - 1] : 0u);
   if (2 * t < B) s_out[2 * t] = ex;
   if (2 * t + 1 < B) s_out[2 * t + 1] = ex + a;
   __syncthreads();
 }
 
+// Tile transpose of a rows x cols u32 matrix (row-major) into cols x rows.
+__global__ void bk_transpose(const uint32_t* __restrict__ in, uint64_t rows, uint32_t cols,
+                             uint32_t* __restrict__ out) {
+  __shared__ uint32_t tile[32][33];
+  const uint64_t r0 = uint64_t(blockIdx.y) * 32, c0 = uint64_t(blockIdx.x) * 32;
+  for (uint32_t i = threadIdx.y; i < 32; i += blockDim.y) {
+    const uint64_t r = r0 + i, c = c0 + threadIdx.x;
+    if (r < rows && c < cols) tile[i][threadIdx.x] = in[r * cols + c];
+  }
+  __syncthreads();
+  for (uint32_t i = threadIdx.y; i < 32; i += blockDim.y) {
+    const uint64_t c = c0 + i, r = r0 + threadIdx.x;
+    if (r < rows && c < cols) out[c * rows + r] = tile[threadIdx.x][i];
+  }
+}
+
 // Pass 1: bucket of every query (bq, u16) and the per-chunk histograms, stored
-// bucket-major: tab[b * chunks + c] = #queries of chunk c in bucket b.
+// chunk-major: tabT[c * B + b] = #queries of chunk c in bucket b (coalesced; the
+// scan runs on its bucket-major transpose).
 template <typename K>
 __global__ void __launch_bounds__(kThreads) bk_count(const K* __restrict__ q, uint64_t m, const K* __restrict__ sp,
                                                      const uint32_t* __restrict__ dir, uint32_t B, uint64_t chunks,
@@ -203,21 +231,21 @@ __global__ void __launch_bounds__(kThreads) bk_count(const K* __restrict__ q, ui
       }
     }
     __syncthreads();
-    for (uint32_t b = threadIdx.x; b < B; b += kThreads) tab[uint64_t(b) * chunks + c] = s_h[b];
+    for (uint32_t b = threadIdx.x; b < B; b += kThreads) tab[c * B + b] = s_h[b];
     __syncthreads();
   }
 }
 
-// Per-chunk bucket layout shared by the scatter and the gather: s_cnt (this
-// chunk's count per bucket), s_lb (their exclusive scan = the bucket's start in
+// Per-chunk bucket layout shared by the scatter and the gather (tab, gb
+// chunk-major): s_cnt (this chunk's count per bucket), s_lb (their exclusive scan = the bucket's start in
 // the chunk's bucket-sorted order), s_gb (the run's first global slot).
 template <int TH = kThreads>
 __device__ __forceinline__ void chunk_layout(const uint32_t* __restrict__ tab, const uint32_t* __restrict__ gb,
                                              uint32_t B, uint64_t chunks, uint64_t c, uint32_t* s_cnt,
                                              uint32_t* s_lb, uint32_t* s_gb, uint32_t* s_tmp) {
-  for (uint32_t b = threadIdx.x; b < B; b += TH) {
-    s_cnt[b] = tab[uint64_t(b) * chunks + c];
-    s_gb[b] = gb[uint64_t(b) * chunks + c];
+  for (uint32_t b = threadIdx.x; b < B; b += TH) {  // chunk-major rows: coalesced
+    s_cnt[b] = tab[c * B + b];
+    s_gb[b] = gb[c * B + b];
   }
   __syncthreads();
   block_exclusive_scan<TH>(s_cnt, s_lb, B, s_tmp);
@@ -538,7 +566,8 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
   // pf_s + v_s (plain search) or 16 B records (item directory: o_pf .. o_pf + 16 m)
   const uint64_t o_pf = al(m * sizeof(K)), o_v = o_pf + al(m * 8), o_bq = o_v + al(m * 8),
                  o_li = o_bq + al(m * 2), o_tab = o_li + al(m * 2), o_gb = o_tab + al(ntab * 4),
-                 o_bs = o_gb + al(ntab * 4), o_tmp = o_bs + al((uint64_t(B) + 1) * 8),
+                 o_bm = o_gb + al(ntab * 4), o_bm2 = o_bm + al(ntab * 4),
+                 o_bs = o_bm2 + al(ntab * 4), o_tmp = o_bs + al((uint64_t(B) + 1) * 8),
                  total = o_tmp + al(scan_bytes);
   void* buf = nullptr;
   HBT_CUDA_TRY(scratch_alloc(&buf, total, s));
@@ -580,10 +609,22 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
     mark(0);
     bk_count<K><<<grid, kThreads, smem_count, s>>>((const K*)q, m, (const K*)bs.d_sp, bs.d_dir, B, chunks, bq, tab);
     mark(1);
-    if (cub::DeviceScan::ExclusiveSum(base + o_tmp, scan_bytes, tab, gb, ntab, s) != cudaSuccess) {
-      set_error("bucket scan failed");
-      rc = HBT_ECUDA;
-      break;
+    {
+      // chunk-major counts -> bucket-major, exclusive scan (run starts), -> chunk-major
+      uint32_t* tab_bm = reinterpret_cast<uint32_t*>(base + o_bm);
+      uint32_t* gb_bm = reinterpret_cast<uint32_t*>(base + o_bm2);
+      const dim3 tb(32, 8);
+      bk_transpose<<<dim3((B + 31) / 32, unsigned((chunks + 31) / 32)), tb, 0, s>>>(tab, chunks, B, tab_bm);
+      if (cub::DeviceScan::ExclusiveSum(base + o_tmp, scan_bytes, tab_bm, gb_bm, ntab, s) != cudaSuccess) {
+        set_error("bucket scan failed");
+        rc = HBT_ECUDA;
+        break;
+      }
+      bk_transpose<<<dim3(unsigned((chunks + 31) / 32), (B + 31) / 32), tb, 0, s>>>(gb_bm, B, uint32_t(chunks), gb);
+      if (bs.items) {
+        uint64_t* bstart = reinterpret_cast<uint64_t*>(base + o_bs);
+        bk_bstart<<<(B + 256) / 256, 256, 0, s>>>(gb_bm, chunks, B, m, bstart);
+      }
     }
     mark(2);
     bk_scatter<K><<<grid, kThreads, smem_scatter, s>>>((const K*)q, m, bq, tab, gb, B, chunks, qs, linv);
@@ -595,7 +636,6 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
     mark(3);
     if (bs.items) {
       uint64_t* bstart = reinterpret_cast<uint64_t*>(base + o_bs);
-      bk_bstart<<<(B + 256) / 256, 256, 0, s>>>(gb, chunks, B, m, bstart);
       ItemDir d;
       d.M = bs.d_M;
       d.chain = t->form == HBT_REGULAR ? t->r.d_chain : nullptr;
@@ -625,8 +665,8 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
       break;
     }
     mark(5);
-    // count, CUB scan (2), scatter, [bucket starts,] search, gather
-    bw.launches = bs.items ? 7u : 6u;
+    // count, transpose, CUB scan (2), transpose, [bucket starts,] scatter, search, gather
+    bw.launches = bs.items ? 9u : 8u;
     bw.timed = timing;
   } while (0);
   scratch_free(buf, s);

@@ -151,7 +151,7 @@ def test_c3_full_size_bench_launch(hbt):
     t.set_param("phase_timing", 1)
     pf, val = t.search(dq)
     torch.cuda.synchronize()
-    assert t.last_phases()["launches"] == 7  # count, scan x2, scatter, starts, item search, gather
+    assert t.last_phases()["launches"] == 9  # count, transpose, scan x2, transpose, starts, scatter, search, gather
     pf = pf.cpu().numpy().view(np.uint64)
     val = from_dev(val, 8)
     u = gen.uniform_indices(m, n + n_ins, sq).astype(np.int64)
