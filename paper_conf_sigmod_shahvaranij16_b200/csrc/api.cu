@@ -77,7 +77,7 @@ static void free_tree(hbt_tree* t) {
 }
 
 static int device_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
-  if (bucketed_enabled(t, m)) return bucketed_search(t, q, m, pf, v, s);
+  if (bucketed_enabled(t, m)) return bucketed_search(t, q, m, pf, v, 0, s);
   return t->form == HBT_REGULAR ? regular_search(t, q, m, pf, v, s) : implicit_search(t, q, m, pf, v, s);
 }
 
@@ -310,6 +310,7 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "bucket_items" && (value == 0 || value == 1)) { c.bucket_items = uint32_t(value); t->bk.valid = false; }
   else if (n == "bucket_cap" && value >= 0 && value < (1 << 20)) { c.bucket_cap = uint32_t(value); t->bk.valid = false; }
   else if (n == "phase_timing" && (value == 0 || value == 1)) c.phase_timing = uint32_t(value);
+  else if (n == "leaf256" && (value == 0 || value == 1)) c.leaf256 = uint32_t(value);
   else {
     set_error("bad parameter %s = %lld", name, (long long)value);
     return HBT_EINVAL;

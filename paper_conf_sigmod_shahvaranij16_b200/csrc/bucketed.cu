@@ -550,8 +550,8 @@ int prepare_splitters(const hbt_tree* t, cudaStream_t s) {
 }
 
 template <typename K>
-int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s,
-               int (*search)(const hbt_tree*, const void*, uint64_t, uint64_t*, void*, cudaStream_t)) {
+int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
+               cudaStream_t s) {
   int rc = prepare_splitters<K>(t, s);
   if (rc != HBT_OK) return rc;
   const BucketState& bs = t->bk;
@@ -645,12 +645,14 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
       d.level = bs.level;
       d.span = bs.span;
       d.nunits = bs.nunits;
+      d.pos_base = pos_base;
       d.cap = t->cfg.bucket_cap ? std::min<uint32_t>(t->cfg.bucket_cap, uint32_t(item_cap(t, B)))
                                 : uint32_t(item_cap(t, B));
       rc = t->form == HBT_IMPLICIT ? implicit_search_items(t, qs, m, pf_s, v_s, d, s)
                                    : regular_search_items(t, qs, m, pf_s, v_s, d, s);
     } else {
-      rc = search(t, qs, m, pf_s, v_s, s);
+      rc = t->form == HBT_REGULAR ? regular_search(t, qs, m, pf_s, v_s, s)
+                                  : implicit_search_base(t, qs, m, pf_s, v_s, pos_base, s);
     }
     if (rc != HBT_OK) break;
     mark(4);
@@ -677,21 +679,29 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
 
 bool bucketed_enabled(const hbt_tree* t, uint64_t m) {
   const uint32_t mode = t->cfg.bucket;
-  if (mode == 0) return false;
-  if (m >= (1ull << 32) || pick_buckets(t) < 2) return false;
+  if (mode == 0 || m >= (1ull << 32)) return false;
+  if (mode == 2 && m < (1ull << 22)) return false;  // auto: small batches never (no host calls)
+  if (pick_buckets(t) < 2) return false;
   if (mode == 1) return true;
-  // auto: regular trees well beyond the L2 and batches large enough to share
-  // lines (measured, profiles/r01_bucket_*: c3 10.8 -> 15.2 G q/s; the implicit
-  // c5 tree under Zipf queries already hits L2 and loses, 23.1 -> 19.6)
-  int l2 = 0;
-  cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, t->device);
-  return t->form == HBT_REGULAR && tree_bytes(t) > 8ull * uint64_t(l2) && m >= (1ull << 22);
+  // auto: batches large enough to share lines, regular trees beyond 8x the L2
+  // (measured: c3 10.9 -> 21.0 G q/s), implicit trees beyond 64x (the 2.1 GB c5
+  // tree gains nothing under uniform values, 18.3 -> 18.8, and loses under Zipf,
+  // 23.1 -> 19.9, whose hot set already lives in L2)
+  static int l2 = 0;  // one device model per process
+  if (!l2) cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, t->device);
+  return t->form == HBT_REGULAR ? tree_bytes(t) > 8ull * uint64_t(l2) : tree_bytes(t) > 64ull * uint64_t(l2);
 }
 
-int bucketed_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
-  auto search = t->form == HBT_REGULAR ? regular_search : implicit_search;
-  return t->width == 4 ? bucketed_t<uint32_t>(t, q, m, pf, v, s, search)
-                       : bucketed_t<uint64_t>(t, q, m, pf, v, s, search);
+int bucketed_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
+                    cudaStream_t s) {
+  return t->width == 4 ? bucketed_t<uint32_t>(t, q, m, pf, v, pos_base, s)
+                       : bucketed_t<uint64_t>(t, q, m, pf, v, pos_base, s);
+}
+
+int shard_local_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
+                       cudaStream_t s) {
+  if (bucketed_enabled(t, m)) return bucketed_search(t, q, m, pf, v, pos_base, s);
+  return implicit_search_base(t, q, m, pf, v, pos_base, s);
 }
 
 void bucket_free(hbt_tree* t) {

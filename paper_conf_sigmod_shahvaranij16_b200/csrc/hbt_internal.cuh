@@ -41,6 +41,7 @@ struct LevelTable {
   uint32_t dcount;  // mode 2/3: nodes at level T; mode 4: sectors at level T
   uint32_t dbits;   // mode 2/3/4: directory prefix bits
   uint32_t full_mask;  // bit d: read level d's nodes whole (not index + sector)
+  uint32_t leaf256;    // leaf line read as one 64 B request (two 256-bit lane loads)
 };
 
 struct SearchConfig {
@@ -59,6 +60,7 @@ struct SearchConfig {
   uint32_t bucket_items = 1;     // bucketed search: bucket-local shared-memory directory (ItemDir)
   uint32_t bucket_cap = 0;       // item directory: shared-memory entries (0 = derived; tests force the fallback)
   uint32_t phase_timing = 0;     // bucketed search: CUDA events around each phase (hbt_last_phases)
+  uint32_t leaf256 = 1;          // leaf line by two 256-bit lane loads (one 64 B request per group)
 };
 
 // Bucket-local directory of the bucketed search (bucketed.cu): after the
@@ -80,6 +82,7 @@ struct ItemDir {
   uint64_t span = 1;   // implicit: leaf lines per unit; regular: entries per chain leaf
   uint64_t nunits = 0; // entries of M
   uint32_t cap = 0;    // shared-memory entries (larger ranges search M in global memory)
+  uint64_t pos_base = 0;  // implicit: added to every reported position (key-range shards)
 };
 
 // Query-bucketing state (bucketed.cu): B splitter keys and a prefix directory,
@@ -273,6 +276,10 @@ int regular_search_items(const hbt_tree* t, const void* q, uint64_t m, uint64_t*
                          const ItemDir& d, cudaStream_t s);
 // bucketed.cu
 bool bucketed_enabled(const hbt_tree* t, uint64_t m);
-int bucketed_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s);
+int bucketed_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
+                    cudaStream_t s);
+// the owner-side search of the sharded paths: bucketed when enabled, positions + pos_base
+int shard_local_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
+                       cudaStream_t s);
 void bucket_free(hbt_tree* t);
 }  // namespace hbt

@@ -51,6 +51,26 @@ __device__ __forceinline__ void ld16(V16<K>& v, const uint8_t* p) {
   v.u = __ldg(reinterpret_cast<const uint4*>(p));
 }
 
+// 32 B held by one lane (a whole sector), loaded with one 256-bit load (sm_100).
+template <typename K>
+union L256 {
+  unsigned long long u[4];
+  K k[32 / sizeof(K)];
+};
+
+template <typename K>
+__device__ __forceinline__ void ld32(L256<K>& v, const uint8_t* p) {
+  asm volatile("ld.global.nc.v4.u64 {%0, %1, %2, %3}, [%4];"
+               : "=l"(v.u[0]), "=l"(v.u[1]), "=l"(v.u[2]), "=l"(v.u[3])
+               : "l"(p));
+}
+
+template <typename K>
+__device__ __forceinline__ void fill_max32(L256<K>& v) {
+#pragma unroll
+  for (int e = 0; e < 4; ++e) v.u[e] = ~0ull;
+}
+
 template <typename K>
 __device__ __forceinline__ void fill_max(V16<K>& v) {
 #pragma unroll
@@ -167,6 +187,36 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
 #pragma unroll
     for (int j = 0; j < QPG; ++j) node[j] = node[j] * F + sec[j] * C::KPS + count_less16(kv[j], q[j], gmask);
   }
+  uint64_t my_pf[QPG / C::G];
+  K my_v[QPG / C::G];
+  if (lt.leaf256) {
+    // ---- leaf line [P keys | P values] in ONE 64 B request per group: lane 0 loads
+    //      the key sector, lane 1 the value sector with 256-bit loads (sm_100).
+    //      s = #{keys < q} on lane 0, broadcast; key / value picked by lanes 0 / 1.
+    L256<K> lw[QPG];
+#pragma unroll
+    for (int j = 0; j < QPG; ++j) {
+      if (k < 2) ld32(lw[j], leaf + uint64_t(node[j]) * 64 + k * 32);
+      else fill_max32(lw[j]);
+    }
+#pragma unroll
+    for (int j = 0; j < QPG; ++j) {
+      uint32_t c = 0;
+#pragma unroll
+      for (int e = 0; e < C::P; ++e) c += (lw[j].k[e] < q[j]) ? 1u : 0u;
+      const uint32_t s = __shfl_sync(0xffffffffu, c, g * C::G);
+      const uint32_t sc = s < uint32_t(C::P) ? s : uint32_t(C::P - 1);
+      const K x = pick(lw[j].k, sc);
+      const K key_s = __shfl_sync(0xffffffffu, x, g * C::G);
+      const K val_s = __shfl_sync(0xffffffffu, x, g * C::G + 1);
+      const uint64_t r = uint64_t(node[j]) * C::P + s;
+      const bool found = (s < uint32_t(C::P)) && (r < n) && (key_s == q[j]);
+      if (j % C::G == k) {
+        my_pf[j / C::G] = (r < n ? r + pos_base : kEnd) | (found ? kFound : 0ull);
+        my_v[j / C::G] = found ? val_s : K(0);
+      }
+    }
+  } else {
   // ---- leaf line [P keys | P values]: lanes 0 and 1 of the group each load one
   //      16 B half of the key sector and of the value sector, so every load
   //      instruction touches exactly one 32 B sector per group.
@@ -183,8 +233,6 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
       fill_max(lval[j]);
     }
   }
-  uint64_t my_pf[QPG / C::G];
-  K my_v[QPG / C::G];
 #pragma unroll
   for (int j = 0; j < QPG; ++j) {
     const uint32_t s = count_less16(lkey[j], q[j], gmask);  // lanes >= 2 hold MAX
@@ -198,6 +246,7 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
       my_pf[j / C::G] = (r < n ? r + pos_base : kEnd) | (found ? kFound : 0ull);
       my_v[j / C::G] = found ? val_s : K(0);
     }
+  }
   }
   // lane (g, k) stores slots j = k + G*t: round queries (k + G*t)*NG + g
 #pragma unroll
@@ -475,7 +524,7 @@ implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* _
         sec0[j] = 0;
       }
       descend_and_store<K, F, QPG, true>(inner, inner_idx, leaf, lt, d.level, false, q, node, sec0, g, k, gmask,
-                                         base, p1 + 1, n, 0, out_pf, out_v);
+                                         base, p1 + 1, n, d.pos_base, out_pf, out_v);
     }
     __syncthreads();
   }
@@ -501,6 +550,7 @@ struct Launch {
     // Levels whose cumulative footprint (from the first global level down) exceeds
     // the L2-resident budget are read as whole nodes (see the kernel).
     lt.full_mask = 0;
+    lt.leaf256 = t->cfg.leaf256;
     size_t smem;
     if (MODE == 4) {
       lt.SL = t->dir_T;
@@ -595,6 +645,7 @@ struct Launch {
     for (uint32_t x = 0; x <= t->H; ++x) lt.offset[x] = t->offset[x];
     lt.H = t->H;
     lt.SL = d.level;
+    lt.leaf256 = t->cfg.leaf256;
     {
       uint64_t cum = 0;
       const uint64_t budget = t->cfg.l2_levels_bytes ? t->cfg.l2_levels_bytes : (32ull << 20);

@@ -193,6 +193,7 @@ struct RView {
   uint32_t root_leaf; // big leaf when U == 0
   uint64_t smem_first;  // pool index of the first staged upper node
   uint64_t smem_nodes;
+  uint32_t leaf256;     // item search: key line and leaf line by 256-bit lane loads
 };
 
 template <typename K, int N>
@@ -208,6 +209,26 @@ union V16 {
   uint4 u;
   K k[16 / sizeof(K)];
 };
+
+// 32 B held by one lane, loaded with one 256-bit load (sm_100)
+template <typename K>
+union L256 {
+  unsigned long long u[4];
+  K k[32 / sizeof(K)];
+};
+
+template <typename K>
+__device__ __forceinline__ void ld32(L256<K>& v, const uint8_t* p) {
+  asm volatile("ld.global.nc.v4.u64 {%0, %1, %2, %3}, [%4];"
+               : "=l"(v.u[0]), "=l"(v.u[1]), "=l"(v.u[2]), "=l"(v.u[3])
+               : "l"(p));
+}
+
+template <typename K>
+__device__ __forceinline__ void fill_max32(L256<K>& v) {
+#pragma unroll
+  for (int e = 0; e < 4; ++e) v.u[e] = ~0ull;
+}
 
 template <typename K>
 __device__ __forceinline__ V16<K> ld16g(const uint8_t* p) {
@@ -672,6 +693,53 @@ regular_search_items_kernel(const RView rv, const ItemDir d, const K* __restrict
         cur[j] = __shfl_sync(0xffffffffu, myv, src);
         t[j] = __shfl_sync(0xffffffffu, myt, src);
       }
+      uint64_t my_pf = 0;
+      K my_v = 0;
+      if (LINE >= 32 && rv.leaf256) {
+        // 256-bit lane loads: the key line and the leaf line each in ONE 64 B request
+        // per group (lane k holds bytes [32k, 32k+32) of the line)
+        L256<K> kw[QPG];
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          if (uint32_t(k) * 32 < LINE) ld32(kw[j], rv.lkeys + (uint64_t(cur[j]) * F + t[j] * KPL) * S + k * 32);
+          else fill_max32(kw[j]);
+        }
+        uint32_t line[QPG];
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          uint32_t c = 0;
+#pragma unroll
+          for (uint32_t x = 0; x < 32 / S; ++x) c += kw[j].k[x] < q[j] ? 1u : 0u;
+          c += __shfl_xor_sync(0xffffffffu, c, 1);
+          line[j] = t[j] * KPL + c;
+        }
+        L256<K> lw[QPG];
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) ld32(lw[j], rv.leaf + (uint64_t(cur[j]) * F + line[j]) * 64 + k * 32);
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          uint32_t c = 0;
+#pragma unroll
+          for (uint32_t x = 0; x < P; ++x) c += lw[j].k[x] < q[j] ? 1u : 0u;
+          const uint32_t sl = __shfl_sync(0xffffffffu, c, g * G);  // lane 0 holds the keys
+          const uint32_t sc = sl < P ? sl : P - 1;
+          const K xk = pick(lw[j].k, sc);
+          const K key_s = __shfl_sync(0xffffffffu, xk, g * G);
+          const K val_s = __shfl_sync(0xffffffffu, xk, g * G + 1);
+          bool end = (sl == P);
+          if (!end && key_s == key_max<K>()) {
+            // MAX slot: padding unless it is a counted entry ("must read the node size")
+            const int64_t in_line = int64_t(__ldg(rv.count + cur[j])) - int64_t(line[j]) * P;
+            const int64_t lim = in_line < int64_t(P) ? in_line : int64_t(P);
+            end = int64_t(sl) >= lim;
+          }
+          const bool found = !end && key_s == q[j];
+          if (j == k) {
+            my_pf = end ? kEnd : (((uint64_t(cur[j]) * F + line[j]) * P + sl) | (found ? kFound : 0ull));
+            my_v = found ? val_s : K(0);
+          }
+        }
+      } else {
       // key line t of last-level node cur: lane k holds 16 B chunks k and k + 2
       V16<K> kv[QPG][2];
 #pragma unroll
@@ -703,8 +771,6 @@ regular_search_items_kernel(const RView rv, const ItemDir d, const K* __restrict
         lk[j] = ld16g<K>(p);
         lvv[j] = ld16g<K>(p + 32);
       }
-      uint64_t my_pf = 0;
-      K my_v = 0;
 #pragma unroll
       for (int j = 0; j < QPG; ++j) {
         uint32_t sl = 0;
@@ -726,6 +792,7 @@ regular_search_items_kernel(const RView rv, const ItemDir d, const K* __restrict
           my_pf = end ? kEnd : (((uint64_t(cur[j]) * F + line[j]) * P + sl) | (found ? kFound : 0ull));
           my_v = found ? val_s : K(0);
         }
+      }
       }
       const uint64_t o = base + uint64_t(k) * NG + g;
       if (o <= p1)  // 16 B record {pos|found, value}: the bucket gather reads records
@@ -871,6 +938,7 @@ int search_items_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* 
   rv.lkeys = (const uint8_t*)r.d_lkeys;
   rv.lidx = (const uint8_t*)r.d_lidx;
   rv.U = r.U;
+  rv.leaf256 = t->cfg.leaf256;
   const size_t smem = (d.B + 1) * 8 + size_t(d.cap) * (sizeof(K) + 4) + ((1u << kPrefixBits) + 1) * 4;
   static bool attr = false;
   if (!attr) {

@@ -255,7 +255,7 @@ int search_local_t(hbt_tree* const* shards, int G, const void* const* queries, c
   // 3. owners search with their global rank base
   for (int d = 0; d < G; ++d) {
     Scratch& sc = shards[d]->shard_scratch;
-    int rc = implicit_search_base(shards[d], sc.recv_q, recv[d], sc.res_pf, sc.res_v, shards[d]->shard.base[d], st);
+    int rc = shard_local_search(shards[d], sc.recv_q, recv[d], sc.res_pf, sc.res_v, shards[d]->shard.base[d], st);
     if (rc) return rc;
   }
   // 4. results back in send order, 5. unpermute
@@ -318,7 +318,7 @@ int search_nccl_t(const hbt_tree* tc, const void* queries, uint64_t m, hbt_out o
     ro += rcnt[p];
   }
   NCCL_TRY(ncclGroupEnd());
-  rc = implicit_search_base(t, sc.recv_q, recv, sc.res_pf, sc.res_v, sm.base[me], st);
+  rc = shard_local_search(t, sc.recv_q, recv, sc.res_pf, sc.res_v, sm.base[me], st);
   if (rc) return rc;
   // results back, in the order they came
   NCCL_TRY(ncclGroupStart());

@@ -267,7 +267,7 @@ int search_and_return(hbt_tree* t, FusedState* f, const PeerTable& pt, int me, u
   if ((rc = ensure(&f->tmp_v, &f->tmp_v_cap, (nrecv ? nrecv : 1) * sizeof(K)))) return rc;
   if (!nrecv) return HBT_OK;
   const Win& w = pt.w[me];
-  rc = implicit_search_base(t, w.recv_q, nrecv, f->tmp_pf, f->tmp_v, t->shard.base[me], st);
+  rc = shard_local_search(t, w.recv_q, nrecv, f->tmp_pf, f->tmp_v, t->shard.base[me], st);
   if (rc) return rc;
   f_return<K><<<grid_for(nrecv), kThreads, 0, st>>>(pt, me, nrecv, f->tmp_pf, (const K*)f->tmp_v);
   HBT_CUDA_TRY(cudaGetLastError());

@@ -26,13 +26,14 @@ def _oracle(layout, k, v, F, width):
     return (oracle.ITree if layout == "implicit" else oracle.RTree).from_pairs(k, v, F, width)
 
 
-ITEM_MODES = [(0, 0), (1, 0), (1, 7)]  # (bucket_items, bucket_cap): plain search, smem directory, global fallback
+# (bucket_items, bucket_cap, leaf256): plain search, smem directory, global fallback, 128-bit lane loads
+ITEM_MODES = [(0, 0, 1), (1, 0, 1), (1, 7, 1), (1, 0, 0)]
 
 
 @pytest.mark.parametrize("layout", ["implicit", "regular"])
 @pytest.mark.parametrize("width,F", [(4, 8), (8, 16), (8, 32), (4, 32)])
-@pytest.mark.parametrize("items,cap", ITEM_MODES)
-def test_bucketed_edge_suite(hbt, layout, width, F, items, cap):
+@pytest.mark.parametrize("items,cap,leaf256", ITEM_MODES)
+def test_bucketed_edge_suite(hbt, layout, width, F, items, cap, leaf256):
     P = 64 // (2 * width)
     rng = np.random.default_rng(900 + 10 * F + width)
     for n in sorted({0, 1, 2, P + 1, F * P + 1, 5 * F * P + 3, 30011}):
@@ -45,6 +46,7 @@ def test_bucketed_edge_suite(hbt, layout, width, F, items, cap):
         t.set_param("bucket", 1)
         t.set_param("bucket_items", items)
         t.set_param("bucket_cap", cap)
+        t.set_param("leaf256", leaf256)
         for slice_bytes in (1, 4096, 1 << 16):  # 1 B: one bucket per unit up to the 1024 cap
             t.set_param("bucket_slice", slice_bytes)
             pf, val = gpu_search(t, q, width)
@@ -55,8 +57,8 @@ def test_bucketed_edge_suite(hbt, layout, width, F, items, cap):
 
 
 @pytest.mark.parametrize("layout,F", [("implicit", 16), ("regular", 32)])
-@pytest.mark.parametrize("items,cap", ITEM_MODES)
-def test_bucketed_scaled_workload(hbt, layout, F, items, cap):
+@pytest.mark.parametrize("items,cap,leaf256", ITEM_MODES)
+def test_bucketed_scaled_workload(hbt, layout, F, items, cap, leaf256):
     """c2 / c3 recipes at reduced size, several bucket counts, every output vs the oracle."""
     cfg = "c2" if layout == "implicit" else "c3"
     n, m = 1 << 19, 1 << 20
@@ -68,6 +70,7 @@ def test_bucketed_scaled_workload(hbt, layout, F, items, cap):
     t.set_param("bucket", 1)
     t.set_param("bucket_items", items)
     t.set_param("bucket_cap", cap)
+    t.set_param("leaf256", leaf256)
     for slice_bytes in (1 << 16, 1 << 20, 1 << 22):
         t.set_param("bucket_slice", slice_bytes)
         pf, val = gpu_search(t, q, 8)
@@ -79,8 +82,8 @@ def test_bucketed_scaled_workload(hbt, layout, F, items, cap):
 
 
 @pytest.mark.parametrize("layout", ["implicit", "regular"])
-@pytest.mark.parametrize("items,cap", ITEM_MODES)
-def test_bucketed_after_update(hbt, layout, items, cap):
+@pytest.mark.parametrize("items,cap,leaf256", ITEM_MODES)
+def test_bucketed_after_update(hbt, layout, items, cap, leaf256):
     """The splitters follow the tree: search, update (keys move between buckets,
     regular leaves split / empty), search again."""
     width, F = 8, 8
@@ -92,6 +95,7 @@ def test_bucketed_after_update(hbt, layout, items, cap):
     t.set_param("bucket", 1)
     t.set_param("bucket_items", items)
     t.set_param("bucket_cap", cap)
+    t.set_param("leaf256", leaf256)
     t.set_param("bucket_slice", 2048)
     q = query_set(k, width, rng, 4000)
     pf, val = gpu_search(t, q, width)

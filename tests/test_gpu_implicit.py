@@ -76,15 +76,17 @@ def expected_index_bytes(o, width):
                                                      (200 * 1024, 512, 2, 1), (64 * 1024, 256, 1, 1),
                                                      (100 * 1024, 512, 2, 0), (0, 1024, 1, 2), (0, 512, 1, 2),
                                                      (0, 1024, 2, 2), (0, 1024, 1, 0)])
-def test_launch_shape_variants(hbt, width, F, budget, threads, qpl, mode):
+@pytest.mark.parametrize("leaf256", [1, 0])
+def test_launch_shape_variants(hbt, width, F, budget, threads, qpl, mode, leaf256):
     """Results must not depend on how many top levels sit in shared memory, the
-    CTA size or the queries in flight per lane."""
+    CTA size, the queries in flight per lane or how the leaf line is loaded."""
     rng = np.random.default_rng(budget + threads + qpl + F + mode)
     k, v = gen_keys(300000, width, rng)
     o = oracle.ITree.from_pairs(k, v, F, width)
     t = gpu_build(hbt, k, v, F, width)
     t.set_search_config(smem_bytes=budget, threads_per_cta=threads, queries_per_lane=qpl, smem_mode=mode,
                         carveout=100 if mode == 1 else -1)
+    t.set_param("leaf256", leaf256)
     q = query_set(k[:5000], width, rng, 20011)
     pf, val = gpu_search(t, q, width)
     epf, ev = o.search(q)

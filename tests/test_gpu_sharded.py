@@ -45,9 +45,12 @@ def queries(allk, rng, m):
                            np.array([0, 2**64 - 1, allk[0], allk[-1], allk[-1] + 1, allk[0] - 1], np.uint64)])
 
 
+@pytest.mark.parametrize("bucket", [0, 1])
 @pytest.mark.parametrize("exchange", [0, 1])
 @pytest.mark.parametrize("G,empty", [(1, []), (2, []), (3, [1]), (5, [0, 4]), (8, []), (8, [2, 3])])
-def test_virtual_shards_match_unsharded_oracle(hbt, G, empty, exchange):
+def test_virtual_shards_match_unsharded_oracle(hbt, G, empty, exchange, bucket):
+    """bucket = 1: the owner side searches its received queries through the bucketed
+    path (item directory, global positions = shard base + local rank)."""
     n = 200000
     allk = gen.stratified_keys(n, gen.stream_seed(4, gen.STREAM_K))
     allv = gen.values(n, 8, gen.stream_seed(4, gen.STREAM_V))
@@ -59,6 +62,9 @@ def test_virtual_shards_match_unsharded_oracle(hbt, G, empty, exchange):
         perm = np.random.default_rng(lo).permutation(len(k))  # unsorted within the shard is fine
         trees.append(hbt.Tree(to_dev(k[perm], 8), to_dev(v[perm], 8), fanout=16))
         trees[-1].set_param("exchange", exchange)
+        if bucket:
+            trees[-1].set_param("bucket", 1)
+            trees[-1].set_param("bucket_slice", 4096)
     grp = hbt.LocalShardGroup(trees)
     rng = np.random.default_rng(G)
     for rep in range(2):  # second batch: larger, forces the windows to grow
