@@ -199,6 +199,10 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *                 global-memory fallback, for tests)
  *   "phase_timing" 1 = record CUDA events around the phases of each bucketed search (read
  *                 them with hbt_last_phases), 0 = off (default)
+ *   "leaf256"     1 (default) = the leaf line (and the regular item search's key line) is read
+ *                 by two lanes' 256-bit loads, one 64 B request per lane group; 0 = 16 B loads
+ *   "sec256"      implicit L2 levels: index / key sector by one lane's 256-bit load (1) or two
+ *                 lanes' 16 B loads (0, default; measured faster on c2)
  * Unknown names or out-of-range values return HBT_EINVAL. */
 HBT_API int hbt_set_param(hbt_tree* t, const char* name, int64_t value);
 

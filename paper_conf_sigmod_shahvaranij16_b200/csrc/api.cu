@@ -311,6 +311,7 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "bucket_cap" && value >= 0 && value < (1 << 20)) { c.bucket_cap = uint32_t(value); t->bk.valid = false; }
   else if (n == "phase_timing" && (value == 0 || value == 1)) c.phase_timing = uint32_t(value);
   else if (n == "leaf256" && (value == 0 || value == 1)) c.leaf256 = uint32_t(value);
+  else if (n == "sec256" && (value == 0 || value == 1)) c.sec256 = uint32_t(value);
   else {
     set_error("bad parameter %s = %lld", name, (long long)value);
     return HBT_EINVAL;

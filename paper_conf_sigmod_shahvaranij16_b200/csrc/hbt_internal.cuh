@@ -42,6 +42,7 @@ struct LevelTable {
   uint32_t dbits;   // mode 2/3/4: directory prefix bits
   uint32_t full_mask;  // bit d: read level d's nodes whole (not index + sector)
   uint32_t leaf256;    // leaf line read as one 64 B request (two 256-bit lane loads)
+  uint32_t sec256;     // index / key sectors of L2 levels by one lane's 256-bit load
 };
 
 struct SearchConfig {
@@ -61,6 +62,7 @@ struct SearchConfig {
   uint32_t bucket_cap = 0;       // item directory: shared-memory entries (0 = derived; tests force the fallback)
   uint32_t phase_timing = 0;     // bucketed search: CUDA events around each phase (hbt_last_phases)
   uint32_t leaf256 = 1;          // leaf line by two 256-bit lane loads (one 64 B request per group)
+  uint32_t sec256 = 0;           // implicit L2 levels: index / key sector by one lane's 256-bit load
 };
 
 // Bucket-local directory of the bucketed search (bucketed.cu): after the

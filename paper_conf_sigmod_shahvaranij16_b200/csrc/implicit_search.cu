@@ -160,6 +160,40 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
         continue;
       }
     }
+    if constexpr (C::IDXB == 32 && C::SECB == 32) {
+      if (lt.sec256 && !sec_known) {
+        // index sector, then the chosen key sector, each by ONE lane's 256-bit load
+        // (the group's other lanes idle): fewer L1 wavefronts per level
+        const uint8_t* lidx = inner_idx + lt.offset[d] * C::IDXB;
+        L256<K> w[QPG];
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          if (k == 0) ld32(w[j], lidx + uint64_t(node[j]) * C::IDXB);
+          else fill_max32(w[j]);
+        }
+        uint32_t sec[QPG];
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          uint32_t c = 0;
+#pragma unroll
+          for (int e = 0; e < C::NSEC; ++e) c += (w[j].k[e] < q[j]) ? 1u : 0u;
+          sec[j] = __shfl_sync(0xffffffffu, c, g * C::G);
+        }
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          if (k == 0) ld32(w[j], lvl + uint64_t(node[j]) * C::NODE_BYTES + sec[j] * 32);
+          else fill_max32(w[j]);
+        }
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          uint32_t c = 0;
+#pragma unroll
+          for (int e = 0; e < C::KPS; ++e) c += (w[j].k[e] < q[j]) ? 1u : 0u;
+          node[j] = node[j] * F + sec[j] * C::KPS + __shfl_sync(0xffffffffu, c, g * C::G);
+        }
+        continue;
+      }
+    }
     uint32_t sec[QPG];
     if (C::HAS_IDX && sec_known) {
 #pragma unroll
@@ -551,6 +585,7 @@ struct Launch {
     // the L2-resident budget are read as whole nodes (see the kernel).
     lt.full_mask = 0;
     lt.leaf256 = t->cfg.leaf256;
+    lt.sec256 = t->cfg.sec256;
     size_t smem;
     if (MODE == 4) {
       lt.SL = t->dir_T;
@@ -646,6 +681,7 @@ struct Launch {
     lt.H = t->H;
     lt.SL = d.level;
     lt.leaf256 = t->cfg.leaf256;
+    lt.sec256 = t->cfg.sec256;
     {
       uint64_t cum = 0;
       const uint64_t budget = t->cfg.l2_levels_bytes ? t->cfg.l2_levels_bytes : (32ull << 20);

@@ -301,3 +301,20 @@ def test_c5_full_size_bench_launch(hbt):
     epf, ev = o.search(q[idx], nthreads=oracle.default_threads())
     assert np.array_equal(pf[idx], epf) and np.array_equal(val[idx], ev)
     t.close()
+
+
+@pytest.mark.parametrize("width,F", [(8, 16), (4, 8), (8, 32), (4, 32), (8, 4)])
+def test_sec256_opt_in_parity(hbt, width, F):
+    """Opt-in "sec256" (L2-level index / key sectors by one lane's 256-bit load; measured
+    slower on c2, kept as a knob): bit-exact on every node shape, including those it skips."""
+    rng = np.random.default_rng(77 + F + width)
+    for n in (1, 1000, 300000):
+        k, v = gen_keys(n, width, rng, dup=True, with_max=(n == 1000))
+        o = oracle.ITree.from_pairs(k, v, F, width)
+        t = gpu_build(hbt, k, v, F, width)
+        t.set_param("sec256", 1)
+        q = query_set(k[:5000], width, rng, 20011)
+        pf, val = gpu_search(t, q, width)
+        epf, ev = o.search(q)
+        assert np.array_equal(pf, epf) and np.array_equal(val, ev), (n, F, width)
+        t.close()
