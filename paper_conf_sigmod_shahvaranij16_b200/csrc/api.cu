@@ -6,6 +6,7 @@
 #include <stdarg.h>
 #include <stdio.h>
 
+#include <algorithm>
 #include <string>
 
 #include "hbt_internal.cuh"
@@ -30,7 +31,12 @@ cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t s) {
   if (configured != dev) {
     cudaMemPool_t pool;
     if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-      uint64_t keep = 4ull << 30;
+      // keep up to a quarter of the device between calls: a bucketed search of
+      // 2^28 queries needs 7.5 GB of scratch, and returning it to the driver
+      // after every call costs ~100 ms (c4, measured)
+      size_t free_b = 0, total_b = 0;
+      cudaMemGetInfo(&free_b, &total_b);
+      uint64_t keep = std::max<uint64_t>(4ull << 30, uint64_t(total_b) / 4);
       cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
     }
     configured = dev;

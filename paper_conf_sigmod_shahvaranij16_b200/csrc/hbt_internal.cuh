@@ -29,7 +29,7 @@ static inline uint64_t ceil_div_u64(uint64_t a, uint64_t b) { return (a + b - 1)
 // Scratch of builds and updates comes from the device's stream-ordered pool
 // (cudaMallocAsync): after the first use, repeated updates allocate without
 // cudaMalloc / cudaFree (which synchronise the device).  The pool keeps up to
-// 4 GiB between calls (api.cu sets the release threshold once).
+// a quarter of the device between calls (api.cu sets the release threshold once).
 cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t s);
 void scratch_free(void* p, cudaStream_t s);
 
