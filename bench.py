@@ -60,6 +60,7 @@ def parse():
     ap.add_argument("--bucket-items", type=int, default=None, help="bucket-local shared-memory directory: 0 | 1")
     ap.add_argument("--leaf256", type=int, default=None, help="leaf / key lines by 256-bit lane loads: 0 | 1")
     ap.add_argument("--sec256", type=int, default=None, help="implicit L2-level sectors by one lane's 256-bit load")
+    ap.add_argument("--full-levels", type=int, default=None, help="implicit: bit mask of levels read whole")
     ap.add_argument("--queries", default=None, choices=["normal", "gamma", "zipf_clustered", "uniform_values"],
                     help="replace the config's queries by the paper's skewed VALUE distributions (P:346-352)")
     ap.add_argument("--update-frac", type=float, default=0.0,
@@ -229,6 +230,8 @@ def make_work(cfg_name, rank, world, args):
         tree.set_param("leaf256", args.leaf256)
     if args.sec256 is not None:
         tree.set_param("sec256", args.sec256)
+    if args.full_levels is not None:
+        tree.set_param("full_levels", args.full_levels)
     out_pos = torch.empty(m, dtype=torch.int64, device="cuda")
     out_val = torch.empty(m, dtype=sdt, device="cuda")
     hi = None

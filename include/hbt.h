@@ -203,6 +203,8 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *                 by two lanes' 256-bit loads, one 64 B request per lane group; 0 = 16 B loads
  *   "sec256"      implicit L2 levels: index / key sector by one lane's 256-bit load (1) or two
  *                 lanes' 16 B loads (0, default; measured faster on c2)
+ *   "full_levels" implicit: bit d set = level d's nodes are read whole in one round trip
+ *                 (0 = default: by the "l2_levels_bytes" budget)
  * Unknown names or out-of-range values return HBT_EINVAL. */
 HBT_API int hbt_set_param(hbt_tree* t, const char* name, int64_t value);
 

@@ -63,6 +63,7 @@ struct SearchConfig {
   uint32_t phase_timing = 0;     // bucketed search: CUDA events around each phase (hbt_last_phases)
   uint32_t leaf256 = 1;          // leaf line by two 256-bit lane loads (one 64 B request per group)
   uint32_t sec256 = 0;           // implicit L2 levels: index / key sector by one lane's 256-bit load
+  uint32_t full_levels = 0;      // implicit: bit d = read level d's nodes whole (0 = by the L2 budget)
 };
 
 // Bucket-local directory of the bucketed search (bucketed.cu): after the

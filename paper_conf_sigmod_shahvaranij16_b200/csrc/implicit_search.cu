@@ -621,6 +621,7 @@ struct Launch {
         cum += t->nodes[d] * uint64_t(C::NODE_BYTES + C::IDXB);
         if (C::HAS_IDX && cum > budget && d < 32) lt.full_mask |= 1u << d;
       }
+      if (t->cfg.full_levels) lt.full_mask = C::HAS_IDX ? uint32_t(t->cfg.full_levels) : 0u;  // explicit override
     }
     // occupancy of this instantiation for this smem size (cached: the query costs
     // microseconds, which dominate small batches)
