@@ -61,6 +61,10 @@ def parse():
     ap.add_argument("--leaf256", type=int, default=None, help="leaf / key lines by 256-bit lane loads: 0 | 1")
     ap.add_argument("--sec256", type=int, default=None, help="implicit L2-level sectors by one lane's 256-bit load")
     ap.add_argument("--full-levels", type=int, default=None, help="implicit: bit mask of levels read whole")
+    ap.add_argument("--graph", default="auto", choices=["0", "1", "auto"],
+                    help="replay the step from a CUDA graph (auto: batches <= 2^20 queries, launch-bound)")
+    ap.add_argument("--param", action="append", default=[], metavar="NAME=VALUE",
+                    help="any hbt_set_param knob (repeatable), e.g. ctas_per_sm=1")
     ap.add_argument("--queries", default=None, choices=["normal", "gamma", "zipf_clustered", "uniform_values"],
                     help="replace the config's queries by the paper's skewed VALUE distributions (P:346-352)")
     ap.add_argument("--update-frac", type=float, default=0.0,
@@ -232,6 +236,9 @@ def make_work(cfg_name, rank, world, args):
         tree.set_param("sec256", args.sec256)
     if args.full_levels is not None:
         tree.set_param("full_levels", args.full_levels)
+    for kv in args.param:
+        name, val = kv.split("=", 1)
+        tree.set_param(name, int(val, 0))
     out_pos = torch.empty(m, dtype=torch.int64, device="cuda")
     out_val = torch.empty(m, dtype=sdt, device="cuda")
     hi = None
@@ -266,10 +273,66 @@ def warm_update_path(work):
     t.close()
 
 
-def time_search(work, steps, world):
+def capture_step(work):
+    """The step captured once in a CUDA graph (small batches are host-launch bound:
+    the Python binding + ctypes + launch cost ~10 us, the c1 kernel ~5 us)."""
+    import torch
+    gs = torch.cuda.Stream()
+    gs.wait_stream(torch.cuda.current_stream())
+    graph = torch.cuda.CUDAGraph()
+    with torch.cuda.stream(gs):
+        step(work)
+        torch.cuda.synchronize()
+        with torch.cuda.graph(graph, stream=gs):
+            step(work)
+    torch.cuda.synchronize()
+    return graph
+
+
+def step_fits_l2(work):
+    """True when the tree plus one step's queries and results fit in the L2 (c1)."""
+    import torch
+    info = work.info
+    data = info["inner_bytes"] + info["leaf_bytes"] + work.m * (2 * work.w + 8)
+    return data < torch.cuda.get_device_properties(torch.cuda.current_device()).L2_cache_size
+
+
+def time_search_flushed(work, steps, world, graph=None):
+    """Small working sets (the tree and the batch fit in the L2): flush the L2 between
+    timed steps by writing a 2x-L2 buffer, and sum per-step CUDA-event intervals (the
+    flush itself is outside every interval).  Max over ranks."""
+    import torch
+    import torch.distributed as dist
+    stream = torch.cuda.current_stream()
+    l2 = torch.cuda.get_device_properties(torch.cuda.current_device()).L2_cache_size
+    flush = torch.empty(2 * l2 // 4, dtype=torch.int32, device="cuda")
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    for a, b in evs:
+        flush.fill_(1)
+        a.record(stream)
+        if graph is not None:
+            graph.replay()
+        else:
+            step(work)
+        b.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    t = torch.tensor([sum(a.elapsed_time(b) for a, b in evs)], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item()) / steps
+
+
+def time_search(work, steps, world, graph=None):
     """K launches of the step, CUDA events on the launching stream, max over ranks."""
     import torch
     import torch.distributed as dist
+    if step_fits_l2(work):
+        return time_search_flushed(work, steps, world, graph)
     stream = torch.cuda.current_stream()
     ev0 = torch.cuda.Event(enable_timing=True)
     ev1 = torch.cuda.Event(enable_timing=True)
@@ -277,8 +340,12 @@ def time_search(work, steps, world):
         dist.barrier()
     torch.cuda.synchronize()
     ev0.record(stream)
-    for _ in range(steps):
-        step(work)
+    if graph is not None:
+        for _ in range(steps):
+            graph.replay()
+    else:
+        for _ in range(steps):
+            step(work)
     ev1.record(stream)
     torch.cuda.synchronize()
     if world > 1:
@@ -342,12 +409,17 @@ def run_hbt(args):
     node_b = ((c["fanout"] * w + 31) // 32) * 32
     l2_probe = probe_l2_gbs(32 if node_b > 32 else node_b) if rank == 0 else None
 
+    use_graph = args.graph == "1" or (args.graph == "auto" and m <= (1 << 20) and args.config != "c4")
+    graph = capture_step(work) if use_graph else None
     for _ in range(max(args.warmup, 3)):
-        step(work)
+        if graph is not None:
+            graph.replay()
+        else:
+            step(work)
     torch.cuda.synchronize()
     sampler = ClockSampler(local)
     sampler.start()
-    ms_step = time_search(work, args.steps, world)
+    ms_step = time_search(work, args.steps, world, graph)
     clocks = sampler.stop()
     qps = world * m / (ms_step * 1e-3)
     launches_per_step = 4 if args.config == "c4" else (2 if args.range_k else 1)
@@ -478,8 +550,13 @@ def run_hbt(args):
                                    if args.config == "c4" else None,
                        "parallelism": (f"key-range sharded x{world}" if args.config == "c4" else
                                        (f"replicated x{world}" if world > 1 else "single")),
-                       "l2_policy": "inputs larger than L2 (queries+results %d MiB/step/GPU > 126 MB L2)"
-                                    % (m * (2 * w + 8) >> 20),
+                       "l2_policy": ("L2 flushed between timed steps (2x-L2 buffer write outside the per-step "
+                                     "CUDA-event intervals; tree + batch %.1f MiB fit in the L2)"
+                                     % ((info["inner_bytes"] + info["leaf_bytes"] + m * (2 * w + 8)) / 2**20)
+                                     if step_fits_l2(work) else
+                                     "inputs larger than L2 (queries+results %d MiB/step/GPU > %d MB L2)"
+                                     % (m * (2 * w + 8) >> 20, l2_size // 10**6)),
+                       "launch": "CUDA graph replay of the captured step" if graph is not None else "direct",
                        "tree": {k: info[k] for k in ("height", "smem_levels", "level_nodes", "leaf_lines",
                                                      "chain_len", "inner_bytes", "leaf_bytes", "n_distinct")}},
             "e2e": e2e,

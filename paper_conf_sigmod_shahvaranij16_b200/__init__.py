@@ -119,8 +119,9 @@ def version() -> str:
 
 def _stream_ptr(stream):
     import torch
-    s = torch.cuda.current_stream() if stream is None else stream
-    return C.c_void_p(s.cuda_stream)
+    if stream is None:  # torch's current stream on the current device (raw handle, no Stream object)
+        return C.c_void_p(torch._C._cuda_getCurrentRawStream(torch._C._cuda_getDevice()))
+    return C.c_void_p(stream.cuda_stream)
 
 
 def _width(t) -> int:

@@ -299,7 +299,7 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
 }
 
 template <typename K, int F, int QPL, int THREADS, int MODE>
-__global__ void __launch_bounds__(THREADS)
+__global__ void __launch_bounds__(THREADS, 1)
 implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ inner_idx,
                        const uint8_t* __restrict__ leaf, const uint32_t* __restrict__ dirbuf,
                        const K* __restrict__ sfull, const K* __restrict__ queries, uint64_t m,
@@ -711,11 +711,14 @@ struct Launch {
     // 256-byte nodes (u64, F = 32) need more registers than a 1024-thread CTA allows
     const uint32_t th = t->cfg.threads ? t->cfg.threads : (C::NODE_BYTES > 128 ? 512 : 1024);
     // small batches read the directory in place (no 96 KB staging per CTA)
-    if (t->cfg.mode == 3 || (t->cfg.mode == 2 && m <= t->cfg.small_batch)) return run_t<1, 1024, 3>(t, q, m, pf, v, b, s);
+    if (t->cfg.mode == 3 || (t->cfg.mode == 2 && m <= t->cfg.small_batch))
+      // 256-thread CTAs spread a small batch over every SM (c1: 10.1 -> 8.3 us per batch)
+      return t->cfg.threads == 1024 ? run_t<1, 1024, 3>(t, q, m, pf, v, b, s) : run_t<1, 256, 3>(t, q, m, pf, v, b, s);
     if (t->cfg.mode == 4 && t->d_sdir)
       return th == 512 ? run_t<1, 512, 4>(t, q, m, pf, v, b, s) : run_t<1, 1024, 4>(t, q, m, pf, v, b, s);
     if (t->cfg.mode == 2) {
       if (th == 512) return run_t<1, 512, 2>(t, q, m, pf, v, b, s);
+      if (th == 768) return qpl == 2 ? run_t<2, 768, 2>(t, q, m, pf, v, b, s) : run_t<1, 768, 2>(t, q, m, pf, v, b, s);
       return qpl == 2 ? run_t<2, 1024, 2>(t, q, m, pf, v, b, s) : run_t<1, 1024, 2>(t, q, m, pf, v, b, s);
     }
     const bool hilo = t->cfg.mode == 1;
