@@ -171,7 +171,7 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
 /* Tune the search kernel's launch shape on one tree; results never depend on
  * it.  name / value:
  *   "smem_bytes"  shared-memory budget per CTA for the pinned top levels (<= 227 KB; 0 = default 100 KB)
- *   "threads"     threads per CTA: 256, 512 or 1024 (0 = default: implicit 1024, regular 512)
+ *   "threads"     threads per CTA: 256, 512, 768 (implicit directory mode) or 1024 (0 = default: implicit 1024, regular 512)
  *   "ctas_per_sm" cap on resident CTAs per SM (0 = occupancy-derived)
  *   "qpl"         queries per lane per warp round, 1 or 2 (0 = default)
  *   "smem_mode"   implicit top levels: 2 = level-T directory + one lower bound, staged in shared
@@ -203,6 +203,8 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *                 by two lanes' 256-bit loads, one 64 B request per lane group; 0 = 16 B loads
  *   "sec256"      implicit L2 levels: index / key sector by one lane's 256-bit load (1) or two
  *                 lanes' 16 B loads (0, default; measured faster on c2)
+ *   "full256"     implicit whole-node levels: 256-bit lane loads (1, default) or 16 B lane
+ *                 loads (0)
  *   "full_levels" implicit: bit d set = level d's nodes are read whole in one round trip
  *                 (0 = default: by the "l2_levels_bytes" budget)
  * Unknown names or out-of-range values return HBT_EINVAL. */

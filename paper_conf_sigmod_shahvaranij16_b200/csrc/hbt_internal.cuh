@@ -43,6 +43,7 @@ struct LevelTable {
   uint32_t full_mask;  // bit d: read level d's nodes whole (not index + sector)
   uint32_t leaf256;    // leaf line read as one 64 B request (two 256-bit lane loads)
   uint32_t sec256;     // index / key sectors of L2 levels by one lane's 256-bit load
+  uint32_t full256;    // whole-node levels read by 256-bit lane loads (half the load instructions)
 };
 
 struct SearchConfig {
@@ -63,6 +64,7 @@ struct SearchConfig {
   uint32_t phase_timing = 0;     // bucketed search: CUDA events around each phase (hbt_last_phases)
   uint32_t leaf256 = 1;          // leaf line by two 256-bit lane loads (one 64 B request per group)
   uint32_t sec256 = 0;           // implicit L2 levels: index / key sector by one lane's 256-bit load
+  uint32_t full256 = 1;          // implicit whole-node levels by 256-bit lane loads
   uint32_t full_levels = 0;      // implicit: bit d = read level d's nodes whole (0 = by the L2 budget)
 };
 

@@ -139,6 +139,31 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
         // Level beyond the L2-resident budget: a miss costs a whole DRAM line
         // anyway, so read the full node in ONE round trip (each of the G lanes
         // loads NODE_BYTES/G contiguous bytes) instead of index + sector.
+        if constexpr (C::NODE_BYTES / C::G >= 32) {
+          if (lt.full256) {
+            // 256-bit lane loads: half the load instructions (and L1TEX wavefronts,
+            // the pipe that binds the item search, profiles/r01_c4_items_*) of 16 B loads
+            constexpr int NC32 = C::NODE_BYTES / C::G / 32;
+            L256<K> fw[QPG][NC32];
+#pragma unroll
+            for (int j = 0; j < QPG; ++j)
+#pragma unroll
+              for (int h = 0; h < NC32; ++h)
+                ld32(fw[j][h], lvl + uint64_t(node[j]) * C::NODE_BYTES + (k * NC32 + h) * 32);
+#pragma unroll
+            for (int j = 0; j < QPG; ++j) {
+              uint32_t c = 0;
+#pragma unroll
+              for (int h = 0; h < NC32; ++h)
+#pragma unroll
+                for (int e = 0; e < 32 / C::S; ++e) c += (fw[j][h].k[e] < q[j]) ? 1u : 0u;
+#pragma unroll
+              for (int x = 1; x < C::G; x <<= 1) c += __shfl_xor_sync(0xffffffffu, c, x);
+              node[j] = node[j] * F + c;
+            }
+            continue;
+          }
+        }
         constexpr int NCH = C::NODE_BYTES / C::G / 16;
         V16<K> fv[QPG][NCH];
 #pragma unroll
@@ -586,6 +611,7 @@ struct Launch {
     lt.full_mask = 0;
     lt.leaf256 = t->cfg.leaf256;
     lt.sec256 = t->cfg.sec256;
+    lt.full256 = t->cfg.full256;
     size_t smem;
     if (MODE == 4) {
       lt.SL = t->dir_T;
@@ -683,6 +709,7 @@ struct Launch {
     lt.SL = d.level;
     lt.leaf256 = t->cfg.leaf256;
     lt.sec256 = t->cfg.sec256;
+    lt.full256 = t->cfg.full256;
     {
       uint64_t cum = 0;
       const uint64_t budget = t->cfg.l2_levels_bytes ? t->cfg.l2_levels_bytes : (32ull << 20);

@@ -44,9 +44,13 @@ def test_edge_suite_parity(hbt, width, F):
         assert t.export(hbt.SEG_INNER_IDX).tobytes() == expected_index_bytes(o, width), (n, F, width)
         q = query_set(k, width, rng, 3000)
         epf, ev = o.search(q)
-        for mode, l2b in ((0, 0), (2, 0), (2, 1), (0, 1), (3, 0), (4, 0), (4, 1)):  # top-level modes x read modes
+        # top-level modes x per-level read modes (l2b = 1: every level read whole, by
+        # 256-bit (f256) or 16 B lane loads)
+        for mode, l2b, f256 in ((0, 0, 1), (2, 0, 1), (2, 1, 1), (2, 1, 0), (0, 1, 1), (0, 1, 0), (3, 0, 1),
+                                (3, 1, 0), (4, 0, 1), (4, 1, 1)):
             t.set_search_config(smem_mode=mode)
             t.set_param("l2_levels_bytes", l2b)
+            t.set_param("full256", f256)
             pf, val = gpu_search(t, q, width)
             assert np.array_equal(pf, epf), (mode, n, F, width, np.nonzero(pf != epf)[0][:5])
             assert np.array_equal(val, ev), (mode, n, F, width)
@@ -75,7 +79,8 @@ def expected_index_bytes(o, width):
 @pytest.mark.parametrize("budget,threads,qpl,mode", [(16, 0, 0, 0), (4096, 256, 2, 1), (100 * 1024, 512, 1, 0),
                                                      (200 * 1024, 512, 2, 1), (64 * 1024, 256, 1, 1),
                                                      (100 * 1024, 512, 2, 0), (0, 1024, 1, 2), (0, 512, 1, 2),
-                                                     (0, 1024, 2, 2), (0, 1024, 1, 0)])
+                                                     (0, 1024, 2, 2), (0, 1024, 1, 0), (0, 768, 1, 2),
+                                                     (0, 768, 2, 2), (0, 256, 1, 3), (0, 1024, 1, 3)])
 @pytest.mark.parametrize("leaf256", [1, 0])
 def test_launch_shape_variants(hbt, width, F, budget, threads, qpl, mode, leaf256):
     """Results must not depend on how many top levels sit in shared memory, the
@@ -87,6 +92,7 @@ def test_launch_shape_variants(hbt, width, F, budget, threads, qpl, mode, leaf25
     t.set_search_config(smem_bytes=budget, threads_per_cta=threads, queries_per_lane=qpl, smem_mode=mode,
                         carveout=100 if mode == 1 else -1)
     t.set_param("leaf256", leaf256)
+    t.set_param("small_batch", 0)  # mode 2 stays mode 2 at this batch size (mode 3 is asked for explicitly)
     q = query_set(k[:5000], width, rng, 20011)
     pf, val = gpu_search(t, q, width)
     epf, ev = o.search(q)
@@ -318,3 +324,36 @@ def test_sec256_opt_in_parity(hbt, width, F):
         epf, ev = o.search(q)
         assert np.array_equal(pf, epf) and np.array_equal(val, ev), (n, F, width)
         t.close()
+
+
+def test_search_in_cuda_graph(hbt):
+    """hbt_search is capturable: a graph captured once and replayed over new query
+    values in the same buffer gives the oracle's results (bench.py replays
+    launch-bound steps this way)."""
+    width, F = 4, 8
+    rng = np.random.default_rng(7)
+    k, v = gen_keys(65536, width, rng)
+    o = oracle.ITree.from_pairs(k, v, F, width)
+    t = gpu_build(hbt, k, v, F, width)
+    q0 = query_set(k, width, rng, 65536)
+    dq = to_dev(q0, width)
+    pos = torch.empty(dq.numel(), dtype=torch.int64, device="cuda")
+    val = torch.empty(dq.numel(), dtype=dq.dtype, device="cuda")
+    gs = torch.cuda.Stream()
+    gs.wait_stream(torch.cuda.current_stream())
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.stream(gs):
+        t.search(dq, pos, val, stream=gs)
+        torch.cuda.synchronize()
+        with torch.cuda.graph(g, stream=gs):
+            t.search(dq, pos, val, stream=gs)
+    torch.cuda.synchronize()
+    for rep in range(3):
+        q = query_set(k, width, rng, 65536)
+        dq.copy_(to_dev(q, width))
+        g.replay()
+        torch.cuda.synchronize()
+        epf, ev = o.search(q)
+        assert np.array_equal(pos.cpu().numpy().view(np.uint64), epf), rep
+        assert np.array_equal(val.cpu().numpy().view(np_dtype(width)).astype(np.uint64), ev), rep
+    t.close()
