@@ -267,11 +267,12 @@ __global__ void __launch_bounds__(kThreads, 2) bk_scatter(const K* __restrict__ 
   uint32_t* s_gb = s_lb + kMaxBuckets;
   uint32_t* s_rank = s_gb + kMaxBuckets;
   uint32_t* s_tmp = s_rank + kMaxBuckets;
+  // the chunk's queries and bucket ids are loaded before its layout row is scanned,
+  // so the two DRAM round trips overlap
+  constexpr int LPT = int(kMaxBuckets) / kThreads;  // layout entries per thread
   for (uint64_t c = blockIdx.x; c < chunks; c += gridDim.x) {
     const uint64_t lo = c * kChunk;
     const uint32_t nc = uint32_t(m - lo < kChunk ? m - lo : kChunk);
-    for (uint32_t b = threadIdx.x; b < B; b += kThreads) s_rank[b] = 0;
-    chunk_layout(tab, gb, B, chunks, c, s_cnt, s_lb, s_gb, s_tmp);
     K qq[kQPT];
     uint32_t bb[kQPT];
 #pragma unroll
@@ -284,6 +285,17 @@ __global__ void __launch_bounds__(kThreads, 2) bk_scatter(const K* __restrict__ 
         bb[j] = __ldcs(reinterpret_cast<const unsigned short*>(bq) + lo + t);
       }
     }
+#pragma unroll
+    for (int e = 0; e < LPT; ++e) {
+      const uint32_t b = uint32_t(e) * kThreads + threadIdx.x;
+      if (b < B) {
+        s_rank[b] = 0;
+        s_cnt[b] = tab[c * B + b];
+        s_gb[b] = gb[c * B + b];
+      }
+    }
+    __syncthreads();
+    block_exclusive_scan(s_cnt, s_lb, B, s_tmp);
 #pragma unroll
     for (int j = 0; j < kQPT; ++j) {
       const uint32_t t = uint32_t(j) * kThreads + threadIdx.x;
@@ -399,6 +411,11 @@ __global__ void __launch_bounds__(kGThreads) bk_gather_rec(const uint16_t* __res
                                                            const uint32_t* __restrict__ gb, uint32_t B,
                                                            uint64_t chunks, const ulonglong2* __restrict__ rec,
                                                            uint64_t* __restrict__ out_pf, K* __restrict__ out_v) {
+  // B <= kMaxBuckets == kGThreads: thread b owns bucket b's layout entries.  The next
+  // chunk's layout row is loaded while this chunk's records are stored, and all of a
+  // thread's record and linv loads are issued together (the kernel was latency
+  // bound: long-scoreboard stalls 38 per issue, one CTA per SM).
+  static_assert(kMaxBuckets <= kGThreads, "one bucket per thread");
   constexpr int PT = int(kChunk) / kGThreads;
   extern __shared__ __align__(16) uint8_t smem[];
   ulonglong2* s_rec = reinterpret_cast<ulonglong2*>(smem);
@@ -407,37 +424,54 @@ __global__ void __launch_bounds__(kGThreads) bk_gather_rec(const uint16_t* __res
   uint32_t* s_lb = s_cnt + kMaxBuckets;
   uint32_t* s_gb = s_lb + kMaxBuckets;
   uint32_t* s_tmp = s_gb + kMaxBuckets;
+  const uint32_t tb = threadIdx.x;
+  uint32_t nx_cnt = 0, nx_gb = 0;
+  if (blockIdx.x < chunks && tb < B) {
+    nx_cnt = tab[uint64_t(blockIdx.x) * B + tb];
+    nx_gb = gb[uint64_t(blockIdx.x) * B + tb];
+  }
   for (uint64_t c = blockIdx.x; c < chunks; c += gridDim.x) {
     const uint64_t lo = c * kChunk;
     const uint32_t nc = uint32_t(m - lo < kChunk ? m - lo : kChunk);
-    chunk_layout<kGThreads>(tab, gb, B, chunks, c, s_cnt, s_lb, s_gb, s_tmp);
-    for (uint32_t b = threadIdx.x; b < B; b += kGThreads)
-      for (uint32_t k = 0, n = s_cnt[b], p = s_lb[b]; k < n; ++k) s_b[p + k] = uint16_t(b);
-    __syncthreads();
-#pragma unroll 1
-    for (int h = 0; h < PT; h += 4) {
-      ulonglong2 x[4];
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const uint32_t t = uint32_t(h + j) * kGThreads + threadIdx.x;
-        if (t < nc) {
-          const uint32_t b = s_b[t];
-          x[j] = __ldcs(rec + s_gb[b] + (t - s_lb[b]));
-        }
-      }
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const uint32_t t = uint32_t(h + j) * kGThreads + threadIdx.x;
-        if (t < nc) s_rec[t] = x[j];
-      }
+    if (tb < B) {
+      s_cnt[tb] = nx_cnt;
+      s_gb[tb] = nx_gb;
     }
     __syncthreads();
+    block_exclusive_scan<kGThreads>(s_cnt, s_lb, B, s_tmp);
+    if (tb < B)
+      for (uint32_t k = 0, n = s_cnt[tb], p = s_lb[tb]; k < n; ++k) s_b[p + k] = uint16_t(tb);
+    __syncthreads();
     const unsigned short* li = reinterpret_cast<const unsigned short*>(linv) + lo;
+    ulonglong2 x[PT];
+    unsigned short l[PT];
 #pragma unroll
     for (int j = 0; j < PT; ++j) {
-      const uint32_t t = uint32_t(j) * kGThreads + threadIdx.x;
+      const uint32_t t = uint32_t(j) * kGThreads + tb;
       if (t < nc) {
-        const ulonglong2 r = s_rec[__ldcs(li + t)];
+        const uint32_t b = s_b[t];
+        x[j] = __ldcs(rec + s_gb[b] + (t - s_lb[b]));
+        l[j] = __ldcs(li + t);
+      }
+    }
+    {  // next chunk's layout row, in flight during the stores below
+      const uint64_t cn = c + gridDim.x;
+      if (cn < chunks && tb < B) {
+        nx_cnt = tab[cn * B + tb];
+        nx_gb = gb[cn * B + tb];
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < PT; ++j) {
+      const uint32_t t = uint32_t(j) * kGThreads + tb;
+      if (t < nc) s_rec[t] = x[j];
+    }
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < PT; ++j) {
+      const uint32_t t = uint32_t(j) * kGThreads + tb;
+      if (t < nc) {
+        const ulonglong2 r = s_rec[l[j]];
         __stcs(reinterpret_cast<unsigned long long*>(out_pf) + lo + t, r.x);
         if constexpr (sizeof(K) == 8)
           __stcs(reinterpret_cast<unsigned long long*>(out_v) + lo + t, r.y);
