@@ -518,6 +518,9 @@ def run_hbt(args):
     roof["kernel_ms"] = round(t_kernel * 1e3, 4)
     roof["frac_hbm"] = roof_hbm["frac"]
     roof["frac_l2"] = roof_l2["frac"] if roof_l2 else None
+    if m <= (1 << 20) and not args.range_k:
+        roof["note"] = ("latency-bound batch: %d queries are one wave of the GPU, so the step is the launch "
+                        "plus one query's chain of dependent memory round trips; no byte roofline binds" % m)
 
     if phases and e2e:  # each 4 Mi-query chunk of hbt_search_host runs the bucketed pipeline
         e2e["gpu_launches_per_step"] *= phases["launches"]
