@@ -187,6 +187,8 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *                 as whole nodes beyond it (0 = default 32 MB; 1 = every level whole)
  *   "exchange"    sharded search: 0 = fused peer-memory exchange (CUDA IPC windows, default),
  *                 1 = NCCL send/recv (multi-process) / device copies (hbt_search_sharded_local)
+ *   "g1_direct"   hbt_search_sharded on a ONE-shard tree with exchange 0: 1 (default) = search
+ *                 in place (nothing to route or exchange), 0 = run the full fused pipeline
  *   "bucket"      query bucketing before the tree walk (north_star "queries bucketed per batch"):
  *                 0 = off, 1 = on, 2 = auto (default: regular trees larger than 8x the L2 and
  *                 batches of >= 4 Mi queries).  The batch is partitioned into B key-range

@@ -329,6 +329,7 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "l2_persist" && value >= 0) c.l2_persist = uint64_t(value);
   else if (n == "l2_levels_bytes" && value >= 0) c.l2_levels_bytes = uint64_t(value);
   else if (n == "exchange" && (value == 0 || value == 1)) c.exchange = uint32_t(value);
+  else if (n == "g1_direct" && (value == 0 || value == 1)) c.g1_direct = uint32_t(value);
   else if (n == "bucket" && value >= 0 && value <= 2) c.bucket = uint32_t(value);
   else if (n == "bucket_slice" && value >= 0) { c.bucket_slice = uint64_t(value); t->bk.valid = false; }
   else if (n == "bucket_items" && (value == 0 || value == 1)) { c.bucket_items = uint32_t(value); t->bk.valid = false; }

@@ -56,6 +56,7 @@ struct SearchConfig {
   uint64_t l2_persist = 0;       // bytes of the I-segment to keep in a persisting L2 window (0 = off)
   uint64_t l2_levels_bytes = 0;  // L2-resident budget for index+sector levels (0 = default 32 MB)
   uint32_t exchange = 0;         // sharded search: 0 = fused peer-memory exchange, 1 = NCCL send/recv
+  uint32_t g1_direct = 1;        // sharded search with ONE shard: search directly (no route / exchange)
   uint64_t small_batch = 1u << 16;  // mode 2: batches up to this size read the directory in place (mode 3)
   uint32_t bucket = 2;           // query bucketing (bucketed.cu): 0 = off, 1 = on, 2 = auto
   uint64_t bucket_slice = 0;     // tree bytes per bucket (0 = default 1 MB)

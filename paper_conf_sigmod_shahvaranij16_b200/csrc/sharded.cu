@@ -454,6 +454,13 @@ int hbt_search_sharded(const hbt_tree* t, const void* queries_local, uint64_t m_
                        void* stream) {
   if (!t || !t->shard.comm) { set_error("not a sharded tree"); return HBT_EINVAL; }
   cudaStream_t st = (cudaStream_t)stream;
+  if (t->shard.G == 1 && t->cfg.exchange == 0 && t->cfg.g1_direct) {
+    // One shard owns every key: routing would send every query to this rank and the
+    // exchange would only copy, so search in place (global pos = the shard's base rank).
+    if (m_local == 0) return HBT_OK;
+    if (!queries_local || !out_local.pos_found || !out_local.values) { set_error("NULL buffer"); return HBT_EINVAL; }
+    return shard_local_search(t, queries_local, m_local, out_local.pos_found, out_local.values, t->shard.base[0], st);
+  }
   if (t->cfg.exchange == 0) return fused_search_nccl(t, queries_local, m_local, out_local, st);
   if (!t->shard.comm->comm) { set_error("exchange=1 needs an NCCL communicator"); return HBT_EUNSUPPORTED; }
   return t->width == 4 ? search_nccl_t<uint32_t>(t, queries_local, m_local, out_local, st)

@@ -85,10 +85,11 @@ def test_virtual_shards_reject_overlap(hbt):
         hbt.LocalShardGroup([a, b])
 
 
-@pytest.mark.parametrize("exchange", [0, 1])
-def test_nccl_path_one_rank(hbt, exchange):
+@pytest.mark.parametrize("exchange,g1_direct", [(0, 0), (0, 1), (1, 1)])
+def test_nccl_path_one_rank(hbt, exchange, g1_direct):
     """One rank over the real communicator: exchange 0 = fused peer-memory path
-    (IPC window export/all-gather, device barriers), 1 = NCCL send/recv."""
+    (IPC window export/all-gather, device barriers; g1_direct = 1 searches the single
+    shard in place), 1 = NCCL send/recv."""
     uid = hbt.unique_id()
     comm = hbt.Comm(1, 0, uid)
     n = 100000
@@ -96,6 +97,7 @@ def test_nccl_path_one_rank(hbt, exchange):
     allv = gen.values(n, 8, 9)
     t = hbt.ShardedTree(comm, to_dev(allk, 8), to_dev(allv, 8), fanout=16)
     t.set_param("exchange", exchange)
+    t.set_param("g1_direct", g1_direct)
     o = oracle.ITree.from_pairs(allk, allv, 16, 8)
     for rep in range(3):
         q = queries(allk, np.random.default_rng(rep), 20000 * (1 + rep))
