@@ -469,7 +469,7 @@ def run_hbt(args):
         t_kernel = phases["search"] * 1e-3
         kernel = ("regular_search_items_kernel" if c["layout"] == "regular" else "implicit_search_items_kernel")
         # c4: the sharded step's own kernels (count / publish / barrier / return) + the pipeline
-        launches_per_step = phases["launches"] + (3 if args.config == "c4" else 0)
+        launches_per_step = phases["launches"] + (3 if args.config == "c4" and world > 1 else 0)
         model_desc = "bucketed search: query + 16 B record + distinct tree lines per pass (tools/roofline.py)"
     else:
         mdl = roofline.model(info, l2_size, work.hit_rate)
