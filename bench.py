@@ -61,6 +61,8 @@ def parse():
     ap.add_argument("--leaf256", type=int, default=None, help="leaf / key lines by 256-bit lane loads: 0 | 1")
     ap.add_argument("--sec256", type=int, default=None, help="implicit L2-level sectors by one lane's 256-bit load")
     ap.add_argument("--full-levels", type=int, default=None, help="implicit: bit mask of levels read whole")
+    ap.add_argument("--leaf-host", action="store_true",
+                    help="implicit trees: L-segment in pinned host memory (the paper's split, SURVEY f4)")
     ap.add_argument("--graph", default="auto", choices=["0", "1", "auto"],
                     help="replay the step from a CUDA graph (auto: batches <= 2^20 queries, launch-bound)")
     ap.add_argument("--param", action="append", default=[], metavar="NAME=VALUE",
@@ -129,6 +131,23 @@ class ClockSampler:
         reasons = sorted({names[i] for r in rows for i in range(4) if r[5 + i].lower().startswith("active")})
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
                 "reasons": reasons, "samples": len(rows)}
+
+
+def measure_h2d_gbs():
+    """Pinned host -> device copy bandwidth (1 GiB, best of 3, CUDA events)."""
+    import torch
+    h = torch.empty(1 << 30, dtype=torch.uint8).pin_memory()
+    d = torch.empty(1 << 30, dtype=torch.uint8, device="cuda")
+    best = 0.0
+    for _ in range(3):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        d.copy_(h, non_blocking=True)
+        b.record()
+        torch.cuda.synchronize()
+        best = max(best, (1 << 30) / (a.elapsed_time(b) * 1e-3) / 1e9)
+    del h, d
+    return best
 
 
 def probe_l2_gbs(chunk):
@@ -236,6 +255,9 @@ def make_work(cfg_name, rank, world, args):
         tree.set_param("sec256", args.sec256)
     if args.full_levels is not None:
         tree.set_param("full_levels", args.full_levels)
+    if args.leaf_host:
+        tree.set_leaf_placement("host")  # f4: L-segment in pinned host memory
+        qdesc += "; L-segment in pinned host memory, leaf lines read by zero-copy loads over the host link"
     for kv in args.param:
         name, val = kv.split("=", 1)
         tree.set_param(name, int(val, 0))
@@ -518,6 +540,13 @@ def run_hbt(args):
     roof["kernel_ms"] = round(t_kernel * 1e3, 4)
     roof["frac_hbm"] = roof_hbm["frac"]
     roof["frac_l2"] = roof_l2["frac"] if roof_l2 else None
+    if args.leaf_host:  # the leaf line crosses the host link once per query
+        h2d = measure_h2d_gbs()
+        link_ach = 64 * m / t_kernel / 1e9
+        roof["link"] = {"bound": "host link (zero-copy leaf reads)", "bytes_per_query": 64,
+                        "achieved": round(link_ach, 1), "unit": "GB/s", "peak": round(h2d, 1),
+                        "peak_source": "measured in this run: pinned H2D cudaMemcpy of 1 GiB",
+                        "frac": round(link_ach / h2d, 4)}
     if m <= (1 << 20) and not args.range_k:
         roof["note"] = ("latency-bound batch: %d queries are one wave of the GPU, so the step is the launch "
                         "plus one query's chain of dependent memory round trips; no byte roofline binds" % m)

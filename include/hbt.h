@@ -145,6 +145,18 @@ HBT_API int hbt_search(const hbt_tree* t, const void* queries, uint64_t m, hbt_o
 HBT_API int hbt_search_host(const hbt_tree* t, const void* host_queries, uint64_t m,
                     uint64_t* host_pos_found, void* host_values, void* stream);
 
+/* L-segment placement (the paper's split: the I-segment on the GPU, the
+ * L-segment in host memory).  where = 0: HBM (default);
+ * 1: pinned host memory mapped into the device address space — the search, range
+ * and bucketing kernels then read each query's leaf line with zero-copy loads over
+ * the host link (PCIe / NVLink-C2C), so a tree's leaves may exceed HBM while its
+ * inner levels stay in HBM.  Results are identical in both placements.
+ * IMPLICIT trees only (HBT_EUNSUPPORTED for regular or multi-shard trees); a rebuild
+ * by hbt_bulk_update keeps the placement.  Synchronises the device (no search may be
+ * in flight); HBT_ENOMEM when the pinned allocation fails (the tree is unchanged). */
+HBT_API int hbt_set_leaf_placement(hbt_tree* t, uint32_t where);
+HBT_API int hbt_get_leaf_placement(const hbt_tree* t, uint32_t* where);
+
 /* Range scan (the range-query experiment of P:392): for each of the m
  * queries, the first up-to-k pairs with lo[i] <= key <= hi[i] in key order.
  * lo/hi: device arrays (width S, length m).  out_keys/out_values: device arrays

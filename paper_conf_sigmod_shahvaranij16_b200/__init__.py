@@ -37,7 +37,8 @@ UPSERT, DELETE = 0, 1
 EXPORTED = ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
             "hbt_info", "hbt_export", "hbt_set_param", "hbt_last_error", "hbt_version",
             "hbt_range", "hbt_comm_unique_id", "hbt_comm_init", "hbt_comm_init_host", "hbt_comm_destroy", "hbt_bulk_build_sharded",
-            "hbt_search_sharded", "hbt_shard_local_init", "hbt_search_sharded_local", "hbt_last_phases"]
+            "hbt_search_sharded", "hbt_shard_local_init", "hbt_search_sharded_local", "hbt_last_phases",
+            "hbt_set_leaf_placement", "hbt_get_leaf_placement"]
 
 
 class HBTError(RuntimeError):
@@ -94,13 +95,16 @@ def _load():
     L.hbt_search_sharded_local.argtypes = [C.POINTER(vp), C.c_int, C.POINTER(vp), C.POINTER(u64),
                                            C.POINTER(_Out), vp]
     L.hbt_last_phases.argtypes = [vp, vp]
+    L.hbt_set_leaf_placement.argtypes = [vp, u32]
+    L.hbt_get_leaf_placement.argtypes = [vp, C.POINTER(u32)]
     L.hbt_last_error.restype = C.c_char_p
     L.hbt_version.restype = C.c_char_p
     for f in ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
               "hbt_info", "hbt_export", "hbt_set_param", "hbt_range", "hbt_comm_unique_id", "hbt_comm_init",
               "hbt_comm_init_host",
               "hbt_comm_destroy", "hbt_bulk_build_sharded", "hbt_search_sharded", "hbt_shard_local_init",
-              "hbt_search_sharded_local", "hbt_last_phases"]:
+              "hbt_search_sharded_local", "hbt_last_phases", "hbt_set_leaf_placement",
+              "hbt_get_leaf_placement"]:
         getattr(L, f).restype = C.c_int
     return L
 
@@ -196,6 +200,17 @@ class Tree:
             _check(lib.hbt_search(self._h, C.c_void_p(queries.data_ptr()), m,
                                   _Out(out_pos.data_ptr(), out_vals.data_ptr()), _stream_ptr(stream)))
         return out_pos, out_vals
+
+    # -- placement of the L-segment (hbt_set_leaf_placement)
+    def set_leaf_placement(self, where: str):
+        """'device' (HBM) or 'host' (pinned host memory read by zero-copy loads)."""
+        _check(lib.hbt_set_leaf_placement(self._h, {"device": 0, "host": 1}[where]))
+
+    @property
+    def leaf_placement(self) -> str:
+        w = C.c_uint32()
+        _check(lib.hbt_get_leaf_placement(self._h, C.byref(w)))
+        return "host" if w.value else "device"
 
     def search_host(self, queries, out_pos, out_vals, stream=None):
         """End-to-end lookups from/to HOST buffers (numpy arrays or pinned CPU tensors)."""

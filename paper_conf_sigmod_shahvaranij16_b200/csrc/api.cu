@@ -78,13 +78,59 @@ static bool is_device_ptr(const void* p) {
   return true;
 }
 
+void leaf_free(hbt_tree* t) {
+  if (t->h_leaf) cudaFreeHost(t->h_leaf);
+  else cudaFree(t->d_leaf);
+  t->h_leaf = nullptr;
+  t->d_leaf = nullptr;
+}
+
+// Move the implicit L-segment between HBM and pinned, mapped host memory.  The
+// search kernels read leaf lines through d_leaf either way (zero-copy loads over the
+// host link when it lives on the host), so results are identical.
+int leaf_place(hbt_tree* t, uint32_t where) {
+  const bool on_host = t->h_leaf != nullptr;
+  if ((where == 1) == on_host) { t->leaf_where = where; return HBT_OK; }
+  const uint64_t bytes = t->leaf_bytes ? t->leaf_bytes : 64;
+  if (where == 1) {
+    void* h = nullptr;
+    void* d = nullptr;
+    if (cudaHostAlloc(&h, bytes, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) {
+      cudaGetLastError();
+      set_error("cudaHostAlloc of %llu bytes for the L-segment failed", (unsigned long long)bytes);
+      return HBT_ENOMEM;
+    }
+    if (t->leaf_bytes) {
+      cudaError_t e = cudaMemcpy(h, t->d_leaf, t->leaf_bytes, cudaMemcpyDefault);
+      if (e != cudaSuccess) { cudaFreeHost(h); set_error("L-segment copy: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
+    }
+    cudaError_t e = cudaHostGetDevicePointer(&d, h, 0);
+    if (e != cudaSuccess) { cudaFreeHost(h); set_error("no device alias of the host L-segment: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
+    cudaFree(t->d_leaf);
+    t->h_leaf = h;
+    t->d_leaf = d;
+  } else {
+    void* d = nullptr;
+    HBT_CUDA_TRY(cudaMalloc(&d, bytes));
+    if (t->leaf_bytes) {
+      cudaError_t e = cudaMemcpy(d, t->h_leaf, t->leaf_bytes, cudaMemcpyDefault);
+      if (e != cudaSuccess) { cudaFree(d); set_error("L-segment copy: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
+    }
+    cudaFreeHost(t->h_leaf);
+    t->h_leaf = nullptr;
+    t->d_leaf = d;
+  }
+  t->leaf_where = where;
+  return HBT_OK;
+}
+
 static void free_tree(hbt_tree* t) {
   if (!t) return;
   cudaFree(t->d_inner);  // also holds d_inner_idx
   cudaFree(t->d_dir);
   cudaFree(t->d_sdir);
   cudaFree(t->d_sdir_full);
-  cudaFree(t->d_leaf);
+  leaf_free(t);
   regular_free(t);
   shard_free(t);
   fused_free(t);
@@ -299,7 +345,23 @@ int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t bytes, u
   }
   if (written) *written = len;
   if (bytes < len) { set_error("destination too small: need %llu bytes", (unsigned long long)len); return HBT_EINVAL; }
-  if (len) HBT_CUDA_TRY(cudaMemcpy(dst, src, len, cudaMemcpyDeviceToHost));
+  if (len) HBT_CUDA_TRY(cudaMemcpy(dst, src, len, cudaMemcpyDefault));  // src may be the mapped host L-segment
+  return HBT_OK;
+}
+
+int hbt_set_leaf_placement(hbt_tree* t, uint32_t where) {
+  g_err.clear();
+  if (!t) { set_error("tree is NULL"); return HBT_EINVAL; }
+  if (where > 1) { set_error("placement must be 0 (HBM) or 1 (host)"); return HBT_EINVAL; }
+  if (t->form != HBT_IMPLICIT) { set_error("leaf placement: implicit trees only"); return HBT_EUNSUPPORTED; }
+  if (t->shard.G > 1) { set_error("leaf placement: not for sharded trees"); return HBT_EUNSUPPORTED; }
+  HBT_CUDA_TRY(cudaDeviceSynchronize());  // no search may be reading the old copy
+  return leaf_place(t, where);
+}
+
+int hbt_get_leaf_placement(const hbt_tree* t, uint32_t* where) {
+  if (!t || !where) { set_error("NULL argument"); return HBT_EINVAL; }
+  *where = t->h_leaf ? 1u : 0u;
   return HBT_OK;
 }
 

@@ -225,6 +225,11 @@ struct hbt_tree {
   void* d_leaf = nullptr;
   uint64_t L0 = 0;
   uint64_t leaf_bytes = 0;
+  // L-segment placement (hbt_set_leaf_placement): 0 = HBM; 1 = pinned host memory
+  // mapped into the device address space (h_leaf = its host address, d_leaf = the
+  // device alias), the paper's I-segment-on-GPU / L-segment-in-host split
+  uint32_t leaf_where = 0;
+  void* h_leaf = nullptr;
   // ---- regular ----
   hbt::RegularState r;
   // ---- key-range sharding ----
@@ -288,4 +293,8 @@ int bucketed_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, 
 int shard_local_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
                        cudaStream_t s);
 void bucket_free(hbt_tree* t);
+// implicit L-segment placement (api.cu): free the current L-segment wherever it lives;
+// move it to HBM (0) or mapped pinned host memory (1)
+void leaf_free(hbt_tree* t);
+int leaf_place(hbt_tree* t, uint32_t where);
 }  // namespace hbt

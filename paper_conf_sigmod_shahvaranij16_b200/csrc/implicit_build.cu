@@ -434,7 +434,8 @@ int implicit_update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
     cudaFree(nt.d_leaf); cudaFree(nt.d_inner); cudaFree(nt.d_dir); cudaFree(nt.d_sdir); cudaFree(nt.d_sdir_full);
     return rc;
   }
-  cudaFree(t->d_leaf);
+  const uint32_t where = t->leaf_where;
+  leaf_free(t);
   cudaFree(t->d_inner);  // also holds the derived index
   cudaFree(t->d_dir);
   cudaFree(t->d_sdir);
@@ -450,7 +451,8 @@ int implicit_update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   t->d_sdir = nt.d_sdir; t->d_sdir_full = nt.d_sdir_full; t->sdir_bytes = nt.sdir_bytes;
   t->sdir_count = nt.sdir_count; t->sdir_bits = nt.sdir_bits;
   nt.d_leaf = nt.d_inner = nt.d_inner_idx = nt.d_dir = nt.d_sdir = nt.d_sdir_full = nullptr;
-  return HBT_OK;
+  // the rebuilt L-segment goes back where the caller placed the old one
+  return where ? leaf_place(t, where) : HBT_OK;
 }
 
 }  // namespace

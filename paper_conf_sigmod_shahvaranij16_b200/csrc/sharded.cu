@@ -189,8 +189,8 @@ int first_last_keys(const hbt_tree* t, uint64_t* kmin, uint64_t* kmax) {
   const uint32_t S = t->width, P = t->P;
   const uint64_t last = t->n - 1;
   uint64_t a = 0, b = 0;
-  HBT_CUDA_TRY(cudaMemcpy(&a, (const uint8_t*)t->d_leaf, S, cudaMemcpyDeviceToHost));
-  HBT_CUDA_TRY(cudaMemcpy(&b, (const uint8_t*)t->d_leaf + (last / P) * 64 + (last % P) * S, S, cudaMemcpyDeviceToHost));
+  HBT_CUDA_TRY(cudaMemcpy(&a, (const uint8_t*)t->d_leaf, S, cudaMemcpyDefault));
+  HBT_CUDA_TRY(cudaMemcpy(&b, (const uint8_t*)t->d_leaf + (last / P) * 64 + (last % P) * S, S, cudaMemcpyDefault));
   *kmin = a;
   *kmax = b;
   return HBT_OK;

@@ -48,6 +48,9 @@ def test_invalid_arguments_without_launch():
     assert b"fanout" in L.hbt_last_error() or True
     assert L.hbt_search(None, None, 1, hbt._Out(0, 0), None) == hbt.EINVAL
     assert L.hbt_destroy(None) == hbt.EINVAL
+    assert L.hbt_set_leaf_placement(None, 1) == hbt.EINVAL
+    w = C.c_uint32()
+    assert L.hbt_get_leaf_placement(None, C.byref(w)) == hbt.EINVAL
     assert L.hbt_info(None, None) == hbt.EINVAL
     assert hbt.version().startswith("hbt")
 

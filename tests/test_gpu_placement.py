@@ -1,0 +1,98 @@
+"""GPU parity with the L-segment in pinned HOST memory (hbt_set_leaf_placement, the
+paper's I-segment-on-GPU / L-segment-in-host split; SURVEY 8(f)
+f4): every search mode, the bucketed search, range scans and rebuilding updates must
+give the oracle's results with the leaf lines read by zero-copy loads, and the
+placement must survive an update and move back to HBM."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from gpu_util import from_dev, gpu_build, gpu_search, to_dev
+from test_gpu_implicit import expected_implicit_bytes
+from test_gpu_range import check as range_check, ranges
+from test_oracle_implicit import gen_keys, query_set
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def hbt():
+    import paper_conf_sigmod_shahvaranij16_b200 as m
+    assert torch.cuda.is_available(), "gpu tests need a CUDA device"
+    return m
+
+
+@pytest.mark.parametrize("width,F", [(8, 16), (4, 8), (8, 32), (4, 4)])
+def test_host_leaves_search_modes(hbt, width, F):
+    rng = np.random.default_rng(31 * F + width)
+    P = 64 // (2 * width)
+    for n in [0, 1, P + 1, F * P + 1, 5000, 300000]:
+        k, v = gen_keys(n, width, rng, dup=(n % 2 == 1), with_max=(n % 3 == 0))
+        o = oracle.ITree.from_pairs(k, v, F, width)
+        t = gpu_build(hbt, k, v, F, width)
+        t.set_leaf_placement("host")
+        assert t.leaf_placement == "host"
+        inner, leaf = expected_implicit_bytes(o, width)
+        assert t.export(hbt.SEG_LEAF).tobytes() == leaf  # the copy is bitwise the build
+        q = query_set(k, width, rng, 20000)
+        epf, ev = o.search(q)
+        for mode, l2b in ((2, 0), (2, 1), (3, 0), (0, 0)):
+            t.set_search_config(smem_mode=mode)
+            t.set_param("l2_levels_bytes", l2b)
+            t.set_param("small_batch", 0)
+            pf, val = gpu_search(t, q, width)
+            assert np.array_equal(pf, epf), (n, mode, l2b)
+            assert np.array_equal(val, ev), (n, mode, l2b)
+        t.set_search_config(smem_mode=2)
+        t.set_param("bucket", 1)  # bucketed search (splitters and item directory read the host leaves)
+        pf, val = gpu_search(t, q, width)
+        assert np.array_equal(pf, epf) and np.array_equal(val, ev), n
+        t.set_param("bucket", 2)
+        t.set_leaf_placement("device")
+        assert t.leaf_placement == "device"
+        assert t.export(hbt.SEG_LEAF).tobytes() == leaf
+        pf, val = gpu_search(t, q, width)
+        assert np.array_equal(pf, epf) and np.array_equal(val, ev), n
+        t.close()
+
+
+@pytest.mark.parametrize("width", [4, 8])
+def test_host_leaves_update_and_range(hbt, width):
+    rng = np.random.default_rng(5 + width)
+    F = 8
+    k, v = gen_keys(20000, width, rng, dup=True)
+    o = oracle.ITree.from_pairs(k, v, F, width)
+    t = gpu_build(hbt, k, v, F, width)
+    t.set_leaf_placement("host")
+    mx = (1 << (8 * width)) - 1
+    for _ in range(3):
+        nops = 3000
+        ok = np.where(rng.random(nops) < 0.5, k[rng.integers(0, len(k), nops)],
+                      rng.integers(0, mx, nops, dtype=np.uint64, endpoint=True)).astype(np.uint64)
+        ov = rng.integers(0, mx, nops, dtype=np.uint64, endpoint=True)
+        op = (rng.random(nops) < 0.4).astype(np.uint8)
+        o = o.update(ok, ov, op)
+        t.update(to_dev(ok, width), to_dev(ov, width), torch.from_numpy(op).cuda())
+        assert t.leaf_placement == "host"  # the rebuild keeps the placement
+        inner, leaf = expected_implicit_bytes(o, width)
+        assert t.export(hbt.SEG_INNER).tobytes() == inner
+        assert t.export(hbt.SEG_LEAF).tobytes() == leaf
+        q = query_set(ok[:500], width, rng, 4000)
+        pf, val = gpu_search(t, q, width)
+        epf, ev = o.search(q)
+        assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+    Kd, _ = oracle.dedupe(k, v)
+    lo, hi = ranges(Kd, width, rng, 500)
+    for kk in (1, 9, 40):
+        range_check(t, o, lo, hi, kk, width)
+    t.close()
+
+
+def test_host_leaves_rejected_for_regular(hbt):
+    k = np.arange(1, 1001, dtype=np.uint64) * 3
+    t = gpu_build(hbt, k, k, 8, 8, layout="regular")
+    with pytest.raises(hbt.HBTError) as e:
+        t.set_leaf_placement("host")
+    assert e.value.code == hbt.EUNSUPPORTED
+    t.close()
