@@ -219,6 +219,12 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *                 lanes' 16 B loads (0, default; measured faster on c2)
  *   "full256"     implicit whole-node levels: 256-bit lane loads (1, default) or 16 B lane
  *                 loads (0)
+ *   "leaf_stream" L-segment in host memory (hbt_set_leaf_placement): 0 = zero-copy leaf
+ *                 reads; 1 = bucket the batch and stream each bucket's leaf slice into HBM
+ *                 (double-buffered copies overlapping the previous bucket's search);
+ *                 2 = auto (default: stream when 160 B x m exceeds the L-segment bytes)
+ *   "stream_slice" host L-segment bytes per streamed bucket (0 = default 8 MB; at most
+ *                 1024 buckets)
  *   "full_levels" implicit: bit d set = level d's nodes are read whole in one round trip
  *                 (0 = default: by the "l2_levels_bytes" budget)
  * Unknown names or out-of-range values return HBT_EINVAL. */

@@ -147,6 +147,7 @@ static void free_tree(hbt_tree* t) {
 }
 
 static int device_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+  if (t->h_leaf && leaf_stream_enabled(t, m)) return streamed_search(t, q, m, pf, v, 0, s);
   if (bucketed_enabled(t, m)) return bucketed_search(t, q, m, pf, v, 0, s);
   return t->form == HBT_REGULAR ? regular_search(t, q, m, pf, v, s) : implicit_search(t, q, m, pf, v, s);
 }
@@ -278,6 +279,7 @@ int hbt_bulk_update(hbt_tree* t, const hbt_batch* batch, void* stream) {
   }
   cudaStream_t s = (cudaStream_t)stream;
   t->bk.valid = false;  // bucket splitters follow the tree
+  t->bks.valid = false;
   return t->form == HBT_REGULAR ? regular_update(t, batch, s) : implicit_update(t, batch, s);
 }
 
@@ -396,6 +398,8 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "bucket_slice" && value >= 0) { c.bucket_slice = uint64_t(value); t->bk.valid = false; }
   else if (n == "bucket_items" && (value == 0 || value == 1)) { c.bucket_items = uint32_t(value); t->bk.valid = false; }
   else if (n == "bucket_cap" && value >= 0 && value < (1 << 20)) { c.bucket_cap = uint32_t(value); t->bk.valid = false; }
+  else if (n == "leaf_stream" && value >= 0 && value <= 2) c.leaf_stream = uint32_t(value);
+  else if (n == "stream_slice" && value >= 0) { c.stream_slice = uint64_t(value); t->bks.valid = false; }
   else if (n == "phase_timing" && (value == 0 || value == 1)) c.phase_timing = uint32_t(value);
   else if (n == "leaf256" && (value == 0 || value == 1)) c.leaf256 = uint32_t(value);
   else if (n == "sec256" && (value == 0 || value == 1)) c.sec256 = uint32_t(value);

@@ -32,6 +32,8 @@
 // on its own; only the order in which queries are processed changes).
 // Extra HBM traffic per query (u64): 8 + 2 | 2 + 8 + 8 + 2 | - | 2 + 16 + 16.
 #include <algorithm>
+#include <mutex>
+#include <vector>
 
 #include <cub/cub.cuh>
 
@@ -483,6 +485,22 @@ __global__ void __launch_bounds__(kGThreads) bk_gather_rec(const uint16_t* __res
   }
 }
 
+// Dynamic shared memory beyond 48 KB for the partition kernels (once per process).
+void set_bucket_attrs() {
+  static bool attr = false;
+  if (attr) return;
+  const int lim = 120 * 1024;
+  cudaFuncSetAttribute(bk_count<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
+  cudaFuncSetAttribute(bk_count<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
+  cudaFuncSetAttribute(bk_scatter<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
+  cudaFuncSetAttribute(bk_scatter<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
+  cudaFuncSetAttribute(bk_gather<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
+  cudaFuncSetAttribute(bk_gather<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
+  cudaFuncSetAttribute(bk_gather_rec<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+  cudaFuncSetAttribute(bk_gather_rec<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+  attr = true;
+}
+
 uint64_t tree_bytes(const hbt_tree* t) {
   if (t->form == HBT_IMPLICIT) return t->inner_bytes + t->inner_idx_bytes + t->leaf_bytes;
   const RegularState& r = t->r;
@@ -513,9 +531,7 @@ uint64_t item_cap(const hbt_tree* t, uint32_t B) {
 }
 
 template <typename K>
-int prepare_splitters(const hbt_tree* t, cudaStream_t s) {
-  BucketState& bs = t->bk;
-  const uint32_t B = pick_buckets(t);
+int prepare_splitters(const hbt_tree* t, cudaStream_t s, BucketState& bs, uint32_t B, bool want_items) {
   if (bs.valid && bs.B == B) return HBT_OK;
   if (!bs.d_sp) {
     HBT_CUDA_TRY(cudaMalloc(&bs.d_sp, kMaxBuckets * 8));
@@ -533,7 +549,7 @@ int prepare_splitters(const hbt_tree* t, cudaStream_t s) {
   // Item directory: the deepest unit level whose range for two buckets fits the
   // shared-memory capacity.
   bs.items = false;
-  if (t->cfg.bucket_items) {
+  if (want_items && t->cfg.bucket_items) {
     const uint64_t cap = item_cap(t, B);
     uint64_t nunits = 0;
     if (t->form == HBT_IMPLICIT) {
@@ -586,7 +602,7 @@ int prepare_splitters(const hbt_tree* t, cudaStream_t s) {
 template <typename K>
 int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
                cudaStream_t s) {
-  int rc = prepare_splitters<K>(t, s);
+  int rc = prepare_splitters<K>(t, s, t->bk, pick_buckets(t), true);
   if (rc != HBT_OK) return rc;
   const BucketState& bs = t->bk;
   const uint32_t B = bs.B;
@@ -626,19 +642,7 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
     const size_t smem_scatter = kChunk * (sizeof(K) + 2) + kMaxBuckets * 4 * 4 + kThreads * 4;
     const size_t smem_gather = kChunk * (8 + 2) + kMaxBuckets * 4 * 3 + kThreads * 4;
     const size_t smem_gather_rec = kChunk * (16 + 2) + kMaxBuckets * 4 * 3 + kGThreads * 4;
-    static bool attr = false;
-    if (!attr) {
-      const int lim = 120 * 1024;
-      cudaFuncSetAttribute(bk_count<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
-      cudaFuncSetAttribute(bk_count<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
-      cudaFuncSetAttribute(bk_scatter<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
-      cudaFuncSetAttribute(bk_scatter<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
-      cudaFuncSetAttribute(bk_gather<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
-      cudaFuncSetAttribute(bk_gather<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
-      cudaFuncSetAttribute(bk_gather_rec<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-      cudaFuncSetAttribute(bk_gather_rec<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-      attr = true;
-    }
+    set_bucket_attrs();
     const unsigned grid = unsigned(std::min<uint64_t>(chunks, uint64_t(t->num_sms) * 2));
     mark(0);
     bk_count<K><<<grid, kThreads, smem_count, s>>>((const K*)q, m, (const K*)bs.d_sp, bs.d_dir, B, chunks, bq, tab);
@@ -709,7 +713,149 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
   return rc;
 }
 
+// ---- streamed host L-segment (the paper's bucket pipeline with double
+// buffering, turned around: the BATCH is bucketed on the GPU and the
+// L-SEGMENT slices stream host -> HBM).  With the L-segment in pinned host memory a
+// batch that touches most of it is cheaper to serve by copying each bucket's leaf
+// slice into HBM at the link's copy rate than by one random 64 B zero-copy read per
+// query (measured 22 GB/s vs a 55 GB/s copy rate).  Bucket b's queries all answer in
+// the leaf lines [floor(bU/B), floor((b+1)U/B)) (sp[b-1] < q <= sp[b], DESIGN.md
+// 'Bucketed search'), so its search reads only that staged slice; the inner levels
+// stay in HBM.  Slice copies (one stream) alternate between two staging slots and
+// overlap the previous bucket's search; results are identical.
+uint64_t stream_slice_bytes(const hbt_tree* t) {
+  return t->cfg.stream_slice ? t->cfg.stream_slice : (8ull << 20);
+}
+
+uint32_t pick_stream_buckets(const hbt_tree* t) {
+  uint64_t B = (t->leaf_bytes + stream_slice_bytes(t) - 1) / stream_slice_bytes(t);
+  B = std::min<uint64_t>(B, kMaxBuckets);
+  B = std::min<uint64_t>(B, t->L0);
+  return uint32_t(std::max<uint64_t>(B, 1));
+}
+
+template <typename K>
+int streamed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
+               cudaStream_t s) {
+  // one user of the staging slots at a time (not pipe.mu: hbt_search_host holds it
+  // while its chunks come through here)
+  std::lock_guard<std::mutex> lock(t->stream_mu);
+  BucketState& bs = t->bks;
+  const uint32_t B = pick_stream_buckets(t);
+  int rc = prepare_splitters<K>(t, s, bs, B, false);
+  if (rc != HBT_OK) return rc;
+  const uint64_t U = t->L0;
+  const uint64_t slice_lines = (U + B - 1) / B + 1;
+  if (bs.stage_cap < slice_lines * 64) {
+    cudaFree(bs.d_stage[0]);
+    bs.d_stage[0] = bs.d_stage[1] = nullptr;
+    bs.stage_cap = 0;
+    HBT_CUDA_TRY(cudaMalloc(&bs.d_stage[0], 2 * slice_lines * 64));
+    bs.d_stage[1] = static_cast<uint8_t*>(bs.d_stage[0]) + slice_lines * 64;
+    bs.stage_cap = slice_lines * 64;
+  }
+  if (!bs.cs) {
+    HBT_CUDA_TRY(cudaStreamCreateWithFlags(&bs.cs, cudaStreamNonBlocking));
+    for (int i = 0; i < 2; ++i) {
+      HBT_CUDA_TRY(cudaEventCreateWithFlags(&bs.ev_copy[i], cudaEventDisableTiming));
+      HBT_CUDA_TRY(cudaEventCreateWithFlags(&bs.ev_done[i], cudaEventDisableTiming));
+      HBT_CUDA_TRY(cudaEventRecord(bs.ev_done[i], s));  // slots start free
+    }
+  }
+  const uint64_t chunks = (m + kChunk - 1) / kChunk;
+  const uint64_t ntab = uint64_t(B) * chunks;
+  size_t scan_bytes = 0;
+  HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, scan_bytes, (const uint32_t*)nullptr, (uint32_t*)nullptr,
+                                             ntab, s));
+  auto al = [](uint64_t x) { return (x + 255) & ~uint64_t(255); };
+  const uint64_t o_pf = al(m * sizeof(K)), o_v = o_pf + al(m * 8), o_bq = o_v + al(m * sizeof(K)),
+                 o_li = o_bq + al(m * 2), o_tab = o_li + al(m * 2), o_gb = o_tab + al(ntab * 4),
+                 o_bm = o_gb + al(ntab * 4), o_bm2 = o_bm + al(ntab * 4), o_bs = o_bm2 + al(ntab * 4),
+                 o_tmp = o_bs + al((uint64_t(B) + 1) * 8), total = o_tmp + al(scan_bytes);
+  void* buf = nullptr;
+  HBT_CUDA_TRY(scratch_alloc(&buf, total, s));
+  uint8_t* base = static_cast<uint8_t*>(buf);
+  K* qs = reinterpret_cast<K*>(base);
+  uint64_t* pf_s = reinterpret_cast<uint64_t*>(base + o_pf);
+  K* v_s = reinterpret_cast<K*>(base + o_v);
+  uint16_t* bq = reinterpret_cast<uint16_t*>(base + o_bq);
+  uint16_t* linv = reinterpret_cast<uint16_t*>(base + o_li);
+  uint32_t* tab = reinterpret_cast<uint32_t*>(base + o_tab);
+  uint32_t* gb = reinterpret_cast<uint32_t*>(base + o_gb);
+  uint32_t* tab_bm = reinterpret_cast<uint32_t*>(base + o_bm);
+  uint32_t* gb_bm = reinterpret_cast<uint32_t*>(base + o_bm2);
+  uint64_t* bstart = reinterpret_cast<uint64_t*>(base + o_bs);
+  std::vector<uint64_t> hb(B + 1);
+  do {
+    const size_t smem_count = (1u << kDirBits) * 4 + kMaxBuckets * 4 + kMaxBuckets * sizeof(K);
+    const size_t smem_scatter = kChunk * (sizeof(K) + 2) + kMaxBuckets * 4 * 4 + kThreads * 4;
+    const size_t smem_gather = kChunk * (8 + 2) + kMaxBuckets * 4 * 3 + kThreads * 4;
+    const unsigned grid = unsigned(std::min<uint64_t>(chunks, uint64_t(t->num_sms) * 2));
+    set_bucket_attrs();
+    bk_count<K><<<grid, kThreads, smem_count, s>>>((const K*)q, m, (const K*)bs.d_sp, bs.d_dir, B, chunks, bq, tab);
+    const dim3 tb(32, 8);
+    bk_transpose<<<dim3((B + 31) / 32, unsigned((chunks + 31) / 32)), tb, 0, s>>>(tab, chunks, B, tab_bm);
+    if (cub::DeviceScan::ExclusiveSum(base + o_tmp, scan_bytes, tab_bm, gb_bm, ntab, s) != cudaSuccess) {
+      set_error("bucket scan failed");
+      rc = HBT_ECUDA;
+      break;
+    }
+    bk_transpose<<<dim3(unsigned((chunks + 31) / 32), (B + 31) / 32), tb, 0, s>>>(gb_bm, B, uint32_t(chunks), gb);
+    bk_bstart<<<(B + 256) / 256, 256, 0, s>>>(gb_bm, chunks, B, m, bstart);
+    bk_scatter<K><<<grid, kThreads, smem_scatter, s>>>((const K*)q, m, bq, tab, gb, B, chunks, qs, linv);
+    if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) {
+      set_error("bucketing kernels failed to launch: %s", cudaGetErrorString(e));
+      rc = HBT_ECUDA;
+      break;
+    }
+    // the bucket boundaries drive the host loop below (one sync per batch)
+    HBT_CUDA_TRY(cudaMemcpyAsync(hb.data(), bstart, (B + 1) * 8, cudaMemcpyDeviceToHost, s));
+    HBT_CUDA_TRY(cudaStreamSynchronize(s));
+    const uint8_t* hl = static_cast<const uint8_t*>(t->h_leaf);
+    uint32_t j = 0;
+    for (uint32_t b = 0; b < B && rc == HBT_OK; ++b) {
+      const uint64_t cnt = hb[b + 1] - hb[b];
+      if (!cnt) continue;
+      const uint64_t u_lo = (uint64_t(b) * U) / B, u_hi = ((uint64_t(b) + 1) * U) / B;
+      const int slot = int(j++ & 1);
+      uint8_t* st = static_cast<uint8_t*>(bs.d_stage[slot]);
+      HBT_CUDA_TRY(cudaStreamWaitEvent(bs.cs, bs.ev_done[slot], 0));
+      HBT_CUDA_TRY(cudaMemcpyAsync(st, hl + u_lo * 64, (u_hi - u_lo) * 64, cudaMemcpyHostToDevice, bs.cs));
+      HBT_CUDA_TRY(cudaEventRecord(bs.ev_copy[slot], bs.cs));
+      HBT_CUDA_TRY(cudaStreamWaitEvent(s, bs.ev_copy[slot], 0));
+      rc = implicit_search_leaf(t, qs + hb[b], cnt, pf_s + hb[b], v_s + hb[b], pos_base,
+                                st - int64_t(u_lo) * 64, s);
+      HBT_CUDA_TRY(cudaEventRecord(bs.ev_done[slot], s));
+    }
+    if (rc != HBT_OK) break;
+    bk_gather<K><<<grid, kThreads, smem_gather, s>>>(linv, m, tab, gb, B, chunks, pf_s, v_s, pf, (K*)v);
+    if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) {
+      set_error("bucket gather failed to launch: %s", cudaGetErrorString(e));
+      rc = HBT_ECUDA;
+      break;
+    }
+  } while (0);
+  scratch_free(buf, s);
+  return rc;
+}
+
 }  // namespace
+
+bool leaf_stream_enabled(const hbt_tree* t, uint64_t m) {
+  if (t->form != HBT_IMPLICIT || !t->h_leaf || m == 0 || m >= (1ull << 32)) return false;
+  const uint32_t mode = t->cfg.leaf_stream;
+  if (mode == 0 || pick_stream_buckets(t) < 2) return false;
+  if (mode == 1) return true;
+  // auto: stream when the batch's random 64 B link reads (~22 GB/s measured) would
+  // cost more than copying the whole L-segment (~55 GB/s): m * 64 / 22 > L / 55
+  return m * 160 > t->leaf_bytes;
+}
+
+int streamed_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
+                    cudaStream_t s) {
+  return t->width == 4 ? streamed_t<uint32_t>(t, q, m, pf, v, pos_base, s)
+                       : streamed_t<uint64_t>(t, q, m, pf, v, pos_base, s);
+}
 
 bool bucketed_enabled(const hbt_tree* t, uint64_t m) {
   const uint32_t mode = t->cfg.bucket;
@@ -738,13 +884,24 @@ int shard_local_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* p
   return implicit_search_base(t, q, m, pf, v, pos_base, s);
 }
 
-void bucket_free(hbt_tree* t) {
-  for (auto& e : t->bk.ev)
+static void bucket_state_free(BucketState& b) {
+  for (auto& e : b.ev)
     if (e) cudaEventDestroy(e);
-  cudaFree(t->bk.d_sp);
-  cudaFree(t->bk.d_dir);
-  cudaFree(t->bk.d_M);
-  t->bk = BucketState{};
+  for (int i = 0; i < 2; ++i) {
+    if (b.ev_copy[i]) cudaEventDestroy(b.ev_copy[i]);
+    if (b.ev_done[i]) cudaEventDestroy(b.ev_done[i]);
+  }
+  if (b.cs) cudaStreamDestroy(b.cs);
+  cudaFree(b.d_stage[0]);
+  cudaFree(b.d_sp);
+  cudaFree(b.d_dir);
+  cudaFree(b.d_M);
+  b = BucketState{};
+}
+
+void bucket_free(hbt_tree* t) {
+  bucket_state_free(t->bk);
+  bucket_state_free(t->bks);
 }
 
 }  // namespace hbt

@@ -63,6 +63,9 @@ struct SearchConfig {
   uint32_t bucket_items = 1;     // bucketed search: bucket-local shared-memory directory (ItemDir)
   uint32_t bucket_cap = 0;       // item directory: shared-memory entries (0 = derived; tests force the fallback)
   uint32_t phase_timing = 0;     // bucketed search: CUDA events around each phase (hbt_last_phases)
+  uint32_t leaf_stream = 2;      // host L-segment: 0 = zero-copy leaf reads, 1 = stream bucket slices
+                                 // into HBM (bucketed, double-buffered copies), 2 = auto (by batch size)
+  uint64_t stream_slice = 0;     // host L-segment bytes per streamed bucket (0 = 8 MB)
   uint32_t leaf256 = 1;          // leaf line by two 256-bit lane loads (one 64 B request per group)
   uint32_t sec256 = 0;           // implicit L2 levels: index / key sector by one lane's 256-bit load
   uint32_t full256 = 1;          // implicit whole-node levels by 256-bit lane loads
@@ -106,6 +109,12 @@ struct BucketState {
   cudaEvent_t ev[6] = {};        // phase boundaries of the last timed bucketed search
   bool timed = false;
   uint32_t launches = 0;
+  // streamed host L-segment (bucketed.cu, streamed_t): two HBM staging slots for
+  // bucket leaf slices, a copy stream and the events that order slot reuse
+  void* d_stage[2] = {};
+  uint64_t stage_cap = 0;
+  cudaStream_t cs = nullptr;
+  cudaEvent_t ev_copy[2] = {}, ev_done[2] = {};
 };
 
 // Regular-tree device state.  All pools are SoA arrays
@@ -244,6 +253,8 @@ struct hbt_tree {
   hbt::SearchConfig cfg;
   mutable hbt::HostPipe pipe;
   mutable hbt::BucketState bk;
+  mutable hbt::BucketState bks;  // streamed host L-segment (own bucket count)
+  mutable std::mutex stream_mu;   // one user of the streamed staging slots at a time
 };
 
 namespace hbt {
@@ -258,6 +269,13 @@ int implicit_update(hbt_tree* t, const hbt_batch* b, cudaStream_t s);
 // implicit_search.cu
 int implicit_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s);
 // same, reporting global positions base + rank (sharded trees)
+// implicit search reading leaf lines at leafp + line * 64 (a staged slice's base
+// minus its first line; only lines inside the slice are dereferenced)
+int implicit_search_leaf(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
+                         const void* leafp, cudaStream_t s);
+bool leaf_stream_enabled(const hbt_tree* t, uint64_t m);
+int streamed_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
+                    cudaStream_t s);
 int implicit_search_base(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
                          cudaStream_t s);
 void shard_free(hbt_tree* t);

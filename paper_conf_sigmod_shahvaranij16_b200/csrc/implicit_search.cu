@@ -383,13 +383,15 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
 
   // MODE 2 pipelines the query stream across rounds: the next round's queries
   // are loaded while this round walks the tree (their HBM latency was the
-  // largest single stall, profiles/r01_c2_v11_*).
+  // largest single stall, profiles/r01_c2_v11_*).  Lanes past the batch end repeat
+  // the batch's last query (results discarded) so they walk to a leaf line the batch
+  // itself uses: a streamed host L-segment stages only the bucket's slice.
   K nextq[QPL];
   if constexpr (MODE >= 2) {
 #pragma unroll
     for (int u = 0; u < QPL; ++u) {
       const uint64_t i = warp * ROUND + uint64_t(u) * 32 + lane;
-      nextq[u] = (warp < rounds && i < m) ? ldcs(queries + i) : key_max<K>();
+      nextq[u] = warp < rounds ? ldcs(queries + (i < m ? i : m - 1)) : key_max<K>();
     }
   }
   for (uint64_t rd = warp; rd < rounds; rd += nwarps) {
@@ -404,10 +406,10 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
       if constexpr (MODE >= 2) {
         myq[u] = nextq[u];
         const uint64_t i = (rd + nwarps) * ROUND + uint64_t(u) * 32 + lane;
-        nextq[u] = (rd + nwarps < rounds && i < m) ? ldcs(queries + i) : key_max<K>();
+        nextq[u] = rd + nwarps < rounds ? ldcs(queries + (i < m ? i : m - 1)) : key_max<K>();
       } else {
         const uint64_t i = base + uint64_t(u) * 32 + lane;
-        myq[u] = i < m ? ldcs(queries + i) : key_max<K>();
+        myq[u] = ldcs(queries + (i < m ? i : m - 1));
       }
       mynode[u] = 0;
     }
@@ -601,7 +603,7 @@ struct Launch {
 
   template <int QPL, int THREADS, int MODE>
   static int run_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t base,
-                   cudaStream_t s) {
+                   cudaStream_t s, const void* leafp) {
     auto kern = implicit_search_kernel<K, F, QPL, THREADS, MODE>;
     LevelTable lt{};
     for (uint32_t d = 0; d <= t->H; ++d) lt.offset[d] = t->offset[d];
@@ -691,7 +693,7 @@ struct Launch {
       lc.numAttrs = 1;
     }
     HBT_CUDA_TRY(cudaLaunchKernelEx(&lc, kern, (const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
-                                    (const uint8_t*)t->d_leaf,
+                                    (const uint8_t*)leafp,
                                     (const uint32_t*)(MODE == 4 ? t->d_sdir : t->d_dir),
                                     (const K*)t->d_sdir_full, (const K*)q, m, pf, (K*)v, lt, t->n, base));
     HBT_CUDA_TRY(cudaGetLastError());
@@ -733,42 +735,44 @@ struct Launch {
     return HBT_OK;
   }
 
-  static int run(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t b, cudaStream_t s) {
+  static int run(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t b, cudaStream_t s,
+                 const void* lp) {
     const uint32_t qpl = t->cfg.qpl ? t->cfg.qpl : 1;
     // 256-byte nodes (u64, F = 32) need more registers than a 1024-thread CTA allows
     const uint32_t th = t->cfg.threads ? t->cfg.threads : (C::NODE_BYTES > 128 ? 512 : 1024);
     // small batches read the directory in place (no 96 KB staging per CTA)
     if (t->cfg.mode == 3 || (t->cfg.mode == 2 && m <= t->cfg.small_batch))
       // 256-thread CTAs spread a small batch over every SM (c1: 10.1 -> 8.3 us per batch)
-      return t->cfg.threads == 1024 ? run_t<1, 1024, 3>(t, q, m, pf, v, b, s) : run_t<1, 256, 3>(t, q, m, pf, v, b, s);
+      return t->cfg.threads == 1024 ? run_t<1, 1024, 3>(t, q, m, pf, v, b, s, lp) : run_t<1, 256, 3>(t, q, m, pf, v, b, s, lp);
     if (t->cfg.mode == 4 && t->d_sdir)
-      return th == 512 ? run_t<1, 512, 4>(t, q, m, pf, v, b, s) : run_t<1, 1024, 4>(t, q, m, pf, v, b, s);
+      return th == 512 ? run_t<1, 512, 4>(t, q, m, pf, v, b, s, lp) : run_t<1, 1024, 4>(t, q, m, pf, v, b, s, lp);
     if (t->cfg.mode == 2) {
-      if (th == 512) return run_t<1, 512, 2>(t, q, m, pf, v, b, s);
-      if (th == 768) return qpl == 2 ? run_t<2, 768, 2>(t, q, m, pf, v, b, s) : run_t<1, 768, 2>(t, q, m, pf, v, b, s);
-      return qpl == 2 ? run_t<2, 1024, 2>(t, q, m, pf, v, b, s) : run_t<1, 1024, 2>(t, q, m, pf, v, b, s);
+      if (th == 512) return run_t<1, 512, 2>(t, q, m, pf, v, b, s, lp);
+      if (th == 768) return qpl == 2 ? run_t<2, 768, 2>(t, q, m, pf, v, b, s, lp) : run_t<1, 768, 2>(t, q, m, pf, v, b, s, lp);
+      return qpl == 2 ? run_t<2, 1024, 2>(t, q, m, pf, v, b, s, lp) : run_t<1, 1024, 2>(t, q, m, pf, v, b, s, lp);
     }
     const bool hilo = t->cfg.mode == 1;
     if (hilo) {
-      if (qpl == 2) return th == 256 ? run_t<2, 256, 1>(t, q, m, pf, v, b, s) : run_t<2, 512, 1>(t, q, m, pf, v, b, s);
-      return th == 256 ? run_t<1, 256, 1>(t, q, m, pf, v, b, s) : run_t<1, 512, 1>(t, q, m, pf, v, b, s);
+      if (qpl == 2) return th == 256 ? run_t<2, 256, 1>(t, q, m, pf, v, b, s, lp) : run_t<2, 512, 1>(t, q, m, pf, v, b, s, lp);
+      return th == 256 ? run_t<1, 256, 1>(t, q, m, pf, v, b, s, lp) : run_t<1, 512, 1>(t, q, m, pf, v, b, s, lp);
     }
     if (qpl == 2) {
-      if (th == 1024) return run_t<2, 1024, 0>(t, q, m, pf, v, b, s);
-      return th == 256 ? run_t<2, 256, 0>(t, q, m, pf, v, b, s) : run_t<2, 512, 0>(t, q, m, pf, v, b, s);
+      if (th == 1024) return run_t<2, 1024, 0>(t, q, m, pf, v, b, s, lp);
+      return th == 256 ? run_t<2, 256, 0>(t, q, m, pf, v, b, s, lp) : run_t<2, 512, 0>(t, q, m, pf, v, b, s, lp);
     }
-    if (th == 1024) return run_t<1, 1024, 0>(t, q, m, pf, v, b, s);
-    return th == 256 ? run_t<1, 256, 0>(t, q, m, pf, v, b, s) : run_t<1, 512, 0>(t, q, m, pf, v, b, s);
+    if (th == 1024) return run_t<1, 1024, 0>(t, q, m, pf, v, b, s, lp);
+    return th == 256 ? run_t<1, 256, 0>(t, q, m, pf, v, b, s, lp) : run_t<1, 512, 0>(t, q, m, pf, v, b, s, lp);
   }
 };
 
 template <typename K>
-int dispatch_f(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t b, cudaStream_t s) {
+int dispatch_f(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t b, cudaStream_t s,
+               const void* lp) {
   switch (t->F) {
-    case 4: return Launch<K, 4>::run(t, q, m, pf, v, b, s);
-    case 8: return Launch<K, 8>::run(t, q, m, pf, v, b, s);
-    case 16: return Launch<K, 16>::run(t, q, m, pf, v, b, s);
-    case 32: return Launch<K, 32>::run(t, q, m, pf, v, b, s);
+    case 4: return Launch<K, 4>::run(t, q, m, pf, v, b, s, lp);
+    case 8: return Launch<K, 8>::run(t, q, m, pf, v, b, s, lp);
+    case 16: return Launch<K, 16>::run(t, q, m, pf, v, b, s, lp);
+    case 32: return Launch<K, 32>::run(t, q, m, pf, v, b, s, lp);
   }
   set_error("unsupported fanout %u", t->F);
   return HBT_EINVAL;
@@ -796,8 +800,14 @@ uint32_t implicit_idx_stride(uint32_t F, uint32_t S) {
 
 int implicit_search_base(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t base,
                          cudaStream_t s) {
+  return implicit_search_leaf(t, q, m, pf, v, base, t->d_leaf, s);
+}
+
+int implicit_search_leaf(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t base,
+                         const void* lp, cudaStream_t s) {
   if (m == 0) return HBT_OK;
-  return t->width == 4 ? dispatch_f<uint32_t>(t, q, m, pf, v, base, s) : dispatch_f<uint64_t>(t, q, m, pf, v, base, s);
+  return t->width == 4 ? dispatch_f<uint32_t>(t, q, m, pf, v, base, s, lp)
+                       : dispatch_f<uint64_t>(t, q, m, pf, v, base, s, lp);
 }
 
 int implicit_search_items(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, const ItemDir& d,

@@ -45,6 +45,13 @@ def test_host_leaves_search_modes(hbt, width, F):
             assert np.array_equal(pf, epf), (n, mode, l2b)
             assert np.array_equal(val, ev), (n, mode, l2b)
         t.set_search_config(smem_mode=2)
+        # streamed slices: many small buckets, the 1024-bucket cap, and auto
+        for ls, slice_ in ((1, 4096), (1, 64), (1, 0), (2, 0)):
+            t.set_param("leaf_stream", ls)
+            t.set_param("stream_slice", slice_)
+            pf, val = gpu_search(t, q, width)
+            assert np.array_equal(pf, epf) and np.array_equal(val, ev), (n, ls, slice_)
+        t.set_param("leaf_stream", 0)
         t.set_param("bucket", 1)  # bucketed search (splitters and item directory read the host leaves)
         pf, val = gpu_search(t, q, width)
         assert np.array_equal(pf, epf) and np.array_equal(val, ev), n
@@ -79,9 +86,12 @@ def test_host_leaves_update_and_range(hbt, width):
         assert t.export(hbt.SEG_INNER).tobytes() == inner
         assert t.export(hbt.SEG_LEAF).tobytes() == leaf
         q = query_set(ok[:500], width, rng, 4000)
-        pf, val = gpu_search(t, q, width)
         epf, ev = o.search(q)
-        assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+        for ls in (0, 1):
+            t.set_param("leaf_stream", ls)
+            t.set_param("stream_slice", 2048)
+            pf, val = gpu_search(t, q, width)
+            assert np.array_equal(pf, epf) and np.array_equal(val, ev), ls
     Kd, _ = oracle.dedupe(k, v)
     lo, hi = ranges(Kd, width, rng, 500)
     for kk in (1, 9, 40):
@@ -95,4 +105,24 @@ def test_host_leaves_rejected_for_regular(hbt):
     with pytest.raises(hbt.HBTError) as e:
         t.set_leaf_placement("host")
     assert e.value.code == hbt.EUNSUPPORTED
+    t.close()
+
+
+def test_host_leaves_streamed_through_host_pipeline(hbt):
+    """hbt_search_host (host buffers, chunked over two streams) on a tree whose
+    L-segment streams from host memory: the streamed search runs inside the host
+    pipeline's chunks (its own lock; a shared one deadlocked)."""
+    width, F = 8, 16
+    rng = np.random.default_rng(77)
+    k, v = gen_keys(300000, width, rng)
+    o = oracle.ITree.from_pairs(k, v, F, width)
+    t = gpu_build(hbt, k, v, F, width)
+    t.set_leaf_placement("host")
+    t.set_param("stream_slice", 65536)  # many buckets; auto mode streams this batch
+    q = query_set(k, width, rng, 1 << 20)
+    hp = np.empty(len(q), np.uint64)
+    hv = np.empty(len(q), np.uint64)
+    t.search_host(np.ascontiguousarray(q), hp, hv)
+    epf, ev = o.search(q, nthreads=oracle.default_threads())
+    assert np.array_equal(hp, epf) and np.array_equal(hv, ev)
     t.close()
