@@ -61,6 +61,8 @@ def parse():
     ap.add_argument("--leaf256", type=int, default=None, help="leaf / key lines by 256-bit lane loads: 0 | 1")
     ap.add_argument("--sec256", type=int, default=None, help="implicit L2-level sectors by one lane's 256-bit load")
     ap.add_argument("--full-levels", type=int, default=None, help="implicit: bit mask of levels read whole")
+    ap.add_argument("--origin-rank0", action="store_true",
+                    help="replicated configs: all queries start on rank 0 (NCCL scatter / gather in the step)")
     ap.add_argument("--leaf-host", action="store_true",
                     help="implicit trees: L-segment in pinned host memory (the paper's split, SURVEY f4)")
     ap.add_argument("--graph", default="auto", choices=["0", "1", "auto"],
@@ -74,7 +76,10 @@ def parse():
                          "DELETEs; c3 does 1%% by default) and time search again")
     ap.add_argument("--range-k", type=int, default=0,
                     help="time range scans returning k keys per query (PAPER.md:392) instead of point lookups")
-    return ap.parse_args()
+    a = ap.parse_args()
+    if a.origin_rank0 and a.config == "c4":
+        ap.error("--origin-rank0 is for replicated trees; c4 routes queries by key range")
+    return a
 
 
 def dist_env():
@@ -267,12 +272,41 @@ def make_work(cfg_name, rank, world, args):
     if args.range_k:
         hi = torch.full_like(q, -1)  # MAX: every range returns k keys unless the tree ends
         qdesc += f"; range scans of {args.range_k} keys from each query key"
+    origin = None
+    if args.origin_rank0:
+        # the batch of every rank starts on rank 0 (gathered there once, untimed); each
+        # step scatters it, searches and gathers the results back to rank 0
+        import torch.distributed as dist
+        if world > 1:
+            full = torch.empty(world * m, dtype=q.dtype, device="cuda") if rank == 0 else None
+            dist.gather(q, list(full.chunk(world)) if rank == 0 else None, dst=0)
+        else:
+            full = q.clone()
+        origin = {"full": full, "recv": torch.empty_like(q),
+                  "gpos": torch.empty(world * m, dtype=torch.int64, device="cuda") if rank == 0 else None,
+                  "gval": torch.empty(world * m, dtype=sdt, device="cuda") if rank == 0 else None}
+        qdesc += "; the queries of all ranks originate on rank 0 (scatter + gather inside each step)"
     return Work(c=c, name=cfg_name, tree=tree, q=q, m=m, w=w, hit_rate=hit_rate, qdesc=qdesc, extra=extra,
-                out_pos=out_pos, out_val=out_val, info=tree.info(), range_k=args.range_k, hi=hi)
+                out_pos=out_pos, out_val=out_val, info=tree.info(), range_k=args.range_k, hi=hi,
+                origin=origin, rank=rank, world=world)
 
 
 def step(work):
     """One step: the whole batch through the hot path."""
+    o = getattr(work, "origin", None)
+    if o is not None:  # queries originate on rank 0: scatter, search, gather (SURVEY 8(e).1)
+        import torch.distributed as dist
+        if work.world > 1:
+            dist.scatter(o["recv"], list(o["full"].chunk(work.world)) if work.rank == 0 else None, src=0)
+            work.tree.search(o["recv"], work.out_pos, work.out_val)
+            dist.gather(work.out_pos, list(o["gpos"].chunk(work.world)) if work.rank == 0 else None, dst=0)
+            dist.gather(work.out_val, list(o["gval"].chunk(work.world)) if work.rank == 0 else None, dst=0)
+        else:
+            o["recv"].copy_(o["full"])
+            work.tree.search(o["recv"], work.out_pos, work.out_val)
+            o["gpos"].copy_(work.out_pos)
+            o["gval"].copy_(work.out_val)
+        return
     if work.range_k:
         work.tree.range(work.q, work.hi, work.range_k)
     else:
@@ -431,7 +465,8 @@ def run_hbt(args):
     node_b = ((c["fanout"] * w + 31) // 32) * 32
     l2_probe = probe_l2_gbs(32 if node_b > 32 else node_b) if rank == 0 else None
 
-    use_graph = args.graph == "1" or (args.graph == "auto" and m <= (1 << 20) and args.config != "c4")
+    use_graph = args.graph == "1" or (args.graph == "auto" and m <= (1 << 20) and args.config != "c4"
+                                      and not args.origin_rank0)
     graph = capture_step(work) if use_graph else None
     for _ in range(max(args.warmup, 3)):
         if graph is not None:
