@@ -399,6 +399,7 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "bucket_items" && (value == 0 || value == 1)) { c.bucket_items = uint32_t(value); t->bk.valid = false; }
   else if (n == "bucket_cap" && value >= 0 && value < (1 << 20)) { c.bucket_cap = uint32_t(value); t->bk.valid = false; }
   else if (n == "leaf_stream" && value >= 0 && value <= 2) c.leaf_stream = uint32_t(value);
+  else if (n == "qprefetch" && (value == 0 || value == 1)) c.qprefetch = uint32_t(value);
   else if (n == "stream_slice" && value >= 0) { c.stream_slice = uint64_t(value); t->bks.valid = false; }
   else if (n == "phase_timing" && (value == 0 || value == 1)) c.phase_timing = uint32_t(value);
   else if (n == "leaf256" && (value == 0 || value == 1)) c.leaf256 = uint32_t(value);

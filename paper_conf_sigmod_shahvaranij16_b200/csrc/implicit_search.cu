@@ -547,6 +547,11 @@ implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* _
       }
       const uint64_t lu = threadIdx.x ? ((uint64_t(lo) + 1) * d.U) / d.B - 1 : (uint64_t(lo) * d.U) / d.B;
       s_range[threadIdx.x] = lu / d.span;
+    } else if (threadIdx.x == 32 && d.qprefetch) {
+      // this item's queries (needed from the first round) and the next item's
+      if (it == blockIdx.x) prefetch_l2_range(queries + p0, (p1 - p0 + 1) * sizeof(K));
+      const uint64_t n0 = (it + gridDim.x) * W;
+      if (n0 < m) prefetch_l2_range(queries + n0, ((n0 + W < m ? n0 + W : m) - n0) * sizeof(K));
     }
     __syncthreads();
     const uint64_t u0 = s_range[0], u1 = s_range[1];

@@ -13,6 +13,22 @@ namespace hbt {
 
 constexpr uint32_t kPrefixBits = 10;
 
+// One thread asks the TMA unit to pull a contiguous byte range into the L2
+// (cp.async.bulk.prefetch.L2, sm_90+).  Opt-in ("qprefetch"): the item kernels can
+// prefetch the queries of their current and next work item (ncu source page of the c3
+// item search: 15 % of all stall samples on the first compare with a round's query),
+// but it measured slower (c3 item search 1.55 -> 1.58 ms, c4 11.39 -> 11.62 ms).
+// Only whole 16 B units inside the range are requested, in pieces of <= 64 KB.
+__device__ __forceinline__ void prefetch_l2_range(const void* p, uint64_t bytes) {
+  const uint64_t a = reinterpret_cast<uint64_t>(p);
+  const uint64_t a0 = (a + 15) & ~uint64_t(15);
+  const uint64_t a1 = (a + bytes) & ~uint64_t(15);
+  for (uint64_t x = a0; x < a1; x += 65536) {
+    const uint32_t n = uint32_t(a1 - x < 65536 ? a1 - x : 65536);
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(x), "r"(n) : "memory");
+  }
+}
+
 template <typename K>
 __device__ __forceinline__ uint32_t lb_range(const K* s, uint32_t lo, uint32_t hi, K q) {
   uint32_t len = hi - lo;

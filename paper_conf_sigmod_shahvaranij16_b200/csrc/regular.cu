@@ -651,6 +651,11 @@ regular_search_items_kernel(const RView rv, const ItemDir d, const K* __restrict
         if (s_bstart[mid] <= p) lo = mid; else hi = mid;
       }
       s_range[threadIdx.x] = threadIdx.x ? ((uint64_t(lo) + 1) * d.U) / d.B - 1 : (uint64_t(lo) * d.U) / d.B;
+    } else if (threadIdx.x == 32 && d.qprefetch) {
+      // this item's queries (needed from the first round) and the next item's
+      if (it == blockIdx.x) prefetch_l2_range(queries + p0, (p1 - p0 + 1) * sizeof(K));
+      const uint64_t n0 = (it + gridDim.x) * W;
+      if (n0 < m) prefetch_l2_range(queries + n0, ((n0 + W < m ? n0 + W : m) - n0) * sizeof(K));
     }
     __syncthreads();
     const uint64_t c0 = s_range[0], c1 = s_range[1];

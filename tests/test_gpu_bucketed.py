@@ -73,8 +73,10 @@ def test_bucketed_scaled_workload(hbt, layout, F, items, cap, leaf256):
     t.set_param("leaf256", leaf256)
     for slice_bytes in (1 << 16, 1 << 20, 1 << 22):
         t.set_param("bucket_slice", slice_bytes)
-        pf, val = gpu_search(t, q, 8)
-        assert np.array_equal(pf, epf) and np.array_equal(val, ev), (layout, slice_bytes)
+        for qpf in (0, 1):  # with / without the bulk L2 prefetch of each item's queries
+            t.set_param("qprefetch", qpf)
+            pf, val = gpu_search(t, q, 8)
+            assert np.array_equal(pf, epf) and np.array_equal(val, ev), (layout, slice_bytes, qpf)
     t.set_param("bucket", 0)
     pf, val = gpu_search(t, q, 8)
     assert np.array_equal(pf, epf) and np.array_equal(val, ev)
