@@ -579,7 +579,9 @@ def run_hbt(args):
         # zero-copy: the leaf line crosses the host link once per query; streamed (the
         # library's auto rule, 160 B x m > L-segment): the whole L-segment once per step
         h2d = measure_h2d_gbs()
-        streamed = m * 160 > info["leaf_bytes"] and info["leaf_bytes"] > (8 << 20)
+        ls = dict(kv.split("=", 1) for kv in args.param).get("leaf_stream", "2")
+        streamed = c["layout"] == "implicit" and (ls == "1" or (ls == "2" and m * 160 > info["leaf_bytes"]
+                                                                and info["leaf_bytes"] > (8 << 20)))
         link_b = info["leaf_bytes"] if streamed else 64 * m
         link_ach = link_b / t_kernel / 1e9
         roof["link"] = {"bound": "host link (%s)" % ("L-segment slices streamed into HBM per bucket"

@@ -151,8 +151,11 @@ HBT_API int hbt_search_host(const hbt_tree* t, const void* host_queries, uint64_
  * and bucketing kernels then read each query's leaf line with zero-copy loads over
  * the host link (PCIe / NVLink-C2C), so a tree's leaves may exceed HBM while its
  * inner levels stay in HBM.  Results are identical in both placements.
- * IMPLICIT trees only (HBT_EUNSUPPORTED for regular or multi-shard trees); a rebuild
- * by hbt_bulk_update keeps the placement.  Synchronises the device (no search may be
+ * IMPLICIT: the leaf lines; a batch that touches most of them may instead be served
+ * by streaming bucket slices into HBM ("leaf_stream"); a rebuild by hbt_bulk_update
+ * keeps the placement.  REGULAR: the big-leaf pool (zero-copy only); the update
+ * kernels write leaves over the link and pool growth stays in host memory.
+ * HBT_EUNSUPPORTED for multi-shard trees.  Synchronises the device (no search may be
  * in flight); HBT_ENOMEM when the pinned allocation fails (the tree is unchanged). */
 HBT_API int hbt_set_leaf_placement(hbt_tree* t, uint32_t where);
 HBT_API int hbt_get_leaf_placement(const hbt_tree* t, uint32_t* where);

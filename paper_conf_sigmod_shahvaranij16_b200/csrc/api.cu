@@ -85,10 +85,53 @@ void leaf_free(hbt_tree* t) {
   t->d_leaf = nullptr;
 }
 
-// Move the implicit L-segment between HBM and pinned, mapped host memory.  The
-// search kernels read leaf lines through d_leaf either way (zero-copy loads over the
-// host link when it lives on the host), so results are identical.
+// Move one pool between HBM and pinned, mapped host memory: *d is the device-visible
+// pointer (the host allocation's device alias when on the host), *h the host
+// allocation or NULL.
+static int move_pool(void** d, void** h, uint64_t bytes, uint32_t where) {
+  if (where == 1) {
+    void* hh = nullptr;
+    void* dd = nullptr;
+    if (cudaHostAlloc(&hh, bytes ? bytes : 64, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) {
+      cudaGetLastError();
+      set_error("cudaHostAlloc of %llu bytes for the L-segment failed", (unsigned long long)bytes);
+      return HBT_ENOMEM;
+    }
+    if (bytes) {
+      cudaError_t e = cudaMemcpy(hh, *d, bytes, cudaMemcpyDefault);
+      if (e != cudaSuccess) { cudaFreeHost(hh); set_error("L-segment copy: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
+    }
+    cudaError_t e = cudaHostGetDevicePointer(&dd, hh, 0);
+    if (e != cudaSuccess) { cudaFreeHost(hh); set_error("no device alias of the host L-segment: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
+    cudaFree(*d);
+    *h = hh;
+    *d = dd;
+  } else {
+    void* dd = nullptr;
+    HBT_CUDA_TRY(cudaMalloc(&dd, bytes ? bytes : 64));
+    if (bytes) {
+      cudaError_t e = cudaMemcpy(dd, *h, bytes, cudaMemcpyDefault);
+      if (e != cudaSuccess) { cudaFree(dd); set_error("L-segment copy: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
+    }
+    cudaFreeHost(*h);
+    *h = nullptr;
+    *d = dd;
+  }
+  return HBT_OK;
+}
+
+// Move the L-segment (implicit: the leaf lines; regular: the big-leaf pool) between
+// HBM and pinned, mapped host memory.  The kernels read (and the regular update
+// kernels write) leaf lines through the device-visible pointer either way — zero-copy
+// accesses over the host link when it lives on the host — so results are identical.
 int leaf_place(hbt_tree* t, uint32_t where) {
+  if (t->form == HBT_REGULAR) {
+    RegularState& r = t->r;
+    if ((where == 1) == (r.h_leaf != nullptr)) { t->leaf_where = where; return HBT_OK; }
+    const int rc = move_pool(&r.d_leaf, &r.h_leaf, r.cap * uint64_t(t->F) * 64, where);
+    if (rc == HBT_OK) t->leaf_where = where;
+    return rc;
+  }
   const bool on_host = t->h_leaf != nullptr;
   if ((where == 1) == on_host) { t->leaf_where = where; return HBT_OK; }
   const uint64_t bytes = t->leaf_bytes ? t->leaf_bytes : 64;
@@ -355,7 +398,6 @@ int hbt_set_leaf_placement(hbt_tree* t, uint32_t where) {
   g_err.clear();
   if (!t) { set_error("tree is NULL"); return HBT_EINVAL; }
   if (where > 1) { set_error("placement must be 0 (HBM) or 1 (host)"); return HBT_EINVAL; }
-  if (t->form != HBT_IMPLICIT) { set_error("leaf placement: implicit trees only"); return HBT_EUNSUPPORTED; }
   if (t->shard.G > 1) { set_error("leaf placement: not for sharded trees"); return HBT_EUNSUPPORTED; }
   HBT_CUDA_TRY(cudaDeviceSynchronize());  // no search may be reading the old copy
   return leaf_place(t, where);
@@ -363,7 +405,7 @@ int hbt_set_leaf_placement(hbt_tree* t, uint32_t where) {
 
 int hbt_get_leaf_placement(const hbt_tree* t, uint32_t* where) {
   if (!t || !where) { set_error("NULL argument"); return HBT_EINVAL; }
-  *where = t->h_leaf ? 1u : 0u;
+  *where = (t->form == HBT_REGULAR ? t->r.h_leaf : t->h_leaf) ? 1u : 0u;
   return HBT_OK;
 }
 

@@ -124,7 +124,8 @@ struct BucketState {
 struct RegularState {
   uint32_t kpl = 0, NI = 0, B = 0, b = 0;
   uint64_t pool = 0, cap = 0;            // big leaves allocated / capacity
-  void* d_leaf = nullptr;                // cap x F lines x 64 B
+  void* d_leaf = nullptr;                // cap x F lines x 64 B (device alias of h_leaf when on the host)
+  void* h_leaf = nullptr;                // pinned mapped host pool (hbt_set_leaf_placement), else NULL
   uint32_t* d_count = nullptr;           // cap
   void* d_lkeys = nullptr;               // cap x F keys (last-level inner node)
   void* d_lidx = nullptr;                // cap x NIP index entries (padded to 32 B)

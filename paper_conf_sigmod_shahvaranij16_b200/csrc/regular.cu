@@ -1008,19 +1008,30 @@ int grow_pool(hbt_tree* t, uint64_t need, cudaStream_t s) {
   const uint64_t F = t->F, S = sizeof(K);
   void *leaf = nullptr, *lkeys = nullptr, *lidx = nullptr;
   uint32_t *count = nullptr, *chain = nullptr;
-  HBT_CUDA_TRY(cudaMalloc(&leaf, cap * F * 64));
+  void* hleaf = nullptr;
+  if (r.h_leaf) {  // L-segment placed in host memory: the grown pool stays there
+    if (cudaHostAlloc(&hleaf, cap * F * 64, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) {
+      cudaGetLastError();
+      set_error("cudaHostAlloc of the grown big-leaf pool failed");
+      return HBT_ENOMEM;
+    }
+    HBT_CUDA_TRY(cudaHostGetDevicePointer(&leaf, hleaf, 0));
+  } else {
+    HBT_CUDA_TRY(cudaMalloc(&leaf, cap * F * 64));
+  }
   HBT_CUDA_TRY(cudaMalloc(&count, cap * 4));
   HBT_CUDA_TRY(cudaMalloc(&lkeys, cap * F * S));
   HBT_CUDA_TRY(cudaMalloc(&lidx, cap * 32));
   HBT_CUDA_TRY(cudaMalloc(&chain, cap * 4));
-  HBT_CUDA_TRY(cudaMemcpyAsync(leaf, r.d_leaf, r.pool * F * 64, cudaMemcpyDeviceToDevice, s));
+  HBT_CUDA_TRY(cudaMemcpyAsync(leaf, r.d_leaf, r.pool * F * 64, cudaMemcpyDefault, s));
   HBT_CUDA_TRY(cudaMemcpyAsync(count, r.d_count, r.pool * 4, cudaMemcpyDeviceToDevice, s));
   HBT_CUDA_TRY(cudaMemcpyAsync(lkeys, r.d_lkeys, r.pool * F * S, cudaMemcpyDeviceToDevice, s));
   HBT_CUDA_TRY(cudaMemcpyAsync(lidx, r.d_lidx, r.pool * 32, cudaMemcpyDeviceToDevice, s));
   HBT_CUDA_TRY(cudaMemcpyAsync(chain, r.d_chain, r.nchain * 4, cudaMemcpyDeviceToDevice, s));
   HBT_CUDA_TRY(cudaStreamSynchronize(s));
-  cudaFree(r.d_leaf); cudaFree(r.d_count); cudaFree(r.d_lkeys); cudaFree(r.d_lidx); cudaFree(r.d_chain);
-  r.d_leaf = leaf; r.d_count = count; r.d_lkeys = lkeys; r.d_lidx = lidx; r.d_chain = chain;
+  if (r.h_leaf) cudaFreeHost(r.h_leaf); else cudaFree(r.d_leaf);
+  cudaFree(r.d_count); cudaFree(r.d_lkeys); cudaFree(r.d_lidx); cudaFree(r.d_chain);
+  r.d_leaf = leaf; r.h_leaf = hleaf; r.d_count = count; r.d_lkeys = lkeys; r.d_lidx = lidx; r.d_chain = chain;
   r.cap = cap;
   return HBT_OK;
 }
@@ -1674,7 +1685,8 @@ int regular_update(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
 
 void regular_free(hbt_tree* t) {
   RegularState& r = t->r;
-  cudaFree(r.d_leaf); cudaFree(r.d_count); cudaFree(r.d_lkeys); cudaFree(r.d_lidx); cudaFree(r.d_chain);
+  if (r.h_leaf) cudaFreeHost(r.h_leaf); else cudaFree(r.d_leaf);
+  cudaFree(r.d_count); cudaFree(r.d_lkeys); cudaFree(r.d_lidx); cudaFree(r.d_chain);
   cudaFree(r.d_ukeys); cudaFree(r.d_uidx); cudaFree(r.d_urefs); cudaFree(r.d_seg_of_leaf); cudaFree(r.d_dir);
   cudaFree(r.d_chainpos);
   r = RegularState{};

@@ -99,12 +99,47 @@ def test_host_leaves_update_and_range(hbt, width):
     t.close()
 
 
-def test_host_leaves_rejected_for_regular(hbt):
-    k = np.arange(1, 1001, dtype=np.uint64) * 3
-    t = gpu_build(hbt, k, k, 8, 8, layout="regular")
-    with pytest.raises(hbt.HBTError) as e:
-        t.set_leaf_placement("host")
-    assert e.value.code == hbt.EUNSUPPORTED
+@pytest.mark.parametrize("width,F", [(8, 32), (4, 8)])
+def test_host_leaves_regular(hbt, width, F):
+    """Regular tree with its big-leaf pool in host memory: searches (both kernels and
+    the bucketed item search), updates that split leaves and grow the pool (which
+    stays in host memory), range scans, and the way back to HBM."""
+    rng = np.random.default_rng(11 * F + width)
+    k, v = gen_keys(30000, width, rng, dup=True)
+    o = oracle.RTree.from_pairs(k, v, F, width)
+    t = gpu_build(hbt, k, v, F, width, layout="regular")
+    t.set_leaf_placement("host")
+    assert t.leaf_placement == "host"
+    mx = (1 << (8 * width)) - 1
+    for rep in range(3):
+        q = query_set(k, width, rng, 20000)
+        epf, ev = o.search(q)
+        for mode, bucket in ((2, 0), (0, 0), (2, 1)):
+            t.set_search_config(smem_mode=mode)
+            t.set_param("bucket", bucket)
+            pf, val = gpu_search(t, q, width)
+            assert np.array_equal(pf, epf) and np.array_equal(val, ev), (rep, mode, bucket)
+        t.set_param("bucket", 2)
+        nops = 20000  # mostly inserts of fresh keys: big leaves split, the pool grows
+        ok = rng.integers(0, mx, nops, dtype=np.uint64, endpoint=True)
+        ok[:3000] = k[rng.integers(0, len(k), 3000)]
+        ov = rng.integers(0, mx, nops, dtype=np.uint64, endpoint=True)
+        op = (rng.random(nops) < 0.1).astype(np.uint8)
+        o.update(ok, ov, op)  # the oracle's regular tree updates in place
+        t.update(to_dev(ok, width), to_dev(ov, width), torch.from_numpy(op).cuda())
+        assert t.leaf_placement == "host"
+        k = np.concatenate([k, ok])
+    q = query_set(k, width, rng, 20000)
+    epf, ev = o.search(q)
+    pf, val = gpu_search(t, q, width)
+    assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+    Kd, _ = oracle.dedupe(k, np.zeros(len(k), np.uint64))
+    lo, hi = ranges(Kd, width, rng, 300)
+    for kk in (1, 20):
+        range_check(t, o, lo, hi, kk, width)
+    t.set_leaf_placement("device")
+    pf, val = gpu_search(t, q, width)
+    assert np.array_equal(pf, epf) and np.array_equal(val, ev)
     t.close()
 
 
