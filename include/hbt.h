@@ -28,7 +28,9 @@
  * hbt_bulk_update is a caller-owned DEVICE pointer (cudaMalloc / torch CUDA
  * tensor on the current device).  hbt_search_host is the one entry point taking
  * HOST pointers (pinned recommended).  A tree owns its device memory until
- * hbt_destroy.
+ * hbt_destroy.  Device pointers are validated with cudaPointerGetAttributes
+ * (pageable host pointers -> HBT_EINVAL); the last 8 pointers that validated are
+ * remembered per thread, so small batches do not pay the check on every call.
  *
  * Streams: `stream` is a cudaStream_t passed as void* (NULL = legacy default
  * stream).  hbt_bulk_build and hbt_bulk_update are host-synchronous on return;
