@@ -445,10 +445,10 @@ def time_e2e(work, steps, world):
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
     qps = world * m * steps / float(te.item())
     api = ("H2D + hbt_search_sharded + D2H (pinned host buffers)" if sharded else
-           "hbt_search_host (pinned host buffers, 4 Mi-query buckets double-buffered over 2 streams)")
+           "hbt_search_host (pinned host buffers, 1 Mi-query buckets double-buffered over 2 streams)")
     return {"value": round(qps / 1e6, 2), "unit": "M queries/s", "h2d_bytes_per_step": m * w,
             "d2h_bytes_per_step": m * (8 + w), "api": api,
-            "gpu_launches_per_step": (4 if sharded else -(-m // (1 << 22)))}
+            "gpu_launches_per_step": (4 if sharded else -(-m // (1 << 20)))}
 
 
 def run_hbt(args):
@@ -598,7 +598,7 @@ def run_hbt(args):
         roof["note"] = ("latency-bound batch: %d queries are one wave of the GPU, so the step is the launch "
                         "plus one query's chain of dependent memory round trips; no byte roofline binds" % m)
 
-    if phases and e2e:  # each 4 Mi-query chunk of hbt_search_host runs the bucketed pipeline
+    if phases and e2e and args.bucket == 1:  # forced bucketing: every 1 Mi-query chunk runs the pipeline
         e2e["gpu_launches_per_step"] *= phases["launches"]
 
     cpu = None

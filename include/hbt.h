@@ -233,6 +233,9 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *   "qprefetch"   bucketed item searches: 1 = one thread per CTA prefetches the current and
  *                 next work item's queries into the L2 (cp.async.bulk.prefetch); 0 = off
  *                 (default: measured slower on c3, 1.55 -> 1.58 ms)
+ *   "host_chunk_log2" hbt_search_host: queries per pipeline bucket, log2 in [12, 26]
+ *                 (default 20)
+ *   "host_bufs"   hbt_search_host: (stream, buffer) pairs in flight, 2..4 (default 2)
  *   "full_levels" implicit: bit d set = level d's nodes are read whole in one round trip
  *                 (0 = default: by the "l2_levels_bytes" budget)
  * Unknown names or out-of-range values return HBT_EINVAL. */

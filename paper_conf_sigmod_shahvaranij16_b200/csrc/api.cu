@@ -182,7 +182,7 @@ static void free_tree(hbt_tree* t) {
   cudaFree(t->pipe.d_q);
   cudaFree(t->pipe.d_pf);
   cudaFree(t->pipe.d_v);
-  for (int i = 0; i < 2; ++i) {
+  for (int i = 0; i < kHostBufs; ++i) {
     if (t->pipe.s[i]) cudaStreamDestroy(t->pipe.s[i]);
     if (t->pipe.ev[i]) cudaEventDestroy(t->pipe.ev[i]);
   }
@@ -263,29 +263,39 @@ int hbt_search_host(const hbt_tree* t, const void* host_queries, uint64_t m, uin
   HostPipe& p = t->pipe;
   std::lock_guard<std::mutex> lock(p.mu);
   const uint64_t S = t->width;
-  const uint64_t chunk = uint64_t(1) << 22;  // 4 Mi queries per bucket
-  if (!p.chunk) {
-    HBT_CUDA_TRY(cudaMalloc(&p.d_q, 2 * chunk * S));
-    HBT_CUDA_TRY(cudaMalloc(&p.d_pf, 2 * chunk * sizeof(uint64_t)));
-    HBT_CUDA_TRY(cudaMalloc(&p.d_v, 2 * chunk * S));
-    for (int i = 0; i < 2; ++i) {
+  const uint64_t chunk = uint64_t(1) << t->cfg.host_chunk_log2;  // queries per bucket (default 4 Mi)
+  const int nbuf = int(t->cfg.host_bufs);
+  if (p.chunk != chunk || p.nbuf != nbuf) {
+    for (int i = 0; i < p.nbuf && p.chunk; ++i) HBT_CUDA_TRY(cudaStreamSynchronize(p.s[i]));
+    cudaFree(p.d_q);
+    cudaFree(p.d_pf);
+    cudaFree(p.d_v);
+    p.d_q = p.d_v = nullptr;
+    p.d_pf = nullptr;
+    p.chunk = 0;
+    HBT_CUDA_TRY(cudaMalloc(&p.d_q, nbuf * chunk * S));
+    HBT_CUDA_TRY(cudaMalloc(&p.d_pf, nbuf * chunk * sizeof(uint64_t)));
+    HBT_CUDA_TRY(cudaMalloc(&p.d_v, nbuf * chunk * S));
+    for (int i = 0; i < kHostBufs; ++i) {
+      if (p.s[i]) continue;
       HBT_CUDA_TRY(cudaStreamCreateWithFlags(&p.s[i], cudaStreamNonBlocking));
       HBT_CUDA_TRY(cudaEventCreateWithFlags(&p.ev[i], cudaEventDisableTiming));
     }
     p.chunk = chunk;
+    p.nbuf = nbuf;
   }
   // Order after the caller's stream.
   cudaStream_t cs = (cudaStream_t)stream;
   HBT_CUDA_TRY(cudaEventRecord(p.ev[0], cs));
-  for (int i = 0; i < 2; ++i) HBT_CUDA_TRY(cudaStreamWaitEvent(p.s[i], p.ev[0], 0));
-  // Buckets alternate between two (stream, buffer) pairs: bucket c+1's H2D copy
-  // overlaps bucket c's search and bucket c-1's D2H copy.
+  for (int i = 0; i < nbuf; ++i) HBT_CUDA_TRY(cudaStreamWaitEvent(p.s[i], p.ev[0], 0));
+  // Buckets rotate over nbuf (stream, buffer) pairs: bucket c+1's H2D copy overlaps
+  // bucket c's search and bucket c-1's D2H copy.
   const char* hq = (const char*)host_queries;
   char* hv = (char*)host_values;
   uint64_t c = 0;
   for (uint64_t off = 0; off < m; off += chunk, ++c) {
     const uint64_t len = (m - off < chunk) ? (m - off) : chunk;
-    const int b = int(c & 1);
+    const int b = int(c % uint64_t(nbuf));
     cudaStream_t s = p.s[b];
     char* dq = (char*)p.d_q + b * chunk * S;
     uint64_t* dpf = p.d_pf + b * chunk;
@@ -296,7 +306,7 @@ int hbt_search_host(const hbt_tree* t, const void* host_queries, uint64_t m, uin
     HBT_CUDA_TRY(cudaMemcpyAsync(host_pos_found + off, dpf, len * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
     HBT_CUDA_TRY(cudaMemcpyAsync(hv + off * S, dv, len * S, cudaMemcpyDeviceToHost, s));
   }
-  for (int i = 0; i < 2; ++i) HBT_CUDA_TRY(cudaStreamSynchronize(p.s[i]));
+  for (int i = 0; i < nbuf; ++i) HBT_CUDA_TRY(cudaStreamSynchronize(p.s[i]));
   return HBT_OK;
 }
 
@@ -442,6 +452,8 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "bucket_cap" && value >= 0 && value < (1 << 20)) { c.bucket_cap = uint32_t(value); t->bk.valid = false; }
   else if (n == "leaf_stream" && value >= 0 && value <= 2) c.leaf_stream = uint32_t(value);
   else if (n == "qprefetch" && (value == 0 || value == 1)) c.qprefetch = uint32_t(value);
+  else if (n == "host_chunk_log2" && value >= 12 && value <= 26) c.host_chunk_log2 = uint32_t(value);
+  else if (n == "host_bufs" && value >= 2 && value <= kHostBufs) c.host_bufs = uint32_t(value);
   else if (n == "stream_slice" && value >= 0) { c.stream_slice = uint64_t(value); t->bks.valid = false; }
   else if (n == "phase_timing" && (value == 0 || value == 1)) c.phase_timing = uint32_t(value);
   else if (n == "leaf256" && (value == 0 || value == 1)) c.leaf256 = uint32_t(value);

@@ -66,6 +66,8 @@ struct SearchConfig {
   uint32_t leaf_stream = 2;      // host L-segment: 0 = zero-copy leaf reads, 1 = stream bucket slices
                                  // into HBM (bucketed, double-buffered copies), 2 = auto (by batch size)
   uint64_t stream_slice = 0;     // host L-segment bytes per streamed bucket (0 = 8 MB)
+  uint32_t host_chunk_log2 = 20;  // hbt_search_host: queries per pipeline bucket (log2; c2 e2e 2.78 -> 3.00 G q/s vs 2^22)
+  uint32_t host_bufs = 2;        // hbt_search_host: (stream, buffer) pairs in flight (2..4)
   uint32_t qprefetch = 0;        // item searches: bulk L2 prefetch of each work item's queries (measured slower: c3 item search 1.55 -> 1.58 ms)
   uint32_t leaf256 = 1;          // leaf line by two 256-bit lane loads (one 64 B request per group)
   uint32_t sec256 = 0;           // implicit L2 levels: index / key sector by one lane's 256-bit load
@@ -150,14 +152,16 @@ struct RegularState {
   uint64_t chainpos_cap = 0;
 };
 
+constexpr int kHostBufs = 4;  // most (stream, buffer) pairs of the host pipeline
 struct HostPipe {
   std::mutex mu;
-  void* d_q = nullptr;                   // 2 x chunk queries
-  uint64_t* d_pf = nullptr;              // 2 x chunk
-  void* d_v = nullptr;                   // 2 x chunk
+  void* d_q = nullptr;                   // nbuf x chunk queries
+  uint64_t* d_pf = nullptr;              // nbuf x chunk
+  void* d_v = nullptr;                   // nbuf x chunk
   uint64_t chunk = 0;
-  cudaStream_t s[2] = {nullptr, nullptr};
-  cudaEvent_t ev[2] = {nullptr, nullptr};
+  int nbuf = 0;
+  cudaStream_t s[kHostBufs] = {};
+  cudaEvent_t ev[kHostBufs] = {};
 };
 
 // Key-range shard metadata (sharded.cu): shard g holds global ranks

@@ -118,8 +118,10 @@ def test_bucketed_after_update(hbt, layout, items, cap, leaf256):
     t.close()
 
 
-def test_bucketed_host_pipeline(hbt):
-    """hbt_search_host runs the bucketed path per 4 Mi-query chunk."""
+@pytest.mark.parametrize("chunk_log2,bufs", [(22, 2), (20, 2), (20, 3), (14, 4)])
+def test_bucketed_host_pipeline(hbt, chunk_log2, bufs):
+    """hbt_search_host runs the bucketed path per pipeline chunk, for several chunk
+    sizes and numbers of (stream, buffer) pairs, with a ragged last chunk."""
     n, m = 1 << 16, (1 << 22) + 12345
     k, v = gen.workload_keys_values("c2", n)
     q = gen.workload_queries("c2", k, m)
@@ -127,6 +129,8 @@ def test_bucketed_host_pipeline(hbt):
     t = gpu_build(hbt, k, v, 16, 8)
     t.set_param("bucket", 1)
     t.set_param("bucket_slice", 1 << 14)
+    t.set_param("host_chunk_log2", chunk_log2)
+    t.set_param("host_bufs", bufs)
     pf = np.empty(m, np.uint64)
     val = np.empty(m, np.uint64)
     t.search_host(q.copy(), pf, val)
