@@ -96,6 +96,7 @@ struct ItemDir {
   uint32_t cap = 0;    // shared-memory entries (larger ranges search M in global memory)
   uint64_t pos_base = 0;  // implicit: added to every reported position (key-range shards)
   uint32_t qprefetch = 0; // bulk L2 prefetch of the current / next item's queries
+  uint32_t rounds = 16;   // warp rounds per work item (fewer for small batches: every SM gets items)
 };
 
 // Query-bucketing state (bucketed.cu): B splitter keys and a prefix directory,

@@ -523,7 +523,7 @@ implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* _
                              uint64_t n) {
   using C = Cfg<K, F>;
   constexpr int QPG = 32 / C::NG;
-  constexpr uint64_t W = uint64_t(THREADS) * kItemRounds;
+  const uint64_t W = uint64_t(THREADS) * d.rounds;
   extern __shared__ __align__(16) uint8_t smem[];
   uint64_t* s_bstart = reinterpret_cast<uint64_t*>(smem);
   K* s_M = reinterpret_cast<K*>(s_bstart + d.B + 1);
@@ -570,13 +570,13 @@ implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* _
       nextq = i <= p1 ? ldcs(queries + i) : key_max<K>();
     }
 #pragma unroll 1
-    for (int r = 0; r < kItemRounds; ++r) {
+    for (int r = 0; r < int(d.rounds); ++r) {
       const uint64_t base = p0 + (uint64_t(r) * (THREADS / 32) + wid) * 32;
       if (base > p1) break;
       const K myq = nextq;
       {
         const uint64_t i = base + (THREADS / 32) * 32 + lane;
-        nextq = (r + 1 < kItemRounds && i <= p1) ? ldcs(queries + i) : key_max<K>();
+        nextq = (r + 1 < int(d.rounds) && i <= p1) ? ldcs(queries + i) : key_max<K>();
       }
       const uint32_t lo = in_smem ? prefix_lower_bound(s_M, cnt, s_T, pt, myq) : lb_range(M, 0, cnt, myq);
       const uint32_t mynode = uint32_t(u0) + (lo < cnt ? lo : cnt - 1);
@@ -731,11 +731,13 @@ struct Launch {
       HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
       attr_set = true;
     }
+    ItemDir dd = d;
+    dd.rounds = item_rounds(m, t->num_sms, TH);
     uint64_t grid = t->num_sms;
-    const uint64_t items = (m + uint64_t(TH) * kItemRounds - 1) / (uint64_t(TH) * kItemRounds);
+    const uint64_t items = (m + uint64_t(TH) * dd.rounds - 1) / (uint64_t(TH) * dd.rounds);
     if (items < grid) grid = items ? items : 1;
     kern<<<unsigned(grid), TH, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
-                                          (const uint8_t*)t->d_leaf, d, (const K*)q, m, pf, (K*)v, lt, t->n);
+                                          (const uint8_t*)t->d_leaf, dd, (const K*)q, m, pf, (K*)v, lt, t->n);
     HBT_CUDA_TRY(cudaGetLastError());
     return HBT_OK;
   }

@@ -626,7 +626,7 @@ regular_search_items_kernel(const RView rv, const ItemDir d, const K* __restrict
   constexpr uint32_t E16 = 16 / S;
   constexpr uint32_t LINE = uint32_t(F) * S < 64 ? uint32_t(F) * S : 64;
   constexpr int LCH = int(LINE / 16);
-  constexpr uint64_t W = uint64_t(THREADS) * kItemRounds;
+  const uint64_t W = uint64_t(THREADS) * d.rounds;
   extern __shared__ __align__(16) uint8_t smem[];
   uint64_t* s_bstart = reinterpret_cast<uint64_t*>(smem);
   K* s_M = reinterpret_cast<K*>(s_bstart + d.B + 1);
@@ -677,13 +677,13 @@ regular_search_items_kernel(const RView rv, const ItemDir d, const K* __restrict
       nextq = i <= p1 ? ldcs(queries + i) : key_max<K>();
     }
 #pragma unroll 1
-    for (int r = 0; r < kItemRounds; ++r) {
+    for (int r = 0; r < int(d.rounds); ++r) {
       const uint64_t base = p0 + (uint64_t(r) * (THREADS / 32) + wid) * 32;
       if (base > p1) break;
       const K myq = nextq;
       {
         const uint64_t i = base + (THREADS / 32) * 32 + lane;
-        nextq = (r + 1 < kItemRounds && i <= p1) ? ldcs(queries + i) : key_max<K>();
+        nextq = (r + 1 < int(d.rounds) && i <= p1) ? ldcs(queries + i) : key_max<K>();
       }
       const uint32_t lo = in_smem ? prefix_lower_bound(s_M, cnt, s_T, pt, myq) : lb_range(M, 0, cnt, myq);
       const uint32_t e = lo < cnt ? lo : cnt - 1;
@@ -950,10 +950,12 @@ int search_items_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* 
     HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
     attr = true;
   }
+  ItemDir dd = d;
+  dd.rounds = item_rounds(m, t->num_sms, TH);
   uint64_t grid = t->num_sms;
-  const uint64_t items = (m + uint64_t(TH) * kItemRounds - 1) / (uint64_t(TH) * kItemRounds);
+  const uint64_t items = (m + uint64_t(TH) * dd.rounds - 1) / (uint64_t(TH) * dd.rounds);
   if (items < grid) grid = items ? items : 1;
-  kern<<<unsigned(grid), TH, smem, s>>>(rv, d, (const K*)q, m, pf, (K*)v);
+  kern<<<unsigned(grid), TH, smem, s>>>(rv, dd, (const K*)q, m, pf, (K*)v);
   HBT_CUDA_TRY(cudaGetLastError());
   return HBT_OK;
 }
