@@ -554,6 +554,9 @@ def run_hbt(args):
                 "traffic_gbs": round(traffic_bytes / t_kernel / 1e9, 1) if traffic_bytes else None,
                 "traffic_frac": round(traffic_bytes / t_kernel / 1e9 / peak, 4) if traffic_bytes else None,
                 "bytes_per_query_model": round(mdl["hbm_bytes_per_query"], 2), "peak_source": peak_src,
+                # SURVEY 8(d) reporting: measured B/q from ncu and the fraction of the 8 TB/s spec HBM roof
+                "traffic_bytes_per_query": round(traffic_bytes / m, 2) if traffic_bytes else None,
+                "frac_of_8tbs_spec": round(hbm_ach / 8000.0, 4),
                 "model": model_desc}
     if args.config == "c4" and world > 1:
         a2a_b = (world - 1) / world * (w + 8 + w)
@@ -688,9 +691,30 @@ def cpu_baseline(cfg_name, target_s=8.0):
         if el > target_s or reps >= 50:
             break
     qps = reps * len(q) / el
+    # SURVEY 8(d) oracle timings beside it: one thread, and std::lower_bound over the
+    # sorted array with all threads (bounded samples)
+    q1 = q[: 1 << 18]
+    t0 = time.perf_counter()
+    tree.search(q1, nthreads=1)
+    qps1 = len(q1) / (time.perf_counter() - t0)
+    Kd, Vd = oracle.dedupe(k, v)
+    oracle.lower_bound(Kd, Vd, q[: 1 << 16], nthreads=cores)
+    t0 = time.perf_counter()
+    oracle.lower_bound(Kd, Vd, q, nthreads=cores)
+    qps_lb = len(q) / (time.perf_counter() - t0)
+    cpu_model = ""
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                cpu_model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
     return {"value": round(qps / 1e6, 3), "unit": "M queries/s", "cores": cores, "kind": "oracle",
             "sample": f"{reps} x {len(q)} queries of the same workload, oracle tree search "
-                      f"(scalar node scan, OpenMP static chunks), {el:.1f} s; oracle build {build_s:.1f} s"}
+                      f"(scalar node scan, OpenMP static chunks), {el:.1f} s; oracle build {build_s:.1f} s",
+            "one_thread": round(qps1 / 1e6, 3), "lower_bound_all_threads": round(qps_lb / 1e6, 3),
+            "build_s": round(build_s, 2), "cpu_model": cpu_model, "nproc": os.cpu_count()}
 
 
 def run_reference(args):
