@@ -464,6 +464,8 @@ def run_hbt(args):
     torch.cuda.synchronize()
     node_b = ((c["fanout"] * w + 31) // 32) * 32
     l2_probe = probe_l2_gbs(32 if node_b > 32 else node_b) if rank == 0 else None
+    # the probe at every access granularity of the tree (reported beside the roofline)
+    l2_probe_by_chunk = {str(b): round(probe_l2_gbs(b) or 0.0, 1) for b in (32, 64, 128)} if rank == 0 else None
 
     use_graph = args.graph == "1" or (args.graph == "auto" and m <= (1 << 20) and args.config != "c4"
                                       and not args.origin_rank0)
@@ -569,7 +571,8 @@ def run_hbt(args):
         roof_l2 = {"bound": "l2", "achieved": round(l2_ach, 1), "peak": round(l2_probe, 1), "unit": "GB/s",
                    "frac": round(l2_ach / l2_probe, 4), "bytes_per_query_model": round(mdl["l2_bytes_per_query"], 2),
                    "peak_source": "measured in this run: all-SM random 32 B reads of a 32 MB L2-resident buffer "
-                                  "(tools/probe.cu; SURVEY §8d BW_L2)"}
+                                  "(tools/probe.cu; SURVEY §8d BW_L2)",
+                   "probe_gbs_by_access_bytes": l2_probe_by_chunk}
     # roof time = max(B_HBM / BW_HBM, B_L2 / BW_L2); the binding term is the
     # kernel's roofline, its frac = roof time / measured kernel time.
     roof = dict(roof_l2 if roof_l2 and roof_l2["frac"] > roof_hbm["frac"] else roof_hbm)
