@@ -523,6 +523,7 @@ def run_hbt(args):
         except hbt.HBTError:
             phases = None
     l2_size = torch.cuda.get_device_properties(local).L2_cache_size
+    gran_extra = 0
     if phases:
         mdl = roofline.model_bucketed(info, m)
         t_kernel = phases["search"] * 1e-3
@@ -541,6 +542,7 @@ def run_hbt(args):
         extra_b = ((args.range_k - 1 + P - 1) // P) * 64 + args.range_k * 2 * w + 4
         mdl["hbm_bytes_per_query"] += extra_b
         mdl["l2_bytes_per_query"] += extra_b
+        gran_extra = extra_b
         kernel = "range_scan_kernel"
     peak, peak_src = measured_peaks()
     traffic = None
@@ -567,12 +569,23 @@ def run_hbt(args):
         roof_hbm["frac_with_nvlink"] = round((m / t_kernel) * t_roof, 4)
     roof_l2 = None
     if l2_probe:
+        # the model's L2 bytes by access granularity, each class at the probe of its own
+        # granularity: roof time = sum(bytes_c / BW_c); peak = bytes / roof time
+        gran = roofline.l2_granularity(info, work.hit_rate, bucketed=bool(phases),
+                                       level=info["height"] if phases else None)
+        gran[64] += gran_extra
+        probes = {32: l2_probe_by_chunk.get("32") or l2_probe, 64: l2_probe_by_chunk.get("64") or l2_probe}
+        t_q = sum(b / (probes[g] * 1e9) for g, b in gran.items())
+        l2_peak = mdl["l2_bytes_per_query"] / t_q / 1e9
         l2_ach = mdl["l2_bytes_per_query"] * m / t_kernel / 1e9
-        roof_l2 = {"bound": "l2", "achieved": round(l2_ach, 1), "peak": round(l2_probe, 1), "unit": "GB/s",
-                   "frac": round(l2_ach / l2_probe, 4), "bytes_per_query_model": round(mdl["l2_bytes_per_query"], 2),
-                   "peak_source": "measured in this run: all-SM random 32 B reads of a 32 MB L2-resident buffer "
-                                  "(tools/probe.cu; SURVEY §8d BW_L2)",
-                   "probe_gbs_by_access_bytes": l2_probe_by_chunk}
+        roof_l2 = {"bound": "l2", "achieved": round(l2_ach, 1), "peak": round(l2_peak, 1), "unit": "GB/s",
+                   "frac": round(l2_ach / l2_peak, 4), "bytes_per_query_model": round(mdl["l2_bytes_per_query"], 2),
+                   "bytes_per_query_by_access": {str(g): round(b, 2) for g, b in gran.items()},
+                   "peak_source": "measured in this run: all-SM random reads of a 32 MB L2-resident buffer at 32 B "
+                                  "and 64 B granularity (tools/probe.cu; SURVEY §8d BW_L2), weighted by the model's "
+                                  "bytes at each granularity",
+                   "probe_gbs_by_access_bytes": l2_probe_by_chunk,
+                   "frac_vs_32b_probe": round(l2_ach / l2_probe, 4)}
     # roof time = max(B_HBM / BW_HBM, B_L2 / BW_L2); the binding term is the
     # kernel's roofline, its frac = roof time / measured kernel time.
     roof = dict(roof_l2 if roof_l2 and roof_l2["frac"] > roof_hbm["frac"] else roof_hbm)

@@ -125,3 +125,32 @@ def model_bucketed(info, m, level=None):
         units = L0 if lv >= info["height"] else nodes[lv]
         dram += units * S / m
     return {"hbm_bytes_per_query": io + dram, "l2_bytes_per_query": io + l2, "io_bytes_per_query": io}
+
+
+def l2_granularity(info, hit_rate=1.0, bucketed=False, level=None):
+    """The L2 model bytes per query split by access granularity (bytes per request):
+    {32: random 32 B sectors, 64: random 64 B lines and the coalesced query / result
+    streams}.  bench.py divides each class by the in-run probe of that granularity, so
+    the L2 roof of a mixed pattern is sum(bytes_c / BW_c), not bytes / BW_32."""
+    S, F = info["width"], info["fanout"]
+    io = 2 * S + 8 if not bucketed else S + 16
+    out = {32: 0.0, 64: float(io)}
+    if info["layout"] == 1:  # regular
+        kpl = 64 // S
+        if bucketed:
+            out[64] += 64 + 64  # key line + leaf line (256-bit lane loads: one 64 B request each)
+            return out
+        levels = len(info["level_nodes"]) - (info["smem_levels"] or 0)
+        idx = 32 if F > kpl else 0
+        out[32] += max(0, levels) * (idx + 32) + idx
+        out[64] += max(0, levels) * min(64, F * S) + min(64, F * S) + 32 + 32 * hit_rate
+        return out
+    node = F * S
+    lv = info["smem_levels"] if level is None else level
+    for d in range(lv, info["height"]):
+        if node > 32:
+            out[32] += 64  # index sector + one key sector
+        else:
+            out[32] += _sect(node)
+    out[64] += 32 + 32 * hit_rate  # the leaf line as one request (key + value sectors)
+    return out
