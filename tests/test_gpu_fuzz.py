@@ -1,0 +1,78 @@
+"""Randomised GPU parity: many small trees, each with a random form, key width,
+fanout, size (duplicates, MAX as a real key, empty), query mix (hits, misses, 0,
+MAX, neighbours of keys) and a random combination of the search knobs (top-level
+mode, per-level read widths, CTA size, bucketing with its slice / item directory /
+capacity, L-segment placement and streaming), every output compared with the
+oracle.  Complements the targeted suites: a knob interaction no suite lists still
+has to give the oracle's bits.  Seeded, so a failure reproduces."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from gpu_util import gpu_build, gpu_search
+from test_oracle_implicit import gen_keys, kmax, query_set
+
+pytestmark = pytest.mark.gpu
+
+CASES = 600
+
+
+@pytest.fixture(scope="module")
+def hbt():
+    import paper_conf_sigmod_shahvaranij16_b200 as m
+    assert torch.cuda.is_available(), "gpu tests need a CUDA device"
+    return m
+
+
+def _queries(k, width, rng, m):
+    q = query_set(k, width, rng, m)
+    if len(k):
+        kk = k[rng.integers(0, len(k), min(m, 64))].astype(object)
+        mx = kmax(width)
+        nb = np.array([min(mx, int(x) + 1) for x in kk] + [max(0, int(x) - 1) for x in kk], dtype=np.uint64)
+        q = np.concatenate([q, nb, np.array([0, kmax(width)], dtype=np.uint64)])
+    return q
+
+
+@pytest.mark.parametrize("case", range(CASES))
+def test_random_knob_parity(hbt, case):
+    rng = np.random.default_rng(7000 + case)
+    layout = "regular" if rng.random() < 0.4 else "implicit"
+    width = int(rng.choice([4, 8]))
+    F = int(rng.choice([4, 8, 16, 32]))
+    n = int(rng.choice([0, 1, 2, 3, 7, 17, 64, 65, 500, 4097, 20000, 70000]))
+    k, v = gen_keys(n, width, rng, dup=bool(rng.random() < 0.5), with_max=bool(rng.random() < 0.3))
+    o = (oracle.ITree if layout == "implicit" else oracle.RTree).from_pairs(k, v, F, width)
+    t = gpu_build(hbt, k, v, F, width, layout=layout)
+    knobs = {}
+    if layout == "implicit":
+        knobs["smem_mode"] = int(rng.choice([0, 1, 2, 3, 4]))
+        knobs["l2_levels_bytes"] = int(rng.choice([0, 1, 4096]))
+        knobs["full256"] = int(rng.integers(0, 2))
+        knobs["sec256"] = int(rng.integers(0, 2))
+        knobs["small_batch"] = int(rng.choice([0, 1 << 16]))
+        if knobs["smem_mode"] == 2:
+            knobs["threads"] = int(rng.choice([0, 512, 768, 1024]))
+    else:
+        knobs["smem_mode"] = int(rng.choice([0, 2]))
+    knobs["leaf256"] = int(rng.integers(0, 2))
+    knobs["bucket"] = int(rng.choice([0, 1, 2]))
+    if knobs["bucket"]:
+        knobs["bucket_slice"] = int(rng.choice([1, 4096, 1 << 16, 1 << 20]))
+        knobs["bucket_items"] = int(rng.integers(0, 2))
+        knobs["bucket_cap"] = int(rng.choice([0, 0, 7]))
+    host = bool(rng.random() < 0.25)
+    if host:
+        t.set_leaf_placement("host")
+        if layout == "implicit":
+            knobs["leaf_stream"] = int(rng.choice([0, 1, 2]))
+            knobs["stream_slice"] = int(rng.choice([64, 4096, 0]))
+    for name, val in knobs.items():
+        t.set_param(name, val)
+    q = _queries(k, width, rng, int(rng.choice([1, 31, 1000, 40000])))
+    epf, ev = o.search(q)
+    pf, val = gpu_search(t, q, width)
+    assert np.array_equal(pf, epf), (layout, width, F, n, host, knobs, np.nonzero(pf != epf)[0][:5])
+    assert np.array_equal(val, ev), (layout, width, F, n, host, knobs)
+    t.close()
