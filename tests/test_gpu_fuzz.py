@@ -76,3 +76,46 @@ def test_random_knob_parity(hbt, case):
     assert np.array_equal(pf, epf), (layout, width, F, n, host, knobs, np.nonzero(pf != epf)[0][:5])
     assert np.array_equal(val, ev), (layout, width, F, n, host, knobs)
     t.close()
+
+
+@pytest.mark.parametrize("case", range(150))
+def test_random_update_sequences(hbt, case):
+    """Random UPSERT / DELETE batches (splits, removals, emptying the tree, MAX keys)
+    on both forms, searched after every batch with random knobs."""
+    import torch as _t
+    from gpu_util import to_dev
+    rng = np.random.default_rng(9100 + case)
+    layout = "regular" if rng.random() < 0.6 else "implicit"
+    width = int(rng.choice([4, 8]))
+    F = int(rng.choice([4, 8, 16, 32]))
+    n = int(rng.choice([0, 1, 9, 300, 5000, 30000]))
+    k, v = gen_keys(n, width, rng, dup=bool(rng.random() < 0.5), with_max=bool(rng.random() < 0.3))
+    o = (oracle.ITree if layout == "implicit" else oracle.RTree).from_pairs(k, v, F, width)
+    t = gpu_build(hbt, k, v, F, width, layout=layout)
+    if rng.random() < 0.2:
+        t.set_leaf_placement("host")
+    mx = kmax(width)
+    live = k.copy()
+    for b in range(3):
+        nops = int(rng.choice([1, 50, 2000, 12000]))
+        pool = live if len(live) else np.zeros(1, np.uint64)
+        ok = np.where(rng.random(nops) < 0.5, pool[rng.integers(0, len(pool), nops)],
+                      rng.integers(0, mx, nops, dtype=np.uint64, endpoint=True)).astype(np.uint64)
+        if rng.random() < 0.2:
+            ok[: nops // 3] = mx
+        ov = rng.integers(0, mx, nops, dtype=np.uint64, endpoint=True)
+        pdel = float(rng.choice([0.0, 0.3, 0.9, 1.0]))
+        op = (rng.random(nops) < pdel).astype(np.uint8)
+        r = o.update(ok, ov, op)
+        if layout == "implicit":
+            o = r
+        t.update(to_dev(ok, width), to_dev(ov, width), _t.from_numpy(op).cuda())
+        live = np.concatenate([live, ok])
+        t.set_param("bucket", int(rng.choice([0, 1, 2])))
+        t.set_param("bucket_slice", int(rng.choice([1, 4096, 1 << 20])))
+        q = _queries(live, width, rng, int(rng.choice([100, 5000])))
+        epf, ev = o.search(q)
+        pf, val = gpu_search(t, q, width)
+        assert np.array_equal(pf, epf), (layout, width, F, n, b, np.nonzero(pf != epf)[0][:5])
+        assert np.array_equal(val, ev), (layout, width, F, n, b)
+    t.close()
