@@ -236,6 +236,8 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *   "host_chunk_log2" hbt_search_host: queries per pipeline bucket, log2 in [12, 26]
  *                 (default 20)
  *   "host_bufs"   hbt_search_host: (stream, buffer) pairs in flight, 2..4 (default 2)
+ *   "item_rounds" bucketed item searches: most warp rounds per work item (0 = default 16;
+ *                 fewer are used when the batch would leave SMs idle)
  *   "full_levels" implicit: bit d set = level d's nodes are read whole in one round trip
  *                 (0 = default: by the "l2_levels_bytes" budget)
  * Unknown names or out-of-range values return HBT_EINVAL. */

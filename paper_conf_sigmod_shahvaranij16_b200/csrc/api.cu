@@ -452,6 +452,7 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "bucket_cap" && value >= 0 && value < (1 << 20)) { c.bucket_cap = uint32_t(value); t->bk.valid = false; }
   else if (n == "leaf_stream" && value >= 0 && value <= 2) c.leaf_stream = uint32_t(value);
   else if (n == "qprefetch" && (value == 0 || value == 1)) c.qprefetch = uint32_t(value);
+  else if (n == "item_rounds" && value >= 0 && value <= 64) c.item_rounds = uint32_t(value);
   else if (n == "host_chunk_log2" && value >= 12 && value <= 26) c.host_chunk_log2 = uint32_t(value);
   else if (n == "host_bufs" && value >= 2 && value <= kHostBufs) c.host_bufs = uint32_t(value);
   else if (n == "stream_slice" && value >= 0) { c.stream_slice = uint64_t(value); t->bks.valid = false; }

@@ -68,6 +68,7 @@ struct SearchConfig {
   uint64_t stream_slice = 0;     // host L-segment bytes per streamed bucket (0 = 8 MB)
   uint32_t host_chunk_log2 = 20;  // hbt_search_host: queries per pipeline bucket (log2; c2 e2e 2.78 -> 3.00 G q/s vs 2^22)
   uint32_t host_bufs = 2;        // hbt_search_host: (stream, buffer) pairs in flight (2..4)
+  uint32_t item_rounds = 0;      // item searches: most warp rounds per work item (0 = 16)
   uint32_t qprefetch = 0;        // item searches: bulk L2 prefetch of each work item's queries (measured slower: c3 item search 1.55 -> 1.58 ms)
   uint32_t leaf256 = 1;          // leaf line by two 256-bit lane loads (one 64 B request per group)
   uint32_t sec256 = 0;           // implicit L2 levels: index / key sector by one lane's 256-bit load

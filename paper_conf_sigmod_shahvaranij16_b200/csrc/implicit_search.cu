@@ -732,7 +732,7 @@ struct Launch {
       attr_set = true;
     }
     ItemDir dd = d;
-    dd.rounds = item_rounds(m, t->num_sms, TH);
+    dd.rounds = item_rounds(m, t->num_sms, TH, t->cfg.item_rounds ? t->cfg.item_rounds : 16);
     uint64_t grid = t->num_sms;
     const uint64_t items = (m + uint64_t(TH) * dd.rounds - 1) / (uint64_t(TH) * dd.rounds);
     if (items < grid) grid = items ? items : 1;

@@ -16,9 +16,9 @@ constexpr uint32_t kPrefixBits = 10;
 // Warp rounds per work item of the bucketed item searches: 16 (staging the item's
 // directory is amortised over 16 K queries), fewer when the batch would leave SMs
 // idle (a 2^18-query c3 batch ran its 16 items on 16 SMs: 0.18 ms of search).
-inline uint32_t item_rounds(uint64_t m, uint32_t sms, uint32_t threads) {
+inline uint32_t item_rounds(uint64_t m, uint32_t sms, uint32_t threads, uint32_t cap = 16) {
   const uint64_t per_sm = (m + uint64_t(sms) * threads - 1) / (uint64_t(sms) * threads);
-  return uint32_t(per_sm < 1 ? 1 : (per_sm > 16 ? 16 : per_sm));
+  return uint32_t(per_sm < 1 ? 1 : (per_sm > cap ? cap : per_sm));
 }
 
 // One thread asks the TMA unit to pull a contiguous byte range into the L2

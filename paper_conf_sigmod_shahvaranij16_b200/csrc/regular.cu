@@ -951,7 +951,7 @@ int search_items_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* 
     attr = true;
   }
   ItemDir dd = d;
-  dd.rounds = item_rounds(m, t->num_sms, TH);
+  dd.rounds = item_rounds(m, t->num_sms, TH, t->cfg.item_rounds ? t->cfg.item_rounds : 16);
   uint64_t grid = t->num_sms;
   const uint64_t items = (m + uint64_t(TH) * dd.rounds - 1) / (uint64_t(TH) * dd.rounds);
   if (items < grid) grid = items ? items : 1;
