@@ -238,6 +238,14 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *   "host_bufs"   hbt_search_host: (stream, buffer) pairs in flight, 2..4 (default 2)
  *   "item_rounds" bucketed item searches: most warp rounds per work item (0 = default 16;
  *                 fewer are used when the batch would leave SMs idle)
+ *   "l2_hint"     implicit search: L2 eviction-priority hints (createpolicy + ld ...
+ *                 L2::cache_hint); bit 0 = leaf lines evict-first, bit 1 = whole-node levels
+ *                 evict-last; 4 = auto (default: bit 0 iff the I-segment fits in a quarter of
+ *                 the L2 — measured c2 0.426 -> 0.415 ms, c5 Zipf 2.84 -> 3.00 ms with it on)
+ *   "item_l2_hint" the same bits for the implicit bucketed item search (default 1: c4 item
+ *                 search 10.96 -> 9.50 ms, DRAM reads 171 -> 148 B/query)
+ *   "regular_l2_hint" the same bits for the regular item search (default 0: 1 measured
+ *                 slower on c3, 1.59 -> 1.72 ms)
  *   "full_levels" implicit: bit d set = level d's nodes are read whole in one round trip
  *                 (0 = default: by the "l2_levels_bytes" budget)
  * Unknown names or out-of-range values return HBT_EINVAL. */

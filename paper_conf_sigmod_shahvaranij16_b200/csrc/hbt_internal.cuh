@@ -44,6 +44,7 @@ struct LevelTable {
   uint32_t leaf256;    // leaf line read as one 64 B request (two 256-bit lane loads)
   uint32_t sec256;     // index / key sectors of L2 levels by one lane's 256-bit load
   uint32_t full256;    // whole-node levels read by 256-bit lane loads (half the load instructions)
+  uint32_t l2_hint;    // bit 0: leaf lines loaded L2::evict_first; bit 1: whole-node levels L2::evict_last
 };
 
 struct SearchConfig {
@@ -74,6 +75,10 @@ struct SearchConfig {
   uint32_t sec256 = 0;           // implicit L2 levels: index / key sector by one lane's 256-bit load
   uint32_t full256 = 1;          // implicit whole-node levels by 256-bit lane loads
   uint32_t full_levels = 0;      // implicit: bit d = read level d's nodes whole (0 = by the L2 budget)
+  uint32_t l2_hint = 4;          // implicit search: L2 eviction-priority hints (LevelTable::l2_hint);
+                                 // 4 = auto: leaf lines evict-first iff the I-segment fits in L2 / 4
+  uint32_t item_l2_hint = 1;     // implicit bucketed item search (c4 item search 10.96 -> 9.50 ms)
+  uint32_t regular_l2_hint = 0;  // regular bucketed item search (measured slower with 1: c3 1.59 -> 1.72 ms)
 };
 
 // Bucket-local directory of the bucketed search (bucketed.cu): after the

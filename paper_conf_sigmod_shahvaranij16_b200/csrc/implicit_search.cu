@@ -65,6 +65,25 @@ __device__ __forceinline__ void ld32(L256<K>& v, const uint8_t* p) {
                : "l"(p));
 }
 
+// The same with an L2 eviction-priority policy (createpolicy): leaf lines that are
+// read once per batch go evict-first so they do not push the inner levels out.
+template <typename K>
+__device__ __forceinline__ void ld32_pol(L256<K>& v, const uint8_t* p, uint64_t pol) {
+  asm volatile("ld.global.nc.L2::cache_hint.v4.u64 {%0, %1, %2, %3}, [%4], %5;"
+               : "=l"(v.u[0]), "=l"(v.u[1]), "=l"(v.u[2]), "=l"(v.u[3])
+               : "l"(p), "l"(pol));
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+__device__ __forceinline__ uint64_t policy_evict_last() {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+
 template <typename K>
 __device__ __forceinline__ void fill_max32(L256<K>& v) {
 #pragma unroll
@@ -145,11 +164,20 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
             // the pipe that binds the item search, profiles/r01_c4_items_*) of 16 B loads
             constexpr int NC32 = C::NODE_BYTES / C::G / 32;
             L256<K> fw[QPG][NC32];
+            if (lt.l2_hint & 2u) {
+              const uint64_t pol = policy_evict_last();
 #pragma unroll
-            for (int j = 0; j < QPG; ++j)
+              for (int j = 0; j < QPG; ++j)
 #pragma unroll
-              for (int h = 0; h < NC32; ++h)
-                ld32(fw[j][h], lvl + uint64_t(node[j]) * C::NODE_BYTES + (k * NC32 + h) * 32);
+                for (int h = 0; h < NC32; ++h)
+                  ld32_pol(fw[j][h], lvl + uint64_t(node[j]) * C::NODE_BYTES + (k * NC32 + h) * 32, pol);
+            } else {
+#pragma unroll
+              for (int j = 0; j < QPG; ++j)
+#pragma unroll
+                for (int h = 0; h < NC32; ++h)
+                  ld32(fw[j][h], lvl + uint64_t(node[j]) * C::NODE_BYTES + (k * NC32 + h) * 32);
+            }
 #pragma unroll
             for (int j = 0; j < QPG; ++j) {
               uint32_t c = 0;
@@ -253,10 +281,19 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
     //      the key sector, lane 1 the value sector with 256-bit loads (sm_100).
     //      s = #{keys < q} on lane 0, broadcast; key / value picked by lanes 0 / 1.
     L256<K> lw[QPG];
+    if (lt.l2_hint & 1u) {
+      const uint64_t pol = policy_evict_first();
 #pragma unroll
-    for (int j = 0; j < QPG; ++j) {
-      if (k < 2) ld32(lw[j], leaf + uint64_t(node[j]) * 64 + k * 32);
-      else fill_max32(lw[j]);
+      for (int j = 0; j < QPG; ++j) {
+        if (k < 2) ld32_pol(lw[j], leaf + uint64_t(node[j]) * 64 + k * 32, pol);
+        else fill_max32(lw[j]);
+      }
+    } else {
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) {
+        if (k < 2) ld32(lw[j], leaf + uint64_t(node[j]) * 64 + k * 32);
+        else fill_max32(lw[j]);
+      }
     }
 #pragma unroll
     for (int j = 0; j < QPG; ++j) {
@@ -619,6 +656,16 @@ struct Launch {
     lt.leaf256 = t->cfg.leaf256;
     lt.sec256 = t->cfg.sec256;
     lt.full256 = t->cfg.full256;
+    lt.l2_hint = t->cfg.l2_hint;
+    if (lt.l2_hint == 4) {
+      // auto: while the I-segment fits in a quarter of the L2, the leaf lines (read
+      // about once per batch) go evict-first so they cannot push the inner levels out
+      // (c2 0.426 -> 0.415 ms); a larger I-segment leaves the L2 to whatever the query
+      // distribution repeats (c5 Zipf: 2.84 -> 3.00 ms with the hint)
+      static int l2 = 0;
+      if (!l2) HBT_CUDA_TRY(cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, t->device));
+      lt.l2_hint = (t->inner_bytes + t->inner_idx_bytes) * 4 <= uint64_t(l2) ? 1u : 0u;
+    }
     size_t smem;
     if (MODE == 4) {
       lt.SL = t->dir_T;
@@ -717,6 +764,7 @@ struct Launch {
     lt.leaf256 = t->cfg.leaf256;
     lt.sec256 = t->cfg.sec256;
     lt.full256 = t->cfg.full256;
+    lt.l2_hint = t->cfg.item_l2_hint;
     {
       uint64_t cum = 0;
       const uint64_t budget = t->cfg.l2_levels_bytes ? t->cfg.l2_levels_bytes : (32ull << 20);

@@ -194,6 +194,7 @@ struct RView {
   uint64_t smem_first;  // pool index of the first staged upper node
   uint64_t smem_nodes;
   uint32_t leaf256;     // item search: key line and leaf line by 256-bit lane loads
+  uint32_t l2_hint;     // item search: bit 0 leaf lines L2::evict_first, bit 1 key lines L2::evict_last
 };
 
 template <typename K, int N>
@@ -222,6 +223,24 @@ __device__ __forceinline__ void ld32(L256<K>& v, const uint8_t* p) {
   asm volatile("ld.global.nc.v4.u64 {%0, %1, %2, %3}, [%4];"
                : "=l"(v.u[0]), "=l"(v.u[1]), "=l"(v.u[2]), "=l"(v.u[3])
                : "l"(p));
+}
+
+// 256-bit load with an L2 eviction-priority policy (createpolicy)
+template <typename K>
+__device__ __forceinline__ void ld32_pol(L256<K>& v, const uint8_t* p, uint64_t pol) {
+  asm volatile("ld.global.nc.L2::cache_hint.v4.u64 {%0, %1, %2, %3}, [%4], %5;"
+               : "=l"(v.u[0]), "=l"(v.u[1]), "=l"(v.u[2]), "=l"(v.u[3])
+               : "l"(p), "l"(pol));
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+__device__ __forceinline__ uint64_t policy_evict_last() {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
 }
 
 template <typename K>
@@ -706,8 +725,13 @@ regular_search_items_kernel(const RView rv, const ItemDir d, const K* __restrict
         L256<K> kw[QPG];
 #pragma unroll
         for (int j = 0; j < QPG; ++j) {
-          if (uint32_t(k) * 32 < LINE) ld32(kw[j], rv.lkeys + (uint64_t(cur[j]) * F + t[j] * KPL) * S + k * 32);
-          else fill_max32(kw[j]);
+          if (uint32_t(k) * 32 < LINE) {
+            const uint8_t* a = rv.lkeys + (uint64_t(cur[j]) * F + t[j] * KPL) * S + k * 32;
+            if (rv.l2_hint & 2u) ld32_pol(kw[j], a, policy_evict_last());
+            else ld32(kw[j], a);
+          } else {
+            fill_max32(kw[j]);
+          }
         }
         uint32_t line[QPG];
 #pragma unroll
@@ -719,8 +743,14 @@ regular_search_items_kernel(const RView rv, const ItemDir d, const K* __restrict
           line[j] = t[j] * KPL + c;
         }
         L256<K> lw[QPG];
+        if (rv.l2_hint & 1u) {
+          const uint64_t pol = policy_evict_first();
 #pragma unroll
-        for (int j = 0; j < QPG; ++j) ld32(lw[j], rv.leaf + (uint64_t(cur[j]) * F + line[j]) * 64 + k * 32);
+          for (int j = 0; j < QPG; ++j) ld32_pol(lw[j], rv.leaf + (uint64_t(cur[j]) * F + line[j]) * 64 + k * 32, pol);
+        } else {
+#pragma unroll
+          for (int j = 0; j < QPG; ++j) ld32(lw[j], rv.leaf + (uint64_t(cur[j]) * F + line[j]) * 64 + k * 32);
+        }
 #pragma unroll
         for (int j = 0; j < QPG; ++j) {
           uint32_t c = 0;
@@ -944,6 +974,7 @@ int search_items_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* 
   rv.lidx = (const uint8_t*)r.d_lidx;
   rv.U = r.U;
   rv.leaf256 = t->cfg.leaf256;
+  rv.l2_hint = t->cfg.regular_l2_hint;
   const size_t smem = (d.B + 1) * 8 + size_t(d.cap) * (sizeof(K) + 4) + ((1u << kPrefixBits) + 1) * 4;
   static bool attr = false;
   if (!attr) {

@@ -75,11 +75,15 @@ def test_bucketed_scaled_workload(hbt, layout, F, items, cap, leaf256):
         t.set_param("bucket_slice", slice_bytes)
         for qpf in (0, 1):  # with / without the bulk L2 prefetch of each item's queries
             t.set_param("qprefetch", qpf)
-            pf, val = gpu_search(t, q, 8)
-            assert np.array_equal(pf, epf) and np.array_equal(val, ev), (layout, slice_bytes, qpf)
+            for hint in (0, 1, 3):  # L2 eviction-priority hints on the item search's loads
+                t.set_param("item_l2_hint" if layout == "implicit" else "regular_l2_hint", hint)
+                pf, val = gpu_search(t, q, 8)
+                assert np.array_equal(pf, epf) and np.array_equal(val, ev), (layout, slice_bytes, qpf, hint)
     t.set_param("bucket", 0)
-    pf, val = gpu_search(t, q, 8)
-    assert np.array_equal(pf, epf) and np.array_equal(val, ev)
+    for hint in (0, 1, 2, 3, 4):  # plain search with the same hints (4 = auto)
+        t.set_param("l2_hint", hint)
+        pf, val = gpu_search(t, q, 8)
+        assert np.array_equal(pf, epf) and np.array_equal(val, ev), hint
     t.close()
 
 

@@ -68,6 +68,11 @@ def test_random_knob_parity(hbt, case):
         if layout == "implicit":
             knobs["leaf_stream"] = int(rng.choice([0, 1, 2]))
             knobs["stream_slice"] = int(rng.choice([64, 4096, 0]))
+    # L2 eviction-priority hints (own generator: the cases above keep their draws)
+    hrng = np.random.default_rng(case + 7777)
+    knobs["l2_hint"] = int(hrng.integers(0, 5))
+    knobs["item_l2_hint"] = int(hrng.integers(0, 4))
+    knobs["regular_l2_hint"] = int(hrng.integers(0, 4))
     for name, val in knobs.items():
         t.set_param(name, val)
     q = _queries(k, width, rng, int(rng.choice([1, 31, 1000, 40000])))
