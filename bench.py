@@ -155,13 +155,15 @@ def measure_h2d_gbs():
     return best
 
 
-def probe_l2_gbs(chunk):
+def probe_l2_gbs(chunk, nbytes=32 << 20):
+    """All-SM random reads of `chunk`-byte aligned chunks over an `nbytes` buffer
+    (32 MB: L2-resident; 1 GB: every read misses, i.e. the random-DRAM rate)."""
     import ctypes as C
     try:
         L = C.CDLL(os.path.join(ROOT, "tools", "libhbtprobe.so"))
         L.probe_random_read_gbs.restype = C.c_double
         L.probe_random_read_gbs.argtypes = [C.c_uint64, C.c_int, C.c_int]
-        v = L.probe_random_read_gbs(32 << 20, chunk, 3)
+        v = L.probe_random_read_gbs(nbytes, chunk, 3)
         return v if v > 0 else None
     except OSError:
         return None
@@ -466,6 +468,9 @@ def run_hbt(args):
     l2_probe = probe_l2_gbs(32 if node_b > 32 else node_b) if rank == 0 else None
     # the probe at every access granularity of the tree (reported beside the roofline)
     l2_probe_by_chunk = {str(b): round(probe_l2_gbs(b) or 0.0, 1) for b in (32, 64, 128)} if rank == 0 else None
+    # random 64 B reads over 1 GB (8x the L2): the rate DRAM sustains for the leaf-line access
+    # pattern (row activations, not bytes, bind it) -- context beside the HBM copy peak
+    dram_rand64 = probe_l2_gbs(64, 1 << 30) if rank == 0 else None
 
     use_graph = args.graph == "1" or (args.graph == "auto" and m <= (1 << 20) and args.config != "c4"
                                       and not args.origin_rank0)
@@ -561,6 +566,8 @@ def run_hbt(args):
                 # SURVEY 8(d) reporting: measured B/q from ncu and the fraction of the 8 TB/s spec HBM roof
                 "traffic_bytes_per_query": round(traffic_bytes / m, 2) if traffic_bytes else None,
                 "frac_of_8tbs_spec": round(hbm_ach / 8000.0, 4),
+                "random_64b_read_probe_gbs": round(dram_rand64, 1) if dram_rand64 else None,
+                "frac_of_random_64b_probe": round(hbm_ach / dram_rand64, 4) if dram_rand64 else None,
                 "model": model_desc}
     if args.config == "c4" and world > 1:
         a2a_b = (world - 1) / world * (w + 8 + w)
