@@ -330,6 +330,112 @@ __global__ void __launch_bounds__(kThreads, 2) bk_scatter(const K* __restrict__ 
   }
 }
 
+// Pass 2, paired form (knob "scatter_pair", off by default): one 1024-thread CTA orders TWO
+// consecutive chunks by bucket in shared memory.  The scan runs in (bucket, chunk) order,
+// so run (b, c+1) starts where run (b, c) ends (gb[c+1][b] = gb[c][b] + cnt[c][b]) and
+// the pair is written as B runs of twice the length: random DRAM writes are bound by
+// their count, not their bytes (c4: 8-query runs of 64 B).  linv is unchanged: each
+// query's position in ITS chunk's bucket-sorted order, which the gather reads back.
+// Measured slower (c3 0.47 -> 0.58 ms, c4 1.95 -> 2.31 ms, profiles/r01s5_scatter_pair.log):
+// one CTA per SM with three block scans per pair hides less latency than the longer
+// runs save, so the one-chunk kernel stays the default.
+constexpr int kPThreads = 2 * kThreads;
+template <typename K>
+__global__ void __launch_bounds__(kPThreads, 1) bk_scatter_pair(const K* __restrict__ q, uint64_t m,
+                                                              const uint16_t* __restrict__ bq,
+                                                              const uint32_t* __restrict__ tab,
+                                                              const uint32_t* __restrict__ gb, uint32_t B,
+                                                              uint64_t chunks, K* __restrict__ qs,
+                                                              uint16_t* __restrict__ linv) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  K* s_q = reinterpret_cast<K*>(smem);
+  uint16_t* s_b = reinterpret_cast<uint16_t*>(s_q + 2 * kChunk);
+  uint32_t* s_cnt0 = reinterpret_cast<uint32_t*>(s_b + 2 * kChunk);
+  uint32_t* s_cnt1 = s_cnt0 + kMaxBuckets;
+  uint32_t* s_cc = s_cnt1 + kMaxBuckets;
+  uint32_t* s_lb0 = s_cc + kMaxBuckets;
+  uint32_t* s_lb1 = s_lb0 + kMaxBuckets;
+  uint32_t* s_L = s_lb1 + kMaxBuckets;
+  uint32_t* s_gb = s_L + kMaxBuckets;
+  uint32_t* s_rank = s_gb + kMaxBuckets;  // 2 x kMaxBuckets
+  uint32_t* s_tmp = s_rank + 2 * kMaxBuckets;
+  const uint32_t h = threadIdx.x / kThreads, tl = threadIdx.x % kThreads;  // chunk of the pair, lane in it
+  const uint64_t pairs = (chunks + 1) / 2;
+  for (uint64_t pc = blockIdx.x; pc < pairs; pc += gridDim.x) {
+    const uint64_t c0 = 2 * pc;
+    const bool has1 = c0 + 1 < chunks;
+    const uint64_t lo = (c0 + h) * kChunk;
+    const uint32_t nc = (c0 + h < chunks) ? uint32_t(m - lo < kChunk ? m - lo : kChunk) : 0u;
+    K qq[kQPT];
+    uint32_t bb[kQPT];
+#pragma unroll
+    for (int j = 0; j < kQPT; ++j) {
+      const uint32_t t = uint32_t(j) * kThreads + tl;
+      qq[j] = K(0);
+      bb[j] = 0;
+      if (t < nc) {
+        qq[j] = __ldcs(q + lo + t);
+        bb[j] = __ldcs(reinterpret_cast<const unsigned short*>(bq) + lo + t);
+      }
+    }
+    for (uint32_t b = threadIdx.x; b < B; b += kPThreads) {
+      s_rank[b] = 0;
+      s_rank[kMaxBuckets + b] = 0;
+      const uint32_t a0 = tab[c0 * B + b], a1 = has1 ? tab[(c0 + 1) * B + b] : 0u;
+      s_cnt0[b] = a0;
+      s_cnt1[b] = a1;
+      s_cc[b] = a0 + a1;
+      s_gb[b] = gb[c0 * B + b];
+    }
+    __syncthreads();
+    block_exclusive_scan<kPThreads>(s_cnt0, s_lb0, B, s_tmp);
+    block_exclusive_scan<kPThreads>(s_cnt1, s_lb1, B, s_tmp);
+    block_exclusive_scan<kPThreads>(s_cc, s_L, B, s_tmp);
+    const uint32_t* lbh = h ? s_lb1 : s_lb0;
+    uint32_t* rankh = s_rank + h * kMaxBuckets;
+#pragma unroll
+    for (int j = 0; j < kQPT; ++j) {
+      const uint32_t t = uint32_t(j) * kThreads + tl;
+      if (t < nc) {
+        const uint32_t b = bb[j];
+        const uint32_t r = atomicAdd(&rankh[b], 1u);
+        const uint32_t pos = s_L[b] + (h ? s_cnt0[b] : 0u) + r;  // pair order: (bucket, chunk, rank)
+        s_q[pos] = qq[j];
+        s_b[pos] = uint16_t(b);
+        __stcs(reinterpret_cast<unsigned short*>(linv) + lo + t, (unsigned short)(lbh[b] + r));
+      }
+    }
+    __syncthreads();
+    const uint32_t ntot = uint32_t(m - c0 * kChunk < 2 * kChunk ? m - c0 * kChunk : 2 * kChunk);
+#pragma unroll 4
+    for (uint32_t t = threadIdx.x; t < ntot; t += kPThreads) {
+      const uint32_t b = s_b[t];
+      qs[uint64_t(s_gb[b]) + (t - s_L[b])] = s_q[t];
+    }
+    __syncthreads();
+  }
+}
+
+template <typename K>
+size_t scatter_pair_smem() {
+  return 2 * kChunk * (sizeof(K) + 2) + kMaxBuckets * 4 * 9 + 32 * 4;
+}
+
+// Pass 2 launch: the one-chunk kernel (default) or the paired kernel ("scatter_pair" = 1).
+template <typename K>
+void launch_scatter(const hbt_tree* t, unsigned grid, size_t smem_single, const void* q, uint64_t m,
+                    const uint16_t* bq, const uint32_t* tab, const uint32_t* gb, uint32_t B, uint64_t chunks,
+                    K* qs, uint16_t* linv, cudaStream_t s) {
+  if (t->cfg.scatter_pair) {
+    const uint64_t pairs = (chunks + 1) / 2;
+    const unsigned g = unsigned(std::min<uint64_t>(pairs, uint64_t(t->num_sms)));
+    bk_scatter_pair<K><<<g ? g : 1, kPThreads, scatter_pair_smem<K>(), s>>>((const K*)q, m, bq, tab, gb, B, chunks,
+                                                                          qs, linv);
+  } else {
+    bk_scatter<K><<<grid, kThreads, smem_single, s>>>((const K*)q, m, bq, tab, gb, B, chunks, qs, linv);
+  }
+}
+
 // Pass 4: the chunk's results are read back as its B contiguous runs into
 // shared memory (bucket-sorted order), then stored in query order through linv.
 template <typename K>
@@ -503,6 +609,10 @@ void set_bucket_attrs() {
   cudaFuncSetAttribute(bk_count<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
   cudaFuncSetAttribute(bk_scatter<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
   cudaFuncSetAttribute(bk_scatter<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
+  cudaFuncSetAttribute(bk_scatter_pair<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       int(scatter_pair_smem<uint32_t>()));
+  cudaFuncSetAttribute(bk_scatter_pair<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       int(scatter_pair_smem<uint64_t>()));
   cudaFuncSetAttribute(bk_gather<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
   cudaFuncSetAttribute(bk_gather<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
   cudaFuncSetAttribute(bk_gather_rec<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
@@ -674,7 +784,7 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
       }
     }
     mark(2);
-    bk_scatter<K><<<grid, kThreads, smem_scatter, s>>>((const K*)q, m, bq, tab, gb, B, chunks, qs, linv);
+    launch_scatter<K>(t, grid, smem_scatter, q, m, bq, tab, gb, B, chunks, qs, linv, s);
     if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) {
       set_error("bucketing kernels failed to launch: %s", cudaGetErrorString(e));
       rc = HBT_ECUDA;
@@ -812,7 +922,7 @@ int streamed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
     }
     bk_transpose<<<dim3(unsigned((chunks + 31) / 32), (B + 31) / 32), tb, 0, s>>>(gb_bm, B, uint32_t(chunks), gb);
     bk_bstart<<<(B + 256) / 256, 256, 0, s>>>(gb_bm, chunks, B, m, bstart);
-    bk_scatter<K><<<grid, kThreads, smem_scatter, s>>>((const K*)q, m, bq, tab, gb, B, chunks, qs, linv);
+    launch_scatter<K>(t, grid, smem_scatter, q, m, bq, tab, gb, B, chunks, qs, linv, s);
     if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) {
       set_error("bucketing kernels failed to launch: %s", cudaGetErrorString(e));
       rc = HBT_ECUDA;

@@ -78,6 +78,8 @@ struct SearchConfig {
   uint32_t l2_hint = 4;          // implicit search: L2 eviction-priority hints (LevelTable::l2_hint);
                                  // 4 = auto: leaf lines evict-first iff the I-segment fits in L2 / 4
   uint32_t item_l2_hint = 1;     // implicit bucketed item search (c4 item search 10.96 -> 9.50 ms)
+  uint32_t scatter_pair = 0;     // bucketed search: scatter two chunks per CTA (runs twice as long; measured
+                                 // slower: c3 scatter 0.47 -> 0.58 ms, c4 1.95 -> 2.31 ms)
   uint32_t regular_l2_hint = 0;  // regular bucketed item search (measured slower with 1: c3 1.59 -> 1.72 ms)
 };
 
