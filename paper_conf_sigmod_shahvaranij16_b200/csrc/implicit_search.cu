@@ -105,7 +105,9 @@ __device__ __forceinline__ void stcs(uint64_t* p, uint64_t v) {
   __stcs(reinterpret_cast<unsigned long long*>(p), (unsigned long long)v);
 }
 
-template <typename K, int F>
+// GMIN: smallest lane group (2; 4 lets a 128 B whole node be read by ONE 256-bit load per
+// lane, one L1TEX wavefront per query instead of two -- the item search's "item_group4")
+template <typename K, int F, int GMIN = 2>
 struct Cfg {
   static constexpr int S = int(sizeof(K));
   static constexpr int NODE_BYTES = F * S;
@@ -116,7 +118,7 @@ struct Cfg {
   static constexpr int IL = IDXB / 16;                                    // lanes loading the index
   static constexpr int SECB = NODE_BYTES < 32 ? NODE_BYTES : 32;          // bytes read after the index
   static constexpr int SL_ = SECB / 16;                                   // lanes loading them
-  static constexpr int G = IL > 2 ? IL : 2;                               // lanes per query group
+  static constexpr int G = IL > GMIN ? IL : GMIN;                         // lanes per query group
   static constexpr int NG = 32 / G;                                       // groups per warp
   static constexpr int P = 64 / (2 * S);                                  // pairs per leaf line
 };
@@ -140,7 +142,7 @@ __device__ __forceinline__ uint32_t count_less16(const V16<K>& v, K q, unsigned 
 // Phase 2 of a warp round: levels [d0, H) by lane groups, the leaf line, and the
 // results of the round (slot j of group g = round query j*NG + g, stored at
 // base + j*NG + g).  sec_known: the sector of level d0 is already in sec0.
-template <typename K, int F, int QPG, bool REC = false>
+template <typename K, int F, int QPG, bool REC = false, int GM = 2>
 __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ inner,
                                                   const uint8_t* __restrict__ inner_idx,
                                                   const uint8_t* __restrict__ leaf, const LevelTable& lt,
@@ -148,7 +150,7 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
                                                   const uint32_t (&sec0)[QPG], int g, int k, unsigned gmask,
                                                   uint64_t base, uint64_t m, uint64_t n, uint64_t pos_base,
                                                   uint64_t* __restrict__ out_pf, K* __restrict__ out_v) {
-  using C = Cfg<K, F>;
+  using C = Cfg<K, F, GM>;
   const uint32_t H = lt.H;
   for (uint32_t d = d0; d < H; ++d) {
     const uint8_t* lvl = inner + lt.offset[d] * C::NODE_BYTES;
@@ -552,13 +554,13 @@ __device__ __forceinline__ void stage_keys(K* dst, const K* __restrict__ src, ui
   }
 }
 
-template <typename K, int F, int THREADS>
+template <typename K, int F, int THREADS, int GM = 2>
 __global__ void __launch_bounds__(THREADS)
 implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ inner_idx,
                              const uint8_t* __restrict__ leaf, const ItemDir d, const K* __restrict__ queries,
                              uint64_t m, uint64_t* __restrict__ out_pf, K* __restrict__ out_v, const LevelTable lt,
                              uint64_t n) {
-  using C = Cfg<K, F>;
+  using C = Cfg<K, F, GM>;
   constexpr int QPG = 32 / C::NG;
   const uint64_t W = uint64_t(THREADS) * d.rounds;
   extern __shared__ __align__(16) uint8_t smem[];
@@ -626,7 +628,7 @@ implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* _
         node[j] = __shfl_sync(0xffffffffu, mynode, src);
         sec0[j] = 0;
       }
-      descend_and_store<K, F, QPG, true>(inner, inner_idx, leaf, lt, d.level, false, q, node, sec0, g, k, gmask,
+      descend_and_store<K, F, QPG, true, GM>(inner, inner_idx, leaf, lt, d.level, false, q, node, sec0, g, k, gmask,
                                          base, p1 + 1, n, d.pos_base, out_pf, out_v);
     }
     __syncthreads();
@@ -756,7 +758,9 @@ struct Launch {
   static int run_items(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, const ItemDir& d,
                        cudaStream_t s) {
     constexpr int TH = C::NODE_BYTES > 128 ? 512 : 1024;
-    auto kern = implicit_search_items_kernel<K, F, TH>;
+    // 128 B nodes: 4-lane groups on request (one 256-bit whole-node load per lane)
+    auto kern = (C::NODE_BYTES == 128 && C::G < 4 && t->cfg.item_group4) ? implicit_search_items_kernel<K, F, TH, 4>
+                                                                         : implicit_search_items_kernel<K, F, TH>;
     LevelTable lt{};
     for (uint32_t x = 0; x <= t->H; ++x) lt.offset[x] = t->offset[x];
     lt.H = t->H;
@@ -774,10 +778,11 @@ struct Launch {
       }
     }
     const size_t smem = (d.B + 1) * 8 + size_t(d.cap) * C::S + ((1u << kPrefixBits) + 1) * 4;
-    static bool attr_set = false;
-    if (!attr_set) {
+    static bool attr_set[2] = {false, false};  // per kernel variant
+    const int av = kern == implicit_search_items_kernel<K, F, TH> ? 0 : 1;
+    if (!attr_set[av]) {
       HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
-      attr_set = true;
+      attr_set[av] = true;
     }
     ItemDir dd = d;
     dd.rounds = item_rounds(m, t->num_sms, TH, t->cfg.item_rounds ? t->cfg.item_rounds : 16);
