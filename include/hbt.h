@@ -248,6 +248,8 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *                 queries per 1024-thread CTA, so every bucket run it writes is twice as long;
  *                 0 (default) = one chunk per 512-thread CTA (measured faster: c3 scatter
  *                 0.47 vs 0.58 ms)
+ *   "small_threads" small-batch search (directory read in place): CTA size 128, 256 or 1024
+ *                 (0 = default 256; 128 measured the same on c1, 1024 slower)
  *   "item_group4" implicit item search with 128 B nodes: 1 = 4-lane query groups (one 256-bit
  *                 whole-node load per lane); 0 (default, measured faster: c4 9.50 vs 10.8 ms)
  *   "regular_l2_hint" the same bits for the regular item search (default 0: 1 measured

@@ -80,6 +80,7 @@ struct SearchConfig {
   uint32_t item_l2_hint = 1;     // implicit bucketed item search (c4 item search 10.96 -> 9.50 ms)
   uint32_t scatter_pair = 0;     // bucketed search: scatter two chunks per CTA (runs twice as long; measured
                                  // slower: c3 scatter 0.47 -> 0.58 ms, c4 1.95 -> 2.31 ms)
+  uint32_t small_threads = 0;    // small-batch (in-place directory) search: CTA size 128 / 256 / 1024 (0 = 256)
   uint32_t item_group4 = 0;      // implicit item search, 128 B nodes: 4-lane groups (one 256-bit load per lane;
                                  // measured slower: c4 item search 9.50 -> 10.8 ms, 56 B of spills)
   uint32_t regular_l2_hint = 0;  // regular bucketed item search (measured slower with 1: c3 1.59 -> 1.72 ms)

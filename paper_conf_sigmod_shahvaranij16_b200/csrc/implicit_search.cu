@@ -803,7 +803,9 @@ struct Launch {
     // small batches read the directory in place (no 96 KB staging per CTA)
     if (t->cfg.mode == 3 || (t->cfg.mode == 2 && m <= t->cfg.small_batch))
       // 256-thread CTAs spread a small batch over every SM (c1: 10.1 -> 8.3 us per batch)
-      return t->cfg.threads == 1024 ? run_t<1, 1024, 3>(t, q, m, pf, v, b, s, lp) : run_t<1, 256, 3>(t, q, m, pf, v, b, s, lp);
+      return (t->cfg.threads == 1024 || t->cfg.small_threads == 1024) ? run_t<1, 1024, 3>(t, q, m, pf, v, b, s, lp)
+             : t->cfg.small_threads == 128                               ? run_t<1, 128, 3>(t, q, m, pf, v, b, s, lp)
+                                                                         : run_t<1, 256, 3>(t, q, m, pf, v, b, s, lp);
     if (t->cfg.mode == 4 && t->d_sdir)
       return th == 512 ? run_t<1, 512, 4>(t, q, m, pf, v, b, s, lp) : run_t<1, 1024, 4>(t, q, m, pf, v, b, s, lp);
     if (t->cfg.mode == 2) {

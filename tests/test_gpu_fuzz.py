@@ -75,6 +75,7 @@ def test_random_knob_parity(hbt, case):
     knobs["regular_l2_hint"] = int(hrng.integers(0, 4))
     knobs["scatter_pair"] = int(hrng.integers(0, 2))
     knobs["item_group4"] = int(hrng.integers(0, 2))
+    knobs["small_threads"] = int(hrng.choice([0, 128, 256, 1024]))
     for name, val in knobs.items():
         t.set_param(name, val)
     q = _queries(k, width, rng, int(rng.choice([1, 31, 1000, 40000])))
