@@ -74,6 +74,7 @@ PROBE_API double probe_random_read_gbs(uint64_t bytes, int chunk, int reps) {
     cudaEventRecord(a);
     if (chunk == 32) l2_random_read<32, 8><<<grid, threads>>>(buf, nchunks, iters, r, sink);
     else if (chunk == 64) l2_random_read<64, 8><<<grid, threads>>>(buf, nchunks, iters, r, sink);
+    else if (chunk == 256) l2_random_read<256, 8><<<grid, threads>>>(buf, nchunks, iters, r, sink);
     else l2_random_read<128, 8><<<grid, threads>>>(buf, nchunks, iters, r, sink);
     cudaEventRecord(b);
     cudaEventSynchronize(b);
