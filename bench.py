@@ -1,21 +1,29 @@
 #!/usr/bin/env python
 """bench.py — batched HB+-tree lookups on B200 (one JSON line on rank 0).
 
-Default workload = BASELINE.json configs[1] (c2), the metric's 1-GPU config:
-implicit tree, 2^23 uint64 keys, fanout 16, 2^24 uniform hit queries per GPU.
-A "step" is one hbt_search over the whole batch (every hot-path row: the
-top-level directory / node search through every level, the leaf search and
-the result write).  Inputs are seeded synthetic (gen/) generated
-on the device; queries + results per step exceed the 126 MB L2, so no L2 flush
-is done between steps.
+Default workload = BASELINE.json configs[3] (c4), the north_star's sharded
+config and the largest one that fits one B200: an implicit tree of 2^31
+stratified uint64 keys (fanout 16, 36 GiB of tree) and 2^28 uniform hit
+queries in total.  At N = 1 the whole tree sits on one GPU; at N > 1 it is
+key-range sharded over the N ranks (2^31/N keys and 2^28/N queries per rank,
+every query routed to its owner shard and its result returned),
+so the total work is fixed: "scaling": "strong".  A "step" is one search of the
+whole batch (every hot-path row: routing, bucketing, the bucket-local directory /
+node search through every level, the leaf search, the result write and, at
+N > 1, the exchange both ways).  Inputs are seeded synthetic (gen/, SURVEY
+§8(d)) generated on the device; queries + results per step exceed the 126 MB
+L2, so no L2 flush is done between steps.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--config c1|c2|c3|c4|c5]
   python bench.py --impl reference ...   # the CPU oracle arm (rank 0 only)
 
-Multi-GPU (torchrun, one process per GPU): c1/c2/c3/c5 run one replica per
-rank, each searching its own batch (weak scaling, no collective on the data
-path); c4 is the key-range-sharded tree (2^31 keys split over
-the ranks, 2^28 queries in total, NCCL all-to-all of queries and results).
+--gpus N without a torchrun environment re-launches itself under
+torch.distributed.run with N local ranks (127.0.0.1).  When there are more ranks
+than visible GPUs (a dry run of the multi-rank path on one GPU) the ranks share
+the devices round-robin, the process group is gloo and the sharded tree uses the
+host-callback communicator with the fused peer-memory exchange.
+c1/c2/c3/c5 at N > 1 run one replica per rank, each searching its own batch
+(weak scaling, no collective on the data path).
 """
 from __future__ import annotations
 
@@ -44,7 +52,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=400)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="hbt", choices=["hbt", "reference"])
-    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c4", "c5"])
+    ap.add_argument("--config", default="c4", choices=["c1", "c2", "c3", "c4", "c5"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--smem", type=int, default=0, help="override smem budget (bytes)")
@@ -84,6 +92,86 @@ def parse():
 
 def dist_env():
     return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
+
+
+def maybe_spawn(args):
+    """--gpus N outside torchrun: re-launch this script under torch.distributed.run
+    with N local ranks (rendezvous on 127.0.0.1) and return its exit code."""
+    if args.gpus <= 1 or "WORLD_SIZE" in os.environ or args.impl == "reference":
+        return None
+    import socket
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
+class Dist:
+    """The process group of a run: NCCL with one rank per GPU; gloo (CPU tensors)
+    when more ranks than visible GPUs share the devices (multi-rank dry run)."""
+
+    def __init__(self, rank, world, local):
+        import torch
+        import torch.distributed as dist
+        self.rank, self.world = rank, world
+        ndev = max(torch.cuda.device_count(), 1)
+        self.device = local % ndev
+        self.shared_gpus = world > ndev
+        self.backend = None
+        torch.cuda.set_device(self.device)
+        if world > 1:
+            self.backend = "gloo" if self.shared_gpus else "nccl"
+            if self.backend == "nccl":
+                dist.init_process_group("nccl", device_id=torch.device("cuda", self.device))
+            else:
+                dist.init_process_group("gloo")
+
+    def barrier(self):
+        import torch.distributed as dist
+        if self.world > 1:
+            dist.barrier()
+
+    def max(self, x: float) -> float:
+        """max over ranks (device tensor under NCCL, CPU tensor under gloo)."""
+        import torch
+        import torch.distributed as dist
+        if self.world == 1:
+            return float(x)
+        t = torch.tensor([x], dtype=torch.float64, device="cuda" if self.backend == "nccl" else "cpu")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def close(self):
+        import torch.distributed as dist
+        if self.world > 1:
+            dist.destroy_process_group()
+
+
+def probe_a2a_gbs(d: "Dist", nbytes=256 << 20):
+    """In-run NVLink probe (SURVEY §8(d) BW_NVL): NCCL all_to_all_single of `nbytes`
+    per rank, best of 3; returns the bytes each GPU sends to its peers per second
+    ((N-1)/N of the buffer) in GB/s, or None (one rank, or ranks sharing a GPU)."""
+    import torch
+    import torch.distributed as dist
+    if d.world == 1 or d.backend != "nccl":
+        return None
+    a = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    b = torch.empty_like(a)
+    best = 0.0
+    for _ in range(4):
+        d.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        dist.all_to_all_single(b, a)
+        e1.record()
+        torch.cuda.synchronize()
+        t = d.max(e0.elapsed_time(e1) * 1e-3)
+        best = max(best, nbytes * (d.world - 1) / d.world / t / 1e9)
+    del a, b
+    return best
 
 
 def measured_peaks():
@@ -179,12 +267,13 @@ class Work:
         self.__dict__.update(kw)
 
 
-def make_work(cfg_name, rank, world, args):
+def make_work(cfg_name, d, args):
     import torch
 
     import paper_conf_sigmod_shahvaranij16_b200 as hbt
     from gen.device import GenLib
 
+    rank, world = d.rank, d.world
     g = GenLib()
     c = gen.CONFIGS[cfg_name]
     n, m, w, F = c["n"], c["m"], c["width"], c["fanout"]
@@ -200,8 +289,15 @@ def make_work(cfg_name, rank, world, args):
         vals = g.mix_stream(hi - lo, w, sv, start=lo)
         m_local = m // world
         q = g.stratified_queries(m_local, n, sq, sk, start=rank * m_local)
-        comm = hbt.Comm.from_torch() if world > 1 else hbt.Comm(1, 0, hbt.unique_id())
+        if world == 1:
+            comm = hbt.Comm(1, 0, hbt.unique_id())
+        elif d.backend == "nccl":
+            comm = hbt.Comm.from_torch()
+        else:  # ranks sharing a GPU: NCCL refuses them; host all-gathers over gloo + IPC windows
+            comm = hbt.Comm.from_torch_host()
         tree = hbt.ShardedTree(comm, keys, vals, fanout=F)
+        if d.backend == "gloo":
+            tree.set_param("exchange", 0)
         qdesc = f"uniform hits over all {n} keys, {m_local} per rank, routed to their owner shard"
         extra["comm"] = comm
         m = m_local
@@ -290,7 +386,7 @@ def make_work(cfg_name, rank, world, args):
         qdesc += "; the queries of all ranks originate on rank 0 (scatter + gather inside each step)"
     return Work(c=c, name=cfg_name, tree=tree, q=q, m=m, w=w, hit_rate=hit_rate, qdesc=qdesc, extra=extra,
                 out_pos=out_pos, out_val=out_val, info=tree.info(), range_k=args.range_k, hi=hi,
-                origin=origin, rank=rank, world=world)
+                origin=origin, rank=rank, world=world, dist=d)
 
 
 def step(work):
@@ -355,18 +451,17 @@ def step_fits_l2(work):
     return data < torch.cuda.get_device_properties(torch.cuda.current_device()).L2_cache_size
 
 
-def time_search_flushed(work, steps, world, graph=None):
+def time_search_flushed(work, steps, graph=None):
     """Small working sets (the tree and the batch fit in the L2): flush the L2 between
     timed steps by writing a 2x-L2 buffer, and sum per-step CUDA-event intervals (the
     flush itself is outside every interval).  Max over ranks."""
     import torch
-    import torch.distributed as dist
+    d = work.dist
     stream = torch.cuda.current_stream()
     l2 = torch.cuda.get_device_properties(torch.cuda.current_device()).L2_cache_size
     flush = torch.empty(2 * l2 // 4, dtype=torch.int32, device="cuda")
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
-    if world > 1:
-        dist.barrier()
+    d.barrier()
     torch.cuda.synchronize()
     for a, b in evs:
         flush.fill_(1)
@@ -377,25 +472,20 @@ def time_search_flushed(work, steps, world, graph=None):
             step(work)
         b.record(stream)
     torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
-    t = torch.tensor([sum(a.elapsed_time(b) for a, b in evs)], dtype=torch.float64, device="cuda")
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    return float(t.item()) / steps
+    d.barrier()
+    return d.max(sum(a.elapsed_time(b) for a, b in evs)) / steps
 
 
-def time_search(work, steps, world, graph=None):
+def time_search(work, steps, graph=None):
     """K launches of the step, CUDA events on the launching stream, max over ranks."""
     import torch
-    import torch.distributed as dist
     if step_fits_l2(work):
-        return time_search_flushed(work, steps, world, graph)
+        return time_search_flushed(work, steps, graph)
+    d = work.dist
     stream = torch.cuda.current_stream()
     ev0 = torch.cuda.Event(enable_timing=True)
     ev1 = torch.cuda.Event(enable_timing=True)
-    if world > 1:
-        dist.barrier()
+    d.barrier()
     torch.cuda.synchronize()
     ev0.record(stream)
     if graph is not None:
@@ -406,18 +496,14 @@ def time_search(work, steps, world, graph=None):
             step(work)
     ev1.record(stream)
     torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
-    t = torch.tensor([ev0.elapsed_time(ev1)], dtype=torch.float64, device="cuda")
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    return float(t.item()) / steps
+    d.barrier()
+    return d.max(ev0.elapsed_time(ev1)) / steps
 
 
-def time_e2e(work, steps, world):
+def time_e2e(work, steps):
     """Same metric through the public API with pinned HOST buffers (H2D + D2H inside)."""
     import torch
-    import torch.distributed as dist
+    d = work.dist
     m, w = work.m, work.w
     hq = work.q.cpu().pin_memory()
     hp = torch.empty(m, dtype=torch.int64).pin_memory()
@@ -435,22 +521,17 @@ def time_e2e(work, steps, world):
             work.tree.search_host(hq, hp, hv)
 
     one()
-    if world > 1:
-        dist.barrier()
+    d.barrier()
     torch.cuda.synchronize()
     t0 = time.perf_counter()
     for _ in range(steps):
         one()
-    el = time.perf_counter() - t0
-    te = torch.tensor([el], dtype=torch.float64, device="cuda")
-    if world > 1:
-        dist.all_reduce(te, op=dist.ReduceOp.MAX)
-    qps = world * m * steps / float(te.item())
+    el = d.max(time.perf_counter() - t0)
+    qps = d.world * m * steps / el
     api = ("H2D + hbt_search_sharded + D2H (pinned host buffers)" if sharded else
            "hbt_search_host (pinned host buffers, 1 Mi-query buckets double-buffered over 2 streams)")
     return {"value": round(qps / 1e6, 2), "unit": "M queries/s", "h2d_bytes_per_step": m * w,
-            "d2h_bytes_per_step": m * (8 + w), "api": api,
-            "gpu_launches_per_step": (4 if sharded else -(-m // (1 << 20)))}
+            "d2h_bytes_per_step": m * (8 + w), "api": api}
 
 
 def run_hbt(args):
@@ -458,10 +539,8 @@ def run_hbt(args):
     import torch.distributed as dist
 
     rank, world, local = dist_env()
-    torch.cuda.set_device(local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    work = make_work(args.config, rank, world, args)
+    d = Dist(rank, world, local)
+    work = make_work(args.config, d, args)
     c, m, w, info = work.c, work.m, work.w, work.info
     torch.cuda.synchronize()
     node_b = ((c["fanout"] * w + 31) // 32) * 32
@@ -471,6 +550,8 @@ def run_hbt(args):
     # random 64 B reads over 1 GB (8x the L2): the rate DRAM sustains for the leaf-line access
     # pattern (row activations, not bytes, bind it) -- context beside the HBM copy peak
     dram_rand64 = probe_l2_gbs(64, 1 << 30) if rank == 0 else None
+    # NVLink (SURVEY 8(d) BW_NVL) for the sharded config's a2a term, measured in this run
+    a2a_gbs = probe_a2a_gbs(d) if args.config == "c4" else None
 
     use_graph = args.graph == "1" or (args.graph == "auto" and m <= (1 << 20) and args.config != "c4"
                                       and not args.origin_rank0)
@@ -481,9 +562,9 @@ def run_hbt(args):
         else:
             step(work)
     torch.cuda.synchronize()
-    sampler = ClockSampler(local)
+    sampler = ClockSampler(d.device)
     sampler.start()
-    ms_step = time_search(work, args.steps, world, graph)
+    ms_step = time_search(work, args.steps, graph)
     clocks = sampler.stop()
     qps = world * m / (ms_step * 1e-3)
     launches_per_step = 4 if args.config == "c4" else (2 if args.range_k else 1)
@@ -499,14 +580,14 @@ def run_hbt(args):
         upd_s = time.perf_counter() - t0
         for _ in range(3):
             work.tree.search(work.q, work.out_pos, work.out_val)
-        ms_after = time_search(work, args.steps, world)
+        ms_after = time_search(work, args.steps)
         after = {"update_ops": int(bk.numel()), "update_ms": round(upd_s * 1e3, 3),
                  "update_ops_per_s": round(bk.numel() / upd_s, 1),
                  "search_after_update": {"value": round(world * m / (ms_after * 1e-3) / 1e6, 2),
                                          "unit": "M queries/s", "ms_per_step": round(ms_after, 4)},
                  "n_distinct_after": work.tree.info()["n_distinct"]}
 
-    e2e = time_e2e(work, args.e2e_steps, world) if not args.range_k else None
+    e2e = time_e2e(work, args.e2e_steps) if not args.range_k else None
 
     # ---- roofline of the step's dominant kernel.  Unbucketed: the step IS one search
     # launch.  Bucketed (regular trees beyond the L2, csrc/bucketed.cu): the step is
@@ -527,7 +608,7 @@ def run_hbt(args):
             phases = {k_: (round(v_ / reps, 4) if k_ != "launches" else int(v_ / reps)) for k_, v_ in acc.items()}
         except hbt.HBTError:
             phases = None
-    l2_size = torch.cuda.get_device_properties(local).L2_cache_size
+    l2_size = torch.cuda.get_device_properties(d.device).L2_cache_size
     gran_extra = 0
     if phases:
         mdl = roofline.model_bucketed(info, m)
@@ -571,8 +652,12 @@ def run_hbt(args):
                 "model": model_desc}
     if args.config == "c4" and world > 1:
         a2a_b = (world - 1) / world * (w + 8 + w)
-        t_roof = mdl["hbm_bytes_per_query"] / (peak * 1e9) + a2a_b / (NVLINK_GBS * 1e9)
+        bw_nvl = a2a_gbs or NVLINK_GBS
+        t_roof = mdl["hbm_bytes_per_query"] / (peak * 1e9) + a2a_b / (bw_nvl * 1e9)
         roof_hbm["a2a_bytes_per_query"] = round(a2a_b, 2)
+        roof_hbm["nvlink_gbs"] = round(bw_nvl, 1)
+        roof_hbm["nvlink_source"] = ("measured in this run (NCCL all_to_all_single)" if a2a_gbs else
+                                     "B200_PROFILING.md peer copy 770 GB/s per direction (fallback)")
         roof_hbm["frac_with_nvlink"] = round((m / t_kernel) * t_roof, 4)
     roof_l2 = None
     if l2_probe:
@@ -624,15 +709,11 @@ def run_hbt(args):
         roof["note"] = ("latency-bound batch: %d queries are one wave of the GPU, so the step is the launch "
                         "plus one query's chain of dependent memory round trips; no byte roofline binds" % m)
 
-    if phases and e2e and args.bucket == 1:  # forced bucketing: every 1 Mi-query chunk runs the pipeline
-        e2e["gpu_launches_per_step"] *= phases["launches"]
-
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(args.config)
 
-    if world > 1:
-        dist.barrier()
+    d.barrier()
     if rank == 0:
         line = {
             "metric": "lookups/sec (M queries/s)",
@@ -643,42 +724,67 @@ def run_hbt(args):
             "warmup": max(args.warmup, 3),
             "ms_per_step": round(ms_step, 4),
             "higher_is_better": True,
-            "scaling": "weak",
+            "scaling": "strong" if args.config == "c4" else "weak",
             "vs_baseline": None,
             "dtype": "u64" if w == 8 else "u32",
             "data": "synthetic (seeded counter-based generators, gen/)",
-            "config": {"workload": f"{args.config}: {c['layout']} tree, n={c['n']} keys (u{8 * w}), fanout "
-                                   f"{c['fanout']}, m={m} queries/GPU ({work.qdesc})",
-                       "n_keys": c["n"], "queries_per_gpu": m, "fanout": c["fanout"], "layout": c["layout"],
-                       "key_bits": 8 * w,
-                       "exchange": ("fused peer-memory (CUDA IPC windows)" if not args.exchange else "NCCL send/recv")
-                                   if args.config == "c4" else None,
-                       "parallelism": (f"key-range sharded x{world}" if args.config == "c4" else
-                                       (f"replicated x{world}" if world > 1 else "single")),
-                       "l2_policy": ("L2 flushed between timed steps (2x-L2 buffer write outside the per-step "
-                                     "CUDA-event intervals; tree + batch %.1f MiB fit in the L2)"
-                                     % ((info["inner_bytes"] + info["leaf_bytes"] + m * (2 * w + 8)) / 2**20)
-                                     if step_fits_l2(work) else
-                                     "inputs larger than L2 (queries+results %d MiB/step/GPU > %d MB L2)"
-                                     % (m * (2 * w + 8) >> 20, l2_size // 10**6)),
-                       "launch": "CUDA graph replay of the captured step" if graph is not None else "direct",
-                       "tree": {k: info[k] for k in ("height", "smem_levels", "level_nodes", "leaf_lines",
-                                                     "chain_len", "inner_bytes", "leaf_bytes", "n_distinct")}},
+            "config": bench_config(args, world),
             "e2e": e2e,
             "gpu_launches": args.steps * launches_per_step,
+            "gpu_launches_per_step": launches_per_step,
             "roofline": roof,
             "roofline_hbm": roof_hbm,
             "roofline_l2": roof_l2,
             "phases_ms": phases,
             "clocks": clocks,
             "cpu_baseline": cpu,
+            "launch": "CUDA graph replay of the captured step" if graph is not None else "direct",
+            "tree": {k: info[k] for k in ("height", "smem_levels", "level_nodes", "leaf_lines", "chain_len",
+                                          "inner_bytes", "leaf_bytes", "n_distinct")},
+            "ranks_share_gpus": d.shared_gpus,
+            "process_group": d.backend,
             "context": "paper: up to 240 M queries/s (HB+ implicit, GTX 780 + Xeon E5-2665, PAPER.md:9,57)",
         }
+        if args.config == "c4":
+            line["nvlink"] = {"a2a_gbs_measured": round(a2a_gbs, 1) if a2a_gbs else None,
+                              "a2a_bytes_per_query": round((world - 1) / world * (w + 8 + w), 2),
+                              "probe": ("NCCL all_to_all_single of 256 MiB per rank in this run, bytes leaving "
+                                        "each GPU per second" if a2a_gbs else
+                                        "not measured (one rank, or ranks sharing a GPU)")}
         if after:
             line["update"] = after
         print(json.dumps(line), flush=True)
-    if world > 1:
-        dist.destroy_process_group()
+    d.close()
+
+
+def bench_config(args, world):
+    """The workload description shared by both arms (this one and --impl reference),
+    from the configuration alone (BASELINE.json configs[], gen.CONFIGS)."""
+    c = gen.CONFIGS[args.config]
+    w = c["width"]
+    m_total = c["m"] if args.config == "c4" else c["m"] * world
+    qk = {"uniform": "uniform hits with replacement", "stratified": "uniform hits over all keys",
+          "uniform_ins": "uniform over key indices [0, n + n_ins) (misses = not-yet-inserted keys)",
+          "shuffle": "Knuth shuffle of the keys (PAPER.md:298)",
+          "zipf": f"Zipf({c.get('theta')}) over key ranks, scrambled through the key order"}[c["queries"]]
+    if args.queries:
+        qk = f"{args.queries} query values on [0, 1] mapped to [0, MAX] (PAPER.md:346-352)"
+    keys = "stratified (i << 33 | mix64 low bits), sorted" if args.config == "c4" else "mix64 / fmix32 stream"
+    if args.config == "c4":
+        par = f"key-range sharded x{world}" if world > 1 else "single GPU, whole tree (one shard)"
+    else:
+        par = f"replicated x{world}" if world > 1 else "single"
+    fits_l2 = args.config == "c1"
+    return {"workload": f"{args.config}: {c['layout']} tree, n={c['n']} keys (u{8 * w}, {keys}), fanout "
+                        f"{c['fanout']}, m={m_total} queries in total ({qk})"
+                        + (f"; range scans of {args.range_k} keys" if args.range_k else ""),
+            "n_keys": c["n"], "queries_total": m_total, "queries_per_rank": m_total // world if world else m_total,
+            "fanout": c["fanout"], "layout": c["layout"], "key_bits": 8 * w, "parallelism": par,
+            "exchange": (("fused peer-memory (CUDA IPC windows)" if not args.exchange else "NCCL send/recv")
+                         if args.config == "c4" and world > 1 else None),
+            "l2_policy": ("L2 flushed between timed steps (2x-L2 buffer write outside the per-step CUDA-event "
+                          "intervals; the tree and the batch fit in the L2)" if fits_l2 else
+                          "inputs larger than L2 (queries + results per step exceed the 126 MB L2)")}
 
 
 def _oracle_workload(cfg_name, m):
@@ -693,13 +799,55 @@ def _oracle_workload(cfg_name, m):
     return c, k, v, gen.workload_queries(cfg_name, k, m)
 
 
+C4_SLICE = 1 << 26  # keys of the contiguous c4 slice the oracle builds (2^26 of 2^31)
+
+
+def c4_oracle_sample(m):
+    """c4 for the oracle, bounded: the contiguous slice of the first 2^26 stratified keys
+    (a complete subtree of the 2^31-key tree: global rank = slice rank), and m queries
+    of the same recipe restricted to it (q = K_u, u uniform over the slice)."""
+    c = gen.CONFIGS["c4"]
+    sk = gen.stream_seed(c["cfg"], gen.STREAM_K)
+    sv = gen.stream_seed(c["cfg"], gen.STREAM_V)
+    sq = gen.stream_seed(c["cfg"], gen.STREAM_Q)
+    k = gen.stratified_keys(C4_SLICE, sk)
+    v = gen.values(C4_SLICE, 8, sv)
+    q = k[gen.uniform_indices(m, C4_SLICE, sq).astype(np.int64)]
+    return c, k, v, q
+
+
+def c4_closed_form_qps(chunk=1 << 24):
+    """SURVEY §8(c).4 pin timed as a CPU program: the stratified closed form over ALL
+    2^28 c4 queries (i = q >> 33, r = i + (q > K_i), found iff q == K_i), numpy on
+    the host, in chunks.  Query generation is outside the timed part."""
+    c = gen.CONFIGS["c4"]
+    sk = gen.stream_seed(c["cfg"], gen.STREAM_K)
+    sv = gen.stream_seed(c["cfg"], gen.STREAM_V)
+    sq = gen.stream_seed(c["cfg"], gen.STREAM_Q)
+    n, m = c["n"], c["m"]
+    el = 0.0
+    for s in range(0, m, chunk):
+        u = gen.uniform_indices(min(chunk, m - s), n, sq, start=s)
+        q = (u << np.uint64(33)) | (gen.mix64(u ^ np.uint64(sk)) & np.uint64((1 << 33) - 1))
+        t0 = time.perf_counter()
+        i = q >> np.uint64(33)
+        ki = (i << np.uint64(33)) | (gen.mix64(i ^ np.uint64(sk)) & np.uint64((1 << 33) - 1))
+        r = i + (q > ki).astype(np.uint64)
+        found = q == ki
+        val = np.where(found, gen.mix64(i ^ np.uint64(sv)), np.uint64(0))
+        pf = np.where(r < np.uint64(n), r, np.uint64(0x7FFFFFFFFFFFFFFF)) | (found.astype(np.uint64) << np.uint64(63))
+        el += time.perf_counter() - t0
+        del pf, val
+    return m / el, el
+
+
 def cpu_baseline(cfg_name, target_s=8.0):
     """The oracle as it stands, on this host's cores, over a bounded sample."""
     import oracle
     if cfg_name == "c4":
-        return {"value": None, "unit": "M queries/s", "cores": oracle.default_threads(), "kind": "oracle",
-                "sample": "not run: the 2^31-key oracle tree needs ~80 GB of host RAM and minutes to build"}
-    c, k, v, q = _oracle_workload(cfg_name, 1 << 20)
+        c, k, v, q = c4_oracle_sample(1 << 20)
+    else:
+        c, k, v, q = _oracle_workload(cfg_name, 1 << 20)
     t0 = time.perf_counter()
     tree = (oracle.ITree if c["layout"] == "implicit" else oracle.RTree).from_pairs(k, v, c["fanout"], c["width"])
     build_s = time.perf_counter() - t0
@@ -725,6 +873,7 @@ def cpu_baseline(cfg_name, target_s=8.0):
     t0 = time.perf_counter()
     oracle.lower_bound(Kd, Vd, q, nthreads=cores)
     qps_lb = len(q) / (time.perf_counter() - t0)
+    del tree
     cpu_model = ""
     try:
         for line in open("/proc/cpuinfo"):
@@ -733,21 +882,38 @@ def cpu_baseline(cfg_name, target_s=8.0):
                 break
     except OSError:
         pass
-    return {"value": round(qps / 1e6, 3), "unit": "M queries/s", "cores": cores, "kind": "oracle",
-            "sample": f"{reps} x {len(q)} queries of the same workload, oracle tree search "
-                      f"(scalar node scan, OpenMP static chunks), {el:.1f} s; oracle build {build_s:.1f} s",
-            "one_thread": round(qps1 / 1e6, 3), "lower_bound_all_threads": round(qps_lb / 1e6, 3),
-            "build_s": round(build_s, 2), "cpu_model": cpu_model, "nproc": os.cpu_count()}
+    sample = (f"{reps} x {len(q)} queries of the same workload, oracle tree search "
+              f"(scalar node scan, OpenMP static chunks), {el:.1f} s; oracle build {build_s:.1f} s")
+    out = {"value": round(qps / 1e6, 3), "unit": "M queries/s", "cores": cores, "kind": "oracle",
+           "sample": sample, "one_thread": round(qps1 / 1e6, 3), "lower_bound_all_threads": round(qps_lb / 1e6, 3),
+           "build_s": round(build_s, 2), "cpu_model": cpu_model, "nproc": os.cpu_count()}
+    if cfg_name == "c4":
+        out["sample"] = (f"c4 slice: the oracle tree built on the first {C4_SLICE} stratified keys (a complete "
+                         f"subtree of the 2^31-key tree), {reps} x {len(q)} uniform hit queries over that slice; "
+                         + sample)
+        cf_qps, cf_s = c4_closed_form_qps()
+        out["closed_form_all_queries"] = {
+            "value": round(cf_qps / 1e6, 3), "unit": "M queries/s", "seconds": round(cf_s, 2), "cores": 1,
+            "what": "SURVEY 8(c).4 stratified closed form (i = q >> 33, r = i + (q > K_i)) over all 2^28 queries, "
+                    "numpy, one thread: not a tree search, only valid for this key generator"}
+    return out
 
 
 def run_reference(args):
-    """--impl reference: the CPU oracle on this host, same config/metric/unit."""
+    """--impl reference: the CPU oracle on this host, same config/metric/unit.  c4: the
+    oracle tree of the contiguous 2^26-key slice (built once, untimed), each step a
+    2^20-query sample of the c4 recipe restricted to that slice."""
     rank, world, _ = dist_env()
     if rank != 0:
         return
     import oracle
-    cfg = args.config if args.config != "c4" else "c2"
-    c, k, v, q = _oracle_workload(cfg, 1 << 20)
+    if args.config == "c4":
+        c, k, v, q = c4_oracle_sample(1 << 20)
+        what = (f"oracle tree of the first {C4_SLICE} c4 keys (contiguous slice), {len(q)} uniform hit "
+                f"queries over that slice per step")
+    else:
+        c, k, v, q = _oracle_workload(args.config, 1 << 20)
+        what = f"{len(q)} queries of {args.config} per step"
     tree = (oracle.ITree if c["layout"] == "implicit" else oracle.RTree).from_pairs(k, v, c["fanout"], c["width"])
     cores = oracle.default_threads()
     for _ in range(max(args.warmup, 1)):
@@ -762,11 +928,11 @@ def run_reference(args):
     line = {
         "impl": "reference", "metric": "lookups/sec (M queries/s)", "value": val, "unit": "M queries/s",
         "n_gpus": world, "steps": steps, "warmup": args.warmup, "ms_per_step": round(el / steps * 1e3, 3),
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64" if c["width"] == 8 else "u32",
-        "data": "synthetic", "config": {"workload": f"{cfg} (oracle tree search on {cores} host threads, "
-                                                     f"{len(q)}-query sample per step)"},
+        "higher_is_better": True, "scaling": "strong" if args.config == "c4" else "weak", "vs_baseline": None,
+        "dtype": "u64" if c["width"] == 8 else "u32", "data": "synthetic (seeded counter-based generators, gen/)",
+        "config": bench_config(args, world),
         "cpu_baseline": {"value": val, "unit": "M queries/s", "cores": cores, "kind": "oracle",
-                         "sample": f"{len(q)} queries of {cfg} per step, {steps} steps"},
+                         "sample": f"{what}, {steps} steps, OpenMP static chunks on {cores} threads"},
         "e2e": {"value": val, "unit": "M queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -774,6 +940,9 @@ def run_reference(args):
 
 def main():
     args = parse()
+    rc = maybe_spawn(args)
+    if rc is not None:
+        sys.exit(rc)
     if args.impl == "reference":
         run_reference(args)
     else:
