@@ -290,7 +290,7 @@ def make_work(cfg_name, d, args):
         m_local = m // world
         q = g.stratified_queries(m_local, n, sq, sk, start=rank * m_local)
         if world == 1:
-            comm = hbt.Comm(1, 0, hbt.unique_id())
+            comm = hbt.Comm.single()  # no NCCL at one rank
         elif d.backend == "nccl":
             comm = hbt.Comm.from_torch()
         else:  # ranks sharing a GPU: NCCL refuses them; host all-gathers over gloo + IPC windows

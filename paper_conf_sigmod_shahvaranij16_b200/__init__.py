@@ -349,6 +349,21 @@ class Comm:
         self._h, self.nranks, self.rank = h, world, rank
         return self
 
+    @classmethod
+    def single(cls):
+        """A one-rank communicator without NCCL (the host all-gather is a copy)."""
+        self = cls.__new__(cls)
+
+        def allgather(send, recv, nbytes, ctx):
+            C.memmove(recv, send, nbytes)
+            return 0
+
+        self._fn = ALLGATHER_FN(allgather)
+        h = C.c_void_p()
+        _check(lib.hbt_comm_init_host(1, 0, self._fn, None, C.byref(h)))
+        self._h, self.nranks, self.rank = h, 1, 0
+        return self
+
     def close(self):
         if getattr(self, "_h", None) and self._h.value:
             lib.hbt_comm_destroy(self._h)

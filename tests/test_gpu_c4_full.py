@@ -53,7 +53,7 @@ def c4():
     g = GenLib()
     keys = g.stratified_keys(n, sk)
     vals = g.mix_stream(n, 8, sv)
-    comm = hbt.Comm(1, 0, hbt.unique_id())
+    comm = hbt.Comm.single()  # as bench.py at N = 1 (no NCCL)
     tree = hbt.ShardedTree(comm, keys, vals, fanout=c["fanout"])
     del keys, vals
     torch.cuda.empty_cache()
@@ -92,7 +92,8 @@ def test_c4_misses_and_edges_closed_form(c4):
     hit = (u << np.uint64(33)) | (gen.mix64(u ^ np.uint64(sk)) & LOW)
     q = np.concatenate([hit[: mq // 4] + np.uint64(1), hit[mq // 4: mq // 2] - np.uint64(1),
                         rng.integers(0, 2**64 - 1, mq // 2, dtype=np.uint64, endpoint=True),
-                        np.array([0, 1, 2**64 - 1, 2**64 - 2, (n - 1) << 33, n << 33], np.uint64)])
+                        np.array([0, 1, 2**64 - 1, 2**64 - 2, (n - 1) << 33, ((n - 1) << 33) | ((1 << 33) - 1),
+                                  (n // 2) << 33], np.uint64)])
     t = c4["tree"]
     pf, val = t.search(to_dev(q, 8))
     torch.cuda.synchronize()
