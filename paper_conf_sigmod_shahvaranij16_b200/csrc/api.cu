@@ -468,6 +468,7 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "regular_l2_hint" && value >= 0 && value <= 3) c.regular_l2_hint = uint32_t(value);
   else if (n == "item_l2_hint" && value >= 0 && value <= 3) c.item_l2_hint = uint32_t(value);
   else if (n == "full_levels" && value >= 0 && value <= 0xFFFFFFFFll) c.full_levels = uint32_t(value);
+  else if (n == "item_sched" && (value == 0 || value == 1)) c.item_sched = uint32_t(value);
   else {
     set_error("bad parameter %s = %lld", name, (long long)value);
     return HBT_EINVAL;

@@ -84,6 +84,8 @@ struct SearchConfig {
   uint32_t item_group4 = 0;      // implicit item search, 128 B nodes: 4-lane groups (one 256-bit load per lane;
                                  // measured slower: c4 item search 9.50 -> 10.8 ms, 56 B of spills)
   uint32_t regular_l2_hint = 0;  // regular bucketed item search (measured slower with 1: c3 1.59 -> 1.72 ms)
+  uint32_t item_sched = 1;       // implicit item search: 1 = strided items (all CTAs move through the
+                                 // bucketed order together), 0 = contiguous 16-round items
 };
 
 // Bucket-local directory of the bucketed search (bucketed.cu): after the
@@ -108,6 +110,11 @@ struct ItemDir {
   uint64_t pos_base = 0;  // implicit: added to every reported position (key-range shards)
   uint32_t qprefetch = 0; // bulk L2 prefetch of the current / next item's queries
   uint32_t rounds = 16;   // warp rounds per work item (fewer for small batches: every SM gets items)
+  // strided schedule (implicit item search, "item_sched" = 1): item (CTA j, s) is rounds
+  // s*R .. s*R+R-1 of CTA j, round g's queries being [(g*grid + j)*T, +T), so all CTAs
+  // work through the bucketed order together (implicit_search.cu)
+  uint32_t strided = 0;
+  uint32_t pbits = 10;    // prefix-table bits of the staged directory (<= 12)
 };
 
 // Query-bucketing state (bucketed.cu): B splitter keys and a prefix directory,

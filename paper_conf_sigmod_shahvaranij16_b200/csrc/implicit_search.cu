@@ -540,6 +540,7 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
 // reaches (every level picks the first child whose subtree max is >= q,
 // DESIGN.md R1/R3).  The rest of the walk is descend_and_store from that level.
 constexpr int kItemRounds = 16;
+constexpr uint32_t kStridedPrefixBits = 12;  // strided items stage ~4x more maxima
 
 // Cooperative copy of cnt keys into shared memory, four loads in flight per thread.
 template <typename K>
@@ -574,9 +575,22 @@ implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* _
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int g = lane / C::G, k = lane % C::G;
   const unsigned gmask = ((1u << C::G) - 1u) << (g * C::G);
-  const uint64_t items = (m + W - 1) / W;
-  for (uint64_t it = blockIdx.x; it < items; it += gridDim.x) {
-    const uint64_t p0 = it * W, p1 = (p0 + W < m ? p0 + W : m) - 1;
+  // strided: superstep x covers queries [x * SW, (x + 1) * SW), CTA j takes its slice
+  // [(x * grid + j) * THREADS, + THREADS); item s of CTA j = supersteps [s R, s R + R)
+  const uint64_t SW = uint64_t(gridDim.x) * THREADS;
+  const uint64_t steps = (m + SW - 1) / SW;
+  const uint64_t items = d.strided ? (steps + d.rounds - 1) / d.rounds : (m + W - 1) / W;
+  for (uint64_t it = d.strided ? 0 : blockIdx.x; it < items; it += d.strided ? 1 : gridDim.x) {
+    uint64_t p0, p1;
+    if (d.strided) {
+      p0 = (it * d.rounds * gridDim.x + blockIdx.x) * uint64_t(THREADS);
+      if (p0 >= m) break;
+      const uint64_t xl = std::min<uint64_t>((it + 1) * d.rounds, steps) - 1;
+      p1 = std::min<uint64_t>(m, (xl * gridDim.x + blockIdx.x + 1) * uint64_t(THREADS)) - 1;
+    } else {
+      p0 = it * W;
+      p1 = (p0 + W < m ? p0 + W : m) - 1;
+    }
     if (threadIdx.x < 2) {
       const uint64_t p = threadIdx.x ? p1 : p0;
       uint32_t lo = 0, hi = d.B;  // largest b with bstart[b] <= p
@@ -599,23 +613,27 @@ implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* _
     if (in_smem) stage_keys(s_M, gM + u0, cnt, THREADS);
     __syncthreads();
     PrefixTab<K> pt{};
-    if (in_smem) pt = build_prefix(s_M, cnt, s_T, THREADS);
+    if (in_smem) pt = build_prefix(s_M, cnt, s_T, THREADS, d.pbits);
     __syncthreads();
     const K* M = in_smem ? s_M : gM + u0;
+    // consecutive rounds of a warp: THREADS queries apart (contiguous items) or one
+    // superstep apart (strided items)
+    const uint64_t rstride = d.strided ? SW : uint64_t(THREADS);
+    const uint64_t lim = d.strided ? m - 1 : p1;  // last valid query index
     // the next round's queries are loaded while this round walks the tree
     K nextq;
     {
       const uint64_t i = p0 + uint64_t(wid) * 32 + lane;
-      nextq = i <= p1 ? ldcs(queries + i) : key_max<K>();
+      nextq = i <= lim ? ldcs(queries + i) : key_max<K>();
     }
 #pragma unroll 1
     for (int r = 0; r < int(d.rounds); ++r) {
-      const uint64_t base = p0 + (uint64_t(r) * (THREADS / 32) + wid) * 32;
-      if (base > p1) break;
+      const uint64_t base = p0 + uint64_t(r) * rstride + uint64_t(wid) * 32;
+      if (base > lim) break;
       const K myq = nextq;
       {
-        const uint64_t i = base + (THREADS / 32) * 32 + lane;
-        nextq = (r + 1 < int(d.rounds) && i <= p1) ? ldcs(queries + i) : key_max<K>();
+        const uint64_t i = base + rstride + lane;
+        nextq = (r + 1 < int(d.rounds) && i <= lim) ? ldcs(queries + i) : key_max<K>();
       }
       const uint32_t lo = in_smem ? prefix_lower_bound(s_M, cnt, s_T, pt, myq) : lb_range(M, 0, cnt, myq);
       const uint32_t mynode = uint32_t(u0) + (lo < cnt ? lo : cnt - 1);
@@ -629,7 +647,7 @@ implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* _
         sec0[j] = 0;
       }
       descend_and_store<K, F, QPG, true, GM>(inner, inner_idx, leaf, lt, d.level, false, q, node, sec0, g, k, gmask,
-                                         base, p1 + 1, n, d.pos_base, out_pf, out_v);
+                                         base, lim + 1, n, d.pos_base, out_pf, out_v);
     }
     __syncthreads();
   }
@@ -777,7 +795,7 @@ struct Launch {
         if (C::HAS_IDX && cum > budget && x < 32) lt.full_mask |= 1u << x;
       }
     }
-    const size_t smem = (d.B + 1) * 8 + size_t(d.cap) * C::S + ((1u << kPrefixBits) + 1) * 4;
+    const size_t smem = (d.B + 1) * 8 + size_t(d.cap) * C::S + ((1u << kStridedPrefixBits) + 1) * 4;
     static bool attr_set[2] = {false, false};  // per kernel variant
     const int av = kern == implicit_search_items_kernel<K, F, TH> ? 0 : 1;
     if (!attr_set[av]) {
@@ -785,10 +803,23 @@ struct Launch {
       attr_set[av] = true;
     }
     ItemDir dd = d;
-    dd.rounds = item_rounds(m, t->num_sms, TH, t->cfg.item_rounds ? t->cfg.item_rounds : 16);
     uint64_t grid = t->num_sms;
-    const uint64_t items = (m + uint64_t(TH) * dd.rounds - 1) / (uint64_t(TH) * dd.rounds);
-    if (items < grid) grid = items ? items : 1;
+    if (d.strided && m >= uint64_t(t->num_sms) * TH * 2) {
+      // strided items: R rounds per item such that the item's unit range (R supersteps of
+      // grid * TH queries, uniform keys assumed; wider items fall back to the global
+      // directory) fits the staging capacity
+      const double per_step = double(uint64_t(t->num_sms) * TH) / double(m) * double(d.nunits);
+      const double edge = 2.0 * double(d.nunits) / double(d.B);  // whole buckets at both ends
+      const uint32_t R = double(d.cap) > edge ? uint32_t((double(d.cap) - edge) / (per_step * 1.15)) : 1u;
+      const uint32_t rmax = t->cfg.item_rounds ? t->cfg.item_rounds : 16;
+      dd.rounds = std::max<uint32_t>(1, std::min<uint32_t>(R, rmax));
+      dd.pbits = kStridedPrefixBits;
+    } else {
+      dd.strided = 0;
+      dd.rounds = item_rounds(m, t->num_sms, TH, t->cfg.item_rounds ? t->cfg.item_rounds : 16);
+      const uint64_t items = (m + uint64_t(TH) * dd.rounds - 1) / (uint64_t(TH) * dd.rounds);
+      if (items < grid) grid = items ? items : 1;
+    }
     kern<<<unsigned(grid), TH, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
                                           (const uint8_t*)t->d_leaf, dd, (const K*)q, m, pf, (K*)v, lt, t->n);
     HBT_CUDA_TRY(cudaGetLastError());

@@ -53,19 +53,20 @@ struct PrefixTab {
   uint32_t sh;
 };
 
-// Builds s_T[p] = #{s_M < lo + p * 2^sh} for p in [0, 2^kPrefixBits] (cnt past
-// the range); (span >> sh) < 2^kPrefixBits.  Caller synchronises before use.
+// Builds s_T[p] = #{s_M < lo + p * 2^sh} for p in [0, 2^PB] (cnt past the range; PB <= 12);
+// (span >> sh) < 2^PB.  Caller synchronises before use.
 template <typename K>
-__device__ __forceinline__ PrefixTab<K> build_prefix(const K* s_M, uint32_t cnt, uint32_t* s_T, uint32_t threads) {
+__device__ __forceinline__ PrefixTab<K> build_prefix(const K* s_M, uint32_t cnt, uint32_t* s_T, uint32_t threads,
+                                                     uint32_t PB = kPrefixBits) {
   PrefixTab<K> pt;
   pt.lo = s_M[0];
   pt.span = K(s_M[cnt - 1] - pt.lo);
   const uint32_t bits = pt.span ? uint32_t(8 * sizeof(K)) - uint32_t(sizeof(K) == 8 ? __clzll((long long)pt.span)
                                                                                     : __clz(int(pt.span)))
                                 : 0u;
-  pt.sh = bits > kPrefixBits ? bits - kPrefixBits : 0u;
+  pt.sh = bits > PB ? bits - PB : 0u;
   const K pmax = K(pt.span >> pt.sh);
-  for (uint32_t p = threadIdx.x; p <= (1u << kPrefixBits); p += threads)
+  for (uint32_t p = threadIdx.x; p <= (1u << PB); p += threads)
     s_T[p] = K(p) > pmax ? cnt : lb_range(s_M, 0, cnt, K(pt.lo + (K(p) << pt.sh)));
   return pt;
 }
