@@ -84,7 +84,7 @@ struct SearchConfig {
   uint32_t item_group4 = 0;      // implicit item search, 128 B nodes: 4-lane groups (one 256-bit load per lane;
                                  // measured slower: c4 item search 9.50 -> 10.8 ms, 56 B of spills)
   uint32_t regular_l2_hint = 0;  // regular bucketed item search (measured slower with 1: c3 1.59 -> 1.72 ms)
-  uint32_t item_sched = 1;       // implicit item search: 1 = strided items (all CTAs move through the
+  uint32_t item_sched = 0;       // implicit item search: 1 = strided items (all CTAs move through the
                                  // bucketed order together), 0 = contiguous 16-round items
 };
 

@@ -795,7 +795,6 @@ struct Launch {
         if (C::HAS_IDX && cum > budget && x < 32) lt.full_mask |= 1u << x;
       }
     }
-    const size_t smem = (d.B + 1) * 8 + size_t(d.cap) * C::S + ((1u << kStridedPrefixBits) + 1) * 4;
     static bool attr_set[2] = {false, false};  // per kernel variant
     const int av = kern == implicit_search_items_kernel<K, F, TH> ? 0 : 1;
     if (!attr_set[av]) {
@@ -808,18 +807,24 @@ struct Launch {
       // strided items: R rounds per item such that the item's unit range (R supersteps of
       // grid * TH queries, uniform keys assumed; wider items fall back to the global
       // directory) fits the staging capacity
+      // the larger prefix table comes out of the staging capacity, so the CTA's shared
+      // memory (and with it the L1 carve-out: 9.5 vs 10.9 ms on c4 when it grew) stays
+      // that of the contiguous items
+      dd.pbits = kStridedPrefixBits;
+      const uint32_t extra = (((1u << kStridedPrefixBits) - (1u << kPrefixBits)) * 4 + C::S - 1) / C::S;
+      if (dd.cap > extra + 64) dd.cap -= extra;
       const double per_step = double(uint64_t(t->num_sms) * TH) / double(m) * double(d.nunits);
       const double edge = 2.0 * double(d.nunits) / double(d.B);  // whole buckets at both ends
-      const uint32_t R = double(d.cap) > edge ? uint32_t((double(d.cap) - edge) / (per_step * 1.15)) : 1u;
+      const uint32_t R = double(dd.cap) > edge ? uint32_t((double(dd.cap) - edge) / (per_step * 1.15)) : 1u;
       const uint32_t rmax = t->cfg.item_rounds ? t->cfg.item_rounds : 16;
       dd.rounds = std::max<uint32_t>(1, std::min<uint32_t>(R, rmax));
-      dd.pbits = kStridedPrefixBits;
     } else {
       dd.strided = 0;
       dd.rounds = item_rounds(m, t->num_sms, TH, t->cfg.item_rounds ? t->cfg.item_rounds : 16);
       const uint64_t items = (m + uint64_t(TH) * dd.rounds - 1) / (uint64_t(TH) * dd.rounds);
       if (items < grid) grid = items ? items : 1;
     }
+    const size_t smem = (d.B + 1) * 8 + size_t(dd.cap) * C::S + ((1u << dd.pbits) + 1) * 4;
     kern<<<unsigned(grid), TH, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
                                           (const uint8_t*)t->d_leaf, dd, (const K*)q, m, pf, (K*)v, lt, t->n);
     HBT_CUDA_TRY(cudaGetLastError());
