@@ -315,6 +315,32 @@ HBT_API int hbt_shard_local_init(hbt_tree* const* shards, int G);
 HBT_API int hbt_search_sharded_local(hbt_tree* const* shards, int G, const void* const* queries,
                                      const uint64_t* m, const hbt_out* outs, void* stream);
 
+/* ---- versioned trees: searches concurrent with bulk updates (
+ * the paper's concurrent search/update queries, App. B.3, and its batch
+ * update, §5.6) ----
+ * A versioned handle owns a sequence of immutable tree versions 0, 1, 2, ...
+ * hbt_versioned_search reads the version that is current when it is called (its number
+ * goes to *version, may be NULL), asynchronously on `stream`, exactly like hbt_search.
+ * hbt_versioned_update derives version k+1 from the current version k on `stream`
+ * (IMPLICIT: merge + rebuild into fresh arrays; REGULAR: a device copy of
+ * version k, then the in-place batch update of hbt_bulk_update), host-synchronously,
+ * while searches on OTHER streams and threads keep reading version k; then publishes
+ * k+1 (*version).  Updates are serialised; searches never block on one.  A replaced
+ * version is freed once no call is inside it and every search launched on it has
+ * completed (CUDA events), so device memory peaks at two versions during an update.
+ * Error: the current version is unchanged.  Not for key-range shards or trees whose
+ * L-segment is in host memory (HBT_EUNSUPPORTED). */
+typedef struct hbt_versioned hbt_versioned;
+/* Takes ownership of t (it becomes version 0; do not hbt_destroy it). */
+HBT_API int hbt_versioned_create(hbt_tree* t, hbt_versioned** out);
+HBT_API int hbt_versioned_search(hbt_versioned* v, const void* queries, uint64_t m, hbt_out out, void* stream,
+                                 uint64_t* version);
+HBT_API int hbt_versioned_update(hbt_versioned* v, const hbt_batch* batch, void* stream, uint64_t* version);
+/* The current version's tree (borrowed: valid until the next update retires it; for
+ * hbt_info / hbt_export / hbt_set_param on the current version). */
+HBT_API int hbt_versioned_current(hbt_versioned* v, hbt_tree** t, uint64_t* version);
+HBT_API int hbt_versioned_destroy(hbt_versioned* v);
+
 HBT_API const char* hbt_last_error(void);
 /* Library version string, e.g. "hbt 0.1 sm_100a". */
 HBT_API const char* hbt_version(void);

@@ -38,7 +38,8 @@ EXPORTED = ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update"
             "hbt_info", "hbt_export", "hbt_set_param", "hbt_last_error", "hbt_version",
             "hbt_range", "hbt_comm_unique_id", "hbt_comm_init", "hbt_comm_init_host", "hbt_comm_destroy", "hbt_bulk_build_sharded",
             "hbt_search_sharded", "hbt_shard_local_init", "hbt_search_sharded_local", "hbt_last_phases",
-            "hbt_set_leaf_placement", "hbt_get_leaf_placement"]
+            "hbt_set_leaf_placement", "hbt_get_leaf_placement", "hbt_versioned_create", "hbt_versioned_search",
+            "hbt_versioned_update", "hbt_versioned_current", "hbt_versioned_destroy"]
 
 
 class HBTError(RuntimeError):
@@ -97,6 +98,11 @@ def _load():
     L.hbt_last_phases.argtypes = [vp, vp]
     L.hbt_set_leaf_placement.argtypes = [vp, u32]
     L.hbt_get_leaf_placement.argtypes = [vp, C.POINTER(u32)]
+    L.hbt_versioned_create.argtypes = [vp, C.POINTER(vp)]
+    L.hbt_versioned_search.argtypes = [vp, vp, u64, _Out, vp, C.POINTER(u64)]
+    L.hbt_versioned_update.argtypes = [vp, C.POINTER(_Batch), vp, C.POINTER(u64)]
+    L.hbt_versioned_current.argtypes = [vp, C.POINTER(vp), C.POINTER(u64)]
+    L.hbt_versioned_destroy.argtypes = [vp]
     L.hbt_last_error.restype = C.c_char_p
     L.hbt_version.restype = C.c_char_p
     for f in ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
@@ -104,7 +110,8 @@ def _load():
               "hbt_comm_init_host",
               "hbt_comm_destroy", "hbt_bulk_build_sharded", "hbt_search_sharded", "hbt_shard_local_init",
               "hbt_search_sharded_local", "hbt_last_phases", "hbt_set_leaf_placement",
-              "hbt_get_leaf_placement"]:
+              "hbt_get_leaf_placement", "hbt_versioned_create", "hbt_versioned_search", "hbt_versioned_update",
+              "hbt_versioned_current", "hbt_versioned_destroy"]:
         getattr(L, f).restype = C.c_int
     return L
 
@@ -284,6 +291,59 @@ class Tree:
                 self.set_param(k, v)
 
 
+class VersionedTree:
+    """Searches concurrent with bulk updates (hbt_versioned_*): every search reads the
+    version current at its call; update() derives and publishes the next version
+    while searches on other streams keep reading the previous one."""
+
+    def __init__(self, tree: Tree):
+        h = C.c_void_p()
+        _check(lib.hbt_versioned_create(tree._h, C.byref(h)))
+        tree._h = C.c_void_p()  # owned by the versioned handle now
+        self._h, self.width, self._torch = h, tree.width, tree._torch
+
+    def search(self, queries, out_pos=None, out_vals=None, stream=None):
+        """Returns (pos_found, values, version)."""
+        torch = self._torch
+        queries = queries.contiguous()
+        m = queries.numel()
+        if out_pos is None:
+            out_pos = torch.empty(m, dtype=torch.int64, device=queries.device)
+        if out_vals is None:
+            out_vals = torch.empty(m, dtype=_dtype(self.width), device=queries.device)
+        ver = C.c_uint64(0)
+        if m:
+            _check(lib.hbt_versioned_search(self._h, C.c_void_p(queries.data_ptr()), m,
+                                            _Out(out_pos.data_ptr(), out_vals.data_ptr()), _stream_ptr(stream),
+                                            C.byref(ver)))
+        return out_pos, out_vals, ver.value
+
+    def update(self, keys, values, ops, stream=None) -> int:
+        keys, values, ops = keys.contiguous(), values.contiguous(), ops.contiguous()
+        b = _Batch(keys.data_ptr() if keys.numel() else 0, values.data_ptr() if values.numel() else 0,
+                   ops.data_ptr() if ops.numel() else 0, keys.numel())
+        ver = C.c_uint64(0)
+        _check(lib.hbt_versioned_update(self._h, C.byref(b), _stream_ptr(stream), C.byref(ver)))
+        return ver.value
+
+    @property
+    def version(self) -> int:
+        t, ver = C.c_void_p(), C.c_uint64(0)
+        _check(lib.hbt_versioned_current(self._h, C.byref(t), C.byref(ver)))
+        return ver.value
+
+    def close(self):
+        if getattr(self, "_h", None) and self._h.value:
+            lib.hbt_versioned_destroy(self._h)
+            self._h = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
 # ---------------------------------------------------------------- sharding
 
 
@@ -390,6 +450,10 @@ class ShardedTree(Tree):
                                           C.c_void_p(values.data_ptr() if values.numel() else 0), keys.numel(),
                                           fanout, word, _stream_ptr(stream), C.byref(h)))
         self._h = h
+
+    def update(self, keys, values, ops, stream=None):
+        raise HBTError(EUNSUPPORTED, "bulk update of a key-range shard is not supported "
+                                     "(rebuild the sharded tree)")
 
     def search(self, queries, out_pos=None, out_vals=None, stream=None):
         torch = self._torch

@@ -167,7 +167,7 @@ int leaf_place(hbt_tree* t, uint32_t where) {
   return HBT_OK;
 }
 
-static void free_tree(hbt_tree* t) {
+void free_tree(hbt_tree* t) {
   if (!t) return;
   cudaFree(t->d_inner);  // also holds d_inner_idx
   cudaFree(t->d_dir);
@@ -189,7 +189,14 @@ static void free_tree(hbt_tree* t) {
   delete t;
 }
 
-static int device_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
+// Mark the bucket states stale (re-derived by the next bucketed search, bucketed.cu).
+void invalidate_buckets(hbt_tree* t) {
+  std::lock_guard<std::mutex> lock(t->bk_mu);
+  t->bk.valid = false;
+  t->bks.valid = false;
+}
+
+int device_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
   if (t->h_leaf && leaf_stream_enabled(t, m)) return streamed_search(t, q, m, pf, v, 0, s);
   if (bucketed_enabled(t, m)) return bucketed_search(t, q, m, pf, v, 0, s);
   return t->form == HBT_REGULAR ? regular_search(t, q, m, pf, v, s) : implicit_search(t, q, m, pf, v, s);
@@ -330,9 +337,14 @@ int hbt_bulk_update(hbt_tree* t, const hbt_batch* batch, void* stream) {
     set_error("batch arrays must be device pointers");
     return HBT_EINVAL;
   }
+  if (t->shard.G >= 1) {
+    // a shard's (n', base, max) are part of every rank's routing table: a local update
+    // would leave the other ranks routing by stale maxima and bases
+    set_error("bulk update of a key-range shard is not supported (rebuild the sharded tree)");
+    return HBT_EUNSUPPORTED;
+  }
   cudaStream_t s = (cudaStream_t)stream;
-  t->bk.valid = false;  // bucket splitters follow the tree
-  t->bks.valid = false;
+  invalidate_buckets(t);  // bucket splitters follow the tree
   return t->form == HBT_REGULAR ? regular_update(t, batch, s) : implicit_update(t, batch, s);
 }
 
@@ -447,15 +459,15 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "exchange" && (value == 0 || value == 1)) c.exchange = uint32_t(value);
   else if (n == "g1_direct" && (value == 0 || value == 1)) c.g1_direct = uint32_t(value);
   else if (n == "bucket" && value >= 0 && value <= 2) c.bucket = uint32_t(value);
-  else if (n == "bucket_slice" && value >= 0) { c.bucket_slice = uint64_t(value); t->bk.valid = false; }
-  else if (n == "bucket_items" && (value == 0 || value == 1)) { c.bucket_items = uint32_t(value); t->bk.valid = false; }
-  else if (n == "bucket_cap" && value >= 0 && value < (1 << 20)) { c.bucket_cap = uint32_t(value); t->bk.valid = false; }
+  else if (n == "bucket_slice" && value >= 0) { c.bucket_slice = uint64_t(value); invalidate_buckets(t); }
+  else if (n == "bucket_items" && (value == 0 || value == 1)) { c.bucket_items = uint32_t(value); invalidate_buckets(t); }
+  else if (n == "bucket_cap" && value >= 0 && value < (1 << 20)) { c.bucket_cap = uint32_t(value); invalidate_buckets(t); }
   else if (n == "leaf_stream" && value >= 0 && value <= 2) c.leaf_stream = uint32_t(value);
   else if (n == "qprefetch" && (value == 0 || value == 1)) c.qprefetch = uint32_t(value);
   else if (n == "item_rounds" && value >= 0 && value <= 64) c.item_rounds = uint32_t(value);
   else if (n == "host_chunk_log2" && value >= 12 && value <= 26) c.host_chunk_log2 = uint32_t(value);
   else if (n == "host_bufs" && value >= 2 && value <= kHostBufs) c.host_bufs = uint32_t(value);
-  else if (n == "stream_slice" && value >= 0) { c.stream_slice = uint64_t(value); t->bks.valid = false; }
+  else if (n == "stream_slice" && value >= 0) { c.stream_slice = uint64_t(value); invalidate_buckets(t); }
   else if (n == "phase_timing" && (value == 0 || value == 1)) c.phase_timing = uint32_t(value);
   else if (n == "leaf256" && (value == 0 || value == 1)) c.leaf256 = uint32_t(value);
   else if (n == "sec256" && (value == 0 || value == 1)) c.sec256 = uint32_t(value);

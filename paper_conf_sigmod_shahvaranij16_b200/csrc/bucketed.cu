@@ -649,9 +649,19 @@ uint64_t item_cap(const hbt_tree* t, uint32_t B) {
   return budget / per;
 }
 
+// Splitters, prefix directory and item-directory maxima of one bucket state, derived
+// from the tree on first use and after every update / bucketing knob change.  The
+// arrays are shared by every search on the tree, so preparation is serialised
+// (t->bk_mu) and completes on the HOST before it is marked valid: a search on another
+// stream can never read half-written splitters.  A re-preparation rewrites the arrays
+// in place, so it first waits for the device to drain (searches in flight on other
+// streams may still read the old ones).
 template <typename K>
 int prepare_splitters(const hbt_tree* t, cudaStream_t s, BucketState& bs, uint32_t B, bool want_items) {
+  std::lock_guard<std::mutex> lock(t->bk_mu);
   if (bs.valid && bs.B == B) return HBT_OK;
+  bs.valid = false;
+  if (bs.d_sp) HBT_CUDA_TRY(cudaDeviceSynchronize());
   if (!bs.d_sp) {
     HBT_CUDA_TRY(cudaMalloc(&bs.d_sp, kMaxBuckets * 8));
     HBT_CUDA_TRY(cudaMalloc(&bs.d_dir, (1u << kDirBits) * 4));
@@ -713,6 +723,7 @@ int prepare_splitters(const hbt_tree* t, cudaStream_t s, BucketState& bs, uint32
       HBT_CUDA_TRY(cudaGetLastError());
     }
   }
+  HBT_CUDA_TRY(cudaStreamSynchronize(s));
   bs.B = B;
   bs.valid = true;
   return HBT_OK;

@@ -271,16 +271,15 @@ struct hbt_tree {
   hbt::ShardMeta shard;
   hbt::Scratch shard_scratch;
   void* fused = nullptr;  // sharded_fused.cu state (peer windows)
-  // range-scan scratch (lower bounds of the range starts)
-  uint64_t* d_rpf = nullptr;
-  void* d_rv = nullptr;
-  uint64_t rcap = 0;
   // ---- search ----
   hbt::SearchConfig cfg;
   mutable hbt::HostPipe pipe;
   mutable hbt::BucketState bk;
   mutable hbt::BucketState bks;  // streamed host L-segment (own bucket count)
   mutable std::mutex stream_mu;   // one user of the streamed staging slots at a time
+  // serialises (re)preparation of the bucket splitters / item directory (bucketed.cu):
+  // preparation completes on the host before any search may use them
+  mutable std::mutex bk_mu;
 };
 
 namespace hbt {
@@ -292,6 +291,15 @@ int implicit_build_sorted(hbt_tree* t, const void* sk, const void* sv, uint64_t 
 int sort_dedupe(uint32_t width, const void* keys, const void* values, uint64_t n, void** out_k,
                 void** out_v, uint64_t* nd, cudaStream_t s);
 int implicit_update(hbt_tree* t, const hbt_batch* b, cudaStream_t s);
+// merge t's pairs with the batch and build the result into the empty tree nt (t unchanged)
+int implicit_merge_rebuild(const hbt_tree* t, const hbt_batch* b, hbt_tree* nt, cudaStream_t s);
+// api.cu: the search dispatch of hbt_search (streamed / bucketed / plain), tree teardown,
+// bucket-state invalidation
+int device_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s);
+void free_tree(hbt_tree* t);
+void invalidate_buckets(hbt_tree* t);
+// regular.cu: deep copy of a regular tree's device state into the empty tree dst
+int regular_clone(const hbt_tree* src, hbt_tree* dst, cudaStream_t s);
 // implicit_search.cu
 int implicit_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s);
 // same, reporting global positions base + rank (sharded trees)

@@ -369,8 +369,12 @@ int build_sorted_t(hbt_tree* t, const K* kd, const K* vd, uint64_t nd, cudaStrea
   return HBT_OK;
 }
 
+// Merge the batch into t's sorted pairs (read from its L-segment) and build the result
+// into the EMPTY tree `nt` (form / width / F / device set by the caller); t is not
+// modified.  hbt_bulk_update swaps nt into t; a versioned tree keeps t as the version
+// that searches still read (versioned.cu).
 template <typename K>
-int implicit_update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
+int implicit_merge_rebuild_t(const hbt_tree* t, const hbt_batch* b, hbt_tree* nt, cudaStream_t s) {
   const uint64_t nb = t->n, m = b->count, total = nb + m;
   if (total >= (1ull << 32)) { set_error("update: n + batch must be < 2^32"); return HBT_EUNSUPPORTED; }
   K *ck = nullptr, *sk = nullptr, *base_v = nullptr, *mv = nullptr, *kd = nullptr, *vd = nullptr;
@@ -425,15 +429,22 @@ int implicit_update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   TRY(cudaMemcpyAsync(&h_nsel, d_nsel, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
   TRY(cudaStreamSynchronize(s));
 #undef TRY
-  // Rebuild into a fresh layout, then swap it in.
-  hbt_tree nt;
-  nt.form = t->form; nt.width = t->width; nt.F = t->F; nt.device = t->device; nt.num_sms = t->num_sms;
-  int rc = build_sorted_t<K>(&nt, kd, vd, uint64_t(h_nsel), s);
+  // Rebuild into a fresh layout.
+  int rc = build_sorted_t<K>(nt, kd, vd, uint64_t(h_nsel), s);
   cleanup();
   if (rc != HBT_OK) {
-    cudaFree(nt.d_leaf); cudaFree(nt.d_inner); cudaFree(nt.d_dir); cudaFree(nt.d_sdir); cudaFree(nt.d_sdir_full);
-    return rc;
+    cudaFree(nt->d_leaf); cudaFree(nt->d_inner); cudaFree(nt->d_dir); cudaFree(nt->d_sdir); cudaFree(nt->d_sdir_full);
+    nt->d_leaf = nt->d_inner = nt->d_inner_idx = nt->d_dir = nt->d_sdir = nt->d_sdir_full = nullptr;
   }
+  return rc;
+}
+
+template <typename K>
+int implicit_update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
+  hbt_tree nt;
+  nt.form = t->form; nt.width = t->width; nt.F = t->F; nt.device = t->device; nt.num_sms = t->num_sms;
+  int rc = implicit_merge_rebuild_t<K>(t, b, &nt, s);
+  if (rc != HBT_OK) return rc;
   const uint32_t where = t->leaf_where;
   leaf_free(t);
   cudaFree(t->d_inner);  // also holds the derived index
@@ -490,6 +501,10 @@ int implicit_build(hbt_tree* t, const void* keys, const void* values, uint64_t n
 
 int implicit_update(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   return t->width == 4 ? implicit_update_t<uint32_t>(t, b, s) : implicit_update_t<uint64_t>(t, b, s);
+}
+
+int implicit_merge_rebuild(const hbt_tree* t, const hbt_batch* b, hbt_tree* nt, cudaStream_t s) {
+  return t->width == 4 ? implicit_merge_rebuild_t<uint32_t>(t, b, nt, s) : implicit_merge_rebuild_t<uint64_t>(t, b, nt, s);
 }
 
 }  // namespace hbt

@@ -132,48 +132,45 @@ inline unsigned warps_grid(uint64_t m, uint32_t L) {
 template <typename K>
 int range_t(hbt_tree* t, const void* lo, const void* hi, uint64_t m, uint32_t k, void* ok, void* ov, uint32_t* oc,
             cudaStream_t s) {
-  if (m > t->rcap) {
-    cudaFree(t->d_rpf);
-    cudaFree(t->d_rv);
-    t->d_rpf = nullptr;
-    t->d_rv = nullptr;
-    t->rcap = 0;
-    HBT_CUDA_TRY(cudaMalloc(&t->d_rpf, m * 8));
-    HBT_CUDA_TRY(cudaMalloc(&t->d_rv, m * sizeof(K)));
-    t->rcap = m;
+  // lower bounds of the range starts in per-call scratch from the stream-ordered pool:
+  // concurrent range scans on other streams each get their own
+  void* buf = nullptr;
+  const uint64_t off_v = (m * 8 + 255) & ~uint64_t(255);
+  HBT_CUDA_TRY(scratch_alloc(&buf, off_v + m * sizeof(K), s));
+  uint64_t* rpf = static_cast<uint64_t*>(buf);
+  K* rv = reinterpret_cast<K*>(static_cast<uint8_t*>(buf) + off_v);
+  int rc = t->form == HBT_REGULAR ? regular_search(t, lo, m, rpf, rv, s) : implicit_search(t, lo, m, rpf, rv, s);
+  if (rc) {
+    scratch_free(buf, s);
+    return rc;
   }
-  int rc = t->form == HBT_REGULAR ? regular_search(t, lo, m, t->d_rpf, t->d_rv, s)
-                                  : implicit_search(t, lo, m, t->d_rpf, t->d_rv, s);
-  if (rc) return rc;
   uint32_t L = 1;
   while (L < k && L < 32) L <<= 1;
   if (t->form == HBT_REGULAR) {
     const RegularState& r = t->r;
     range_regular<K><<<warps_grid(m, L), 256, 0, s>>>((const K*)r.d_leaf, r.d_count, r.d_chain, r.d_chainpos,
-                                                      r.nchain, t->F, t->d_rpf, (const K*)hi, m, k, L, (K*)ok,
+                                                      r.nchain, t->F, rpf, (const K*)hi, m, k, L, (K*)ok,
                                                       (K*)ov, oc);
   } else {
-    range_implicit<K><<<warps_grid(m, L), 256, 0, s>>>((const K*)t->d_leaf, t->n, t->d_rpf, (const K*)hi, m, k, L,
+    range_implicit<K><<<warps_grid(m, L), 256, 0, s>>>((const K*)t->d_leaf, t->n, rpf, (const K*)hi, m, k, L,
                                                        (K*)ok, (K*)ov, oc);
   }
-  HBT_CUDA_TRY(cudaGetLastError());
+  const cudaError_t e = cudaGetLastError();
+  scratch_free(buf, s);
+  if (e != cudaSuccess) {
+    set_error("range scan launch: %s", cudaGetErrorString(e));
+    return HBT_ECUDA;
+  }
   return HBT_OK;
 }
 
 }  // namespace
 
-void range_free(hbt_tree* t) {
-  cudaFree(t->d_rpf);
-  cudaFree(t->d_rv);
-  t->d_rpf = nullptr;
-  t->d_rv = nullptr;
-  t->rcap = 0;
-}
+void range_free(hbt_tree*) {}
 
 int range_scan(const hbt_tree* tc, const void* lo, const void* hi, uint64_t m, uint32_t k, void* ok, void* ov,
                uint32_t* oc, cudaStream_t s) {
   hbt_tree* t = const_cast<hbt_tree*>(tc);
-  std::lock_guard<std::mutex> lock(t->pipe.mu);
   return t->width == 4 ? range_t<uint32_t>(t, lo, hi, m, k, ok, ov, oc, s) : range_t<uint64_t>(t, lo, hi, m, k, ok, ov, oc, s);
 }
 

@@ -1069,9 +1069,65 @@ int grow_pool(hbt_tree* t, uint64_t need, cudaStream_t s) {
   return HBT_OK;
 }
 
-// Regroup every upper level from the chain (reading R11).
+// Upper-level node count for a chain of c big leaves (levels bottom-up).
+inline uint64_t upper_nodes_for(uint64_t c, uint32_t F) {
+  uint64_t total = 0;
+  while (c > 1) {
+    c = ceil_div_u64(c, F);
+    total += c;
+  }
+  return total;
+}
+
+// Before an update mutates anything: grow every array the update and the rebuild after
+// it may need (big-leaf pool, upper levels, chain positions), copying the live contents,
+// so that an allocation failure leaves the tree unchanged (hbt.h error contract).
 template <typename K>
-int rebuild_upper(hbt_tree* t, cudaStream_t s) {
+int reserve_for_update(hbt_tree* t, uint64_t pool_need, uint64_t nchain_bound, cudaStream_t s) {
+  RegularState& r = t->r;
+  const uint32_t F = t->F;
+  int rc = grow_pool<K>(t, pool_need, s);
+  if (rc != HBT_OK) return rc;
+  const uint64_t total = upper_nodes_for(nchain_bound, F);
+  if (total > r.ucap) {
+    const uint64_t cap = total + total / 4 + 16;
+    void *uk = nullptr, *ui = nullptr;
+    uint32_t* ur = nullptr;
+    auto undo = [&]() { cudaFree(uk); cudaFree(ui); cudaFree(ur); };
+    if (cudaMalloc(&uk, cap * F * sizeof(K)) != cudaSuccess || cudaMalloc(&ui, cap * 32) != cudaSuccess ||
+        cudaMalloc(&ur, cap * F * 4) != cudaSuccess) {
+      cudaGetLastError();
+      undo();
+      set_error("no device memory for the grown upper levels");
+      return HBT_ENOMEM;
+    }
+    const uint64_t live = r.uoff[r.U];
+    if (live) {
+      HBT_CUDA_TRY(cudaMemcpyAsync(uk, r.d_ukeys, live * F * sizeof(K), cudaMemcpyDeviceToDevice, s));
+      HBT_CUDA_TRY(cudaMemcpyAsync(ui, r.d_uidx, live * 32, cudaMemcpyDeviceToDevice, s));
+      HBT_CUDA_TRY(cudaMemcpyAsync(ur, r.d_urefs, live * F * 4, cudaMemcpyDeviceToDevice, s));
+    }
+    HBT_CUDA_TRY(cudaStreamSynchronize(s));
+    cudaFree(r.d_ukeys); cudaFree(r.d_uidx); cudaFree(r.d_urefs);
+    r.d_ukeys = uk; r.d_uidx = ui; r.d_urefs = ur; r.ucap = cap;
+  }
+  if (r.chainpos_cap < r.cap) {
+    uint32_t* cp = nullptr;
+    HBT_CUDA_TRY(cudaMalloc(&cp, r.cap * 4));
+    if (r.chainpos_cap) HBT_CUDA_TRY(cudaMemcpyAsync(cp, r.d_chainpos, r.chainpos_cap * 4, cudaMemcpyDeviceToDevice, s));
+    HBT_CUDA_TRY(cudaStreamSynchronize(s));
+    cudaFree(r.d_chainpos);
+    r.d_chainpos = cp;
+    r.chainpos_cap = r.cap;
+  }
+  return HBT_OK;
+}
+
+// Regroup every upper level from the chain (reading R11).  mx: optional
+// scratch of 2 x (nchain + 1) keys (the update passes preallocated scratch, so it
+// cannot fail for memory after it has modified the leaves).
+template <typename K>
+int rebuild_upper(hbt_tree* t, cudaStream_t s, K* mx = nullptr) {
   RegularState& r = t->r;
   const uint32_t F = t->F;
   uint64_t c = r.nchain, total = 0;
@@ -1100,8 +1156,14 @@ int rebuild_upper(hbt_tree* t, cudaStream_t s) {
   }
   if (U == 0) return HBT_OK;
   K *mx_a = nullptr, *mx_b = nullptr;
-  HBT_CUDA_TRY(scratch_alloc((void**)&mx_a, r.nchain * sizeof(K), s));
-  HBT_CUDA_TRY(scratch_alloc((void**)&mx_b, (unodes[0] + 1) * sizeof(K), s));
+  const bool own = mx == nullptr;
+  if (own) {
+    HBT_CUDA_TRY(scratch_alloc((void**)&mx_a, r.nchain * sizeof(K), s));
+    HBT_CUDA_TRY(scratch_alloc((void**)&mx_b, (unodes[0] + 1) * sizeof(K), s));
+  } else {
+    mx_a = mx;
+    mx_b = mx + r.nchain + 1;
+  }
   chain_leaf_max<K><<<grid_for(r.nchain), 256, 0, s>>>((const K*)r.d_leaf, r.d_count, r.d_chain, r.nchain, F, mx_a);
   uint64_t below = r.nchain;
   for (uint32_t u = 0; u < U; ++u) {
@@ -1112,8 +1174,10 @@ int rebuild_upper(hbt_tree* t, cudaStream_t s) {
     below = unodes[u];
   }
   cudaError_t e = cudaGetLastError();
-  scratch_free(mx_a, s);
-  scratch_free(mx_b, s);
+  if (own) {
+    scratch_free(mx_a, s);
+    scratch_free(mx_b, s);
+  }
   cudaStreamSynchronize(s);
   if (e != cudaSuccess) { set_error("rebuild_upper: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
   return HBT_OK;
@@ -1249,17 +1313,20 @@ __global__ void segment_flags(const uint32_t* __restrict__ leaf_of, uint64_t m, 
 
 // segment s = ops [seg_off[s], seg_off[s+1]) of leaf seg_leaf[s]
 __global__ void segment_tables(const uint32_t* __restrict__ leaf_of, const uint32_t* __restrict__ seg_incl, uint64_t m,
-                               uint32_t* __restrict__ seg_off, uint32_t* __restrict__ seg_leaf,
-                               uint32_t* __restrict__ seg_of_leaf) {
+                               uint32_t* __restrict__ seg_off, uint32_t* __restrict__ seg_leaf) {
   GRID_STRIDE(i, m) {
     if (i == 0 || leaf_of[i] != leaf_of[i - 1]) {
       const uint32_t sgi = seg_incl[i] - 1;
       seg_off[sgi] = uint32_t(i);
       seg_leaf[sgi] = leaf_of[i];
-      seg_of_leaf[leaf_of[i]] = sgi;
     }
     if (i + 1 == m) seg_off[seg_incl[i]] = uint32_t(m);
   }
+}
+
+// leaf -> its update segment (tree-owned map, reset to "none" after the update)
+__global__ void mark_seg_of_leaf(const uint32_t* __restrict__ seg_leaf, uint64_t nseg, uint32_t* __restrict__ seg_of_leaf) {
+  GRID_STRIDE(sg, nseg) seg_of_leaf[seg_leaf[sg]] = uint32_t(sg);
 }
 
 // Big-leaf entry e of leaf v (dense order): line e/P, slot e%P.
@@ -1526,7 +1593,7 @@ int update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   gather_ops<K><<<grid_for(m), 256, 0, s>>>(didx.as<uint32_t>(), m, (const K*)b->values, b->ops, dv.as<K>(),
                                             dop.as<uint8_t>());
   // 2. locate each op's big leaf through the pre-update tree
-  DevBuf leaf_of, start, incl, seg_off, seg_leaf, seg_delta, lb, ins, insx, new_cnt, extra, new_base, dirty;
+  DevBuf leaf_of, start, incl, seg_off, seg_leaf, seg_delta, lb, ins, insx, new_cnt, extra, new_base;
   leaf_of.s = s;
   HBT_CUDA_TRY(scratch_alloc(&leaf_of.p, m * 4, s));
   const uint32_t root_leaf = r.root_leaf;
@@ -1556,7 +1623,7 @@ int update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   HBT_CUDA_TRY(scratch_alloc(&seg_delta.p, nseg * 4, s));
   HBT_CUDA_TRY(cudaMemsetAsync(seg_delta.p, 0, nseg * 4, s));
   segment_tables<<<grid_for(m), 256, 0, s>>>(leaf_of.as<uint32_t>(), incl.as<uint32_t>(), m, seg_off.as<uint32_t>(),
-                                             seg_leaf.as<uint32_t>(), r.d_seg_of_leaf);
+                                             seg_leaf.as<uint32_t>());
   // 4. classify ops against their leaf; new counts; new pool indices (key order)
   lb.s = s;
   HBT_CUDA_TRY(scratch_alloc(&lb.p, m * 4, s));
@@ -1593,13 +1660,33 @@ int update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   const uint64_t n_new = uint64_t(last_base) + last_extra;
   const uint64_t old_pool = r.pool;
   if (old_pool + n_new >= (1ull << 32) - 1) { set_error("pool index overflow"); return HBT_EUNSUPPORTED; }
-  add_base<<<grid_for(nseg), 256, 0, s>>>(new_base.as<uint32_t>(), nseg, old_pool);
-  int rc = grow_pool<K>(t, old_pool + n_new, s);
+  // ---- every allocation of the update happens before its first change to the tree
+  //      (hbt.h: on error the tree is unchanged)
+  const uint64_t nchain_bound = r.nchain + n_new;
+  int rc = reserve_for_update<K>(t, old_pool + n_new, nchain_bound, s);
   if (rc != HBT_OK) return rc;
-  r.pool = old_pool + n_new;
+  DevBuf dirty, parts, ppos, nchain_buf, tmp5, mxbuf, sum;
   dirty.s = s;
-  HBT_CUDA_TRY(scratch_alloc(&dirty.p, r.pool, s));
-  HBT_CUDA_TRY(cudaMemsetAsync(dirty.p, 0, r.pool, s));
+  HBT_CUDA_TRY(scratch_alloc(&dirty.p, old_pool + n_new, s));
+  parts.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&parts.p, (r.nchain + 1) * 4, s));
+  ppos.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&ppos.p, (r.nchain + 1) * 4, s));
+  nchain_buf.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&nchain_buf.p, (nchain_bound + 1) * 4, s));
+  tb2 = 0;
+  HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb2, parts.as<uint32_t>(), ppos.as<uint32_t>(), r.nchain, s));
+  tmp5.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&tmp5.p, tb2 + 256, s));
+  mxbuf.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&mxbuf.p, 2 * (nchain_bound + 2) * sizeof(K), s));
+  sum.s = s;
+  HBT_CUDA_TRY(scratch_alloc(&sum.p, 8, s));
+  HBT_CUDA_TRY(cudaMemsetAsync(dirty.p, 0, old_pool + n_new, s));
+  // ---- mutation starts here
+  add_base<<<grid_for(nseg), 256, 0, s>>>(new_base.as<uint32_t>(), nseg, old_pool);
+  mark_seg_of_leaf<<<grid_for(nseg), 256, 0, s>>>(seg_leaf.as<uint32_t>(), nseg, r.d_seg_of_leaf);
+  r.pool = old_pool + n_new;
   // 5. merge + split + pad, one warp per affected leaf
   {
     constexpr int MAXB = 32 * Geo<K>::P;  // F <= 32
@@ -1611,25 +1698,14 @@ int update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
     HBT_CUDA_TRY(cudaGetLastError());
   }
   // 6. new chain (key order): every old position expands to its parts
-  DevBuf parts, ppos, nchain_buf;
-  parts.s = s;
-  HBT_CUDA_TRY(scratch_alloc(&parts.p, (r.nchain + 1) * 4, s));
-  ppos.s = s;
-  HBT_CUDA_TRY(scratch_alloc(&ppos.p, (r.nchain + 1) * 4, s));
   chain_parts<<<grid_for(r.nchain), 256, 0, s>>>(r.d_chain, r.nchain, r.d_seg_of_leaf, new_cnt.as<uint32_t>(), B,
                                                  parts.as<uint32_t>());
-  DevBuf tmp5;
-  HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb2, parts.as<uint32_t>(), ppos.as<uint32_t>(), r.nchain, s));
-  tmp5.s = s;
-  HBT_CUDA_TRY(scratch_alloc(&tmp5.p, tb2 + 256, s));
   HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp5.p, tb2, parts.as<uint32_t>(), ppos.as<uint32_t>(), r.nchain, s));
   uint32_t lp = 0, lpart = 0;
   HBT_CUDA_TRY(cudaMemcpyAsync(&lp, ppos.as<uint32_t>() + r.nchain - 1, 4, cudaMemcpyDeviceToHost, s));
   HBT_CUDA_TRY(cudaMemcpyAsync(&lpart, parts.as<uint32_t>() + r.nchain - 1, 4, cudaMemcpyDeviceToHost, s));
   HBT_CUDA_TRY(cudaStreamSynchronize(s));
   const uint64_t new_nchain = uint64_t(lp) + lpart;
-  nchain_buf.s = s;
-  HBT_CUDA_TRY(scratch_alloc(&nchain_buf.p, (new_nchain + 1) * 4, s));
   chain_write<<<grid_for(r.nchain), 256, 0, s>>>(r.d_chain, r.nchain, r.d_seg_of_leaf, parts.as<uint32_t>(),
                                                  ppos.as<uint32_t>(), new_base.as<uint32_t>(), nchain_buf.as<uint32_t>());
   reset_seg_of_leaf<<<grid_for(nseg), 256, 0, s>>>(seg_leaf.as<uint32_t>(), nseg, r.d_seg_of_leaf);
@@ -1648,15 +1724,12 @@ int update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   HBT_CUDA_TRY(cudaStreamSynchronize(s));
   HBT_CUDA_TRY(cudaMemcpyAsync(&r.root_leaf, r.d_chain, 4, cudaMemcpyDeviceToHost, s));
   HBT_CUDA_TRY(cudaStreamSynchronize(s));
-  rc = rebuild_upper<K>(t, s);
+  rc = rebuild_upper<K>(t, s, mxbuf.as<K>());
   if (rc != HBT_OK) return rc;
   rc = rebuild_dir<K>(t, s);
   if (rc != HBT_OK) return rc;
   // live key count n' = sum of the chain's counts
   {
-    DevBuf sum;
-    sum.s = s;
-  HBT_CUDA_TRY(scratch_alloc(&sum.p, 8, s));
     HBT_CUDA_TRY(cudaMemsetAsync(sum.p, 0, 8, s));
     chain_count_sum<<<grid_for(r.nchain), 256, 0, s>>>(r.d_chain, r.nchain, r.d_count, sum.as<unsigned long long>());
     uint64_t nn = 0;
@@ -1714,6 +1787,34 @@ int regular_update(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
     r.seg_cap = worst;
   }
   return t->width == 4 ? update_t<uint32_t>(t, b, s) : update_t<uint64_t>(t, b, s);
+}
+
+int regular_clone(const hbt_tree* src, hbt_tree* dst, cudaStream_t s) {
+  const RegularState& a = src->r;
+  RegularState& b = dst->r;
+  if (a.h_leaf) { set_error("clone of a host-placed big-leaf pool is not supported"); return HBT_EUNSUPPORTED; }
+  const uint64_t F = src->F, S = src->width;
+  b = a;  // scalars; every device pointer is replaced below
+  b.d_leaf = b.d_lkeys = b.d_lidx = b.d_ukeys = b.d_uidx = b.d_dir = nullptr;
+  b.d_count = b.d_chain = b.d_urefs = b.d_seg_of_leaf = b.d_chainpos = nullptr;
+  b.h_leaf = nullptr;
+  auto dup = [&](void** d, const void* p, uint64_t bytes) -> int {
+    if (!p || !bytes) return HBT_OK;
+    HBT_CUDA_TRY(cudaMalloc(d, bytes));
+    HBT_CUDA_TRY(cudaMemcpyAsync(*d, p, bytes, cudaMemcpyDeviceToDevice, s));
+    return HBT_OK;
+  };
+  int rc;
+  if ((rc = dup(&b.d_leaf, a.d_leaf, a.cap * F * 64)) || (rc = dup((void**)&b.d_count, a.d_count, a.cap * 4)) ||
+      (rc = dup(&b.d_lkeys, a.d_lkeys, a.cap * F * S)) || (rc = dup(&b.d_lidx, a.d_lidx, a.cap * 32)) ||
+      (rc = dup((void**)&b.d_chain, a.d_chain, a.cap * 4)) || (rc = dup(&b.d_ukeys, a.d_ukeys, a.ucap * F * S)) ||
+      (rc = dup(&b.d_uidx, a.d_uidx, a.ucap * 32)) || (rc = dup((void**)&b.d_urefs, a.d_urefs, a.ucap * F * 4)) ||
+      (rc = dup((void**)&b.d_seg_of_leaf, a.d_seg_of_leaf, a.seg_cap * 4)) ||
+      (rc = dup(&b.d_dir, a.d_dir, a.dir_cap)) ||
+      (rc = dup((void**)&b.d_chainpos, a.d_chainpos, a.chainpos_cap * 4)))
+    return rc;
+  HBT_CUDA_TRY(cudaStreamSynchronize(s));
+  return HBT_OK;
 }
 
 void regular_free(hbt_tree* t) {
