@@ -58,7 +58,8 @@ def test_versioned_search_during_updates(hbt, layout, width, F):
     o = T.from_pairs(k, v, F, width)
     expect = [o.search(q)]
     for bk, bv, bo in batches:
-        o.update(bk, bv, bo)
+        r = o.update(bk, bv, bo)  # ITree.update returns the rebuilt tree, RTree updates in place
+        o = r if layout == "implicit" else o
         expect.append(o.search(q))
     vt = hbt.VersionedTree(gpu_build(hbt, k, v, F, width, layout=layout))
     dq = to_dev(q, width)
