@@ -244,10 +244,6 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *                 the L2 — measured c2 0.426 -> 0.415 ms, c5 Zipf 2.84 -> 3.00 ms with it on)
  *   "item_l2_hint" the same bits for the implicit bucketed item search (default 1: c4 item
  *                 search 10.96 -> 9.50 ms, DRAM reads 171 -> 148 B/query)
- *   "scatter_pair" bucketed search: 1 = the partition's scatter orders TWO chunks of 8192
- *                 queries per 1024-thread CTA, so every bucket run it writes is twice as long;
- *                 0 (default) = one chunk per 512-thread CTA (measured faster: c3 scatter
- *                 0.47 vs 0.58 ms)
  *   "small_threads" small-batch search (directory read in place): CTA size 128, 256 or 1024
  *                 (0 = default 256; 128 measured the same on c1, 1024 slower)
  *   "item_group4" implicit item search with 128 B nodes: 1 = 4-lane query groups (one 256-bit

@@ -476,7 +476,6 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "small_threads" && (value == 0 || value == 128 || value == 256 || value == 1024))
     c.small_threads = uint32_t(value);
   else if (n == "item_group4" && (value == 0 || value == 1)) c.item_group4 = uint32_t(value);
-  else if (n == "scatter_pair" && (value == 0 || value == 1)) c.scatter_pair = uint32_t(value);
   else if (n == "regular_l2_hint" && value >= 0 && value <= 3) c.regular_l2_hint = uint32_t(value);
   else if (n == "item_l2_hint" && value >= 0 && value <= 3) c.item_l2_hint = uint32_t(value);
   else if (n == "full_levels" && value >= 0 && value <= 0xFFFFFFFFll) c.full_levels = uint32_t(value);

@@ -10,32 +10,34 @@
 // bucket lets the queries of a bucket share the slice's lines: they are
 // fetched from DRAM about once per bucket instead of once per query.
 //
-// The batch is cut into chunks of kChunk queries.  Per chunk and bucket the
-// queries form one contiguous RUN in the bucketed order (bucket-major, chunk
-// order inside a bucket), so both reorderings move whole runs:
+// The batch is cut into chunks of kChunk queries, and the chunks into NSEG contiguous
+// SEGMENTS, each handled in chunk order by one CTA in every pass.  Per chunk and
+// bucket the queries form one contiguous RUN in the bucketed order (bucket-major,
+// then segment, then chunk inside a segment), so both reorderings move whole runs:
 //   splitters   sp[b] = max key of unit floor((b+1) U / B) - 1 (units = leaf
 //               lines of the implicit tree / chain big leaves of the regular
 //               tree), sp[B-1] = MAX; bucket(q) = #{sp < q} (a lower bound, the
 //               node-search rule R1 of DESIGN.md applied to the splitters)
 //   directory   dir[p] = [bucket(p << sh), bucket(((p+1) << sh) - 1)] over the
 //               top D bits of the key, so a query binary-searches a short range
-//   bk_count    bucket of every query (u16) + per-chunk histograms tab[b][c]
-//   scan        gb = exclusive scan of tab in (bucket, chunk) order = the
-//               first global slot of every run (CUB)
-//   bk_scatter  per chunk: queries ordered by bucket in shared memory, written
-//               as runs; linv[i] = position of query i in the chunk's order
-//   search      the normal implicit / regular search kernels on the bucketed
-//               queries
-//   bk_gather   per chunk: result runs read into shared memory, stored in
-//               query order through linv
+//   bk_count    bucket of every query (u16), per-chunk histograms tab[c][b] and
+//               per-segment column sums seg[j][b]
+//   bk_seg_scan one CTA: run start of every (segment, bucket), segoff[j][b] =
+//               sum_{b'<b} total(b') + sum_{j'<j} seg[j'][b], and the bucket starts
+//   bk_scatter  per segment, chunk after chunk: queries ordered by bucket in shared
+//               memory and written as runs at a running per-bucket offset (segoff +
+//               earlier chunks' counts); linv[i] = the query's position in its
+//               chunk's bucket-sorted order
+//   search      the item searches (bucket-local directory) on the bucketed queries
+//   bk_gather   per segment, the same running offsets: result runs read into
+//               shared memory, stored in query order through linv
 // Results are bit-identical to the unbucketed search (each query is searched
 // on its own; only the order in which queries are processed changes).
-// Extra HBM traffic per query (u64): 8 + 2 | 2 + 8 + 8 + 2 | - | 2 + 16 + 16.
+// Extra HBM traffic per query (u64): 8 + 2 | - | 2 + 8 + 8 + 2 | - | 2 + 16 + 16.
 #include <algorithm>
+#include <functional>
 #include <mutex>
 #include <vector>
-
-#include <cub/cub.cuh>
 
 #include "hbt_internal.cuh"
 #include "item_dir.cuh"
@@ -121,13 +123,6 @@ __global__ void bk_keyline_max(const uint8_t* __restrict__ leaf, const uint32_t*
   }
 }
 
-__global__ void bk_bstart(const uint32_t* __restrict__ gb, uint64_t chunks, uint32_t B, uint64_t m,
-                          uint64_t* __restrict__ bstart) {
-  const uint32_t b = blockIdx.x * blockDim.x + threadIdx.x;
-  if (b < B) bstart[b] = gb[uint64_t(b) * chunks];
-  if (b == B) bstart[b] = m;
-}
-
 template <typename K>
 __device__ __forceinline__ uint32_t lower_bound_in(const K* sp, uint32_t lo, uint32_t hi, K q) {
   while (lo < hi) {
@@ -189,87 +184,110 @@ __device__ __forceinline__ void block_exclusive_scan(const uint32_t* s_in, uint3
   __syncthreads();
 }
 
-// Tile transpose of a rows x cols u32 matrix (row-major) into cols x rows.
-__global__ void bk_transpose(const uint32_t* __restrict__ in, uint64_t rows, uint32_t cols,
-                             uint32_t* __restrict__ out) {
-  __shared__ uint32_t tile[32][33];
-  const uint64_t r0 = uint64_t(blockIdx.y) * 32, c0 = uint64_t(blockIdx.x) * 32;
-  for (uint32_t i = threadIdx.y; i < 32; i += blockDim.y) {
-    const uint64_t r = r0 + i, c = c0 + threadIdx.x;
-    if (r < rows && c < cols) tile[i][threadIdx.x] = in[r * cols + c];
-  }
-  __syncthreads();
-  for (uint32_t i = threadIdx.y; i < 32; i += blockDim.y) {
-    const uint64_t c = c0 + i, r = r0 + threadIdx.x;
-    if (r < rows && c < cols) out[c * rows + r] = tile[threadIdx.x][i];
-  }
-}
-
-// Pass 1: bucket of every query (bq, u16) and the per-chunk histograms, stored
-// chunk-major: tabT[c * B + b] = #queries of chunk c in bucket b (coalesced; the
-// scan runs on its bucket-major transpose).
+// Pass 1: bucket of every query (bq, u16), the per-chunk histograms (chunk-major:
+// tab[c * B + b] = #queries of chunk c in bucket b) and the per-segment column sums
+// seg[j * B + b] (segment j = chunks [j * kps, (j + 1) * kps), in chunk order).
 template <typename K>
 __global__ void __launch_bounds__(kThreads) bk_count(const K* __restrict__ q, uint64_t m, const K* __restrict__ sp,
                                                      const uint32_t* __restrict__ dir, uint32_t B, uint64_t chunks,
-                                                     uint16_t* __restrict__ bq, uint32_t* __restrict__ tab) {
+                                                     uint64_t kps, uint64_t nseg, uint16_t* __restrict__ bq,
+                                                     uint32_t* __restrict__ tab, uint32_t* __restrict__ seg) {
   extern __shared__ __align__(16) uint8_t smem[];
   uint32_t* s_dir = reinterpret_cast<uint32_t*>(smem);
   uint32_t* s_h = s_dir + (1u << kDirBits);
-  K* s_sp = reinterpret_cast<K*>(s_h + kMaxBuckets);
+  uint32_t* s_sh = s_h + kMaxBuckets;
+  K* s_sp = reinterpret_cast<K*>(s_sh + kMaxBuckets);
   for (uint32_t i = threadIdx.x; i < B; i += kThreads) s_sp[i] = sp[i];
   for (uint32_t i = threadIdx.x; i < (1u << kDirBits); i += kThreads) s_dir[i] = dir[i];
-  for (uint64_t c = blockIdx.x; c < chunks; c += gridDim.x) {
-    if (kStreamPrefetch && threadIdx.x == 0 && c + gridDim.x < chunks) {  // next chunk's queries -> L2
-      const uint64_t n0 = (c + gridDim.x) * kChunk;
-      prefetch_l2_range(q + n0, (m - n0 < kChunk ? m - n0 : kChunk) * sizeof(K));
-    }
-    for (uint32_t i = threadIdx.x; i < B; i += kThreads) s_h[i] = 0;
-    __syncthreads();
-    const uint64_t lo = c * kChunk;
-    K qq[kQPT];
-#pragma unroll
-    for (int j = 0; j < kQPT; ++j) {
-      const uint64_t i = lo + uint64_t(j) * kThreads + threadIdx.x;
-      qq[j] = i < m ? __ldcs(q + i) : K(0);
-    }
-#pragma unroll
-    for (int j = 0; j < kQPT; ++j) {
-      const uint64_t i = lo + uint64_t(j) * kThreads + threadIdx.x;
-      if (i < m) {
-        const uint32_t b = bucket_of(qq[j], s_sp, s_dir);
-        bq[i] = uint16_t(b);
-        atomicAdd(&s_h[b], 1u);
+  for (uint64_t j = blockIdx.x; j < nseg; j += gridDim.x) {
+    const uint64_t c0 = j * kps, c1 = c0 + kps < chunks ? c0 + kps : chunks;
+    for (uint32_t i = threadIdx.x; i < B; i += kThreads) s_sh[i] = 0;
+    for (uint64_t c = c0; c < c1; ++c) {
+      if (kStreamPrefetch && threadIdx.x == 0 && c + 1 < c1) {  // next chunk's queries -> L2
+        const uint64_t n0 = (c + 1) * kChunk;
+        prefetch_l2_range(q + n0, (m - n0 < kChunk ? m - n0 : kChunk) * sizeof(K));
       }
+      for (uint32_t i = threadIdx.x; i < B; i += kThreads) s_h[i] = 0;
+      __syncthreads();
+      const uint64_t lo = c * kChunk;
+      K qq[kQPT];
+#pragma unroll
+      for (int x = 0; x < kQPT; ++x) {
+        const uint64_t i = lo + uint64_t(x) * kThreads + threadIdx.x;
+        qq[x] = i < m ? __ldcs(q + i) : K(0);
+      }
+#pragma unroll
+      for (int x = 0; x < kQPT; ++x) {
+        const uint64_t i = lo + uint64_t(x) * kThreads + threadIdx.x;
+        if (i < m) {
+          const uint32_t b = bucket_of(qq[x], s_sp, s_dir);
+          bq[i] = uint16_t(b);
+          atomicAdd(&s_h[b], 1u);
+        }
+      }
+      __syncthreads();
+      for (uint32_t b = threadIdx.x; b < B; b += kThreads) {
+        tab[c * B + b] = s_h[b];
+        s_sh[b] += s_h[b];
+      }
+      __syncthreads();
     }
-    __syncthreads();
-    for (uint32_t b = threadIdx.x; b < B; b += kThreads) tab[c * B + b] = s_h[b];
-    __syncthreads();
+    for (uint32_t b = threadIdx.x; b < B; b += kThreads) seg[j * B + b] = s_sh[b];
   }
 }
 
-// Per-chunk bucket layout shared by the scatter and the gather (tab, gb
-// chunk-major): s_cnt (this chunk's count per bucket), s_lb (their exclusive scan = the bucket's start in
-// the chunk's bucket-sorted order), s_gb (the run's first global slot).
-template <int TH = kThreads>
-__device__ __forceinline__ void chunk_layout(const uint32_t* __restrict__ tab, const uint32_t* __restrict__ gb,
-                                             uint32_t B, uint64_t chunks, uint64_t c, uint32_t* s_cnt,
-                                             uint32_t* s_lb, uint32_t* s_gb, uint32_t* s_tmp) {
-  for (uint32_t b = threadIdx.x; b < B; b += TH) {  // chunk-major rows: coalesced
-    s_cnt[b] = tab[c * B + b];
-    s_gb[b] = gb[c * B + b];
+// Run starts (one CTA; B <= 1024): bucket b's runs follow segment after segment,
+// buckets in order, so segoff[j * B + b] = bstart[b] + sum_{j' < j} seg[j' * B + b]
+// with bstart[b] = the exclusive scan of the bucket totals (bstart[B] = m).
+constexpr int kScanThreads = 1024;
+__global__ void __launch_bounds__(kScanThreads) bk_seg_scan(const uint32_t* __restrict__ seg, uint32_t B, uint64_t nseg,
+                                                            uint64_t m, uint32_t* __restrict__ segoff,
+                                                            uint64_t* __restrict__ bstart) {
+  __shared__ uint32_t s_T[kScanThreads], s_base[kScanThreads], s_tmp[32];
+  const uint32_t b = threadIdx.x;
+  uint32_t tot = 0;
+  if (b < B) {
+#pragma unroll 8
+    for (uint64_t j = 0; j < nseg; ++j) tot += seg[j * B + b];
   }
+  s_T[b] = tot;
+  __syncthreads();
+  block_exclusive_scan<kScanThreads>(s_T, s_base, B, s_tmp);
+  if (b < B) {
+    uint32_t run = s_base[b];
+#pragma unroll 8
+    for (uint64_t j = 0; j < nseg; ++j) {
+      const uint32_t x = seg[j * B + b];
+      segoff[j * B + b] = run;
+      run += x;
+    }
+    bstart[b] = s_base[b];
+  }
+  if (b == 0) bstart[B] = m;
+}
+
+// Per-chunk bucket layout shared by the scatter and the gather: s_cnt (this chunk's
+// count per bucket, from tab) and s_lb (their exclusive scan = the bucket's start in
+// the chunk's bucket-sorted order).  s_gb (the run's first global slot) is the
+// caller's running per-bucket offset.
+template <int TH = kThreads>
+__device__ __forceinline__ void chunk_layout(const uint32_t* __restrict__ tab, uint32_t B, uint64_t c, uint32_t* s_cnt,
+                                             uint32_t* s_lb, uint32_t* s_tmp) {
+  for (uint32_t b = threadIdx.x; b < B; b += TH) s_cnt[b] = tab[c * B + b];  // chunk-major row: coalesced
   __syncthreads();
   block_exclusive_scan<TH>(s_cnt, s_lb, B, s_tmp);
 }
 
-// Pass 2: each chunk's queries are ordered by bucket in shared memory, then
-// written as B contiguous runs (the run of bucket b at global slot gb[b][c]);
+// Pass 2: per segment, chunk after chunk: each chunk's queries are ordered by bucket
+// in shared memory, then written as B contiguous runs, the run of bucket b at the
+// segment's running offset s_gb[b] (segoff + the segment's earlier chunks' counts);
 // linv[i] (u16) = the query's position in the chunk's bucket-sorted order.
 template <typename K>
 __global__ void __launch_bounds__(kThreads, 2) bk_scatter(const K* __restrict__ q, uint64_t m,
                                                        const uint16_t* __restrict__ bq, const uint32_t* __restrict__ tab,
-                                                       const uint32_t* __restrict__ gb, uint32_t B, uint64_t chunks,
-                                                       K* __restrict__ qs, uint16_t* __restrict__ linv) {
+                                                       const uint32_t* __restrict__ segoff, uint32_t B, uint64_t chunks,
+                                                       uint64_t kps, uint64_t nseg, K* __restrict__ qs,
+                                                       uint16_t* __restrict__ linv) {
   extern __shared__ __align__(16) uint8_t smem[];
   K* s_q = reinterpret_cast<K*>(smem);
   uint16_t* s_b = reinterpret_cast<uint16_t*>(s_q + kChunk);
@@ -280,159 +298,65 @@ __global__ void __launch_bounds__(kThreads, 2) bk_scatter(const K* __restrict__ 
   uint32_t* s_tmp = s_rank + kMaxBuckets;
   // the chunk's queries and bucket ids are loaded before its layout row is scanned,
   // so the two DRAM round trips overlap
-  constexpr int LPT = int(kMaxBuckets) / kThreads;  // layout entries per thread
-  for (uint64_t c = blockIdx.x; c < chunks; c += gridDim.x) {
-    const uint64_t lo = c * kChunk;
-    const uint32_t nc = uint32_t(m - lo < kChunk ? m - lo : kChunk);
-    K qq[kQPT];
-    uint32_t bb[kQPT];
-#pragma unroll
-    for (int j = 0; j < kQPT; ++j) {
-      const uint32_t t = uint32_t(j) * kThreads + threadIdx.x;
-      qq[j] = K(0);
-      bb[j] = 0;
-      if (t < nc) {
-        qq[j] = __ldcs(q + lo + t);
-        bb[j] = __ldcs(reinterpret_cast<const unsigned short*>(bq) + lo + t);
-      }
-    }
+  constexpr int LPT = int(kMaxBuckets) / kThreads;  // layout entries per thread (thread-owned buckets)
+  for (uint64_t j = blockIdx.x; j < nseg; j += gridDim.x) {
+    const uint64_t c0 = j * kps, c1 = c0 + kps < chunks ? c0 + kps : chunks;
 #pragma unroll
     for (int e = 0; e < LPT; ++e) {
       const uint32_t b = uint32_t(e) * kThreads + threadIdx.x;
-      if (b < B) {
-        s_rank[b] = 0;
-        s_cnt[b] = tab[c * B + b];
-        s_gb[b] = gb[c * B + b];
-      }
+      if (b < B) s_gb[b] = segoff[j * B + b];
     }
-    __syncthreads();
-    block_exclusive_scan(s_cnt, s_lb, B, s_tmp);
+    for (uint64_t c = c0; c < c1; ++c) {
+      const uint64_t lo = c * kChunk;
+      const uint32_t nc = uint32_t(m - lo < kChunk ? m - lo : kChunk);
+      K qq[kQPT];
+      uint32_t bb[kQPT];
 #pragma unroll
-    for (int j = 0; j < kQPT; ++j) {
-      const uint32_t t = uint32_t(j) * kThreads + threadIdx.x;
-      if (t < nc) {
-        const uint32_t pos = s_lb[bb[j]] + atomicAdd(&s_rank[bb[j]], 1u);
-        s_q[pos] = qq[j];
-        s_b[pos] = uint16_t(bb[j]);
-        __stcs(reinterpret_cast<unsigned short*>(linv) + lo + t, (unsigned short)pos);
+      for (int x = 0; x < kQPT; ++x) {
+        const uint32_t t = uint32_t(x) * kThreads + threadIdx.x;
+        qq[x] = K(0);
+        bb[x] = 0;
+        if (t < nc) {
+          qq[x] = __ldcs(q + lo + t);
+          bb[x] = __ldcs(reinterpret_cast<const unsigned short*>(bq) + lo + t);
+        }
       }
-    }
-    __syncthreads();
 #pragma unroll
-    for (int j = 0; j < kQPT; ++j) {
-      const uint32_t t = uint32_t(j) * kThreads + threadIdx.x;
-      if (t < nc) {
-        const uint32_t b = s_b[t];
-        qs[uint64_t(s_gb[b]) + (t - s_lb[b])] = s_q[t];
+      for (int e = 0; e < LPT; ++e) {
+        const uint32_t b = uint32_t(e) * kThreads + threadIdx.x;
+        if (b < B) {
+          s_rank[b] = 0;
+          s_cnt[b] = tab[c * B + b];
+        }
       }
-    }
-    __syncthreads();
-  }
-}
-
-// Pass 2, paired form (knob "scatter_pair", off by default): one 1024-thread CTA orders TWO
-// consecutive chunks by bucket in shared memory.  The scan runs in (bucket, chunk) order,
-// so run (b, c+1) starts where run (b, c) ends (gb[c+1][b] = gb[c][b] + cnt[c][b]) and
-// the pair is written as B runs of twice the length: random DRAM writes are bound by
-// their count, not their bytes (c4: 8-query runs of 64 B).  linv is unchanged: each
-// query's position in ITS chunk's bucket-sorted order, which the gather reads back.
-// Measured slower (c3 0.47 -> 0.58 ms, c4 1.95 -> 2.31 ms, profiles/r01s5_scatter_pair.log):
-// one CTA per SM with three block scans per pair hides less latency than the longer
-// runs save, so the one-chunk kernel stays the default.
-constexpr int kPThreads = 2 * kThreads;
-template <typename K>
-__global__ void __launch_bounds__(kPThreads, 1) bk_scatter_pair(const K* __restrict__ q, uint64_t m,
-                                                              const uint16_t* __restrict__ bq,
-                                                              const uint32_t* __restrict__ tab,
-                                                              const uint32_t* __restrict__ gb, uint32_t B,
-                                                              uint64_t chunks, K* __restrict__ qs,
-                                                              uint16_t* __restrict__ linv) {
-  extern __shared__ __align__(16) uint8_t smem[];
-  K* s_q = reinterpret_cast<K*>(smem);
-  uint16_t* s_b = reinterpret_cast<uint16_t*>(s_q + 2 * kChunk);
-  uint32_t* s_cnt0 = reinterpret_cast<uint32_t*>(s_b + 2 * kChunk);
-  uint32_t* s_cnt1 = s_cnt0 + kMaxBuckets;
-  uint32_t* s_cc = s_cnt1 + kMaxBuckets;
-  uint32_t* s_lb0 = s_cc + kMaxBuckets;
-  uint32_t* s_lb1 = s_lb0 + kMaxBuckets;
-  uint32_t* s_L = s_lb1 + kMaxBuckets;
-  uint32_t* s_gb = s_L + kMaxBuckets;
-  uint32_t* s_rank = s_gb + kMaxBuckets;  // 2 x kMaxBuckets
-  uint32_t* s_tmp = s_rank + 2 * kMaxBuckets;
-  const uint32_t h = threadIdx.x / kThreads, tl = threadIdx.x % kThreads;  // chunk of the pair, lane in it
-  const uint64_t pairs = (chunks + 1) / 2;
-  for (uint64_t pc = blockIdx.x; pc < pairs; pc += gridDim.x) {
-    const uint64_t c0 = 2 * pc;
-    const bool has1 = c0 + 1 < chunks;
-    const uint64_t lo = (c0 + h) * kChunk;
-    const uint32_t nc = (c0 + h < chunks) ? uint32_t(m - lo < kChunk ? m - lo : kChunk) : 0u;
-    K qq[kQPT];
-    uint32_t bb[kQPT];
+      __syncthreads();
+      block_exclusive_scan(s_cnt, s_lb, B, s_tmp);
 #pragma unroll
-    for (int j = 0; j < kQPT; ++j) {
-      const uint32_t t = uint32_t(j) * kThreads + tl;
-      qq[j] = K(0);
-      bb[j] = 0;
-      if (t < nc) {
-        qq[j] = __ldcs(q + lo + t);
-        bb[j] = __ldcs(reinterpret_cast<const unsigned short*>(bq) + lo + t);
+      for (int x = 0; x < kQPT; ++x) {
+        const uint32_t t = uint32_t(x) * kThreads + threadIdx.x;
+        if (t < nc) {
+          const uint32_t pos = s_lb[bb[x]] + atomicAdd(&s_rank[bb[x]], 1u);
+          s_q[pos] = qq[x];
+          s_b[pos] = uint16_t(bb[x]);
+          __stcs(reinterpret_cast<unsigned short*>(linv) + lo + t, (unsigned short)pos);
+        }
       }
-    }
-    for (uint32_t b = threadIdx.x; b < B; b += kPThreads) {
-      s_rank[b] = 0;
-      s_rank[kMaxBuckets + b] = 0;
-      const uint32_t a0 = tab[c0 * B + b], a1 = has1 ? tab[(c0 + 1) * B + b] : 0u;
-      s_cnt0[b] = a0;
-      s_cnt1[b] = a1;
-      s_cc[b] = a0 + a1;
-      s_gb[b] = gb[c0 * B + b];
-    }
-    __syncthreads();
-    block_exclusive_scan<kPThreads>(s_cnt0, s_lb0, B, s_tmp);
-    block_exclusive_scan<kPThreads>(s_cnt1, s_lb1, B, s_tmp);
-    block_exclusive_scan<kPThreads>(s_cc, s_L, B, s_tmp);
-    const uint32_t* lbh = h ? s_lb1 : s_lb0;
-    uint32_t* rankh = s_rank + h * kMaxBuckets;
+      __syncthreads();
 #pragma unroll
-    for (int j = 0; j < kQPT; ++j) {
-      const uint32_t t = uint32_t(j) * kThreads + tl;
-      if (t < nc) {
-        const uint32_t b = bb[j];
-        const uint32_t r = atomicAdd(&rankh[b], 1u);
-        const uint32_t pos = s_L[b] + (h ? s_cnt0[b] : 0u) + r;  // pair order: (bucket, chunk, rank)
-        s_q[pos] = qq[j];
-        s_b[pos] = uint16_t(b);
-        __stcs(reinterpret_cast<unsigned short*>(linv) + lo + t, (unsigned short)(lbh[b] + r));
+      for (int x = 0; x < kQPT; ++x) {
+        const uint32_t t = uint32_t(x) * kThreads + threadIdx.x;
+        if (t < nc) {
+          const uint32_t b = s_b[t];
+          qs[uint64_t(s_gb[b]) + (t - s_lb[b])] = s_q[t];
+        }
+      }
+      __syncthreads();
+#pragma unroll
+      for (int e = 0; e < LPT; ++e) {  // the next chunk's runs follow this one's
+        const uint32_t b = uint32_t(e) * kThreads + threadIdx.x;
+        if (b < B) s_gb[b] += s_cnt[b];
       }
     }
-    __syncthreads();
-    const uint32_t ntot = uint32_t(m - c0 * kChunk < 2 * kChunk ? m - c0 * kChunk : 2 * kChunk);
-#pragma unroll 4
-    for (uint32_t t = threadIdx.x; t < ntot; t += kPThreads) {
-      const uint32_t b = s_b[t];
-      qs[uint64_t(s_gb[b]) + (t - s_L[b])] = s_q[t];
-    }
-    __syncthreads();
-  }
-}
-
-template <typename K>
-size_t scatter_pair_smem() {
-  return 2 * kChunk * (sizeof(K) + 2) + kMaxBuckets * 4 * 9 + 32 * 4;
-}
-
-// Pass 2 launch: the one-chunk kernel (default) or the paired kernel ("scatter_pair" = 1).
-template <typename K>
-void launch_scatter(const hbt_tree* t, unsigned grid, size_t smem_single, const void* q, uint64_t m,
-                    const uint16_t* bq, const uint32_t* tab, const uint32_t* gb, uint32_t B, uint64_t chunks,
-                    K* qs, uint16_t* linv, cudaStream_t s) {
-  if (t->cfg.scatter_pair) {
-    const uint64_t pairs = (chunks + 1) / 2;
-    const unsigned g = unsigned(std::min<uint64_t>(pairs, uint64_t(t->num_sms)));
-    bk_scatter_pair<K><<<g ? g : 1, kPThreads, scatter_pair_smem<K>(), s>>>((const K*)q, m, bq, tab, gb, B, chunks,
-                                                                          qs, linv);
-  } else {
-    bk_scatter<K><<<grid, kThreads, smem_single, s>>>((const K*)q, m, bq, tab, gb, B, chunks, qs, linv);
   }
 }
 
@@ -440,8 +364,9 @@ void launch_scatter(const hbt_tree* t, unsigned grid, size_t smem_single, const 
 // shared memory (bucket-sorted order), then stored in query order through linv.
 template <typename K>
 __global__ void __launch_bounds__(kThreads, 2) bk_gather(const uint16_t* __restrict__ linv, uint64_t m,
-                                                      const uint32_t* __restrict__ tab, const uint32_t* __restrict__ gb,
-                                                      uint32_t B, uint64_t chunks, const uint64_t* __restrict__ pf_s,
+                                                      const uint32_t* __restrict__ tab, const uint32_t* __restrict__ segoff,
+                                                      uint32_t B, uint64_t chunks, uint64_t kps, uint64_t nseg,
+                                                      const uint64_t* __restrict__ pf_s,
                                                       const K* __restrict__ v_s, uint64_t* __restrict__ out_pf,
                                                       K* __restrict__ out_v) {
   extern __shared__ __align__(16) uint8_t smem[];
@@ -451,10 +376,13 @@ __global__ void __launch_bounds__(kThreads, 2) bk_gather(const uint16_t* __restr
   uint32_t* s_lb = s_cnt + kMaxBuckets;
   uint32_t* s_gb = s_lb + kMaxBuckets;
   uint32_t* s_tmp = s_gb + kMaxBuckets;
-  for (uint64_t c = blockIdx.x; c < chunks; c += gridDim.x) {
+  for (uint64_t sj = blockIdx.x; sj < nseg; sj += gridDim.x) {
+  const uint64_t c0 = sj * kps, c1 = c0 + kps < chunks ? c0 + kps : chunks;
+  for (uint32_t b = threadIdx.x; b < B; b += kThreads) s_gb[b] = segoff[sj * B + b];  // thread-owned buckets
+  for (uint64_t c = c0; c < c1; ++c) {
     const uint64_t lo = c * kChunk;
     const uint32_t nc = uint32_t(m - lo < kChunk ? m - lo : kChunk);
-    chunk_layout(tab, gb, B, chunks, c, s_cnt, s_lb, s_gb, s_tmp);
+    chunk_layout(tab, B, c, s_cnt, s_lb, s_tmp);
     for (uint32_t b = threadIdx.x; b < B; b += kThreads)
       for (uint32_t k = 0, n = s_cnt[b], p = s_lb[b]; k < n; ++k) s_b[p + k] = uint16_t(b);
     __syncthreads();
@@ -513,6 +441,8 @@ __global__ void __launch_bounds__(kThreads, 2) bk_gather(const uint16_t* __restr
       }
     }
     __syncthreads();
+    for (uint32_t b = threadIdx.x; b < B; b += kThreads) s_gb[b] += s_cnt[b];
+  }
   }
 }
 
@@ -522,16 +452,21 @@ __global__ void __launch_bounds__(kThreads, 2) bk_gather(const uint16_t* __restr
 // makes each half's stores partial sectors and costs DRAM read-modify-writes,
 // 0.77 -> 0.88 ms on c3.)
 constexpr int kGThreads = 1024;
-template <typename K>
+template <typename K, bool REMOTE>
 __global__ void __launch_bounds__(kGThreads) bk_gather_rec(const uint16_t* __restrict__ linv, uint64_t m,
                                                            const uint32_t* __restrict__ tab,
-                                                           const uint32_t* __restrict__ gb, uint32_t B,
-                                                           uint64_t chunks, const ulonglong2* __restrict__ rec,
-                                                           uint64_t* __restrict__ out_pf, K* __restrict__ out_v) {
-  // B <= kMaxBuckets == kGThreads: thread b owns bucket b's layout entries.  The next
-  // chunk's layout row is loaded while this chunk's records are stored, and all of a
-  // thread's record and linv loads are issued together (the kernel was latency
-  // bound: long-scoreboard stalls 38 per issue, one CTA per SM).
+                                                           const uint32_t* __restrict__ segoff, uint32_t B,
+                                                           uint64_t chunks, uint64_t kps, uint64_t nseg,
+                                                           const ulonglong2* __restrict__ rec,
+                                                           uint64_t* __restrict__ out_pf, K* __restrict__ out_v,
+                                                           const RemoteOut ro) {
+  // B <= kMaxBuckets == kGThreads: thread b owns bucket b's layout entries and its
+  // running run offset.  The next chunk's layout row is loaded while this chunk's
+  // records are stored, and all of a thread's record and linv loads are issued
+  // together (the kernel was latency bound: long-scoreboard stalls 38 per issue, one
+  // CTA per SM).  REMOTE (the owner side of the fused sharded exchange): query i of
+  // the receive window came from rank org[i] >> 40, index org[i] & (2^40 - 1) there,
+  // and its record is stored straight into THAT rank's result window (peer memory).
   static_assert(kMaxBuckets <= kGThreads, "one bucket per thread");
   constexpr int PT = int(kChunk) / kGThreads;
   extern __shared__ __align__(16) uint8_t smem[];
@@ -539,64 +474,80 @@ __global__ void __launch_bounds__(kGThreads) bk_gather_rec(const uint16_t* __res
   uint16_t* s_b = reinterpret_cast<uint16_t*>(s_rec + kChunk);
   uint32_t* s_cnt = reinterpret_cast<uint32_t*>(s_b + kChunk);
   uint32_t* s_lb = s_cnt + kMaxBuckets;
-  uint32_t* s_gb = s_lb + kMaxBuckets;
-  uint32_t* s_tmp = s_gb + kMaxBuckets;
+  uint32_t* s_tmp = s_lb + kMaxBuckets;
   const uint32_t tb = threadIdx.x;
-  uint32_t nx_cnt = 0, nx_gb = 0;
-  if (blockIdx.x < chunks && tb < B) {
-    nx_cnt = tab[uint64_t(blockIdx.x) * B + tb];
-    nx_gb = gb[uint64_t(blockIdx.x) * B + tb];
-  }
-  for (uint64_t c = blockIdx.x; c < chunks; c += gridDim.x) {
-    const uint64_t lo = c * kChunk;
-    const uint32_t nc = uint32_t(m - lo < kChunk ? m - lo : kChunk);
-    if (tb < B) {
-      s_cnt[tb] = nx_cnt;
-      s_gb[tb] = nx_gb;
-    }
-    __syncthreads();
-    block_exclusive_scan<kGThreads>(s_cnt, s_lb, B, s_tmp);
-    if (tb < B)
-      for (uint32_t k = 0, n = s_cnt[tb], p = s_lb[tb]; k < n; ++k) s_b[p + k] = uint16_t(tb);
-    __syncthreads();
-    const unsigned short* li = reinterpret_cast<const unsigned short*>(linv) + lo;
-    ulonglong2 x[PT];
-    unsigned short l[PT];
-#pragma unroll
-    for (int j = 0; j < PT; ++j) {
-      const uint32_t t = uint32_t(j) * kGThreads + tb;
-      if (t < nc) {
-        const uint32_t b = s_b[t];
-        x[j] = __ldcs(rec + s_gb[b] + (t - s_lb[b]));
-        l[j] = __ldcs(li + t);
+  for (uint64_t sj = blockIdx.x; sj < nseg; sj += gridDim.x) {
+    const uint64_t c0 = sj * kps, c1 = c0 + kps < chunks ? c0 + kps : chunks;
+    uint32_t run = tb < B ? segoff[sj * B + tb] : 0u;
+    uint32_t nx_cnt = tb < B ? tab[c0 * B + tb] : 0u;
+    for (uint64_t c = c0; c < c1; ++c) {
+      const uint64_t lo = c * kChunk;
+      const uint32_t nc = uint32_t(m - lo < kChunk ? m - lo : kChunk);
+      const uint32_t gbt = run;  // this chunk's run of bucket tb starts here
+      if (tb < B) s_cnt[tb] = nx_cnt;
+      __syncthreads();
+      block_exclusive_scan<kGThreads>(s_cnt, s_lb, B, s_tmp);
+      if (tb < B) {
+        for (uint32_t k = 0, n = s_cnt[tb], p = s_lb[tb]; k < n; ++k) s_b[p + k] = uint16_t(tb);
+        run += s_cnt[tb];
       }
-    }
-    {  // next chunk's layout row, in flight during the stores below
-      const uint64_t cn = c + gridDim.x;
-      if (cn < chunks && tb < B) {
-        nx_cnt = tab[cn * B + tb];
-        nx_gb = gb[cn * B + tb];
-      }
-    }
+      // run starts of this chunk by bucket: s_cnt is free again after the scan, reuse it
+      __syncthreads();
+      if (tb < B) s_cnt[tb] = gbt;
+      __syncthreads();
+      const unsigned short* li = reinterpret_cast<const unsigned short*>(linv) + lo;
+      ulonglong2 x[PT];
+      unsigned short l[PT];
 #pragma unroll
-    for (int j = 0; j < PT; ++j) {
-      const uint32_t t = uint32_t(j) * kGThreads + tb;
-      if (t < nc) s_rec[t] = x[j];
-    }
-    __syncthreads();
-#pragma unroll
-    for (int j = 0; j < PT; ++j) {
-      const uint32_t t = uint32_t(j) * kGThreads + tb;
-      if (t < nc) {
-        const ulonglong2 r = s_rec[l[j]];
-        __stcs(reinterpret_cast<unsigned long long*>(out_pf) + lo + t, r.x);
-        if constexpr (sizeof(K) == 8)
-          __stcs(reinterpret_cast<unsigned long long*>(out_v) + lo + t, r.y);
-        else
-          __stcs(reinterpret_cast<unsigned int*>(out_v) + lo + t, (unsigned int)r.y);
+      for (int j = 0; j < PT; ++j) {
+        const uint32_t t = uint32_t(j) * kGThreads + tb;
+        if (t < nc) {
+          const uint32_t b = s_b[t];
+          x[j] = __ldcs(rec + s_cnt[b] + (t - s_lb[b]));
+          l[j] = __ldcs(li + t);
+        }
       }
+      if (c + 1 < c1 && tb < B) nx_cnt = tab[(c + 1) * B + tb];  // in flight during the stores below
+#pragma unroll
+      for (int j = 0; j < PT; ++j) {
+        const uint32_t t = uint32_t(j) * kGThreads + tb;
+        if (t < nc) s_rec[t] = x[j];
+      }
+      __syncthreads();
+      if constexpr (REMOTE) {
+        uint64_t o[PT];
+#pragma unroll
+        for (int j = 0; j < PT; ++j) {
+          const uint32_t t = uint32_t(j) * kGThreads + tb;
+          o[j] = t < nc ? __ldcs(reinterpret_cast<const unsigned long long*>(ro.org) + lo + t) : 0ull;
+        }
+#pragma unroll
+        for (int j = 0; j < PT; ++j) {
+          const uint32_t t = uint32_t(j) * kGThreads + tb;
+          if (t < nc) {
+            const ulonglong2 r = s_rec[l[j]];
+            const uint32_t src = uint32_t(o[j] >> kRemoteOrgShift);
+            const uint64_t idx = o[j] & ((1ull << kRemoteOrgShift) - 1);
+            ro.pf[src][idx] = r.x;
+            reinterpret_cast<K*>(ro.v[src])[idx] = K(r.y);
+          }
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < PT; ++j) {
+          const uint32_t t = uint32_t(j) * kGThreads + tb;
+          if (t < nc) {
+            const ulonglong2 r = s_rec[l[j]];
+            __stcs(reinterpret_cast<unsigned long long*>(out_pf) + lo + t, r.x);
+            if constexpr (sizeof(K) == 8)
+              __stcs(reinterpret_cast<unsigned long long*>(out_v) + lo + t, r.y);
+            else
+              __stcs(reinterpret_cast<unsigned int*>(out_v) + lo + t, (unsigned int)r.y);
+          }
+        }
+      }
+      __syncthreads();
     }
-    __syncthreads();
   }
 }
 
@@ -609,14 +560,12 @@ void set_bucket_attrs() {
   cudaFuncSetAttribute(bk_count<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
   cudaFuncSetAttribute(bk_scatter<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
   cudaFuncSetAttribute(bk_scatter<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
-  cudaFuncSetAttribute(bk_scatter_pair<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                       int(scatter_pair_smem<uint32_t>()));
-  cudaFuncSetAttribute(bk_scatter_pair<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                       int(scatter_pair_smem<uint64_t>()));
   cudaFuncSetAttribute(bk_gather<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
   cudaFuncSetAttribute(bk_gather<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
-  cudaFuncSetAttribute(bk_gather_rec<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-  cudaFuncSetAttribute(bk_gather_rec<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+  cudaFuncSetAttribute(bk_gather_rec<uint32_t, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+  cudaFuncSetAttribute(bk_gather_rec<uint64_t, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+  cudaFuncSetAttribute(bk_gather_rec<uint32_t, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+  cudaFuncSetAttribute(bk_gather_rec<uint64_t, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
   attr = true;
 }
 
@@ -729,37 +678,88 @@ int prepare_splitters(const hbt_tree* t, cudaStream_t s, BucketState& bs, uint32
   return HBT_OK;
 }
 
+// Scratch layout and geometry of one partitioned batch (stream-ordered pool).
+struct Part {
+  uint32_t B = 0;
+  uint64_t chunks = 0, kps = 0, nseg = 0;
+  uint8_t* base = nullptr;
+  uint64_t o_pf = 0, o_v = 0, o_bq = 0, o_li = 0, o_tab = 0, o_seg = 0, o_so = 0, o_bs = 0, total = 0;
+  template <typename T> T* at(uint64_t o) const { return reinterpret_cast<T*>(base + o); }
+};
+
+// qs (m x S) | results: pf_s (m x 8) + v_s (m x 8), or 16 B records over the same
+// 16 m bytes | bq (u16) | linv (u16) | tab (chunks x B) | seg, segoff (nseg x B) |
+// bucket starts (B + 1)
+template <typename K>
+Part part_layout(uint64_t m, uint32_t B, uint32_t sms) {
+  Part p;
+  p.B = B;
+  p.chunks = (m + kChunk - 1) / kChunk;
+  const uint64_t want = std::min<uint64_t>(p.chunks, uint64_t(sms) * 2);
+  p.kps = (p.chunks + want - 1) / want;
+  p.nseg = (p.chunks + p.kps - 1) / p.kps;
+  auto al = [](uint64_t x) { return (x + 255) & ~uint64_t(255); };
+  p.o_pf = al(m * sizeof(K));
+  p.o_v = p.o_pf + al(m * 8);
+  p.o_bq = p.o_v + al(m * 8);
+  p.o_li = p.o_bq + al(m * 2);
+  p.o_tab = p.o_li + al(m * 2);
+  p.o_seg = p.o_tab + al(p.chunks * B * 4);
+  p.o_so = p.o_seg + al(p.nseg * B * 4);
+  p.o_bs = p.o_so + al(p.nseg * B * 4);
+  p.total = p.o_bs + al((uint64_t(B) + 1) * 8);
+  return p;
+}
+
+constexpr size_t kSmemCount = (1u << kDirBits) * 4 + kMaxBuckets * 4 * 2 + kMaxBuckets * 8;
+template <typename K>
+constexpr size_t smem_scatter() { return kChunk * (sizeof(K) + 2) + kMaxBuckets * 4 * 4 + kThreads * 4; }
+constexpr size_t kSmemGather = kChunk * (8 + 2) + kMaxBuckets * 4 * 3 + kThreads * 4;
+constexpr size_t kSmemGatherRec = kChunk * (16 + 2) + kMaxBuckets * 4 * 2 + kGThreads * 4;
+
+// count -> run starts -> scatter: the batch q in bucket order at qs (Part::base).
+template <typename K>
+int partition(const hbt_tree* t, const BucketState& bs, const void* q, uint64_t m, const Part& p, cudaStream_t s,
+              const std::function<void(int)>& mark) {
+  set_bucket_attrs();
+  const unsigned grid = unsigned(std::min<uint64_t>(p.nseg, uint64_t(t->num_sms) * 2));
+  mark(0);
+  bk_count<K><<<grid, kThreads, kSmemCount, s>>>((const K*)q, m, (const K*)bs.d_sp, bs.d_dir, p.B, p.chunks, p.kps,
+                                                 p.nseg, p.at<uint16_t>(p.o_bq), p.at<uint32_t>(p.o_tab),
+                                                 p.at<uint32_t>(p.o_seg));
+  mark(1);
+  bk_seg_scan<<<1, kScanThreads, 0, s>>>(p.at<uint32_t>(p.o_seg), p.B, p.nseg, m, p.at<uint32_t>(p.o_so),
+                                         p.at<uint64_t>(p.o_bs));
+  mark(2);
+  bk_scatter<K><<<grid, kThreads, smem_scatter<K>(), s>>>((const K*)q, m, p.at<uint16_t>(p.o_bq),
+                                                          p.at<uint32_t>(p.o_tab), p.at<uint32_t>(p.o_so), p.B,
+                                                          p.chunks, p.kps, p.nseg, p.at<K>(0),
+                                                          p.at<uint16_t>(p.o_li));
+  if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) {
+    set_error("bucketing kernels failed to launch: %s", cudaGetErrorString(e));
+    return HBT_ECUDA;
+  }
+  mark(3);
+  return HBT_OK;
+}
+
 template <typename K>
 int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
-               cudaStream_t s) {
+               cudaStream_t s, const RemoteOut* ro) {
   int rc = prepare_splitters<K>(t, s, t->bk, pick_buckets(t), true);
   if (rc != HBT_OK) return rc;
   const BucketState& bs = t->bk;
-  const uint32_t B = bs.B;
-  const uint64_t chunks = (m + kChunk - 1) / kChunk;
-  const uint64_t ntab = uint64_t(B) * chunks;
-  size_t scan_bytes = 0;
-  HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, scan_bytes, (const uint32_t*)nullptr, (uint32_t*)nullptr,
-                                             ntab, s));
-  // scratch (stream-ordered pool): qs, pf_s, v_s, bq, linv, tab, gb, scan temp
-  auto al = [](uint64_t x) { return (x + 255) & ~uint64_t(255); };
-  // pf_s + v_s (plain search) or 16 B records (item directory: o_pf .. o_pf + 16 m)
-  const uint64_t o_pf = al(m * sizeof(K)), o_v = o_pf + al(m * 8), o_bq = o_v + al(m * 8),
-                 o_li = o_bq + al(m * 2), o_tab = o_li + al(m * 2), o_gb = o_tab + al(ntab * 4),
-                 o_bm = o_gb + al(ntab * 4), o_bm2 = o_bm + al(ntab * 4),
-                 o_bs = o_bm2 + al(ntab * 4), o_tmp = o_bs + al((uint64_t(B) + 1) * 8),
-                 total = o_tmp + al(scan_bytes);
+  if (ro && !bs.items) {
+    set_error("remote result stores need the bucket-local item directory");
+    return HBT_EUNSUPPORTED;
+  }
+  Part p = part_layout<K>(m, bs.B, uint32_t(t->num_sms));
   void* buf = nullptr;
-  HBT_CUDA_TRY(scratch_alloc(&buf, total, s));
-  uint8_t* base = static_cast<uint8_t*>(buf);
-  K* qs = reinterpret_cast<K*>(base);
-  uint64_t* pf_s = reinterpret_cast<uint64_t*>(base + o_pf);
-  K* v_s = reinterpret_cast<K*>(base + o_v);
-  uint16_t* bq = reinterpret_cast<uint16_t*>(base + o_bq);
-  uint16_t* linv = reinterpret_cast<uint16_t*>(base + o_li);
-  uint32_t* tab = reinterpret_cast<uint32_t*>(base + o_tab);
-  uint32_t* gb = reinterpret_cast<uint32_t*>(base + o_gb);
-  rc = HBT_OK;
+  HBT_CUDA_TRY(scratch_alloc(&buf, p.total, s));
+  p.base = static_cast<uint8_t*>(buf);
+  K* qs = p.at<K>(0);
+  uint64_t* pf_s = p.at<uint64_t>(p.o_pf);
+  K* v_s = p.at<K>(p.o_v);
   BucketState& bw = t->bk;
   const bool timing = t->cfg.phase_timing != 0;
   if (timing && !bw.ev[0])
@@ -768,55 +768,21 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
     if (timing) cudaEventRecord(bw.ev[i], s);
   };
   do {
-    const size_t smem_count = (1u << kDirBits) * 4 + kMaxBuckets * 4 + kMaxBuckets * sizeof(K);
-    const size_t smem_scatter = kChunk * (sizeof(K) + 2) + kMaxBuckets * 4 * 4 + kThreads * 4;
-    const size_t smem_gather = kChunk * (8 + 2) + kMaxBuckets * 4 * 3 + kThreads * 4;
-    const size_t smem_gather_rec = kChunk * (16 + 2) + kMaxBuckets * 4 * 3 + kGThreads * 4;
-    set_bucket_attrs();
-    const unsigned grid = unsigned(std::min<uint64_t>(chunks, uint64_t(t->num_sms) * 2));
-    mark(0);
-    bk_count<K><<<grid, kThreads, smem_count, s>>>((const K*)q, m, (const K*)bs.d_sp, bs.d_dir, B, chunks, bq, tab);
-    mark(1);
-    {
-      // chunk-major counts -> bucket-major, exclusive scan (run starts), -> chunk-major
-      uint32_t* tab_bm = reinterpret_cast<uint32_t*>(base + o_bm);
-      uint32_t* gb_bm = reinterpret_cast<uint32_t*>(base + o_bm2);
-      const dim3 tb(32, 8);
-      bk_transpose<<<dim3((B + 31) / 32, unsigned((chunks + 31) / 32)), tb, 0, s>>>(tab, chunks, B, tab_bm);
-      if (cub::DeviceScan::ExclusiveSum(base + o_tmp, scan_bytes, tab_bm, gb_bm, ntab, s) != cudaSuccess) {
-        set_error("bucket scan failed");
-        rc = HBT_ECUDA;
-        break;
-      }
-      bk_transpose<<<dim3(unsigned((chunks + 31) / 32), (B + 31) / 32), tb, 0, s>>>(gb_bm, B, uint32_t(chunks), gb);
-      if (bs.items) {
-        uint64_t* bstart = reinterpret_cast<uint64_t*>(base + o_bs);
-        bk_bstart<<<(B + 256) / 256, 256, 0, s>>>(gb_bm, chunks, B, m, bstart);
-      }
-    }
-    mark(2);
-    launch_scatter<K>(t, grid, smem_scatter, q, m, bq, tab, gb, B, chunks, qs, linv, s);
-    if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) {
-      set_error("bucketing kernels failed to launch: %s", cudaGetErrorString(e));
-      rc = HBT_ECUDA;
-      break;
-    }
-    mark(3);
+    if ((rc = partition<K>(t, bs, q, m, p, s, mark)) != HBT_OK) break;
     if (bs.items) {
-      uint64_t* bstart = reinterpret_cast<uint64_t*>(base + o_bs);
       ItemDir d;
       d.M = bs.d_M;
       d.chain = t->form == HBT_REGULAR ? t->r.d_chain : nullptr;
-      d.bstart = bstart;
-      d.B = B;
+      d.bstart = p.at<uint64_t>(p.o_bs);
+      d.B = p.B;
       d.U = t->form == HBT_IMPLICIT ? t->L0 : t->r.nchain;
       d.level = bs.level;
       d.span = bs.span;
       d.nunits = bs.nunits;
       d.pos_base = pos_base;
       d.qprefetch = t->cfg.qprefetch;
-      d.cap = t->cfg.bucket_cap ? std::min<uint32_t>(t->cfg.bucket_cap, uint32_t(item_cap(t, B)))
-                                : uint32_t(item_cap(t, B));
+      d.cap = t->cfg.bucket_cap ? std::min<uint32_t>(t->cfg.bucket_cap, uint32_t(item_cap(t, p.B)))
+                                : uint32_t(item_cap(t, p.B));
       d.strided = t->form == HBT_IMPLICIT ? t->cfg.item_sched : 0u;
       rc = t->form == HBT_IMPLICIT ? implicit_search_items(t, qs, m, pf_s, v_s, d, s)
                                    : regular_search_items(t, qs, m, pf_s, v_s, d, s);
@@ -826,19 +792,30 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
     }
     if (rc != HBT_OK) break;
     mark(4);
-    if (bs.items)
-      bk_gather_rec<K><<<unsigned(std::min<uint64_t>(chunks, t->num_sms)), kGThreads, smem_gather_rec, s>>>(
-          linv, m, tab, gb, B, chunks, reinterpret_cast<const ulonglong2*>(pf_s), pf, (K*)v);
-    else
-      bk_gather<K><<<grid, kThreads, smem_gather, s>>>(linv, m, tab, gb, B, chunks, pf_s, v_s, pf, (K*)v);
+    const uint16_t* linv = p.at<uint16_t>(p.o_li);
+    const uint32_t* tab = p.at<uint32_t>(p.o_tab);
+    const uint32_t* so = p.at<uint32_t>(p.o_so);
+    if (bs.items) {
+      const unsigned g = unsigned(std::min<uint64_t>(p.nseg, t->num_sms));
+      const ulonglong2* rec = reinterpret_cast<const ulonglong2*>(pf_s);
+      if (ro)
+        bk_gather_rec<K, true><<<g, kGThreads, kSmemGatherRec, s>>>(linv, m, tab, so, p.B, p.chunks, p.kps, p.nseg,
+                                                                    rec, nullptr, nullptr, *ro);
+      else
+        bk_gather_rec<K, false><<<g, kGThreads, kSmemGatherRec, s>>>(linv, m, tab, so, p.B, p.chunks, p.kps, p.nseg,
+                                                                     rec, pf, (K*)v, RemoteOut{});
+    } else {
+      const unsigned g = unsigned(std::min<uint64_t>(p.nseg, uint64_t(t->num_sms) * 2));
+      bk_gather<K><<<g, kThreads, kSmemGather, s>>>(linv, m, tab, so, p.B, p.chunks, p.kps, p.nseg, pf_s, v_s, pf,
+                                                   (K*)v);
+    }
     if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) {
       set_error("bucket gather failed to launch: %s", cudaGetErrorString(e));
       rc = HBT_ECUDA;
       break;
     }
     mark(5);
-    // count, transpose, CUB scan (2), transpose, [bucket starts,] scatter, search, gather
-    bw.launches = bs.items ? 9u : 8u;
+    bw.launches = 5;  // count, run starts, scatter, search, gather
     bw.timed = timing;
   } while (0);
   scratch_free(buf, s);
@@ -894,54 +871,18 @@ int streamed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
       HBT_CUDA_TRY(cudaEventRecord(bs.ev_done[i], s));  // slots start free
     }
   }
-  const uint64_t chunks = (m + kChunk - 1) / kChunk;
-  const uint64_t ntab = uint64_t(B) * chunks;
-  size_t scan_bytes = 0;
-  HBT_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, scan_bytes, (const uint32_t*)nullptr, (uint32_t*)nullptr,
-                                             ntab, s));
-  auto al = [](uint64_t x) { return (x + 255) & ~uint64_t(255); };
-  const uint64_t o_pf = al(m * sizeof(K)), o_v = o_pf + al(m * 8), o_bq = o_v + al(m * sizeof(K)),
-                 o_li = o_bq + al(m * 2), o_tab = o_li + al(m * 2), o_gb = o_tab + al(ntab * 4),
-                 o_bm = o_gb + al(ntab * 4), o_bm2 = o_bm + al(ntab * 4), o_bs = o_bm2 + al(ntab * 4),
-                 o_tmp = o_bs + al((uint64_t(B) + 1) * 8), total = o_tmp + al(scan_bytes);
+  Part p = part_layout<K>(m, B, uint32_t(t->num_sms));
   void* buf = nullptr;
-  HBT_CUDA_TRY(scratch_alloc(&buf, total, s));
-  uint8_t* base = static_cast<uint8_t*>(buf);
-  K* qs = reinterpret_cast<K*>(base);
-  uint64_t* pf_s = reinterpret_cast<uint64_t*>(base + o_pf);
-  K* v_s = reinterpret_cast<K*>(base + o_v);
-  uint16_t* bq = reinterpret_cast<uint16_t*>(base + o_bq);
-  uint16_t* linv = reinterpret_cast<uint16_t*>(base + o_li);
-  uint32_t* tab = reinterpret_cast<uint32_t*>(base + o_tab);
-  uint32_t* gb = reinterpret_cast<uint32_t*>(base + o_gb);
-  uint32_t* tab_bm = reinterpret_cast<uint32_t*>(base + o_bm);
-  uint32_t* gb_bm = reinterpret_cast<uint32_t*>(base + o_bm2);
-  uint64_t* bstart = reinterpret_cast<uint64_t*>(base + o_bs);
+  HBT_CUDA_TRY(scratch_alloc(&buf, p.total, s));
+  p.base = static_cast<uint8_t*>(buf);
+  K* qs = p.at<K>(0);
+  uint64_t* pf_s = p.at<uint64_t>(p.o_pf);
+  K* v_s = p.at<K>(p.o_v);
   std::vector<uint64_t> hb(B + 1);
   do {
-    const size_t smem_count = (1u << kDirBits) * 4 + kMaxBuckets * 4 + kMaxBuckets * sizeof(K);
-    const size_t smem_scatter = kChunk * (sizeof(K) + 2) + kMaxBuckets * 4 * 4 + kThreads * 4;
-    const size_t smem_gather = kChunk * (8 + 2) + kMaxBuckets * 4 * 3 + kThreads * 4;
-    const unsigned grid = unsigned(std::min<uint64_t>(chunks, uint64_t(t->num_sms) * 2));
-    set_bucket_attrs();
-    bk_count<K><<<grid, kThreads, smem_count, s>>>((const K*)q, m, (const K*)bs.d_sp, bs.d_dir, B, chunks, bq, tab);
-    const dim3 tb(32, 8);
-    bk_transpose<<<dim3((B + 31) / 32, unsigned((chunks + 31) / 32)), tb, 0, s>>>(tab, chunks, B, tab_bm);
-    if (cub::DeviceScan::ExclusiveSum(base + o_tmp, scan_bytes, tab_bm, gb_bm, ntab, s) != cudaSuccess) {
-      set_error("bucket scan failed");
-      rc = HBT_ECUDA;
-      break;
-    }
-    bk_transpose<<<dim3(unsigned((chunks + 31) / 32), (B + 31) / 32), tb, 0, s>>>(gb_bm, B, uint32_t(chunks), gb);
-    bk_bstart<<<(B + 256) / 256, 256, 0, s>>>(gb_bm, chunks, B, m, bstart);
-    launch_scatter<K>(t, grid, smem_scatter, q, m, bq, tab, gb, B, chunks, qs, linv, s);
-    if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) {
-      set_error("bucketing kernels failed to launch: %s", cudaGetErrorString(e));
-      rc = HBT_ECUDA;
-      break;
-    }
+    if ((rc = partition<K>(t, bs, q, m, p, s, [](int) {})) != HBT_OK) break;
     // the bucket boundaries drive the host loop below (one sync per batch)
-    HBT_CUDA_TRY(cudaMemcpyAsync(hb.data(), bstart, (B + 1) * 8, cudaMemcpyDeviceToHost, s));
+    HBT_CUDA_TRY(cudaMemcpyAsync(hb.data(), p.at<uint64_t>(p.o_bs), (B + 1) * 8, cudaMemcpyDeviceToHost, s));
     HBT_CUDA_TRY(cudaStreamSynchronize(s));
     const uint8_t* hl = static_cast<const uint8_t*>(t->h_leaf);
     uint32_t j = 0;
@@ -960,7 +901,10 @@ int streamed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
       HBT_CUDA_TRY(cudaEventRecord(bs.ev_done[slot], s));
     }
     if (rc != HBT_OK) break;
-    bk_gather<K><<<grid, kThreads, smem_gather, s>>>(linv, m, tab, gb, B, chunks, pf_s, v_s, pf, (K*)v);
+    const unsigned g = unsigned(std::min<uint64_t>(p.nseg, uint64_t(t->num_sms) * 2));
+    bk_gather<K><<<g, kThreads, kSmemGather, s>>>(p.at<uint16_t>(p.o_li), m, p.at<uint32_t>(p.o_tab),
+                                                 p.at<uint32_t>(p.o_so), B, p.chunks, p.kps, p.nseg, pf_s, v_s, pf,
+                                                 (K*)v);
     if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) {
       set_error("bucket gather failed to launch: %s", cudaGetErrorString(e));
       rc = HBT_ECUDA;
@@ -1005,9 +949,9 @@ bool bucketed_enabled(const hbt_tree* t, uint64_t m) {
 }
 
 int bucketed_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
-                    cudaStream_t s) {
-  return t->width == 4 ? bucketed_t<uint32_t>(t, q, m, pf, v, pos_base, s)
-                       : bucketed_t<uint64_t>(t, q, m, pf, v, pos_base, s);
+                    cudaStream_t s, const RemoteOut* ro) {
+  return t->width == 4 ? bucketed_t<uint32_t>(t, q, m, pf, v, pos_base, s, ro)
+                       : bucketed_t<uint64_t>(t, q, m, pf, v, pos_base, s, ro);
 }
 
 int shard_local_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,

@@ -78,8 +78,6 @@ struct SearchConfig {
   uint32_t l2_hint = 4;          // implicit search: L2 eviction-priority hints (LevelTable::l2_hint);
                                  // 4 = auto: leaf lines evict-first iff the I-segment fits in L2 / 4
   uint32_t item_l2_hint = 1;     // implicit bucketed item search (c4 item search 10.96 -> 9.50 ms)
-  uint32_t scatter_pair = 0;     // bucketed search: scatter two chunks per CTA (runs twice as long; measured
-                                 // slower: c3 scatter 0.47 -> 0.58 ms, c4 1.95 -> 2.31 ms)
   uint32_t small_threads = 0;    // small-batch (in-place directory) search: CTA size 128 / 256 / 1024 (0 = 256)
   uint32_t item_group4 = 0;      // implicit item search, 128 B nodes: 4-lane groups (one 256-bit load per lane;
                                  // measured slower: c4 item search 9.50 -> 10.8 ms, 56 B of spills)
@@ -115,6 +113,16 @@ struct ItemDir {
   // work through the bucketed order together (implicit_search.cu)
   uint32_t strided = 0;
   uint32_t pbits = 10;    // prefix-table bits of the staged directory (<= 12)
+};
+
+// Owner side of the fused sharded exchange (sharded_fused.cu): the bucketed search's
+// gather stores each received query's result straight into the REQUESTER's result
+// window (mapped peer memory) at the query's original index.
+constexpr int kRemoteOrgShift = 40;  // org = (source rank << 40) | index at the source
+struct RemoteOut {
+  const uint64_t* org = nullptr;  // per received query (receive-window order)
+  uint64_t* pf[64] = {};          // per source rank: its result window
+  uint8_t* v[64] = {};
 };
 
 // Query-bucketing state (bucketed.cu): B splitter keys and a prefix directory,
@@ -340,7 +348,7 @@ int regular_search_items(const hbt_tree* t, const void* q, uint64_t m, uint64_t*
 // bucketed.cu
 bool bucketed_enabled(const hbt_tree* t, uint64_t m);
 int bucketed_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
-                    cudaStream_t s);
+                    cudaStream_t s, const RemoteOut* ro = nullptr);
 // the owner-side search of the sharded paths: bucketed when enabled, positions + pos_base
 int shard_local_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,
                        cudaStream_t s);

@@ -1,23 +1,31 @@
 // sharded_fused.cu — the key-range-sharded search with a FUSED exchange over
-// peer memory (NVLink 5 / NVSwitch): no NCCL on the data path.
+// peer memory (NVLink 5 / NVSwitch): no NCCL and no host collective on the data path.
 //
 // Every rank owns one window (one cudaMalloc, exported with CUDA IPC and
 // mapped by every peer):
-//   [flags: 64 x u32 | matrix: 64 x 64 u64 | res_pf: cap_m u64 | res_v: cap_m x S
-//    | recv_q: cap_r x S | recv_org: cap_r u64]
-// Per batch (all kernels stream-ordered; barriers are device-side flag
-// exchanges over peer memory):
-//   1. route_count (sharded.cu's owner rule) + publish: this rank's count row
-//      is stored into EVERY peer's matrix                         -> barrier
-//   2. route_put: every query is stored straight into its owner's receive
-//      window at (prefix of earlier sources' counts) + a CTA-reserved slot,
-//      with its origin (source rank, index)                       -> barrier
-//   3. the owner searches its receive window (pos_base = its first global rank)
-//   4. return_put: each result is stored straight into the requester's result
-//      window at its ORIGINAL index (no unpermute pass)           -> barrier
+//   [flags: 64 x u32 | matrix: 2 x 64 x 64 u64 (parity of the batch) | res_pf: cap_m u64
+//    | res_v: cap_m x S | recv_q: cap_r x S | recv_org: cap_r u64]
+// Per batch b (all kernels stream-ordered; barriers are device-side flag exchanges
+// over peer memory):
+//   1. f_count (the owner rule of sharded.cu) counts queries per destination, and
+//      f_publish stores this rank's count row into EVERY peer's matrix[b & 1]
+//                                                                 -> barrier
+//   2. the host reads its own matrix[b & 1] (the full G x G count matrix, one small
+//      D2H) to size the owner search; every rank sees the same matrix, so a window
+//      regrowth is decided identically everywhere (a collective re-export)
+//   3. f_put: every query is stored straight into its owner's receive window at
+//      (earlier sources' counts) + a CTA-reserved slot, with its origin (rank, index)
+//                                                                 -> barrier
+//   4. the owner searches its receive window (pos_base = its first global rank); the
+//      bucketed search's final gather stores each result straight into the
+//      REQUESTER's result window at the query's original index (bucketed.cu,
+//      RemoteOut); small batches search into scratch and f_return stores them
+//                                                                 -> barrier
 //   5. the requester copies its result window into the caller's out arrays.
-// The same kernels run for G virtual shards on one GPU (peer table = local
-// windows, barriers = stream order), which is how they are tested here.
+// The matrix is double-buffered by batch parity, so step 1 of batch b+1 (stores into
+// the peers' other matrix) cannot disturb a peer still reading batch b's.  The same
+// kernels run for G virtual shards on one GPU (peer table = local windows, barriers =
+// stream order), which is how they are tested on one device.
 #include <nccl.h>
 
 #include <vector>
@@ -29,11 +37,12 @@ namespace {
 
 constexpr int kMaxG = 64;
 constexpr int kThreads = 256;
-constexpr uint64_t kOrgShift = 40;  // recv_org = (source rank << 40) | origin index
+constexpr uint64_t kOrgShift = kRemoteOrgShift;  // recv_org = (source rank << 40) | origin index
+constexpr uint64_t kMat = uint64_t(kMaxG) * kMaxG;  // one parity of the count matrix
 
 struct Win {
   uint32_t* flags;
-  unsigned long long* matrix;  // [src][dst]
+  unsigned long long* matrix;  // [parity][src][dst]
   uint64_t* res_pf;
   uint8_t* res_v;
   uint8_t* recv_q;
@@ -59,7 +68,7 @@ inline unsigned grid_for(uint64_t n) {
 
 uint64_t win_bytes(uint64_t cap_m, uint64_t cap_r, uint32_t S) {
   auto al = [](uint64_t x) { return (x + 255) & ~uint64_t(255); };
-  return al(kMaxG * 4) + al(kMaxG * kMaxG * 8) + al(cap_m * 8) + al(cap_m * S) + al(cap_r * S) + al(cap_r * 8);
+  return al(kMaxG * 4) + al(2 * kMat * 8) + al(cap_m * 8) + al(cap_m * S) + al(cap_r * S) + al(cap_r * 8);
 }
 
 Win carve(uint8_t* base, uint64_t cap_m, uint64_t cap_r, uint32_t S) {
@@ -67,7 +76,7 @@ Win carve(uint8_t* base, uint64_t cap_m, uint64_t cap_r, uint32_t S) {
   Win w;
   uint64_t o = 0;
   w.flags = (uint32_t*)(base + o); o += al(kMaxG * 4);
-  w.matrix = (unsigned long long*)(base + o); o += al(kMaxG * kMaxG * 8);
+  w.matrix = (unsigned long long*)(base + o); o += al(2 * kMat * 8);
   w.res_pf = (uint64_t*)(base + o); o += al(cap_m * 8);
   w.res_v = base + o; o += al(cap_m * S);
   w.recv_q = base + o; o += al(cap_r * S);
@@ -99,18 +108,18 @@ __global__ void __launch_bounds__(kThreads) f_count(const K* __restrict__ q, uin
     if (h[i]) atomicAdd(cnt + i, (unsigned long long)h[i]);
 }
 
-// Store this rank's count row into every peer's matrix (row `me`).
-__global__ void f_publish(const PeerTable pt, int me, const unsigned long long* __restrict__ cnt) {
+// Store this rank's count row into every peer's matrix[parity] (row `me`).
+__global__ void f_publish(const PeerTable pt, int me, const unsigned long long* __restrict__ cnt, int parity) {
   for (int x = threadIdx.x; x < pt.G * pt.G; x += blockDim.x) {
     const int d = x / pt.G, c = x % pt.G;
-    pt.w[d].matrix[me * kMaxG + c] = cnt[c];
+    pt.w[d].matrix[parity * kMat + me * kMaxG + c] = cnt[c];
   }
 }
 
 // Route + put: queries go straight into their owner's receive window.
 template <typename K>
 __global__ void __launch_bounds__(kThreads) f_put(const K* __restrict__ q, uint64_t m, const uint8_t* __restrict__ dest,
-                                                  const PeerTable pt, int me,
+                                                  const PeerTable pt, int me, int parity,
                                                   unsigned long long* __restrict__ cursor, uint64_t chunk) {
   __shared__ unsigned int h[kMaxG];
   __shared__ unsigned long long base[kMaxG];
@@ -121,7 +130,7 @@ __global__ void __launch_bounds__(kThreads) f_put(const K* __restrict__ q, uint6
   __syncthreads();
   for (uint64_t i = lo + threadIdx.x; i < hi; i += blockDim.x) atomicAdd(&h[dest[i]], 1u);
   __syncthreads();
-  const unsigned long long* M = pt.w[me].matrix;  // full matrix (every row published)
+  const unsigned long long* M = pt.w[me].matrix + parity * kMat;  // full matrix (every row published)
   for (int d = threadIdx.x; d < G; d += blockDim.x) {
     unsigned long long start = 0;  // earlier sources' share of destination d
     for (int s = 0; s < me; ++s) start += M[s * kMaxG + d];
@@ -203,7 +212,9 @@ struct FusedState {
   uint64_t* tmp_pf = nullptr; uint64_t tmp_pf_cap = 0;
   uint8_t* tmp_v = nullptr; uint64_t tmp_v_cap = 0;
   unsigned long long* cnt = nullptr;  // 2 x kMaxG: counts, cursors
+  unsigned long long* h_mat = nullptr;  // pinned host copy of one count matrix
   uint32_t epoch = 0;
+  uint64_t batch = 0;                 // parity of the count matrix
 };
 
 void fused_free(hbt_tree* t) {
@@ -212,6 +223,7 @@ void fused_free(hbt_tree* t) {
   for (int g = 0; g < kMaxG; ++g)
     if (f->peer[g] && f->peer[g] != f->win) cudaIpcCloseMemHandle(f->peer[g]);
   cudaFree(f->win); cudaFree(f->dest); cudaFree(f->tmp_pf); cudaFree(f->tmp_v); cudaFree(f->cnt);
+  if (f->h_mat) cudaFreeHost(f->h_mat);
   delete f;
   t->fused = nullptr;
 }
@@ -227,7 +239,7 @@ int alloc_window(FusedState* f, uint64_t cap_m, uint64_t cap_r, uint32_t S) {
   cudaFree(f->win);
   f->win = nullptr;
   HBT_CUDA_TRY(cudaMalloc(&f->win, win_bytes(cap_m, cap_r, S)));
-  HBT_CUDA_TRY(cudaMemset(f->win, 0, 256 * ((kMaxG * 4 + 255) / 256)));  // flags
+  HBT_CUDA_TRY(cudaMemset(f->win, 0, 256 * ((kMaxG * 4 + 255) / 256) + 2 * kMat * 8));  // flags + matrices
   f->cap_m = cap_m;
   f->cap_r = cap_r;
   f->epoch = 0;
@@ -238,6 +250,7 @@ int prep_local(FusedState* f, uint64_t m) {
   int rc;
   if ((rc = ensure(&f->dest, &f->dest_cap, m ? m : 1))) return rc;
   if (!f->cnt) HBT_CUDA_TRY(cudaMalloc(&f->cnt, 2 * kMaxG * sizeof(unsigned long long)));
+  if (!f->h_mat) HBT_CUDA_TRY(cudaMallocHost(&f->h_mat, kMat * sizeof(unsigned long long)));
   return HBT_OK;
 }
 
@@ -252,10 +265,11 @@ int route_and_count(FusedState* f, const K* q, uint64_t m, const RouteTab& rt, i
 }
 
 template <typename K>
-int put_queries(FusedState* f, const K* q, uint64_t m, const PeerTable& pt, int me, cudaStream_t st) {
+int put_queries(FusedState* f, const K* q, uint64_t m, const PeerTable& pt, int me, int parity, cudaStream_t st) {
   if (!m) return HBT_OK;
   const uint64_t chunk = 4096;
-  f_put<K><<<unsigned((m + chunk - 1) / chunk), kThreads, 0, st>>>(q, m, f->dest, pt, me, f->cnt + kMaxG, chunk);
+  f_put<K><<<unsigned((m + chunk - 1) / chunk), kThreads, 0, st>>>(q, m, f->dest, pt, me, parity, f->cnt + kMaxG,
+                                                                   chunk);
   HBT_CUDA_TRY(cudaGetLastError());
   return HBT_OK;
 }
@@ -263,10 +277,22 @@ int put_queries(FusedState* f, const K* q, uint64_t m, const PeerTable& pt, int 
 template <typename K>
 int search_and_return(hbt_tree* t, FusedState* f, const PeerTable& pt, int me, uint64_t nrecv, cudaStream_t st) {
   int rc;
-  if ((rc = ensure(&f->tmp_pf, &f->tmp_pf_cap, nrecv ? nrecv : 1))) return rc;
-  if ((rc = ensure(&f->tmp_v, &f->tmp_v_cap, (nrecv ? nrecv : 1) * sizeof(K)))) return rc;
   if (!nrecv) return HBT_OK;
   const Win& w = pt.w[me];
+  if (bucketed_enabled(t, nrecv)) {
+    // fused return: the bucketed search's gather stores each result straight into the
+    // requester's result window (no staging, no f_return pass)
+    RemoteOut ro;
+    ro.org = w.recv_org;
+    for (int g = 0; g < pt.G; ++g) {
+      ro.pf[g] = pt.w[g].res_pf;
+      ro.v[g] = pt.w[g].res_v;
+    }
+    rc = bucketed_search(t, w.recv_q, nrecv, nullptr, nullptr, t->shard.base[me], st, &ro);
+    if (rc != HBT_EUNSUPPORTED) return rc;  // EUNSUPPORTED: no item directory, stage + f_return
+  }
+  if ((rc = ensure(&f->tmp_pf, &f->tmp_pf_cap, nrecv))) return rc;
+  if ((rc = ensure(&f->tmp_v, &f->tmp_v_cap, nrecv * sizeof(K)))) return rc;
   rc = shard_local_search(t, w.recv_q, nrecv, f->tmp_pf, f->tmp_v, t->shard.base[me], st);
   if (rc) return rc;
   f_return<K><<<grid_for(nrecv), kThreads, 0, st>>>(pt, me, nrecv, f->tmp_pf, (const K*)f->tmp_v);
@@ -310,11 +336,11 @@ int local_t(hbt_tree* const* shards, int G, const void* const* queries, const ui
     pt.w[g] = carve(fs[g]->win, fs[g]->cap_m, fs[g]->cap_r, S);
   }
   for (int s = 0; s < G; ++s) {
-    f_publish<<<1, 256, 0, st>>>(pt, s, fs[s]->cnt);
+    f_publish<<<1, 256, 0, st>>>(pt, s, fs[s]->cnt, 0);
     HBT_CUDA_TRY(cudaGetLastError());
   }
   for (int s = 0; s < G; ++s) {
-    int rc = put_queries<K>(fs[s], (const K*)queries[s], m[s], pt, s, st);
+    int rc = put_queries<K>(fs[s], (const K*)queries[s], m[s], pt, s, 0, st);
     if (rc) return rc;
   }
   for (int d = 0; d < G; ++d) {
@@ -344,9 +370,17 @@ int local_t(hbt_tree* const* shards, int G, const void* const* queries, const ui
 
 // (Re)allocate this rank's window and map every peer's (collective).
 int exchange_windows(FusedState* f, hbt_comm* c, uint64_t cap_m, uint64_t cap_r, uint32_t S, cudaStream_t st) {
+  HBT_CUDA_TRY(cudaStreamSynchronize(st));  // no kernel of ours still touches a peer window
   for (int g = 0; g < kMaxG; ++g) {
     if (f->peer[g] && f->peer[g] != f->win) cudaIpcCloseMemHandle(f->peer[g]);
     f->peer[g] = nullptr;
+  }
+  if (f->win) {
+    // every peer must have closed its mapping of our old window before it is freed
+    uint8_t one = 1;
+    std::vector<uint8_t> all(c->nranks);
+    int rc0 = comm_allgather_host(c, &one, all.data(), 1, st);
+    if (rc0) return rc0;
   }
   int rc = alloc_window(f, cap_m, cap_r, S);
   if (rc) return rc;
@@ -372,17 +406,32 @@ int nccl_fused_t(hbt_tree* t, const void* queries, uint64_t m, hbt_out out, cuda
   FusedState* f = state_of(t);
   int rc = prep_local(f, m);
   if (rc) return rc;
-  // agree on window capacities: every rank needs m_s <= cap_m and recv_d <= cap_r.
-  // The count row is all-gathered by NCCL once per batch on the host path (small),
-  // the data path itself is peer stores.
   const RouteTab rt = table_of(t->shard);
   rc = route_and_count<K>(f, (const K*)queries, m, rt, G, st);
   if (rc) return rc;
-  std::vector<unsigned long long> mine(G), mat(G * G);
-  HBT_CUDA_TRY(cudaMemcpyAsync(mine.data(), f->cnt, G * 8, cudaMemcpyDeviceToHost, st));
-  HBT_CUDA_TRY(cudaStreamSynchronize(st));
-  rc = comm_allgather_host(c, mine.data(), mat.data(), G * 8, st);
-  if (rc) return rc;
+  const int par = int(f->batch & 1);
+  std::vector<unsigned long long> mat(G * G);
+  PeerTable pt{};
+  pt.G = G;
+  const bool had_windows = f->win != nullptr;
+  if (had_windows) {
+    // steady state: the count rows travel by peer stores, no host collective
+    for (int g = 0; g < G; ++g) pt.w[g] = carve(f->peer[g], f->cap_m, f->cap_r, S);
+    f_publish<<<1, 256, 0, st>>>(pt, me, f->cnt, par);
+    f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);
+    HBT_CUDA_TRY(cudaGetLastError());
+    HBT_CUDA_TRY(cudaMemcpyAsync(f->h_mat, pt.w[me].matrix + par * kMat, kMat * 8, cudaMemcpyDeviceToHost, st));
+    HBT_CUDA_TRY(cudaStreamSynchronize(st));
+    for (int s = 0; s < G; ++s)
+      for (int x = 0; x < G; ++x) mat[s * G + x] = f->h_mat[s * kMaxG + x];
+  } else {
+    // first batch: no windows to store into yet; the count rows go through the host
+    std::vector<unsigned long long> mine(G);
+    HBT_CUDA_TRY(cudaMemcpyAsync(mine.data(), f->cnt, G * 8, cudaMemcpyDeviceToHost, st));
+    HBT_CUDA_TRY(cudaStreamSynchronize(st));
+    rc = comm_allgather_host(c, mine.data(), mat.data(), G * 8, st);
+    if (rc) return rc;
+  }
   uint64_t need_m = 1, need_r = 1;
   for (int x = 0; x < G; ++x) {
     uint64_t row = 0, col = 0;
@@ -390,21 +439,18 @@ int nccl_fused_t(hbt_tree* t, const void* queries, uint64_t m, hbt_out out, cuda
     need_m = std::max<uint64_t>(need_m, row);
     need_r = std::max<uint64_t>(need_r, col);
   }
-  if (!f->win || f->cap_m < need_m || f->cap_r < need_r) {
+  if (!had_windows || f->cap_m < need_m || f->cap_r < need_r) {
+    // every rank holds the same matrix, so every rank takes this branch (collective)
     rc = exchange_windows(f, c, need_m + need_m / 8, need_r + need_r / 8, S, st);
     if (rc) return rc;
+    for (int g = 0; g < G; ++g) pt.w[g] = carve(f->peer[g], f->cap_m, f->cap_r, S);
+    std::vector<unsigned long long> full(kMat, 0);
+    for (int s = 0; s < G; ++s)
+      for (int x = 0; x < G; ++x) full[s * kMaxG + x] = mat[s * G + x];
+    HBT_CUDA_TRY(cudaMemcpyAsync(pt.w[me].matrix + par * kMat, full.data(), kMat * 8, cudaMemcpyHostToDevice, st));
+    f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);  // every window exists and holds its matrix
   }
-  PeerTable pt{};
-  pt.G = G;
-  for (int g = 0; g < G; ++g) pt.w[g] = carve(f->peer[g], f->cap_m, f->cap_r, S);
-  // the full matrix is known: write it into our own window (no peer publish needed)
-  std::vector<unsigned long long> full(kMaxG * kMaxG, 0);
-  for (int s = 0; s < G; ++s)
-    for (int x = 0; x < G; ++x) full[s * kMaxG + x] = mat[s * G + x];
-  HBT_CUDA_TRY(cudaMemcpyAsync(pt.w[me].matrix, full.data(), full.size() * 8, cudaMemcpyHostToDevice, st));
-  // everybody's previous batch must be finished with our windows
-  f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);
-  rc = put_queries<K>(f, (const K*)queries, m, pt, me, st);
+  rc = put_queries<K>(f, (const K*)queries, m, pt, me, par, st);
   if (rc) return rc;
   f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);
   uint64_t nrecv = 0;
@@ -417,6 +463,7 @@ int nccl_fused_t(hbt_tree* t, const void* queries, uint64_t m, hbt_out out, cuda
     HBT_CUDA_TRY(cudaMemcpyAsync(out.pos_found, pt.w[me].res_pf, m * 8, cudaMemcpyDeviceToDevice, st));
     HBT_CUDA_TRY(cudaMemcpyAsync(out.values, pt.w[me].res_v, m * S, cudaMemcpyDeviceToDevice, st));
   }
+  ++f->batch;
   return HBT_OK;
 }
 

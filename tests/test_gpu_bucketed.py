@@ -49,7 +49,6 @@ def test_bucketed_edge_suite(hbt, layout, width, F, items, cap, leaf256):
         t.set_param("leaf256", leaf256)
         for slice_bytes in (1, 4096, 1 << 16):  # 1 B: one bucket per unit up to the 1024 cap
             t.set_param("bucket_slice", slice_bytes)
-            t.set_param("scatter_pair", int(slice_bytes != 4096))  # one-chunk (default) and paired scatter
             t.set_param("item_group4", int(slice_bytes == 4096))
             pf, val = gpu_search(t, q, width)
             assert np.array_equal(pf, epf), (layout, n, F, width, slice_bytes, items, cap,
@@ -77,7 +76,6 @@ def test_bucketed_scaled_workload(hbt, layout, F, items, cap, leaf256):
         t.set_param("bucket_slice", slice_bytes)
         for qpf in (0, 1):  # with / without the bulk L2 prefetch of each item's queries
             t.set_param("qprefetch", qpf)
-            t.set_param("scatter_pair", 1 - qpf)  # both scatter kernels
             t.set_param("item_group4", qpf)  # 2- and 4-lane groups in the implicit item search
             for hint in (0, 1, 3):  # L2 eviction-priority hints on the item search's loads
                 t.set_param("item_l2_hint" if layout == "implicit" else "regular_l2_hint", hint)
@@ -171,7 +169,7 @@ def test_c3_full_size_bench_launch(hbt):
     t.set_param("phase_timing", 1)
     pf, val = t.search(dq)
     torch.cuda.synchronize()
-    assert t.last_phases()["launches"] == 9  # count, transpose, scan x2, transpose, starts, scatter, search, gather
+    assert t.last_phases()["launches"] == 5  # count, run starts, scatter, search, gather
     pf = pf.cpu().numpy().view(np.uint64)
     val = from_dev(val, 8)
     u = gen.uniform_indices(m, n + n_ins, sq).astype(np.int64)

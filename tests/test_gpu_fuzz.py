@@ -73,7 +73,6 @@ def test_random_knob_parity(hbt, case):
     knobs["l2_hint"] = int(hrng.integers(0, 5))
     knobs["item_l2_hint"] = int(hrng.integers(0, 4))
     knobs["regular_l2_hint"] = int(hrng.integers(0, 4))
-    knobs["scatter_pair"] = int(hrng.integers(0, 2))
     knobs["item_group4"] = int(hrng.integers(0, 2))
     knobs["small_threads"] = int(hrng.choice([0, 128, 256, 1024]))
     for name, val in knobs.items():

@@ -20,6 +20,7 @@ import paper_conf_sigmod_shahvaranij16_b200 as hbt  # noqa: E402
 
 def main():
     exchange = int(sys.argv[1]) if len(sys.argv) > 1 else 0
+    bucket = int(sys.argv[2]) if len(sys.argv) > 2 else 2  # 1: owner search bucketed (fused remote gather)
     dist.init_process_group("gloo")
     rank, world = dist.get_rank(), dist.get_world_size()
     torch.cuda.set_device(0)
@@ -32,11 +33,16 @@ def main():
     v = torch.from_numpy(allv[lo:hi].view(np.int64)).cuda()
     t = hbt.ShardedTree(comm, k, v, fanout=16)
     t.set_param("exchange", exchange)
+    t.set_param("bucket", bucket)
+    if bucket == 1:
+        t.set_param("bucket_slice", 4096)
     full = oracle.ITree.from_pairs(allk, allv, 16, 8)
     ok = True
-    for rep in range(3):
+    # batch sizes grow (window regrowth, a collective re-export) and shrink; several
+    # batches in a row exercise the device-side count publication (matrix parity)
+    for rep, mq in enumerate([30000, 90000, 20000, 250000, 10000, 400000, 5000]):
         rng = np.random.default_rng(100 * rank + rep)
-        q = np.concatenate([allk[rng.integers(0, n, 30000 * (rep + 1))],
+        q = np.concatenate([allk[rng.integers(0, n, mq * (rank + 1))],
                             rng.integers(0, 2**64 - 1, 5000, dtype=np.uint64, endpoint=True)])
         pf, vals = t.search(torch.from_numpy(q.view(np.int64)).cuda())
         torch.cuda.synchronize()
