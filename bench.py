@@ -704,7 +704,7 @@ def run_hbt(args):
         if streamed:  # partition (count, run starts, scatter) + one search per bucket + gather
             slice_b = int(dict(kv.split("=", 1) for kv in args.param).get("stream_slice", "0"), 0) or (8 << 20)
             nb = min(1024, -(-info["leaf_bytes"] // slice_b), info["leaf_lines"])
-            launches_per_step = 4 + nb
+            launches_per_step = 5 + nb
     if m <= (1 << 20) and not args.range_k:
         roof["note"] = ("latency-bound batch: %d queries are one wave of the GPU, so the step is the launch "
                         "plus one query's chain of dependent memory round trips; no byte roofline binds" % m)

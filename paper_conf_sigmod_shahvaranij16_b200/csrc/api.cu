@@ -214,6 +214,7 @@ const char* hbt_version(void) { return "hbt 0.1 (HB+-tree lookups, sm_100a)"; }
 
 int hbt_bulk_build(const void* keys, const void* values, uint64_t n, uint32_t fanout, uint32_t layout,
                    void* stream, hbt_tree** out) {
+  NvtxRange nvtx_("hbt_bulk_build");
   g_err.clear();
   if (!out) { set_error("out is NULL"); return HBT_EINVAL; }
   *out = nullptr;
@@ -253,6 +254,7 @@ int hbt_bulk_build(const void* keys, const void* values, uint64_t n, uint32_t fa
 }
 
 int hbt_search(const hbt_tree* t, const void* queries, uint64_t m, hbt_out out, void* stream) {
+  NvtxRange nvtx_("hbt_search");
   if (!t) { set_error("tree is NULL"); return HBT_EINVAL; }
   if (m == 0) return HBT_OK;
   if (!is_device_ptr(queries) || !is_device_ptr(out.pos_found) || !is_device_ptr(out.values)) {
@@ -264,6 +266,7 @@ int hbt_search(const hbt_tree* t, const void* queries, uint64_t m, hbt_out out, 
 
 int hbt_search_host(const hbt_tree* t, const void* host_queries, uint64_t m, uint64_t* host_pos_found,
                     void* host_values, void* stream) {
+  NvtxRange nvtx_("hbt_search_host");
   if (!t) { set_error("tree is NULL"); return HBT_EINVAL; }
   if (m == 0) return HBT_OK;
   if (!host_queries || !host_pos_found || !host_values) { set_error("NULL host buffer"); return HBT_EINVAL; }
@@ -319,6 +322,7 @@ int hbt_search_host(const hbt_tree* t, const void* host_queries, uint64_t m, uin
 
 int hbt_range(const hbt_tree* t, const void* lo, const void* hi, uint64_t m, uint32_t k, void* out_keys,
               void* out_values, uint32_t* out_count, void* stream) {
+  NvtxRange nvtx_("hbt_range");
   if (!t) { set_error("tree is NULL"); return HBT_EINVAL; }
   if (m == 0) return HBT_OK;
   if (k == 0 || k > 4096) { set_error("k must be in [1, 4096]"); return HBT_EINVAL; }
@@ -331,6 +335,7 @@ int hbt_range(const hbt_tree* t, const void* lo, const void* hi, uint64_t m, uin
 }
 
 int hbt_bulk_update(hbt_tree* t, const hbt_batch* batch, void* stream) {
+  NvtxRange nvtx_("hbt_bulk_update");
   if (!t || !batch) { set_error("tree/batch is NULL"); return HBT_EINVAL; }
   if (batch->count == 0) return HBT_OK;
   if (!is_device_ptr(batch->keys) || !is_device_ptr(batch->values) || !is_device_ptr(batch->ops)) {

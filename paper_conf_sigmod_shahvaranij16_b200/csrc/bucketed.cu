@@ -266,28 +266,52 @@ __global__ void __launch_bounds__(kScanThreads) bk_seg_scan(const uint32_t* __re
   if (b == 0) bstart[B] = m;
 }
 
-// Per-chunk bucket layout shared by the scatter and the gather: s_cnt (this chunk's
-// count per bucket, from tab) and s_lb (their exclusive scan = the bucket's start in
-// the chunk's bucket-sorted order).  s_gb (the run's first global slot) is the
-// caller's running per-bucket offset.
+// Run start of every (chunk, bucket), chunk-major: gb[c * B + b] = segoff[j][b] + the
+// counts of segment j's earlier chunks (one CTA per segment walks its chunks in order;
+// rows are coalesced).  The scatter and the gather take chunks interleaved over the
+// CTAs (c = blockIdx, blockIdx + grid, ...): the runs they write / read at the same
+// time are then neighbours in memory and share L2 lines and DRAM pages (contiguous
+// per-CTA segments measured slower: c4 scatter 1.95 -> 2.57 ms, gather 2.14 -> 2.44).
+__global__ void __launch_bounds__(kScanThreads) bk_run_starts(const uint32_t* __restrict__ tab,
+                                                              const uint32_t* __restrict__ segoff, uint32_t B,
+                                                              uint64_t chunks, uint64_t kps,
+                                                              uint32_t* __restrict__ gb) {
+  const uint64_t j = blockIdx.x;
+  const uint32_t b = threadIdx.x;
+  if (b >= B) return;
+  const uint64_t c0 = j * kps, c1 = c0 + kps < chunks ? c0 + kps : chunks;
+  uint32_t run = segoff[j * B + b];
+#pragma unroll 4
+  for (uint64_t c = c0; c < c1; ++c) {
+    const uint32_t x = tab[c * B + b];
+    gb[c * B + b] = run;
+    run += x;
+  }
+}
+
+// Per-chunk bucket layout shared by the scatter and the gather (tab, gb
+// chunk-major): s_cnt (this chunk's count per bucket), s_lb (their exclusive scan = the
+// bucket's start in the chunk's bucket-sorted order), s_gb (the run's first global slot).
 template <int TH = kThreads>
-__device__ __forceinline__ void chunk_layout(const uint32_t* __restrict__ tab, uint32_t B, uint64_t c, uint32_t* s_cnt,
-                                             uint32_t* s_lb, uint32_t* s_tmp) {
-  for (uint32_t b = threadIdx.x; b < B; b += TH) s_cnt[b] = tab[c * B + b];  // chunk-major row: coalesced
+__device__ __forceinline__ void chunk_layout(const uint32_t* __restrict__ tab, const uint32_t* __restrict__ gb,
+                                             uint32_t B, uint64_t c, uint32_t* s_cnt, uint32_t* s_lb, uint32_t* s_gb,
+                                             uint32_t* s_tmp) {
+  for (uint32_t b = threadIdx.x; b < B; b += TH) {  // chunk-major rows: coalesced
+    s_cnt[b] = tab[c * B + b];
+    s_gb[b] = gb[c * B + b];
+  }
   __syncthreads();
   block_exclusive_scan<TH>(s_cnt, s_lb, B, s_tmp);
 }
 
-// Pass 2: per segment, chunk after chunk: each chunk's queries are ordered by bucket
-// in shared memory, then written as B contiguous runs, the run of bucket b at the
-// segment's running offset s_gb[b] (segoff + the segment's earlier chunks' counts);
+// Pass 2: each chunk's queries are ordered by bucket in shared memory, then
+// written as B contiguous runs (the run of bucket b at global slot gb[c][b]);
 // linv[i] (u16) = the query's position in the chunk's bucket-sorted order.
 template <typename K>
 __global__ void __launch_bounds__(kThreads, 2) bk_scatter(const K* __restrict__ q, uint64_t m,
                                                        const uint16_t* __restrict__ bq, const uint32_t* __restrict__ tab,
-                                                       const uint32_t* __restrict__ segoff, uint32_t B, uint64_t chunks,
-                                                       uint64_t kps, uint64_t nseg, K* __restrict__ qs,
-                                                       uint16_t* __restrict__ linv) {
+                                                       const uint32_t* __restrict__ gb, uint32_t B, uint64_t chunks,
+                                                       K* __restrict__ qs, uint16_t* __restrict__ linv) {
   extern __shared__ __align__(16) uint8_t smem[];
   K* s_q = reinterpret_cast<K*>(smem);
   uint16_t* s_b = reinterpret_cast<uint16_t*>(s_q + kChunk);
@@ -298,65 +322,53 @@ __global__ void __launch_bounds__(kThreads, 2) bk_scatter(const K* __restrict__ 
   uint32_t* s_tmp = s_rank + kMaxBuckets;
   // the chunk's queries and bucket ids are loaded before its layout row is scanned,
   // so the two DRAM round trips overlap
-  constexpr int LPT = int(kMaxBuckets) / kThreads;  // layout entries per thread (thread-owned buckets)
-  for (uint64_t j = blockIdx.x; j < nseg; j += gridDim.x) {
-    const uint64_t c0 = j * kps, c1 = c0 + kps < chunks ? c0 + kps : chunks;
+  constexpr int LPT = int(kMaxBuckets) / kThreads;  // layout entries per thread
+  for (uint64_t c = blockIdx.x; c < chunks; c += gridDim.x) {
+    const uint64_t lo = c * kChunk;
+    const uint32_t nc = uint32_t(m - lo < kChunk ? m - lo : kChunk);
+    K qq[kQPT];
+    uint32_t bb[kQPT];
+#pragma unroll
+    for (int x = 0; x < kQPT; ++x) {
+      const uint32_t t = uint32_t(x) * kThreads + threadIdx.x;
+      qq[x] = K(0);
+      bb[x] = 0;
+      if (t < nc) {
+        qq[x] = __ldcs(q + lo + t);
+        bb[x] = __ldcs(reinterpret_cast<const unsigned short*>(bq) + lo + t);
+      }
+    }
 #pragma unroll
     for (int e = 0; e < LPT; ++e) {
       const uint32_t b = uint32_t(e) * kThreads + threadIdx.x;
-      if (b < B) s_gb[b] = segoff[j * B + b];
-    }
-    for (uint64_t c = c0; c < c1; ++c) {
-      const uint64_t lo = c * kChunk;
-      const uint32_t nc = uint32_t(m - lo < kChunk ? m - lo : kChunk);
-      K qq[kQPT];
-      uint32_t bb[kQPT];
-#pragma unroll
-      for (int x = 0; x < kQPT; ++x) {
-        const uint32_t t = uint32_t(x) * kThreads + threadIdx.x;
-        qq[x] = K(0);
-        bb[x] = 0;
-        if (t < nc) {
-          qq[x] = __ldcs(q + lo + t);
-          bb[x] = __ldcs(reinterpret_cast<const unsigned short*>(bq) + lo + t);
-        }
-      }
-#pragma unroll
-      for (int e = 0; e < LPT; ++e) {
-        const uint32_t b = uint32_t(e) * kThreads + threadIdx.x;
-        if (b < B) {
-          s_rank[b] = 0;
-          s_cnt[b] = tab[c * B + b];
-        }
-      }
-      __syncthreads();
-      block_exclusive_scan(s_cnt, s_lb, B, s_tmp);
-#pragma unroll
-      for (int x = 0; x < kQPT; ++x) {
-        const uint32_t t = uint32_t(x) * kThreads + threadIdx.x;
-        if (t < nc) {
-          const uint32_t pos = s_lb[bb[x]] + atomicAdd(&s_rank[bb[x]], 1u);
-          s_q[pos] = qq[x];
-          s_b[pos] = uint16_t(bb[x]);
-          __stcs(reinterpret_cast<unsigned short*>(linv) + lo + t, (unsigned short)pos);
-        }
-      }
-      __syncthreads();
-#pragma unroll
-      for (int x = 0; x < kQPT; ++x) {
-        const uint32_t t = uint32_t(x) * kThreads + threadIdx.x;
-        if (t < nc) {
-          const uint32_t b = s_b[t];
-          qs[uint64_t(s_gb[b]) + (t - s_lb[b])] = s_q[t];
-        }
-      }
-      __syncthreads();
-#pragma unroll
-      for (int e = 0; e < LPT; ++e) {  // the next chunk's runs follow this one's
-        const uint32_t b = uint32_t(e) * kThreads + threadIdx.x;
-        if (b < B) s_gb[b] += s_cnt[b];
+      if (b < B) {
+        s_rank[b] = 0;
+        s_cnt[b] = tab[c * B + b];
+        s_gb[b] = gb[c * B + b];
       }
     }
+    __syncthreads();
+    block_exclusive_scan(s_cnt, s_lb, B, s_tmp);
+#pragma unroll
+    for (int x = 0; x < kQPT; ++x) {
+      const uint32_t t = uint32_t(x) * kThreads + threadIdx.x;
+      if (t < nc) {
+        const uint32_t pos = s_lb[bb[x]] + atomicAdd(&s_rank[bb[x]], 1u);
+        s_q[pos] = qq[x];
+        s_b[pos] = uint16_t(bb[x]);
+        __stcs(reinterpret_cast<unsigned short*>(linv) + lo + t, (unsigned short)pos);
+      }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int x = 0; x < kQPT; ++x) {
+      const uint32_t t = uint32_t(x) * kThreads + threadIdx.x;
+      if (t < nc) {
+        const uint32_t b = s_b[t];
+        qs[uint64_t(s_gb[b]) + (t - s_lb[b])] = s_q[t];
+      }
+    }
+    __syncthreads();
   }
 }
 
@@ -364,9 +376,8 @@ __global__ void __launch_bounds__(kThreads, 2) bk_scatter(const K* __restrict__ 
 // shared memory (bucket-sorted order), then stored in query order through linv.
 template <typename K>
 __global__ void __launch_bounds__(kThreads, 2) bk_gather(const uint16_t* __restrict__ linv, uint64_t m,
-                                                      const uint32_t* __restrict__ tab, const uint32_t* __restrict__ segoff,
-                                                      uint32_t B, uint64_t chunks, uint64_t kps, uint64_t nseg,
-                                                      const uint64_t* __restrict__ pf_s,
+                                                      const uint32_t* __restrict__ tab, const uint32_t* __restrict__ gb,
+                                                      uint32_t B, uint64_t chunks, const uint64_t* __restrict__ pf_s,
                                                       const K* __restrict__ v_s, uint64_t* __restrict__ out_pf,
                                                       K* __restrict__ out_v) {
   extern __shared__ __align__(16) uint8_t smem[];
@@ -376,13 +387,10 @@ __global__ void __launch_bounds__(kThreads, 2) bk_gather(const uint16_t* __restr
   uint32_t* s_lb = s_cnt + kMaxBuckets;
   uint32_t* s_gb = s_lb + kMaxBuckets;
   uint32_t* s_tmp = s_gb + kMaxBuckets;
-  for (uint64_t sj = blockIdx.x; sj < nseg; sj += gridDim.x) {
-  const uint64_t c0 = sj * kps, c1 = c0 + kps < chunks ? c0 + kps : chunks;
-  for (uint32_t b = threadIdx.x; b < B; b += kThreads) s_gb[b] = segoff[sj * B + b];  // thread-owned buckets
-  for (uint64_t c = c0; c < c1; ++c) {
+  for (uint64_t c = blockIdx.x; c < chunks; c += gridDim.x) {
     const uint64_t lo = c * kChunk;
     const uint32_t nc = uint32_t(m - lo < kChunk ? m - lo : kChunk);
-    chunk_layout(tab, B, c, s_cnt, s_lb, s_tmp);
+    chunk_layout(tab, gb, B, c, s_cnt, s_lb, s_gb, s_tmp);
     for (uint32_t b = threadIdx.x; b < B; b += kThreads)
       for (uint32_t k = 0, n = s_cnt[b], p = s_lb[b]; k < n; ++k) s_b[p + k] = uint16_t(b);
     __syncthreads();
@@ -441,8 +449,6 @@ __global__ void __launch_bounds__(kThreads, 2) bk_gather(const uint16_t* __restr
       }
     }
     __syncthreads();
-    for (uint32_t b = threadIdx.x; b < B; b += kThreads) s_gb[b] += s_cnt[b];
-  }
   }
 }
 
@@ -455,18 +461,17 @@ constexpr int kGThreads = 1024;
 template <typename K, bool REMOTE>
 __global__ void __launch_bounds__(kGThreads) bk_gather_rec(const uint16_t* __restrict__ linv, uint64_t m,
                                                            const uint32_t* __restrict__ tab,
-                                                           const uint32_t* __restrict__ segoff, uint32_t B,
-                                                           uint64_t chunks, uint64_t kps, uint64_t nseg,
-                                                           const ulonglong2* __restrict__ rec,
+                                                           const uint32_t* __restrict__ gb, uint32_t B,
+                                                           uint64_t chunks, const ulonglong2* __restrict__ rec,
                                                            uint64_t* __restrict__ out_pf, K* __restrict__ out_v,
                                                            const RemoteOut ro) {
-  // B <= kMaxBuckets == kGThreads: thread b owns bucket b's layout entries and its
-  // running run offset.  The next chunk's layout row is loaded while this chunk's
-  // records are stored, and all of a thread's record and linv loads are issued
-  // together (the kernel was latency bound: long-scoreboard stalls 38 per issue, one
-  // CTA per SM).  REMOTE (the owner side of the fused sharded exchange): query i of
-  // the receive window came from rank org[i] >> 40, index org[i] & (2^40 - 1) there,
-  // and its record is stored straight into THAT rank's result window (peer memory).
+  // B <= kMaxBuckets == kGThreads: thread b owns bucket b's layout entries.  The next
+  // chunk's layout row is loaded while this chunk's records are stored, and all of a
+  // thread's record and linv loads are issued together (the kernel was latency
+  // bound: long-scoreboard stalls 38 per issue, one CTA per SM).  REMOTE (the owner
+  // side of the fused sharded exchange): query i of the receive window came from
+  // rank org[i] >> 40, index org[i] & (2^40 - 1) there, and its record is stored
+  // straight into THAT rank's result window (peer memory).
   static_assert(kMaxBuckets <= kGThreads, "one bucket per thread");
   constexpr int PT = int(kChunk) / kGThreads;
   extern __shared__ __align__(16) uint8_t smem[];
@@ -474,80 +479,84 @@ __global__ void __launch_bounds__(kGThreads) bk_gather_rec(const uint16_t* __res
   uint16_t* s_b = reinterpret_cast<uint16_t*>(s_rec + kChunk);
   uint32_t* s_cnt = reinterpret_cast<uint32_t*>(s_b + kChunk);
   uint32_t* s_lb = s_cnt + kMaxBuckets;
-  uint32_t* s_tmp = s_lb + kMaxBuckets;
+  uint32_t* s_gb = s_lb + kMaxBuckets;
+  uint32_t* s_tmp = s_gb + kMaxBuckets;
   const uint32_t tb = threadIdx.x;
-  for (uint64_t sj = blockIdx.x; sj < nseg; sj += gridDim.x) {
-    const uint64_t c0 = sj * kps, c1 = c0 + kps < chunks ? c0 + kps : chunks;
-    uint32_t run = tb < B ? segoff[sj * B + tb] : 0u;
-    uint32_t nx_cnt = tb < B ? tab[c0 * B + tb] : 0u;
-    for (uint64_t c = c0; c < c1; ++c) {
-      const uint64_t lo = c * kChunk;
-      const uint32_t nc = uint32_t(m - lo < kChunk ? m - lo : kChunk);
-      const uint32_t gbt = run;  // this chunk's run of bucket tb starts here
-      if (tb < B) s_cnt[tb] = nx_cnt;
-      __syncthreads();
-      block_exclusive_scan<kGThreads>(s_cnt, s_lb, B, s_tmp);
-      if (tb < B) {
-        for (uint32_t k = 0, n = s_cnt[tb], p = s_lb[tb]; k < n; ++k) s_b[p + k] = uint16_t(tb);
-        run += s_cnt[tb];
+  uint32_t nx_cnt = 0, nx_gb = 0;
+  if (blockIdx.x < chunks && tb < B) {
+    nx_cnt = tab[uint64_t(blockIdx.x) * B + tb];
+    nx_gb = gb[uint64_t(blockIdx.x) * B + tb];
+  }
+  for (uint64_t c = blockIdx.x; c < chunks; c += gridDim.x) {
+    const uint64_t lo = c * kChunk;
+    const uint32_t nc = uint32_t(m - lo < kChunk ? m - lo : kChunk);
+    if (tb < B) {
+      s_cnt[tb] = nx_cnt;
+      s_gb[tb] = nx_gb;
+    }
+    __syncthreads();
+    block_exclusive_scan<kGThreads>(s_cnt, s_lb, B, s_tmp);
+    if (tb < B)
+      for (uint32_t k = 0, n = s_cnt[tb], p = s_lb[tb]; k < n; ++k) s_b[p + k] = uint16_t(tb);
+    __syncthreads();
+    const unsigned short* li = reinterpret_cast<const unsigned short*>(linv) + lo;
+    ulonglong2 x[PT];
+    unsigned short l[PT];
+#pragma unroll
+    for (int j = 0; j < PT; ++j) {
+      const uint32_t t = uint32_t(j) * kGThreads + tb;
+      if (t < nc) {
+        const uint32_t b = s_b[t];
+        x[j] = __ldcs(rec + s_gb[b] + (t - s_lb[b]));
+        l[j] = __ldcs(li + t);
       }
-      // run starts of this chunk by bucket: s_cnt is free again after the scan, reuse it
-      __syncthreads();
-      if (tb < B) s_cnt[tb] = gbt;
-      __syncthreads();
-      const unsigned short* li = reinterpret_cast<const unsigned short*>(linv) + lo;
-      ulonglong2 x[PT];
-      unsigned short l[PT];
+    }
+    {  // next chunk's layout row, in flight during the stores below
+      const uint64_t cn = c + gridDim.x;
+      if (cn < chunks && tb < B) {
+        nx_cnt = tab[cn * B + tb];
+        nx_gb = gb[cn * B + tb];
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < PT; ++j) {
+      const uint32_t t = uint32_t(j) * kGThreads + tb;
+      if (t < nc) s_rec[t] = x[j];
+    }
+    __syncthreads();
+    if constexpr (REMOTE) {
+      uint64_t o[PT];
+#pragma unroll
+      for (int j = 0; j < PT; ++j) {
+        const uint32_t t = uint32_t(j) * kGThreads + tb;
+        o[j] = t < nc ? __ldcs(reinterpret_cast<const unsigned long long*>(ro.org) + lo + t) : 0ull;
+      }
 #pragma unroll
       for (int j = 0; j < PT; ++j) {
         const uint32_t t = uint32_t(j) * kGThreads + tb;
         if (t < nc) {
-          const uint32_t b = s_b[t];
-          x[j] = __ldcs(rec + s_cnt[b] + (t - s_lb[b]));
-          l[j] = __ldcs(li + t);
+          const ulonglong2 r = s_rec[l[j]];
+          const uint32_t src = uint32_t(o[j] >> kRemoteOrgShift);
+          const uint64_t idx = o[j] & ((1ull << kRemoteOrgShift) - 1);
+          ro.pf[src][idx] = r.x;
+          reinterpret_cast<K*>(ro.v[src])[idx] = K(r.y);
         }
       }
-      if (c + 1 < c1 && tb < B) nx_cnt = tab[(c + 1) * B + tb];  // in flight during the stores below
+    } else {
 #pragma unroll
       for (int j = 0; j < PT; ++j) {
         const uint32_t t = uint32_t(j) * kGThreads + tb;
-        if (t < nc) s_rec[t] = x[j];
-      }
-      __syncthreads();
-      if constexpr (REMOTE) {
-        uint64_t o[PT];
-#pragma unroll
-        for (int j = 0; j < PT; ++j) {
-          const uint32_t t = uint32_t(j) * kGThreads + tb;
-          o[j] = t < nc ? __ldcs(reinterpret_cast<const unsigned long long*>(ro.org) + lo + t) : 0ull;
-        }
-#pragma unroll
-        for (int j = 0; j < PT; ++j) {
-          const uint32_t t = uint32_t(j) * kGThreads + tb;
-          if (t < nc) {
-            const ulonglong2 r = s_rec[l[j]];
-            const uint32_t src = uint32_t(o[j] >> kRemoteOrgShift);
-            const uint64_t idx = o[j] & ((1ull << kRemoteOrgShift) - 1);
-            ro.pf[src][idx] = r.x;
-            reinterpret_cast<K*>(ro.v[src])[idx] = K(r.y);
-          }
-        }
-      } else {
-#pragma unroll
-        for (int j = 0; j < PT; ++j) {
-          const uint32_t t = uint32_t(j) * kGThreads + tb;
-          if (t < nc) {
-            const ulonglong2 r = s_rec[l[j]];
-            __stcs(reinterpret_cast<unsigned long long*>(out_pf) + lo + t, r.x);
-            if constexpr (sizeof(K) == 8)
-              __stcs(reinterpret_cast<unsigned long long*>(out_v) + lo + t, r.y);
-            else
-              __stcs(reinterpret_cast<unsigned int*>(out_v) + lo + t, (unsigned int)r.y);
-          }
+        if (t < nc) {
+          const ulonglong2 r = s_rec[l[j]];
+          __stcs(reinterpret_cast<unsigned long long*>(out_pf) + lo + t, r.x);
+          if constexpr (sizeof(K) == 8)
+            __stcs(reinterpret_cast<unsigned long long*>(out_v) + lo + t, r.y);
+          else
+            __stcs(reinterpret_cast<unsigned int*>(out_v) + lo + t, (unsigned int)r.y);
         }
       }
-      __syncthreads();
     }
+    __syncthreads();
   }
 }
 
@@ -683,12 +692,12 @@ struct Part {
   uint32_t B = 0;
   uint64_t chunks = 0, kps = 0, nseg = 0;
   uint8_t* base = nullptr;
-  uint64_t o_pf = 0, o_v = 0, o_bq = 0, o_li = 0, o_tab = 0, o_seg = 0, o_so = 0, o_bs = 0, total = 0;
+  uint64_t o_pf = 0, o_v = 0, o_bq = 0, o_li = 0, o_tab = 0, o_gb = 0, o_seg = 0, o_so = 0, o_bs = 0, total = 0;
   template <typename T> T* at(uint64_t o) const { return reinterpret_cast<T*>(base + o); }
 };
 
 // qs (m x S) | results: pf_s (m x 8) + v_s (m x 8), or 16 B records over the same
-// 16 m bytes | bq (u16) | linv (u16) | tab (chunks x B) | seg, segoff (nseg x B) |
+// 16 m bytes | bq (u16) | linv (u16) | tab, gb (chunks x B) | seg, segoff (nseg x B) |
 // bucket starts (B + 1)
 template <typename K>
 Part part_layout(uint64_t m, uint32_t B, uint32_t sms) {
@@ -704,7 +713,8 @@ Part part_layout(uint64_t m, uint32_t B, uint32_t sms) {
   p.o_bq = p.o_v + al(m * 8);
   p.o_li = p.o_bq + al(m * 2);
   p.o_tab = p.o_li + al(m * 2);
-  p.o_seg = p.o_tab + al(p.chunks * B * 4);
+  p.o_gb = p.o_tab + al(p.chunks * B * 4);
+  p.o_seg = p.o_gb + al(p.chunks * B * 4);
   p.o_so = p.o_seg + al(p.nseg * B * 4);
   p.o_bs = p.o_so + al(p.nseg * B * 4);
   p.total = p.o_bs + al((uint64_t(B) + 1) * 8);
@@ -715,12 +725,13 @@ constexpr size_t kSmemCount = (1u << kDirBits) * 4 + kMaxBuckets * 4 * 2 + kMaxB
 template <typename K>
 constexpr size_t smem_scatter() { return kChunk * (sizeof(K) + 2) + kMaxBuckets * 4 * 4 + kThreads * 4; }
 constexpr size_t kSmemGather = kChunk * (8 + 2) + kMaxBuckets * 4 * 3 + kThreads * 4;
-constexpr size_t kSmemGatherRec = kChunk * (16 + 2) + kMaxBuckets * 4 * 2 + kGThreads * 4;
+constexpr size_t kSmemGatherRec = kChunk * (16 + 2) + kMaxBuckets * 4 * 3 + kGThreads * 4;
 
 // count -> run starts -> scatter: the batch q in bucket order at qs (Part::base).
 template <typename K>
 int partition(const hbt_tree* t, const BucketState& bs, const void* q, uint64_t m, const Part& p, cudaStream_t s,
               const std::function<void(int)>& mark) {
+  NvtxRange nvtx_("bucket.partition");
   set_bucket_attrs();
   const unsigned grid = unsigned(std::min<uint64_t>(p.nseg, uint64_t(t->num_sms) * 2));
   mark(0);
@@ -730,11 +741,13 @@ int partition(const hbt_tree* t, const BucketState& bs, const void* q, uint64_t 
   mark(1);
   bk_seg_scan<<<1, kScanThreads, 0, s>>>(p.at<uint32_t>(p.o_seg), p.B, p.nseg, m, p.at<uint32_t>(p.o_so),
                                          p.at<uint64_t>(p.o_bs));
+  bk_run_starts<<<unsigned(p.nseg), kScanThreads, 0, s>>>(p.at<uint32_t>(p.o_tab), p.at<uint32_t>(p.o_so), p.B,
+                                                          p.chunks, p.kps, p.at<uint32_t>(p.o_gb));
   mark(2);
-  bk_scatter<K><<<grid, kThreads, smem_scatter<K>(), s>>>((const K*)q, m, p.at<uint16_t>(p.o_bq),
-                                                          p.at<uint32_t>(p.o_tab), p.at<uint32_t>(p.o_so), p.B,
-                                                          p.chunks, p.kps, p.nseg, p.at<K>(0),
-                                                          p.at<uint16_t>(p.o_li));
+  const unsigned sgrid = unsigned(std::min<uint64_t>(p.chunks, uint64_t(t->num_sms) * 2));
+  bk_scatter<K><<<sgrid, kThreads, smem_scatter<K>(), s>>>((const K*)q, m, p.at<uint16_t>(p.o_bq),
+                                                           p.at<uint32_t>(p.o_tab), p.at<uint32_t>(p.o_gb), p.B,
+                                                           p.chunks, p.at<K>(0), p.at<uint16_t>(p.o_li));
   if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) {
     set_error("bucketing kernels failed to launch: %s", cudaGetErrorString(e));
     return HBT_ECUDA;
@@ -794,20 +807,19 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
     mark(4);
     const uint16_t* linv = p.at<uint16_t>(p.o_li);
     const uint32_t* tab = p.at<uint32_t>(p.o_tab);
-    const uint32_t* so = p.at<uint32_t>(p.o_so);
+    const uint32_t* gb = p.at<uint32_t>(p.o_gb);
     if (bs.items) {
-      const unsigned g = unsigned(std::min<uint64_t>(p.nseg, t->num_sms));
+      const unsigned g = unsigned(std::min<uint64_t>(p.chunks, t->num_sms));
       const ulonglong2* rec = reinterpret_cast<const ulonglong2*>(pf_s);
       if (ro)
-        bk_gather_rec<K, true><<<g, kGThreads, kSmemGatherRec, s>>>(linv, m, tab, so, p.B, p.chunks, p.kps, p.nseg,
-                                                                    rec, nullptr, nullptr, *ro);
+        bk_gather_rec<K, true><<<g, kGThreads, kSmemGatherRec, s>>>(linv, m, tab, gb, p.B, p.chunks, rec, nullptr,
+                                                                    nullptr, *ro);
       else
-        bk_gather_rec<K, false><<<g, kGThreads, kSmemGatherRec, s>>>(linv, m, tab, so, p.B, p.chunks, p.kps, p.nseg,
-                                                                     rec, pf, (K*)v, RemoteOut{});
+        bk_gather_rec<K, false><<<g, kGThreads, kSmemGatherRec, s>>>(linv, m, tab, gb, p.B, p.chunks, rec, pf, (K*)v,
+                                                                     RemoteOut{});
     } else {
-      const unsigned g = unsigned(std::min<uint64_t>(p.nseg, uint64_t(t->num_sms) * 2));
-      bk_gather<K><<<g, kThreads, kSmemGather, s>>>(linv, m, tab, so, p.B, p.chunks, p.kps, p.nseg, pf_s, v_s, pf,
-                                                   (K*)v);
+      const unsigned g = unsigned(std::min<uint64_t>(p.chunks, uint64_t(t->num_sms) * 2));
+      bk_gather<K><<<g, kThreads, kSmemGather, s>>>(linv, m, tab, gb, p.B, p.chunks, pf_s, v_s, pf, (K*)v);
     }
     if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) {
       set_error("bucket gather failed to launch: %s", cudaGetErrorString(e));
@@ -815,7 +827,7 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
       break;
     }
     mark(5);
-    bw.launches = 5;  // count, run starts, scatter, search, gather
+    bw.launches = 6;  // count, run-start scan, run starts, scatter, search, gather
     bw.timed = timing;
   } while (0);
   scratch_free(buf, s);
@@ -901,10 +913,9 @@ int streamed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
       HBT_CUDA_TRY(cudaEventRecord(bs.ev_done[slot], s));
     }
     if (rc != HBT_OK) break;
-    const unsigned g = unsigned(std::min<uint64_t>(p.nseg, uint64_t(t->num_sms) * 2));
+    const unsigned g = unsigned(std::min<uint64_t>(p.chunks, uint64_t(t->num_sms) * 2));
     bk_gather<K><<<g, kThreads, kSmemGather, s>>>(p.at<uint16_t>(p.o_li), m, p.at<uint32_t>(p.o_tab),
-                                                 p.at<uint32_t>(p.o_so), B, p.chunks, p.kps, p.nseg, pf_s, v_s, pf,
-                                                 (K*)v);
+                                                 p.at<uint32_t>(p.o_gb), B, p.chunks, pf_s, v_s, pf, (K*)v);
     if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) {
       set_error("bucket gather failed to launch: %s", cudaGetErrorString(e));
       rc = HBT_ECUDA;

@@ -4,6 +4,7 @@
 
 #include <cuda_runtime.h>
 #include <nccl.h>
+#include <nvtx3/nvToolsExt.h>
 #include <stdint.h>
 
 #include <mutex>
@@ -25,6 +26,16 @@ void set_error(const char* fmt, ...);
   } while (0)
 
 static inline uint64_t ceil_div_u64(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+
+// NVTX range around a host-side phase (build, search, update, exchange steps): shows
+// up in nsys / ncu --nvtx timelines; free when no tool is attached (NVTX v3 is
+// header-only and does nothing until a tool injects itself).
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+  NvtxRange(const NvtxRange&) = delete;
+  NvtxRange& operator=(const NvtxRange&) = delete;
+};
 
 // Scratch of builds and updates comes from the device's stream-ordered pool
 // (cudaMallocAsync): after the first use, repeated updates allocate without

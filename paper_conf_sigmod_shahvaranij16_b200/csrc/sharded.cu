@@ -284,6 +284,19 @@ int search_local_t(hbt_tree* const* shards, int G, const void* const* queries, c
 
 ncclDataType_t u8() { return ncclUint8; }
 
+// Poll the communicator's asynchronous error state (a peer failure or a network error
+// surfaces here, not in the enqueue calls' return codes).
+int nccl_async_ok(ncclComm_t comm) {
+  ncclResult_t a = ncclSuccess;
+  ncclResult_t r = ncclCommGetAsyncError(comm, &a);
+  if (r != ncclSuccess) { set_error("ncclCommGetAsyncError: %s", ncclGetErrorString(r)); return HBT_ENCCL; }
+  if (a != ncclSuccess && a != ncclInProgress) {
+    set_error("NCCL asynchronous error: %s", ncclGetErrorString(a));
+    return HBT_ENCCL;
+  }
+  return HBT_OK;
+}
+
 template <typename K>
 int search_nccl_t(const hbt_tree* tc, const void* queries, uint64_t m, hbt_out out, cudaStream_t st) {
   hbt_tree* t = const_cast<hbt_tree*>(tc);
@@ -305,6 +318,7 @@ int search_nccl_t(const hbt_tree* tc, const void* queries, uint64_t m, hbt_out o
   std::vector<unsigned long long> rcnt(G, 0);
   HBT_CUDA_TRY(cudaMemcpyAsync(rcnt.data(), sc.counts + kMaxShards, G * 8, cudaMemcpyDeviceToHost, st));
   HBT_CUDA_TRY(cudaStreamSynchronize(st));
+  if ((rc = nccl_async_ok(c->comm))) return rc;
   uint64_t recv = 0;
   for (int g = 0; g < G; ++g) recv += rcnt[g];
   if ((rc = prepare(sc, m, recv, S))) return rc;
@@ -341,7 +355,7 @@ int search_nccl_t(const hbt_tree* tc, const void* queries, uint64_t m, hbt_out o
                                                    (K*)out.values);
     HBT_CUDA_TRY(cudaGetLastError());
   }
-  return HBT_OK;
+  return nccl_async_ok(c->comm);
 }
 
 }  // namespace
@@ -363,7 +377,7 @@ int comm_allgather_host(hbt_comm* c, const void* send, void* recv, uint64_t byte
   cudaFree(d);
   if (r != ncclSuccess) { set_error("ncclAllGather: %s", ncclGetErrorString(r)); return HBT_ENCCL; }
   if (e != cudaSuccess) { set_error("all-gather: %s", cudaGetErrorString(e)); return HBT_ECUDA; }
-  return HBT_OK;
+  return nccl_async_ok(c->comm);
 }
 
 void shard_free(hbt_tree* t) { free_scratch(t->shard_scratch); }
@@ -425,6 +439,7 @@ int hbt_comm_destroy(hbt_comm* c) {
 
 int hbt_bulk_build_sharded(hbt_comm* c, const void* keys_local, const void* values_local, uint64_t n_local,
                            uint32_t fanout, uint32_t layout, void* stream, hbt_tree** out) {
+  NvtxRange nvtx_("hbt_bulk_build_sharded");
   if (!c || !out) { set_error("NULL argument"); return HBT_EINVAL; }
   if ((layout & 0x1) != HBT_IMPLICIT) { set_error("sharded trees are implicit"); return HBT_EUNSUPPORTED; }
   int rc = hbt_bulk_build(keys_local, values_local, n_local, fanout, layout, stream, out);
@@ -452,6 +467,7 @@ int hbt_bulk_build_sharded(hbt_comm* c, const void* keys_local, const void* valu
 
 int hbt_search_sharded(const hbt_tree* t, const void* queries_local, uint64_t m_local, hbt_out out_local,
                        void* stream) {
+  NvtxRange nvtx_("hbt_search_sharded");
   if (!t || !t->shard.comm) { set_error("not a sharded tree"); return HBT_EINVAL; }
   cudaStream_t st = (cudaStream_t)stream;
   if (t->shard.G == 1 && t->cfg.exchange == 0 && t->cfg.g1_direct) {

@@ -407,7 +407,10 @@ int nccl_fused_t(hbt_tree* t, const void* queries, uint64_t m, hbt_out out, cuda
   int rc = prep_local(f, m);
   if (rc) return rc;
   const RouteTab rt = table_of(t->shard);
-  rc = route_and_count<K>(f, (const K*)queries, m, rt, G, st);
+  {
+    NvtxRange r("exchange.count");
+    rc = route_and_count<K>(f, (const K*)queries, m, rt, G, st);
+  }
   if (rc) return rc;
   const int par = int(f->batch & 1);
   std::vector<unsigned long long> mat(G * G);
@@ -450,12 +453,18 @@ int nccl_fused_t(hbt_tree* t, const void* queries, uint64_t m, hbt_out out, cuda
     HBT_CUDA_TRY(cudaMemcpyAsync(pt.w[me].matrix + par * kMat, full.data(), kMat * 8, cudaMemcpyHostToDevice, st));
     f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);  // every window exists and holds its matrix
   }
-  rc = put_queries<K>(f, (const K*)queries, m, pt, me, par, st);
+  {
+    NvtxRange r("exchange.put");
+    rc = put_queries<K>(f, (const K*)queries, m, pt, me, par, st);
+  }
   if (rc) return rc;
   f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);
   uint64_t nrecv = 0;
   for (int s = 0; s < G; ++s) nrecv += mat[s * G + me];
-  rc = search_and_return<K>(t, f, pt, me, nrecv, st);
+  {
+    NvtxRange r("owner_search_and_return");
+    rc = search_and_return<K>(t, f, pt, me, nrecv, st);
+  }
   if (rc) return rc;
   f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);
   HBT_CUDA_TRY(cudaGetLastError());

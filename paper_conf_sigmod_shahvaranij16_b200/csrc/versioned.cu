@@ -112,6 +112,7 @@ int hbt_versioned_create(hbt_tree* t, hbt_versioned** out) {
 int hbt_versioned_search(hbt_versioned* v, const void* queries, uint64_t m, hbt_out out, void* stream,
                          uint64_t* version) {
   if (!v) { set_error("NULL handle"); return HBT_EINVAL; }
+  NvtxRange nvtx_("hbt_versioned_search");
   hbt_tree* t;
   {
     std::lock_guard<std::mutex> lock(v->mu);
@@ -142,6 +143,7 @@ int hbt_versioned_search(hbt_versioned* v, const void* queries, uint64_t m, hbt_
 
 int hbt_versioned_update(hbt_versioned* v, const hbt_batch* batch, void* stream, uint64_t* version) {
   if (!v || !batch) { set_error("NULL argument"); return HBT_EINVAL; }
+  NvtxRange nvtx_("hbt_versioned_update");
   std::lock_guard<std::mutex> ulock(v->update_mu);
   cudaStream_t s = (cudaStream_t)stream;
   hbt_tree* base;

@@ -169,7 +169,7 @@ def test_c3_full_size_bench_launch(hbt):
     t.set_param("phase_timing", 1)
     pf, val = t.search(dq)
     torch.cuda.synchronize()
-    assert t.last_phases()["launches"] == 5  # count, run starts, scatter, search, gather
+    assert t.last_phases()["launches"] == 6  # count, run-start scan, run starts, scatter, search, gather
     pf = pf.cpu().numpy().view(np.uint64)
     val = from_dev(val, 8)
     u = gen.uniform_indices(m, n + n_ins, sq).astype(np.int64)
