@@ -55,19 +55,13 @@ def parse():
     ap.add_argument("--config", default="c4", choices=["c1", "c2", "c3", "c4", "c5"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--smem", type=int, default=0, help="override smem budget (bytes)")
-    ap.add_argument("--qpl", type=int, default=0, help="queries per lane per warp round (1|2)")
-    ap.add_argument("--threads", type=int, default=0, help="threads per CTA (256|512|1024)")
-    ap.add_argument("--smem-mode", type=int, default=None, help="2 = directory (default), 0 = staged levels, 1 = hi/lo")
-    ap.add_argument("--carveout", type=int, default=-1, help="smem carve-out percent (-1 default)")
-    ap.add_argument("--l2-persist", type=int, default=None, help="bytes of I-segment in a persisting L2 window")
+    ap.add_argument("--smem-mode", type=int, default=None, help="implicit directory: 2 = staged (default), 3 = in place")
     ap.add_argument("--l2-levels", type=int, default=None, help="L2 budget for index+sector levels (bytes)")
     ap.add_argument("--exchange", type=int, default=None, help="c4: 0 = fused peer-memory exchange, 1 = NCCL")
     ap.add_argument("--bucket", type=int, default=None, help="query bucketing: 0 = off, 1 = on, 2 = auto (default)")
     ap.add_argument("--bucket-slice", type=int, default=None, help="tree bytes per query bucket")
     ap.add_argument("--bucket-items", type=int, default=None, help="bucket-local shared-memory directory: 0 | 1")
     ap.add_argument("--leaf256", type=int, default=None, help="leaf / key lines by 256-bit lane loads: 0 | 1")
-    ap.add_argument("--sec256", type=int, default=None, help="implicit L2-level sectors by one lane's 256-bit load")
     ap.add_argument("--full-levels", type=int, default=None, help="implicit: bit mask of levels read whole")
     ap.add_argument("--origin-rank0", action="store_true",
                     help="replicated configs: all queries start on rank 0 (NCCL scatter / gather in the step)")
@@ -338,10 +332,8 @@ def make_work(cfg_name, d, args):
         hit_rate = 0.0
         qdesc = f"{args.queries} query values on [0, 1] mapped to [0, MAX] (PAPER.md:346-352)"
     del keys, vals
-    tree.set_search_config(smem_bytes=args.smem, threads_per_cta=args.threads, queries_per_lane=args.qpl,
-                           smem_mode=args.smem_mode, carveout=args.carveout)
-    if args.l2_persist is not None:
-        tree.set_param("l2_persist", args.l2_persist)
+    if args.smem_mode is not None:
+        tree.set_param("smem_mode", args.smem_mode)
     if args.l2_levels is not None and c["layout"] == "implicit":
         tree.set_param("l2_levels_bytes", args.l2_levels)
     if args.exchange is not None:
@@ -354,8 +346,6 @@ def make_work(cfg_name, d, args):
         tree.set_param("bucket_items", args.bucket_items)
     if args.leaf256 is not None:
         tree.set_param("leaf256", args.leaf256)
-    if args.sec256 is not None:
-        tree.set_param("sec256", args.sec256)
     if args.full_levels is not None:
         tree.set_param("full_levels", args.full_levels)
     if args.leaf_host:

@@ -185,74 +185,53 @@ HBT_API int hbt_info(const hbt_tree* t, hbt_info_t* info);
  * `bytes` bytes (HBT_EINVAL if too small); *written receives the byte count. */
 HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t bytes, uint64_t* written);
 
-/* Tune the search kernel's launch shape on one tree; results never depend on
- * it.  name / value:
- *   "smem_bytes"  shared-memory budget per CTA for the pinned top levels (<= 227 KB; 0 = default 100 KB)
- *   "threads"     threads per CTA: 256, 512, 768 (implicit directory mode) or 1024 (0 = default: implicit 1024, regular 512)
+/* Tune the search and bucketing of one tree; results never depend on it.  name / value:
  *   "ctas_per_sm" cap on resident CTAs per SM (0 = occupancy-derived)
- *   "qpl"         queries per lane per warp round, 1 or 2 (0 = default)
- *   "smem_mode"   implicit top levels: 2 = level-T directory + one lower bound, staged in shared
- *                 memory (default), 3 = the same read in place from L2 (used automatically for
- *                 batches <= "small_batch"), 0 = per-level binary search of staged nodes,
- *                 1 = the same on 32-bit hi/lo planes
- *   "small_batch" mode 2: batches of at most this many queries use mode 3 (default 65536)
- *   "carveout"    preferred shared-memory carve-out percent, -1 = driver default
- *   "l2_persist"  implicit: keep up to this many bytes of the I-segment (+ index) in a
- *                 persisting L2 access-policy window (sets the device persisting-L2 limit), 0 = off
- *   "l2_levels_bytes" implicit: inner levels below the shared-memory top are read as index
- *                 sector + one key sector while their cumulative bytes fit this L2 budget,
- *                 as whole nodes beyond it (0 = default 32 MB; 1 = every level whole)
- *   "exchange"    sharded search: 0 = fused peer-memory exchange (CUDA IPC windows, default),
- *                 1 = NCCL send/recv (multi-process) / device copies (hbt_search_sharded_local)
+ *   "smem_mode"   implicit level-T directory (lower_bound over the level-T maxima plus a prefix
+ *                 table): 2 = staged in shared memory once per CTA (default), 3 = read in place
+ *                 from L2 (used automatically for batches <= "small_batch")
+ *   "small_batch" batches of at most this many queries use smem_mode 3 (default 65536)
+ *   "l2_levels_bytes" implicit: inner levels below the directory are read as index sector + one
+ *                 key sector while their cumulative bytes fit this L2 budget, as whole nodes
+ *                 beyond it (0 = default 32 MB; 1 = every level whole)
+ *   "full_levels" implicit: bit d set = level d's nodes are read whole (0 = by the budget above)
+ *   "exchange"    sharded search: 0 = fused peer-memory exchange (CUDA IPC windows, device
+ *                 barriers, count rows and queries by peer stores; default), 1 = NCCL send/recv
+ *                 (multi-process) / device copies (hbt_search_sharded_local)
  *   "g1_direct"   hbt_search_sharded on a ONE-shard tree with exchange 0: 1 (default) = search
  *                 in place (nothing to route or exchange), 0 = run the full fused pipeline
  *   "bucket"      query bucketing before the tree walk (north_star "queries bucketed per batch"):
  *                 0 = off, 1 = on, 2 = auto (default: regular trees larger than 8x the L2 and
- *                 batches of >= 4 Mi queries).  The batch is partitioned into B key-range
- *                 buckets, searched bucket after bucket, and the results are gathered back
- *                 to query order; outputs are identical to the unbucketed search.
+ *                 implicit trees larger than 64x, batches of >= 4 Mi queries).  The batch is
+ *                 partitioned into B key-range buckets, searched bucket after bucket, and the
+ *                 results are gathered back to query order; outputs are identical.
  *   "bucket_slice" tree bytes per bucket (0 = default 1 MB; B <= 1024)
  *   "bucket_items" bucketed search through a bucket-local shared-memory directory (1, default)
  *                 or the normal search kernel on the bucketed queries (0)
  *   "bucket_cap"  item-directory shared-memory entries (0 = derived; small values force the
  *                 global-memory fallback, for tests)
+ *   "item_rounds" bucketed item searches: most warp rounds per work item (0 = default 16;
+ *                 fewer are used when the batch would leave SMs idle)
  *   "phase_timing" 1 = record CUDA events around the phases of each bucketed search (read
  *                 them with hbt_last_phases), 0 = off (default)
- *   "leaf256"     1 (default) = the leaf line (and the regular item search's key line) is read
- *                 by two lanes' 256-bit loads, one 64 B request per lane group; 0 = 16 B loads
- *   "sec256"      implicit L2 levels: index / key sector by one lane's 256-bit load (1) or two
- *                 lanes' 16 B loads (0, default; measured faster on c2)
- *   "full256"     implicit whole-node levels: 256-bit lane loads (1, default) or 16 B lane
- *                 loads (0)
  *   "leaf_stream" L-segment in host memory (hbt_set_leaf_placement): 0 = zero-copy leaf
  *                 reads; 1 = bucket the batch and stream each bucket's leaf slice into HBM
  *                 (double-buffered copies overlapping the previous bucket's search);
  *                 2 = auto (default: stream when 160 B x m exceeds the L-segment bytes)
- *   "stream_slice" host L-segment bytes per streamed bucket (0 = default 8 MB; at most
- *                 1024 buckets)
- *   "qprefetch"   bucketed item searches: 1 = one thread per CTA prefetches the current and
- *                 next work item's queries into the L2 (cp.async.bulk.prefetch); 0 = off
- *                 (default: measured slower on c3, 1.55 -> 1.58 ms)
- *   "host_chunk_log2" hbt_search_host: queries per pipeline bucket, log2 in [12, 26]
- *                 (default 20)
+ *   "stream_slice" host L-segment bytes per streamed bucket (0 = default 8 MB; <= 1024 buckets)
+ *   "host_chunk_log2" hbt_search_host: queries per pipeline bucket, log2 in [12, 26] (default 20)
  *   "host_bufs"   hbt_search_host: (stream, buffer) pairs in flight, 2..4 (default 2)
- *   "item_rounds" bucketed item searches: most warp rounds per work item (0 = default 16;
- *                 fewer are used when the batch would leave SMs idle)
+ *   "leaf256"     1 (default) = the leaf line (and the regular item search's key line) is read
+ *                 by two lanes' 256-bit loads, one 64 B request per lane group; 0 = 16 B loads
+ *   "full256"     implicit whole-node levels: 256-bit lane loads (1, default) or 16 B loads (0)
  *   "l2_hint"     implicit search: L2 eviction-priority hints (createpolicy + ld ...
  *                 L2::cache_hint); bit 0 = leaf lines evict-first, bit 1 = whole-node levels
  *                 evict-last; 4 = auto (default: bit 0 iff the I-segment fits in a quarter of
- *                 the L2 — measured c2 0.426 -> 0.415 ms, c5 Zipf 2.84 -> 3.00 ms with it on)
+ *                 the L2 -- measured c2 0.426 -> 0.415 ms, c5 Zipf 2.84 -> 3.00 ms with it on)
  *   "item_l2_hint" the same bits for the implicit bucketed item search (default 1: c4 item
  *                 search 10.96 -> 9.50 ms, DRAM reads 171 -> 148 B/query)
- *   "small_threads" small-batch search (directory read in place): CTA size 128, 256 or 1024
- *                 (0 = default 256; 128 measured the same on c1, 1024 slower)
- *   "item_group4" implicit item search with 128 B nodes: 1 = 4-lane query groups (one 256-bit
- *                 whole-node load per lane); 0 (default, measured faster: c4 9.50 vs 10.8 ms)
- *   "regular_l2_hint" the same bits for the regular item search (default 0: 1 measured
- *                 slower on c3, 1.59 -> 1.72 ms)
- *   "full_levels" implicit: bit d set = level d's nodes are read whole in one round trip
- *                 (0 = default: by the "l2_levels_bytes" budget)
- * Unknown names or out-of-range values return HBT_EINVAL. */
+ * Variants measured slower were removed (DESIGN.md §8 keeps their numbers).  Unknown
+ * names or out-of-range values return HBT_EINVAL. */
 HBT_API int hbt_set_param(hbt_tree* t, const char* name, int64_t value);
 
 /* Device time of the phases of the tree's last BUCKETED search (hbt_search with

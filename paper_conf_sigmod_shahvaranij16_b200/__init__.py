@@ -283,12 +283,11 @@ class Tree:
         d["launches"] = int(p.launches)
         return d
 
-    def set_search_config(self, smem_bytes: int = 0, threads_per_cta: int = 0, ctas_per_sm: int = 0,
-                          queries_per_lane: int = 0, smem_mode=None, carveout: int = -1):
-        for k, v in [("smem_bytes", smem_bytes), ("threads", threads_per_cta), ("ctas_per_sm", ctas_per_sm),
-                     ("qpl", queries_per_lane), ("smem_mode", smem_mode), ("carveout", carveout)]:
-            if v is not None:
-                self.set_param(k, v)
+    def set_search_config(self, ctas_per_sm: int = 0, smem_mode=None):
+        """Launch-shape knobs of the search (results never depend on them)."""
+        self.set_param("ctas_per_sm", ctas_per_sm)
+        if smem_mode is not None:
+            self.set_param("smem_mode", smem_mode)
 
 
 class VersionedTree:

@@ -171,8 +171,6 @@ void free_tree(hbt_tree* t) {
   if (!t) return;
   cudaFree(t->d_inner);  // also holds d_inner_idx
   cudaFree(t->d_dir);
-  cudaFree(t->d_sdir);
-  cudaFree(t->d_sdir_full);
   leaf_free(t);
   regular_free(t);
   shard_free(t);
@@ -370,7 +368,7 @@ int hbt_info(const hbt_tree* t, hbt_info_t* info) {
   info->n_distinct = t->n;
   if (t->form == HBT_IMPLICIT) {
     info->height = t->H;
-    info->smem_levels = t->cfg.mode >= 2 ? t->dir_T : implicit_smem_levels(t, t->cfg.smem_budget);
+    info->smem_levels = t->dir_T;
     for (uint32_t d = 0; d < t->H; ++d) info->level_nodes[d] = t->nodes[d];
     info->leaf_lines = t->L0;
     info->chain_len = t->L0;
@@ -379,7 +377,7 @@ int hbt_info(const hbt_tree* t, hbt_info_t* info) {
   } else {
     const RegularState& r = t->r;
     info->height = r.U + 1;
-    info->smem_levels = regular_smem_levels(t, t->cfg.smem_budget);
+    info->smem_levels = r.dir_T;
     for (uint32_t u = 0; u < r.U; ++u) info->level_nodes[u] = r.unodes[u];
     info->leaf_lines = r.pool;
     info->chain_len = r.nchain;
@@ -452,39 +450,27 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   if (!t || !name) { set_error("NULL argument"); return HBT_EINVAL; }
   const std::string n(name);
   SearchConfig& c = t->cfg;
-  if (n == "smem_bytes" && value >= 0 && value <= 227 * 1024) c.smem_budget = uint32_t(value);
-  else if (n == "threads" && (value == 0 || value == 256 || value == 512 || value == 768 || value == 1024)) c.threads = uint32_t(value);
-  else if (n == "ctas_per_sm" && value >= 0 && value <= 32) c.ctas_per_sm = uint32_t(value);
-  else if (n == "qpl" && value >= 0 && value <= 2) c.qpl = uint32_t(value);
-  else if (n == "smem_mode" && value >= 0 && value <= 4) c.mode = uint32_t(value);
+  if (n == "ctas_per_sm" && value >= 0 && value <= 32) c.ctas_per_sm = uint32_t(value);
+  else if (n == "smem_mode" && (value == 2 || value == 3)) c.mode = uint32_t(value);
   else if (n == "small_batch" && value >= 0) c.small_batch = uint64_t(value);
-  else if (n == "carveout" && value >= -1 && value <= 100) c.carveout = int(value);
-  else if (n == "l2_persist" && value >= 0) c.l2_persist = uint64_t(value);
   else if (n == "l2_levels_bytes" && value >= 0) c.l2_levels_bytes = uint64_t(value);
+  else if (n == "full_levels" && value >= 0 && value <= 0xFFFFFFFFll) c.full_levels = uint32_t(value);
   else if (n == "exchange" && (value == 0 || value == 1)) c.exchange = uint32_t(value);
   else if (n == "g1_direct" && (value == 0 || value == 1)) c.g1_direct = uint32_t(value);
   else if (n == "bucket" && value >= 0 && value <= 2) c.bucket = uint32_t(value);
   else if (n == "bucket_slice" && value >= 0) { c.bucket_slice = uint64_t(value); invalidate_buckets(t); }
   else if (n == "bucket_items" && (value == 0 || value == 1)) { c.bucket_items = uint32_t(value); invalidate_buckets(t); }
   else if (n == "bucket_cap" && value >= 0 && value < (1 << 20)) { c.bucket_cap = uint32_t(value); invalidate_buckets(t); }
-  else if (n == "leaf_stream" && value >= 0 && value <= 2) c.leaf_stream = uint32_t(value);
-  else if (n == "qprefetch" && (value == 0 || value == 1)) c.qprefetch = uint32_t(value);
   else if (n == "item_rounds" && value >= 0 && value <= 64) c.item_rounds = uint32_t(value);
+  else if (n == "phase_timing" && (value == 0 || value == 1)) c.phase_timing = uint32_t(value);
+  else if (n == "leaf_stream" && value >= 0 && value <= 2) c.leaf_stream = uint32_t(value);
+  else if (n == "stream_slice" && value >= 0) { c.stream_slice = uint64_t(value); invalidate_buckets(t); }
   else if (n == "host_chunk_log2" && value >= 12 && value <= 26) c.host_chunk_log2 = uint32_t(value);
   else if (n == "host_bufs" && value >= 2 && value <= kHostBufs) c.host_bufs = uint32_t(value);
-  else if (n == "stream_slice" && value >= 0) { c.stream_slice = uint64_t(value); invalidate_buckets(t); }
-  else if (n == "phase_timing" && (value == 0 || value == 1)) c.phase_timing = uint32_t(value);
   else if (n == "leaf256" && (value == 0 || value == 1)) c.leaf256 = uint32_t(value);
-  else if (n == "sec256" && (value == 0 || value == 1)) c.sec256 = uint32_t(value);
   else if (n == "full256" && (value == 0 || value == 1)) c.full256 = uint32_t(value);
   else if (n == "l2_hint" && value >= 0 && value <= 4) c.l2_hint = uint32_t(value);
-  else if (n == "small_threads" && (value == 0 || value == 128 || value == 256 || value == 1024))
-    c.small_threads = uint32_t(value);
-  else if (n == "item_group4" && (value == 0 || value == 1)) c.item_group4 = uint32_t(value);
-  else if (n == "regular_l2_hint" && value >= 0 && value <= 3) c.regular_l2_hint = uint32_t(value);
   else if (n == "item_l2_hint" && value >= 0 && value <= 3) c.item_l2_hint = uint32_t(value);
-  else if (n == "full_levels" && value >= 0 && value <= 0xFFFFFFFFll) c.full_levels = uint32_t(value);
-  else if (n == "item_sched" && (value == 0 || value == 1)) c.item_sched = uint32_t(value);
   else {
     set_error("bad parameter %s = %lld", name, (long long)value);
     return HBT_EINVAL;

@@ -793,10 +793,8 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
       d.span = bs.span;
       d.nunits = bs.nunits;
       d.pos_base = pos_base;
-      d.qprefetch = t->cfg.qprefetch;
       d.cap = t->cfg.bucket_cap ? std::min<uint32_t>(t->cfg.bucket_cap, uint32_t(item_cap(t, p.B)))
                                 : uint32_t(item_cap(t, p.B));
-      d.strided = t->form == HBT_IMPLICIT ? t->cfg.item_sched : 0u;
       rc = t->form == HBT_IMPLICIT ? implicit_search_items(t, qs, m, pf_s, v_s, d, s)
                                    : regular_search_items(t, qs, m, pf_s, v_s, d, s);
     } else {

@@ -48,53 +48,42 @@ void scratch_free(void* p, cudaStream_t s);
 struct LevelTable {
   uint64_t offset[HBT_MAX_LEVELS + 1];
   uint32_t H;   // inner levels
-  uint32_t SL;  // levels [0, SL) searched in shared memory (mode 2: = the directory level T)
-  uint32_t dcount;  // mode 2/3: nodes at level T; mode 4: sectors at level T
-  uint32_t dbits;   // mode 2/3/4: directory prefix bits
+  uint32_t SL;  // first level walked by lane groups (the directory level T, or the item directory's level)
+  uint32_t dcount;  // nodes at level T (directory entries)
+  uint32_t dbits;   // directory prefix bits
   uint32_t full_mask;  // bit d: read level d's nodes whole (not index + sector)
   uint32_t leaf256;    // leaf line read as one 64 B request (two 256-bit lane loads)
-  uint32_t sec256;     // index / key sectors of L2 levels by one lane's 256-bit load
   uint32_t full256;    // whole-node levels read by 256-bit lane loads (half the load instructions)
   uint32_t l2_hint;    // bit 0: leaf lines loaded L2::evict_first; bit 1: whole-node levels L2::evict_last
 };
 
+// Search / bucketing configuration of one tree (hbt_set_param, include/hbt.h).  Results
+// never depend on it.  Variants measured slower in round 1 and 2 were removed; their
+// numbers stay in DESIGN.md §8.
 struct SearchConfig {
-  uint32_t smem_budget = 0;      // bytes per CTA for pinned levels (0 = default)
-  uint32_t threads = 0;          // threads per CTA (0 = default)
   uint32_t ctas_per_sm = 0;      // 0 = occupancy-derived
-  uint32_t qpl = 0;              // queries per lane per warp round (0 = default)
-  uint32_t mode = 2;             // top-level mode: 0 = staged levels (K words), 1 = hi/lo planes, 2 = directory
-  int carveout = -1;             // shared-memory carve-out percent (-1 = driver default)
-  uint64_t l2_persist = 0;       // bytes of the I-segment to keep in a persisting L2 window (0 = off)
+  uint32_t mode = 2;             // implicit directory: 2 = staged in shared memory, 3 = read in place
+  uint64_t small_batch = 1u << 16;  // mode 2: batches up to this size read the directory in place (mode 3)
   uint64_t l2_levels_bytes = 0;  // L2-resident budget for index+sector levels (0 = default 32 MB)
+  uint32_t full_levels = 0;      // implicit: bit d = read level d's nodes whole (0 = by the L2 budget)
   uint32_t exchange = 0;         // sharded search: 0 = fused peer-memory exchange, 1 = NCCL send/recv
   uint32_t g1_direct = 1;        // sharded search with ONE shard: search directly (no route / exchange)
-  uint64_t small_batch = 1u << 16;  // mode 2: batches up to this size read the directory in place (mode 3)
   uint32_t bucket = 2;           // query bucketing (bucketed.cu): 0 = off, 1 = on, 2 = auto
   uint64_t bucket_slice = 0;     // tree bytes per bucket (0 = default 1 MB)
   uint32_t bucket_items = 1;     // bucketed search: bucket-local shared-memory directory (ItemDir)
   uint32_t bucket_cap = 0;       // item directory: shared-memory entries (0 = derived; tests force the fallback)
+  uint32_t item_rounds = 0;      // item searches: most warp rounds per work item (0 = 16)
   uint32_t phase_timing = 0;     // bucketed search: CUDA events around each phase (hbt_last_phases)
   uint32_t leaf_stream = 2;      // host L-segment: 0 = zero-copy leaf reads, 1 = stream bucket slices
                                  // into HBM (bucketed, double-buffered copies), 2 = auto (by batch size)
   uint64_t stream_slice = 0;     // host L-segment bytes per streamed bucket (0 = 8 MB)
   uint32_t host_chunk_log2 = 20;  // hbt_search_host: queries per pipeline bucket (log2; c2 e2e 2.78 -> 3.00 G q/s vs 2^22)
   uint32_t host_bufs = 2;        // hbt_search_host: (stream, buffer) pairs in flight (2..4)
-  uint32_t item_rounds = 0;      // item searches: most warp rounds per work item (0 = 16)
-  uint32_t qprefetch = 0;        // item searches: bulk L2 prefetch of each work item's queries (measured slower: c3 item search 1.55 -> 1.58 ms)
   uint32_t leaf256 = 1;          // leaf line by two 256-bit lane loads (one 64 B request per group)
-  uint32_t sec256 = 0;           // implicit L2 levels: index / key sector by one lane's 256-bit load
   uint32_t full256 = 1;          // implicit whole-node levels by 256-bit lane loads
-  uint32_t full_levels = 0;      // implicit: bit d = read level d's nodes whole (0 = by the L2 budget)
   uint32_t l2_hint = 4;          // implicit search: L2 eviction-priority hints (LevelTable::l2_hint);
                                  // 4 = auto: leaf lines evict-first iff the I-segment fits in L2 / 4
   uint32_t item_l2_hint = 1;     // implicit bucketed item search (c4 item search 10.96 -> 9.50 ms)
-  uint32_t small_threads = 0;    // small-batch (in-place directory) search: CTA size 128 / 256 / 1024 (0 = 256)
-  uint32_t item_group4 = 0;      // implicit item search, 128 B nodes: 4-lane groups (one 256-bit load per lane;
-                                 // measured slower: c4 item search 9.50 -> 10.8 ms, 56 B of spills)
-  uint32_t regular_l2_hint = 0;  // regular bucketed item search (measured slower with 1: c3 1.59 -> 1.72 ms)
-  uint32_t item_sched = 0;       // implicit item search: 1 = strided items (all CTAs move through the
-                                 // bucketed order together), 0 = contiguous 16-round items
 };
 
 // Bucket-local directory of the bucketed search (bucketed.cu): after the
@@ -117,13 +106,7 @@ struct ItemDir {
   uint64_t nunits = 0; // entries of M
   uint32_t cap = 0;    // shared-memory entries (larger ranges search M in global memory)
   uint64_t pos_base = 0;  // implicit: added to every reported position (key-range shards)
-  uint32_t qprefetch = 0; // bulk L2 prefetch of the current / next item's queries
   uint32_t rounds = 16;   // warp rounds per work item (fewer for small batches: every SM gets items)
-  // strided schedule (implicit item search, "item_sched" = 1): item (CTA j, s) is rounds
-  // s*R .. s*R+R-1 of CTA j, round g's queries being [(g*grid + j)*T, +T), so all CTAs
-  // work through the bucketed order together (implicit_search.cu)
-  uint32_t strided = 0;
-  uint32_t pbits = 10;    // prefix-table bits of the staged directory (<= 12)
 };
 
 // Owner side of the fused sharded exchange (sharded_fused.cu): the bucketed search's
@@ -269,13 +252,6 @@ struct hbt_tree {
   uint32_t dir_T = 0;       // target level (H = leaf lines)
   uint32_t dir_count = 0;   // nodes at level T
   uint32_t dir_bits = 0;
-  // Sector directory (search mode 4): over the key SECTORS of level T.
-  // d_sdir = [hi 32 bits of Msec (sdir_count u32) | 2^sdir_bits x (u16 lo, u16 hi)];
-  // d_sdir_full = Msec at full width (tie fallback when the high words are equal).
-  void* d_sdir = nullptr;
-  void* d_sdir_full = nullptr;
-  uint64_t sdir_bytes = 0;
-  uint32_t sdir_count = 0, sdir_bits = 0;
   void* d_leaf = nullptr;
   uint64_t L0 = 0;
   uint64_t leaf_bytes = 0;
@@ -341,7 +317,6 @@ void fused_free(hbt_tree* t);
 int fused_search_local(hbt_tree* const* shards, int G, const void* const* queries, const uint64_t* m,
                        const hbt_out* outs, cudaStream_t st);
 int fused_search_nccl(const hbt_tree* t, const void* queries, uint64_t m, hbt_out out, cudaStream_t st);
-uint32_t implicit_smem_levels(const hbt_tree* t, uint32_t budget);
 // index bytes per implicit node (0 when F*S <= 32)
 uint32_t implicit_idx_stride(uint32_t F, uint32_t S);
 // regular_*.cu
@@ -349,7 +324,6 @@ int regular_build(hbt_tree* t, const void* keys, const void* values, uint64_t n,
 int regular_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s);
 int regular_update(hbt_tree* t, const hbt_batch* b, cudaStream_t s);
 void regular_free(hbt_tree* t);
-uint32_t regular_smem_levels(const hbt_tree* t, uint32_t budget);
 // Item-directory searches write 16 B records {pos|found, value (zero-extended)}
 // at pf (v is unused): rec[i] = (pf[2i], pf[2i+1]).
 int implicit_search_items(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v,

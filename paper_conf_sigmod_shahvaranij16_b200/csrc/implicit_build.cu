@@ -130,25 +130,6 @@ __global__ void build_dir_table(const K* __restrict__ M, uint32_t count, uint32_
   }
 }
 
-// Sector directory (mode 4): Msec[j*NSEC + t] = the max key of key sector t of
-// level-T node j, except that the LAST sector of every non-last node takes the
-// node's subtree max M_T[j] (its index entry is MAX).  Then Msec is sorted and
-// lower_bound(Msec, q) = j*NSEC + t with j = the node the descent reaches and t =
-// its index step's answer: nodes before j have every entry <= M_T[j-1] < q, and
-// inside node j the first sector with max >= q is the index step's t (the last
-// sector qualifies because M_T[j] >= q).  hi holds the high 32 bits.
-template <typename K>
-__global__ void build_sec_max(const K* __restrict__ idx, uint32_t idx_entries, const K* __restrict__ MT,
-                              uint64_t nodes, uint32_t nsec, K* __restrict__ full, uint32_t* __restrict__ hi) {
-  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < nodes * nsec;
-       x += uint64_t(gridDim.x) * blockDim.x) {
-    const uint64_t j = x / nsec;
-    const uint32_t t = uint32_t(x % nsec);
-    const K v = (j + 1 < nodes && t + 1 == nsec) ? MT[j] : idx[j * idx_entries + t];
-    full[x] = v;
-    hi[x] = uint32_t(uint64_t(v) >> (8 * sizeof(K) - 32));
-  }
-}
 
 template <typename K>
 __global__ void unpack_leaf_lines(const K* __restrict__ leaf, uint64_t nd, K* __restrict__ kd, K* __restrict__ vd) {
@@ -345,25 +326,6 @@ int build_sorted_t(hbt_tree* t, const K* kd, const K* vd, uint64_t nd, cudaStrea
     HBT_CUDA_TRY(cudaGetLastError());
     build_dir_table<K><<<grid_for(1ull << bits), 256, 0, s>>>(M, uint32_t(cnt), bits, dir);
     HBT_CUDA_TRY(cudaGetLastError());
-    // sector directory (mode 4) when level T is an inner level of multi-sector nodes
-    const uint32_t nsec = (F * sizeof(K)) / 32;
-    if (T < H && nsec > 1 && cnt * nsec <= 32768) {
-      const uint64_t ns = cnt * nsec;
-      uint32_t sb = 1;
-      while ((1ull << sb) < ns && sb < 13) ++sb;
-      t->sdir_count = uint32_t(ns);
-      t->sdir_bits = sb;
-      t->sdir_bytes = ns * 4 + (4ull << sb);
-      HBT_CUDA_TRY(cudaMalloc(&t->d_sdir, t->sdir_bytes));
-      HBT_CUDA_TRY(cudaMalloc(&t->d_sdir_full, ns * sizeof(K)));
-      const uint32_t ie = t->idx_stride / sizeof(K);
-      const K* idx_T = (const K*)t->d_inner_idx + t->offset[T] * ie;
-      build_sec_max<K><<<grid_for(ns), 256, 0, s>>>(idx_T, ie, M, cnt, nsec, (K*)t->d_sdir_full,
-                                                      (uint32_t*)t->d_sdir);
-      build_dir_table<K><<<grid_for(1ull << sb), 256, 0, s>>>((const K*)t->d_sdir_full, uint32_t(ns), sb,
-                                                               (uint32_t*)((uint8_t*)t->d_sdir + ns * 4));
-      HBT_CUDA_TRY(cudaGetLastError());
-    }
   }
   HBT_CUDA_TRY(cudaStreamSynchronize(s));
   return HBT_OK;
@@ -433,8 +395,8 @@ int implicit_merge_rebuild_t(const hbt_tree* t, const hbt_batch* b, hbt_tree* nt
   int rc = build_sorted_t<K>(nt, kd, vd, uint64_t(h_nsel), s);
   cleanup();
   if (rc != HBT_OK) {
-    cudaFree(nt->d_leaf); cudaFree(nt->d_inner); cudaFree(nt->d_dir); cudaFree(nt->d_sdir); cudaFree(nt->d_sdir_full);
-    nt->d_leaf = nt->d_inner = nt->d_inner_idx = nt->d_dir = nt->d_sdir = nt->d_sdir_full = nullptr;
+    cudaFree(nt->d_leaf); cudaFree(nt->d_inner); cudaFree(nt->d_dir);
+    nt->d_leaf = nt->d_inner = nt->d_inner_idx = nt->d_dir = nullptr;
   }
   return rc;
 }
@@ -449,8 +411,6 @@ int implicit_update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   leaf_free(t);
   cudaFree(t->d_inner);  // also holds the derived index
   cudaFree(t->d_dir);
-  cudaFree(t->d_sdir);
-  cudaFree(t->d_sdir_full);
   t->n = nt.n; t->L0 = nt.L0; t->H = nt.H; t->P = nt.P;
   for (int d = 0; d < HBT_MAX_LEVELS; ++d) t->nodes[d] = nt.nodes[d];
   for (int d = 0; d <= HBT_MAX_LEVELS; ++d) t->offset[d] = nt.offset[d];
@@ -459,9 +419,7 @@ int implicit_update_t(hbt_tree* t, const hbt_batch* b, cudaStream_t s) {
   t->d_inner_idx = nt.d_inner_idx; t->inner_idx_bytes = nt.inner_idx_bytes; t->idx_stride = nt.idx_stride;
   t->d_dir = nt.d_dir; t->dir_bytes = nt.dir_bytes; t->dir_T = nt.dir_T; t->dir_count = nt.dir_count;
   t->dir_bits = nt.dir_bits;
-  t->d_sdir = nt.d_sdir; t->d_sdir_full = nt.d_sdir_full; t->sdir_bytes = nt.sdir_bytes;
-  t->sdir_count = nt.sdir_count; t->sdir_bits = nt.sdir_bits;
-  nt.d_leaf = nt.d_inner = nt.d_inner_idx = nt.d_dir = nt.d_sdir = nt.d_sdir_full = nullptr;
+  nt.d_leaf = nt.d_inner = nt.d_inner_idx = nt.d_dir = nullptr;
   // the rebuilt L-segment goes back where the caller placed the old one
   return where ? leaf_place(t, where) : HBT_OK;
 }

@@ -3,21 +3,24 @@
 // Node search = "the minimum i such that q <= sep[i]" = #{t : sep[t] < q}
 // (PAPER.md:190 read with the comments of Snippets 1/2, P:520 / P:566; reading
 // R1), then descend to child node*F + i (Snippet 3's
-// (nodeIndex+result)<<3).  Two phases per warp round of 32*QPL queries:
+// (nodeIndex+result)<<3).  Two phases per warp round of 32 queries:
 //
-//  1. Shared-memory levels (the top SL levels, staged once per persistent CTA —
-//     the I-segment-in-fast-memory principle of P:178): ONE lane per query runs
-//     a branchless binary search over the node's F sorted keys (log2 F probes,
-//     each one LDS; the last key is MAX, so no size is needed).
+//  1. The top of the I-segment in the fastest memory, in its B200
+//     form: the root-first descent through levels 0..T-1 always reaches the FIRST
+//     level-T node whose subtree max is >= q, i.e. lower_bound(M_T, q) over the
+//     level-T maxima; M_T and a prefix directory are staged in shared memory once
+//     per persistent CTA and ONE lane per query does one directory probe plus a
+//     short binary search.
 //  2. L2/HBM levels: a GROUP of G = 2 (4 for 256-byte nodes) lanes per query.
 //     A node wider than one 32 B sector is read through its index sector
 //     (entry t = max key of sector t, the paper's index line of P:134 applied
 //     to implicit nodes): t = popc(ballot(idx < q)), then ONLY key sector t is
 //     read: i = t*KPS + popc(ballot(key < q)).  So a level moves 64 B instead of
 //     F*S bytes, with 16 B vector loads, no divergence and no barriers (Snippet
-//     3 needs two __syncthreads per level).  Each group keeps QPG
-//     queries in flight level-synchronously (the GPU form of the software
-//     pipelining of Alg. 2).
+//     3 needs two __syncthreads per level).  Levels beyond the L2
+//     budget are read whole in one round trip (256-bit lane loads).  Each group
+//     keeps QPG queries in flight level-synchronously (the GPU form of the
+//     software pipelining of Alg. 2).
 //  Leaf: the 64 B line [P keys | P values] is read by the group in one round
 //  trip; s = popc(ballot(key < q)); r = line*P + s; found = r < n' && key[s] == q.
 // Queries and results stream with evict-first (.cs) accesses so they do not
@@ -32,10 +35,6 @@ namespace {
 
 constexpr uint64_t kEnd = HBT_POS_END;
 constexpr uint64_t kFound = HBT_FOUND_BIT;
-// Pinned-level budget per CTA (measured on B200, profiles/r01_sweep_v*.log): with
-// the padded node stride, c2's 4 top levels (74 KB) beat 3 levels (29.3 -> 31.5
-// G q/s); the carve-out is left to the driver so the L2 levels keep L1 hits.
-constexpr uint32_t kDefaultSmemBudget = 100 * 1024;
 
 template <typename K>
 __device__ __forceinline__ K key_max() { return K(~K(0)); }
@@ -105,9 +104,7 @@ __device__ __forceinline__ void stcs(uint64_t* p, uint64_t v) {
   __stcs(reinterpret_cast<unsigned long long*>(p), (unsigned long long)v);
 }
 
-// GMIN: smallest lane group (2; 4 lets a 128 B whole node be read by ONE 256-bit load per
-// lane, one L1TEX wavefront per query instead of two -- the item search's "item_group4")
-template <typename K, int F, int GMIN = 2>
+template <typename K, int F>
 struct Cfg {
   static constexpr int S = int(sizeof(K));
   static constexpr int NODE_BYTES = F * S;
@@ -118,7 +115,7 @@ struct Cfg {
   static constexpr int IL = IDXB / 16;                                    // lanes loading the index
   static constexpr int SECB = NODE_BYTES < 32 ? NODE_BYTES : 32;          // bytes read after the index
   static constexpr int SL_ = SECB / 16;                                   // lanes loading them
-  static constexpr int G = IL > GMIN ? IL : GMIN;                         // lanes per query group
+  static constexpr int G = IL > 2 ? IL : 2;                               // lanes per query group
   static constexpr int NG = 32 / G;                                       // groups per warp
   static constexpr int P = 64 / (2 * S);                                  // pairs per leaf line
 };
@@ -141,22 +138,21 @@ __device__ __forceinline__ uint32_t count_less16(const V16<K>& v, K q, unsigned 
 
 // Phase 2 of a warp round: levels [d0, H) by lane groups, the leaf line, and the
 // results of the round (slot j of group g = round query j*NG + g, stored at
-// base + j*NG + g).  sec_known: the sector of level d0 is already in sec0.
-template <typename K, int F, int QPG, bool REC = false, int GM = 2>
+// base + j*NG + g).
+template <typename K, int F, int QPG, bool REC = false>
 __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ inner,
                                                   const uint8_t* __restrict__ inner_idx,
                                                   const uint8_t* __restrict__ leaf, const LevelTable& lt,
-                                                  uint32_t d0, bool sec_known_d0, K (&q)[QPG], uint32_t (&node)[QPG],
-                                                  const uint32_t (&sec0)[QPG], int g, int k, unsigned gmask,
-                                                  uint64_t base, uint64_t m, uint64_t n, uint64_t pos_base,
-                                                  uint64_t* __restrict__ out_pf, K* __restrict__ out_v) {
-  using C = Cfg<K, F, GM>;
+                                                  uint32_t d0, K (&q)[QPG], uint32_t (&node)[QPG], int g, int k,
+                                                  unsigned gmask, uint64_t base, uint64_t m, uint64_t n,
+                                                  uint64_t pos_base, uint64_t* __restrict__ out_pf,
+                                                  K* __restrict__ out_v) {
+  using C = Cfg<K, F>;
   const uint32_t H = lt.H;
   for (uint32_t d = d0; d < H; ++d) {
     const uint8_t* lvl = inner + lt.offset[d] * C::NODE_BYTES;
-    const bool sec_known = sec_known_d0 && d == d0;  // mode 4: the sector directory chose it
     if constexpr (C::HAS_IDX) {
-      if (!sec_known && ((lt.full_mask >> d) & 1u)) {
+      if ((lt.full_mask >> d) & 1u) {
         // Level beyond the L2-resident budget: a miss costs a whole DRAM line
         // anyway, so read the full node in ONE round trip (each of the G lanes
         // loads NODE_BYTES/G contiguous bytes) instead of index + sector.
@@ -215,45 +211,8 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
         continue;
       }
     }
-    if constexpr (C::IDXB == 32 && C::SECB == 32) {
-      if (lt.sec256 && !sec_known) {
-        // index sector, then the chosen key sector, each by ONE lane's 256-bit load
-        // (the group's other lanes idle): fewer L1 wavefronts per level
-        const uint8_t* lidx = inner_idx + lt.offset[d] * C::IDXB;
-        L256<K> w[QPG];
-#pragma unroll
-        for (int j = 0; j < QPG; ++j) {
-          if (k == 0) ld32(w[j], lidx + uint64_t(node[j]) * C::IDXB);
-          else fill_max32(w[j]);
-        }
-        uint32_t sec[QPG];
-#pragma unroll
-        for (int j = 0; j < QPG; ++j) {
-          uint32_t c = 0;
-#pragma unroll
-          for (int e = 0; e < C::NSEC; ++e) c += (w[j].k[e] < q[j]) ? 1u : 0u;
-          sec[j] = __shfl_sync(0xffffffffu, c, g * C::G);
-        }
-#pragma unroll
-        for (int j = 0; j < QPG; ++j) {
-          if (k == 0) ld32(w[j], lvl + uint64_t(node[j]) * C::NODE_BYTES + sec[j] * 32);
-          else fill_max32(w[j]);
-        }
-#pragma unroll
-        for (int j = 0; j < QPG; ++j) {
-          uint32_t c = 0;
-#pragma unroll
-          for (int e = 0; e < C::KPS; ++e) c += (w[j].k[e] < q[j]) ? 1u : 0u;
-          node[j] = node[j] * F + sec[j] * C::KPS + __shfl_sync(0xffffffffu, c, g * C::G);
-        }
-        continue;
-      }
-    }
     uint32_t sec[QPG];
-    if (C::HAS_IDX && sec_known) {
-#pragma unroll
-      for (int j = 0; j < QPG; ++j) sec[j] = sec0[j];
-    } else if constexpr (C::HAS_IDX) {
+    if constexpr (C::HAS_IDX) {
       const uint8_t* lidx = inner_idx + lt.offset[d] * C::IDXB;
       V16<K> iv[QPG];
 #pragma unroll
@@ -362,53 +321,31 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
   }
 }
 
-template <typename K, int F, int QPL, int THREADS, int MODE>
+// The plain (unbucketed) search: one persistent pass over the batch, one query per
+// lane in phase 1 (the level-T directory), lane groups in phase 2 (descend_and_store).
+// MODE 2: the directory [M_T | prefix table] is staged in shared memory once per CTA;
+// MODE 3 (small batches): it is read in place from L2 (staging ~70 KB per CTA would
+// dominate a launch that serves only a few warp rounds).
+template <typename K, int F, int THREADS, int MODE>
 __global__ void __launch_bounds__(THREADS, 1)
 implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ inner_idx,
                        const uint8_t* __restrict__ leaf, const uint32_t* __restrict__ dirbuf,
-                       const K* __restrict__ sfull, const K* __restrict__ queries, uint64_t m,
-                       uint64_t* __restrict__ out_pf, K* __restrict__ out_v, const LevelTable lt, uint64_t n,
-                       uint64_t pos_base) {
+                       const K* __restrict__ queries, uint64_t m, uint64_t* __restrict__ out_pf,
+                       K* __restrict__ out_v, const LevelTable lt, uint64_t n, uint64_t pos_base) {
+  static_assert(MODE == 2 || MODE == 3, "directory staged (2) or read in place (3)");
   using C = Cfg<K, F>;
-  constexpr int ROUND = 32 * QPL;        // queries per warp round (QPL per lane in phase 1)
+  constexpr int ROUND = 32;              // queries per warp round
   constexpr int QPG = ROUND / C::NG;     // queries per group in phase 2
   static_assert(QPG % C::G == 0, "every group lane stores QPG/G results");
   extern __shared__ __align__(16) uint8_t smem[];
-  const uint32_t SL = lt.SL, H = lt.H;
-  // Stage the top SL levels (root-first, contiguous) once per persistent CTA
-  // with a padded node stride of F+1 keys: with a 128 B stride, key i of every
-  // node would sit in the same bank and the lanes' probes into different nodes
-  // would serialise.  MODE 1 splits 64-bit keys into 32-bit hi / lo planes.
-  constexpr uint32_t FP = F + 1;
-  const uint32_t s_nodes = MODE >= 2 ? 0u : uint32_t(lt.offset[SL]);
-  K* s_keys = reinterpret_cast<K*>(smem);
-  uint32_t* s_hi = reinterpret_cast<uint32_t*>(smem);
-  uint32_t* s_lo = s_hi + s_nodes * FP;
+  uint32_t* s_words = reinterpret_cast<uint32_t*>(smem);
   if constexpr (MODE == 2) {
     // directory: [M_T (dcount keys) | 2^dbits x (u16 lo, u16 hi)]
     const uint32_t words = (lt.dcount * uint32_t(sizeof(K)) + (4u << lt.dbits)) / 4;
-    for (uint32_t i = threadIdx.x; i < words; i += THREADS) s_hi[i] = __ldg(dirbuf + i);
-  } else if constexpr (MODE == 4) {
-    // sector directory: [hi words of Msec (dcount u32) | 2^dbits x (u16 lo, u16 hi)]
-    const uint32_t words = lt.dcount + (1u << lt.dbits);
-    for (uint32_t i = threadIdx.x; i < words; i += THREADS) s_hi[i] = __ldg(dirbuf + i);
-  } else if constexpr (MODE == 3) {
-    // small batches: the directory is read from L2 in place (staging 96 KB per
-    // CTA would dominate a launch that serves only a few warp rounds)
-  } else {
-    for (uint32_t i = threadIdx.x; i < s_nodes * F; i += THREADS) {
-      const K key = __ldg(reinterpret_cast<const K*>(inner) + i);
-      const uint32_t a = (i / F) * FP + i % F;
-      if constexpr (MODE == 1 && sizeof(K) == 8) {
-        s_hi[a] = uint32_t(uint64_t(key) >> 32);
-        s_lo[a] = uint32_t(key);
-      } else {
-        s_keys[a] = key;
-      }
-    }
+    for (uint32_t i = threadIdx.x; i < words; i += THREADS) s_words[i] = __ldg(dirbuf + i);
   }
   __syncthreads();
-  const K* d_M = MODE == 3 ? reinterpret_cast<const K*>(dirbuf) : s_keys;
+  const K* d_M = MODE == 3 ? reinterpret_cast<const K*>(dirbuf) : reinterpret_cast<const K*>(smem);
   const uint32_t* d_dir = MODE == 3 ? reinterpret_cast<const uint32_t*>(reinterpret_cast<const uint8_t*>(dirbuf) +
                                                                          lt.dcount * sizeof(K))
                                     : reinterpret_cast<const uint32_t*>(smem + lt.dcount * sizeof(K));
@@ -420,127 +357,67 @@ implicit_search_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restr
   const uint64_t nwarps = (uint64_t(gridDim.x) * THREADS) >> 5;
   const uint64_t rounds = (m + ROUND - 1) / ROUND;
 
-  // MODE 2 pipelines the query stream across rounds: the next round's queries
-  // are loaded while this round walks the tree (their HBM latency was the
-  // largest single stall, profiles/r01_c2_v11_*).  Lanes past the batch end repeat
-  // the batch's last query (results discarded) so they walk to a leaf line the batch
-  // itself uses: a streamed host L-segment stages only the bucket's slice.
-  K nextq[QPL];
-  if constexpr (MODE >= 2) {
-#pragma unroll
-    for (int u = 0; u < QPL; ++u) {
-      const uint64_t i = warp * ROUND + uint64_t(u) * 32 + lane;
-      nextq[u] = warp < rounds ? ldcs(queries + (i < m ? i : m - 1)) : key_max<K>();
-    }
+  // The query stream is pipelined across rounds: the next round's queries are
+  // loaded while this round walks the tree (their HBM latency was the largest single
+  // stall, profiles/r01_c2_v11_*).  Lanes past the batch end repeat the batch's last
+  // query (results discarded) so they walk to a leaf line the batch itself uses: a
+  // streamed host L-segment stages only the bucket's slice.
+  K nextq;
+  {
+    const uint64_t i = warp * ROUND + lane;
+    nextq = warp < rounds ? ldcs(queries + (i < m ? i : m - 1)) : key_max<K>();
   }
   for (uint64_t rd = warp; rd < rounds; rd += nwarps) {
     const uint64_t base = rd * ROUND;
     // ---- phase 1: one lane per query; coalesced query loads
-    K myq[QPL];
-    uint32_t mynode[QPL];
-    uint32_t mysec[QPL];
-#pragma unroll
-    for (int u = 0; u < QPL; ++u) {
-      mysec[u] = 0;
-      if constexpr (MODE >= 2) {
-        myq[u] = nextq[u];
-        const uint64_t i = (rd + nwarps) * ROUND + uint64_t(u) * 32 + lane;
-        nextq[u] = rd + nwarps < rounds ? ldcs(queries + (i < m ? i : m - 1)) : key_max<K>();
-      } else {
-        const uint64_t i = base + uint64_t(u) * 32 + lane;
-        myq[u] = ldcs(queries + (i < m ? i : m - 1));
-      }
-      mynode[u] = 0;
+    const K myq = nextq;
+    {
+      const uint64_t i = (rd + nwarps) * ROUND + lane;
+      nextq = rd + nwarps < rounds ? ldcs(queries + (i < m ? i : m - 1)) : key_max<K>();
     }
-    if constexpr (MODE == 4) {
-      // (level-T node, key sector) = lower_bound(Msec, q) over 32-bit high words;
-      // equal high words fall back to the full key (global, L2-resident)
-      constexpr uint32_t NSEC = C::NSEC;
-      const uint32_t* s_sdir = s_hi + lt.dcount;
-#pragma unroll
-      for (int u = 0; u < QPL; ++u) {
-        const uint32_t qh = uint32_t(uint64_t(myq[u]) >> (8 * sizeof(K) - 32));
-        const uint32_t e = s_sdir[uint32_t(myq[u] >> (8 * sizeof(K) - lt.dbits))];
-        uint32_t lo = e & 0xFFFFu, hi = e >> 16;
-        while (lo < hi) {
-          const uint32_t mid = (lo + hi) >> 1;
-          const uint32_t mh = s_hi[mid];
-          bool lt_ = mh < qh;
-          if (sizeof(K) == 8 && mh == qh) lt_ = __ldg(sfull + mid) < myq[u];
-          if (lt_) lo = mid + 1; else hi = mid;
-        }
-        mynode[u] = lo / NSEC;
-        mysec[u] = lo % NSEC;
+    // level-T node = lower_bound(M_T, q), narrowed by the prefix directory
+    uint32_t mynode;
+    {
+      const uint32_t e = d_dir[uint32_t(myq >> (8 * sizeof(K) - lt.dbits))];
+      uint32_t lo = e & 0xFFFFu, hi = e >> 16;
+      while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (d_M[mid] < myq) lo = mid + 1; else hi = mid;
       }
-    } else if constexpr (MODE >= 2) {
-      // level-T node = lower_bound(M_T, q), narrowed by the prefix directory
-#pragma unroll
-      for (int u = 0; u < QPL; ++u) {
-        const uint32_t e = d_dir[uint32_t(myq[u] >> (8 * sizeof(K) - lt.dbits))];
-        uint32_t lo = e & 0xFFFFu, hi = e >> 16;
-        while (lo < hi) {
-          const uint32_t mid = (lo + hi) >> 1;
-          if (d_M[mid] < myq[u]) lo = mid + 1; else hi = mid;
-        }
-        mynode[u] = lo;
-      }
-    } else {
-    for (uint32_t d = 0; d < SL; ++d) {
-      const uint32_t lvl = uint32_t(lt.offset[d]) * FP;
-      uint32_t pos[QPL];
-#pragma unroll
-      for (int u = 0; u < QPL; ++u) pos[u] = 0;
-#pragma unroll
-      for (int step = F / 2; step >= 1; step /= 2) {
-#pragma unroll
-        for (int u = 0; u < QPL; ++u) {
-          const uint32_t a = lvl + mynode[u] * FP + pos[u] + step - 1;
-          bool lt_;
-          if constexpr (MODE == 1 && sizeof(K) == 8) {
-            const uint32_t qh = uint32_t(uint64_t(myq[u]) >> 32), ql = uint32_t(myq[u]);
-            const uint32_t kh = s_hi[a], kl = s_lo[a];
-            lt_ = (kh < qh) | ((kh == qh) & (kl < ql));
-          } else {
-            lt_ = s_keys[a] < myq[u];
-          }
-          pos[u] += lt_ ? uint32_t(step) : 0u;
-        }
-      }
-#pragma unroll
-      for (int u = 0; u < QPL; ++u) mynode[u] = mynode[u] * F + pos[u];
-    }
+      mynode = lo;
     }
     // ---- phase 2: lane groups; slot j of group g is round query j*NG + g,
-    //      owned in phase 1 by lane (j*NG)%32 + g, slot (j*NG)/32
+    //      owned in phase 1 by lane (j*NG)%32 + g
     K q[QPG];
     uint32_t node[QPG];
-    uint32_t sec0[QPG];
 #pragma unroll
     for (int j = 0; j < QPG; ++j) {
       const int src = (j * C::NG) % 32 + g;
-      q[j] = __shfl_sync(0xffffffffu, myq[(j * C::NG) / 32], src);
-      node[j] = __shfl_sync(0xffffffffu, mynode[(j * C::NG) / 32], src);
-      sec0[j] = MODE == 4 ? __shfl_sync(0xffffffffu, mysec[(j * C::NG) / 32], src) : 0u;
+      q[j] = __shfl_sync(0xffffffffu, myq, src);
+      node[j] = __shfl_sync(0xffffffffu, mynode, src);
     }
-    descend_and_store<K, F, QPG>(inner, inner_idx, leaf, lt, SL, MODE == 4, q, node, sec0, g, k, gmask, base, m, n,
-                                 pos_base, out_pf, out_v);
+    descend_and_store<K, F, QPG>(inner, inner_idx, leaf, lt, lt.SL, q, node, g, k, gmask, base, m, n, pos_base,
+                                 out_pf, out_v);
   }
 }
 
-
 // Bucketed search with a bucket-local directory (bucketed.cu, ItemDir).  One
-// persistent CTA works through items of kItemRounds * THREADS consecutive
-// bucketed queries.  Per item: the item's first and last queries give its bucket
-// range [b0, b1] (binary search over the staged bucket starts), hence a
-// contiguous range of level-`level` nodes [u0, u1] that contains every query's
-// node at that level: all nodes before u0 end at or below splitter b0-1 < q and
-// q <= splitter b1 <= max of node u1.  The maxima of [u0, u1] are staged in
-// shared memory; a query's node is u0 + lower_bound(maxima, q) (clamped to u1,
-// which only binds past the last key), exactly the node the root-first descent
-// reaches (every level picks the first child whose subtree max is >= q,
-// DESIGN.md R1/R3).  The rest of the walk is descend_and_store from that level.
-constexpr int kItemRounds = 16;
-constexpr uint32_t kStridedPrefixBits = 12;  // strided items stage ~4x more maxima
+// persistent CTA works through items of rounds * THREADS consecutive bucketed
+// queries.  Per item: the item's first and last queries give its bucket range
+// [b0, b1] (binary search over the staged bucket starts), hence a contiguous range
+// of level-`level` nodes [u0, u1] that contains every query's node at that level:
+// all nodes before u0 end at or below splitter b0-1 < q and q <= splitter b1 <= max
+// of node u1.  The maxima of [u0, u1] are staged in shared memory; a query's node is
+// u0 + lower_bound(maxima, q) (clamped to u1, which only binds past the last key),
+// exactly the node the root-first descent reaches (every level picks the first
+// child whose subtree max is >= q, R1/R3).  The rest of the walk is
+// descend_and_store from that level.
+//
+// Measured and dropped (profiles/r02_c4_*): a strided item schedule in which all
+// CTAs move through the bucketed order together cut c4's DRAM reads 40.1 -> 29.2 GB
+// per launch (the leaf slices stay L2-resident while their bucket's queries arrive)
+// but ran slower (9.9 -> 10.5 ms): this kernel is bound by latency and the LSU pipe,
+// not by DRAM, and the wider per-item directory cost more than the saved bytes.
 
 // Cooperative copy of cnt keys into shared memory, four loads in flight per thread.
 template <typename K>
@@ -555,13 +432,13 @@ __device__ __forceinline__ void stage_keys(K* dst, const K* __restrict__ src, ui
   }
 }
 
-template <typename K, int F, int THREADS, int GM = 2>
+template <typename K, int F, int THREADS>
 __global__ void __launch_bounds__(THREADS)
 implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ inner_idx,
                              const uint8_t* __restrict__ leaf, const ItemDir d, const K* __restrict__ queries,
                              uint64_t m, uint64_t* __restrict__ out_pf, K* __restrict__ out_v, const LevelTable lt,
                              uint64_t n) {
-  using C = Cfg<K, F, GM>;
+  using C = Cfg<K, F>;
   constexpr int QPG = 32 / C::NG;
   const uint64_t W = uint64_t(THREADS) * d.rounds;
   extern __shared__ __align__(16) uint8_t smem[];
@@ -575,22 +452,9 @@ implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* _
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int g = lane / C::G, k = lane % C::G;
   const unsigned gmask = ((1u << C::G) - 1u) << (g * C::G);
-  // strided: superstep x covers queries [x * SW, (x + 1) * SW), CTA j takes its slice
-  // [(x * grid + j) * THREADS, + THREADS); item s of CTA j = supersteps [s R, s R + R)
-  const uint64_t SW = uint64_t(gridDim.x) * THREADS;
-  const uint64_t steps = (m + SW - 1) / SW;
-  const uint64_t items = d.strided ? (steps + d.rounds - 1) / d.rounds : (m + W - 1) / W;
-  for (uint64_t it = d.strided ? 0 : blockIdx.x; it < items; it += d.strided ? 1 : gridDim.x) {
-    uint64_t p0, p1;
-    if (d.strided) {
-      p0 = (it * d.rounds * gridDim.x + blockIdx.x) * uint64_t(THREADS);
-      if (p0 >= m) break;
-      const uint64_t xl = std::min<uint64_t>((it + 1) * d.rounds, steps) - 1;
-      p1 = std::min<uint64_t>(m, (xl * gridDim.x + blockIdx.x + 1) * uint64_t(THREADS)) - 1;
-    } else {
-      p0 = it * W;
-      p1 = (p0 + W < m ? p0 + W : m) - 1;
-    }
+  const uint64_t items = (m + W - 1) / W;
+  for (uint64_t it = blockIdx.x; it < items; it += gridDim.x) {
+    const uint64_t p0 = it * W, p1 = (p0 + W < m ? p0 + W : m) - 1;
     if (threadIdx.x < 2) {
       const uint64_t p = threadIdx.x ? p1 : p0;
       uint32_t lo = 0, hi = d.B;  // largest b with bstart[b] <= p
@@ -600,11 +464,6 @@ implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* _
       }
       const uint64_t lu = threadIdx.x ? ((uint64_t(lo) + 1) * d.U) / d.B - 1 : (uint64_t(lo) * d.U) / d.B;
       s_range[threadIdx.x] = lu / d.span;
-    } else if (threadIdx.x == 32 && d.qprefetch) {
-      // this item's queries (needed from the first round) and the next item's
-      if (it == blockIdx.x) prefetch_l2_range(queries + p0, (p1 - p0 + 1) * sizeof(K));
-      const uint64_t n0 = (it + gridDim.x) * W;
-      if (n0 < m) prefetch_l2_range(queries + n0, ((n0 + W < m ? n0 + W : m) - n0) * sizeof(K));
     }
     __syncthreads();
     const uint64_t u0 = s_range[0], u1 = s_range[1];
@@ -613,41 +472,36 @@ implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* _
     if (in_smem) stage_keys(s_M, gM + u0, cnt, THREADS);
     __syncthreads();
     PrefixTab<K> pt{};
-    if (in_smem) pt = build_prefix(s_M, cnt, s_T, THREADS, d.pbits);
+    if (in_smem) pt = build_prefix(s_M, cnt, s_T, THREADS);
     __syncthreads();
     const K* M = in_smem ? s_M : gM + u0;
-    // consecutive rounds of a warp: THREADS queries apart (contiguous items) or one
-    // superstep apart (strided items)
-    const uint64_t rstride = d.strided ? SW : uint64_t(THREADS);
-    const uint64_t lim = d.strided ? m - 1 : p1;  // last valid query index
     // the next round's queries are loaded while this round walks the tree
     K nextq;
     {
       const uint64_t i = p0 + uint64_t(wid) * 32 + lane;
-      nextq = i <= lim ? ldcs(queries + i) : key_max<K>();
+      nextq = i <= p1 ? ldcs(queries + i) : key_max<K>();
     }
 #pragma unroll 1
     for (int r = 0; r < int(d.rounds); ++r) {
-      const uint64_t base = p0 + uint64_t(r) * rstride + uint64_t(wid) * 32;
-      if (base > lim) break;
+      const uint64_t base = p0 + (uint64_t(r) * (THREADS / 32) + wid) * 32;
+      if (base > p1) break;
       const K myq = nextq;
       {
-        const uint64_t i = base + rstride + lane;
-        nextq = (r + 1 < int(d.rounds) && i <= lim) ? ldcs(queries + i) : key_max<K>();
+        const uint64_t i = base + (THREADS / 32) * 32 + lane;
+        nextq = (r + 1 < int(d.rounds) && i <= p1) ? ldcs(queries + i) : key_max<K>();
       }
       const uint32_t lo = in_smem ? prefix_lower_bound(s_M, cnt, s_T, pt, myq) : lb_range(M, 0, cnt, myq);
       const uint32_t mynode = uint32_t(u0) + (lo < cnt ? lo : cnt - 1);
       K q[QPG];
-      uint32_t node[QPG], sec0[QPG];
+      uint32_t node[QPG];
 #pragma unroll
       for (int j = 0; j < QPG; ++j) {
         const int src = (j * C::NG) % 32 + g;
         q[j] = __shfl_sync(0xffffffffu, myq, src);
         node[j] = __shfl_sync(0xffffffffu, mynode, src);
-        sec0[j] = 0;
       }
-      descend_and_store<K, F, QPG, true, GM>(inner, inner_idx, leaf, lt, d.level, false, q, node, sec0, g, k, gmask,
-                                         base, lim + 1, n, d.pos_base, out_pf, out_v);
+      descend_and_store<K, F, QPG, true>(inner, inner_idx, leaf, lt, d.level, q, node, g, k, gmask, base, p1 + 1, n,
+                                         d.pos_base, out_pf, out_v);
     }
     __syncthreads();
   }
@@ -657,24 +511,28 @@ template <typename K, int F>
 struct Launch {
   using C = Cfg<K, F>;
 
-  static uint32_t smem_levels(const hbt_tree* t, uint32_t budget) {
-    uint32_t SL = 0;
-    while (SL < t->H && t->offset[SL + 1] * uint64_t(C::NODE_BYTES + C::S) <= budget) ++SL;
-    return SL;
+  // Levels below the shared-memory top are read as index sector + one key sector while
+  // their cumulative bytes fit the L2 budget, as whole nodes beyond it.
+  static uint32_t full_mask(const hbt_tree* t, uint32_t first) {
+    uint32_t mask = 0;
+    uint64_t cum = 0;
+    const uint64_t budget = t->cfg.l2_levels_bytes ? t->cfg.l2_levels_bytes : (32ull << 20);
+    for (uint32_t d = first; d < t->H; ++d) {
+      cum += t->nodes[d] * uint64_t(C::NODE_BYTES + C::IDXB);
+      if (C::HAS_IDX && cum > budget && d < 32) mask |= 1u << d;
+    }
+    if (t->cfg.full_levels) mask = C::HAS_IDX ? uint32_t(t->cfg.full_levels) : 0u;  // explicit override
+    return mask;
   }
 
-  template <int QPL, int THREADS, int MODE>
+  template <int THREADS, int MODE>
   static int run_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t base,
                    cudaStream_t s, const void* leafp) {
-    auto kern = implicit_search_kernel<K, F, QPL, THREADS, MODE>;
+    auto kern = implicit_search_kernel<K, F, THREADS, MODE>;
     LevelTable lt{};
     for (uint32_t d = 0; d <= t->H; ++d) lt.offset[d] = t->offset[d];
     lt.H = t->H;
-    // Levels whose cumulative footprint (from the first global level down) exceeds
-    // the L2-resident budget are read as whole nodes (see the kernel).
-    lt.full_mask = 0;
     lt.leaf256 = t->cfg.leaf256;
-    lt.sec256 = t->cfg.sec256;
     lt.full256 = t->cfg.full256;
     lt.l2_hint = t->cfg.l2_hint;
     if (lt.l2_hint == 4) {
@@ -686,145 +544,61 @@ struct Launch {
       if (!l2) HBT_CUDA_TRY(cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, t->device));
       lt.l2_hint = (t->inner_bytes + t->inner_idx_bytes) * 4 <= uint64_t(l2) ? 1u : 0u;
     }
-    size_t smem;
-    if (MODE == 4) {
-      lt.SL = t->dir_T;
-      lt.dcount = t->sdir_count;
-      lt.dbits = t->sdir_bits;
-      smem = t->sdir_bytes;
-    } else if (MODE >= 2) {
-      lt.SL = t->dir_T;
-      lt.dcount = t->dir_count;
-      lt.dbits = t->dir_bits;
-      smem = MODE == 2 ? t->dir_bytes : 0;
-    } else {
-      lt.SL = smem_levels(t, t->cfg.smem_budget ? t->cfg.smem_budget : kDefaultSmemBudget);
-      lt.dcount = 0;
-      lt.dbits = 0;
-      smem = size_t(lt.offset[lt.SL]) * (C::NODE_BYTES + C::S);  // (F+1)*S bytes per staged node
-    }
+    lt.SL = t->dir_T;
+    lt.dcount = t->dir_count;
+    lt.dbits = t->dir_bits;
+    lt.full_mask = full_mask(t, lt.SL);
+    const size_t smem = MODE == 2 ? t->dir_bytes : 0;
     static bool attr_set = false;  // per instantiation
     if (!attr_set) {
       HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
       attr_set = true;
     }
-    static int carve = -2;  // per instantiation: last carve-out applied
-    if (carve != t->cfg.carveout) {
-      HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout,
-                                        t->cfg.carveout >= 0 ? t->cfg.carveout : int(cudaSharedmemCarveoutDefault)));
-      carve = t->cfg.carveout;
-    }
-    {
-      uint64_t cum = 0;
-      const uint64_t budget = t->cfg.l2_levels_bytes ? t->cfg.l2_levels_bytes : (32ull << 20);
-      for (uint32_t d = lt.SL; d < t->H; ++d) {
-        cum += t->nodes[d] * uint64_t(C::NODE_BYTES + C::IDXB);
-        if (C::HAS_IDX && cum > budget && d < 32) lt.full_mask |= 1u << d;
-      }
-      if (t->cfg.full_levels) lt.full_mask = C::HAS_IDX ? uint32_t(t->cfg.full_levels) : 0u;  // explicit override
-    }
     // occupancy of this instantiation for this smem size (cached: the query costs
     // microseconds, which dominate small batches)
     static size_t occ_smem = ~size_t(0);
     static int occ_cached = 0;
-    int occ = 0;
     if (occ_smem != smem) {
       HBT_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_cached, kern, THREADS, smem));
       occ_smem = smem;
     }
-    occ = occ_cached;
+    int occ = occ_cached;
     if (t->cfg.ctas_per_sm && int(t->cfg.ctas_per_sm) < occ) occ = int(t->cfg.ctas_per_sm);
     if (occ < 1) occ = 1;
-    const uint64_t rounds = (m + 32 * QPL - 1) / (32 * QPL);
+    const uint64_t rounds = (m + 31) / 32;
     uint64_t grid = uint64_t(t->num_sms) * occ;
     const uint64_t need = (rounds + THREADS / 32 - 1) / (THREADS / 32);
     if (need < grid) grid = need ? need : 1;
-    cudaLaunchConfig_t lc = {};
-    lc.gridDim = dim3(unsigned(grid));
-    lc.blockDim = dim3(THREADS);
-    lc.dynamicSmemBytes = smem;
-    lc.stream = s;
-    cudaLaunchAttribute attr[1];
-    lc.attrs = attr;
-    lc.numAttrs = 0;
-    if (t->cfg.l2_persist && t->d_inner) {
-      // Keep the inner levels resident against the leaf / query / result streams.
-      static uint64_t limit_set = 0;
-      const uint64_t win = std::min<uint64_t>(t->cfg.l2_persist,
-                                              ((t->inner_bytes + 255) & ~uint64_t(255)) + t->inner_idx_bytes);
-      if (limit_set < win) {
-        HBT_CUDA_TRY(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, win));
-        limit_set = win;
-      }
-      attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
-      attr[0].val.accessPolicyWindow.base_ptr = t->d_inner;
-      attr[0].val.accessPolicyWindow.num_bytes = win;
-      attr[0].val.accessPolicyWindow.hitRatio = 1.0f;
-      attr[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-      attr[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-      lc.numAttrs = 1;
-    }
-    HBT_CUDA_TRY(cudaLaunchKernelEx(&lc, kern, (const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
-                                    (const uint8_t*)leafp,
-                                    (const uint32_t*)(MODE == 4 ? t->d_sdir : t->d_dir),
-                                    (const K*)t->d_sdir_full, (const K*)q, m, pf, (K*)v, lt, t->n, base));
+    kern<<<unsigned(grid), THREADS, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
+                                              (const uint8_t*)leafp, (const uint32_t*)t->d_dir, (const K*)q, m, pf,
+                                              (K*)v, lt, t->n, base);
     HBT_CUDA_TRY(cudaGetLastError());
     return HBT_OK;
   }
 
-
   static int run_items(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, const ItemDir& d,
                        cudaStream_t s) {
     constexpr int TH = C::NODE_BYTES > 128 ? 512 : 1024;
-    // 128 B nodes: 4-lane groups on request (one 256-bit whole-node load per lane)
-    auto kern = (C::NODE_BYTES == 128 && C::G < 4 && t->cfg.item_group4) ? implicit_search_items_kernel<K, F, TH, 4>
-                                                                         : implicit_search_items_kernel<K, F, TH>;
+    auto kern = implicit_search_items_kernel<K, F, TH>;
     LevelTable lt{};
     for (uint32_t x = 0; x <= t->H; ++x) lt.offset[x] = t->offset[x];
     lt.H = t->H;
     lt.SL = d.level;
     lt.leaf256 = t->cfg.leaf256;
-    lt.sec256 = t->cfg.sec256;
     lt.full256 = t->cfg.full256;
     lt.l2_hint = t->cfg.item_l2_hint;
-    {
-      uint64_t cum = 0;
-      const uint64_t budget = t->cfg.l2_levels_bytes ? t->cfg.l2_levels_bytes : (32ull << 20);
-      for (uint32_t x = d.level; x < t->H; ++x) {
-        cum += t->nodes[x] * uint64_t(C::NODE_BYTES + C::IDXB);
-        if (C::HAS_IDX && cum > budget && x < 32) lt.full_mask |= 1u << x;
-      }
-    }
-    static bool attr_set[2] = {false, false};  // per kernel variant
-    const int av = kern == implicit_search_items_kernel<K, F, TH> ? 0 : 1;
-    if (!attr_set[av]) {
+    lt.full_mask = full_mask(t, d.level);
+    static bool attr_set = false;
+    if (!attr_set) {
       HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
-      attr_set[av] = true;
+      attr_set = true;
     }
     ItemDir dd = d;
+    dd.rounds = item_rounds(m, t->num_sms, TH, t->cfg.item_rounds ? t->cfg.item_rounds : 16);
     uint64_t grid = t->num_sms;
-    if (d.strided && m >= uint64_t(t->num_sms) * TH * 2) {
-      // strided items: R rounds per item such that the item's unit range (R supersteps of
-      // grid * TH queries, uniform keys assumed; wider items fall back to the global
-      // directory) fits the staging capacity
-      // the larger prefix table comes out of the staging capacity, so the CTA's shared
-      // memory (and with it the L1 carve-out: 9.5 vs 10.9 ms on c4 when it grew) stays
-      // that of the contiguous items
-      dd.pbits = kStridedPrefixBits;
-      const uint32_t extra = (((1u << kStridedPrefixBits) - (1u << kPrefixBits)) * 4 + C::S - 1) / C::S;
-      if (dd.cap > extra + 64) dd.cap -= extra;
-      const double per_step = double(uint64_t(t->num_sms) * TH) / double(m) * double(d.nunits);
-      const double edge = 2.0 * double(d.nunits) / double(d.B);  // whole buckets at both ends
-      const uint32_t R = double(dd.cap) > edge ? uint32_t((double(dd.cap) - edge) / (per_step * 1.15)) : 1u;
-      const uint32_t rmax = t->cfg.item_rounds ? t->cfg.item_rounds : 16;
-      dd.rounds = std::max<uint32_t>(1, std::min<uint32_t>(R, rmax));
-    } else {
-      dd.strided = 0;
-      dd.rounds = item_rounds(m, t->num_sms, TH, t->cfg.item_rounds ? t->cfg.item_rounds : 16);
-      const uint64_t items = (m + uint64_t(TH) * dd.rounds - 1) / (uint64_t(TH) * dd.rounds);
-      if (items < grid) grid = items ? items : 1;
-    }
-    const size_t smem = (d.B + 1) * 8 + size_t(dd.cap) * C::S + ((1u << dd.pbits) + 1) * 4;
+    const uint64_t items = (m + uint64_t(TH) * dd.rounds - 1) / (uint64_t(TH) * dd.rounds);
+    if (items < grid) grid = items ? items : 1;
+    const size_t smem = (d.B + 1) * 8 + size_t(dd.cap) * C::S + ((1u << kPrefixBits) + 1) * 4;
     kern<<<unsigned(grid), TH, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
                                           (const uint8_t*)t->d_leaf, dd, (const K*)q, m, pf, (K*)v, lt, t->n);
     HBT_CUDA_TRY(cudaGetLastError());
@@ -833,33 +607,11 @@ struct Launch {
 
   static int run(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t b, cudaStream_t s,
                  const void* lp) {
-    const uint32_t qpl = t->cfg.qpl ? t->cfg.qpl : 1;
+    // small batches read the directory in place with 256-thread CTAs, so a one-wave
+    // batch spreads over every SM (c1: 10.1 -> 8.3 us per batch)
+    if (t->cfg.mode == 3 || (t->cfg.mode == 2 && m <= t->cfg.small_batch)) return run_t<256, 3>(t, q, m, pf, v, b, s, lp);
     // 256-byte nodes (u64, F = 32) need more registers than a 1024-thread CTA allows
-    const uint32_t th = t->cfg.threads ? t->cfg.threads : (C::NODE_BYTES > 128 ? 512 : 1024);
-    // small batches read the directory in place (no 96 KB staging per CTA)
-    if (t->cfg.mode == 3 || (t->cfg.mode == 2 && m <= t->cfg.small_batch))
-      // 256-thread CTAs spread a small batch over every SM (c1: 10.1 -> 8.3 us per batch)
-      return (t->cfg.threads == 1024 || t->cfg.small_threads == 1024) ? run_t<1, 1024, 3>(t, q, m, pf, v, b, s, lp)
-             : t->cfg.small_threads == 128                               ? run_t<1, 128, 3>(t, q, m, pf, v, b, s, lp)
-                                                                         : run_t<1, 256, 3>(t, q, m, pf, v, b, s, lp);
-    if (t->cfg.mode == 4 && t->d_sdir)
-      return th == 512 ? run_t<1, 512, 4>(t, q, m, pf, v, b, s, lp) : run_t<1, 1024, 4>(t, q, m, pf, v, b, s, lp);
-    if (t->cfg.mode == 2) {
-      if (th == 512) return run_t<1, 512, 2>(t, q, m, pf, v, b, s, lp);
-      if (th == 768) return qpl == 2 ? run_t<2, 768, 2>(t, q, m, pf, v, b, s, lp) : run_t<1, 768, 2>(t, q, m, pf, v, b, s, lp);
-      return qpl == 2 ? run_t<2, 1024, 2>(t, q, m, pf, v, b, s, lp) : run_t<1, 1024, 2>(t, q, m, pf, v, b, s, lp);
-    }
-    const bool hilo = t->cfg.mode == 1;
-    if (hilo) {
-      if (qpl == 2) return th == 256 ? run_t<2, 256, 1>(t, q, m, pf, v, b, s, lp) : run_t<2, 512, 1>(t, q, m, pf, v, b, s, lp);
-      return th == 256 ? run_t<1, 256, 1>(t, q, m, pf, v, b, s, lp) : run_t<1, 512, 1>(t, q, m, pf, v, b, s, lp);
-    }
-    if (qpl == 2) {
-      if (th == 1024) return run_t<2, 1024, 0>(t, q, m, pf, v, b, s, lp);
-      return th == 256 ? run_t<2, 256, 0>(t, q, m, pf, v, b, s, lp) : run_t<2, 512, 0>(t, q, m, pf, v, b, s, lp);
-    }
-    if (th == 1024) return run_t<1, 1024, 0>(t, q, m, pf, v, b, s, lp);
-    return th == 256 ? run_t<1, 256, 0>(t, q, m, pf, v, b, s, lp) : run_t<1, 512, 0>(t, q, m, pf, v, b, s, lp);
+    return C::NODE_BYTES > 128 ? run_t<512, 2>(t, q, m, pf, v, b, s, lp) : run_t<1024, 2>(t, q, m, pf, v, b, s, lp);
   }
 };
 
@@ -874,17 +626,6 @@ int dispatch_f(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
   }
   set_error("unsupported fanout %u", t->F);
   return HBT_EINVAL;
-}
-
-template <typename K>
-uint32_t smem_levels_f(const hbt_tree* t, uint32_t budget) {
-  switch (t->F) {
-    case 4: return Launch<K, 4>::smem_levels(t, budget);
-    case 8: return Launch<K, 8>::smem_levels(t, budget);
-    case 16: return Launch<K, 16>::smem_levels(t, budget);
-    case 32: return Launch<K, 32>::smem_levels(t, budget);
-  }
-  return 0;
 }
 
 }  // namespace
@@ -927,11 +668,6 @@ int implicit_search_items(const hbt_tree* t, const void* q, uint64_t m, uint64_t
 
 int implicit_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
   return implicit_search_base(t, q, m, pf, v, 0, s);
-}
-
-uint32_t implicit_smem_levels(const hbt_tree* t, uint32_t budget) {
-  if (!budget) budget = kDefaultSmemBudget;
-  return t->width == 4 ? smem_levels_f<uint32_t>(t, budget) : smem_levels_f<uint64_t>(t, budget);
 }
 
 }  // namespace hbt

@@ -22,11 +22,9 @@ inline uint32_t item_rounds(uint64_t m, uint32_t sms, uint32_t threads, uint32_t
 }
 
 // One thread asks the TMA unit to pull a contiguous byte range into the L2
-// (cp.async.bulk.prefetch.L2, sm_90+).  Opt-in ("qprefetch"): the item kernels can
-// prefetch the queries of their current and next work item (ncu source page of the c3
-// item search: 15 % of all stall samples on the first compare with a round's query),
-// but it measured slower (c3 item search 1.55 -> 1.58 ms, c4 11.39 -> 11.62 ms).
-// Only whole 16 B units inside the range are requested, in pieces of <= 64 KB.
+// (cp.async.bulk.prefetch.L2, sm_90+): the bucket count pass prefetches its next
+// chunk's queries this way (c3 count 0.167 -> 0.158 ms).  Only whole 16 B units inside
+// the range are requested, in pieces of <= 64 KB.
 __device__ __forceinline__ void prefetch_l2_range(const void* p, uint64_t bytes) {
   const uint64_t a = reinterpret_cast<uint64_t>(p);
   const uint64_t a0 = (a + 15) & ~uint64_t(15);

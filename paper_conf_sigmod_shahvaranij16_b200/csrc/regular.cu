@@ -189,12 +189,7 @@ struct RView {
   const uint32_t* urefs;
   uint64_t uoff[HBT_MAX_LEVELS + 1];
   uint32_t U;
-  uint32_t SL;        // top upper levels staged in shared memory
-  uint32_t root_leaf; // big leaf when U == 0
-  uint64_t smem_first;  // pool index of the first staged upper node
-  uint64_t smem_nodes;
   uint32_t leaf256;     // item search: key line and leaf line by 256-bit lane loads
-  uint32_t l2_hint;     // item search: bit 0 leaf lines L2::evict_first, bit 1 key lines L2::evict_last
 };
 
 template <typename K, int N>
@@ -225,24 +220,6 @@ __device__ __forceinline__ void ld32(L256<K>& v, const uint8_t* p) {
                : "l"(p));
 }
 
-// 256-bit load with an L2 eviction-priority policy (createpolicy)
-template <typename K>
-__device__ __forceinline__ void ld32_pol(L256<K>& v, const uint8_t* p, uint64_t pol) {
-  asm volatile("ld.global.nc.L2::cache_hint.v4.u64 {%0, %1, %2, %3}, [%4], %5;"
-               : "=l"(v.u[0]), "=l"(v.u[1]), "=l"(v.u[2]), "=l"(v.u[3])
-               : "l"(p), "l"(pol));
-}
-__device__ __forceinline__ uint64_t policy_evict_first() {
-  uint64_t pol;
-  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-  return pol;
-}
-__device__ __forceinline__ uint64_t policy_evict_last() {
-  uint64_t pol;
-  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
-  return pol;
-}
-
 template <typename K>
 __device__ __forceinline__ void fill_max32(L256<K>& v) {
 #pragma unroll
@@ -255,198 +232,12 @@ __device__ __forceinline__ V16<K> ld16g(const uint8_t* p) {
   v.u = __ldg(reinterpret_cast<const uint4*>(p));
   return v;
 }
-template <typename K>
-__device__ __forceinline__ V16<K> ld16s(const uint8_t* p) {
-  V16<K> v;
-  v.u = *reinterpret_cast<const uint4*>(p);
-  return v;
-}
 
 __device__ __forceinline__ uint32_t ldcs(const uint32_t* p) { return __ldcs(p); }
 __device__ __forceinline__ uint64_t ldcs(const uint64_t* p) { return __ldcs(reinterpret_cast<const unsigned long long*>(p)); }
 __device__ __forceinline__ void stcs(uint32_t* p, uint32_t v) { __stcs(p, v); }
 __device__ __forceinline__ void stcs(uint64_t* p, uint64_t v) { __stcs(reinterpret_cast<unsigned long long*>(p), (unsigned long long)v); }
 
-// Group of G = 4 lanes per query; each lane holds 16 B of a 64 B key line / leaf
-// line; QPG queries in flight per group (8 groups x QPG = 32 queries per warp round).
-template <typename K, int F, int QPG, int THREADS>
-__global__ void __launch_bounds__(THREADS)
-regular_search_kernel(const RView rv, const K* __restrict__ queries, uint64_t m, uint64_t* __restrict__ out_pf,
-                      K* __restrict__ out_v) {
-  constexpr int G = 4, NG = 8, ROUND = NG * QPG;
-  constexpr uint32_t S = sizeof(K), P = Geo<K>::P, KPL = Geo<K>::KPL, NIP = Geo<K>::NIP;
-  constexpr uint32_t E16 = 16 / S;                       // entries per 16 B lane chunk
-  constexpr uint32_t NI = uint32_t(F) > KPL ? uint32_t(F) / KPL : 1;
-  constexpr uint32_t LINE = uint32_t(F) * S < 64 ? uint32_t(F) * S : 64;  // bytes of one key line
-  constexpr int KL = int(LINE / 16) ? int(LINE / 16) : 1;                 // lanes loading it
-  static_assert(ROUND <= 32, "tiling");
-  extern __shared__ __align__(16) uint8_t smem[];
-  // stage the top SL upper levels: keys | idx | refs (contiguous pool range)
-  const uint64_t NS = rv.smem_nodes;
-  uint8_t* s_keys = smem;
-  uint8_t* s_idx = smem + NS * F * S;
-  uint32_t* s_refs = reinterpret_cast<uint32_t*>(smem + NS * (F * S + NIP * S));
-  {
-    const uint4* a = reinterpret_cast<const uint4*>(rv.ukeys + rv.smem_first * F * S);
-    const uint4* b = reinterpret_cast<const uint4*>(rv.uidx + rv.smem_first * NIP * S);
-    const uint4* c = reinterpret_cast<const uint4*>(rv.urefs + rv.smem_first * F);
-    for (uint64_t i = threadIdx.x; i < NS * F * S / 16; i += THREADS) reinterpret_cast<uint4*>(s_keys)[i] = __ldg(a + i);
-    for (uint64_t i = threadIdx.x; i < NS * NIP * S / 16; i += THREADS) reinterpret_cast<uint4*>(s_idx)[i] = __ldg(b + i);
-    for (uint64_t i = threadIdx.x; i < NS * F * 4 / 16; i += THREADS) reinterpret_cast<uint4*>(s_refs)[i] = __ldg(c + i);
-  }
-  __syncthreads();
-
-  const int lane = threadIdx.x & 31;
-  const int g = lane / G, k = lane % G;
-  const unsigned gmask = 0xFu << (g * G);
-  const uint64_t warp = (uint64_t(blockIdx.x) * THREADS + threadIdx.x) >> 5;
-  const uint64_t nwarps = (uint64_t(gridDim.x) * THREADS) >> 5;
-  const uint64_t rounds = (m + ROUND - 1) / ROUND;
-  const uint32_t U = rv.U, SL = rv.SL;
-
-  for (uint64_t rd = warp; rd < rounds; rd += nwarps) {
-    const uint64_t my_i = rd * ROUND + uint64_t(k) * NG + g;
-    const bool my_ok = (k < QPG) && (my_i < m);
-    const K myq = my_ok ? ldcs(queries + my_i) : key_max<K>();
-    K q[QPG];
-    uint32_t cur[QPG];
-#pragma unroll
-    for (int j = 0; j < QPG; ++j) {
-      q[j] = __shfl_sync(0xffffffffu, myq, g * G + j);
-      cur[j] = U ? uint32_t(rv.uoff[U] - 1) : rv.root_leaf;
-    }
-    // ---- upper levels, root first
-    for (uint32_t l = 0; l < U; ++l) {
-      const bool sm = l < SL;
-      uint32_t t[QPG];
-      if constexpr (NI > 1) {  // (1) index sector: t = #{idx < q}
-        V16<K> iv[QPG];
-#pragma unroll
-        for (int j = 0; j < QPG; ++j) {
-          if (k < 2) {
-            iv[j] = sm ? ld16s<K>(s_idx + (cur[j] - rv.smem_first) * NIP * S + k * 16)
-                       : ld16g<K>(rv.uidx + uint64_t(cur[j]) * NIP * S + k * 16);
-          } else {
-#pragma unroll
-            for (uint32_t e = 0; e < E16; ++e) iv[j].k[e] = key_max<K>();
-          }
-        }
-#pragma unroll
-        for (int j = 0; j < QPG; ++j) {
-          uint32_t c = 0;
-#pragma unroll
-          for (uint32_t e = 0; e < E16; ++e) c += __popc(__ballot_sync(0xffffffffu, iv[j].k[e] < q[j]) & gmask);
-          t[j] = c;
-        }
-      } else {
-#pragma unroll
-        for (int j = 0; j < QPG; ++j) t[j] = 0;
-      }
-      // (2) key line t
-      V16<K> kv[QPG];
-#pragma unroll
-      for (int j = 0; j < QPG; ++j) {
-        if (k < KL) {
-          const uint64_t off = (uint64_t(cur[j]) * F + t[j] * KPL) * S + k * 16;
-          kv[j] = sm ? ld16s<K>(s_keys + (uint64_t(cur[j] - rv.smem_first) * F + t[j] * KPL) * S + k * 16)
-                     : ld16g<K>(rv.ukeys + off);
-        } else {
-#pragma unroll
-          for (uint32_t e = 0; e < E16; ++e) kv[j].k[e] = key_max<K>();
-        }
-      }
-      uint32_t slot[QPG];
-#pragma unroll
-      for (int j = 0; j < QPG; ++j) {
-        uint32_t c = 0;
-#pragma unroll
-        for (uint32_t e = 0; e < E16; ++e) c += __popc(__ballot_sync(0xffffffffu, kv[j].k[e] < q[j]) & gmask);
-        slot[j] = t[j] * KPL + c;
-      }
-      // (3) child reference
-#pragma unroll
-      for (int j = 0; j < QPG; ++j)
-        cur[j] = sm ? s_refs[uint64_t(cur[j] - rv.smem_first) * F + slot[j]]
-                    : __ldg(rv.urefs + uint64_t(cur[j]) * F + slot[j]);
-    }
-    // ---- last level (shares pool index with the big leaf): index sector + key line -> line j
-    uint32_t lj[QPG];
-    {
-      uint32_t t[QPG];
-      if constexpr (NI > 1) {
-        V16<K> iv[QPG];
-#pragma unroll
-        for (int j = 0; j < QPG; ++j) {
-          if (k < 2) iv[j] = ld16g<K>(rv.lidx + uint64_t(cur[j]) * NIP * S + k * 16);
-          else {
-#pragma unroll
-            for (uint32_t e = 0; e < E16; ++e) iv[j].k[e] = key_max<K>();
-          }
-        }
-#pragma unroll
-        for (int j = 0; j < QPG; ++j) {
-          uint32_t c = 0;
-#pragma unroll
-          for (uint32_t e = 0; e < E16; ++e) c += __popc(__ballot_sync(0xffffffffu, iv[j].k[e] < q[j]) & gmask);
-          t[j] = c;
-        }
-      } else {
-#pragma unroll
-        for (int j = 0; j < QPG; ++j) t[j] = 0;
-      }
-      V16<K> kv[QPG];
-#pragma unroll
-      for (int j = 0; j < QPG; ++j) {
-        if (k < KL) kv[j] = ld16g<K>(rv.lkeys + (uint64_t(cur[j]) * F + t[j] * KPL) * S + k * 16);
-        else {
-#pragma unroll
-          for (uint32_t e = 0; e < E16; ++e) kv[j].k[e] = key_max<K>();
-        }
-      }
-#pragma unroll
-      for (int j = 0; j < QPG; ++j) {
-        uint32_t c = 0;
-#pragma unroll
-        for (uint32_t e = 0; e < E16; ++e) c += __popc(__ballot_sync(0xffffffffu, kv[j].k[e] < q[j]) & gmask);
-        lj[j] = t[j] * KPL + c;
-      }
-    }
-    // ---- leaf line (v*F + j): lanes 0-1 keys, 2-3 values
-    V16<K> lv[QPG];
-#pragma unroll
-    for (int j = 0; j < QPG; ++j)
-      lv[j] = ld16g<K>(rv.leaf + (uint64_t(cur[j]) * F + lj[j]) * 64 + k * 16);
-    uint64_t my_pf = 0;
-    K my_v = 0;
-#pragma unroll
-    for (int j = 0; j < QPG; ++j) {
-      uint32_t s = 0;
-#pragma unroll
-      for (uint32_t e = 0; e < E16; ++e) s += __popc(__ballot_sync(0xffffffffu, (k < 2) && (lv[j].k[e] < q[j])) & gmask);
-      const uint32_t sc = s < P ? s : P - 1;
-      const K sel = pick(lv[j].k, sc % E16);
-      const int src = g * G + int(sc / E16);
-      const K key_s = __shfl_sync(0xffffffffu, sel, src);
-      const K val_s = __shfl_sync(0xffffffffu, sel, src + 2);
-      bool end = (s == P);
-      if (!end && key_s == key_max<K>()) {
-        // MAX slot: padding unless it is a counted entry ("must read the node size")
-        const int64_t in_line = int64_t(__ldg(rv.count + cur[j])) - int64_t(lj[j]) * P;
-        const int64_t lim = in_line < int64_t(P) ? in_line : int64_t(P);
-        end = int64_t(s) >= lim;
-      }
-      const bool found = !end && key_s == q[j];
-      if (j == k) {
-        my_pf = end ? kEnd : (((uint64_t(cur[j]) * F + lj[j]) * P + s) | (found ? kFound : 0ull));
-        my_v = found ? val_s : K(0);
-      }
-    }
-    if (my_ok) {
-      stcs(out_pf + my_i, my_pf);
-      stcs(out_v + my_i, my_v);
-    }
-  }
-}
 
 // Search v2 (mode 2, default).  Phase 1: ONE lane per query finds its node at
 // root-first level T through the directory + a lower bound over M_T (shared
@@ -670,11 +461,6 @@ regular_search_items_kernel(const RView rv, const ItemDir d, const K* __restrict
         if (s_bstart[mid] <= p) lo = mid; else hi = mid;
       }
       s_range[threadIdx.x] = threadIdx.x ? ((uint64_t(lo) + 1) * d.U) / d.B - 1 : (uint64_t(lo) * d.U) / d.B;
-    } else if (threadIdx.x == 32 && d.qprefetch) {
-      // this item's queries (needed from the first round) and the next item's
-      if (it == blockIdx.x) prefetch_l2_range(queries + p0, (p1 - p0 + 1) * sizeof(K));
-      const uint64_t n0 = (it + gridDim.x) * W;
-      if (n0 < m) prefetch_l2_range(queries + n0, ((n0 + W < m ? n0 + W : m) - n0) * sizeof(K));
     }
     __syncthreads();
     const uint64_t c0 = s_range[0], c1 = s_range[1];
@@ -726,9 +512,7 @@ regular_search_items_kernel(const RView rv, const ItemDir d, const K* __restrict
 #pragma unroll
         for (int j = 0; j < QPG; ++j) {
           if (uint32_t(k) * 32 < LINE) {
-            const uint8_t* a = rv.lkeys + (uint64_t(cur[j]) * F + t[j] * KPL) * S + k * 32;
-            if (rv.l2_hint & 2u) ld32_pol(kw[j], a, policy_evict_last());
-            else ld32(kw[j], a);
+            ld32(kw[j], rv.lkeys + (uint64_t(cur[j]) * F + t[j] * KPL) * S + k * 32);
           } else {
             fill_max32(kw[j]);
           }
@@ -743,14 +527,8 @@ regular_search_items_kernel(const RView rv, const ItemDir d, const K* __restrict
           line[j] = t[j] * KPL + c;
         }
         L256<K> lw[QPG];
-        if (rv.l2_hint & 1u) {
-          const uint64_t pol = policy_evict_first();
 #pragma unroll
-          for (int j = 0; j < QPG; ++j) ld32_pol(lw[j], rv.leaf + (uint64_t(cur[j]) * F + line[j]) * 64 + k * 32, pol);
-        } else {
-#pragma unroll
-          for (int j = 0; j < QPG; ++j) ld32(lw[j], rv.leaf + (uint64_t(cur[j]) * F + line[j]) * 64 + k * 32);
-        }
+        for (int j = 0; j < QPG; ++j) ld32(lw[j], rv.leaf + (uint64_t(cur[j]) * F + line[j]) * 64 + k * 32);
 #pragma unroll
         for (int j = 0; j < QPG; ++j) {
           uint32_t c = 0;
@@ -837,62 +615,6 @@ regular_search_items_kernel(const RView rv, const ItemDir d, const K* __restrict
   }
 }
 
-constexpr int kThreads = 512;
-constexpr int kQPG = 4;
-
-template <typename K>
-uint64_t upper_node_bytes(uint32_t F) { return uint64_t(F) * sizeof(K) + Geo<K>::NIP * sizeof(K) + 4ull * F; }
-
-template <typename K>
-uint32_t smem_levels_t(const hbt_tree* t, uint32_t budget) {
-  const RegularState& r = t->r;
-  uint32_t SL = 0;
-  while (SL < r.U) {
-    const uint64_t nodes = r.uoff[r.U] - r.uoff[r.U - SL - 1];
-    if (nodes * upper_node_bytes<K>(t->F) > budget) break;
-    ++SL;
-  }
-  return SL;
-}
-
-template <typename K, int F>
-int search_v1_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
-  const RegularState& r = t->r;
-  auto kern = regular_search_kernel<K, F, kQPG, kThreads>;
-  RView rv{};
-  rv.leaf = (const uint8_t*)r.d_leaf;
-  rv.count = r.d_count;
-  rv.lkeys = (const uint8_t*)r.d_lkeys;
-  rv.lidx = (const uint8_t*)r.d_lidx;
-  rv.ukeys = (const uint8_t*)r.d_ukeys;
-  rv.uidx = (const uint8_t*)r.d_uidx;
-  rv.urefs = r.d_urefs;
-  for (uint32_t u = 0; u <= r.U; ++u) rv.uoff[u] = r.uoff[u];
-  rv.U = r.U;
-  rv.root_leaf = r.root_leaf;
-  const uint32_t budget = t->cfg.smem_budget ? t->cfg.smem_budget : 100 * 1024;
-  rv.SL = smem_levels_t<K>(t, budget);
-  rv.smem_first = rv.SL ? r.uoff[r.U - rv.SL] : 0;
-  rv.smem_nodes = rv.SL ? r.uoff[r.U] - rv.smem_first : 0;
-  const size_t smem = rv.smem_nodes * upper_node_bytes<K>(F);
-  static bool attr = false;
-  if (!attr) {
-    HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
-    attr = true;
-  }
-  int occ = 0;
-  HBT_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, smem));
-  if (t->cfg.ctas_per_sm && int(t->cfg.ctas_per_sm) < occ) occ = int(t->cfg.ctas_per_sm);
-  if (occ < 1) occ = 1;
-  const uint64_t rounds = (m + 8 * kQPG - 1) / (8 * kQPG);
-  uint64_t grid = uint64_t(t->num_sms) * occ;
-  const uint64_t need = (rounds + kThreads / 32 - 1) / (kThreads / 32);
-  if (need < grid) grid = need ? need : 1;
-  kern<<<unsigned(grid), kThreads, smem, s>>>(rv, (const K*)q, m, pf, (K*)v);
-  HBT_CUDA_TRY(cudaGetLastError());
-  return HBT_OK;
-}
-
 template <typename K, int F, int QPL, int THREADS>
 int search_v2_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
   const RegularState& r = t->r;
@@ -936,25 +658,6 @@ int search_v2_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf,
   lc.blockDim = dim3(THREADS);
   lc.dynamicSmemBytes = smem;
   lc.stream = s;
-  cudaLaunchAttribute la[1];
-  lc.attrs = la;
-  lc.numAttrs = 0;
-  if (t->cfg.l2_persist) {
-    // keep the last level's index sectors (one 32 B sector per big leaf) resident
-    static uint64_t limit_set = 0;
-    const uint64_t win = std::min<uint64_t>(t->cfg.l2_persist, r.pool * 32);
-    if (limit_set < win) {
-      HBT_CUDA_TRY(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, win));
-      limit_set = win;
-    }
-    la[0].id = cudaLaunchAttributeAccessPolicyWindow;
-    la[0].val.accessPolicyWindow.base_ptr = r.d_lidx;
-    la[0].val.accessPolicyWindow.num_bytes = win;
-    la[0].val.accessPolicyWindow.hitRatio = 1.0f;
-    la[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-    la[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-    lc.numAttrs = 1;
-  }
   HBT_CUDA_TRY(cudaLaunchKernelEx(&lc, kern, rv, rd, (const uint32_t*)r.d_dir, (const uint32_t*)r.d_chain, (const K*)q,
                                   m, pf, (K*)v));
   return HBT_OK;
@@ -974,7 +677,6 @@ int search_items_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* 
   rv.lidx = (const uint8_t*)r.d_lidx;
   rv.U = r.U;
   rv.leaf256 = t->cfg.leaf256;
-  rv.l2_hint = t->cfg.regular_l2_hint;
   const size_t smem = (d.B + 1) * 8 + size_t(d.cap) * (sizeof(K) + 4) + ((1u << kPrefixBits) + 1) * 4;
   static bool attr = false;
   if (!attr) {
@@ -993,15 +695,7 @@ int search_items_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* 
 
 template <typename K, int F>
 int search_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
-  if (t->cfg.mode == 2) {
-    const uint32_t th = t->cfg.threads ? t->cfg.threads : 1024;
-    const uint32_t qpl = t->cfg.qpl ? t->cfg.qpl : 1;
-    if (qpl == 2) return th == 512 ? search_v2_launch<K, F, 2, 512>(t, q, m, pf, v, s)
-                                   : search_v2_launch<K, F, 2, 1024>(t, q, m, pf, v, s);
-    return th == 512 ? search_v2_launch<K, F, 1, 512>(t, q, m, pf, v, s)
-                     : search_v2_launch<K, F, 1, 1024>(t, q, m, pf, v, s);
-  }
-  return search_v1_launch<K, F>(t, q, m, pf, v, s);
+  return search_v2_launch<K, F, 1, 1024>(t, q, m, pf, v, s);
 }
 
 template <typename K>
@@ -1114,6 +808,7 @@ int reserve_for_update(hbt_tree* t, uint64_t pool_need, uint64_t nchain_bound, c
   if (r.chainpos_cap < r.cap) {
     uint32_t* cp = nullptr;
     HBT_CUDA_TRY(cudaMalloc(&cp, r.cap * 4));
+    HBT_CUDA_TRY(cudaMemsetAsync(cp, 0xFF, r.cap * 4, s));
     if (r.chainpos_cap) HBT_CUDA_TRY(cudaMemcpyAsync(cp, r.d_chainpos, r.chainpos_cap * 4, cudaMemcpyDeviceToDevice, s));
     HBT_CUDA_TRY(cudaStreamSynchronize(s));
     cudaFree(r.d_chainpos);
@@ -1195,6 +890,7 @@ int rebuild_dir(hbt_tree* t, cudaStream_t s) {
     r.d_chainpos = nullptr;
     r.chainpos_cap = 0;
     HBT_CUDA_TRY(cudaMalloc(&r.d_chainpos, r.cap * 4));
+    HBT_CUDA_TRY(cudaMemsetAsync(r.d_chainpos, 0xFF, r.cap * 4, s));  // dead leaves: no position
     r.chainpos_cap = r.cap;
   }
   chain_positions<<<grid_for(r.nchain), 256, 0, s>>>(r.d_chain, r.nchain, r.d_chainpos);
@@ -1798,20 +1494,27 @@ int regular_clone(const hbt_tree* src, hbt_tree* dst, cudaStream_t s) {
   b.d_leaf = b.d_lkeys = b.d_lidx = b.d_ukeys = b.d_uidx = b.d_dir = nullptr;
   b.d_count = b.d_chain = b.d_urefs = b.d_seg_of_leaf = b.d_chainpos = nullptr;
   b.h_leaf = nullptr;
-  auto dup = [&](void** d, const void* p, uint64_t bytes) -> int {
-    if (!p || !bytes) return HBT_OK;
-    HBT_CUDA_TRY(cudaMalloc(d, bytes));
-    HBT_CUDA_TRY(cudaMemcpyAsync(*d, p, bytes, cudaMemcpyDeviceToDevice, s));
+  // same capacities; only the live prefix of each array is copied (the rest is
+  // never read before it is written)
+  auto dup = [&](void** d, const void* p, uint64_t cap_bytes, uint64_t live_bytes) -> int {
+    if (!p || !cap_bytes) return HBT_OK;
+    HBT_CUDA_TRY(cudaMalloc(d, cap_bytes));
+    if (live_bytes) HBT_CUDA_TRY(cudaMemcpyAsync(*d, p, live_bytes, cudaMemcpyDeviceToDevice, s));
     return HBT_OK;
   };
+  const uint64_t up = a.uoff[a.U];
   int rc;
-  if ((rc = dup(&b.d_leaf, a.d_leaf, a.cap * F * 64)) || (rc = dup((void**)&b.d_count, a.d_count, a.cap * 4)) ||
-      (rc = dup(&b.d_lkeys, a.d_lkeys, a.cap * F * S)) || (rc = dup(&b.d_lidx, a.d_lidx, a.cap * 32)) ||
-      (rc = dup((void**)&b.d_chain, a.d_chain, a.cap * 4)) || (rc = dup(&b.d_ukeys, a.d_ukeys, a.ucap * F * S)) ||
-      (rc = dup(&b.d_uidx, a.d_uidx, a.ucap * 32)) || (rc = dup((void**)&b.d_urefs, a.d_urefs, a.ucap * F * 4)) ||
-      (rc = dup((void**)&b.d_seg_of_leaf, a.d_seg_of_leaf, a.seg_cap * 4)) ||
-      (rc = dup(&b.d_dir, a.d_dir, a.dir_cap)) ||
-      (rc = dup((void**)&b.d_chainpos, a.d_chainpos, a.chainpos_cap * 4)))
+  if ((rc = dup(&b.d_leaf, a.d_leaf, a.cap * F * 64, a.pool * F * 64)) ||
+      (rc = dup((void**)&b.d_count, a.d_count, a.cap * 4, a.pool * 4)) ||
+      (rc = dup(&b.d_lkeys, a.d_lkeys, a.cap * F * S, a.pool * F * S)) ||
+      (rc = dup(&b.d_lidx, a.d_lidx, a.cap * 32, a.pool * 32)) ||
+      (rc = dup((void**)&b.d_chain, a.d_chain, a.cap * 4, a.nchain * 4)) ||
+      (rc = dup(&b.d_ukeys, a.d_ukeys, a.ucap * F * S, up * F * S)) ||
+      (rc = dup(&b.d_uidx, a.d_uidx, a.ucap * 32, up * 32)) ||
+      (rc = dup((void**)&b.d_urefs, a.d_urefs, a.ucap * F * 4, up * F * 4)) ||
+      (rc = dup((void**)&b.d_seg_of_leaf, a.d_seg_of_leaf, a.seg_cap * 4, a.seg_cap * 4)) ||
+      (rc = dup(&b.d_dir, a.d_dir, a.dir_cap, a.dir_bytes)) ||
+      (rc = dup((void**)&b.d_chainpos, a.d_chainpos, a.chainpos_cap * 4, a.chainpos_cap * 4)))
     return rc;
   HBT_CUDA_TRY(cudaStreamSynchronize(s));
   return HBT_OK;
@@ -1826,9 +1529,5 @@ void regular_free(hbt_tree* t) {
   r = RegularState{};
 }
 
-uint32_t regular_smem_levels(const hbt_tree* t, uint32_t budget) {
-  if (!budget) budget = 100 * 1024;
-  return t->width == 4 ? smem_levels_t<uint32_t>(t, budget) : smem_levels_t<uint64_t>(t, budget);
-}
 
 }  // namespace hbt

@@ -49,7 +49,6 @@ def test_bucketed_edge_suite(hbt, layout, width, F, items, cap, leaf256):
         t.set_param("leaf256", leaf256)
         for slice_bytes in (1, 4096, 1 << 16):  # 1 B: one bucket per unit up to the 1024 cap
             t.set_param("bucket_slice", slice_bytes)
-            t.set_param("item_group4", int(slice_bytes == 4096))
             pf, val = gpu_search(t, q, width)
             assert np.array_equal(pf, epf), (layout, n, F, width, slice_bytes, items, cap,
                                              np.nonzero(pf != epf)[0][:5])
@@ -74,11 +73,11 @@ def test_bucketed_scaled_workload(hbt, layout, F, items, cap, leaf256):
     t.set_param("leaf256", leaf256)
     for slice_bytes in (1 << 16, 1 << 20, 1 << 22):
         t.set_param("bucket_slice", slice_bytes)
-        for qpf in (0, 1):  # with / without the bulk L2 prefetch of each item's queries
-            t.set_param("qprefetch", qpf)
-            t.set_param("item_group4", qpf)  # 2- and 4-lane groups in the implicit item search
+        for qpf in (0, 1):  # default and single-round work items
+            t.set_param("item_rounds", 1 if qpf else 0)
             for hint in (0, 1, 3):  # L2 eviction-priority hints on the item search's loads
-                t.set_param("item_l2_hint" if layout == "implicit" else "regular_l2_hint", hint)
+                if layout == "implicit":
+                    t.set_param("item_l2_hint", hint)
                 pf, val = gpu_search(t, q, 8)
                 assert np.array_equal(pf, epf) and np.array_equal(val, ev), (layout, slice_bytes, qpf, hint)
     t.set_param("bucket", 0)

@@ -47,15 +47,11 @@ def test_random_knob_parity(hbt, case):
     t = gpu_build(hbt, k, v, F, width, layout=layout)
     knobs = {}
     if layout == "implicit":
-        knobs["smem_mode"] = int(rng.choice([0, 1, 2, 3, 4]))
+        knobs["smem_mode"] = int(rng.choice([2, 3]))
         knobs["l2_levels_bytes"] = int(rng.choice([0, 1, 4096]))
         knobs["full256"] = int(rng.integers(0, 2))
-        knobs["sec256"] = int(rng.integers(0, 2))
         knobs["small_batch"] = int(rng.choice([0, 1 << 16]))
-        if knobs["smem_mode"] == 2:
-            knobs["threads"] = int(rng.choice([0, 512, 768, 1024]))
-    else:
-        knobs["smem_mode"] = int(rng.choice([0, 2]))
+        knobs["ctas_per_sm"] = int(rng.choice([0, 1, 2]))
     knobs["leaf256"] = int(rng.integers(0, 2))
     knobs["bucket"] = int(rng.choice([0, 1, 2]))
     if knobs["bucket"]:
@@ -72,9 +68,7 @@ def test_random_knob_parity(hbt, case):
     hrng = np.random.default_rng(case + 7777)
     knobs["l2_hint"] = int(hrng.integers(0, 5))
     knobs["item_l2_hint"] = int(hrng.integers(0, 4))
-    knobs["regular_l2_hint"] = int(hrng.integers(0, 4))
-    knobs["item_group4"] = int(hrng.integers(0, 2))
-    knobs["small_threads"] = int(hrng.choice([0, 128, 256, 1024]))
+    knobs["item_rounds"] = int(hrng.choice([0, 1, 3, 16]))
     for name, val in knobs.items():
         t.set_param(name, val)
     q = _queries(k, width, rng, int(rng.choice([1, 31, 1000, 40000])))

@@ -37,7 +37,7 @@ def test_host_leaves_search_modes(hbt, width, F):
         assert t.export(hbt.SEG_LEAF).tobytes() == leaf  # the copy is bitwise the build
         q = query_set(k, width, rng, 20000)
         epf, ev = o.search(q)
-        for mode, l2b in ((2, 0), (2, 1), (3, 0), (0, 0)):
+        for mode, l2b in ((2, 0), (2, 1), (3, 0), (3, 1)):
             t.set_search_config(smem_mode=mode)
             t.set_param("l2_levels_bytes", l2b)
             t.set_param("small_batch", 0)
@@ -114,7 +114,7 @@ def test_host_leaves_regular(hbt, width, F):
     for rep in range(3):
         q = query_set(k, width, rng, 20000)
         epf, ev = o.search(q)
-        for mode, bucket in ((2, 0), (0, 0), (2, 1)):
+        for mode, bucket in ((2, 0), (3, 0), (2, 1)):
             t.set_search_config(smem_mode=mode)
             t.set_param("bucket", bucket)
             pf, val = gpu_search(t, q, width)

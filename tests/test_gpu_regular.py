@@ -60,11 +60,11 @@ def test_regular_edge_suite_parity(hbt, width, F):
         check_arrays(hbt, t, o, width)
         q = query_set(k, width, rng, 3000)
         epf, ev = o.search(q)
-        for mode, th, qpl in ((2, 0, 0), (0, 0, 0), (2, 512, 2)):  # directory v2 / staged v1 / shapes
-            t.set_search_config(smem_mode=mode, threads_per_cta=th, queries_per_lane=qpl)
+        for ctas in (0, 1):  # launch shapes
+            t.set_search_config(ctas_per_sm=ctas)
             pf, val = gpu_search(t, q, width)
-            assert np.array_equal(pf, epf), (mode, n, F, width, np.nonzero(pf != epf)[0][:5])
-            assert np.array_equal(val, ev), (mode, n, F, width)
+            assert np.array_equal(pf, epf), (ctas, n, F, width, np.nonzero(pf != epf)[0][:5])
+            assert np.array_equal(val, ev), (ctas, n, F, width)
         t.close()
 
 
@@ -102,11 +102,9 @@ def test_regular_update_parity(hbt, width, F):
             check_arrays(hbt, t, o, width)
             q = query_set(ok[:300], width, rng, 3000)
             epf, ev = o.search(q)
-            for mode in (2, 0):
-                t.set_search_config(smem_mode=mode)
-                pf, val = gpu_search(t, q, width)
-                assert np.array_equal(pf, epf), (mode, trial, batch)
-                assert np.array_equal(val, ev), (mode, trial, batch)
+            pf, val = gpu_search(t, q, width)
+            assert np.array_equal(pf, epf), (trial, batch)
+            assert np.array_equal(val, ev), (trial, batch)
         assert t.info()["n_distinct"] == 0
 
 
