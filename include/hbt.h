@@ -136,7 +136,10 @@ HBT_API int hbt_bulk_build(const void* keys, const void* values, uint64_t n, uin
                    uint32_t layout, void* stream, hbt_tree** out);
 
 /* Look up m queries (device array of width S) into out (device arrays, length
- * m).  Asynchronous on `stream`.  m = 0 is a no-op. */
+ * m): the paper's batched search (the problem statement of §4.1; node
+ * search rule P:190, reading R1; implicit child index P:126; regular node P:134-138).
+ * Asynchronous on `stream`.  m = 0 is a no-op.  Large batches over trees far beyond the
+ * L2 are partitioned by key range first ("bucket"); results are identical either way. */
 HBT_API int hbt_search(const hbt_tree* t, const void* queries, uint64_t m, hbt_out out, void* stream);
 
 /* End-to-end lookup with HOST buffers: copies queries host->device, searches and
@@ -272,14 +275,27 @@ HBT_API int hbt_comm_init(int nranks, int rank, const void* id128, hbt_comm** ou
  * (exchange = 0).  Works with any number of ranks per GPU. */
 HBT_API int hbt_comm_init_host(int nranks, int rank, hbt_allgather_fn fn, void* ctx, hbt_comm** out);
 HBT_API int hbt_comm_destroy(hbt_comm* c);
+/* Collective, host only (no device work): all-gather every rank's (n', min key, max key)
+ * through the communicator and check that the non-empty shards are in key order.
+ * Writes, per rank g (arrays of nranks entries): counts[g] = n'_g, bases[g] = the
+ * shard's first global rank (sum of earlier counts), maxima[g] = its max key (the
+ * routing table of owner(q) = #(shard_max < q)).  HBT_EINVAL if ranges overlap or are
+ * out of order.  hbt_bulk_build_sharded calls it after building the local shard. */
+HBT_API int hbt_comm_shard_table(hbt_comm* c, uint64_t n_local, uint64_t kmin, uint64_t kmax, uint64_t* counts,
+                                 uint64_t* bases, uint64_t* maxima);
 /* Collective: every rank builds its shard from its local (device) pairs, then the
  * ranks all-gather (n', min, max).  HBT_EINVAL if shard ranges overlap. */
 HBT_API int hbt_bulk_build_sharded(hbt_comm* c, const void* keys_local, const void* values_local,
                                    uint64_t n_local, uint32_t fanout, uint32_t layout, void* stream,
                                    hbt_tree** out);
-/* Collective: every rank searches its local batch; queries and results cross
- * NVLink by NCCL send/recv (an all-to-all).  Host-synchronous on the count
- * exchange (one small D2H per batch). */
+/* Collective: every rank searches its local batch (the north_star's routed search,
+ * SURVEY §8(e).2, P:186-196 per shard).  Exchange "exchange" = 0 (default): the fused
+ * peer-memory exchange — count rows and queries are stored straight into the owners'
+ * IPC-mapped windows, device flag barriers order the steps, and the owner's bucketed
+ * gather stores each result into the requester's window (sharded_fused.cu); 1: NCCL
+ * send/recv of counts, queries and results (an all-to-all) + unpermute.  One small D2H
+ * of the count matrix per batch (host-synchronous there).  A ONE-shard tree searches in
+ * place ("g1_direct").  Positions are global (shard base rank + local rank). */
 HBT_API int hbt_search_sharded(const hbt_tree* t, const void* queries_local, uint64_t m_local,
                                hbt_out out_local, void* stream);
 /* Single-process shard group on ONE device (tests, capacity planning): mark G

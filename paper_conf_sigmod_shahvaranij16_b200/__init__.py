@@ -39,7 +39,7 @@ EXPORTED = ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update"
             "hbt_range", "hbt_comm_unique_id", "hbt_comm_init", "hbt_comm_init_host", "hbt_comm_destroy", "hbt_bulk_build_sharded",
             "hbt_search_sharded", "hbt_shard_local_init", "hbt_search_sharded_local", "hbt_last_phases",
             "hbt_set_leaf_placement", "hbt_get_leaf_placement", "hbt_versioned_create", "hbt_versioned_search",
-            "hbt_versioned_update", "hbt_versioned_current", "hbt_versioned_destroy"]
+            "hbt_versioned_update", "hbt_versioned_current", "hbt_versioned_destroy", "hbt_comm_shard_table"]
 
 
 class HBTError(RuntimeError):
@@ -103,6 +103,7 @@ def _load():
     L.hbt_versioned_update.argtypes = [vp, C.POINTER(_Batch), vp, C.POINTER(u64)]
     L.hbt_versioned_current.argtypes = [vp, C.POINTER(vp), C.POINTER(u64)]
     L.hbt_versioned_destroy.argtypes = [vp]
+    L.hbt_comm_shard_table.argtypes = [vp, u64, u64, u64, vp, vp, vp]
     L.hbt_last_error.restype = C.c_char_p
     L.hbt_version.restype = C.c_char_p
     for f in ["hbt_bulk_build", "hbt_search", "hbt_search_host", "hbt_bulk_update", "hbt_destroy",
@@ -111,7 +112,7 @@ def _load():
               "hbt_comm_destroy", "hbt_bulk_build_sharded", "hbt_search_sharded", "hbt_shard_local_init",
               "hbt_search_sharded_local", "hbt_last_phases", "hbt_set_leaf_placement",
               "hbt_get_leaf_placement", "hbt_versioned_create", "hbt_versioned_search", "hbt_versioned_update",
-              "hbt_versioned_current", "hbt_versioned_destroy"]:
+              "hbt_versioned_current", "hbt_versioned_destroy", "hbt_comm_shard_table"]:
         getattr(L, f).restype = C.c_int
     return L
 
@@ -422,6 +423,14 @@ class Comm:
         _check(lib.hbt_comm_init_host(1, 0, self._fn, None, C.byref(h)))
         self._h, self.nranks, self.rank = h, 1, 0
         return self
+
+    def shard_table(self, n_local: int, kmin: int, kmax: int):
+        """Collective, host only: (counts, bases, maxima) of every rank's shard (uint64
+        numpy arrays), the routing table of the key-range-sharded search."""
+        arr = [np.zeros(self.nranks, np.uint64) for _ in range(3)]
+        _check(lib.hbt_comm_shard_table(self._h, int(n_local), int(kmin), int(kmax),
+                                        *[C.c_void_p(a.ctypes.data) for a in arr]))
+        return tuple(arr)
 
     def close(self):
         if getattr(self, "_h", None) and self._h.value:

@@ -437,6 +437,27 @@ int hbt_comm_destroy(hbt_comm* c) {
   return HBT_OK;
 }
 
+int hbt_comm_shard_table(hbt_comm* c, uint64_t n_local, uint64_t kmin, uint64_t kmax, uint64_t* counts,
+                         uint64_t* bases, uint64_t* maxima) {
+  if (!c || !counts || !bases || !maxima) { set_error("NULL argument"); return HBT_EINVAL; }
+  NvtxRange nvtx_("hbt_comm_shard_table");
+  const int G = c->nranks;
+  uint64_t mine[3] = {n_local, kmin, kmax};
+  std::vector<uint64_t> all(3 * G);
+  int rc = comm_allgather_host(c, mine, all.data(), sizeof(mine), nullptr);
+  if (rc) return rc;
+  std::vector<uint64_t> cn(G), mnv(G), mxv(G);
+  for (int g = 0; g < G; ++g) { cn[g] = all[3 * g]; mnv[g] = all[3 * g + 1]; mxv[g] = all[3 * g + 2]; }
+  ShardMeta sm;
+  if ((rc = validate_and_set(sm, cn, mnv, mxv, G))) return rc;
+  for (int g = 0; g < G; ++g) {
+    counts[g] = sm.count[g];
+    bases[g] = sm.base[g];
+    maxima[g] = sm.max[g];
+  }
+  return HBT_OK;
+}
+
 int hbt_bulk_build_sharded(hbt_comm* c, const void* keys_local, const void* values_local, uint64_t n_local,
                            uint32_t fanout, uint32_t layout, void* stream, hbt_tree** out) {
   NvtxRange nvtx_("hbt_bulk_build_sharded");
@@ -448,18 +469,19 @@ int hbt_bulk_build_sharded(hbt_comm* c, const void* keys_local, const void* valu
   const int G = c->nranks;
   uint64_t mn = 0, mx = 0;
   if ((rc = first_last_keys(t, &mn, &mx))) { hbt_destroy(t); *out = nullptr; return rc; }
-  // all-gather (n', min, max) of every shard
-  cudaStream_t st = (cudaStream_t)stream;
-  uint64_t mine[3] = {t->n, mn, mx};
-  std::vector<uint64_t> all(3 * G);
-  if ((rc = comm_allgather_host(c, mine, all.data(), sizeof(mine), st))) {
+  // all-gather (n', min, max) of every shard, validate the key order, set the routing table
+  std::vector<uint64_t> cn(G), bs(G), mxv(G);
+  if ((rc = hbt_comm_shard_table(c, t->n, mn, mx, cn.data(), bs.data(), mxv.data()))) {
     hbt_destroy(t);
     *out = nullptr;
     return rc;
   }
-  std::vector<uint64_t> cn(G), mnv(G), mxv(G);
-  for (int g = 0; g < G; ++g) { cn[g] = all[3 * g]; mnv[g] = all[3 * g + 1]; mxv[g] = all[3 * g + 2]; }
-  if ((rc = validate_and_set(t->shard, cn, mnv, mxv, G))) { hbt_destroy(t); *out = nullptr; return rc; }
+  t->shard.G = G;
+  for (int g = 0; g < G; ++g) {
+    t->shard.count[g] = cn[g];
+    t->shard.base[g] = bs[g];
+    t->shard.max[g] = mxv[g];
+  }
   t->shard.comm = c;
   t->shard.rank = c->rank;
   return HBT_OK;

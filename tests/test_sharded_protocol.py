@@ -156,3 +156,63 @@ def test_host_allgather_communicator_two_ranks_gloo():
         p.join(timeout=60)
         assert p.exitcode == 0
     assert all(ok for _, ok in res), res
+
+
+def _shard_table_worker(rank, world, port, case, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import paper_conf_sigmod_shahvaranij16_b200 as hbt
+        comm = hbt.Comm.from_torch_host()
+        n = 3000
+        allk = gen.stratified_keys(n, 11)
+        lo, hi = hbt.shard_plan(n, world, rank)
+        if case == "empty_middle" and rank == 1:
+            lo = hi = 0
+        if case == "overlap" and rank == 1:
+            lo -= 5  # shares five keys with rank 0's range
+        if case == "out_of_order":  # rank 0 holds the upper range
+            lo, hi = hbt.shard_plan(n, world, world - 1 - rank)
+        k = allk[lo:hi]
+        try:
+            counts, bases, maxima = comm.shard_table(len(k), int(k.min()) if len(k) else 0,
+                                                     int(k.max()) if len(k) else 0)
+            got = ("ok", counts.tolist(), bases.tolist(), maxima.tolist())
+        except hbt.HBTError as e:
+            got = ("err", e.code)
+        comm.close()
+        q.put((rank, got))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("case", ["even3", "empty_middle", "overlap", "out_of_order"])
+def test_library_shard_table_gloo(case):
+    """The library's own multi-process host path (hbt_comm_shard_table: all-gather of
+    every rank's (n', min, max) through the host-callback communicator over gloo, key-order
+    validation, bases and maxima of the routing table), no GPU needed."""
+    world = 3 if case in ("even3", "empty_middle") else 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_shard_table_worker, args=(r, world, port, case, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=300) for _ in procs)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    import paper_conf_sigmod_shahvaranij16_b200 as hbt
+    if case in ("overlap", "out_of_order"):
+        assert all(r == ("err", hbt.EINVAL) for r in res.values()), res
+        return
+    allk = gen.stratified_keys(3000, 11)
+    spans = [hbt.shard_plan(3000, world, r) for r in range(world)]
+    if case == "empty_middle":
+        spans[1] = (0, 0)
+    counts = [hi - lo for lo, hi in spans]
+    bases = list(np.cumsum([0] + counts)[:-1])
+    maxima = [int(allk[hi - 1]) if hi > lo else 0 for lo, hi in spans]
+    for r in range(world):
+        assert res[r] == ("ok", counts, bases, maxima), (r, res[r])
