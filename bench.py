@@ -351,9 +351,17 @@ def make_work(cfg_name, d, args):
     if args.leaf_host:
         tree.set_leaf_placement("host")  # f4: L-segment in pinned host memory
         qdesc += "; L-segment in pinned host memory, leaf lines read by zero-copy loads over the host link"
+    params = {}
     for kv in args.param:
         name, val = kv.split("=", 1)
-        tree.set_param(name, int(val, 0))
+        params[name] = int(val, 0)
+    # the host pipeline of the e2e number: c4's 2^28-query batch in 4 Mi-query chunks, each
+    # chunk's search bucketed, copies both ways overlapping the searches (D2H-bound:
+    # 1.99 -> 3.27 G q/s against H2D + search + D2H in sequence, profiles/r02_c4_e2e_sweep.jsonl)
+    params.setdefault("host_chunk_log2", 22 if cfg_name == "c4" else 20)
+    params.setdefault("host_bufs", 2)
+    for name, val in params.items():
+        tree.set_param(name, val)
     out_pos = torch.empty(m, dtype=torch.int64, device="cuda")
     out_val = torch.empty(m, dtype=sdt, device="cuda")
     hi = None
@@ -375,6 +383,7 @@ def make_work(cfg_name, d, args):
                   "gval": torch.empty(world * m, dtype=sdt, device="cuda") if rank == 0 else None}
         qdesc += "; the queries of all ranks originate on rank 0 (scatter + gather inside each step)"
     return Work(c=c, name=cfg_name, tree=tree, q=q, m=m, w=w, hit_rate=hit_rate, qdesc=qdesc, extra=extra,
+                host_chunk_log2=params["host_chunk_log2"], host_bufs=params["host_bufs"],
                 out_pos=out_pos, out_val=out_val, info=tree.info(), range_k=args.range_k, hi=hi,
                 origin=origin, rank=rank, world=world, dist=d)
 
@@ -498,7 +507,9 @@ def time_e2e(work, steps):
     hq = work.q.cpu().pin_memory()
     hp = torch.empty(m, dtype=torch.int64).pin_memory()
     hv = torch.empty(m, dtype=work.q.dtype).pin_memory()
-    sharded = work.name == "c4"
+    # a multi-rank sharded search is a collective over every rank's whole batch; one
+    # shard (N = 1) is an ordinary tree for the host pipeline (global pos = local rank)
+    sharded = work.name == "c4" and d.world > 1
 
     def one():
         if sharded:  # H2D, collective search, D2H on the current stream
@@ -519,7 +530,8 @@ def time_e2e(work, steps):
     el = d.max(time.perf_counter() - t0)
     qps = d.world * m * steps / el
     api = ("H2D + hbt_search_sharded + D2H (pinned host buffers)" if sharded else
-           "hbt_search_host (pinned host buffers, 1 Mi-query buckets double-buffered over 2 streams)")
+           "hbt_search_host (pinned host buffers; chunks of 2^%d queries: H2D, search, D2H pipelined over %d "
+           "streams)" % (work.host_chunk_log2, work.host_bufs))
     return {"value": round(qps / 1e6, 2), "unit": "M queries/s", "h2d_bytes_per_step": m * w,
             "d2h_bytes_per_step": m * (8 + w), "api": api}
 
