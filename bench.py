@@ -617,7 +617,9 @@ def run_hbt(args):
         t_kernel = phases["search"] * 1e-3
         kernel = ("regular_search_items_kernel" if c["layout"] == "regular" else "implicit_search_items_kernel")
         # c4: the sharded step's own kernels (count / publish / barrier / return) + the pipeline
-        launches_per_step = phases["launches"] + (3 if args.config == "c4" and world > 1 else 0)
+        # c4 at N > 1, fused exchange: f_count, f_publish, f_put and three device barriers
+        # around the owner's bucketed search (whose gather stores into the requesters' windows)
+        launches_per_step = phases["launches"] + (6 if args.config == "c4" and world > 1 else 0)
         model_desc = "bucketed search: query + 16 B record + distinct tree lines per pass (tools/roofline.py)"
     else:
         mdl = roofline.model(info, l2_size, work.hit_rate)
