@@ -116,14 +116,21 @@ __global__ void f_publish(const PeerTable pt, int me, const unsigned long long* 
   }
 }
 
-// Route + put: queries go straight into their owner's receive window.
+// Route + put: queries go straight into their owner's receive window.  Each CTA
+// reserves one block per destination for its chunk of the batch and fills it in SOURCE
+// ORDER (warp match + a per-destination prefix over the CTA's warps), so a run of the
+// owner's window holds one source chunk's queries in index order and the results the
+// owner stores back into the requester's window land on nearly consecutive indices.
 template <typename K>
 __global__ void __launch_bounds__(kThreads) f_put(const K* __restrict__ q, uint64_t m, const uint8_t* __restrict__ dest,
                                                   const PeerTable pt, int me, int parity,
                                                   unsigned long long* __restrict__ cursor, uint64_t chunk) {
+  constexpr int W = kThreads / 32;
   __shared__ unsigned int h[kMaxG];
   __shared__ unsigned long long base[kMaxG];
+  __shared__ unsigned int wc[W][kMaxG];
   const int G = pt.G;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const uint64_t lo = blockIdx.x * chunk;
   const uint64_t hi = lo + chunk < m ? lo + chunk : m;
   for (int i = threadIdx.x; i < G; i += blockDim.x) h[i] = 0;
@@ -135,14 +142,34 @@ __global__ void __launch_bounds__(kThreads) f_put(const K* __restrict__ q, uint6
     unsigned long long start = 0;  // earlier sources' share of destination d
     for (int s = 0; s < me; ++s) start += M[s * kMaxG + d];
     base[d] = h[d] ? start + atomicAdd(cursor + d, (unsigned long long)h[d]) : 0ull;
-    h[d] = 0;
+    h[d] = 0;  // from here on: queries of this chunk already placed, per destination
   }
-  __syncthreads();
-  for (uint64_t i = lo + threadIdx.x; i < hi; i += blockDim.x) {
-    const uint32_t d = dest[i];
-    const uint64_t slot = base[d] + atomicAdd(&h[d], 1u);
-    reinterpret_cast<K*>(pt.w[d].recv_q)[slot] = q[i];
-    pt.w[d].recv_org[slot] = (uint64_t(me) << kOrgShift) | i;
+  for (uint64_t r0 = lo; r0 < hi; r0 += blockDim.x) {
+    __syncwarp();  // every lane of this warp has read its row of the previous round
+    for (int d = lane; d < G; d += 32) wc[w][d] = 0;
+    __syncthreads();  // base / h ready (first round), previous round's slots read
+    const uint64_t i = r0 + threadIdx.x;
+    const bool v = i < hi;
+    const uint32_t d = v ? dest[i] : 0xFFu;
+    const unsigned peers = __match_any_sync(0xffffffffu, d);
+    const unsigned before = peers & ((1u << lane) - 1u);
+    if (v && before == 0) wc[w][d] = __popc(peers);
+    __syncthreads();
+    if (threadIdx.x < G) {  // exclusive prefix over the warps, continuing the chunk's count
+      unsigned run = h[threadIdx.x];
+      for (int x = 0; x < W; ++x) {
+        const unsigned c = wc[x][threadIdx.x];
+        wc[x][threadIdx.x] = run;
+        run += c;
+      }
+      h[threadIdx.x] = run;
+    }
+    __syncthreads();
+    if (v) {
+      const uint64_t slot = base[d] + wc[w][d] + __popc(before);
+      reinterpret_cast<K*>(pt.w[d].recv_q)[slot] = q[i];
+      pt.w[d].recv_org[slot] = (uint64_t(me) << kOrgShift) | i;
+    }
   }
 }
 
