@@ -471,8 +471,9 @@ __global__ void __launch_bounds__(kGThreads) bk_gather_rec(const uint16_t* __res
   // thread's record and linv loads are issued together (the kernel was latency
   // bound: long-scoreboard stalls 38 per issue, one CTA per SM).  REMOTE (the owner
   // side of the fused sharded exchange): query i of the receive window came from
-  // rank org[i] >> 40, index org[i] & (2^40 - 1) there, and its record is stored
-  // straight into THAT rank's result window (peer memory).
+  // rank s = org[i] >> 40, and its record is stored straight into THAT rank's result
+  // window (peer memory) at i - start[s] + dst[s]: consecutive receive slots of one
+  // source land on consecutive result slots there (coalesced peer stores).
   static_assert(kMaxBuckets <= kGThreads, "one bucket per thread");
   constexpr int PT = int(kChunk) / kGThreads;
   extern __shared__ __align__(16) uint8_t smem[];
@@ -538,9 +539,9 @@ __global__ void __launch_bounds__(kGThreads) bk_gather_rec(const uint16_t* __res
         if (t < nc) {
           const ulonglong2 r = s_rec[l[j]];
           const uint32_t src = uint32_t(o[j] >> kRemoteOrgShift);
-          const uint64_t idx = o[j] & ((1ull << kRemoteOrgShift) - 1);
-          ro.pf[src][idx] = r.x;
-          reinterpret_cast<K*>(ro.v[src])[idx] = K(r.y);
+          const uint64_t slot = lo + t - ro.start[src] + ro.dst[src];
+          ro.pf[src][slot] = r.x;
+          reinterpret_cast<K*>(ro.v[src])[slot] = K(r.y);
         }
       }
     } else {

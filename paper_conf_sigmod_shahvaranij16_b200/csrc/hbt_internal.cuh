@@ -111,12 +111,16 @@ struct ItemDir {
 
 // Owner side of the fused sharded exchange (sharded_fused.cu): the bucketed search's
 // gather stores each received query's result straight into the REQUESTER's result
-// window (mapped peer memory) at the query's original index.
+// window (mapped peer memory).  Receive slot j of source s (s = org[j] >> 40) goes to
+// slot j - start[s] + dst[s] there: the owner's run of s's queries comes back as ONE
+// contiguous run (coalesced peer stores); the requester maps it to query order.
 constexpr int kRemoteOrgShift = 40;  // org = (source rank << 40) | index at the source
 struct RemoteOut {
   const uint64_t* org = nullptr;  // per received query (receive-window order)
   uint64_t* pf[64] = {};          // per source rank: its result window
   uint8_t* v[64] = {};
+  uint64_t start[64] = {};        // per source: first slot of its run in the owner's window
+  uint64_t dst[64] = {};          // per source: where this owner's results start in its window
 };
 
 // Query-bucketing state (bucketed.cu): B splitter keys and a prefix directory,

@@ -18,10 +18,11 @@
 //                                                                 -> barrier
 //   4. the owner searches its receive window (pos_base = its first global rank); the
 //      bucketed search's final gather stores each result straight into the
-//      REQUESTER's result window at the query's original index (bucketed.cu,
-//      RemoteOut); small batches search into scratch and f_return stores them
-//                                                                 -> barrier
-//   5. the requester copies its result window into the caller's out arrays.
+//      REQUESTER's result window, the owner's run of that requester's queries as one
+//      contiguous run (coalesced peer stores; bucketed.cu, RemoteOut); small batches
+//      search into scratch and f_return stores them the same way  -> barrier
+//   5. the requester moves its result window (one run per owner) into query order
+//      through rpos[i], the result slot f_put recorded for query i (f_collect).
 // The matrix is double-buffered by batch parity, so step 1 of batch b+1 (stores into
 // the peers' other matrix) cannot disturb a peer still reading batch b's.  The same
 // kernels run for G virtual shards on one GPU (peer table = local windows, barriers =
@@ -121,13 +122,18 @@ __global__ void f_publish(const PeerTable pt, int me, const unsigned long long* 
 // ORDER (warp match + a per-destination prefix over the CTA's warps), so a run of the
 // owner's window holds one source chunk's queries in index order and the results the
 // owner stores back into the requester's window land on nearly consecutive indices.
+// rpos[i] = where query i's result will land in this rank's result window: the owner
+// stores its run of our queries back as one run starting at (our earlier destinations'
+// counts), in the order of its receive slots.
 template <typename K>
 __global__ void __launch_bounds__(kThreads) f_put(const K* __restrict__ q, uint64_t m, const uint8_t* __restrict__ dest,
                                                   const PeerTable pt, int me, int parity,
-                                                  unsigned long long* __restrict__ cursor, uint64_t chunk) {
+                                                  unsigned long long* __restrict__ cursor, uint64_t chunk,
+                                                  uint32_t* __restrict__ rpos) {
   constexpr int W = kThreads / 32;
   __shared__ unsigned int h[kMaxG];
   __shared__ unsigned long long base[kMaxG];
+  __shared__ unsigned long long roff[kMaxG];  // base[d] - (start of our share of d) + (our row prefix)
   __shared__ unsigned int wc[W][kMaxG];
   const int G = pt.G;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -141,7 +147,11 @@ __global__ void __launch_bounds__(kThreads) f_put(const K* __restrict__ q, uint6
   for (int d = threadIdx.x; d < G; d += blockDim.x) {
     unsigned long long start = 0;  // earlier sources' share of destination d
     for (int s = 0; s < me; ++s) start += M[s * kMaxG + d];
-    base[d] = h[d] ? start + atomicAdd(cursor + d, (unsigned long long)h[d]) : 0ull;
+    unsigned long long row = 0;    // our queries to earlier destinations
+    for (int x = 0; x < d; ++x) row += M[me * kMaxG + x];
+    const unsigned long long off = h[d] ? atomicAdd(cursor + d, (unsigned long long)h[d]) : 0ull;
+    base[d] = start + off;
+    roff[d] = row + off;
     h[d] = 0;  // from here on: queries of this chunk already placed, per destination
   }
   for (uint64_t r0 = lo; r0 < hi; r0 += blockDim.x) {
@@ -166,24 +176,37 @@ __global__ void __launch_bounds__(kThreads) f_put(const K* __restrict__ q, uint6
     }
     __syncthreads();
     if (v) {
-      const uint64_t slot = base[d] + wc[w][d] + __popc(before);
+      const uint64_t k = wc[w][d] + __popc(before);
+      const uint64_t slot = base[d] + k;
       reinterpret_cast<K*>(pt.w[d].recv_q)[slot] = q[i];
       pt.w[d].recv_org[slot] = (uint64_t(me) << kOrgShift) | i;
+      rpos[i] = uint32_t(roff[d] + k);
     }
   }
 }
 
-// Results straight into the requester's result window at the original index.
+// Results straight into the requester's result window, each source's run as one
+// contiguous run (RemoteOut: slot i - start[s] + dst[s] of source s).
 template <typename K>
 __global__ void f_return(const PeerTable pt, int me, uint64_t nrecv, const uint64_t* __restrict__ pf,
-                         const K* __restrict__ v) {
+                         const K* __restrict__ v, const RemoteOut ro) {
   const Win& mine = pt.w[me];
   for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < nrecv; i += uint64_t(gridDim.x) * blockDim.x) {
-    const uint64_t org = mine.recv_org[i];
-    const int src = int(org >> kOrgShift);
-    const uint64_t idx = org & ((1ull << kOrgShift) - 1);
-    pt.w[src].res_pf[idx] = pf[i];
-    reinterpret_cast<K*>(pt.w[src].res_v)[idx] = v[i];
+    const int src = int(mine.recv_org[i] >> kOrgShift);
+    const uint64_t slot = i - ro.start[src] + ro.dst[src];
+    pt.w[src].res_pf[slot] = pf[i];
+    reinterpret_cast<K*>(pt.w[src].res_v)[slot] = v[i];
+  }
+}
+
+// Requester: results from the result window (runs per destination) into query order.
+template <typename K>
+__global__ void f_collect(const uint32_t* __restrict__ rpos, uint64_t m, const uint64_t* __restrict__ res_pf,
+                          const K* __restrict__ res_v, uint64_t* __restrict__ out_pf, K* __restrict__ out_v) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < m; i += uint64_t(gridDim.x) * blockDim.x) {
+    const uint32_t p = __ldcs(rpos + i);
+    __stcs(reinterpret_cast<unsigned long long*>(out_pf) + i, (unsigned long long)res_pf[p]);
+    out_v[i] = res_v[p];
   }
 }
 
@@ -236,6 +259,7 @@ struct FusedState {
   uint64_t cap_m = 0, cap_r = 0;
   uint8_t* peer[kMaxG] = {};     // mapped peer windows (multi-process)
   uint8_t* dest = nullptr; uint64_t dest_cap = 0;
+  uint32_t* rpos = nullptr; uint64_t rpos_cap = 0;   // per query: its slot in our result window
   uint64_t* tmp_pf = nullptr; uint64_t tmp_pf_cap = 0;
   uint8_t* tmp_v = nullptr; uint64_t tmp_v_cap = 0;
   unsigned long long* cnt = nullptr;  // 2 x kMaxG: counts, cursors
@@ -249,7 +273,7 @@ void fused_free(hbt_tree* t) {
   if (!f) return;
   for (int g = 0; g < kMaxG; ++g)
     if (f->peer[g] && f->peer[g] != f->win) cudaIpcCloseMemHandle(f->peer[g]);
-  cudaFree(f->win); cudaFree(f->dest); cudaFree(f->tmp_pf); cudaFree(f->tmp_v); cudaFree(f->cnt);
+  cudaFree(f->win); cudaFree(f->dest); cudaFree(f->rpos); cudaFree(f->tmp_pf); cudaFree(f->tmp_v); cudaFree(f->cnt);
   if (f->h_mat) cudaFreeHost(f->h_mat);
   delete f;
   t->fused = nullptr;
@@ -276,6 +300,7 @@ int alloc_window(FusedState* f, uint64_t cap_m, uint64_t cap_r, uint32_t S) {
 int prep_local(FusedState* f, uint64_t m) {
   int rc;
   if ((rc = ensure(&f->dest, &f->dest_cap, m ? m : 1))) return rc;
+  if ((rc = ensure(&f->rpos, &f->rpos_cap, m ? m : 1))) return rc;
   if (!f->cnt) HBT_CUDA_TRY(cudaMalloc(&f->cnt, 2 * kMaxG * sizeof(unsigned long long)));
   if (!f->h_mat) HBT_CUDA_TRY(cudaMallocHost(&f->h_mat, kMat * sizeof(unsigned long long)));
   return HBT_OK;
@@ -296,25 +321,37 @@ int put_queries(FusedState* f, const K* q, uint64_t m, const PeerTable& pt, int 
   if (!m) return HBT_OK;
   const uint64_t chunk = 4096;
   f_put<K><<<unsigned((m + chunk - 1) / chunk), kThreads, 0, st>>>(q, m, f->dest, pt, me, parity, f->cnt + kMaxG,
-                                                                   chunk);
+                                                                   chunk, f->rpos);
   HBT_CUDA_TRY(cudaGetLastError());
   return HBT_OK;
 }
 
+// The owner's search of its receive window, results stored straight back into the
+// requesters' result windows.  mat = the G x G count matrix [src][dst] of this batch:
+// source s's run in our window starts at sum_{s' < s} mat[s'][me], and its results go
+// to s's window from sum_{d < me} mat[s][d] on (where s's f_put pointed its rpos).
 template <typename K>
-int search_and_return(hbt_tree* t, FusedState* f, const PeerTable& pt, int me, uint64_t nrecv, cudaStream_t st) {
+int search_and_return(hbt_tree* t, FusedState* f, const PeerTable& pt, int me, uint64_t nrecv,
+                      const std::vector<unsigned long long>& mat, cudaStream_t st) {
   int rc;
   if (!nrecv) return HBT_OK;
   const Win& w = pt.w[me];
+  const int G = pt.G;
+  RemoteOut ro;
+  ro.org = w.recv_org;
+  uint64_t start = 0;
+  for (int g = 0; g < G; ++g) {
+    ro.pf[g] = pt.w[g].res_pf;
+    ro.v[g] = pt.w[g].res_v;
+    ro.start[g] = start;
+    start += mat[g * G + me];
+    uint64_t dst = 0;
+    for (int d = 0; d < me; ++d) dst += mat[g * G + d];
+    ro.dst[g] = dst;
+  }
   if (bucketed_enabled(t, nrecv)) {
     // fused return: the bucketed search's gather stores each result straight into the
     // requester's result window (no staging, no f_return pass)
-    RemoteOut ro;
-    ro.org = w.recv_org;
-    for (int g = 0; g < pt.G; ++g) {
-      ro.pf[g] = pt.w[g].res_pf;
-      ro.v[g] = pt.w[g].res_v;
-    }
     rc = bucketed_search(t, w.recv_q, nrecv, nullptr, nullptr, t->shard.base[me], st, &ro);
     if (rc != HBT_EUNSUPPORTED) return rc;  // EUNSUPPORTED: no item directory, stage + f_return
   }
@@ -322,7 +359,7 @@ int search_and_return(hbt_tree* t, FusedState* f, const PeerTable& pt, int me, u
   if ((rc = ensure(&f->tmp_v, &f->tmp_v_cap, nrecv * sizeof(K)))) return rc;
   rc = shard_local_search(t, w.recv_q, nrecv, f->tmp_pf, f->tmp_v, t->shard.base[me], st);
   if (rc) return rc;
-  f_return<K><<<grid_for(nrecv), kThreads, 0, st>>>(pt, me, nrecv, f->tmp_pf, (const K*)f->tmp_v);
+  f_return<K><<<grid_for(nrecv), kThreads, 0, st>>>(pt, me, nrecv, f->tmp_pf, (const K*)f->tmp_v, ro);
   HBT_CUDA_TRY(cudaGetLastError());
   return HBT_OK;
 }
@@ -370,16 +407,20 @@ int local_t(hbt_tree* const* shards, int G, const void* const* queries, const ui
     int rc = put_queries<K>(fs[s], (const K*)queries[s], m[s], pt, s, 0, st);
     if (rc) return rc;
   }
+  std::vector<unsigned long long> mat(G * G);
+  for (int s = 0; s < G; ++s)
+    for (int d = 0; d < G; ++d) mat[s * G + d] = cnt[s][d];
   for (int d = 0; d < G; ++d) {
     uint64_t r = 0;
     for (int s = 0; s < G; ++s) r += cnt[s][d];
-    int rc = search_and_return<K>(shards[d], fs[d], pt, d, r, st);
+    int rc = search_and_return<K>(shards[d], fs[d], pt, d, r, mat, st);
     if (rc) return rc;
   }
   for (int s = 0; s < G; ++s) {
     if (!m[s]) continue;
-    HBT_CUDA_TRY(cudaMemcpyAsync(outs[s].pos_found, pt.w[s].res_pf, m[s] * 8, cudaMemcpyDeviceToDevice, st));
-    HBT_CUDA_TRY(cudaMemcpyAsync(outs[s].values, pt.w[s].res_v, m[s] * S, cudaMemcpyDeviceToDevice, st));
+    f_collect<K><<<grid_for(m[s]), kThreads, 0, st>>>(fs[s]->rpos, m[s], pt.w[s].res_pf, (const K*)pt.w[s].res_v,
+                                                      outs[s].pos_found, (K*)outs[s].values);
+    HBT_CUDA_TRY(cudaGetLastError());
   }
   return HBT_OK;
 }
@@ -490,14 +531,15 @@ int nccl_fused_t(hbt_tree* t, const void* queries, uint64_t m, hbt_out out, cuda
   for (int s = 0; s < G; ++s) nrecv += mat[s * G + me];
   {
     NvtxRange r("owner_search_and_return");
-    rc = search_and_return<K>(t, f, pt, me, nrecv, st);
+    rc = search_and_return<K>(t, f, pt, me, nrecv, mat, st);
   }
   if (rc) return rc;
   f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);
   HBT_CUDA_TRY(cudaGetLastError());
-  if (m) {
-    HBT_CUDA_TRY(cudaMemcpyAsync(out.pos_found, pt.w[me].res_pf, m * 8, cudaMemcpyDeviceToDevice, st));
-    HBT_CUDA_TRY(cudaMemcpyAsync(out.values, pt.w[me].res_v, m * S, cudaMemcpyDeviceToDevice, st));
+  if (m) {  // our results, one run per owner in our window, back into query order
+    f_collect<K><<<grid_for(m), kThreads, 0, st>>>(f->rpos, m, pt.w[me].res_pf, (const K*)pt.w[me].res_v,
+                                                   out.pos_found, (K*)out.values);
+    HBT_CUDA_TRY(cudaGetLastError());
   }
   ++f->batch;
   return HBT_OK;
