@@ -462,6 +462,7 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "bucket_items" && (value == 0 || value == 1)) { c.bucket_items = uint32_t(value); invalidate_buckets(t); }
   else if (n == "bucket_cap" && value >= 0 && value < (1 << 20)) { c.bucket_cap = uint32_t(value); invalidate_buckets(t); }
   else if (n == "item_rounds" && value >= 0 && value <= 64) c.item_rounds = uint32_t(value);
+  else if (n == "scatter_tma" && (value == 0 || value == 1)) c.scatter_tma = uint32_t(value);
   else if (n == "phase_timing" && (value == 0 || value == 1)) c.phase_timing = uint32_t(value);
   else if (n == "leaf_stream" && value >= 0 && value <= 2) c.leaf_stream = uint32_t(value);
   else if (n == "stream_slice" && value >= 0) { c.stream_slice = uint64_t(value); invalidate_buckets(t); }

@@ -58,6 +58,10 @@ constexpr bool kStreamPrefetch = true;
 template <typename K>
 __device__ __forceinline__ K kmax() { return K(~K(0)); }
 
+// Row stride of the chunk-major tables tab / gb: B rounded up to 4 entries, so every
+// chunk's row starts 16 B aligned (bulk copies of a row into shared memory).
+__host__ __device__ __forceinline__ uint32_t row_stride(uint32_t B) { return (B + 3u) & ~3u; }
+
 template <typename K>
 __device__ __forceinline__ K load_key(const uint8_t* p) { return *reinterpret_cast<const K*>(p); }
 
@@ -185,7 +189,7 @@ __device__ __forceinline__ void block_exclusive_scan(const uint32_t* s_in, uint3
 }
 
 // Pass 1: bucket of every query (bq, u16), the per-chunk histograms (chunk-major:
-// tab[c * B + b] = #queries of chunk c in bucket b) and the per-segment column sums
+// tab[c * Bp + b] = #queries of chunk c in bucket b, Bp = row_stride(B)) and the per-segment column sums
 // seg[j * B + b] (segment j = chunks [j * kps, (j + 1) * kps), in chunk order).
 template <typename K>
 __global__ void __launch_bounds__(kThreads) bk_count(const K* __restrict__ q, uint64_t m, const K* __restrict__ sp,
@@ -227,7 +231,7 @@ __global__ void __launch_bounds__(kThreads) bk_count(const K* __restrict__ q, ui
       }
       __syncthreads();
       for (uint32_t b = threadIdx.x; b < B; b += kThreads) {
-        tab[c * B + b] = s_h[b];
+        tab[c * row_stride(B) + b] = s_h[b];
         s_sh[b] += s_h[b];
       }
       __syncthreads();
@@ -266,7 +270,7 @@ __global__ void __launch_bounds__(kScanThreads) bk_seg_scan(const uint32_t* __re
   if (b == 0) bstart[B] = m;
 }
 
-// Run start of every (chunk, bucket), chunk-major: gb[c * B + b] = segoff[j][b] + the
+// Run start of every (chunk, bucket), chunk-major: gb[c * Bp + b] = segoff[j][b] + the
 // counts of segment j's earlier chunks (one CTA per segment walks its chunks in order;
 // rows are coalesced).  The scatter and the gather take chunks interleaved over the
 // CTAs (c = blockIdx, blockIdx + grid, ...): the runs they write / read at the same
@@ -283,8 +287,8 @@ __global__ void __launch_bounds__(kScanThreads) bk_run_starts(const uint32_t* __
   uint32_t run = segoff[j * B + b];
 #pragma unroll 4
   for (uint64_t c = c0; c < c1; ++c) {
-    const uint32_t x = tab[c * B + b];
-    gb[c * B + b] = run;
+    const uint32_t x = tab[c * row_stride(B) + b];
+    gb[c * row_stride(B) + b] = run;
     run += x;
   }
 }
@@ -297,8 +301,8 @@ __device__ __forceinline__ void chunk_layout(const uint32_t* __restrict__ tab, c
                                              uint32_t B, uint64_t c, uint32_t* s_cnt, uint32_t* s_lb, uint32_t* s_gb,
                                              uint32_t* s_tmp) {
   for (uint32_t b = threadIdx.x; b < B; b += TH) {  // chunk-major rows: coalesced
-    s_cnt[b] = tab[c * B + b];
-    s_gb[b] = gb[c * B + b];
+    s_cnt[b] = tab[c * row_stride(B) + b];
+    s_gb[b] = gb[c * row_stride(B) + b];
   }
   __syncthreads();
   block_exclusive_scan<TH>(s_cnt, s_lb, B, s_tmp);
@@ -344,8 +348,8 @@ __global__ void __launch_bounds__(kThreads, 2) bk_scatter(const K* __restrict__ 
       const uint32_t b = uint32_t(e) * kThreads + threadIdx.x;
       if (b < B) {
         s_rank[b] = 0;
-        s_cnt[b] = tab[c * B + b];
-        s_gb[b] = gb[c * B + b];
+        s_cnt[b] = tab[c * row_stride(B) + b];
+        s_gb[b] = gb[c * row_stride(B) + b];
       }
     }
     __syncthreads();
@@ -364,6 +368,151 @@ __global__ void __launch_bounds__(kThreads, 2) bk_scatter(const K* __restrict__ 
 #pragma unroll
     for (int x = 0; x < kQPT; ++x) {
       const uint32_t t = uint32_t(x) * kThreads + threadIdx.x;
+      if (t < nc) {
+        const uint32_t b = s_b[t];
+        qs[uint64_t(s_gb[b]) + (t - s_lb[b])] = s_q[t];
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// ---- Pass 2 with bulk-copy staging (default for full chunks).  One elected thread
+// streams the NEXT chunk's queries, bucket ids and layout rows (88 KB for u64) into a
+// shared staging buffer with cp.async.bulk (TMA 1D bulk copies, completion on an
+// mbarrier) while the CTA sorts and writes the current chunk, so no warp waits on
+// DRAM for its inputs and no registers hold them in flight.  1024 threads, 8 queries
+// each; the sort and the run writes are those of bk_scatter.
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return uint32_t(__cvta_generic_to_shared(p)); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      " .reg .pred p;\n"
+      "WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra WAIT_%=;\n"
+      "}\n" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+
+constexpr int kTThreads = 1024;
+constexpr int kTQPT = int(kChunk) / kTThreads;  // 8 queries per thread
+
+template <typename K>
+size_t smem_scatter_tma(uint32_t B) {
+  const size_t bp = row_stride(B);
+  return kChunk * (sizeof(K) + 2) * 2 + bp * 4 * 2 + kMaxBuckets * 4 * 3 + 32 * 4 + 64;
+}
+
+template <typename K>
+__global__ void __launch_bounds__(kTThreads, 1) bk_scatter_tma(const K* __restrict__ q, uint64_t m,
+                                                               const uint16_t* __restrict__ bq,
+                                                               const uint32_t* __restrict__ tab,
+                                                               const uint32_t* __restrict__ gb, uint32_t B,
+                                                               uint64_t chunks, K* __restrict__ qs,
+                                                               uint16_t* __restrict__ linv) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  const uint32_t BP = row_stride(B);
+  // staging: [q | bq | tab row | gb row]; sorted: [s_q | s_b]; layout arrays
+  K* st_q = reinterpret_cast<K*>(smem);
+  uint16_t* st_b = reinterpret_cast<uint16_t*>(st_q + kChunk);
+  uint32_t* st_cnt = reinterpret_cast<uint32_t*>(st_b + kChunk);
+  uint32_t* st_gb = st_cnt + BP;
+  K* s_q = reinterpret_cast<K*>(st_gb + BP);
+  uint16_t* s_b = reinterpret_cast<uint16_t*>(s_q + kChunk);
+  uint32_t* s_lb = reinterpret_cast<uint32_t*>(s_b + kChunk);
+  uint32_t* s_rank = s_lb + kMaxBuckets;
+  uint32_t* s_gb = s_rank + kMaxBuckets;
+  uint32_t* s_tmp = s_gb + kMaxBuckets;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(s_tmp + 32);
+  const uint32_t bytes = uint32_t(kChunk * (sizeof(K) + 2) + 2 * BP * 4);
+  auto issue = [&](uint64_t c) {  // one thread: the whole chunk c into the staging buffer
+    mbar_expect_tx(bar, bytes);
+    bulk_g2s(st_q, q + c * kChunk, uint32_t(kChunk * sizeof(K)), bar);
+    bulk_g2s(st_b, bq + c * kChunk, uint32_t(kChunk * 2), bar);
+    bulk_g2s(st_cnt, tab + c * BP, BP * 4, bar);
+    bulk_g2s(st_gb, gb + c * BP, BP * 4, bar);
+  };
+  const uint64_t full = m / kChunk;  // chunks served by bulk copies; the tail chunk reads directly
+  if (threadIdx.x == 0) {
+    mbar_init(bar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if (threadIdx.x == 0 && blockIdx.x < full) issue(blockIdx.x);
+  uint32_t parity = 0;
+  for (uint64_t c = blockIdx.x; c < chunks; c += gridDim.x) {
+    const uint64_t lo = c * kChunk;
+    const uint32_t nc = uint32_t(m - lo < kChunk ? m - lo : kChunk);
+    K qq[kTQPT];
+    uint32_t bb[kTQPT];
+    if (c < full) {
+      mbar_wait(bar, parity);
+      parity ^= 1u;
+#pragma unroll
+      for (int x = 0; x < kTQPT; ++x) {
+        const uint32_t t = uint32_t(x) * kTThreads + threadIdx.x;
+        qq[x] = st_q[t];
+        bb[x] = st_b[t];
+      }
+      for (uint32_t b = threadIdx.x; b < B; b += kTThreads) {
+        s_rank[b] = 0;
+        s_gb[b] = st_gb[b];
+        s_lb[b] = st_cnt[b];  // counts for the scan below (in place)
+      }
+    } else {
+#pragma unroll
+      for (int x = 0; x < kTQPT; ++x) {
+        const uint32_t t = uint32_t(x) * kTThreads + threadIdx.x;
+        qq[x] = K(0);
+        bb[x] = 0;
+        if (t < nc) {
+          qq[x] = __ldcs(q + lo + t);
+          bb[x] = __ldcs(reinterpret_cast<const unsigned short*>(bq) + lo + t);
+        }
+      }
+      for (uint32_t b = threadIdx.x; b < B; b += kTThreads) {
+        s_rank[b] = 0;
+        s_gb[b] = gb[c * BP + b];
+        s_lb[b] = tab[c * BP + b];
+      }
+    }
+    __syncthreads();  // the staging buffer is consumed: stream the next chunk into it
+    if (threadIdx.x == 0) {
+      const uint64_t cn = c + gridDim.x;
+      if (cn < full) {
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        issue(cn);
+      }
+    }
+    block_exclusive_scan<kTThreads>(s_lb, s_lb, B, s_tmp);
+#pragma unroll
+    for (int x = 0; x < kTQPT; ++x) {
+      const uint32_t t = uint32_t(x) * kTThreads + threadIdx.x;
+      if (t < nc) {
+        const uint32_t pos = s_lb[bb[x]] + atomicAdd(&s_rank[bb[x]], 1u);
+        s_q[pos] = qq[x];
+        s_b[pos] = uint16_t(bb[x]);
+        __stcs(reinterpret_cast<unsigned short*>(linv) + lo + t, (unsigned short)pos);
+      }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int x = 0; x < kTQPT; ++x) {
+      const uint32_t t = uint32_t(x) * kTThreads + threadIdx.x;
       if (t < nc) {
         const uint32_t b = s_b[t];
         qs[uint64_t(s_gb[b]) + (t - s_lb[b])] = s_q[t];
@@ -486,8 +635,8 @@ __global__ void __launch_bounds__(kGThreads) bk_gather_rec(const uint16_t* __res
   const uint32_t tb = threadIdx.x;
   uint32_t nx_cnt = 0, nx_gb = 0;
   if (blockIdx.x < chunks && tb < B) {
-    nx_cnt = tab[uint64_t(blockIdx.x) * B + tb];
-    nx_gb = gb[uint64_t(blockIdx.x) * B + tb];
+    nx_cnt = tab[uint64_t(blockIdx.x) * row_stride(B) + tb];
+    nx_gb = gb[uint64_t(blockIdx.x) * row_stride(B) + tb];
   }
   for (uint64_t c = blockIdx.x; c < chunks; c += gridDim.x) {
     const uint64_t lo = c * kChunk;
@@ -516,8 +665,8 @@ __global__ void __launch_bounds__(kGThreads) bk_gather_rec(const uint16_t* __res
     {  // next chunk's layout row, in flight during the stores below
       const uint64_t cn = c + gridDim.x;
       if (cn < chunks && tb < B) {
-        nx_cnt = tab[cn * B + tb];
-        nx_gb = gb[cn * B + tb];
+        nx_cnt = tab[cn * row_stride(B) + tb];
+        nx_gb = gb[cn * row_stride(B) + tb];
       }
     }
 #pragma unroll
@@ -571,6 +720,10 @@ void set_bucket_attrs() {
   cudaFuncSetAttribute(bk_count<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
   cudaFuncSetAttribute(bk_scatter<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
   cudaFuncSetAttribute(bk_scatter<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
+  cudaFuncSetAttribute(bk_scatter_tma<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       int(smem_scatter_tma<uint32_t>(kMaxBuckets)));
+  cudaFuncSetAttribute(bk_scatter_tma<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       int(smem_scatter_tma<uint64_t>(kMaxBuckets)));
   cudaFuncSetAttribute(bk_gather<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
   cudaFuncSetAttribute(bk_gather<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, lim);
   cudaFuncSetAttribute(bk_gather_rec<uint32_t, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
@@ -715,8 +868,8 @@ Part part_layout(uint64_t m, uint32_t B, uint32_t sms) {
   p.o_bq = p.o_v + al(m * 8);
   p.o_li = p.o_bq + al(m * 2);
   p.o_tab = p.o_li + al(m * 2);
-  p.o_gb = p.o_tab + al(p.chunks * B * 4);
-  p.o_seg = p.o_gb + al(p.chunks * B * 4);
+  p.o_gb = p.o_tab + al(p.chunks * row_stride(B) * 4);
+  p.o_seg = p.o_gb + al(p.chunks * row_stride(B) * 4);
   p.o_so = p.o_seg + al(p.nseg * B * 4);
   p.o_bs = p.o_so + al(p.nseg * B * 4);
   p.total = p.o_bs + al((uint64_t(B) + 1) * 8);
@@ -746,10 +899,17 @@ int partition(const hbt_tree* t, const BucketState& bs, const void* q, uint64_t 
   bk_run_starts<<<unsigned(p.nseg), kScanThreads, 0, s>>>(p.at<uint32_t>(p.o_tab), p.at<uint32_t>(p.o_so), p.B,
                                                           p.chunks, p.kps, p.at<uint32_t>(p.o_gb));
   mark(2);
-  const unsigned sgrid = unsigned(std::min<uint64_t>(p.chunks, uint64_t(t->num_sms) * 2));
-  bk_scatter<K><<<sgrid, kThreads, smem_scatter<K>(), s>>>((const K*)q, m, p.at<uint16_t>(p.o_bq),
-                                                           p.at<uint32_t>(p.o_tab), p.at<uint32_t>(p.o_gb), p.B,
-                                                           p.chunks, p.at<K>(0), p.at<uint16_t>(p.o_li));
+  if (t->cfg.scatter_tma && m >= kChunk && (reinterpret_cast<uintptr_t>(q) & 15u) == 0) {
+    const unsigned sgrid = unsigned(std::min<uint64_t>(p.chunks, uint64_t(t->num_sms)));
+    bk_scatter_tma<K><<<sgrid, kTThreads, smem_scatter_tma<K>(p.B), s>>>(
+        (const K*)q, m, p.at<uint16_t>(p.o_bq), p.at<uint32_t>(p.o_tab), p.at<uint32_t>(p.o_gb), p.B, p.chunks,
+        p.at<K>(0), p.at<uint16_t>(p.o_li));
+  } else {
+    const unsigned sgrid = unsigned(std::min<uint64_t>(p.chunks, uint64_t(t->num_sms) * 2));
+    bk_scatter<K><<<sgrid, kThreads, smem_scatter<K>(), s>>>((const K*)q, m, p.at<uint16_t>(p.o_bq),
+                                                             p.at<uint32_t>(p.o_tab), p.at<uint32_t>(p.o_gb), p.B,
+                                                             p.chunks, p.at<K>(0), p.at<uint16_t>(p.o_li));
+  }
   if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) {
     set_error("bucketing kernels failed to launch: %s", cudaGetErrorString(e));
     return HBT_ECUDA;

@@ -73,6 +73,7 @@ struct SearchConfig {
   uint32_t bucket_items = 1;     // bucketed search: bucket-local shared-memory directory (ItemDir)
   uint32_t bucket_cap = 0;       // item directory: shared-memory entries (0 = derived; tests force the fallback)
   uint32_t item_rounds = 0;      // item searches: most warp rounds per work item (0 = 16)
+  uint32_t scatter_tma = 1;      // bucketed scatter: inputs streamed into shared memory by bulk copies (1)
   uint32_t phase_timing = 0;     // bucketed search: CUDA events around each phase (hbt_last_phases)
   uint32_t leaf_stream = 2;      // host L-segment: 0 = zero-copy leaf reads, 1 = stream bucket slices
                                  // into HBM (bucketed, double-buffered copies), 2 = auto (by batch size)
