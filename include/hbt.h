@@ -204,8 +204,8 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *   "g1_direct"   hbt_search_sharded on a ONE-shard tree with exchange 0: 1 (default) = search
  *                 in place (nothing to route or exchange), 0 = run the full fused pipeline
  *   "bucket"      query bucketing before the tree walk (north_star "queries bucketed per batch"):
- *                 0 = off, 1 = on, 2 = auto (default: regular trees larger than 8x the L2 and
- *                 implicit trees larger than 64x, batches of >= 4 Mi queries).  The batch is
+ *                 0 = off, 1 = on, 2 = auto (default: trees larger than 8x the L2, batches of
+ *                 >= 4 Mi queries: c3, c4, c5).  The batch is
  *                 partitioned into B key-range buckets, searched bucket after bucket, and the
  *                 results are gathered back to query order; outputs are identical.
  *   "bucket_slice" tree bytes per bucket (0 = default 1 MB; B <= 1024)

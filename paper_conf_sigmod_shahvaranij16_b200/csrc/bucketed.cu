@@ -1110,13 +1110,13 @@ bool bucketed_enabled(const hbt_tree* t, uint64_t m) {
   if (mode == 2 && m < (1ull << 22)) return false;  // auto: small batches never (no host calls)
   if (pick_buckets(t) < 2) return false;
   if (mode == 1) return true;
-  // auto: batches large enough to share lines, regular trees beyond 8x the L2
-  // (measured: c3 10.9 -> 21.0 G q/s), implicit trees beyond 64x (the 2.1 GB c5
-  // tree gains nothing under uniform values, 18.3 -> 18.8, and loses under Zipf,
-  // 23.1 -> 19.9, whose hot set already lives in L2)
+  // auto: batches large enough to share lines, trees beyond 8x the L2 (measured: c3
+  // regular 10.9 -> 24 G q/s; c5 implicit Zipf 2^27 keys 2.84 -> 2.71 ms once the scatter
+  // used bulk-copy staging, profiles/r02_c5_c2_bucket_ab.jsonl; c2's 150 MB tree stays
+  // unbucketed: 0.41 vs 0.66 ms)
   static int l2 = 0;  // one device model per process
   if (!l2) cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, t->device);
-  return t->form == HBT_REGULAR ? tree_bytes(t) > 8ull * uint64_t(l2) : tree_bytes(t) > 64ull * uint64_t(l2);
+  return tree_bytes(t) > 8ull * uint64_t(l2);
 }
 
 int bucketed_search(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t pos_base,

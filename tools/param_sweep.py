@@ -32,6 +32,10 @@ def main():
     if a.config == "c4":
         keys, vals = g.stratified_keys(n, sk), g.mix_stream(n, w, sv)
         q = g.stratified_queries(m, n, sq, sk)
+    elif c["queries"] == "zipf":
+        keys, vals = g.mix_stream(n, w, sk), g.mix_stream(n, w, sv)
+        hk = gen.keys(n, w, sk)
+        q = torch.from_numpy(hk[gen.zipf_ranks(m, n, c["theta"], sq) - 1].view("int64")).cuda()
     else:
         keys, vals = g.mix_stream(n, w, sk), g.mix_stream(n, w, sv)
         q = g.uniform_queries(m, n, w, sq, sk)
