@@ -3,6 +3,10 @@
 # steady-state DRAM traffic per config, and ncu --set full of the c4 item search.
 cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out
 TAG=${1:-r02}
+timeout 2400 python -m pytest tests -x -q -m gpu > gpurun_out/${TAG}_pytest_gpu.log 2>&1
+echo "rc=$?" >> gpurun_out/${TAG}_pytest_gpu.log
+python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${TAG}_smoke.log 2>&1
+bash tools/sanitize.sh
 for c in c1 c2 c3 c5; do
   timeout 900 python bench.py --config $c --steps 50 --warmup 5 > gpurun_out/${TAG}_bench_$c.log 2>&1
 done
