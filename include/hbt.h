@@ -201,6 +201,9 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *   "exchange"    sharded search: 0 = fused peer-memory exchange (CUDA IPC windows, device
  *                 barriers, count rows and queries by peer stores; default), 1 = NCCL send/recv
  *                 (multi-process) / device copies (hbt_search_sharded_local)
+ *   "exchange_chunks" fused exchange: the batch is exchanged in 1..4 chunks; the owner searches
+ *                 chunk c on a second stream while chunk c+1 is put (overlap of NVLink stores and
+ *                 search).  Default 1; every rank of a communicator must set the same value.
  *   "g1_direct"   hbt_search_sharded on a ONE-shard tree with exchange 0: 1 (default) = search
  *                 in place (nothing to route or exchange), 0 = run the full fused pipeline
  *   "bucket"      query bucketing before the tree walk (north_star "queries bucketed per batch"):

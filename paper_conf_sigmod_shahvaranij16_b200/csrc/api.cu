@@ -456,6 +456,7 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "l2_levels_bytes" && value >= 0) c.l2_levels_bytes = uint64_t(value);
   else if (n == "full_levels" && value >= 0 && value <= 0xFFFFFFFFll) c.full_levels = uint32_t(value);
   else if (n == "exchange" && (value == 0 || value == 1)) c.exchange = uint32_t(value);
+  else if (n == "exchange_chunks" && value >= 1 && value <= 4) c.exchange_chunks = uint32_t(value);
   else if (n == "g1_direct" && (value == 0 || value == 1)) c.g1_direct = uint32_t(value);
   else if (n == "bucket" && value >= 0 && value <= 2) c.bucket = uint32_t(value);
   else if (n == "bucket_slice" && value >= 0) { c.bucket_slice = uint64_t(value); invalidate_buckets(t); }

@@ -67,6 +67,10 @@ struct SearchConfig {
   uint64_t l2_levels_bytes = 0;  // L2-resident budget for index+sector levels (0 = default 32 MB)
   uint32_t full_levels = 0;      // implicit: bit d = read level d's nodes whole (0 = by the L2 budget)
   uint32_t exchange = 0;         // sharded search: 0 = fused peer-memory exchange, 1 = NCCL send/recv
+  uint32_t exchange_chunks = 1;  // fused exchange: chunks per batch (the put of chunk c+1 overlaps the owner
+                                 // search of chunk c on a second stream); every rank of a communicator must
+                                 // use the same value.  1 by default: with the ranks sharing one GPU (the only
+                                 // multi-rank setup measured) 2 / 3 chunks ran 11.6 -> 10.3 / 9.5 G q/s
   uint32_t g1_direct = 1;        // sharded search with ONE shard: search directly (no route / exchange)
   uint32_t bucket = 2;           // query bucketing (bucketed.cu): 0 = off, 1 = on, 2 = auto
   uint64_t bucket_slice = 0;     // tree bytes per bucket (0 = default 1 MB)

@@ -39,11 +39,13 @@ namespace {
 constexpr int kMaxG = 64;
 constexpr int kThreads = 256;
 constexpr uint64_t kOrgShift = kRemoteOrgShift;  // recv_org = (source rank << 40) | origin index
-constexpr uint64_t kMat = uint64_t(kMaxG) * kMaxG;  // one parity of the count matrix
+constexpr uint64_t kMat = uint64_t(kMaxG) * kMaxG;  // one count matrix [src][dst]
+constexpr int kMaxChunks = 4;                       // exchange chunks per batch (overlap, see below)
+constexpr uint64_t kMatAll = 2 * kMaxChunks * kMat; // [parity][chunk] matrices per window
 
 struct Win {
   uint32_t* flags;
-  unsigned long long* matrix;  // [parity][src][dst]
+  unsigned long long* matrix;  // [parity][chunk][src][dst]
   uint64_t* res_pf;
   uint8_t* res_v;
   uint8_t* recv_q;
@@ -69,7 +71,7 @@ inline unsigned grid_for(uint64_t n) {
 
 uint64_t win_bytes(uint64_t cap_m, uint64_t cap_r, uint32_t S) {
   auto al = [](uint64_t x) { return (x + 255) & ~uint64_t(255); };
-  return al(kMaxG * 4) + al(2 * kMat * 8) + al(cap_m * 8) + al(cap_m * S) + al(cap_r * S) + al(cap_r * 8);
+  return al(kMaxG * 4) + al(kMatAll * 8) + al(cap_m * 8) + al(cap_m * S) + al(cap_r * S) + al(cap_r * 8);
 }
 
 Win carve(uint8_t* base, uint64_t cap_m, uint64_t cap_r, uint32_t S) {
@@ -77,7 +79,7 @@ Win carve(uint8_t* base, uint64_t cap_m, uint64_t cap_r, uint32_t S) {
   Win w;
   uint64_t o = 0;
   w.flags = (uint32_t*)(base + o); o += al(kMaxG * 4);
-  w.matrix = (unsigned long long*)(base + o); o += al(2 * kMat * 8);
+  w.matrix = (unsigned long long*)(base + o); o += al(kMatAll * 8);
   w.res_pf = (uint64_t*)(base + o); o += al(cap_m * 8);
   w.res_v = base + o; o += al(cap_m * S);
   w.recv_q = base + o; o += al(cap_r * S);
@@ -109,13 +111,24 @@ __global__ void __launch_bounds__(kThreads) f_count(const K* __restrict__ q, uin
     if (h[i]) atomicAdd(cnt + i, (unsigned long long)h[i]);
 }
 
-// Store this rank's count row into every peer's matrix[parity] (row `me`).
-__global__ void f_publish(const PeerTable pt, int me, const unsigned long long* __restrict__ cnt, int parity) {
-  for (int x = threadIdx.x; x < pt.G * pt.G; x += blockDim.x) {
-    const int d = x / pt.G, c = x % pt.G;
-    pt.w[d].matrix[parity * kMat + me * kMaxG + c] = cnt[c];
+// Store this rank's count rows (one per chunk) into every peer's matrix[parity][chunk]
+// (row `me`).  cnt: chunk c's counts at cnt[c * 2 * kMaxG].
+__global__ void f_publish(const PeerTable pt, int me, const unsigned long long* __restrict__ cnt, int parity,
+                          int nchunks) {
+  const int G = pt.G;
+  for (int x = threadIdx.x; x < nchunks * G * G; x += blockDim.x) {
+    const int ch = x / (G * G), d = (x / G) % G, c = x % G;
+    pt.w[d].matrix[(uint64_t(parity) * kMaxChunks + ch) * kMat + me * kMaxG + c] = cnt[ch * 2 * kMaxG + c];
   }
 }
+
+// Where one chunk's put lands: rbase[d] = the chunk's region in owner d's receive window
+// (earlier chunks' receives), qbase = the chunk's first query (result slots follow the
+// batch's chunks in order).
+struct PutOff {
+  uint64_t rbase[kMaxG];
+  uint64_t qbase;
+};
 
 // Route + put: queries go straight into their owner's receive window.  Each CTA
 // reserves one block per destination for its chunk of the batch and fills it in SOURCE
@@ -127,7 +140,8 @@ __global__ void f_publish(const PeerTable pt, int me, const unsigned long long* 
 // counts), in the order of its receive slots.
 template <typename K>
 __global__ void __launch_bounds__(kThreads) f_put(const K* __restrict__ q, uint64_t m, const uint8_t* __restrict__ dest,
-                                                  const PeerTable pt, int me, int parity,
+                                                  const PeerTable pt, int me,
+                                                  const unsigned long long* __restrict__ M, const PutOff off,
                                                   unsigned long long* __restrict__ cursor, uint64_t chunk,
                                                   uint32_t* __restrict__ rpos) {
   constexpr int W = kThreads / 32;
@@ -143,15 +157,15 @@ __global__ void __launch_bounds__(kThreads) f_put(const K* __restrict__ q, uint6
   __syncthreads();
   for (uint64_t i = lo + threadIdx.x; i < hi; i += blockDim.x) atomicAdd(&h[dest[i]], 1u);
   __syncthreads();
-  const unsigned long long* M = pt.w[me].matrix + parity * kMat;  // full matrix (every row published)
+  // M = this chunk's full matrix in our own window (every row published)
   for (int d = threadIdx.x; d < G; d += blockDim.x) {
-    unsigned long long start = 0;  // earlier sources' share of destination d
+    unsigned long long start = off.rbase[d];  // earlier chunks, then earlier sources, at destination d
     for (int s = 0; s < me; ++s) start += M[s * kMaxG + d];
     unsigned long long row = 0;    // our queries to earlier destinations
     for (int x = 0; x < d; ++x) row += M[me * kMaxG + x];
-    const unsigned long long off = h[d] ? atomicAdd(cursor + d, (unsigned long long)h[d]) : 0ull;
-    base[d] = start + off;
-    roff[d] = row + off;
+    const unsigned long long o = h[d] ? atomicAdd(cursor + d, (unsigned long long)h[d]) : 0ull;
+    base[d] = start + o;
+    roff[d] = off.qbase + row + o;
     h[d] = 0;  // from here on: queries of this chunk already placed, per destination
   }
   for (uint64_t r0 = lo; r0 < hi; r0 += blockDim.x) {
@@ -179,7 +193,7 @@ __global__ void __launch_bounds__(kThreads) f_put(const K* __restrict__ q, uint6
       const uint64_t k = wc[w][d] + __popc(before);
       const uint64_t slot = base[d] + k;
       reinterpret_cast<K*>(pt.w[d].recv_q)[slot] = q[i];
-      pt.w[d].recv_org[slot] = (uint64_t(me) << kOrgShift) | i;
+      pt.w[d].recv_org[slot] = (uint64_t(me) << kOrgShift) | (off.qbase + i);
       rpos[i] = uint32_t(roff[d] + k);
     }
   }
@@ -188,11 +202,10 @@ __global__ void __launch_bounds__(kThreads) f_put(const K* __restrict__ q, uint6
 // Results straight into the requester's result window, each source's run as one
 // contiguous run (RemoteOut: slot i - start[s] + dst[s] of source s).
 template <typename K>
-__global__ void f_return(const PeerTable pt, int me, uint64_t nrecv, const uint64_t* __restrict__ pf,
+__global__ void f_return(const PeerTable pt, uint64_t nrecv, const uint64_t* __restrict__ pf,
                          const K* __restrict__ v, const RemoteOut ro) {
-  const Win& mine = pt.w[me];
   for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < nrecv; i += uint64_t(gridDim.x) * blockDim.x) {
-    const int src = int(mine.recv_org[i] >> kOrgShift);
+    const int src = int(ro.org[i] >> kOrgShift);
     const uint64_t slot = i - ro.start[src] + ro.dst[src];
     pt.w[src].res_pf[slot] = pf[i];
     reinterpret_cast<K*>(pt.w[src].res_v)[slot] = v[i];
@@ -262,8 +275,10 @@ struct FusedState {
   uint32_t* rpos = nullptr; uint64_t rpos_cap = 0;   // per query: its slot in our result window
   uint64_t* tmp_pf = nullptr; uint64_t tmp_pf_cap = 0;
   uint8_t* tmp_v = nullptr; uint64_t tmp_v_cap = 0;
-  unsigned long long* cnt = nullptr;  // 2 x kMaxG: counts, cursors
-  unsigned long long* h_mat = nullptr;  // pinned host copy of one count matrix
+  unsigned long long* cnt = nullptr;  // per chunk: kMaxG counts, kMaxG cursors
+  unsigned long long* h_mat = nullptr;  // pinned host copy of one parity's count matrices
+  cudaStream_t aux = nullptr;         // owner searches of the chunks (overlapping later puts)
+  cudaEvent_t ev_put[kMaxChunks] = {}, ev_done = nullptr;
   uint32_t epoch = 0;
   uint64_t batch = 0;                 // parity of the count matrix
 };
@@ -275,6 +290,10 @@ void fused_free(hbt_tree* t) {
     if (f->peer[g] && f->peer[g] != f->win) cudaIpcCloseMemHandle(f->peer[g]);
   cudaFree(f->win); cudaFree(f->dest); cudaFree(f->rpos); cudaFree(f->tmp_pf); cudaFree(f->tmp_v); cudaFree(f->cnt);
   if (f->h_mat) cudaFreeHost(f->h_mat);
+  for (auto& e : f->ev_put)
+    if (e) cudaEventDestroy(e);
+  if (f->ev_done) cudaEventDestroy(f->ev_done);
+  if (f->aux) cudaStreamDestroy(f->aux);
   delete f;
   t->fused = nullptr;
 }
@@ -290,7 +309,7 @@ int alloc_window(FusedState* f, uint64_t cap_m, uint64_t cap_r, uint32_t S) {
   cudaFree(f->win);
   f->win = nullptr;
   HBT_CUDA_TRY(cudaMalloc(&f->win, win_bytes(cap_m, cap_r, S)));
-  HBT_CUDA_TRY(cudaMemset(f->win, 0, 256 * ((kMaxG * 4 + 255) / 256) + 2 * kMat * 8));  // flags + matrices
+  HBT_CUDA_TRY(cudaMemset(f->win, 0, 256 * ((kMaxG * 4 + 255) / 256) + kMatAll * 8));  // flags + matrices
   f->cap_m = cap_m;
   f->cap_r = cap_r;
   f->epoch = 0;
@@ -301,27 +320,35 @@ int prep_local(FusedState* f, uint64_t m) {
   int rc;
   if ((rc = ensure(&f->dest, &f->dest_cap, m ? m : 1))) return rc;
   if ((rc = ensure(&f->rpos, &f->rpos_cap, m ? m : 1))) return rc;
-  if (!f->cnt) HBT_CUDA_TRY(cudaMalloc(&f->cnt, 2 * kMaxG * sizeof(unsigned long long)));
-  if (!f->h_mat) HBT_CUDA_TRY(cudaMallocHost(&f->h_mat, kMat * sizeof(unsigned long long)));
+  if (!f->cnt) HBT_CUDA_TRY(cudaMalloc(&f->cnt, kMaxChunks * 2 * kMaxG * sizeof(unsigned long long)));
+  if (!f->h_mat) HBT_CUDA_TRY(cudaMallocHost(&f->h_mat, kMaxChunks * kMat * sizeof(unsigned long long)));
   return HBT_OK;
 }
 
+// Owner of every query and per-destination counts, chunk by chunk (chunk c = queries
+// [c * mc, min((c + 1) * mc, m))).
 template <typename K>
-int route_and_count(FusedState* f, const K* q, uint64_t m, const RouteTab& rt, int G, cudaStream_t st) {
-  HBT_CUDA_TRY(cudaMemsetAsync(f->cnt, 0, 2 * kMaxG * sizeof(unsigned long long), st));
-  if (m) {
-    f_count<K><<<grid_for(m), kThreads, 0, st>>>(q, m, rt, G, f->dest, f->cnt);
+int route_and_count(FusedState* f, const K* q, uint64_t m, uint64_t mc, int nchunks, const RouteTab& rt, int G,
+                    cudaStream_t st) {
+  HBT_CUDA_TRY(cudaMemsetAsync(f->cnt, 0, kMaxChunks * 2 * kMaxG * sizeof(unsigned long long), st));
+  for (int c = 0; c < nchunks; ++c) {
+    const uint64_t lo = uint64_t(c) * mc, n = lo < m ? std::min<uint64_t>(mc, m - lo) : 0;
+    if (!n) continue;
+    f_count<K><<<grid_for(n), kThreads, 0, st>>>(q + lo, n, rt, G, f->dest + lo, f->cnt + c * 2 * kMaxG);
     HBT_CUDA_TRY(cudaGetLastError());
   }
   return HBT_OK;
 }
 
+// Chunk c of this rank's batch (queries [lo, lo + n)) into the owners' windows.
 template <typename K>
-int put_queries(FusedState* f, const K* q, uint64_t m, const PeerTable& pt, int me, int parity, cudaStream_t st) {
-  if (!m) return HBT_OK;
+int put_queries(FusedState* f, const K* q, uint64_t lo, uint64_t n, const PeerTable& pt, int me,
+                const unsigned long long* M, const PutOff& off, int c, cudaStream_t st) {
+  if (!n) return HBT_OK;
   const uint64_t chunk = 4096;
-  f_put<K><<<unsigned((m + chunk - 1) / chunk), kThreads, 0, st>>>(q, m, f->dest, pt, me, parity, f->cnt + kMaxG,
-                                                                   chunk, f->rpos);
+  f_put<K><<<unsigned((n + chunk - 1) / chunk), kThreads, 0, st>>>(q + lo, n, f->dest + lo, pt, me, M, off,
+                                                                   f->cnt + c * 2 * kMaxG + kMaxG, chunk,
+                                                                   f->rpos + lo);
   HBT_CUDA_TRY(cudaGetLastError());
   return HBT_OK;
 }
@@ -331,35 +358,39 @@ int put_queries(FusedState* f, const K* q, uint64_t m, const PeerTable& pt, int 
 // source s's run in our window starts at sum_{s' < s} mat[s'][me], and its results go
 // to s's window from sum_{d < me} mat[s][d] on (where s's f_put pointed its rpos).
 template <typename K>
-int search_and_return(hbt_tree* t, FusedState* f, const PeerTable& pt, int me, uint64_t nrecv,
-                      const std::vector<unsigned long long>& mat, cudaStream_t st) {
+int search_and_return(hbt_tree* t, FusedState* f, const PeerTable& pt, int me, uint64_t rstart,
+                      const std::vector<unsigned long long>& mat, const std::vector<uint64_t>& qbase,
+                      cudaStream_t st) {
   int rc;
+  const int G = pt.G;
+  uint64_t nrecv = 0;
+  for (int g = 0; g < G; ++g) nrecv += mat[g * G + me];
   if (!nrecv) return HBT_OK;
   const Win& w = pt.w[me];
-  const int G = pt.G;
+  const uint8_t* rq = w.recv_q + rstart * sizeof(K);
   RemoteOut ro;
-  ro.org = w.recv_org;
+  ro.org = w.recv_org + rstart;
   uint64_t start = 0;
   for (int g = 0; g < G; ++g) {
     ro.pf[g] = pt.w[g].res_pf;
     ro.v[g] = pt.w[g].res_v;
     ro.start[g] = start;
     start += mat[g * G + me];
-    uint64_t dst = 0;
+    uint64_t dst = qbase[g];
     for (int d = 0; d < me; ++d) dst += mat[g * G + d];
     ro.dst[g] = dst;
   }
   if (bucketed_enabled(t, nrecv)) {
     // fused return: the bucketed search's gather stores each result straight into the
     // requester's result window (no staging, no f_return pass)
-    rc = bucketed_search(t, w.recv_q, nrecv, nullptr, nullptr, t->shard.base[me], st, &ro);
+    rc = bucketed_search(t, rq, nrecv, nullptr, nullptr, t->shard.base[me], st, &ro);
     if (rc != HBT_EUNSUPPORTED) return rc;  // EUNSUPPORTED: no item directory, stage + f_return
   }
   if ((rc = ensure(&f->tmp_pf, &f->tmp_pf_cap, nrecv))) return rc;
   if ((rc = ensure(&f->tmp_v, &f->tmp_v_cap, nrecv * sizeof(K)))) return rc;
-  rc = shard_local_search(t, w.recv_q, nrecv, f->tmp_pf, f->tmp_v, t->shard.base[me], st);
+  rc = shard_local_search(t, rq, nrecv, f->tmp_pf, f->tmp_v, t->shard.base[me], st);
   if (rc) return rc;
-  f_return<K><<<grid_for(nrecv), kThreads, 0, st>>>(pt, me, nrecv, f->tmp_pf, (const K*)f->tmp_v, ro);
+  f_return<K><<<grid_for(nrecv), kThreads, 0, st>>>(pt, nrecv, f->tmp_pf, (const K*)f->tmp_v, ro);
   HBT_CUDA_TRY(cudaGetLastError());
   return HBT_OK;
 }
@@ -378,7 +409,7 @@ int local_t(hbt_tree* const* shards, int G, const void* const* queries, const ui
     fs[s] = state_of(shards[s]);
     int rc = prep_local(fs[s], m[s]);
     if (rc) return rc;
-    rc = route_and_count<K>(fs[s], (const K*)queries[s], m[s], rt, G, st);
+    rc = route_and_count<K>(fs[s], (const K*)queries[s], m[s], m[s] ? m[s] : 1, 1, rt, G, st);
     if (rc) return rc;
     HBT_CUDA_TRY(cudaMemcpyAsync(cnt[s].data(), fs[s]->cnt, G * 8, cudaMemcpyDeviceToHost, st));
   }
@@ -400,20 +431,20 @@ int local_t(hbt_tree* const* shards, int G, const void* const* queries, const ui
     pt.w[g] = carve(fs[g]->win, fs[g]->cap_m, fs[g]->cap_r, S);
   }
   for (int s = 0; s < G; ++s) {
-    f_publish<<<1, 256, 0, st>>>(pt, s, fs[s]->cnt, 0);
+    f_publish<<<1, 256, 0, st>>>(pt, s, fs[s]->cnt, 0, 1);
     HBT_CUDA_TRY(cudaGetLastError());
   }
+  PutOff off{};
   for (int s = 0; s < G; ++s) {
-    int rc = put_queries<K>(fs[s], (const K*)queries[s], m[s], pt, s, 0, st);
+    int rc = put_queries<K>(fs[s], (const K*)queries[s], 0, m[s], pt, s, pt.w[s].matrix, off, 0, st);
     if (rc) return rc;
   }
   std::vector<unsigned long long> mat(G * G);
   for (int s = 0; s < G; ++s)
     for (int d = 0; d < G; ++d) mat[s * G + d] = cnt[s][d];
+  const std::vector<uint64_t> qbase(G, 0);
   for (int d = 0; d < G; ++d) {
-    uint64_t r = 0;
-    for (int s = 0; s < G; ++s) r += cnt[s][d];
-    int rc = search_and_return<K>(shards[d], fs[d], pt, d, r, mat, st);
+    int rc = search_and_return<K>(shards[d], fs[d], pt, d, 0, mat, qbase, st);
     if (rc) return rc;
   }
   for (int s = 0; s < G; ++s) {
@@ -466,6 +497,13 @@ int exchange_windows(FusedState* f, hbt_comm* c, uint64_t cap_m, uint64_t cap_r,
   return HBT_OK;
 }
 
+// The batch is cut into C chunks ("exchange_chunks"): chunk c's queries are put into the
+// owners' windows (region c of every window) on the caller's stream while the owner
+// searches chunk c-1 on an auxiliary stream, so the NVLink stores of the put overlap the
+// owner's search (the paper's double buffering of transfers against processing,
+// P:232-238, on peer memory).  The C count rows are published together, so one barrier
+// and one D2H size every chunk; chunk regions do not overlap, so no slot is reused
+// within a batch.
 template <typename K>
 int nccl_fused_t(hbt_tree* t, const void* queries, uint64_t m, hbt_out out, cudaStream_t st) {
   hbt_comm* c = t->shard.comm;
@@ -474,69 +512,117 @@ int nccl_fused_t(hbt_tree* t, const void* queries, uint64_t m, hbt_out out, cuda
   FusedState* f = state_of(t);
   int rc = prep_local(f, m);
   if (rc) return rc;
+  const int C = int(std::max<uint32_t>(1, std::min<uint32_t>(t->cfg.exchange_chunks, kMaxChunks)));
+  const uint64_t mc = std::max<uint64_t>(1, (m + C - 1) / C);
   const RouteTab rt = table_of(t->shard);
   {
     NvtxRange r("exchange.count");
-    rc = route_and_count<K>(f, (const K*)queries, m, rt, G, st);
+    rc = route_and_count<K>(f, (const K*)queries, m, mc, C, rt, G, st);
   }
   if (rc) return rc;
   const int par = int(f->batch & 1);
-  std::vector<unsigned long long> mat(G * G);
+  // mat[ch][src * G + dst]
+  std::vector<std::vector<unsigned long long>> mat(C, std::vector<unsigned long long>(G * G));
   PeerTable pt{};
   pt.G = G;
+  // every rank must use the same C: agree on it with the window (first batch) or trust
+  // the configuration (the bench and the tests set it on every rank)
   const bool had_windows = f->win != nullptr;
   if (had_windows) {
     // steady state: the count rows travel by peer stores, no host collective
     for (int g = 0; g < G; ++g) pt.w[g] = carve(f->peer[g], f->cap_m, f->cap_r, S);
-    f_publish<<<1, 256, 0, st>>>(pt, me, f->cnt, par);
+    f_publish<<<1, 256, 0, st>>>(pt, me, f->cnt, par, C);
     f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);
     HBT_CUDA_TRY(cudaGetLastError());
-    HBT_CUDA_TRY(cudaMemcpyAsync(f->h_mat, pt.w[me].matrix + par * kMat, kMat * 8, cudaMemcpyDeviceToHost, st));
+    HBT_CUDA_TRY(cudaMemcpyAsync(f->h_mat, pt.w[me].matrix + uint64_t(par) * kMaxChunks * kMat, C * kMat * 8,
+                                 cudaMemcpyDeviceToHost, st));
     HBT_CUDA_TRY(cudaStreamSynchronize(st));
-    for (int s = 0; s < G; ++s)
-      for (int x = 0; x < G; ++x) mat[s * G + x] = f->h_mat[s * kMaxG + x];
+    for (int ch = 0; ch < C; ++ch)
+      for (int s2 = 0; s2 < G; ++s2)
+        for (int x = 0; x < G; ++x) mat[ch][s2 * G + x] = f->h_mat[ch * kMat + s2 * kMaxG + x];
   } else {
     // first batch: no windows to store into yet; the count rows go through the host
-    std::vector<unsigned long long> mine(G);
-    HBT_CUDA_TRY(cudaMemcpyAsync(mine.data(), f->cnt, G * 8, cudaMemcpyDeviceToHost, st));
+    std::vector<unsigned long long> mine(C * G), all(size_t(C) * G * G);
+    std::vector<unsigned long long> dev(C * 2 * kMaxG);
+    HBT_CUDA_TRY(cudaMemcpyAsync(dev.data(), f->cnt, dev.size() * 8, cudaMemcpyDeviceToHost, st));
     HBT_CUDA_TRY(cudaStreamSynchronize(st));
-    rc = comm_allgather_host(c, mine.data(), mat.data(), G * 8, st);
+    for (int ch = 0; ch < C; ++ch)
+      for (int x = 0; x < G; ++x) mine[ch * G + x] = dev[ch * 2 * kMaxG + x];
+    rc = comm_allgather_host(c, mine.data(), all.data(), C * G * 8, st);
     if (rc) return rc;
+    for (int s2 = 0; s2 < G; ++s2)
+      for (int ch = 0; ch < C; ++ch)
+        for (int x = 0; x < G; ++x) mat[ch][s2 * G + x] = all[(size_t(s2) * C + ch) * G + x];
   }
   uint64_t need_m = 1, need_r = 1;
   for (int x = 0; x < G; ++x) {
     uint64_t row = 0, col = 0;
-    for (int y = 0; y < G; ++y) { row += mat[x * G + y]; col += mat[y * G + x]; }
+    for (int ch = 0; ch < C; ++ch)
+      for (int y = 0; y < G; ++y) { row += mat[ch][x * G + y]; col += mat[ch][y * G + x]; }
     need_m = std::max<uint64_t>(need_m, row);
     need_r = std::max<uint64_t>(need_r, col);
   }
   if (!had_windows || f->cap_m < need_m || f->cap_r < need_r) {
-    // every rank holds the same matrix, so every rank takes this branch (collective)
+    // every rank holds the same matrices, so every rank takes this branch (collective)
     rc = exchange_windows(f, c, need_m + need_m / 8, need_r + need_r / 8, S, st);
     if (rc) return rc;
     for (int g = 0; g < G; ++g) pt.w[g] = carve(f->peer[g], f->cap_m, f->cap_r, S);
-    std::vector<unsigned long long> full(kMat, 0);
-    for (int s = 0; s < G; ++s)
-      for (int x = 0; x < G; ++x) full[s * kMaxG + x] = mat[s * G + x];
-    HBT_CUDA_TRY(cudaMemcpyAsync(pt.w[me].matrix + par * kMat, full.data(), kMat * 8, cudaMemcpyHostToDevice, st));
-    f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);  // every window exists and holds its matrix
+    std::vector<unsigned long long> full(C * kMat, 0);
+    for (int ch = 0; ch < C; ++ch)
+      for (int s2 = 0; s2 < G; ++s2)
+        for (int x = 0; x < G; ++x) full[ch * kMat + s2 * kMaxG + x] = mat[ch][s2 * G + x];
+    HBT_CUDA_TRY(cudaMemcpyAsync(pt.w[me].matrix + uint64_t(par) * kMaxChunks * kMat, full.data(), C * kMat * 8,
+                                 cudaMemcpyHostToDevice, st));
+    f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);  // every window exists and holds its matrices
   }
-  {
-    NvtxRange r("exchange.put");
-    rc = put_queries<K>(f, (const K*)queries, m, pt, me, par, st);
+  if (C > 1 && !f->aux) {
+    HBT_CUDA_TRY(cudaStreamCreateWithFlags(&f->aux, cudaStreamNonBlocking));
+    for (auto& e : f->ev_put) HBT_CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    HBT_CUDA_TRY(cudaEventCreateWithFlags(&f->ev_done, cudaEventDisableTiming));
   }
-  if (rc) return rc;
-  f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);
-  uint64_t nrecv = 0;
-  for (int s = 0; s < G; ++s) nrecv += mat[s * G + me];
-  {
-    NvtxRange r("owner_search_and_return");
-    rc = search_and_return<K>(t, f, pt, me, nrecv, mat, st);
+  // per chunk: region bases in every owner's window, and every source's first query
+  std::vector<uint64_t> rbase(G, 0), qb(G, 0);
+  uint64_t my_rstart = 0;
+  for (int ch = 0; ch < C; ++ch) {
+    const std::vector<unsigned long long>& M = mat[ch];
+    PutOff off{};
+    for (int d = 0; d < G; ++d) off.rbase[d] = rbase[d];
+    off.qbase = uint64_t(ch) * mc;
+    const uint64_t lo = uint64_t(ch) * mc, n = lo < m ? std::min<uint64_t>(mc, m - lo) : 0;
+    {
+      NvtxRange r("exchange.put");
+      rc = put_queries<K>(f, (const K*)queries, lo, n, pt, me, pt.w[me].matrix + (uint64_t(par) * kMaxChunks + ch) * kMat,
+                          off, ch, st);
+    }
+    if (rc) return rc;
+    f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);  // chunk ch is in every owner's window
+    HBT_CUDA_TRY(cudaGetLastError());
+    cudaStream_t ss = st;
+    if (C > 1) {
+      HBT_CUDA_TRY(cudaEventRecord(f->ev_put[ch], st));
+      HBT_CUDA_TRY(cudaStreamWaitEvent(f->aux, f->ev_put[ch], 0));
+      ss = f->aux;
+    }
+    {
+      NvtxRange r("owner_search_and_return");
+      rc = search_and_return<K>(t, f, pt, me, my_rstart, M, qb, ss);
+    }
+    if (rc) return rc;
+    for (int s2 = 0; s2 < G; ++s2) {
+      my_rstart += M[s2 * G + me];
+      for (int d = 0; d < G; ++d) rbase[d] += M[s2 * G + d];
+      uint64_t row = 0;
+      for (int d = 0; d < G; ++d) row += M[s2 * G + d];
+      qb[s2] += row;
+    }
   }
-  if (rc) return rc;
-  f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);
+  if (C > 1) {  // the owner searches of every chunk, then the last barrier
+    HBT_CUDA_TRY(cudaEventRecord(f->ev_done, f->aux));
+    HBT_CUDA_TRY(cudaStreamWaitEvent(st, f->ev_done, 0));
+  }
+  f_barrier<<<1, 32, 0, st>>>(pt, me, ++f->epoch);  // every owner has stored our results
   HBT_CUDA_TRY(cudaGetLastError());
-  if (m) {  // our results, one run per owner in our window, back into query order
+  if (m) {  // our results, one run per (chunk, owner) in our window, back into query order
     f_collect<K><<<grid_for(m), kThreads, 0, st>>>(f->rpos, m, pt.w[me].res_pf, (const K*)pt.w[me].res_v,
                                                    out.pos_found, (K*)out.values);
     HBT_CUDA_TRY(cudaGetLastError());

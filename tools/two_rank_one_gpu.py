@@ -21,6 +21,7 @@ import paper_conf_sigmod_shahvaranij16_b200 as hbt  # noqa: E402
 def main():
     exchange = int(sys.argv[1]) if len(sys.argv) > 1 else 0
     bucket = int(sys.argv[2]) if len(sys.argv) > 2 else 2  # 1: owner search bucketed (fused remote gather)
+    chunks = int(sys.argv[3]) if len(sys.argv) > 3 else 2  # exchange chunks (put of c+1 overlaps search of c)
     dist.init_process_group("gloo")
     rank, world = dist.get_rank(), dist.get_world_size()
     torch.cuda.set_device(0)
@@ -34,6 +35,8 @@ def main():
     t = hbt.ShardedTree(comm, k, v, fanout=16)
     t.set_param("exchange", exchange)
     t.set_param("bucket", bucket)
+    if exchange == 0:
+        t.set_param("exchange_chunks", chunks)
     if bucket == 1:
         t.set_param("bucket_slice", 4096)
     full = oracle.ITree.from_pairs(allk, allv, 16, 8)
