@@ -39,6 +39,7 @@
 #include <mutex>
 #include <vector>
 
+#include "block_util.cuh"
 #include "hbt_internal.cuh"
 #include "item_dir.cuh"
 
@@ -109,6 +110,34 @@ __global__ void bk_level_max(const uint8_t* __restrict__ leaf, uint64_t n, uint3
   }
 }
 
+// Compressed item directory (ItemDir::bd): one CTA per bucket derives the offset
+// origin lo = M[u0] and the shift that fits M[u0 + cnt - 1] - lo in 32 bits, then
+// writes M32[off + i] = (M[u0 + i] - lo) >> sh (padding to 4 entries: ~0).
+template <typename K>
+__global__ void bk_dir32(const K* __restrict__ M, BucketDir32* __restrict__ bd, uint32_t* __restrict__ M32) {
+  __shared__ K s_lo;
+  __shared__ uint32_t s_sh;
+  BucketDir32* d = bd + blockIdx.x;
+  const uint64_t u0 = d->u0, off = d->off;
+  const uint32_t cnt = d->cnt;
+  if (threadIdx.x == 0) {
+    const K lo = M[u0], span = K(M[u0 + cnt - 1] - lo);
+    const uint32_t bits = span ? uint32_t(8 * sizeof(K)) - uint32_t(sizeof(K) == 8 ? __clzll((long long)span)
+                                                                                 : __clz(int(span)))
+                               : 0u;
+    s_lo = lo;
+    s_sh = bits > 32 ? bits - 32 : 0u;
+    d->lo = uint64_t(lo);
+    d->sh = s_sh;
+  }
+  __syncthreads();
+  const K lo = s_lo;
+  const uint32_t sh = s_sh;
+  const uint32_t padded = (cnt + 3u) & ~3u;
+  for (uint32_t i = threadIdx.x; i < padded; i += blockDim.x)
+    M32[off + i] = i < cnt ? uint32_t(K(M[u0 + i] - lo) >> sh) : ~0u;
+}
+
 // Item directory (regular): M[c * NI + t] = true max key of key line t of the
 // last-level node of chain leaf c = the key of entry min(count, (t+1)*KPL*P) - 1
 // (KPL separators per 64 B key line, each covering one leaf line of P entries);
@@ -154,38 +183,6 @@ __device__ __forceinline__ uint32_t bucket_of(K q, const K* s_sp, const uint32_t
   constexpr int sh = 8 * int(sizeof(K)) - int(kDirBits);
   const uint32_t e = s_dir[uint32_t(q >> sh)];
   return lower_bound_in(s_sp, e & 0xFFFFu, e >> 16, q);
-}
-
-// Exclusive scan of s_in[0, B) into s_out (B <= 2 * TH) by one CTA of TH threads:
-// two elements per thread, a shuffle scan per warp, the warp totals (s_tmp) scanned
-// by warp 0.  Ends with a barrier.
-template <int TH = kThreads>
-__device__ __forceinline__ void block_exclusive_scan(const uint32_t* s_in, uint32_t* s_out, uint32_t B,
-                                                     uint32_t* s_tmp) {
-  const uint32_t t = threadIdx.x, lane = t & 31, wid = t >> 5;
-  const uint32_t a = 2 * t < B ? s_in[2 * t] : 0u, b = 2 * t + 1 < B ? s_in[2 * t + 1] : 0u;
-  uint32_t x = a + b;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-    if (lane >= uint32_t(o)) x += y;
-  }
-  if (lane == 31) s_tmp[wid] = x;
-  __syncthreads();
-  if (wid == 0) {
-    uint32_t w = lane < uint32_t(TH / 32) ? s_tmp[lane] : 0u;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t y = __shfl_up_sync(0xffffffffu, w, o);
-      if (lane >= uint32_t(o)) w += y;
-    }
-    if (lane < uint32_t(TH / 32)) s_tmp[lane] = w;
-  }
-  __syncthreads();
-  const uint32_t ex = x - (a + b) + (wid ? s_tmp[wid - 1] : 0u);
-  if (2 * t < B) s_out[2 * t] = ex;
-  if (2 * t + 1 < B) s_out[2 * t + 1] = ex + a;
-  __syncthreads();
 }
 
 // Pass 1: bucket of every query (bq, u16), the per-chunk histograms (chunk-major:
@@ -353,7 +350,7 @@ __global__ void __launch_bounds__(kThreads, 2) bk_scatter(const K* __restrict__ 
       }
     }
     __syncthreads();
-    block_exclusive_scan(s_cnt, s_lb, B, s_tmp);
+    block_exclusive_scan<kThreads>(s_cnt, s_lb, B, s_tmp);
 #pragma unroll
     for (int x = 0; x < kQPT; ++x) {
       const uint32_t t = uint32_t(x) * kThreads + threadIdx.x;
@@ -383,31 +380,6 @@ __global__ void __launch_bounds__(kThreads, 2) bk_scatter(const K* __restrict__ 
 // mbarrier) while the CTA sorts and writes the current chunk, so no warp waits on
 // DRAM for its inputs and no registers hold them in flight.  1024 threads, 8 queries
 // each; the sort and the run writes are those of bk_scatter.
-__device__ __forceinline__ uint32_t smem_u32(const void* p) { return uint32_t(__cvta_generic_to_shared(p)); }
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  asm volatile(
-      "{\n"
-      " .reg .pred p;\n"
-      "WAIT_%=:\n"
-      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-      " @!p bra WAIT_%=;\n"
-      "}\n" ::"r"(smem_u32(bar)),
-      "r"(parity)
-      : "memory");
-}
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                   smem_u32(dst)),
-               "l"(src), "r"(bytes), "r"(smem_u32(bar))
-               : "memory");
-}
-
 constexpr int kTThreads = 1024;
 constexpr int kTQPT = int(kChunk) / kTThreads;  // 8 queries per thread
 
@@ -449,7 +421,7 @@ __global__ void __launch_bounds__(kTThreads, 1) bk_scatter_tma(const K* __restri
   const uint64_t full = m / kChunk;  // chunks served by bulk copies; the tail chunk reads directly
   if (threadIdx.x == 0) {
     mbar_init(bar, 1);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    fence_mbar_init();
   }
   __syncthreads();
   if (threadIdx.x == 0 && blockIdx.x < full) issue(blockIdx.x);
@@ -494,7 +466,7 @@ __global__ void __launch_bounds__(kTThreads, 1) bk_scatter_tma(const K* __restri
     if (threadIdx.x == 0) {
       const uint64_t cn = c + gridDim.x;
       if (cn < full) {
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        fence_proxy_async_smem();
         issue(cn);
       }
     }
@@ -754,6 +726,19 @@ uint32_t pick_buckets(const hbt_tree* t) {
   return uint32_t(std::max<uint64_t>(B, 1));
 }
 
+// Units of bucket b at a directory level of `span` leaf lines per unit (the units
+// holding leaf lines [floor(bU/B), floor((b+1)U/B) - 1], where b's queries end).
+static inline void bucket_units(uint64_t U, uint32_t B, uint32_t b, uint64_t span, uint64_t& u0, uint64_t& u1) {
+  u0 = ((uint64_t(b) * U) / B) / span;
+  u1 = (((uint64_t(b) + 1) * U) / B - 1) / span;
+}
+
+// Shared-memory entries of the compressed directory: ~200 KB per CTA beside the
+// bucket starts, item starts and the 2^12-entry prefix table.
+uint64_t item_cap32(uint32_t B) {
+  return (200 * 1024 - (uint64_t(B) + 1) * 12 - ((1u << 12) + 1) * 4 - 64) / 4;
+}
+
 // Shared-memory entries of the item directory (keys; the regular tree also
 // stages one u32 chain id per NI entries): ~150 KB per CTA beside the bucket starts.
 uint64_t item_cap(const hbt_tree* t, uint32_t B) {
@@ -794,6 +779,7 @@ int prepare_splitters(const hbt_tree* t, cudaStream_t s, BucketState& bs, uint32
   if (want_items && t->cfg.bucket_items) {
     const uint64_t cap = item_cap(t, B);
     uint64_t nunits = 0;
+    bs.d32 = false;
     if (t->form == HBT_IMPLICIT) {
       uint64_t span = 1;
       for (int d = int(t->H); d >= 0; --d) {
@@ -806,6 +792,31 @@ int prepare_splitters(const hbt_tree* t, cudaStream_t s, BucketState& bs, uint32
           break;
         }
         span *= t->F;
+      }
+      // the compressed per-bucket form, where it reaches a deeper level (or when forced)
+      if (t->cfg.item_dir32 && !t->cfg.bucket_cap) {
+        const uint64_t cap32 = item_cap32(B);
+        uint64_t span32 = 1;
+        for (int d = int(t->H); d >= 0; --d) {
+          uint64_t most = 0;
+          for (uint32_t b = 0; b < B; ++b) {
+            uint64_t u0, u1;
+            bucket_units(t->L0, B, b, span32, u0, u1);
+            most = std::max<uint64_t>(most, u1 - u0 + 1);
+          }
+          if (most <= cap32) {
+            if (!bs.items || d > int(bs.level) || t->cfg.item_dir32 == 2) {
+              bs.level = uint32_t(d);
+              bs.span = span32;
+              nunits = d == int(t->H) ? t->L0 : t->nodes[d];
+              bs.items = true;
+              bs.d32 = true;
+              bs.cap32 = uint32_t((most + 3) & ~uint64_t(3));
+            }
+            break;
+          }
+          span32 *= t->F;
+        }
       }
     } else {
       const uint32_t KPL = 64 / sizeof(K);
@@ -833,6 +844,27 @@ int prepare_splitters(const hbt_tree* t, cudaStream_t s, BucketState& bs, uint32
         bk_keyline_max<K><<<t->num_sms * 4, 256, 0, s>>>((const uint8_t*)t->r.d_leaf, t->r.d_count, t->r.d_chain,
                                                           t->r.nchain, t->F, t->P, uint32_t(bs.span),
                                                           uint32_t(64 / sizeof(K)), (K*)bs.d_M);
+      HBT_CUDA_TRY(cudaGetLastError());
+    }
+    if (bs.d32) {
+      std::vector<BucketDir32> h(B);
+      uint64_t total = 0;
+      for (uint32_t b = 0; b < B; ++b) {
+        uint64_t u0, u1;
+        bucket_units(t->L0, B, b, bs.span, u0, u1);
+        h[b] = BucketDir32{u0, total, 0, uint32_t(u1 - u0 + 1), 0};
+        total += (u1 - u0 + 1 + 3) & ~uint64_t(3);
+      }
+      if (!bs.d_bd) HBT_CUDA_TRY(cudaMalloc(&bs.d_bd, kMaxBuckets * sizeof(BucketDir32)));
+      if (bs.M32_cap < total * 4) {
+        cudaFree(bs.d_M32);
+        bs.d_M32 = nullptr;
+        bs.M32_cap = 0;
+        HBT_CUDA_TRY(cudaMalloc(&bs.d_M32, total * 4));
+        bs.M32_cap = total * 4;
+      }
+      HBT_CUDA_TRY(cudaMemcpyAsync(bs.d_bd, h.data(), B * sizeof(BucketDir32), cudaMemcpyHostToDevice, s));
+      bk_dir32<K><<<B, 256, 0, s>>>((const K*)bs.d_M, (BucketDir32*)bs.d_bd, bs.d_M32);
       HBT_CUDA_TRY(cudaGetLastError());
     }
   }
@@ -957,6 +989,11 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
       d.pos_base = pos_base;
       d.cap = t->cfg.bucket_cap ? std::min<uint32_t>(t->cfg.bucket_cap, uint32_t(item_cap(t, p.B)))
                                 : uint32_t(item_cap(t, p.B));
+      if (bs.d32) {
+        d.bd = static_cast<const BucketDir32*>(bs.d_bd);
+        d.M32 = bs.d_M32;
+        d.cap = bs.cap32;
+      }
       rc = t->form == HBT_IMPLICIT ? implicit_search_items(t, qs, m, pf_s, v_s, d, s)
                                    : regular_search_items(t, qs, m, pf_s, v_s, d, s);
     } else {
@@ -1143,6 +1180,8 @@ static void bucket_state_free(BucketState& b) {
   cudaFree(b.d_sp);
   cudaFree(b.d_dir);
   cudaFree(b.d_M);
+  cudaFree(b.d_bd);
+  cudaFree(b.d_M32);
   b = BucketState{};
 }
 

@@ -89,6 +89,8 @@ struct SearchConfig {
   uint32_t l2_hint = 4;          // implicit search: L2 eviction-priority hints (LevelTable::l2_hint);
                                  // 4 = auto: leaf lines evict-first iff the I-segment fits in L2 / 4
   uint32_t item_l2_hint = 1;     // implicit bucketed item search (c4 item search 10.96 -> 9.50 ms)
+  uint32_t item_dir32 = 1;       // implicit item directory in the compressed per-bucket form (ItemDir::bd):
+                                 // 0 = never, 1 = where it reaches a deeper level, 2 = always
 };
 
 // Bucket-local directory of the bucketed search (bucketed.cu): after the
@@ -112,6 +114,21 @@ struct ItemDir {
   uint32_t cap = 0;    // shared-memory entries (larger ranges search M in global memory)
   uint64_t pos_base = 0;  // implicit: added to every reported position (key-range shards)
   uint32_t rounds = 16;   // warp rounds per work item (fewer for small batches: every SM gets items)
+  // Compressed per-bucket directory (implicit trees whose directory level has too many
+  // units per bucket for 8 B keys in shared memory): bucket b's unit maxima as 32-bit
+  // offsets M32[bd[b].off + i] = (M[bd[b].u0 + i] - bd[b].lo) >> bd[b].sh, items cut
+  // inside one bucket each (item search).
+  const struct BucketDir32* bd = nullptr;
+  const uint32_t* M32 = nullptr;
+};
+
+// One bucket of the compressed item directory (ItemDir::bd).
+struct BucketDir32 {
+  uint64_t u0;   // first directory unit of the bucket
+  uint64_t off;  // its first entry in M32 (a multiple of 4: 16 B aligned bulk copies)
+  uint64_t lo;   // M[u0]: the offset origin
+  uint32_t cnt;  // units u0 .. u0 + cnt - 1
+  uint32_t sh;   // right shift that makes M[u0 + cnt - 1] - lo fit 32 bits
 };
 
 // Owner side of the fused sharded exchange (sharded_fused.cu): the bucketed search's
@@ -140,6 +157,11 @@ struct BucketState {
   uint32_t level = 0;            // implicit: directory level
   uint64_t span = 1, nunits = 0;
   bool items = false;            // the item directory is in use
+  bool d32 = false;              // ... in its compressed per-bucket form (ItemDir::bd)
+  void* d_bd = nullptr;          // B x BucketDir32
+  uint32_t* d_M32 = nullptr;     // compressed maxima
+  uint64_t M32_cap = 0;          // bytes allocated
+  uint32_t cap32 = 0;            // largest bucket's unit count, rounded up to 4
   cudaEvent_t ev[6] = {};        // phase boundaries of the last timed bucketed search
   bool timed = false;
   uint32_t launches = 0;

@@ -27,6 +27,7 @@
 // displace the tree from L2.
 #include <algorithm>
 
+#include "block_util.cuh"
 #include "hbt_internal.cuh"
 #include "item_dir.cuh"
 
@@ -507,6 +508,134 @@ implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* _
   }
 }
 
+// The same with the COMPRESSED per-bucket directory (ItemDir::bd / M32), used when
+// it reaches a deeper level than 8 B keys would (c4: the last inner level instead of
+// the one above it, one dependent node read less per query).  Work items are cut
+// inside one bucket each (bucket b's queries split into ceil(cnt_b / W) near-equal
+// items), so an item stages exactly its bucket's unit maxima: one elected thread
+// moves them into shared memory with bulk copies (cp.async.bulk, completion on an
+// mbarrier).  Entry i holds (M[u0+i] - lo) >> sh: order-preserving, so
+// lower_bound(M32, (q - lo) >> sh) is exact except where the truncated values tie
+// with the query's; those few entries are compared exactly against M in global
+// memory (sh = 0, i.e. bucket key spans below 2^32, never ties).
+constexpr uint32_t kPrefixBits32 = 12;
+
+template <typename K>
+__device__ __forceinline__ uint32_t lower_bound32(const uint32_t* s_M, uint32_t cnt, const uint32_t* s_T,
+                                                  const PrefixTab<uint32_t>& pt, K q, K lo, uint32_t sh,
+                                                  const K* __restrict__ gM) {
+  if (q <= lo) return 0;
+  const K dq = K(q - lo) >> sh;
+  if (dq > K(pt.span)) return cnt;  // beyond the bucket's last maximum (pt.lo = s_M[0] = 0)
+  const uint32_t q32 = uint32_t(dq);
+  uint32_t a = prefix_lower_bound(s_M, cnt, s_T, pt, q32);
+  if (sh)
+    while (a < cnt && s_M[a] == q32 && __ldg(gM + a) < q) ++a;
+  return a;
+}
+
+template <typename K, int F, int THREADS>
+__global__ void __launch_bounds__(THREADS)
+implicit_search_items32_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ inner_idx,
+                               const uint8_t* __restrict__ leaf, const ItemDir d, const K* __restrict__ queries,
+                               uint64_t m, uint64_t* __restrict__ out_pf, K* __restrict__ out_v, const LevelTable lt,
+                               uint64_t n) {
+  using C = Cfg<K, F>;
+  constexpr int QPG = 32 / C::NG;
+  constexpr uint32_t PB = kPrefixBits32;
+  const uint64_t W = uint64_t(THREADS) * d.rounds;
+  const uint32_t B = d.B;
+  extern __shared__ __align__(16) uint8_t smem[];
+  // [M32: cap entries | bucket starts: B + 1 u64 | prefix table: 2^PB + 1 | item starts: B + 1]
+  uint32_t* s_M = reinterpret_cast<uint32_t*>(smem);
+  uint64_t* s_bs = reinterpret_cast<uint64_t*>(s_M + d.cap);
+  uint32_t* s_T = reinterpret_cast<uint32_t*>(s_bs + B + 1);
+  uint32_t* s_is = s_T + (1u << PB) + 1;
+  __shared__ uint64_t bar;
+  __shared__ uint32_t s_tmp[32];
+  __shared__ uint64_t s_p[2];
+  __shared__ BucketDir32 s_bd;
+  const K* gM = static_cast<const K*>(d.M);
+  for (uint32_t i = threadIdx.x; i <= B; i += THREADS) s_bs[i] = d.bstart[i];
+  __syncthreads();
+  // items per bucket, then their starts (B <= 2 * THREADS)
+  for (uint32_t b = threadIdx.x; b < B; b += THREADS) s_is[b] = uint32_t((s_bs[b + 1] - s_bs[b] + W - 1) / W);
+  __syncthreads();
+  const uint32_t last = s_is[B - 1];
+  block_exclusive_scan<THREADS>(s_is, s_is, B, s_tmp);
+  if (threadIdx.x == 0) {
+    s_is[B] = s_is[B - 1] + last;
+    mbar_init(&bar, 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  const uint32_t items = s_is[B];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int g = lane / C::G, k = lane % C::G;
+  const unsigned gmask = ((1u << C::G) - 1u) << (g * C::G);
+  uint32_t parity = 0;
+  for (uint32_t it = blockIdx.x; it < items; it += gridDim.x) {
+    if (threadIdx.x == 0) {
+      uint32_t lo = 0, hi = B;  // the bucket: largest b with s_is[b] <= it
+      while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (s_is[mid] <= it) lo = mid; else hi = mid;
+      }
+      const uint64_t nb = s_is[lo + 1] - s_is[lo], j = it - s_is[lo];
+      const uint64_t c0 = s_bs[lo], cnt = s_bs[lo + 1] - c0;
+      s_p[0] = c0 + (cnt * j) / nb;
+      s_p[1] = c0 + (cnt * (j + 1)) / nb - 1;
+      const BucketDir32 bd = d.bd[lo];
+      s_bd = bd;
+      // the previous item's reads of s_M are ordered before this copy by the barrier
+      // that ended it; the proxy fence orders them for the async (bulk copy) proxy
+      fence_proxy_async_smem();
+      const uint32_t bytes = (bd.cnt * 4u + 15u) & ~15u;
+      mbar_expect_tx(&bar, bytes);
+      for (uint32_t o = 0; o < bytes; o += 32768u)
+        bulk_g2s(reinterpret_cast<uint8_t*>(s_M) + o, d.M32 + bd.off + o / 4, bytes - o < 32768u ? bytes - o : 32768u,
+                 &bar);
+    }
+    __syncthreads();
+    const uint64_t p0 = s_p[0], p1 = s_p[1];
+    const uint64_t u0 = s_bd.u0;
+    const uint32_t cnt = s_bd.cnt, sh = s_bd.sh;
+    const K blo = K(s_bd.lo);
+    mbar_wait(&bar, parity);
+    parity ^= 1u;
+    const PrefixTab<uint32_t> pt = build_prefix(s_M, cnt, s_T, THREADS, PB);
+    __syncthreads();
+    K nextq;
+    {
+      const uint64_t i = p0 + uint64_t(wid) * 32 + lane;
+      nextq = i <= p1 ? ldcs(queries + i) : key_max<K>();
+    }
+#pragma unroll 1
+    for (int r = 0; r < int(d.rounds); ++r) {
+      const uint64_t base = p0 + (uint64_t(r) * (THREADS / 32) + wid) * 32;
+      if (base > p1) break;
+      const K myq = nextq;
+      {
+        const uint64_t i = base + (THREADS / 32) * 32 + lane;
+        nextq = (r + 1 < int(d.rounds) && i <= p1) ? ldcs(queries + i) : key_max<K>();
+      }
+      const uint32_t a = lower_bound32(s_M, cnt, s_T, pt, myq, blo, sh, gM + u0);
+      const uint32_t mynode = uint32_t(u0) + (a < cnt ? a : cnt - 1);
+      K q[QPG];
+      uint32_t node[QPG];
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) {
+        const int src = (j * C::NG) % 32 + g;
+        q[j] = __shfl_sync(0xffffffffu, myq, src);
+        node[j] = __shfl_sync(0xffffffffu, mynode, src);
+      }
+      descend_and_store<K, F, QPG, true>(inner, inner_idx, leaf, lt, d.level, q, node, g, k, gmask, base, p1 + 1, n,
+                                         d.pos_base, out_pf, out_v);
+    }
+    __syncthreads();
+  }
+}
+
 template <typename K, int F>
 struct Launch {
   using C = Cfg<K, F>;
@@ -605,6 +734,33 @@ struct Launch {
     return HBT_OK;
   }
 
+  static int run_items32(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, const ItemDir& d,
+                         cudaStream_t s) {
+    constexpr int TH = C::NODE_BYTES > 128 ? 512 : 1024;
+    auto kern = implicit_search_items32_kernel<K, F, TH>;
+    LevelTable lt{};
+    for (uint32_t x = 0; x <= t->H; ++x) lt.offset[x] = t->offset[x];
+    lt.H = t->H;
+    lt.SL = d.level;
+    lt.leaf256 = t->cfg.leaf256;
+    lt.full256 = t->cfg.full256;
+    lt.l2_hint = t->cfg.item_l2_hint;
+    lt.full_mask = full_mask(t, d.level);
+    static bool attr_set = false;
+    if (!attr_set) {
+      HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024));
+      attr_set = true;
+    }
+    ItemDir dd = d;
+    dd.rounds = item_rounds(m, t->num_sms, TH, t->cfg.item_rounds ? t->cfg.item_rounds : 16);
+    const size_t smem = size_t(d.cap) * 4 + (size_t(d.B) + 1) * 8 + ((1u << kPrefixBits32) + 1) * 4 +
+                        (size_t(d.B) + 1) * 4;
+    kern<<<t->num_sms, TH, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
+                                     (const uint8_t*)t->d_leaf, dd, (const K*)q, m, pf, (K*)v, lt, t->n);
+    HBT_CUDA_TRY(cudaGetLastError());
+    return HBT_OK;
+  }
+
   static int run(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, uint64_t b, cudaStream_t s,
                  const void* lp) {
     // small batches read the directory in place with 256-thread CTAs, so a one-wave
@@ -654,6 +810,14 @@ int implicit_search_items(const hbt_tree* t, const void* q, uint64_t m, uint64_t
   if (m == 0) return HBT_OK;
   auto go = [&](auto tag) -> int {
     using K = decltype(tag);
+    if (d.bd) {
+      switch (t->F) {
+        case 4: return Launch<K, 4>::run_items32(t, q, m, pf, v, d, s);
+        case 8: return Launch<K, 8>::run_items32(t, q, m, pf, v, d, s);
+        case 16: return Launch<K, 16>::run_items32(t, q, m, pf, v, d, s);
+        case 32: return Launch<K, 32>::run_items32(t, q, m, pf, v, d, s);
+      }
+    }
     switch (t->F) {
       case 4: return Launch<K, 4>::run_items(t, q, m, pf, v, d, s);
       case 8: return Launch<K, 8>::run_items(t, q, m, pf, v, d, s);

@@ -26,14 +26,15 @@ def _oracle(layout, k, v, F, width):
     return (oracle.ITree if layout == "implicit" else oracle.RTree).from_pairs(k, v, F, width)
 
 
-# (bucket_items, bucket_cap, leaf256): plain search, smem directory, global fallback, 128-bit lane loads
-ITEM_MODES = [(0, 0, 1), (1, 0, 1), (1, 7, 1), (1, 0, 0)]
+# (bucket_items, bucket_cap, leaf256, item_dir32): plain search, 8 B smem directory, global
+# fallback, 128-bit lane loads (directory form auto), compressed per-bucket directory forced
+ITEM_MODES = [(0, 0, 1, 1), (1, 0, 1, 0), (1, 7, 1, 1), (1, 0, 0, 1), (1, 0, 1, 2)]
 
 
 @pytest.mark.parametrize("layout", ["implicit", "regular"])
 @pytest.mark.parametrize("width,F", [(4, 8), (8, 16), (8, 32), (4, 32)])
-@pytest.mark.parametrize("items,cap,leaf256", ITEM_MODES)
-def test_bucketed_edge_suite(hbt, layout, width, F, items, cap, leaf256):
+@pytest.mark.parametrize("items,cap,leaf256,dir32", ITEM_MODES)
+def test_bucketed_edge_suite(hbt, layout, width, F, items, cap, leaf256, dir32):
     P = 64 // (2 * width)
     rng = np.random.default_rng(900 + 10 * F + width)
     for n in sorted({0, 1, 2, P + 1, F * P + 1, 5 * F * P + 3, 30011}):
@@ -47,6 +48,7 @@ def test_bucketed_edge_suite(hbt, layout, width, F, items, cap, leaf256):
         t.set_param("bucket_items", items)
         t.set_param("bucket_cap", cap)
         t.set_param("leaf256", leaf256)
+        t.set_param("item_dir32", dir32)
         for slice_bytes in (1, 4096, 1 << 16):  # 1 B: one bucket per unit up to the 1024 cap
             t.set_param("bucket_slice", slice_bytes)
             pf, val = gpu_search(t, q, width)
@@ -57,8 +59,8 @@ def test_bucketed_edge_suite(hbt, layout, width, F, items, cap, leaf256):
 
 
 @pytest.mark.parametrize("layout,F", [("implicit", 16), ("regular", 32)])
-@pytest.mark.parametrize("items,cap,leaf256", ITEM_MODES)
-def test_bucketed_scaled_workload(hbt, layout, F, items, cap, leaf256):
+@pytest.mark.parametrize("items,cap,leaf256,dir32", ITEM_MODES)
+def test_bucketed_scaled_workload(hbt, layout, F, items, cap, leaf256, dir32):
     """c2 / c3 recipes at reduced size, several bucket counts, every output vs the oracle."""
     cfg = "c2" if layout == "implicit" else "c3"
     n, m = 1 << 19, 1 << 20
@@ -71,6 +73,7 @@ def test_bucketed_scaled_workload(hbt, layout, F, items, cap, leaf256):
     t.set_param("bucket_items", items)
     t.set_param("bucket_cap", cap)
     t.set_param("leaf256", leaf256)
+    t.set_param("item_dir32", dir32)
     for slice_bytes in (1 << 16, 1 << 20, 1 << 22):
         t.set_param("bucket_slice", slice_bytes)
         for qpf in (0, 1):  # default and single-round work items
@@ -89,8 +92,8 @@ def test_bucketed_scaled_workload(hbt, layout, F, items, cap, leaf256):
 
 
 @pytest.mark.parametrize("layout", ["implicit", "regular"])
-@pytest.mark.parametrize("items,cap,leaf256", ITEM_MODES)
-def test_bucketed_after_update(hbt, layout, items, cap, leaf256):
+@pytest.mark.parametrize("items,cap,leaf256,dir32", ITEM_MODES)
+def test_bucketed_after_update(hbt, layout, items, cap, leaf256, dir32):
     """The splitters follow the tree: search, update (keys move between buckets,
     regular leaves split / empty), search again."""
     width, F = 8, 8
@@ -103,6 +106,7 @@ def test_bucketed_after_update(hbt, layout, items, cap, leaf256):
     t.set_param("bucket_items", items)
     t.set_param("bucket_cap", cap)
     t.set_param("leaf256", leaf256)
+    t.set_param("item_dir32", dir32)
     t.set_param("bucket_slice", 2048)
     q = query_set(k, width, rng, 4000)
     pf, val = gpu_search(t, q, width)
@@ -121,6 +125,33 @@ def test_bucketed_after_update(hbt, layout, items, cap, leaf256):
         epf, ev = o.search(q)
         assert np.array_equal(pf, epf) and np.array_equal(val, ev), (layout, trial)
     t.close()
+
+
+@pytest.mark.parametrize("slice_bytes", [1 << 20, 4096, 1])
+def test_compressed_directory_ties(hbt, slice_bytes):
+    """Compressed per-bucket directory (item_dir32) where 32-bit truncation ties: dense
+    small keys share a bucket with keys near 2^63, so the bucket's shift is ~31 and
+    every small maximum truncates to the same value; the tied entries are resolved
+    against the exact maxima.  Also u32 keys (shift 0) and a bucket of one unit."""
+    rng = np.random.default_rng(31)
+    small = np.arange(0, 60000, 3, dtype=np.uint64)
+    big = (np.uint64(1) << np.uint64(63)) + rng.integers(0, 1 << 40, 300, dtype=np.uint64)
+    for width, k in ((8, np.concatenate([small, big])), (4, small)):
+        v = rng.integers(0, kmax(width), len(k), dtype=np.uint64, endpoint=True)
+        o = oracle.ITree.from_pairs(k, v, 16, width)
+        t = gpu_build(hbt, k, v, 16, width)
+        q = np.concatenate([query_set(k, width, rng, 6000), k[::7], k[::11] + np.uint64(1), k[::13] - np.uint64(1)])
+        q = np.concatenate([q, np.array([0, kmax(width)], dtype=np.uint64)]) & np.uint64(kmax(width))
+        epf, ev = o.search(q)
+        t.set_param("bucket", 1)
+        t.set_param("item_dir32", 2)
+        t.set_param("bucket_slice", slice_bytes)
+        for rounds in (0, 1):
+            t.set_param("item_rounds", rounds)
+            pf, val = gpu_search(t, q, width)
+            assert np.array_equal(pf, epf), (width, slice_bytes, np.nonzero(pf != epf)[0][:5])
+            assert np.array_equal(val, ev), (width, slice_bytes)
+        t.close()
 
 
 @pytest.mark.parametrize("chunk_log2,bufs", [(22, 2), (20, 2), (20, 3), (14, 4)])
