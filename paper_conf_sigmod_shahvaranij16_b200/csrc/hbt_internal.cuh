@@ -120,6 +120,7 @@ struct ItemDir {
   // inside one bucket each (item search).
   const struct BucketDir32* bd = nullptr;
   const uint32_t* M32 = nullptr;
+  bool fix = false;  // ties of the truncated maxima resolved by the walk (implicit_search.cu)
 };
 
 // One bucket of the compressed item directory (ItemDir::bd).

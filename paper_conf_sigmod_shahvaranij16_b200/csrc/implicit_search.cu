@@ -140,14 +140,19 @@ __device__ __forceinline__ uint32_t count_less16(const V16<K>& v, K q, unsigned 
 // Phase 2 of a warp round: levels [d0, H) by lane groups, the leaf line, and the
 // results of the round (slot j of group g = round query j*NG + g, stored at
 // base + j*NG + g).
-template <typename K, int F, int QPG, bool REC = false>
+// FIX (compressed item directory): the directory may place a query ONE OR MORE units
+// early at level d0 (a tie of truncated maxima, implicit_search_items32_kernel).  A
+// unit u before the right one has max M_u < q, and its last separator IS M_u (a real,
+// full node / leaf line), so the search of unit u counts every entry below q; then the
+// query moves on to unit u + 1 (at most up to fix_last) and searches again.
+template <typename K, int F, int QPG, bool REC = false, bool FIX = false>
 __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ inner,
                                                   const uint8_t* __restrict__ inner_idx,
                                                   const uint8_t* __restrict__ leaf, const LevelTable& lt,
                                                   uint32_t d0, K (&q)[QPG], uint32_t (&node)[QPG], int g, int k,
                                                   unsigned gmask, uint64_t base, uint64_t m, uint64_t n,
                                                   uint64_t pos_base, uint64_t* __restrict__ out_pf,
-                                                  K* __restrict__ out_v) {
+                                                  K* __restrict__ out_v, uint32_t fix_last = 0) {
   using C = Cfg<K, F>;
   const uint32_t H = lt.H;
   for (uint32_t d = d0; d < H; ++d) {
@@ -163,22 +168,16 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
             // the pipe that binds the item search, profiles/r01_c4_items_*) of 16 B loads
             constexpr int NC32 = C::NODE_BYTES / C::G / 32;
             L256<K> fw[QPG][NC32];
-            if (lt.l2_hint & 2u) {
-              const uint64_t pol = policy_evict_last();
+            const uint64_t pol = policy_evict_last();
+            auto load = [&](int j) {
 #pragma unroll
-              for (int j = 0; j < QPG; ++j)
-#pragma unroll
-                for (int h = 0; h < NC32; ++h)
-                  ld32_pol(fw[j][h], lvl + uint64_t(node[j]) * C::NODE_BYTES + (k * NC32 + h) * 32, pol);
-            } else {
-#pragma unroll
-              for (int j = 0; j < QPG; ++j)
-#pragma unroll
-                for (int h = 0; h < NC32; ++h)
-                  ld32(fw[j][h], lvl + uint64_t(node[j]) * C::NODE_BYTES + (k * NC32 + h) * 32);
-            }
-#pragma unroll
-            for (int j = 0; j < QPG; ++j) {
+              for (int h = 0; h < NC32; ++h) {
+                const uint8_t* p = lvl + uint64_t(node[j]) * C::NODE_BYTES + (k * NC32 + h) * 32;
+                if (lt.l2_hint & 2u) ld32_pol(fw[j][h], p, pol);
+                else ld32(fw[j][h], p);
+              }
+            };
+            auto count = [&](int j) {
               uint32_t c = 0;
 #pragma unroll
               for (int h = 0; h < NC32; ++h)
@@ -186,8 +185,40 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
                 for (int e = 0; e < 32 / C::S; ++e) c += (fw[j][h].k[e] < q[j]) ? 1u : 0u;
 #pragma unroll
               for (int x = 1; x < C::G; x <<= 1) c += __shfl_xor_sync(0xffffffffu, c, x);
-              node[j] = node[j] * F + c;
+              return c;
+            };
+#pragma unroll
+            for (int j = 0; j < QPG; ++j) load(j);
+            uint32_t c[QPG];
+#pragma unroll
+            for (int j = 0; j < QPG; ++j) c[j] = count(j);
+            if constexpr (FIX) {
+              if (d == d0) {
+                uint32_t adv = 0;
+#pragma unroll
+                for (int j = 0; j < QPG; ++j) adv |= (c[j] == uint32_t(F) && node[j] < fix_last) ? 1u << j : 0u;
+                while (__any_sync(0xffffffffu, adv != 0)) {
+#pragma unroll
+                  for (int j = 0; j < QPG; ++j)
+                    if ((adv >> j) & 1u) {
+                      ++node[j];
+                      load(j);
+                    }
+                  uint32_t nadv = 0;
+#pragma unroll
+                  for (int j = 0; j < QPG; ++j) {
+                    const uint32_t cc = count(j);  // every lane shuffles; only advanced slots keep it
+                    if ((adv >> j) & 1u) {
+                      c[j] = cc;
+                      nadv |= (cc == uint32_t(F) && node[j] < fix_last) ? 1u << j : 0u;
+                    }
+                  }
+                  adv = nadv;
+                }
+              }
             }
+#pragma unroll
+            for (int j = 0; j < QPG; ++j) node[j] = node[j] * F + c[j];
             continue;
           }
         }
@@ -243,26 +274,55 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
     //      the key sector, lane 1 the value sector with 256-bit loads (sm_100).
     //      s = #{keys < q} on lane 0, broadcast; key / value picked by lanes 0 / 1.
     L256<K> lw[QPG];
-    if (lt.l2_hint & 1u) {
-      const uint64_t pol = policy_evict_first();
-#pragma unroll
-      for (int j = 0; j < QPG; ++j) {
-        if (k < 2) ld32_pol(lw[j], leaf + uint64_t(node[j]) * 64 + k * 32, pol);
-        else fill_max32(lw[j]);
+    const uint64_t pol = policy_evict_first();
+    auto load = [&](int j) {
+      if (k < 2) {
+        const uint8_t* p = leaf + uint64_t(node[j]) * 64 + k * 32;
+        if (lt.l2_hint & 1u) ld32_pol(lw[j], p, pol);
+        else ld32(lw[j], p);
+      } else {
+        fill_max32(lw[j]);
       }
-    } else {
+    };
+    auto count = [&](int j) {
+      uint32_t c = 0;
 #pragma unroll
-      for (int j = 0; j < QPG; ++j) {
-        if (k < 2) ld32(lw[j], leaf + uint64_t(node[j]) * 64 + k * 32);
-        else fill_max32(lw[j]);
+      for (int e = 0; e < C::P; ++e) c += (lw[j].k[e] < q[j]) ? 1u : 0u;
+      return __shfl_sync(0xffffffffu, c, g * C::G);
+    };
+#pragma unroll
+    for (int j = 0; j < QPG; ++j) load(j);
+    uint32_t sl[QPG];
+#pragma unroll
+    for (int j = 0; j < QPG; ++j) sl[j] = count(j);
+    if constexpr (FIX) {
+      if (d0 == H) {  // the directory named a leaf line directly (see above)
+        uint32_t adv = 0;
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) adv |= (sl[j] == uint32_t(C::P) && node[j] < fix_last) ? 1u << j : 0u;
+        while (__any_sync(0xffffffffu, adv != 0)) {
+#pragma unroll
+          for (int j = 0; j < QPG; ++j)
+            if ((adv >> j) & 1u) {
+              ++node[j];
+              load(j);
+            }
+          uint32_t nadv = 0;
+#pragma unroll
+          for (int j = 0; j < QPG; ++j) {
+            const uint32_t cc = count(j);
+            if ((adv >> j) & 1u) {
+              sl[j] = cc;
+              nadv |= (cc == uint32_t(C::P) && node[j] < fix_last) ? 1u << j : 0u;
+            }
+          }
+          adv = nadv;
+        }
       }
     }
 #pragma unroll
     for (int j = 0; j < QPG; ++j) {
-      uint32_t c = 0;
-#pragma unroll
-      for (int e = 0; e < C::P; ++e) c += (lw[j].k[e] < q[j]) ? 1u : 0u;
-      const uint32_t s = __shfl_sync(0xffffffffu, c, g * C::G);
+      const uint32_t s = sl[j];
       const uint32_t sc = s < uint32_t(C::P) ? s : uint32_t(C::P - 1);
       const K x = pick(lw[j].k, sc);
       const K key_s = __shfl_sync(0xffffffffu, x, g * C::G);
@@ -529,7 +589,7 @@ __device__ __forceinline__ uint32_t lower_bound32(const uint32_t* s_M, uint32_t 
   if (dq > K(pt.span)) return cnt;  // beyond the bucket's last maximum (pt.lo = s_M[0] = 0)
   const uint32_t q32 = uint32_t(dq);
   uint32_t a = prefix_lower_bound(s_M, cnt, s_T, pt, q32);
-  if (sh)
+  if (sh && gM)
     while (a < cnt && s_M[a] == q32 && __ldg(gM + a) < q) ++a;
   return a;
 }
@@ -619,7 +679,9 @@ implicit_search_items32_kernel(const uint8_t* __restrict__ inner, const uint8_t*
         const uint64_t i = base + (THREADS / 32) * 32 + lane;
         nextq = (r + 1 < int(d.rounds) && i <= p1) ? ldcs(queries + i) : key_max<K>();
       }
-      const uint32_t a = lower_bound32(s_M, cnt, s_T, pt, myq, blo, sh, gM + u0);
+      // fixable first level: ties are resolved by the walk (descend_and_store FIX), not
+      // by a dependent read of the exact maxima that would stall the whole warp
+      const uint32_t a = lower_bound32(s_M, cnt, s_T, pt, myq, blo, sh, d.fix ? nullptr : gM + u0);
       const uint32_t mynode = uint32_t(u0) + (a < cnt ? a : cnt - 1);
       K q[QPG];
       uint32_t node[QPG];
@@ -629,8 +691,9 @@ implicit_search_items32_kernel(const uint8_t* __restrict__ inner, const uint8_t*
         q[j] = __shfl_sync(0xffffffffu, myq, src);
         node[j] = __shfl_sync(0xffffffffu, mynode, src);
       }
-      descend_and_store<K, F, QPG, true>(inner, inner_idx, leaf, lt, d.level, q, node, g, k, gmask, base, p1 + 1, n,
-                                         d.pos_base, out_pf, out_v);
+      descend_and_store<K, F, QPG, true, true>(inner, inner_idx, leaf, lt, d.level, q, node, g, k, gmask, base,
+                                               p1 + 1, n, d.pos_base, out_pf, out_v,
+                                               d.fix ? uint32_t(u0) + cnt - 1 : 0u);
     }
     __syncthreads();
   }
@@ -753,6 +816,11 @@ struct Launch {
     }
     ItemDir dd = d;
     dd.rounds = item_rounds(m, t->num_sms, TH, t->cfg.item_rounds ? t->cfg.item_rounds : 16);
+    // the walk can resolve directory ties where the first level is read whole (256-bit
+    // node loads or the 256-bit leaf line)
+    dd.fix = d.level == t->H ? lt.leaf256 != 0
+                             : (((lt.full_mask >> d.level) & 1u) && lt.full256 && C::HAS_IDX &&
+                                C::NODE_BYTES / C::G >= 32);
     const size_t smem = size_t(d.cap) * 4 + (size_t(d.B) + 1) * 8 + ((1u << kPrefixBits32) + 1) * 4 +
                         (size_t(d.B) + 1) * 4;
     kern<<<t->num_sms, TH, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
@@ -767,7 +835,8 @@ struct Launch {
     // batch spreads over every SM (c1: 10.1 -> 8.3 us per batch)
     if (t->cfg.mode == 3 || (t->cfg.mode == 2 && m <= t->cfg.small_batch)) return run_t<256, 3>(t, q, m, pf, v, b, s, lp);
     // 256-byte nodes (u64, F = 32) need more registers than a 1024-thread CTA allows
-    return C::NODE_BYTES > 128 ? run_t<512, 2>(t, q, m, pf, v, b, s, lp) : run_t<1024, 2>(t, q, m, pf, v, b, s, lp);
+    if constexpr (C::NODE_BYTES > 128) return run_t<512, 2>(t, q, m, pf, v, b, s, lp);
+    else return run_t<1024, 2>(t, q, m, pf, v, b, s, lp);
   }
 };
 

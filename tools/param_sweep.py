@@ -24,6 +24,7 @@ def main():
     ap.add_argument("--set", action="append", default=[])
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--m", type=int, default=0)
+    ap.add_argument("--sorted", action="store_true", help="sort the batch first (locality experiments)")
     a = ap.parse_args()
     c = gen.CONFIGS[a.config]
     g = GenLib()
@@ -39,6 +40,8 @@ def main():
     else:
         keys, vals = g.mix_stream(n, w, sk), g.mix_stream(n, w, sv)
         q = g.uniform_queries(m, n, w, sq, sk)
+    if a.sorted:
+        q = (q.view(torch.int64) ^ (1 << 63)).sort().values.__xor__(1 << 63).view(q.dtype)  # unsigned order
     tree = hbt.Tree(keys, vals, fanout=c["fanout"], layout=c["layout"])
     del keys, vals
     torch.cuda.empty_cache()
