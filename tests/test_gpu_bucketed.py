@@ -127,14 +127,17 @@ def test_bucketed_after_update(hbt, layout, items, cap, leaf256, dir32):
     t.close()
 
 
-@pytest.mark.parametrize("slice_bytes", [1 << 20, 4096, 1])
-def test_compressed_directory_ties(hbt, slice_bytes):
+@pytest.mark.parametrize("nsmall,slice_bytes", [(20000, 1 << 20), (20000, 4096), (20000, 1), (400000, 1 << 30)])
+def test_compressed_directory_ties(hbt, nsmall, slice_bytes):
     """Compressed per-bucket directory (item_dir32) where 32-bit truncation ties: dense
     small keys share a bucket with keys near 2^63, so the bucket's shift is ~31 and
-    every small maximum truncates to the same value; the tied entries are resolved
-    against the exact maxima.  Also u32 keys (shift 0) and a bucket of one unit."""
+    every small maximum truncates to the same value.  Ties are resolved by the walk
+    (256-bit whole-node / leaf reads at the directory level) or against the exact
+    maxima (16 B reads, index + sector levels).  The 400 K-key tree in one bucket puts
+    the directory on the last inner level (whole nodes with l2_levels_bytes = 4096);
+    the others on the leaf lines.  Also u32 keys (shift 0)."""
     rng = np.random.default_rng(31)
-    small = np.arange(0, 60000, 3, dtype=np.uint64)
+    small = np.arange(0, 3 * nsmall, 3, dtype=np.uint64)
     big = (np.uint64(1) << np.uint64(63)) + rng.integers(0, 1 << 40, 300, dtype=np.uint64)
     for width, k in ((8, np.concatenate([small, big])), (4, small)):
         v = rng.integers(0, kmax(width), len(k), dtype=np.uint64, endpoint=True)
@@ -146,11 +149,16 @@ def test_compressed_directory_ties(hbt, slice_bytes):
         t.set_param("bucket", 1)
         t.set_param("item_dir32", 2)
         t.set_param("bucket_slice", slice_bytes)
-        for rounds in (0, 1):
+        for rounds, leaf256, full256, l2b in ((0, 1, 1, 0), (0, 1, 1, 4096), (1, 1, 1, 4096), (0, 0, 1, 0),
+                                              (0, 1, 0, 4096), (1, 0, 0, 0)):
             t.set_param("item_rounds", rounds)
+            t.set_param("leaf256", leaf256)
+            t.set_param("full256", full256)
+            t.set_param("l2_levels_bytes", l2b)
             pf, val = gpu_search(t, q, width)
-            assert np.array_equal(pf, epf), (width, slice_bytes, np.nonzero(pf != epf)[0][:5])
-            assert np.array_equal(val, ev), (width, slice_bytes)
+            cfg = (width, slice_bytes, rounds, leaf256, full256, l2b)
+            assert np.array_equal(pf, epf), (cfg, np.nonzero(pf != epf)[0][:5])
+            assert np.array_equal(val, ev), cfg
         t.close()
 
 
