@@ -140,11 +140,14 @@ __device__ __forceinline__ uint32_t count_less16(const V16<K>& v, K q, unsigned 
 // Phase 2 of a warp round: levels [d0, H) by lane groups, the leaf line, and the
 // results of the round (slot j of group g = round query j*NG + g, stored at
 // base + j*NG + g).
-// FIX (compressed item directory): the directory may place a query ONE OR MORE units
-// early at level d0 (a tie of truncated maxima, implicit_search_items32_kernel).  A
-// unit u before the right one has max M_u < q, and its last separator IS M_u (a real,
-// full node / leaf line), so the search of unit u counts every entry below q; then the
-// query moves on to unit u + 1 (at most up to fix_last) and searches again.
+// FIX (compressed item directory, implicit_search_items32_kernel): the directory may
+// place a query ONE unit early (a tie of truncated maxima; runs of ties are settled
+// before the walk).  Every real separator of that unit u is < q and its last key slot
+// is MAX (reading R3), so the walk takes the last child at every level and ends
+// on the LAST leaf line of u's subtree with s = P, which cannot happen on the right
+// unit.  The lower bound then lies in the following lines (u + 1's first lines, in
+// key order): the slot reads line + 1, ... until s < P, at most up to line fix_last
+// (the bucket's last real line).  For hits on ties (c4) that is one extra line.
 template <typename K, int F, int QPG, bool REC = false, bool FIX = false>
 __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ inner,
                                                   const uint8_t* __restrict__ inner_idx,
@@ -192,31 +195,6 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
             uint32_t c[QPG];
 #pragma unroll
             for (int j = 0; j < QPG; ++j) c[j] = count(j);
-            if constexpr (FIX) {
-              if (d == d0) {
-                uint32_t adv = 0;
-#pragma unroll
-                for (int j = 0; j < QPG; ++j) adv |= (c[j] == uint32_t(F) && node[j] < fix_last) ? 1u << j : 0u;
-                while (__any_sync(0xffffffffu, adv != 0)) {
-#pragma unroll
-                  for (int j = 0; j < QPG; ++j)
-                    if ((adv >> j) & 1u) {
-                      ++node[j];
-                      load(j);
-                    }
-                  uint32_t nadv = 0;
-#pragma unroll
-                  for (int j = 0; j < QPG; ++j) {
-                    const uint32_t cc = count(j);  // every lane shuffles; only advanced slots keep it
-                    if ((adv >> j) & 1u) {
-                      c[j] = cc;
-                      nadv |= (cc == uint32_t(F) && node[j] < fix_last) ? 1u << j : 0u;
-                    }
-                  }
-                  adv = nadv;
-                }
-              }
-            }
 #pragma unroll
             for (int j = 0; j < QPG; ++j) node[j] = node[j] * F + c[j];
             continue;
@@ -296,7 +274,7 @@ __device__ __forceinline__ void descend_and_store(const uint8_t* __restrict__ in
 #pragma unroll
     for (int j = 0; j < QPG; ++j) sl[j] = count(j);
     if constexpr (FIX) {
-      if (d0 == H) {  // the directory named a leaf line directly (see above)
+      {
         uint32_t adv = 0;
 #pragma unroll
         for (int j = 0; j < QPG; ++j) adv |= (sl[j] == uint32_t(C::P) && node[j] < fix_last) ? 1u << j : 0u;
@@ -583,14 +561,19 @@ constexpr uint32_t kPrefixBits32 = 12;
 template <typename K>
 __device__ __forceinline__ uint32_t lower_bound32(const uint32_t* s_M, uint32_t cnt, const uint32_t* s_T,
                                                   const PrefixTab<uint32_t>& pt, K q, K lo, uint32_t sh,
-                                                  const K* __restrict__ gM) {
+                                                  const K* __restrict__ gM, bool fixable) {
   if (q <= lo) return 0;
   const K dq = K(q - lo) >> sh;
   if (dq > K(pt.span)) return cnt;  // beyond the bucket's last maximum (pt.lo = s_M[0] = 0)
   const uint32_t q32 = uint32_t(dq);
   uint32_t a = prefix_lower_bound(s_M, cnt, s_T, pt, q32);
-  if (sh && gM)
+  // A tie with ONE truncated maximum leaves a or a + 1, which the walk settles (FIX, when
+  // fixable); a RUN of ties (or no FIX) is settled here against the exact maxima gM, so
+  // the walk never moves on by more than one unit.
+  if (sh && a < cnt && s_M[a] == q32) {
+    if (fixable && (a + 1 >= cnt || s_M[a + 1] != q32)) return a;
     while (a < cnt && s_M[a] == q32 && __ldg(gM + a) < q) ++a;
+  }
   return a;
 }
 
@@ -679,9 +662,9 @@ implicit_search_items32_kernel(const uint8_t* __restrict__ inner, const uint8_t*
         const uint64_t i = base + (THREADS / 32) * 32 + lane;
         nextq = (r + 1 < int(d.rounds) && i <= p1) ? ldcs(queries + i) : key_max<K>();
       }
-      // fixable first level: ties are resolved by the walk (descend_and_store FIX), not
-      // by a dependent read of the exact maxima that would stall the whole warp
-      const uint32_t a = lower_bound32(s_M, cnt, s_T, pt, myq, blo, sh, d.fix ? nullptr : gM + u0);
+      // single ties are resolved by the walk (descend_and_store FIX), not by a dependent
+      // read of the exact maxima that would stall the whole warp
+      const uint32_t a = lower_bound32(s_M, cnt, s_T, pt, myq, blo, sh, gM + u0, d.fix);
       const uint32_t mynode = uint32_t(u0) + (a < cnt ? a : cnt - 1);
       K q[QPG];
       uint32_t node[QPG];
@@ -693,7 +676,7 @@ implicit_search_items32_kernel(const uint8_t* __restrict__ inner, const uint8_t*
       }
       descend_and_store<K, F, QPG, true, true>(inner, inner_idx, leaf, lt, d.level, q, node, g, k, gmask, base,
                                                p1 + 1, n, d.pos_base, out_pf, out_v,
-                                               d.fix ? uint32_t(u0) + cnt - 1 : 0u);
+                                               d.fix ? uint32_t(min((u0 + cnt) * d.span, d.U) - 1) : 0u);
     }
     __syncthreads();
   }
@@ -816,11 +799,8 @@ struct Launch {
     }
     ItemDir dd = d;
     dd.rounds = item_rounds(m, t->num_sms, TH, t->cfg.item_rounds ? t->cfg.item_rounds : 16);
-    // the walk can resolve directory ties where the first level is read whole (256-bit
-    // node loads or the 256-bit leaf line)
-    dd.fix = d.level == t->H ? lt.leaf256 != 0
-                             : (((lt.full_mask >> d.level) & 1u) && lt.full256 && C::HAS_IDX &&
-                                C::NODE_BYTES / C::G >= 32);
+    // the walk resolves directory ties (it detects them on the 256-bit leaf read)
+    dd.fix = lt.leaf256 != 0;
     const size_t smem = size_t(d.cap) * 4 + (size_t(d.B) + 1) * 8 + ((1u << kPrefixBits32) + 1) * 4 +
                         (size_t(d.B) + 1) * 4;
     kern<<<t->num_sms, TH, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
