@@ -129,3 +129,34 @@ def test_c4_sample_vs_oracle_slice(c4):
     exp = (epf & ~FOUND) + np.uint64(s0) | (epf & FOUND)
     assert np.array_equal(got_pf, exp)
     assert np.array_equal(got_v, ev)
+
+
+@pytest.mark.parametrize("slice_bytes", [20_000_000, 0])
+def test_c4_recipe_last_inner_level_directory_ties(slice_bytes):
+    """The c4 recipe at 2^26 keys / 2^24 queries with ~63 buckets (bucket_slice 20 MB):
+    the compressed item directory sits on the LAST INNER level, and hits on the first
+    key of a node whose predecessor's max lies within 2^26 below tie in the directory
+    (regression: the walk must move on to the next lines).  Every output vs the
+    stratified closed form; the default slice as a control."""
+    import paper_conf_sigmod_shahvaranij16_b200 as hbt
+    c = gen.CONFIGS["c4"]
+    n, m = 1 << 26, 1 << 24
+    sk = gen.stream_seed(c["cfg"], gen.STREAM_K)
+    sv = gen.stream_seed(c["cfg"], gen.STREAM_V)
+    sq = gen.stream_seed(c["cfg"], gen.STREAM_Q)
+    g = GenLib()
+    t = hbt.Tree(g.stratified_keys(n, sk), g.mix_stream(n, 8, sv), fanout=16)
+    t.set_param("bucket", 1)
+    t.set_param("bucket_slice", slice_bytes)
+    dq = g.stratified_queries(m, n, sq, sk)
+    # hits, plus misses just above each hit (lower bound = next key)
+    q = torch.cat([dq, dq + 1])
+    pf, val = t.search(q)
+    torch.cuda.synchronize()
+    qh = q.cpu().numpy().view(np.uint64)
+    epf, ev = closed_form(qh, n, sk, sv)
+    got = pf.cpu().numpy().view(np.uint64)
+    bad = np.nonzero(got != epf)[0]
+    assert bad.size == 0, (bad.size, qh[bad[:4]], got[bad[:4]], epf[bad[:4]])
+    assert np.array_equal(from_dev(val, 8), ev)
+    t.close()
