@@ -640,6 +640,9 @@ def run_hbt(args):
     if os.path.exists(tp) and not (args.config == "c4" and world > 1):  # measured on one GPU
         traffic = json.load(open(tp)).get(args.config)
     traffic_bytes = traffic.get("dram_bytes_per_launch") if isinstance(traffic, dict) and not args.range_k else None
+    if traffic_bytes and traffic.get("kernel") and not args.range_k:
+        # the dominant kernel's name as ncu reported it in the traffic capture
+        kernel = traffic["kernel"].split("::")[-1].split("<")[0]
     hbm_ach = mdl["hbm_bytes_per_query"] * m / t_kernel / 1e9
     roof_hbm = {"bound": "hbm", "achieved": round(hbm_ach, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(hbm_ach / peak, 4), "traffic": traffic_bytes,
