@@ -236,9 +236,10 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *                 the L2 -- measured c2 0.426 -> 0.415 ms, c5 Zipf 2.84 -> 3.00 ms with it on)
  *   "item_l2_hint" the same bits for the implicit bucketed item search (default 1: c4 item
  *                 search 10.96 -> 9.50 ms, DRAM reads 171 -> 148 B/query)
- *   "item_dir32"  implicit item directory in its compressed per-bucket form (32-bit offsets
- *                 of each bucket's unit maxima, items cut inside one bucket): 0 = never,
- *                 1 = where it reaches a deeper tree level than 8 B keys (default), 2 = always
+ *   "item_cdir"   item directory in its compressed per-bucket form (16-bit entries under a
+ *                 per-bucket prefix table, items cut inside one bucket; regular trees: the
+ *                 leaf lines): 0 = never, 1 = where it reaches a deeper tree level than 8 B
+ *                 keys and fits (default), 2 = always where it fits
  * Variants measured slower were removed (DESIGN.md §8 keeps their numbers).  Unknown
  * names or out-of-range values return HBT_EINVAL. */
 HBT_API int hbt_set_param(hbt_tree* t, const char* name, int64_t value);

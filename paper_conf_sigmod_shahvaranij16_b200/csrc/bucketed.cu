@@ -110,32 +110,58 @@ __global__ void bk_level_max(const uint8_t* __restrict__ leaf, uint64_t n, uint3
   }
 }
 
-// Compressed item directory (ItemDir::bd): one CTA per bucket derives the offset
-// origin lo = M[u0] and the shift that fits M[u0 + cnt - 1] - lo in 32 bits, then
-// writes M32[off + i] = (M[u0 + i] - lo) >> sh (padding to 4 entries: ~0).
+// Compressed item directory (ItemDir::bd): one CTA per bucket derives the offset origin
+// lo = M[u0], the shift sh that fits M[u0 + cnt - 1] - lo in 32 bits (M' = (M - lo) >> sh),
+// the prefix-table slice shift ssh (2^12 slices over [0, top]) and the entry shift esh,
+// then writes the 16-bit entries E16 = (M' >> esh) & 0xFFFF (padding to 8 entries: ~0) and
+// the prefix table T16[p] = #{M' < p << ssh}, p in [0, 2^12] (padded with cnt).
 template <typename K>
-__global__ void bk_dir32(const K* __restrict__ M, BucketDir32* __restrict__ bd, uint32_t* __restrict__ M32) {
+__global__ void bk_cdir(const K* __restrict__ M, BucketDir* __restrict__ bd, uint16_t* __restrict__ E16,
+                        uint16_t* __restrict__ T16) {
   __shared__ K s_lo;
-  __shared__ uint32_t s_sh;
-  BucketDir32* d = bd + blockIdx.x;
-  const uint64_t u0 = d->u0, off = d->off;
+  __shared__ uint32_t s_sh[3];
+  BucketDir* d = bd + blockIdx.x;
+  const uint64_t u0 = d->u0, off16 = d->off16;
   const uint32_t cnt = d->cnt;
   if (threadIdx.x == 0) {
     const K lo = M[u0], span = K(M[u0 + cnt - 1] - lo);
     const uint32_t bits = span ? uint32_t(8 * sizeof(K)) - uint32_t(sizeof(K) == 8 ? __clzll((long long)span)
                                                                                  : __clz(int(span)))
                                : 0u;
+    const uint32_t sh = bits > 32 ? bits - 32 : 0u;
+    const uint32_t top = uint32_t(span >> sh);
+    const uint32_t tb = top ? 32u - uint32_t(__clz(int(top))) : 0u;
+    const uint32_t ssh = tb > 12 ? tb - 12 : 0u;
     s_lo = lo;
-    s_sh = bits > 32 ? bits - 32 : 0u;
+    s_sh[0] = sh;
+    s_sh[1] = ssh;
+    s_sh[2] = ssh > 16 ? ssh - 16 : 0u;
     d->lo = uint64_t(lo);
-    d->sh = s_sh;
+    d->sh = sh;
+    d->top = top;
+    d->ssh = ssh;
+    d->esh = s_sh[2];
   }
   __syncthreads();
   const K lo = s_lo;
-  const uint32_t sh = s_sh;
-  const uint32_t padded = (cnt + 3u) & ~3u;
-  for (uint32_t i = threadIdx.x; i < padded; i += blockDim.x)
-    M32[off + i] = i < cnt ? uint32_t(K(M[u0 + i] - lo) >> sh) : ~0u;
+  const uint32_t sh = s_sh[0], ssh = s_sh[1], esh = s_sh[2];
+  auto mp = [&](uint32_t i) { return uint32_t(K(M[u0 + i] - lo) >> sh); };
+  const uint32_t padded = (cnt + 7u) & ~7u;
+  for (uint32_t i = threadIdx.x; i < padded; i += blockDim.x) E16[off16 + i] = i < cnt ? uint16_t(mp(i) >> esh) : 0xFFFFu;
+  for (uint32_t p = threadIdx.x; p < kT16; p += blockDim.x) {
+    uint32_t a = 0;
+    if (p > 4096u) {
+      a = cnt;
+    } else {
+      const uint64_t key = uint64_t(p) << ssh;  // lower bound of key over M'
+      uint32_t len = cnt;
+      while (len > 0) {
+        const uint32_t half = len >> 1;
+        if (uint64_t(mp(a + half)) < key) { a += half + 1; len -= half + 1; } else { len = half; }
+      }
+    }
+    T16[uint64_t(blockIdx.x) * kT16 + p] = uint16_t(a);
+  }
 }
 
 // Item directory (regular): M[c * NI + t] = true max key of key line t of the
@@ -733,10 +759,15 @@ static inline void bucket_units(uint64_t U, uint32_t B, uint32_t b, uint64_t spa
   u1 = (((uint64_t(b) + 1) * U) / B - 1) / span;
 }
 
-// Shared-memory entries of the compressed directory: ~200 KB per CTA beside the
-// bucket starts, item starts and the 2^12-entry prefix table.
-uint64_t item_cap32(uint32_t B) {
-  return (200 * 1024 - (uint64_t(B) + 1) * 12 - ((1u << 12) + 1) * 4 - 64) / 4;
+// Entries of the compressed directory per bucket: below 2^16 (16-bit prefix table) and
+// within ~160 KB of shared memory per CTA together with the prefix table, the bucket
+// and item starts (and, regular trees, one chain id per F entries), so the L1 keeps
+// >= 92 KB for the loads in flight (a 200 KB directory measured 30 % slower on c3).
+uint64_t item_cap16(uint32_t B, uint32_t per_chain) {
+  const uint64_t fixed = uint64_t(kT16) * 2 + (uint64_t(B) + 1) * 12 + 64 + (per_chain ? 32 : 0);
+  const uint64_t per = per_chain ? 2 * uint64_t(per_chain) + 4 : 2 * uint64_t(1);  // bytes per `per_chain` entries
+  const uint64_t room = (160 * 1024 - fixed) * (per_chain ? per_chain : 1) / per;
+  return std::min<uint64_t>(room, 65528);
 }
 
 // Shared-memory entries of the item directory (keys; the regular tree also
@@ -779,7 +810,7 @@ int prepare_splitters(const hbt_tree* t, cudaStream_t s, BucketState& bs, uint32
   if (want_items && t->cfg.bucket_items) {
     const uint64_t cap = item_cap(t, B);
     uint64_t nunits = 0;
-    bs.d32 = false;
+    bs.cdir = false;
     if (t->form == HBT_IMPLICIT) {
       uint64_t span = 1;
       for (int d = int(t->H); d >= 0; --d) {
@@ -794,8 +825,8 @@ int prepare_splitters(const hbt_tree* t, cudaStream_t s, BucketState& bs, uint32
         span *= t->F;
       }
       // the compressed per-bucket form, where it reaches a deeper level (or when forced)
-      if (t->cfg.item_dir32 && !t->cfg.bucket_cap) {
-        const uint64_t cap32 = item_cap32(B);
+      if (t->cfg.item_cdir && !t->cfg.bucket_cap) {
+        const uint64_t cap16 = item_cap16(B, 0);
         uint64_t span32 = 1;
         for (int d = int(t->H); d >= 0; --d) {
           uint64_t most = 0;
@@ -804,14 +835,14 @@ int prepare_splitters(const hbt_tree* t, cudaStream_t s, BucketState& bs, uint32
             bucket_units(t->L0, B, b, span32, u0, u1);
             most = std::max<uint64_t>(most, u1 - u0 + 1);
           }
-          if (most <= cap32) {
-            if (!bs.items || d > int(bs.level) || t->cfg.item_dir32 == 2) {
+          if (most <= cap16) {
+            if (!bs.items || d > int(bs.level) || t->cfg.item_cdir == 2) {
               bs.level = uint32_t(d);
               bs.span = span32;
               nunits = d == int(t->H) ? t->L0 : t->nodes[d];
               bs.items = true;
-              bs.d32 = true;
-              bs.cap32 = uint32_t((most + 3) & ~uint64_t(3));
+              bs.cdir = true;
+              bs.cap16 = uint32_t((most + 7) & ~uint64_t(7));
             }
             break;
           }
@@ -825,6 +856,23 @@ int prepare_splitters(const hbt_tree* t, cudaStream_t s, BucketState& bs, uint32
         bs.span = NI;
         nunits = t->r.nchain * NI;
         bs.items = true;
+      }
+      // the compressed per-bucket form on the LEAF LINES (F per chain leaf): the search
+      // goes from the directory straight to the leaf line (regular_search_items32_kernel)
+      if (t->cfg.item_cdir && !t->cfg.bucket_cap) {
+        uint64_t most = 0;
+        for (uint32_t b = 0; b < B; ++b) {
+          uint64_t c0, c1;
+          bucket_units(t->r.nchain, B, b, 1, c0, c1);
+          most = std::max<uint64_t>(most, (c1 - c0 + 1) * t->F);
+        }
+        if (most + 8 <= item_cap16(B, t->F)) {
+          bs.span = t->F;
+          nunits = t->r.nchain * t->F;
+          bs.items = true;
+          bs.cdir = true;
+          bs.cap16 = uint32_t((most + 7) & ~uint64_t(7));
+        }
       }
     }
     if (bs.items) {
@@ -840,31 +888,39 @@ int prepare_splitters(const hbt_tree* t, cudaStream_t s, BucketState& bs, uint32
       if (t->form == HBT_IMPLICIT)
         bk_level_max<K><<<t->num_sms * 4, 256, 0, s>>>((const uint8_t*)t->d_leaf, t->n, t->P, bs.span, nunits,
                                                         (K*)bs.d_M);
-      else
+      else  // key lines (NI per leaf, KPL lines of P each) or, compressed form, leaf lines (F, 1)
         bk_keyline_max<K><<<t->num_sms * 4, 256, 0, s>>>((const uint8_t*)t->r.d_leaf, t->r.d_count, t->r.d_chain,
                                                           t->r.nchain, t->F, t->P, uint32_t(bs.span),
-                                                          uint32_t(64 / sizeof(K)), (K*)bs.d_M);
+                                                          bs.cdir ? 1u : uint32_t(64 / sizeof(K)), (K*)bs.d_M);
       HBT_CUDA_TRY(cudaGetLastError());
     }
-    if (bs.d32) {
-      std::vector<BucketDir32> h(B);
+    if (bs.cdir) {
+      std::vector<BucketDir> h(B);
       uint64_t total = 0;
       for (uint32_t b = 0; b < B; ++b) {
         uint64_t u0, u1;
-        bucket_units(t->L0, B, b, bs.span, u0, u1);
-        h[b] = BucketDir32{u0, total, 0, uint32_t(u1 - u0 + 1), 0};
-        total += (u1 - u0 + 1 + 3) & ~uint64_t(3);
+        if (t->form == HBT_IMPLICIT) {
+          bucket_units(t->L0, B, b, bs.span, u0, u1);
+        } else {  // the lines of chain leaves [c0, c1]
+          bucket_units(t->r.nchain, B, b, 1, u0, u1);
+          u0 *= t->F;
+          u1 = u1 * t->F + t->F - 1;
+        }
+        h[b] = BucketDir{u0, total, 0, uint32_t(u1 - u0 + 1), 0, 0, 0, 0, 0};
+        total += (u1 - u0 + 1 + 7) & ~uint64_t(7);
       }
-      if (!bs.d_bd) HBT_CUDA_TRY(cudaMalloc(&bs.d_bd, kMaxBuckets * sizeof(BucketDir32)));
-      if (bs.M32_cap < total * 4) {
-        cudaFree(bs.d_M32);
-        bs.d_M32 = nullptr;
-        bs.M32_cap = 0;
-        HBT_CUDA_TRY(cudaMalloc(&bs.d_M32, total * 4));
-        bs.M32_cap = total * 4;
+      if (!bs.d_bd) HBT_CUDA_TRY(cudaMalloc(&bs.d_bd, kMaxBuckets * sizeof(BucketDir)));
+      const uint64_t bytes = total * 2 + uint64_t(B) * kT16 * 2;
+      if (bs.E16_cap < bytes) {
+        cudaFree(bs.d_E16);
+        bs.d_E16 = nullptr;
+        bs.E16_cap = 0;
+        HBT_CUDA_TRY(cudaMalloc(&bs.d_E16, bytes));
+        bs.E16_cap = bytes;
       }
-      HBT_CUDA_TRY(cudaMemcpyAsync(bs.d_bd, h.data(), B * sizeof(BucketDir32), cudaMemcpyHostToDevice, s));
-      bk_dir32<K><<<B, 256, 0, s>>>((const K*)bs.d_M, (BucketDir32*)bs.d_bd, bs.d_M32);
+      bs.d_T16 = bs.d_E16 + total;
+      HBT_CUDA_TRY(cudaMemcpyAsync(bs.d_bd, h.data(), B * sizeof(BucketDir), cudaMemcpyHostToDevice, s));
+      bk_cdir<K><<<B, 256, 0, s>>>((const K*)bs.d_M, (BucketDir*)bs.d_bd, bs.d_E16, bs.d_T16);
       HBT_CUDA_TRY(cudaGetLastError());
     }
   }
@@ -989,10 +1045,11 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
       d.pos_base = pos_base;
       d.cap = t->cfg.bucket_cap ? std::min<uint32_t>(t->cfg.bucket_cap, uint32_t(item_cap(t, p.B)))
                                 : uint32_t(item_cap(t, p.B));
-      if (bs.d32) {
-        d.bd = static_cast<const BucketDir32*>(bs.d_bd);
-        d.M32 = bs.d_M32;
-        d.cap = bs.cap32;
+      if (bs.cdir) {
+        d.bd = static_cast<const BucketDir*>(bs.d_bd);
+        d.E16 = bs.d_E16;
+        d.T16 = bs.d_T16;
+        d.cap = bs.cap16;
       }
       rc = t->form == HBT_IMPLICIT ? implicit_search_items(t, qs, m, pf_s, v_s, d, s)
                                    : regular_search_items(t, qs, m, pf_s, v_s, d, s);
@@ -1181,7 +1238,7 @@ static void bucket_state_free(BucketState& b) {
   cudaFree(b.d_dir);
   cudaFree(b.d_M);
   cudaFree(b.d_bd);
-  cudaFree(b.d_M32);
+  cudaFree(b.d_E16);
   b = BucketState{};
 }
 

@@ -89,8 +89,9 @@ struct SearchConfig {
   uint32_t l2_hint = 4;          // implicit search: L2 eviction-priority hints (LevelTable::l2_hint);
                                  // 4 = auto: leaf lines evict-first iff the I-segment fits in L2 / 4
   uint32_t item_l2_hint = 1;     // implicit bucketed item search (c4 item search 10.96 -> 9.50 ms)
-  uint32_t item_dir32 = 1;       // implicit item directory in the compressed per-bucket form (ItemDir::bd):
-                                 // 0 = never, 1 = where it reaches a deeper level, 2 = always
+  uint32_t item_cdir = 1;        // item directory in the compressed per-bucket form (ItemDir::bd): 0 = never,
+                                 // 1 = where it reaches a deeper level (regular: always fits-permitting),
+                                 // 2 = always (implicit: even at the same level)
 };
 
 // Bucket-local directory of the bucketed search (bucketed.cu): after the
@@ -115,21 +116,30 @@ struct ItemDir {
   uint64_t pos_base = 0;  // implicit: added to every reported position (key-range shards)
   uint32_t rounds = 16;   // warp rounds per work item (fewer for small batches: every SM gets items)
   // Compressed per-bucket directory (implicit trees whose directory level has too many
-  // units per bucket for 8 B keys in shared memory): bucket b's unit maxima as 32-bit
-  // offsets M32[bd[b].off + i] = (M[bd[b].u0 + i] - bd[b].lo) >> bd[b].sh, items cut
-  // inside one bucket each (item search).
-  const struct BucketDir32* bd = nullptr;
-  const uint32_t* M32 = nullptr;
-  bool fix = false;  // ties of the truncated maxima resolved by the walk (implicit_search.cu)
+  // units per bucket for 8 B keys in shared memory; regular trees: the leaf lines of the
+  // chain leaves): with M' = (M - bd[b].lo) >> bd[b].sh (32 bits), a prefix table over
+  // 2^12 slices T16[b * kT16 + p] = #{M' < p << ssh} and 16-bit entries
+  // E16[bd[b].off16 + i] = (M'_i >> esh) & 0xFFFF; items are cut inside one bucket
+  // (item search).
+  const struct BucketDir* bd = nullptr;
+  const uint16_t* E16 = nullptr;
+  const uint16_t* T16 = nullptr;
+  bool fix = false;  // single ties of the truncated maxima resolved by the walk
 };
 
+constexpr uint32_t kT16 = 4104;  // per-bucket prefix table: 2^12 + 1 entries, padded to 16 B
+
 // One bucket of the compressed item directory (ItemDir::bd).
-struct BucketDir32 {
-  uint64_t u0;   // first directory unit of the bucket
-  uint64_t off;  // its first entry in M32 (a multiple of 4: 16 B aligned bulk copies)
-  uint64_t lo;   // M[u0]: the offset origin
-  uint32_t cnt;  // units u0 .. u0 + cnt - 1
-  uint32_t sh;   // right shift that makes M[u0 + cnt - 1] - lo fit 32 bits
+struct BucketDir {
+  uint64_t u0;     // first directory unit of the bucket
+  uint64_t off16;  // its first entry in E16 (a multiple of 8: 16 B aligned bulk copies)
+  uint64_t lo;     // M[u0]: the offset origin
+  uint32_t cnt;    // units u0 .. u0 + cnt - 1 (< 2^16)
+  uint32_t sh;     // right shift that makes M[u0 + cnt - 1] - lo fit 32 bits
+  uint32_t top;    // (M[u0 + cnt - 1] - lo) >> sh
+  uint32_t ssh;    // prefix-table slice p holds M' in [p << ssh, (p + 1) << ssh)
+  uint32_t esh;    // entry = (M' >> esh) & 0xFFFF (ssh - 16, or 0)
+  uint32_t pad;
 };
 
 // Owner side of the fused sharded exchange (sharded_fused.cu): the bucketed search's
@@ -158,11 +168,12 @@ struct BucketState {
   uint32_t level = 0;            // implicit: directory level
   uint64_t span = 1, nunits = 0;
   bool items = false;            // the item directory is in use
-  bool d32 = false;              // ... in its compressed per-bucket form (ItemDir::bd)
-  void* d_bd = nullptr;          // B x BucketDir32
-  uint32_t* d_M32 = nullptr;     // compressed maxima
-  uint64_t M32_cap = 0;          // bytes allocated
-  uint32_t cap32 = 0;            // largest bucket's unit count, rounded up to 4
+  bool cdir = false;             // ... in its compressed per-bucket form (ItemDir::bd)
+  void* d_bd = nullptr;          // B x BucketDir
+  uint16_t* d_E16 = nullptr;     // entries | prefix tables
+  uint16_t* d_T16 = nullptr;
+  uint64_t E16_cap = 0;          // bytes allocated
+  uint32_t cap16 = 0;            // largest bucket's unit count, rounded up to 8
   cudaEvent_t ev[6] = {};        // phase boundaries of the last timed bucketed search
   bool timed = false;
   uint32_t launches = 0;

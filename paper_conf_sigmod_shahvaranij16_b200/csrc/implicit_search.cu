@@ -140,7 +140,7 @@ __device__ __forceinline__ uint32_t count_less16(const V16<K>& v, K q, unsigned 
 // Phase 2 of a warp round: levels [d0, H) by lane groups, the leaf line, and the
 // results of the round (slot j of group g = round query j*NG + g, stored at
 // base + j*NG + g).
-// FIX (compressed item directory, implicit_search_items32_kernel): the directory may
+// FIX (compressed item directory, implicit_search_cdir_kernel): the directory may
 // place a query ONE unit early (a tie of truncated maxima; runs of ties are settled
 // before the walk).  Every real separator of that unit u is < q and its last key slot
 // is MAX (reading R3), so the walk takes the last child at every level and ends
@@ -546,58 +546,34 @@ implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* _
   }
 }
 
-// The same with the COMPRESSED per-bucket directory (ItemDir::bd / M32), used when
-// it reaches a deeper level than 8 B keys would (c4: the last inner level instead of
-// the one above it, one dependent node read less per query).  Work items are cut
-// inside one bucket each (bucket b's queries split into ceil(cnt_b / W) near-equal
-// items), so an item stages exactly its bucket's unit maxima: one elected thread
-// moves them into shared memory with bulk copies (cp.async.bulk, completion on an
-// mbarrier).  Entry i holds (M[u0+i] - lo) >> sh: order-preserving, so
-// lower_bound(M32, (q - lo) >> sh) is exact except where the truncated values tie
-// with the query's; those few entries are compared exactly against M in global
-// memory (sh = 0, i.e. bucket key spans below 2^32, never ties).
-constexpr uint32_t kPrefixBits32 = 12;
-
-template <typename K>
-__device__ __forceinline__ uint32_t lower_bound32(const uint32_t* s_M, uint32_t cnt, const uint32_t* s_T,
-                                                  const PrefixTab<uint32_t>& pt, K q, K lo, uint32_t sh,
-                                                  const K* __restrict__ gM, bool fixable) {
-  if (q <= lo) return 0;
-  const K dq = K(q - lo) >> sh;
-  if (dq > K(pt.span)) return cnt;  // beyond the bucket's last maximum (pt.lo = s_M[0] = 0)
-  const uint32_t q32 = uint32_t(dq);
-  uint32_t a = prefix_lower_bound(s_M, cnt, s_T, pt, q32);
-  // A tie with ONE truncated maximum leaves a or a + 1, which the walk settles (FIX, when
-  // fixable); a RUN of ties (or no FIX) is settled here against the exact maxima gM, so
-  // the walk never moves on by more than one unit.
-  if (sh && a < cnt && s_M[a] == q32) {
-    if (fixable && (a + 1 >= cnt || s_M[a + 1] != q32)) return a;
-    while (a < cnt && s_M[a] == q32 && __ldg(gM + a) < q) ++a;
-  }
-  return a;
-}
-
+// The same with the COMPRESSED per-bucket directory (ItemDir::bd, 16-bit entries under a
+// 2^12-slice prefix table), used when it reaches a deeper level than 8 B keys would (c4:
+// the last inner level instead of the one above it, one dependent node read less per
+// query; c5: the leaf lines themselves).  Work items are cut inside one bucket each
+// (bucket b's queries split into ceil(cnt_b / W) near-equal items), so an item stages
+// exactly its bucket's directory: one elected thread moves the entries and the prefix
+// table into shared memory with bulk copies (cp.async.bulk, completion on an mbarrier).
+// Ties of truncated values: lower_bound16 (item_dir.cuh) and descend_and_store FIX.
 template <typename K, int F, int THREADS>
 __global__ void __launch_bounds__(THREADS)
-implicit_search_items32_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ inner_idx,
-                               const uint8_t* __restrict__ leaf, const ItemDir d, const K* __restrict__ queries,
-                               uint64_t m, uint64_t* __restrict__ out_pf, K* __restrict__ out_v, const LevelTable lt,
-                               uint64_t n) {
+implicit_search_cdir_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ inner_idx,
+                            const uint8_t* __restrict__ leaf, const ItemDir d, const K* __restrict__ queries,
+                            uint64_t m, uint64_t* __restrict__ out_pf, K* __restrict__ out_v, const LevelTable lt,
+                            uint64_t n) {
   using C = Cfg<K, F>;
   constexpr int QPG = 32 / C::NG;
-  constexpr uint32_t PB = kPrefixBits32;
   const uint64_t W = uint64_t(THREADS) * d.rounds;
   const uint32_t B = d.B;
   extern __shared__ __align__(16) uint8_t smem[];
-  // [M32: cap entries | bucket starts: B + 1 u64 | prefix table: 2^PB + 1 | item starts: B + 1]
-  uint32_t* s_M = reinterpret_cast<uint32_t*>(smem);
-  uint64_t* s_bs = reinterpret_cast<uint64_t*>(s_M + d.cap);
-  uint32_t* s_T = reinterpret_cast<uint32_t*>(s_bs + B + 1);
-  uint32_t* s_is = s_T + (1u << PB) + 1;
+  // [E16: cap entries | T16: kT16 | bucket starts: B + 1 u64 | item starts: B + 1]
+  uint16_t* s_E = reinterpret_cast<uint16_t*>(smem);
+  uint16_t* s_T = s_E + d.cap;
+  uint64_t* s_bs = reinterpret_cast<uint64_t*>(s_T + kT16);
+  uint32_t* s_is = reinterpret_cast<uint32_t*>(s_bs + B + 1);
   __shared__ uint64_t bar;
   __shared__ uint32_t s_tmp[32];
   __shared__ uint64_t s_p[2];
-  __shared__ BucketDir32 s_bd;
+  __shared__ BucketDir s_bd;
   const K* gM = static_cast<const K*>(d.M);
   for (uint32_t i = threadIdx.x; i <= B; i += THREADS) s_bs[i] = d.bstart[i];
   __syncthreads();
@@ -628,26 +604,22 @@ implicit_search_items32_kernel(const uint8_t* __restrict__ inner, const uint8_t*
       const uint64_t c0 = s_bs[lo], cnt = s_bs[lo + 1] - c0;
       s_p[0] = c0 + (cnt * j) / nb;
       s_p[1] = c0 + (cnt * (j + 1)) / nb - 1;
-      const BucketDir32 bd = d.bd[lo];
+      const BucketDir bd = d.bd[lo];
       s_bd = bd;
-      // the previous item's reads of s_M are ordered before this copy by the barrier
-      // that ended it; the proxy fence orders them for the async (bulk copy) proxy
+      // the previous item's reads of the directory are ordered before this copy by the
+      // barrier that ended it; the proxy fence orders them for the async (bulk copy) proxy
       fence_proxy_async_smem();
-      const uint32_t bytes = (bd.cnt * 4u + 15u) & ~15u;
-      mbar_expect_tx(&bar, bytes);
-      for (uint32_t o = 0; o < bytes; o += 32768u)
-        bulk_g2s(reinterpret_cast<uint8_t*>(s_M) + o, d.M32 + bd.off + o / 4, bytes - o < 32768u ? bytes - o : 32768u,
-                 &bar);
+      const uint32_t eb = ((bd.cnt + 7u) & ~7u) * 2u;
+      mbar_expect_tx(&bar, eb + kT16 * 2u);
+      bulk_g2s(s_E, d.E16 + bd.off16, eb, &bar);
+      bulk_g2s(s_T, d.T16 + uint64_t(lo) * kT16, kT16 * 2u, &bar);
     }
     __syncthreads();
     const uint64_t p0 = s_p[0], p1 = s_p[1];
     const uint64_t u0 = s_bd.u0;
-    const uint32_t cnt = s_bd.cnt, sh = s_bd.sh;
-    const K blo = K(s_bd.lo);
+    const uint32_t cnt = s_bd.cnt;
     mbar_wait(&bar, parity);
     parity ^= 1u;
-    const PrefixTab<uint32_t> pt = build_prefix(s_M, cnt, s_T, THREADS, PB);
-    __syncthreads();
     K nextq;
     {
       const uint64_t i = p0 + uint64_t(wid) * 32 + lane;
@@ -664,7 +636,8 @@ implicit_search_items32_kernel(const uint8_t* __restrict__ inner, const uint8_t*
       }
       // single ties are resolved by the walk (descend_and_store FIX), not by a dependent
       // read of the exact maxima that would stall the whole warp
-      const uint32_t a = lower_bound32(s_M, cnt, s_T, pt, myq, blo, sh, gM + u0, d.fix);
+      const uint32_t a = lower_bound16(s_E, s_T, cnt, myq, K(s_bd.lo), s_bd.sh, s_bd.top, s_bd.ssh, s_bd.esh,
+                                       gM + u0, d.fix);
       const uint32_t mynode = uint32_t(u0) + (a < cnt ? a : cnt - 1);
       K q[QPG];
       uint32_t node[QPG];
@@ -780,10 +753,10 @@ struct Launch {
     return HBT_OK;
   }
 
-  static int run_items32(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, const ItemDir& d,
+  static int run_cdir(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, const ItemDir& d,
                          cudaStream_t s) {
     constexpr int TH = C::NODE_BYTES > 128 ? 512 : 1024;
-    auto kern = implicit_search_items32_kernel<K, F, TH>;
+    auto kern = implicit_search_cdir_kernel<K, F, TH>;
     LevelTable lt{};
     for (uint32_t x = 0; x <= t->H; ++x) lt.offset[x] = t->offset[x];
     lt.H = t->H;
@@ -801,8 +774,7 @@ struct Launch {
     dd.rounds = item_rounds(m, t->num_sms, TH, t->cfg.item_rounds ? t->cfg.item_rounds : 16);
     // the walk resolves directory ties (it detects them on the 256-bit leaf read)
     dd.fix = lt.leaf256 != 0;
-    const size_t smem = size_t(d.cap) * 4 + (size_t(d.B) + 1) * 8 + ((1u << kPrefixBits32) + 1) * 4 +
-                        (size_t(d.B) + 1) * 4;
+    const size_t smem = (size_t(d.cap) + kT16) * 2 + (size_t(d.B) + 1) * 12;
     kern<<<t->num_sms, TH, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
                                      (const uint8_t*)t->d_leaf, dd, (const K*)q, m, pf, (K*)v, lt, t->n);
     HBT_CUDA_TRY(cudaGetLastError());
@@ -861,10 +833,10 @@ int implicit_search_items(const hbt_tree* t, const void* q, uint64_t m, uint64_t
     using K = decltype(tag);
     if (d.bd) {
       switch (t->F) {
-        case 4: return Launch<K, 4>::run_items32(t, q, m, pf, v, d, s);
-        case 8: return Launch<K, 8>::run_items32(t, q, m, pf, v, d, s);
-        case 16: return Launch<K, 16>::run_items32(t, q, m, pf, v, d, s);
-        case 32: return Launch<K, 32>::run_items32(t, q, m, pf, v, d, s);
+        case 4: return Launch<K, 4>::run_cdir(t, q, m, pf, v, d, s);
+        case 8: return Launch<K, 8>::run_cdir(t, q, m, pf, v, d, s);
+        case 16: return Launch<K, 16>::run_cdir(t, q, m, pf, v, d, s);
+        case 32: return Launch<K, 32>::run_cdir(t, q, m, pf, v, d, s);
       }
     }
     switch (t->F) {

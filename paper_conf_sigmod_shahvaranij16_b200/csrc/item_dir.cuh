@@ -80,4 +80,35 @@ __device__ __forceinline__ uint32_t prefix_lower_bound(const K* s_M, uint32_t cn
   return lb_range(s_M, s_T[p], s_T[p + 1], q);
 }
 
+// lower_bound over bucket b's compressed maxima (ItemDir::bd): the prefix table T names
+// the slice of entries whose 32-bit offsets M' share the query's top bits, E holds the
+// next 16 bits.  Truncation is order-preserving, so the result is exact except where
+// the query's truncated value TIES with an entry's (then the answer is that unit or a
+// later one).  A RUN of ties (or fixable = false) is settled against the exact maxima
+// gM; a single tie is left to the caller's walk (the answer is the returned unit or the
+// next one).
+template <typename K>
+__device__ __forceinline__ uint32_t lower_bound16(const uint16_t* E, const uint16_t* T, uint32_t cnt, K q, K lo,
+                                                  uint32_t sh, uint32_t top, uint32_t ssh, uint32_t esh,
+                                                  const K* __restrict__ gM, bool fixable) {
+  if (q <= lo) return 0;
+  const K dq = K(q - lo) >> sh;
+  if (dq > K(top)) return cnt;
+  const uint32_t q32 = uint32_t(dq);
+  const uint32_t p = q32 >> ssh;
+  uint32_t a = T[p];
+  const uint32_t b = T[p + 1];
+  const uint16_t q16 = uint16_t(q32 >> esh);
+  uint32_t len = b - a;
+  while (len > 0) {
+    const uint32_t half = len >> 1;
+    if (E[a + half] < q16) { a += half + 1; len -= half + 1; } else { len = half; }
+  }
+  if ((sh | esh) && a < b && E[a] == q16) {
+    if (fixable && (a + 1 >= b || E[a + 1] != q16)) return a;
+    while (a < b && E[a] == q16 && __ldg(gM + a) < q) ++a;
+  }
+  return a;
+}
+
 }  // namespace hbt

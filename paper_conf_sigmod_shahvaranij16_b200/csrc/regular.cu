@@ -20,6 +20,7 @@
 
 #include <algorithm>
 
+#include "block_util.cuh"
 #include "hbt_internal.cuh"
 #include "item_dir.cuh"
 
@@ -615,6 +616,184 @@ regular_search_items_kernel(const RView rv, const ItemDir d, const K* __restrict
   }
 }
 
+// Item search on the COMPRESSED per-bucket LEAF-LINE directory (ItemDir::bd; units =
+// the F lines of each chain leaf, M = the line's true max, lines past the leaf's last
+// used line repeat the leaf max): a query goes from the directory straight to its leaf
+// line (v = chain[c], line j), one dependent access instead of key line + leaf line.
+// As in implicit_search_cdir_kernel, items are cut inside one bucket and the bucket's
+// 16-bit entries and prefix table are bulk-copied into shared memory per item (plus
+// its chain ids).  A single tie can name the line BEFORE the right one (a run of ties,
+// including a used line and the padding entries repeating its max, is settled exactly
+// by lower_bound16); the leaf then reports "past every real key of the line" (s = P, or
+// a MAX padding slot at or past the line's count), which cannot happen on the
+// right line of a bucket (q <= sp[b]), so the slot moves to the next line in key order
+// (j + 1, or line 0 of the next chain leaf) while inside the bucket.
+template <typename K, int F, int THREADS>
+__global__ void __launch_bounds__(THREADS)
+regular_search_cdir_kernel(const RView rv, const ItemDir d, const K* __restrict__ queries, uint64_t m,
+                           uint64_t* __restrict__ out_pf, K* __restrict__ out_v) {
+  constexpr int G = 2, NG = 16, QPG = 32 / NG;
+  constexpr uint32_t P = Geo<K>::P;
+  const uint64_t W = uint64_t(THREADS) * d.rounds;
+  const uint32_t B = d.B;
+  extern __shared__ __align__(16) uint8_t smem[];
+  // [E16: cap | T16: kT16 | chain ids: cap / F + 4, padded to 4 | bucket starts: B + 1 u64 | item starts: B + 1]
+  uint16_t* s_E = reinterpret_cast<uint16_t*>(smem);
+  uint16_t* s_T = s_E + d.cap;
+  uint32_t* s_chain = reinterpret_cast<uint32_t*>(s_T + kT16);
+  uint64_t* s_bs = reinterpret_cast<uint64_t*>(s_chain + ((d.cap / F + 4 + 3) & ~3u));
+  uint32_t* s_is = reinterpret_cast<uint32_t*>(s_bs + B + 1);
+  __shared__ uint64_t bar;
+  __shared__ uint32_t s_tmp[32];
+  __shared__ uint64_t s_p[2];
+  __shared__ BucketDir s_bd;
+  const K* gM = static_cast<const K*>(d.M);
+  for (uint32_t i = threadIdx.x; i <= B; i += THREADS) s_bs[i] = d.bstart[i];
+  __syncthreads();
+  for (uint32_t b = threadIdx.x; b < B; b += THREADS) s_is[b] = uint32_t((s_bs[b + 1] - s_bs[b] + W - 1) / W);
+  __syncthreads();
+  const uint32_t last = s_is[B - 1];
+  block_exclusive_scan<THREADS>(s_is, s_is, B, s_tmp);
+  if (threadIdx.x == 0) {
+    s_is[B] = s_is[B - 1] + last;
+    mbar_init(&bar, 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  const uint32_t items = s_is[B];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int g = lane / G, k = lane % G;
+  uint32_t parity = 0;
+  for (uint32_t it = blockIdx.x; it < items; it += gridDim.x) {
+    if (threadIdx.x == 0) {
+      uint32_t lo = 0, hi = B;  // the bucket: largest b with s_is[b] <= it
+      while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (s_is[mid] <= it) lo = mid; else hi = mid;
+      }
+      const uint64_t nb = s_is[lo + 1] - s_is[lo], j = it - s_is[lo];
+      const uint64_t c0 = s_bs[lo], cnt = s_bs[lo + 1] - c0;
+      s_p[0] = c0 + (cnt * j) / nb;
+      s_p[1] = c0 + (cnt * (j + 1)) / nb - 1;
+      const BucketDir bd = d.bd[lo];
+      s_bd = bd;
+      fence_proxy_async_smem();  // the previous item's reads of the directory precede this copy
+      const uint32_t eb = ((bd.cnt + 7u) & ~7u) * 2u;
+      mbar_expect_tx(&bar, eb + kT16 * 2u);
+      bulk_g2s(s_E, d.E16 + bd.off16, eb, &bar);
+      bulk_g2s(s_T, d.T16 + uint64_t(lo) * kT16, kT16 * 2u, &bar);
+    }
+    __syncthreads();
+    const uint64_t p0 = s_p[0], p1 = s_p[1];
+    const uint64_t e0 = s_bd.u0;  // first entry = first chain leaf * F
+    const uint32_t cnt = s_bd.cnt, nc = cnt / F;
+    for (uint32_t i = threadIdx.x; i < nc; i += THREADS) s_chain[i] = __ldg(d.chain + e0 / F + i);
+    mbar_wait(&bar, parity);
+    parity ^= 1u;
+    __syncthreads();  // chain ids
+    K nextq;
+    {
+      const uint64_t i = p0 + uint64_t(wid) * 32 + lane;
+      nextq = i <= p1 ? ldcs(queries + i) : key_max<K>();
+    }
+#pragma unroll 1
+    for (int r = 0; r < int(d.rounds); ++r) {
+      const uint64_t base = p0 + (uint64_t(r) * (THREADS / 32) + wid) * 32;
+      if (base > p1) break;
+      const K myq = nextq;
+      {
+        const uint64_t i = base + (THREADS / 32) * 32 + lane;
+        nextq = (r + 1 < int(d.rounds) && i <= p1) ? ldcs(queries + i) : key_max<K>();
+      }
+      const uint32_t a = lower_bound16(s_E, s_T, cnt, myq, K(s_bd.lo), s_bd.sh, s_bd.top, s_bd.ssh, s_bd.esh,
+                                       gM + e0, true);
+      const uint32_t e = a < cnt ? a : cnt - 1;
+      K q[QPG];
+      uint32_t cl[QPG], ln[QPG];
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) {
+        const int src = (j * NG) % 32 + g;
+        q[j] = __shfl_sync(0xffffffffu, myq, src);
+        const uint32_t ej = __shfl_sync(0xffffffffu, e, src);
+        cl[j] = ej / F;
+        ln[j] = ej % F;
+      }
+      // leaf line (v*F + line) by two 256-bit lane loads: keys on lane 0, values on lane 1
+      L256<K> lw[QPG];
+      uint32_t sl[QPG];
+      bool end[QPG];
+      K key_s[QPG], val_s[QPG];
+      auto probe = [&](int j) {
+        const uint32_t v = s_chain[cl[j]];
+        ld32(lw[j], rv.leaf + (uint64_t(v) * F + ln[j]) * 64 + k * 32);
+      };
+      auto settle = [&](int j) {  // every lane shuffles
+        const uint32_t v = s_chain[cl[j]];
+        uint32_t c = 0;
+#pragma unroll
+        for (uint32_t x = 0; x < P; ++x) c += lw[j].k[x] < q[j] ? 1u : 0u;
+        sl[j] = __shfl_sync(0xffffffffu, c, g * G);
+        const uint32_t sc = sl[j] < P ? sl[j] : P - 1;
+        const K xk = pick(lw[j].k, sc);
+        key_s[j] = __shfl_sync(0xffffffffu, xk, g * G);
+        val_s[j] = __shfl_sync(0xffffffffu, xk, g * G + 1);
+        bool en = (sl[j] == P);
+        if (!en && key_s[j] == key_max<K>()) {
+          // MAX slot: padding unless it is a counted entry ("must read the node size")
+          const int64_t in_line = int64_t(__ldg(rv.count + v)) - int64_t(ln[j]) * P;
+          const int64_t lim = in_line < int64_t(P) ? in_line : int64_t(P);
+          en = int64_t(sl[j]) >= lim;
+        }
+        end[j] = en;
+      };
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) probe(j);
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) settle(j);
+#pragma unroll 1
+      for (;;) {
+        // past the line's real keys before the bucket's last line: the next line in key order
+        uint32_t adv = 0;
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) {
+          if (!end[j]) continue;
+          const uint32_t v = s_chain[cl[j]];
+          const uint32_t used = (__ldg(rv.count + v) + P - 1) / P;
+          if (ln[j] + 1 < used) {
+            ++ln[j];
+            adv |= 1u << j;
+          } else if (cl[j] + 1 < nc) {
+            ++cl[j];
+            ln[j] = 0;
+            adv |= 1u << j;
+          }
+        }
+        if (!__any_sync(0xffffffffu, adv != 0)) break;
+#pragma unroll
+        for (int j = 0; j < QPG; ++j)
+          if ((adv >> j) & 1u) probe(j);
+#pragma unroll
+        for (int j = 0; j < QPG; ++j) settle(j);  // unchanged slots settle to the same result
+      }
+      uint64_t my_pf = 0;
+      K my_v = 0;
+#pragma unroll
+      for (int j = 0; j < QPG; ++j) {
+        const uint32_t v = s_chain[cl[j]];
+        const bool found = !end[j] && key_s[j] == q[j];
+        if (j == k) {
+          my_pf = end[j] ? kEnd : (((uint64_t(v) * F + ln[j]) * P + sl[j]) | (found ? kFound : 0ull));
+          my_v = found ? val_s[j] : K(0);
+        }
+      }
+      const uint64_t o = base + uint64_t(k) * NG + g;
+      if (o <= p1)  // 16 B record {pos|found, value}: the bucket gather reads records
+        __stcs(reinterpret_cast<ulonglong2*>(out_pf) + o, make_ulonglong2(my_pf, (unsigned long long)my_v));
+    }
+    __syncthreads();
+  }
+}
+
 template <typename K, int F, int QPL, int THREADS>
 int search_v2_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, cudaStream_t s) {
   const RegularState& r = t->r;
@@ -665,8 +844,33 @@ int search_v2_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf,
 
 
 template <typename K, int F>
+int search_cdir_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, const ItemDir& d,
+                          cudaStream_t s) {
+  constexpr int TH = 1024;
+  const RegularState& r = t->r;
+  auto kern = regular_search_cdir_kernel<K, F, TH>;
+  RView rv{};
+  rv.leaf = (const uint8_t*)r.d_leaf;
+  rv.count = r.d_count;
+  rv.U = r.U;
+  const size_t smem = (size_t(d.cap) + kT16) * 2 + ((size_t(d.cap) / F + 4 + 3) & ~size_t(3)) * 4 +
+                      (size_t(d.B) + 1) * 12;
+  static bool attr = false;
+  if (!attr) {
+    HBT_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024));
+    attr = true;
+  }
+  ItemDir dd = d;
+  dd.rounds = item_rounds(m, t->num_sms, TH, t->cfg.item_rounds ? t->cfg.item_rounds : 16);
+  kern<<<t->num_sms, TH, smem, s>>>(rv, dd, (const K*)q, m, pf, (K*)v);
+  HBT_CUDA_TRY(cudaGetLastError());
+  return HBT_OK;
+}
+
+template <typename K, int F>
 int search_items_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void* v, const ItemDir& d,
                         cudaStream_t s) {
+  if (d.bd) return search_cdir_launch<K, F>(t, q, m, pf, v, d, s);
   constexpr int TH = 1024;
   const RegularState& r = t->r;
   auto kern = regular_search_items_kernel<K, F, TH>;

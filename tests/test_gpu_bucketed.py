@@ -26,7 +26,7 @@ def _oracle(layout, k, v, F, width):
     return (oracle.ITree if layout == "implicit" else oracle.RTree).from_pairs(k, v, F, width)
 
 
-# (bucket_items, bucket_cap, leaf256, item_dir32): plain search, 8 B smem directory, global
+# (bucket_items, bucket_cap, leaf256, item_cdir): plain search, 8 B smem directory, global
 # fallback, 128-bit lane loads (directory form auto), compressed per-bucket directory forced
 ITEM_MODES = [(0, 0, 1, 1), (1, 0, 1, 0), (1, 7, 1, 1), (1, 0, 0, 1), (1, 0, 1, 2)]
 
@@ -48,7 +48,7 @@ def test_bucketed_edge_suite(hbt, layout, width, F, items, cap, leaf256, dir32):
         t.set_param("bucket_items", items)
         t.set_param("bucket_cap", cap)
         t.set_param("leaf256", leaf256)
-        t.set_param("item_dir32", dir32)
+        t.set_param("item_cdir", dir32)
         for slice_bytes in (1, 4096, 1 << 16):  # 1 B: one bucket per unit up to the 1024 cap
             t.set_param("bucket_slice", slice_bytes)
             pf, val = gpu_search(t, q, width)
@@ -73,7 +73,7 @@ def test_bucketed_scaled_workload(hbt, layout, F, items, cap, leaf256, dir32):
     t.set_param("bucket_items", items)
     t.set_param("bucket_cap", cap)
     t.set_param("leaf256", leaf256)
-    t.set_param("item_dir32", dir32)
+    t.set_param("item_cdir", dir32)
     for slice_bytes in (1 << 16, 1 << 20, 1 << 22):
         t.set_param("bucket_slice", slice_bytes)
         for qpf in (0, 1):  # default and single-round work items
@@ -106,7 +106,7 @@ def test_bucketed_after_update(hbt, layout, items, cap, leaf256, dir32):
     t.set_param("bucket_items", items)
     t.set_param("bucket_cap", cap)
     t.set_param("leaf256", leaf256)
-    t.set_param("item_dir32", dir32)
+    t.set_param("item_cdir", dir32)
     t.set_param("bucket_slice", 2048)
     q = query_set(k, width, rng, 4000)
     pf, val = gpu_search(t, q, width)
@@ -127,9 +127,11 @@ def test_bucketed_after_update(hbt, layout, items, cap, leaf256, dir32):
     t.close()
 
 
+@pytest.mark.parametrize("layout,F", [("implicit", 16), ("regular", 32), ("regular", 4)])
 @pytest.mark.parametrize("nsmall,slice_bytes", [(20000, 1 << 20), (20000, 4096), (20000, 1), (400000, 1 << 30)])
-def test_compressed_directory_ties(hbt, nsmall, slice_bytes):
-    """Compressed per-bucket directory (item_dir32) where 32-bit truncation ties: dense
+def test_compressed_directory_ties(hbt, layout, F, nsmall, slice_bytes):
+    """Compressed per-bucket directory (item_cdir; implicit: unit maxima, regular: leaf
+    lines of the chain leaves) where 32-bit truncation ties: dense
     small keys share a bucket with keys near 2^63, so the bucket's shift is ~31 and
     every small maximum truncates to the same value.  Ties are resolved by the walk
     (256-bit whole-node / leaf reads at the directory level) or against the exact
@@ -141,13 +143,13 @@ def test_compressed_directory_ties(hbt, nsmall, slice_bytes):
     big = (np.uint64(1) << np.uint64(63)) + rng.integers(0, 1 << 40, 300, dtype=np.uint64)
     for width, k in ((8, np.concatenate([small, big])), (4, small)):
         v = rng.integers(0, kmax(width), len(k), dtype=np.uint64, endpoint=True)
-        o = oracle.ITree.from_pairs(k, v, 16, width)
-        t = gpu_build(hbt, k, v, 16, width)
+        o = _oracle(layout, k, v, F, width)
+        t = gpu_build(hbt, k, v, F, width, layout=layout)
         q = np.concatenate([query_set(k, width, rng, 6000), k[::7], k[::11] + np.uint64(1), k[::13] - np.uint64(1)])
         q = np.concatenate([q, np.array([0, kmax(width)], dtype=np.uint64)]) & np.uint64(kmax(width))
         epf, ev = o.search(q)
         t.set_param("bucket", 1)
-        t.set_param("item_dir32", 2)
+        t.set_param("item_cdir", 2)
         t.set_param("bucket_slice", slice_bytes)
         for rounds, leaf256, full256, l2b in ((0, 1, 1, 0), (0, 1, 1, 4096), (1, 1, 1, 4096), (0, 0, 1, 0),
                                               (0, 1, 0, 4096), (1, 0, 0, 0)):
@@ -156,7 +158,7 @@ def test_compressed_directory_ties(hbt, nsmall, slice_bytes):
             t.set_param("full256", full256)
             t.set_param("l2_levels_bytes", l2b)
             pf, val = gpu_search(t, q, width)
-            cfg = (width, slice_bytes, rounds, leaf256, full256, l2b)
+            cfg = (layout, F, width, slice_bytes, rounds, leaf256, full256, l2b)
             assert np.array_equal(pf, epf), (cfg, np.nonzero(pf != epf)[0][:5])
             assert np.array_equal(val, ev), cfg
         t.close()
