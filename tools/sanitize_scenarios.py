@@ -51,7 +51,8 @@ def sc_implicit_u64_levels():
 
 
 def sc_bucketed_both_forms():
-    """Bucketed search with the item directory (count, run starts, scatter, item search, gather)."""
+    """Bucketed search with the item directory (count, run starts, scatter, item search, gather),
+    8 B-key directory and compressed per-bucket directory (bulk copies + mbarrier)."""
     for layout, F, cfg in (("implicit", 16, "c2"), ("regular", 32, "c3")):
         k, v = gen.workload_keys_values(cfg, 1 << 16)
         q = gen.workload_queries(cfg, k, 1 << 17)
@@ -59,7 +60,9 @@ def sc_bucketed_both_forms():
         t = hbt.Tree(to_dev(k, 8), to_dev(v, 8), fanout=F, layout=layout)
         t.set_param("bucket", 1)
         t.set_param("bucket_slice", 4096)
-        check(t, o, q, 8)
+        for cdir in (0, 2):
+            t.set_param("item_cdir", cdir)
+            check(t, o, q, 8)
 
 
 def sc_regular_update_splits():
