@@ -377,3 +377,140 @@ PROBE_API double probe_affinity_read_gbs(uint64_t bytes, int mode, const uint8_t
   if (cudaGetLastError() != cudaSuccess) return -2;
   return double(grid) * threads * iters * 8 * 16 / (best_ms * 1e-3) / 1e9;
 }
+
+// ---- Random 64 B line gather from a DRAM-resident buffer (round-2 item-search design
+// probe): how many random line reads per second the SMs sustain as a function of the
+// lines in flight per SM and of how they land.
+//   mode 0: a lane pair per line, one 256-bit load per lane (the item search's leaf read);
+//           U lines in flight per pair.
+//   mode 1: every lane issues cp.async.bulk (TMA) copies of its own lines (64 B each) into
+//           a shared-memory slot; one mbarrier per warp and stage; U lines per lane.
+__device__ __forceinline__ void pb_mbar_init(uint64_t* bar, uint32_t n) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(uint32_t(__cvta_generic_to_shared(bar))), "r"(n));
+}
+__device__ __forceinline__ void pb_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(uint32_t(__cvta_generic_to_shared(bar))),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void pb_bulk(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          uint32_t(__cvta_generic_to_shared(dst))),
+      "l"(src), "r"(bytes), "r"(uint32_t(__cvta_generic_to_shared(bar)))
+      : "memory");
+}
+__device__ __forceinline__ void pb_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n W: mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra W;\n}\n" ::"r"(
+          uint32_t(__cvta_generic_to_shared(bar))),
+      "r"(parity)
+      : "memory");
+}
+
+template <int U>
+__global__ void gather64_ldg(const uint8_t* __restrict__ buf, uint64_t nlines, uint64_t iters, uint64_t seed,
+                             uint64_t* __restrict__ sink) {
+  const int lane = threadIdx.x & 31, k = lane & 1;
+  const uint64_t gid = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 1;
+  uint64_t state = mix64(gid ^ seed), acc = 0;
+  for (uint64_t it = 0; it < iters; ++it) {
+    unsigned long long v[U][4];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      state = mix64(state);
+      const uint8_t* p = buf + __umul64hi(state, nlines) * 64 + k * 32;
+      asm volatile("ld.global.nc.v4.u64 {%0, %1, %2, %3}, [%4];"
+                   : "=l"(v[u][0]), "=l"(v[u][1]), "=l"(v[u][2]), "=l"(v[u][3])
+                   : "l"(p));
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) acc ^= v[u][0] ^ v[u][1] ^ v[u][2] ^ v[u][3];
+  }
+  if (acc == 0x1234567890ull) sink[threadIdx.x] = acc;
+}
+
+template <int U>
+__global__ void gather64_tma(const uint8_t* __restrict__ buf, uint64_t nlines, uint64_t iters, uint64_t seed,
+                             uint64_t* __restrict__ sink) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  __shared__ uint64_t bars[32];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  uint8_t* slot = smem + (size_t(threadIdx.x) * U) * 64;
+  if (lane == 0) pb_mbar_init(&bars[wid], 1);
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  __syncthreads();
+  uint64_t state = mix64((uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) ^ seed), acc = 0;
+  uint32_t parity = 0;
+  for (uint64_t it = 0; it < iters; ++it) {
+    if (lane == 0) pb_expect_tx(&bars[wid], 32u * U * 64u);
+    __syncwarp();
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      state = mix64(state);
+      pb_bulk(slot + u * 64, buf + __umul64hi(state, nlines) * 64, 64, &bars[wid]);
+    }
+    pb_wait(&bars[wid], parity);
+    parity ^= 1u;
+#pragma unroll
+    for (int u = 0; u < U; ++u) acc ^= *reinterpret_cast<const uint64_t*>(slot + u * 64 + (lane & 7) * 8);
+    __syncwarp();
+  }
+  if (acc == 0x1234567890ull) sink[threadIdx.x] = acc;
+}
+
+// Returns random 64 B lines per second (G lines/s) over a `bytes` buffer.
+PROBE_API double probe_gather64(uint64_t bytes, int mode, int u, int threads, int ctas_per_sm, int reps) {
+  uint8_t* buf = nullptr;
+  uint64_t* sink = nullptr;
+  if (cudaMalloc(&buf, bytes) != cudaSuccess) return -1;
+  cudaMalloc(&sink, 1024 * 8);
+  cudaMemset(buf, 1, bytes);
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const uint64_t nlines = bytes / 64, iters = 64;
+  const unsigned grid = sms * ctas_per_sm;
+  const size_t smem = mode == 1 ? size_t(threads) * u * 64 : 0;
+  auto launch = [&](int r) {
+    if (mode == 0) {
+      switch (u) {
+        case 1: gather64_ldg<1><<<grid, threads>>>(buf, nlines, iters, r, sink); break;
+        case 2: gather64_ldg<2><<<grid, threads>>>(buf, nlines, iters, r, sink); break;
+        case 4: gather64_ldg<4><<<grid, threads>>>(buf, nlines, iters, r, sink); break;
+        default: gather64_ldg<8><<<grid, threads>>>(buf, nlines, iters, r, sink); break;
+      }
+    } else {
+      switch (u) {
+        case 1: cudaFuncSetAttribute(gather64_tma<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+                gather64_tma<1><<<grid, threads, smem>>>(buf, nlines, iters, r, sink); break;
+        case 2: cudaFuncSetAttribute(gather64_tma<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+                gather64_tma<2><<<grid, threads, smem>>>(buf, nlines, iters, r, sink); break;
+        case 4: cudaFuncSetAttribute(gather64_tma<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+                gather64_tma<4><<<grid, threads, smem>>>(buf, nlines, iters, r, sink); break;
+        default: cudaFuncSetAttribute(gather64_tma<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+                gather64_tma<8><<<grid, threads, smem>>>(buf, nlines, iters, r, sink); break;
+      }
+    }
+  };
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  float best_ms = 1e30f;
+  for (int r = 0; r < reps + 1; ++r) {
+    cudaEventRecord(a);
+    launch(r);
+    cudaEventRecord(b);
+    cudaEventSynchronize(b);
+    float ms = 0;
+    cudaEventElapsedTime(&ms, a, b);
+    if (r > 0 && ms < best_ms) best_ms = ms;
+  }
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  cudaFree(buf);
+  cudaFree(sink);
+  if (cudaGetLastError() != cudaSuccess) return -2;
+  const double lines = mode == 0 ? double(grid) * threads / 2 * iters * u : double(grid) * threads * iters * u;
+  return lines / (best_ms * 1e-3) / 1e9;
+}
