@@ -237,6 +237,19 @@ def measure_h2d_gbs():
     return best
 
 
+def probe_line_rate(nbytes=8 << 30):
+    """G random 64 B lines/s from a DRAM-resident buffer (tools/probe.cu probe_gather64)."""
+    try:
+        import ctypes as C
+        L = C.CDLL(os.path.join(ROOT, "tools", "libhbtprobe.so"))
+        L.probe_gather64.restype = C.c_double
+        L.probe_gather64.argtypes = [C.c_uint64, C.c_int, C.c_int, C.c_int, C.c_int, C.c_int]
+        v = L.probe_gather64(nbytes, 0, 2, 1024, 1, 3)
+        return v if v > 0 else None
+    except OSError:
+        return None
+
+
 def probe_l2_gbs(chunk, nbytes=32 << 20):
     """All-SM random reads of `chunk`-byte aligned chunks over an `nbytes` buffer
     (32 MB: L2-resident; 1 GB: every read misses, i.e. the random-DRAM rate)."""
@@ -552,6 +565,10 @@ def run_hbt(args):
     # random 64 B reads over 1 GB (8x the L2): the rate DRAM sustains for the leaf-line access
     # pattern (row activations, not bytes, bind it) -- context beside the HBM copy peak
     dram_rand64 = probe_l2_gbs(64, 1 << 30) if rank == 0 else None
+    # random 64 B LINE reads (lane pairs, 256-bit loads) from an 8 GB buffer: the rate the HBM
+    # serves the leaf-line access of the bucketed item search (tools/probe.cu probe_gather64;
+    # saturates with 512 lines in flight per SM, profiles/r02s_gather64_probe.jsonl)
+    line_rate = probe_line_rate() if rank == 0 else None
     # NVLink (SURVEY 8(d) BW_NVL) for the sharded config's a2a term, measured in this run
     a2a_gbs = probe_a2a_gbs(d) if args.config == "c4" else None
 
@@ -656,6 +673,10 @@ def run_hbt(args):
                 "frac_of_8tbs_spec": round(hbm_ach / 8000.0, 4),
                 "random_64b_read_probe_gbs": round(dram_rand64, 1) if dram_rand64 else None,
                 "frac_of_random_64b_probe": round(hbm_ach / dram_rand64, 4) if dram_rand64 else None,
+                # every query reads >= 1 random leaf line: queries/s of the kernel against the
+                # random-line rate of the HBM measured in this run (the access-rate roof)
+                "random_line_probe_glines_per_s": round(line_rate, 2) if line_rate else None,
+                "frac_of_random_line_rate": round(m / t_kernel / 1e9 / line_rate, 4) if line_rate else None,
                 "model": model_desc}
     if args.config == "c4" and world > 1:
         a2a_b = (world - 1) / world * (w + 8 + w)
