@@ -771,7 +771,21 @@ struct Launch {
       attr_set = true;
     }
     ItemDir dd = d;
-    dd.rounds = item_rounds(m, t->num_sms, TH, t->cfg.item_rounds ? t->cfg.item_rounds : 16);
+    // Warp rounds per work item: 16, or 8 when the leaf lines the in-flight items reach
+    // (one item per SM, each anywhere in its bucket's leaf range) exceed twice the L2:
+    // smaller items keep the concurrently searched buckets -- and the DRAM rows their leaf
+    // reads open -- closer together.  c4: 148 items x 16 K queries reach ~300 MB of leaf
+    // lines, 8 rounds: item search 8.9 -> 8.1-8.3 ms (4 rounds: 8.9, the per-item directory
+    // copy is exposed); c5 (74 MB) keeps 16.  Random-line probe over a sliding window:
+    // 36 G lines/s over 512 MB, 44 over 128 MB, 59 over 32 MB (profiles/r02s_*).
+    uint32_t rcap = t->cfg.item_rounds;
+    if (!rcap) {
+      static int l2 = 0;
+      if (!l2) HBT_CUDA_TRY(cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, t->device));
+      const double reach = double(t->num_sms) * TH * 16 / double(m) * double(t->leaf_bytes);
+      rcap = reach > 2.0 * l2 ? 8 : 16;
+    }
+    dd.rounds = item_rounds(m, t->num_sms, TH, rcap);
     // the walk resolves directory ties (it detects them on the 256-bit leaf read)
     dd.fix = lt.leaf256 != 0;
     const size_t smem = (size_t(d.cap) + kT16) * 2 + (size_t(d.B) + 1) * 12;

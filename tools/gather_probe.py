@@ -18,3 +18,10 @@ for mode, u, th, cps in [(0, 1, 1024, 1), (0, 2, 1024, 1), (0, 4, 1024, 1), (0, 
     inflight = th * cps * u // (2 if mode == 0 else 1)
     print(json.dumps({"mode": ["ldg256_pair", "tma_bulk64"][mode], "u": u, "threads": th, "ctas_per_sm": cps,
                       "lines_in_flight_per_sm": inflight, "glines_per_s": round(r, 2)}), flush=True)
+# windowed: all SMs draw random lines from one sliding window (DRAM-row / L2 locality)
+lib.probe_gather64_window.restype = ctypes.c_double
+lib.probe_gather64_window.argtypes = [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_int]
+for wmb in (0, 2048, 512, 128, 64, 32, 16, 8, 2):
+    r = lib.probe_gather64_window(B, wmb << 20, 3)
+    print(json.dumps({"mode": "ldg256_pair_window", "window_mb": wmb or "whole 8 GB", "lines_in_flight_per_sm": 1024,
+                      "glines_per_s": round(r, 2)}), flush=True)

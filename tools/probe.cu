@@ -408,9 +408,12 @@ __device__ __forceinline__ void pb_wait(uint64_t* bar, uint32_t parity) {
       : "memory");
 }
 
+// wlines > 0: every line of iteration `it` lies in the window of wlines lines starting at
+// (it * wlines) mod nlines (all SMs move through the buffer window by window: locality
+// at the DRAM-row / L2 level, not within a warp)
 template <int U>
 __global__ void gather64_ldg(const uint8_t* __restrict__ buf, uint64_t nlines, uint64_t iters, uint64_t seed,
-                             uint64_t* __restrict__ sink) {
+                             uint64_t* __restrict__ sink, uint64_t wlines = 0) {
   const int lane = threadIdx.x & 31, k = lane & 1;
   const uint64_t gid = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 1;
   uint64_t state = mix64(gid ^ seed), acc = 0;
@@ -419,7 +422,9 @@ __global__ void gather64_ldg(const uint8_t* __restrict__ buf, uint64_t nlines, u
 #pragma unroll
     for (int u = 0; u < U; ++u) {
       state = mix64(state);
-      const uint8_t* p = buf + __umul64hi(state, nlines) * 64 + k * 32;
+      const uint64_t line = wlines ? ((it * wlines) % (nlines - wlines + 1)) + __umul64hi(state, wlines)
+                                   : __umul64hi(state, nlines);
+      const uint8_t* p = buf + line * 64 + k * 32;
       asm volatile("ld.global.nc.v4.u64 {%0, %1, %2, %3}, [%4];"
                    : "=l"(v[u][0]), "=l"(v[u][1]), "=l"(v[u][2]), "=l"(v[u][3])
                    : "l"(p));
@@ -513,4 +518,36 @@ PROBE_API double probe_gather64(uint64_t bytes, int mode, int u, int threads, in
   if (cudaGetLastError() != cudaSuccess) return -2;
   const double lines = mode == 0 ? double(grid) * threads / 2 * iters * u : double(grid) * threads * iters * u;
   return lines / (best_ms * 1e-3) / 1e9;
+}
+
+// The windowed form of probe_gather64 mode 0 (u = 2, 1024 threads, 1 CTA per SM): G lines/s.
+PROBE_API double probe_gather64_window(uint64_t bytes, uint64_t window_bytes, int reps) {
+  uint8_t* buf = nullptr;
+  uint64_t* sink = nullptr;
+  if (cudaMalloc(&buf, bytes) != cudaSuccess) return -1;
+  cudaMalloc(&sink, 1024 * 8);
+  cudaMemset(buf, 1, bytes);
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const uint64_t nlines = bytes / 64, iters = 64, wl = window_bytes / 64;
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  float best_ms = 1e30f;
+  for (int r = 0; r < reps + 1; ++r) {
+    cudaEventRecord(a);
+    gather64_ldg<2><<<sms, 1024>>>(buf, nlines, iters, r, sink, wl);
+    cudaEventRecord(b);
+    cudaEventSynchronize(b);
+    float ms = 0;
+    cudaEventElapsedTime(&ms, a, b);
+    if (r > 0 && ms < best_ms) best_ms = ms;
+  }
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  cudaFree(buf);
+  cudaFree(sink);
+  if (cudaGetLastError() != cudaSuccess) return -2;
+  return double(sms) * 1024 / 2 * iters * 2 / (best_ms * 1e-3) / 1e9;
 }
