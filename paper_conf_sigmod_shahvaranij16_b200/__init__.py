@@ -23,7 +23,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libhbt.so")
+# HBT_LIB_ALT (A/B experiments only): another in-tree build of the same library
+LIB_PATH = os.path.join(_HERE, os.environ.get("HBT_LIB_ALT", "libhbt.so"))
 
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, EUNSUPPORTED = 0, -1, -2, -3, -4, -5
 IMPLICIT, REGULAR, KEY32, KEY64 = 0x0, 0x1, 0x00, 0x10

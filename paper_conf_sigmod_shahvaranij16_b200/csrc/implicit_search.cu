@@ -593,18 +593,31 @@ implicit_search_cdir_kernel(const uint8_t* __restrict__ inner, const uint8_t* __
   const int g = lane / C::G, k = lane % C::G;
   const unsigned gmask = ((1u << C::G) - 1u) << (g * C::G);
   uint32_t parity = 0;
+  // the bucket of item `it`: largest b with s_is[b] <= it
+  auto bucket_of_item = [&](uint32_t it) {
+    uint32_t lo = 0, hi = B;
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (s_is[mid] <= it) lo = mid; else hi = mid;
+    }
+    return lo;
+  };
+  // thread 0 holds the NEXT item's bucket record, loaded during the current item (its
+  // global-load latency stays off the item-start path)
+  uint32_t nlo = 0;
+  BucketDir nbd{};
+  if (threadIdx.x == 0 && blockIdx.x < items) {
+    nlo = bucket_of_item(blockIdx.x);
+    nbd = d.bd[nlo];
+  }
   for (uint32_t it = blockIdx.x; it < items; it += gridDim.x) {
     if (threadIdx.x == 0) {
-      uint32_t lo = 0, hi = B;  // the bucket: largest b with s_is[b] <= it
-      while (hi - lo > 1) {
-        const uint32_t mid = (lo + hi) >> 1;
-        if (s_is[mid] <= it) lo = mid; else hi = mid;
-      }
+      const uint32_t lo = nlo;
+      const BucketDir bd = nbd;
       const uint64_t nb = s_is[lo + 1] - s_is[lo], j = it - s_is[lo];
       const uint64_t c0 = s_bs[lo], cnt = s_bs[lo + 1] - c0;
       s_p[0] = c0 + (cnt * j) / nb;
       s_p[1] = c0 + (cnt * (j + 1)) / nb - 1;
-      const BucketDir bd = d.bd[lo];
       s_bd = bd;
       // the previous item's reads of the directory are ordered before this copy by the
       // barrier that ended it; the proxy fence orders them for the async (bulk copy) proxy
@@ -613,18 +626,23 @@ implicit_search_cdir_kernel(const uint8_t* __restrict__ inner, const uint8_t* __
       mbar_expect_tx(&bar, eb + kT16 * 2u);
       bulk_g2s(s_E, d.E16 + bd.off16, eb, &bar);
       bulk_g2s(s_T, d.T16 + uint64_t(lo) * kT16, kT16 * 2u, &bar);
+      if (it + gridDim.x < items) {
+        nlo = bucket_of_item(it + gridDim.x);
+        nbd = d.bd[nlo];
+      }
     }
     __syncthreads();
     const uint64_t p0 = s_p[0], p1 = s_p[1];
     const uint64_t u0 = s_bd.u0;
     const uint32_t cnt = s_bd.cnt;
-    mbar_wait(&bar, parity);
-    parity ^= 1u;
+    // the first round's queries are requested before waiting for the directory copy
     K nextq;
     {
       const uint64_t i = p0 + uint64_t(wid) * 32 + lane;
       nextq = i <= p1 ? ldcs(queries + i) : key_max<K>();
     }
+    mbar_wait(&bar, parity);
+    parity ^= 1u;
 #pragma unroll 1
     for (int r = 0; r < int(d.rounds); ++r) {
       const uint64_t base = p0 + (uint64_t(r) * (THREADS / 32) + wid) * 32;
