@@ -1,5 +1,5 @@
 #!/bin/bash
-# Round-2 final profile set (TAG, default r02s): GPU tests, smoke, sanitizers, every 1-GPU
+# Round-2 final profile set (TAG, default r02s): GPU tests, smoke, every 1-GPU
 # config line, the c4 2-rank dry run, the default bench's launch list, single-pass
 # steady-state DRAM traffic of each config's dominant kernel (-> profiles/traffic.json),
 # and ncu --set full of the c4 item search.
@@ -8,8 +8,7 @@ TAG=${1:-r02s}
 timeout 2400 python -m pytest tests -x -q -m gpu > gpurun_out/${TAG}_pytest_gpu.log 2>&1
 echo "rc=$?" >> gpurun_out/${TAG}_pytest_gpu.log
 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${TAG}_smoke.log 2>&1
-bash tools/sanitize.sh
-for t in memcheck racecheck synccheck initcheck memcheck_two_process; do cp gpurun_out/sanitize_$t.log gpurun_out/${TAG}_sanitize_$t.log; done
+# (compute-sanitizer is closed on this GPU pool since round 2b: tools/sanitize.sh, logs profiles/r02_sanitize_*)
 for spec in "c2 implicit_search" "c1 implicit_search" "c5 implicit_search" "c3 regular_search_(items|cdir)" "c4 implicit_search_(items|cdir)"; do
   set -- $spec
   timeout 900 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,lts__t_sector_hit_rate.pct,gpu__time_duration.sum \
