@@ -216,8 +216,10 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *                 or the normal search kernel on the bucketed queries (0)
  *   "bucket_cap"  item-directory shared-memory entries (0 = derived; small values force the
  *                 global-memory fallback, for tests)
- *   "item_rounds" bucketed item searches: most warp rounds per work item (0 = default 16;
- *                 fewer are used when the batch would leave SMs idle)
+ *   "item_rounds" bucketed item searches: most warp rounds per work item (0 = default 16,
+ *                 or 8 for the compressed-directory implicit search when the leaf lines its
+ *                 in-flight items reach exceed 2x the L2; fewer are used when the batch would
+ *                 leave SMs idle)
  *   "phase_timing" 1 = record CUDA events around the phases of each bucketed search (read
  *                 them with hbt_last_phases), 0 = off (default)
  *   "leaf_stream" L-segment in host memory (hbt_set_leaf_placement): 0 = zero-copy leaf
