@@ -542,11 +542,36 @@ def time_e2e(work, steps):
         one()
     el = d.max(time.perf_counter() - t0)
     qps = d.world * m * steps / el
+    # the host link alone: the step's H2D and D2H bytes copied concurrently on two streams
+    # (no search) -- the ceiling the end-to-end number runs against
+    link = None
+    try:
+        dq = torch.empty_like(work.q)
+        sa, sb = torch.cuda.Stream(), torch.cuda.Stream()
+        best = 1e30
+        for _ in range(3):
+            torch.cuda.synchronize()
+            t1 = time.perf_counter()
+            with torch.cuda.stream(sa):
+                dq.copy_(hq, non_blocking=True)
+            with torch.cuda.stream(sb):
+                hp.copy_(work.out_pos, non_blocking=True)
+                hv.copy_(work.out_val, non_blocking=True)
+            torch.cuda.synchronize()
+            best = min(best, time.perf_counter() - t1)
+        del dq
+        best = d.max(best)
+        link = {"value": round(d.world * m / best / 1e6, 2), "unit": "M queries/s",
+                "frac": round(qps / (d.world * m / best), 4),
+                "what": "the step's H2D (queries) and D2H (pos|found, values) bytes copied concurrently on two "
+                        "streams, no search: the host-link ceiling of e2e"}
+    except RuntimeError:
+        link = None
     api = ("H2D + hbt_search_sharded + D2H (pinned host buffers)" if sharded else
            "hbt_search_host (pinned host buffers; chunks of 2^%d queries: H2D, search, D2H pipelined over %d "
            "streams)" % (work.host_chunk_log2, work.host_bufs))
     return {"value": round(qps / 1e6, 2), "unit": "M queries/s", "h2d_bytes_per_step": m * w,
-            "d2h_bytes_per_step": m * (8 + w), "api": api}
+            "d2h_bytes_per_step": m * (8 + w), "api": api, "link_ceiling": link}
 
 
 def run_hbt(args):
