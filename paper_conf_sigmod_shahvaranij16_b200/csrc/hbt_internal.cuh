@@ -89,6 +89,7 @@ struct SearchConfig {
   uint32_t l2_hint = 4;          // implicit search: L2 eviction-priority hints (LevelTable::l2_hint);
                                  // 4 = auto: leaf lines evict-first iff the I-segment fits in L2 / 4
   uint32_t item_l2_hint = 1;     // implicit bucketed item search (c4 item search 10.96 -> 9.50 ms)
+  uint32_t item_qpf = 1;         // see ItemDir::qpf
   uint32_t item_cdir = 1;        // item directory in the compressed per-bucket form (ItemDir::bd): 0 = never,
                                  // 1 = where it reaches a deeper level (regular: always fits-permitting),
                                  // 2 = always (implicit: even at the same level)
@@ -125,6 +126,7 @@ struct ItemDir {
   const uint16_t* E16 = nullptr;
   const uint16_t* T16 = nullptr;
   bool fix = false;  // single ties of the truncated maxima resolved by the walk
+  uint32_t qpf = 0;  // compressed-directory items: each lane prefetches its query of the round after next into the L2
 };
 
 constexpr uint32_t kT16 = 4104;  // per-bucket prefix table: 2^12 + 1 entries, padded to 16 B

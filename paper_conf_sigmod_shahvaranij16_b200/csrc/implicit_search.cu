@@ -651,6 +651,11 @@ implicit_search_cdir_kernel(const uint8_t* __restrict__ inner, const uint8_t* __
       {
         const uint64_t i = base + (THREADS / 32) * 32 + lane;
         nextq = (r + 1 < int(d.rounds) && i <= p1) ? ldcs(queries + i) : key_max<K>();
+        // the query of the round after next into the L2 now (no register held): the query
+        // loaded one round ahead still waited on DRAM (ncu: 13 % of the stalls; c4 item
+        // search -1..-2 %, c5 -6 %, profiles/r02s_c4_qpf2.jsonl)
+        if (d.qpf && r + 2 < int(d.rounds) && i + (THREADS / 32) * 32 <= p1)
+          asm volatile("prefetch.global.L2 [%0];" ::"l"(queries + i + (THREADS / 32) * 32));
       }
       // single ties are resolved by the walk (descend_and_store FIX), not by a dependent
       // read of the exact maxima that would stall the whole warp
@@ -806,6 +811,7 @@ struct Launch {
     dd.rounds = item_rounds(m, t->num_sms, TH, rcap);
     // the walk resolves directory ties (it detects them on the 256-bit leaf read)
     dd.fix = lt.leaf256 != 0;
+    dd.qpf = t->cfg.item_qpf;
     const size_t smem = (size_t(d.cap) + kT16) * 2 + (size_t(d.B) + 1) * 12;
     kern<<<t->num_sms, TH, smem, s>>>((const uint8_t*)t->d_inner, (const uint8_t*)t->d_inner_idx,
                                      (const uint8_t*)t->d_leaf, dd, (const K*)q, m, pf, (K*)v, lt, t->n);

@@ -704,6 +704,9 @@ regular_search_cdir_kernel(const RView rv, const ItemDir d, const K* __restrict_
       {
         const uint64_t i = base + (THREADS / 32) * 32 + lane;
         nextq = (r + 1 < int(d.rounds) && i <= p1) ? ldcs(queries + i) : key_max<K>();
+        // the query of the round after next into the L2 now (as implicit_search_cdir_kernel)
+        if (d.qpf && r + 2 < int(d.rounds) && i + (THREADS / 32) * 32 <= p1)
+          asm volatile("prefetch.global.L2 [%0];" ::"l"(queries + i + (THREADS / 32) * 32));
       }
       const uint32_t a = lower_bound16(s_E, s_T, cnt, myq, K(s_bd.lo), s_bd.sh, s_bd.top, s_bd.ssh, s_bd.esh,
                                        gM + e0, true);
@@ -862,6 +865,7 @@ int search_cdir_launch(const hbt_tree* t, const void* q, uint64_t m, uint64_t* p
   }
   ItemDir dd = d;
   dd.rounds = item_rounds(m, t->num_sms, TH, t->cfg.item_rounds ? t->cfg.item_rounds : 16);
+  dd.qpf = t->cfg.item_qpf;
   kern<<<t->num_sms, TH, smem, s>>>(rv, dd, (const K*)q, m, pf, (K*)v);
   HBT_CUDA_TRY(cudaGetLastError());
   return HBT_OK;
