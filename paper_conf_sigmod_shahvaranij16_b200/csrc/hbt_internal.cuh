@@ -126,7 +126,8 @@ struct ItemDir {
   const uint16_t* E16 = nullptr;
   const uint16_t* T16 = nullptr;
   bool fix = false;  // single ties of the truncated maxima resolved by the walk
-  uint32_t qpf = 0;  // compressed-directory items: each lane prefetches its query of the round after next into the L2
+  uint32_t qpf = 0;  // compressed-directory items: each lane prefetches its query qpf rounds after the next into
+                     // the L2 (0 = off; 1 measured best, 2-4 slower: profiles/r02s_item_query_prefetch_ab.jsonl)
 };
 
 constexpr uint32_t kT16 = 4104;  // per-bucket prefix table: 2^12 + 1 entries, padded to 16 B

@@ -654,8 +654,8 @@ implicit_search_cdir_kernel(const uint8_t* __restrict__ inner, const uint8_t* __
         // the query of the round after next into the L2 now (no register held): the query
         // loaded one round ahead still waited on DRAM (ncu: 13 % of the stalls; c4 item
         // search -1..-2 %, c5 -6 %, profiles/r02s_c4_qpf2.jsonl)
-        if (d.qpf && r + 2 < int(d.rounds) && i + (THREADS / 32) * 32 <= p1)
-          asm volatile("prefetch.global.L2 [%0];" ::"l"(queries + i + (THREADS / 32) * 32));
+        if (d.qpf && r + 1 + int(d.qpf) < int(d.rounds) && i + d.qpf * (THREADS / 32) * 32 <= p1)
+          asm volatile("prefetch.global.L2 [%0];" ::"l"(queries + i + d.qpf * (THREADS / 32) * 32));
       }
       // single ties are resolved by the walk (descend_and_store FIX), not by a dependent
       // read of the exact maxima that would stall the whole warp

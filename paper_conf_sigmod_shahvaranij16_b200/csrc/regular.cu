@@ -705,8 +705,8 @@ regular_search_cdir_kernel(const RView rv, const ItemDir d, const K* __restrict_
         const uint64_t i = base + (THREADS / 32) * 32 + lane;
         nextq = (r + 1 < int(d.rounds) && i <= p1) ? ldcs(queries + i) : key_max<K>();
         // the query of the round after next into the L2 now (as implicit_search_cdir_kernel)
-        if (d.qpf && r + 2 < int(d.rounds) && i + (THREADS / 32) * 32 <= p1)
-          asm volatile("prefetch.global.L2 [%0];" ::"l"(queries + i + (THREADS / 32) * 32));
+        if (d.qpf && r + 1 + int(d.qpf) < int(d.rounds) && i + d.qpf * (THREADS / 32) * 32 <= p1)
+          asm volatile("prefetch.global.L2 [%0];" ::"l"(queries + i + d.qpf * (THREADS / 32) * 32));
       }
       const uint32_t a = lower_bound16(s_E, s_T, cnt, myq, K(s_bd.lo), s_bd.sh, s_bd.top, s_bd.ssh, s_bd.esh,
                                        gM + e0, true);
