@@ -76,13 +76,16 @@ def test_bucketed_scaled_workload(hbt, layout, F, items, cap, leaf256, dir32):
     t.set_param("item_cdir", dir32)
     for slice_bytes in (1 << 16, 1 << 20, 1 << 22):
         t.set_param("bucket_slice", slice_bytes)
-        for qpf in (0, 1):  # default and single-round work items
-            t.set_param("item_rounds", 1 if qpf else 0)
-            for hint in (0, 1, 3):  # L2 eviction-priority hints on the item search's loads
+        for one_round in (0, 1):  # default and single-round work items
+            t.set_param("item_rounds", 1 if one_round else 0)
+            for hint, qpf in ((0, 0), (1, 1), (3, 3)):  # L2 hints / query-prefetch distance
                 if layout == "implicit":
                     t.set_param("item_l2_hint", hint)
+                t.set_param("item_qpf", qpf)
                 pf, val = gpu_search(t, q, 8)
-                assert np.array_equal(pf, epf) and np.array_equal(val, ev), (layout, slice_bytes, qpf, hint)
+                assert np.array_equal(pf, epf) and np.array_equal(val, ev), (layout, slice_bytes, one_round, hint,
+                                                                             qpf)
+    t.set_param("item_qpf", 1)
     t.set_param("bucket", 0)
     for hint in (0, 1, 2, 3, 4):  # plain search with the same hints (4 = auto)
         t.set_param("l2_hint", hint)
