@@ -554,6 +554,13 @@ implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* _
 // exactly its bucket's directory: one elected thread moves the entries and the prefix
 // table into shared memory with bulk copies (cp.async.bulk, completion on an mbarrier).
 // Ties of truncated values: lower_bound16 (item_dir.cuh) and descend_and_store FIX.
+// Items are handed off on two mbarriers instead of CTA barriers: every warp arrives on
+// `empty` right after its LAST directory lookup of an item; thread 0 waits for all of
+// them, publishes the next item (its range and bucket record, double-buffered by item
+// parity) and starts its directory copy, which completes `full`.  A warp starts the next
+// item as soon as `full` completes -- it does not wait for the other warps' last walks
+// (leaf reads) of the previous item (c4 item search -1..-5 %, c5 -3 %,
+// profiles/r02s_item_pipe_ab.jsonl).
 template <typename K, int F, int THREADS>
 __global__ void __launch_bounds__(THREADS)
 implicit_search_cdir_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ inner_idx,
@@ -562,29 +569,29 @@ implicit_search_cdir_kernel(const uint8_t* __restrict__ inner, const uint8_t* __
                             uint64_t n) {
   using C = Cfg<K, F>;
   constexpr int QPG = 32 / C::NG;
+  constexpr int NW = THREADS / 32;
   const uint64_t W = uint64_t(THREADS) * d.rounds;
   const uint32_t B = d.B;
   extern __shared__ __align__(16) uint8_t smem[];
-  // [E16: cap entries | T16: kT16 | bucket starts: B + 1 u64 | item starts: B + 1]
   uint16_t* s_E = reinterpret_cast<uint16_t*>(smem);
   uint16_t* s_T = s_E + d.cap;
   uint64_t* s_bs = reinterpret_cast<uint64_t*>(s_T + kT16);
   uint32_t* s_is = reinterpret_cast<uint32_t*>(s_bs + B + 1);
-  __shared__ uint64_t bar;
+  __shared__ uint64_t full_bar, empty_bar;
   __shared__ uint32_t s_tmp[32];
-  __shared__ uint64_t s_p[2];
-  __shared__ BucketDir s_bd;
+  __shared__ uint64_t s_p[2][2];
+  __shared__ BucketDir s_bd[2];
   const K* gM = static_cast<const K*>(d.M);
   for (uint32_t i = threadIdx.x; i <= B; i += THREADS) s_bs[i] = d.bstart[i];
   __syncthreads();
-  // items per bucket, then their starts (B <= 2 * THREADS)
   for (uint32_t b = threadIdx.x; b < B; b += THREADS) s_is[b] = uint32_t((s_bs[b + 1] - s_bs[b] + W - 1) / W);
   __syncthreads();
   const uint32_t last = s_is[B - 1];
   block_exclusive_scan<THREADS>(s_is, s_is, B, s_tmp);
   if (threadIdx.x == 0) {
     s_is[B] = s_is[B - 1] + last;
-    mbar_init(&bar, 1);
+    mbar_init(&full_bar, 1);
+    mbar_init(&empty_bar, NW);
     fence_mbar_init();
   }
   __syncthreads();
@@ -592,8 +599,6 @@ implicit_search_cdir_kernel(const uint8_t* __restrict__ inner, const uint8_t* __
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int g = lane / C::G, k = lane % C::G;
   const unsigned gmask = ((1u << C::G) - 1u) << (g * C::G);
-  uint32_t parity = 0;
-  // the bucket of item `it`: largest b with s_is[b] <= it
   auto bucket_of_item = [&](uint32_t it) {
     uint32_t lo = 0, hi = B;
     while (hi - lo > 1) {
@@ -602,65 +607,61 @@ implicit_search_cdir_kernel(const uint8_t* __restrict__ inner, const uint8_t* __
     }
     return lo;
   };
-  // thread 0 holds the NEXT item's bucket record, loaded during the current item (its
-  // global-load latency stays off the item-start path)
-  uint32_t nlo = 0;
-  BucketDir nbd{};
-  if (threadIdx.x == 0 && blockIdx.x < items) {
-    nlo = bucket_of_item(blockIdx.x);
-    nbd = d.bd[nlo];
-  }
-  for (uint32_t it = blockIdx.x; it < items; it += gridDim.x) {
-    if (threadIdx.x == 0) {
-      const uint32_t lo = nlo;
-      const BucketDir bd = nbd;
-      const uint64_t nb = s_is[lo + 1] - s_is[lo], j = it - s_is[lo];
-      const uint64_t c0 = s_bs[lo], cnt = s_bs[lo + 1] - c0;
-      s_p[0] = c0 + (cnt * j) / nb;
-      s_p[1] = c0 + (cnt * (j + 1)) / nb - 1;
-      s_bd = bd;
-      // the previous item's reads of the directory are ordered before this copy by the
-      // barrier that ended it; the proxy fence orders them for the async (bulk copy) proxy
-      fence_proxy_async_smem();
-      const uint32_t eb = ((bd.cnt + 7u) & ~7u) * 2u;
-      mbar_expect_tx(&bar, eb + kT16 * 2u);
-      bulk_g2s(s_E, d.E16 + bd.off16, eb, &bar);
-      bulk_g2s(s_T, d.T16 + uint64_t(lo) * kT16, kT16 * 2u, &bar);
-      if (it + gridDim.x < items) {
-        nlo = bucket_of_item(it + gridDim.x);
-        nbd = d.bd[nlo];
+  // thread 0: the item `it` of bucket lo into metadata slot x, and its directory copy
+  // (the expect_tx arrive releases the metadata writes to the phase's waiters)
+  auto issue = [&](uint32_t it, int x) {
+    const uint32_t lo = bucket_of_item(it);
+    const BucketDir bd = d.bd[lo];
+    const uint64_t nb = s_is[lo + 1] - s_is[lo], j = it - s_is[lo];
+    const uint64_t c0 = s_bs[lo], cnt = s_bs[lo + 1] - c0;
+    s_p[x][0] = c0 + (cnt * j) / nb;
+    s_p[x][1] = c0 + (cnt * (j + 1)) / nb - 1;
+    s_bd[x] = bd;
+    fence_proxy_async_smem();
+    const uint32_t eb = ((bd.cnt + 7u) & ~7u) * 2u;
+    mbar_expect_tx(&full_bar, eb + kT16 * 2u);
+    bulk_g2s(s_E, d.E16 + bd.off16, eb, &full_bar);
+    bulk_g2s(s_T, d.T16 + uint64_t(lo) * kT16, kT16 * 2u, &full_bar);
+  };
+  if (threadIdx.x == 0 && blockIdx.x < items) issue(blockIdx.x, 0);
+  uint32_t kk = 0;
+  for (uint32_t it = blockIdx.x; it < items; it += gridDim.x, ++kk) {
+    const int x = int(kk & 1u);
+    mbar_wait(&full_bar, kk & 1u);
+    const uint64_t p0 = s_p[x][0], p1 = s_p[x][1];
+    const uint64_t u0 = s_bd[x].u0;
+    const uint32_t cnt = s_bd[x].cnt;
+    const uint64_t wb0 = p0 + uint64_t(wid) * 32;
+    const int nr = wb0 > p1 ? 0 : int(min(uint64_t(d.rounds), (p1 - wb0) / (NW * 32) + 1));
+    // past this warp's last directory lookup: release the directory buffer; thread 0 waits
+    // for every warp, then publishes the next item
+    auto done_with_dir = [&]() {
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty_bar);
+      if (threadIdx.x == 0) {
+        mbar_wait(&empty_bar, kk & 1u);
+        if (it + gridDim.x < items) issue(it + gridDim.x, x ^ 1);
       }
-    }
-    __syncthreads();
-    const uint64_t p0 = s_p[0], p1 = s_p[1];
-    const uint64_t u0 = s_bd.u0;
-    const uint32_t cnt = s_bd.cnt;
-    // the first round's queries are requested before waiting for the directory copy
+    };
+    if (nr == 0) done_with_dir();
     K nextq;
     {
-      const uint64_t i = p0 + uint64_t(wid) * 32 + lane;
+      const uint64_t i = wb0 + lane;
       nextq = i <= p1 ? ldcs(queries + i) : key_max<K>();
     }
-    mbar_wait(&bar, parity);
-    parity ^= 1u;
 #pragma unroll 1
-    for (int r = 0; r < int(d.rounds); ++r) {
-      const uint64_t base = p0 + (uint64_t(r) * (THREADS / 32) + wid) * 32;
-      if (base > p1) break;
+    for (int r = 0; r < nr; ++r) {
+      const uint64_t base = wb0 + uint64_t(r) * (NW * 32);
       const K myq = nextq;
       {
-        const uint64_t i = base + (THREADS / 32) * 32 + lane;
-        nextq = (r + 1 < int(d.rounds) && i <= p1) ? ldcs(queries + i) : key_max<K>();
-        // the query of the round after next into the L2 now (no register held): the query
-        // loaded one round ahead still waited on DRAM (ncu: 13 % of the stalls; c4 item
-        // search -1..-2 %, c5 -6 %, profiles/r02s_c4_qpf2.jsonl)
-        if (d.qpf && r + 1 + int(d.qpf) < int(d.rounds) && i + d.qpf * (THREADS / 32) * 32 <= p1)
-          asm volatile("prefetch.global.L2 [%0];" ::"l"(queries + i + d.qpf * (THREADS / 32) * 32));
+        const uint64_t i = base + NW * 32 + lane;
+        nextq = (r + 1 < nr && i <= p1) ? ldcs(queries + i) : key_max<K>();
+        if (d.qpf && r + 1 + int(d.qpf) < nr && i + d.qpf * (NW * 32) <= p1)
+          asm volatile("prefetch.global.L2 [%0];" ::"l"(queries + i + d.qpf * (NW * 32)));
       }
-      // single ties are resolved by the walk (descend_and_store FIX), not by a dependent
-      // read of the exact maxima that would stall the whole warp
-      const uint32_t a = lower_bound16(s_E, s_T, cnt, myq, K(s_bd.lo), s_bd.sh, s_bd.top, s_bd.ssh, s_bd.esh,
-                                       gM + u0, d.fix);
+      const uint32_t a = lower_bound16(s_E, s_T, cnt, myq, K(s_bd[x].lo), s_bd[x].sh, s_bd[x].top, s_bd[x].ssh,
+                                       s_bd[x].esh, gM + u0, d.fix);
+      if (r == nr - 1) done_with_dir();
       const uint32_t mynode = uint32_t(u0) + (a < cnt ? a : cnt - 1);
       K q[QPG];
       uint32_t node[QPG];
@@ -674,7 +675,6 @@ implicit_search_cdir_kernel(const uint8_t* __restrict__ inner, const uint8_t* __
                                                p1 + 1, n, d.pos_base, out_pf, out_v,
                                                d.fix ? uint32_t(min((u0 + cnt) * d.span, d.U) - 1) : 0u);
     }
-    __syncthreads();
   }
 }
 
