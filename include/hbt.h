@@ -242,6 +242,8 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *                 per-bucket prefix table, items cut inside one bucket; regular trees: the
  *                 leaf lines): 0 = never, 1 = where it reaches a deeper tree level than 8 B
  *                 keys and fits (default), 2 = always where it fits
+ *   "item_qpf"    compressed-directory item searches: each lane prefetches its query this many
+ *                 rounds beyond the next into the L2 (0 = off, 1 = default; 0..6)
  * Variants measured slower were removed (DESIGN.md §8 keeps their numbers).  Unknown
  * names or out-of-range values return HBT_EINVAL. */
 HBT_API int hbt_set_param(hbt_tree* t, const char* name, int64_t value);
