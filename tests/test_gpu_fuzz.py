@@ -5,6 +5,8 @@ mode, per-level read widths, CTA size, bucketing with its slice / item directory
 capacity, L-segment placement and streaming), every output compared with the
 oracle.  Complements the targeted suites: a knob interaction no suite lists still
 has to give the oracle's bits.  Seeded, so a failure reproduces."""
+import os
+
 import numpy as np
 import pytest
 import torch
@@ -15,7 +17,9 @@ from test_oracle_implicit import gen_keys, kmax, query_set
 
 pytestmark = pytest.mark.gpu
 
-CASES = 600
+# HBT_FUZZ_CASES / HBT_FUZZ_SEED widen the sweep for long runs (the defaults are the suite's)
+CASES = int(os.environ.get("HBT_FUZZ_CASES", "600"))
+SEED0 = int(os.environ.get("HBT_FUZZ_SEED", "7000"))
 
 
 @pytest.fixture(scope="module")
@@ -37,7 +41,7 @@ def _queries(k, width, rng, m):
 
 @pytest.mark.parametrize("case", range(CASES))
 def test_random_knob_parity(hbt, case):
-    rng = np.random.default_rng(7000 + case)
+    rng = np.random.default_rng(SEED0 + case)
     layout = "regular" if rng.random() < 0.4 else "implicit"
     width = int(rng.choice([4, 8]))
     F = int(rng.choice([4, 8, 16, 32]))
@@ -65,7 +69,7 @@ def test_random_knob_parity(hbt, case):
             knobs["leaf_stream"] = int(rng.choice([0, 1, 2]))
             knobs["stream_slice"] = int(rng.choice([64, 4096, 0]))
     # L2 eviction-priority hints (own generator: the cases above keep their draws)
-    hrng = np.random.default_rng(case + 7777)
+    hrng = np.random.default_rng(SEED0 + case + 777)
     knobs["l2_hint"] = int(hrng.integers(0, 5))
     knobs["item_l2_hint"] = int(hrng.integers(0, 4))
     knobs["item_rounds"] = int(hrng.choice([0, 1, 3, 16]))
