@@ -22,8 +22,9 @@ torch.distributed.run with N local ranks (127.0.0.1).  When there are more ranks
 than visible GPUs (a dry run of the multi-rank path on one GPU) the ranks share
 the devices round-robin, the process group is gloo and the sharded tree uses the
 host-callback communicator with the fused peer-memory exchange.
-c1/c2/c3/c5 at N > 1 run one replica per rank, each searching its own batch
-(weak scaling, no collective on the data path).
+c1/c2/c3 at N > 1 run one replica per rank, each searching its own batch (weak
+scaling); c5 ("query-batch split at 8 GPUs") splits its 2^26-query batch over the
+replicas (strong scaling); no collective on the data path.
 """
 from __future__ import annotations
 
@@ -326,6 +327,9 @@ def make_work(cfg_name, d, args):
             q = torch.from_numpy(gen.workload_queries(cfg_name, hk).view(np.int32 if w == 4 else np.int64)).cuda()
             qdesc = "Knuth shuffle of the keys (PAPER.md:298)"
         elif c["queries"] == "zipf":
+            # c5 = BASELINE configs[4], "query-batch split at 8 GPUs": the 2^26-query batch is
+            # split over the ranks (2^23 each at 8; strong scaling), every rank holding a replica
+            m = m // world
             hk = gen.keys(n, w, sk)
             r = gen.zipf_ranks(m, n, c["theta"], sq, start=rank * m)
             q = torch.from_numpy(hk[r - 1].view(np.int64)).cuda()
@@ -807,7 +811,7 @@ def run_hbt(args):
             "warmup": max(args.warmup, 3),
             "ms_per_step": round(ms_step, 4),
             "higher_is_better": True,
-            "scaling": "strong" if args.config == "c4" else "weak",
+            "scaling": "strong" if args.config in ("c4", "c5") else "weak",
             "vs_baseline": None,
             "dtype": "u64" if w == 8 else "u32",
             "data": "synthetic (seeded counter-based generators, gen/)",
@@ -845,7 +849,7 @@ def bench_config(args, world):
     from the configuration alone (BASELINE.json configs[], gen.CONFIGS)."""
     c = gen.CONFIGS[args.config]
     w = c["width"]
-    m_total = c["m"] if args.config == "c4" else c["m"] * world
+    m_total = c["m"] if args.config in ("c4", "c5") else c["m"] * world
     qk = {"uniform": "uniform hits with replacement", "stratified": "uniform hits over all keys",
           "uniform_ins": "uniform over key indices [0, n + n_ins) (misses = not-yet-inserted keys)",
           "shuffle": "Knuth shuffle of the keys (PAPER.md:298)",
@@ -1011,7 +1015,7 @@ def run_reference(args):
     line = {
         "impl": "reference", "metric": "lookups/sec (M queries/s)", "value": val, "unit": "M queries/s",
         "n_gpus": world, "steps": steps, "warmup": args.warmup, "ms_per_step": round(el / steps * 1e3, 3),
-        "higher_is_better": True, "scaling": "strong" if args.config == "c4" else "weak", "vs_baseline": None,
+        "higher_is_better": True, "scaling": "strong" if args.config in ("c4", "c5") else "weak", "vs_baseline": None,
         "dtype": "u64" if c["width"] == 8 else "u32", "data": "synthetic (seeded counter-based generators, gen/)",
         "config": bench_config(args, world),
         "cpu_baseline": {"value": val, "unit": "M queries/s", "cores": cores, "kind": "oracle",
