@@ -474,6 +474,7 @@ int hbt_set_param(hbt_tree* t, const char* name, int64_t value) {
   else if (n == "l2_hint" && value >= 0 && value <= 4) c.l2_hint = uint32_t(value);
   else if (n == "item_l2_hint" && value >= 0 && value <= 3) c.item_l2_hint = uint32_t(value);
   else if (n == "item_qpf" && value >= 0 && value <= 6) c.item_qpf = uint32_t(value);
+  else if (n == "item_cnode" && value >= 0 && value <= 2) { c.item_cnode = uint32_t(value); invalidate_buckets(t); }
   else if (n == "item_cdir" && value >= 0 && value <= 2) { c.item_cdir = uint32_t(value); invalidate_buckets(t); }
   else {
     set_error("bad parameter %s = %lld", name, (long long)value);

@@ -164,6 +164,67 @@ __global__ void bk_cdir(const K* __restrict__ M, BucketDir* __restrict__ bd, uin
   }
 }
 
+// Compact nodes of the compressed directory's level (implicit, u64 keys, F = 16; ItemDir::
+// cnode): one CTA per bucket.  With M'(x) = (x - lo) >> sh of the bucket (0 below lo), node u
+// becomes 32 B: u32 b0 = M'(sep_0), then for slots 1..14 the u16 (M'(sep_i) - b0) >> nsh, or
+// 0xFFFF for a MAX slot (slot 15 is always MAX, reading R3); nsh is the bucket's shift that
+// keeps every real entry <= 0xFFFE.  Truncation is monotone, so the child the search counts
+// from it is the true child or an earlier one (a tie), never a later one; the walk's FIX
+// moves on from an early leaf line (descend_and_store).  A DRAM transfer of 128 B brings
+// four of them instead of one node.
+__global__ void bk_cnode(const uint64_t* __restrict__ lvl, BucketDir* __restrict__ bd,
+                         uint4* __restrict__ out) {
+  constexpr uint64_t MAXK = ~0ull;
+  __shared__ uint32_t s_w[32];
+  __shared__ uint32_t s_nsh;
+  BucketDir* d = bd + blockIdx.x;
+  const uint64_t u0 = d->u0, lo = d->lo;
+  const uint32_t cnt = d->cnt, sh = d->sh;
+  auto mp = [&](uint64_t x) -> uint32_t {
+    if (x <= lo) return 0u;
+    const uint64_t y = (x - lo) >> sh;
+    return y > 0xFFFFFFFFull ? 0xFFFFFFFFu : uint32_t(y);
+  };
+  uint32_t w = 0;
+  for (uint32_t i = threadIdx.x; i < cnt; i += blockDim.x) {
+    const uint64_t* nd = lvl + (u0 + i) * 16;
+    if (nd[0] == MAXK) continue;
+    const uint32_t b0 = mp(nd[0]);
+    for (int j = 14; j >= 1; --j)
+      if (nd[j] != MAXK) {
+        w = max(w, mp(nd[j]) - b0);
+        break;
+      }
+  }
+  for (int o = 16; o > 0; o >>= 1) w = max(w, __shfl_xor_sync(0xffffffffu, w, o));
+  if ((threadIdx.x & 31) == 0) s_w[threadIdx.x >> 5] = w;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t m = 0;
+    for (uint32_t x = 0; x < blockDim.x / 32; ++x) m = max(m, s_w[x]);
+    uint32_t nsh = 0;
+    while ((m >> nsh) > 0xFFFEu) ++nsh;
+    s_nsh = nsh;
+    d->nsh = nsh;
+  }
+  __syncthreads();
+  const uint32_t nsh = s_nsh;
+  for (uint32_t i = threadIdx.x; i < cnt; i += blockDim.x) {
+    const uint64_t* nd = lvl + (u0 + i) * 16;
+    const uint32_t b0 = nd[0] == MAXK ? 0xFFFFFFFFu : mp(nd[0]);
+    uint32_t wv[8];
+    wv[0] = b0;
+    for (int j = 1; j <= 14; ++j) {
+      const uint32_t e = nd[j] == MAXK ? 0xFFFFu : ((mp(nd[j]) - b0) >> nsh);
+      const int word = (j + 1) / 2, half = (j + 1) & 1;  // u16 slot j at byte 4 + 2 (j - 1)
+      if (half == 0) wv[word] = e; else wv[word] |= e << 16;
+    }
+    uint4* o = out + (u0 + i) * 2;
+    o[0] = make_uint4(wv[0], wv[1], wv[2], wv[3]);
+    o[1] = make_uint4(wv[4], wv[5], wv[6], wv[7]);
+  }
+}
+
 // Item directory (regular): M[c * NI + t] = true max key of key line t of the
 // last-level node of chain leaf c = the key of entry min(count, (t+1)*KPL*P) - 1
 // (KPL separators per 64 B key line, each covering one leaf line of P entries);
@@ -922,6 +983,35 @@ int prepare_splitters(const hbt_tree* t, cudaStream_t s, BucketState& bs, uint32
       HBT_CUDA_TRY(cudaMemcpyAsync(bs.d_bd, h.data(), B * sizeof(BucketDir), cudaMemcpyHostToDevice, s));
       bk_cdir<K><<<B, 256, 0, s>>>((const K*)bs.d_M, (BucketDir*)bs.d_bd, bs.d_E16, bs.d_T16);
       HBT_CUDA_TRY(cudaGetLastError());
+      // compact copies of the directory level's nodes where that level is read as whole
+      // nodes from HBM (c4: the last inner level, 4 GB -> 1 GB)
+      bs.cnode = false;
+      // (the last inner level only: a tie there puts the walk at most a few leaf lines early)
+      if (t->form == HBT_IMPLICIT && sizeof(K) == 8 && t->F == 16 && t->H >= 1 && bs.level == t->H - 1 &&
+          t->cfg.item_cnode) {
+        bool full = t->cfg.item_cnode == 2;
+        if (!full) {
+          uint64_t cum = 0;
+          const uint64_t budget = t->cfg.l2_levels_bytes ? t->cfg.l2_levels_bytes : (32ull << 20);
+          for (uint32_t x = bs.level; x < t->H; ++x) cum += t->nodes[x] * uint64_t(16 * 8 + 32);
+          full = cum > budget;
+        }
+        if (full) {
+          const uint64_t bytes = t->nodes[bs.level] * 32;
+          if (bs.cnode_cap < bytes) {
+            cudaFree(bs.d_cnode);
+            bs.d_cnode = nullptr;
+            bs.cnode_cap = 0;
+            HBT_CUDA_TRY(cudaMalloc(&bs.d_cnode, bytes));
+            bs.cnode_cap = bytes;
+          }
+          bk_cnode<<<B, 256, 0, s>>>(reinterpret_cast<const uint64_t*>(static_cast<const uint8_t*>(t->d_inner) +
+                                                                         t->offset[bs.level] * 128),
+                                     (BucketDir*)bs.d_bd, reinterpret_cast<uint4*>(bs.d_cnode));
+          HBT_CUDA_TRY(cudaGetLastError());
+          bs.cnode = true;
+        }
+      }
     }
   }
   HBT_CUDA_TRY(cudaStreamSynchronize(s));
@@ -1050,6 +1140,7 @@ int bucketed_t(const hbt_tree* t, const void* q, uint64_t m, uint64_t* pf, void*
         d.E16 = bs.d_E16;
         d.T16 = bs.d_T16;
         d.cap = bs.cap16;
+        if (bs.cnode) d.cnode = bs.d_cnode;
       }
       rc = t->form == HBT_IMPLICIT ? implicit_search_items(t, qs, m, pf_s, v_s, d, s)
                                    : regular_search_items(t, qs, m, pf_s, v_s, d, s);
@@ -1239,6 +1330,7 @@ static void bucket_state_free(BucketState& b) {
   cudaFree(b.d_M);
   cudaFree(b.d_bd);
   cudaFree(b.d_E16);
+  cudaFree(b.d_cnode);
   b = BucketState{};
 }
 

@@ -90,6 +90,8 @@ struct SearchConfig {
                                  // 4 = auto: leaf lines evict-first iff the I-segment fits in L2 / 4
   uint32_t item_l2_hint = 1;     // implicit bucketed item search (c4 item search 10.96 -> 9.50 ms)
   uint32_t item_qpf = 1;         // see ItemDir::qpf
+  uint32_t item_cnode = 1;       // compact 32 B directory-level nodes (u64, F = 16): 0 = off, 1 = when that level
+                                 // is read as whole nodes (beyond the L2 budget), 2 = always
   uint32_t item_cdir = 1;        // item directory in the compressed per-bucket form (ItemDir::bd): 0 = never,
                                  // 1 = where it reaches a deeper level (regular: always fits-permitting),
                                  // 2 = always (implicit: even at the same level)
@@ -126,6 +128,9 @@ struct ItemDir {
   const uint16_t* E16 = nullptr;
   const uint16_t* T16 = nullptr;
   bool fix = false;  // single ties of the truncated maxima resolved by the walk
+  // compact 32 B copies of the directory level's nodes (u64 keys, F = 16; bk_cnode): u32
+  // M'(sep_0) + 14 u16 (M'(sep_i) - M'(sep_0)) >> nsh (0xFFFF = MAX slot); null = off
+  const uint8_t* cnode = nullptr;
   uint32_t qpf = 0;  // compressed-directory items: each lane prefetches its query qpf rounds after the next into
                      // the L2 (0 = off; 1 measured best, 2-4 slower: profiles/r02s_item_query_prefetch_ab.jsonl)
 };
@@ -142,7 +147,7 @@ struct BucketDir {
   uint32_t top;    // (M[u0 + cnt - 1] - lo) >> sh
   uint32_t ssh;    // prefix-table slice p holds M' in [p << ssh, (p + 1) << ssh)
   uint32_t esh;    // entry = (M' >> esh) & 0xFFFF (ssh - 16, or 0)
-  uint32_t pad;
+  uint32_t nsh;    // compact directory-level nodes (ItemDir::cnode): entry = (M'(sep) - M'(sep_0)) >> nsh
 };
 
 // Owner side of the fused sharded exchange (sharded_fused.cu): the bucketed search's
@@ -177,6 +182,9 @@ struct BucketState {
   uint16_t* d_T16 = nullptr;
   uint64_t E16_cap = 0;          // bytes allocated
   uint32_t cap16 = 0;            // largest bucket's unit count, rounded up to 8
+  uint8_t* d_cnode = nullptr;    // compact directory-level nodes (ItemDir::cnode), 32 B per unit
+  uint64_t cnode_cap = 0;        // bytes allocated
+  bool cnode = false;            // in use
   cudaEvent_t ev[6] = {};        // phase boundaries of the last timed bucketed search
   bool timed = false;
   uint32_t launches = 0;

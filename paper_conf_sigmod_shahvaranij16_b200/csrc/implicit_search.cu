@@ -661,8 +661,38 @@ implicit_search_cdir_kernel(const uint8_t* __restrict__ inner, const uint8_t* __
       }
       const uint32_t a = lower_bound16(s_E, s_T, cnt, myq, K(s_bd[x].lo), s_bd[x].sh, s_bd[x].top, s_bd[x].ssh,
                                        s_bd[x].esh, gM + u0, d.fix);
+      uint32_t mynode = uint32_t(u0) + (a < cnt ? a : cnt - 1);
+      uint32_t lvl0 = d.level;
+      if constexpr (sizeof(K) == 8 && F == 16) {
+        if (d.cnode) {
+          // the directory unit's compact node (32 B, one 256-bit load per lane): child =
+          // 0 if M'(q) <= b0, else 1 + #{slots 1..14 with entry < (M'(q) - b0) >> nsh}
+          const uint64_t lo = s_bd[x].lo;
+          const uint32_t sh = s_bd[x].sh, nsh = s_bd[x].nsh;
+          L256<K> cn;
+          ld32(cn, d.cnode + uint64_t(mynode) * 32);
+          const uint64_t dq = myq <= lo ? 0ull : (uint64_t(myq) - lo) >> sh;
+          const uint32_t qp = dq > 0xFFFFFFFFull ? 0xFFFFFFFFu : uint32_t(dq);
+          const uint32_t b0 = uint32_t(cn.u[0]);
+          uint32_t c = 0;
+          if (qp > b0) {
+            const uint32_t t16 = min((qp - b0) >> nsh, 0xFFFFu);
+            const uint32_t qq = t16 * 0x10001u;
+            // u16 slots 1..14: two per 32-bit word, words 1..7 (word 0 is b0)
+            const uint32_t cmp = __popc(__vcmpltu2(uint32_t(cn.u[0] >> 32), qq)) +
+                                 __popc(__vcmpltu2(uint32_t(cn.u[1]), qq)) +
+                                 __popc(__vcmpltu2(uint32_t(cn.u[1] >> 32), qq)) +
+                                 __popc(__vcmpltu2(uint32_t(cn.u[2]), qq)) +
+                                 __popc(__vcmpltu2(uint32_t(cn.u[2] >> 32), qq)) +
+                                 __popc(__vcmpltu2(uint32_t(cn.u[3]), qq)) +
+                                 __popc(__vcmpltu2(uint32_t(cn.u[3] >> 32), qq));
+            c = 1 + cmp / 16;
+          }
+          mynode = mynode * 16 + c;
+          lvl0 = d.level + 1;
+        }
+      }
       if (r == nr - 1) done_with_dir();
-      const uint32_t mynode = uint32_t(u0) + (a < cnt ? a : cnt - 1);
       K q[QPG];
       uint32_t node[QPG];
 #pragma unroll
@@ -671,7 +701,7 @@ implicit_search_cdir_kernel(const uint8_t* __restrict__ inner, const uint8_t* __
         q[j] = __shfl_sync(0xffffffffu, myq, src);
         node[j] = __shfl_sync(0xffffffffu, mynode, src);
       }
-      descend_and_store<K, F, QPG, true, true>(inner, inner_idx, leaf, lt, d.level, q, node, g, k, gmask, base,
+      descend_and_store<K, F, QPG, true, true>(inner, inner_idx, leaf, lt, lvl0, q, node, g, k, gmask, base,
                                                p1 + 1, n, d.pos_base, out_pf, out_v,
                                                d.fix ? uint32_t(min((u0 + cnt) * d.span, d.U) - 1) : 0u);
     }

@@ -154,14 +154,16 @@ def test_compressed_directory_ties(hbt, layout, F, nsmall, slice_bytes):
         t.set_param("bucket", 1)
         t.set_param("item_cdir", 2)
         t.set_param("bucket_slice", slice_bytes)
-        for rounds, leaf256, full256, l2b in ((0, 1, 1, 0), (0, 1, 1, 4096), (1, 1, 1, 4096), (0, 0, 1, 0),
-                                              (0, 1, 0, 4096), (1, 0, 0, 0)):
+        for rounds, leaf256, full256, l2b, cnode in ((0, 1, 1, 0, 1), (0, 1, 1, 4096, 1), (1, 1, 1, 4096, 1),
+                                                     (0, 0, 1, 0, 1), (0, 1, 0, 4096, 1), (1, 0, 0, 0, 1),
+                                                     (0, 1, 1, 0, 2), (1, 1, 1, 4096, 2)):
             t.set_param("item_rounds", rounds)
             t.set_param("leaf256", leaf256)
             t.set_param("full256", full256)
             t.set_param("l2_levels_bytes", l2b)
+            t.set_param("item_cnode", cnode)  # 2: compact last-level nodes forced (their own ties)
             pf, val = gpu_search(t, q, width)
-            cfg = (layout, F, width, slice_bytes, rounds, leaf256, full256, l2b)
+            cfg = (layout, F, width, slice_bytes, rounds, leaf256, full256, l2b, cnode)
             assert np.array_equal(pf, epf), (cfg, np.nonzero(pf != epf)[0][:5])
             assert np.array_equal(val, ev), cfg
         t.close()

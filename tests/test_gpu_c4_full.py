@@ -151,12 +151,14 @@ def test_c4_recipe_last_inner_level_directory_ties(slice_bytes):
     dq = g.stratified_queries(m, n, sq, sk)
     # hits, plus misses just above each hit (lower bound = next key)
     q = torch.cat([dq, dq + 1])
-    pf, val = t.search(q)
-    torch.cuda.synchronize()
     qh = q.cpu().numpy().view(np.uint64)
     epf, ev = closed_form(qh, n, sk, sv)
-    got = pf.cpu().numpy().view(np.uint64)
-    bad = np.nonzero(got != epf)[0]
-    assert bad.size == 0, (bad.size, qh[bad[:4]], got[bad[:4]], epf[bad[:4]])
-    assert np.array_equal(from_dev(val, 8), ev)
+    for cnode in (1, 0):  # compact last-inner-level nodes (default, on at this size) and the full nodes
+        t.set_param("item_cnode", cnode)
+        pf, val = t.search(q)
+        torch.cuda.synchronize()
+        got = pf.cpu().numpy().view(np.uint64)
+        bad = np.nonzero(got != epf)[0]
+        assert bad.size == 0, (cnode, bad.size, qh[bad[:4]], got[bad[:4]], epf[bad[:4]])
+        assert np.array_equal(from_dev(val, 8), ev)
     t.close()
