@@ -49,12 +49,15 @@ def test_bucketed_edge_suite(hbt, layout, width, F, items, cap, leaf256, dir32):
         t.set_param("bucket_cap", cap)
         t.set_param("leaf256", leaf256)
         t.set_param("item_cdir", dir32)
-        for slice_bytes in (1, 4096, 1 << 16):  # 1 B: one bucket per unit up to the 1024 cap
+        for slice_bytes, cnode in ((1, 1), (4096, 1), (1 << 16, 1), (4096, 2), (1 << 16, 2)):
+            # 1 B: one bucket per unit up to the 1024 cap; cnode 2: compact last-inner-level
+            # nodes forced wherever the directory sits on the last inner level
             t.set_param("bucket_slice", slice_bytes)
+            t.set_param("item_cnode", cnode)
             pf, val = gpu_search(t, q, width)
-            assert np.array_equal(pf, epf), (layout, n, F, width, slice_bytes, items, cap,
+            assert np.array_equal(pf, epf), (layout, n, F, width, slice_bytes, cnode, items, cap,
                                              np.nonzero(pf != epf)[0][:5])
-            assert np.array_equal(val, ev), (layout, n, F, width, slice_bytes, items, cap)
+            assert np.array_equal(val, ev), (layout, n, F, width, slice_bytes, cnode, items, cap)
         t.close()
 
 
