@@ -246,3 +246,30 @@ def test_c3_full_size_bench_launch(hbt):
     assert bad.size == 0, (bad.size, bad[:5])
     assert np.array_equal(val, ev)
     t.close()
+
+
+@pytest.mark.parametrize("slice_bytes", [1 << 30, 12 << 20, 5 << 20])
+def test_compact_last_level_nodes(hbt, slice_bytes):
+    """Compact last-inner-level nodes (item_cnode; bucketed implicit u64 search, F = 16)
+    on a tree whose compressed directory sits on the last inner level (1, 2 or 3 buckets
+    of a 2^20-key tree: more leaf lines per bucket than the 16-bit directory holds):
+    random keys with duplicates and MAX as a key, hits, misses, 0, MAX and neighbours of
+    keys, compact nodes off / auto / forced against the oracle."""
+    rng = np.random.default_rng(4242)
+    n = 1 << 20
+    k, v = gen_keys(n, 8, rng, dup=True, with_max=True)
+    o = _oracle("implicit", k, v, 16, 8)
+    t = gpu_build(hbt, k, v, 16, 8, layout="implicit")
+    q = query_set(k, 8, rng, 1 << 18)
+    q = np.concatenate([q, k[::5], k[::7] + np.uint64(1), k[::9] - np.uint64(1),
+                        np.array([0, kmax(8)], dtype=np.uint64)])
+    epf, ev = o.search(q, nthreads=oracle.default_threads())
+    t.set_param("bucket", 1)
+    t.set_param("bucket_slice", slice_bytes)
+    t.set_param("l2_levels_bytes", 4096)  # the last inner level read as whole nodes: compact form in auto mode
+    for cnode in (0, 1, 2):
+        t.set_param("item_cnode", cnode)
+        pf, val = gpu_search(t, q, 8)
+        assert np.array_equal(pf, epf), (slice_bytes, cnode, np.nonzero(pf != epf)[0][:5])
+        assert np.array_equal(val, ev), (slice_bytes, cnode)
+    t.close()
