@@ -74,6 +74,7 @@ def test_random_knob_parity(hbt, case):
     knobs["item_l2_hint"] = int(hrng.integers(0, 4))
     knobs["item_rounds"] = int(hrng.choice([0, 1, 3, 16]))
     knobs["item_qpf"] = int(hrng.choice([0, 1, 2]))
+    knobs["item_cnode"] = int(hrng.choice([0, 1, 2]))
     for name, val in knobs.items():
         t.set_param(name, val)
     q = _queries(k, width, rng, int(rng.choice([1, 31, 1000, 40000])))
