@@ -560,7 +560,9 @@ implicit_search_items_kernel(const uint8_t* __restrict__ inner, const uint8_t* _
 // parity) and starts its directory copy, which completes `full`.  A warp starts the next
 // item as soon as `full` completes -- it does not wait for the other warps' last walks
 // (leaf reads) of the previous item (c4 item search -1..-5 %, c5 -3 %,
-// profiles/r02s_item_pipe_ab.jsonl).
+// profiles/r02s_item_pipe_ab.jsonl).  With ItemDir::cnode (u64, F = 16, the directory on the
+// last inner level) a lane reads its unit's 32 B compact node (bk_cnode, bucketed.cu)
+// instead of the 128 B node and goes straight to the leaf line (c4 item search -15 %).
 template <typename K, int F, int THREADS>
 __global__ void __launch_bounds__(THREADS)
 implicit_search_cdir_kernel(const uint8_t* __restrict__ inner, const uint8_t* __restrict__ inner_idx,
