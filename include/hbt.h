@@ -244,6 +244,9 @@ HBT_API int hbt_export(const hbt_tree* t, uint32_t segment, void* dst, uint64_t 
  *                 keys and fits (default), 2 = always where it fits
  *   "item_qpf"    compressed-directory item searches: each lane prefetches its query this many
  *                 rounds beyond the next into the L2 (0 = off, 1 = default; 0..6)
+ *   "item_cnode"  compact 32 B copies of the last inner level's nodes for the bucketed implicit
+ *                 search (u64 keys, F = 16, directory on the last inner level): 0 = off,
+ *                 1 = where that level is read as whole nodes (default), 2 = always
  * Variants measured slower were removed (DESIGN.md §8 keeps their numbers).  Unknown
  * names or out-of-range values return HBT_EINVAL. */
 HBT_API int hbt_set_param(hbt_tree* t, const char* name, int64_t value);
