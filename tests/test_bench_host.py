@@ -61,3 +61,28 @@ def test_c4_oracle_sample_matches_the_stratified_closed_form(monkeypatch):
     assert np.array_equal(val, gen.mix64(i ^ np.uint64(sv)))
     assert np.array_equal(k[i.astype(np.int64)], q)
     assert sk != sv
+
+
+def test_c5_splits_its_batch_over_the_replicas():
+    """BASELINE configs[4] 'query-batch split at 8 GPUs': c5's 2^26 queries are divided
+    among the ranks (strong scaling); c1-c3 keep a full batch per rank (weak)."""
+    for world in (1, 2, 8):
+        c5 = bench.bench_config(_args(config="c5"), world)
+        assert c5["queries_total"] == 1 << 26 and c5["queries_per_rank"] == (1 << 26) // world
+        c3 = bench.bench_config(_args(config="c3"), world)
+        assert c3["queries_total"] == world * (1 << 26) and c3["queries_per_rank"] == 1 << 26
+
+
+def test_roofline_model_bytes_of_the_c4_item_search():
+    """tools/roofline.py's bucketed model as bench.py calls it (the line's algorithmic bytes,
+    DESIGN.md §6): query 8 + record 16 + distinct leaf lines touched by 2^28 uniform queries
+    (64 B each) + one pass over the directory keys at leaf-line granularity (8 B per line):
+    90.4 B/q for the c4 geometry."""
+    from tools import roofline
+    info = {"width": 8, "fanout": 16, "layout": 0, "n_distinct": 1 << 31, "height": 8, "smem_levels": 4,
+            "level_nodes": [1, 2, 32, 512, 8192, 131072, 2097152, 33554432], "leaf_lines": 1 << 29}
+    m = 1 << 28
+    b = roofline.model_bucketed(info, m)["hbm_bytes_per_query"]
+    lines = (1 << 29) * (1 - np.exp(-m / (1 << 29))) * 64 / m
+    assert abs(b - (24 + lines + (1 << 29) * 8 / m)) < 1e-6, b
+    assert abs(b - 90.36) < 0.01
