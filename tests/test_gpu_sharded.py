@@ -110,14 +110,16 @@ def test_nccl_path_one_rank(hbt, exchange, g1_direct):
     comm.close()
 
 
-@pytest.mark.parametrize("bucket,chunks", [(0, 1), (1, 1), (0, 2), (1, 3), (1, 4)])
-def test_fused_exchange_two_processes_one_gpu(bucket, chunks):
+@pytest.mark.parametrize("bucket,chunks,cnode", [(0, 1, 0), (1, 1, 0), (0, 2, 0), (1, 3, 0), (1, 4, 0), (1, 1, 1),
+                                                (1, 2, 1)])
+def test_fused_exchange_two_processes_one_gpu(bucket, chunks, cnode):
     """Two ranks (processes) on one GPU through the host-callback communicator:
     CUDA IPC windows, device flag barriers, count rows published by peer stores and
     queries put into the owner's window (exchange = 0); bucket = 1: the owner's
     bucketed gather stores results straight into the requester's window; chunks > 1:
     the batch is exchanged in chunks, the owner searching chunk c on a second stream
-    while chunk c+1 is put.  Seven
+    while chunk c+1 is put; cnode = 1: a 2^21-key tree whose owner searches read the compact
+    last-inner-level nodes.  Seven
     batches of growing and shrinking size per rank, each rank's results vs the
     unsharded oracle (tools/two_rank_one_gpu.py)."""
     import os
@@ -131,7 +133,8 @@ def test_fused_exchange_two_processes_one_gpu(bucket, chunks):
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nproc-per-node", "2",
                         "--master-addr", "127.0.0.1", "--master-port", str(port),
-                        os.path.join(root, "tools", "two_rank_one_gpu.py"), "0", str(bucket), str(chunks)],
+                        os.path.join(root, "tools", "two_rank_one_gpu.py"), "0", str(bucket), str(chunks),
+                        str(cnode)],
                        capture_output=True, text=True, timeout=600, cwd=root)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
     assert r.stdout.count("ok=True") == 2, r.stdout[-2000:]

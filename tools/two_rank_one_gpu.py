@@ -22,11 +22,14 @@ def main():
     exchange = int(sys.argv[1]) if len(sys.argv) > 1 else 0
     bucket = int(sys.argv[2]) if len(sys.argv) > 2 else 2  # 1: owner search bucketed (fused remote gather)
     chunks = int(sys.argv[3]) if len(sys.argv) > 3 else 2  # exchange chunks (put of c+1 overlaps search of c)
+    # 1: a larger tree with one bucket per shard, so the owner's item directory sits on the last
+    # inner level and the search reads its compact nodes (item_cnode forced)
+    cnode = int(sys.argv[4]) if len(sys.argv) > 4 else 0
     dist.init_process_group("gloo")
     rank, world = dist.get_rank(), dist.get_world_size()
     torch.cuda.set_device(0)
     comm = hbt.Comm.from_torch_host() if exchange == 0 else hbt.Comm.from_torch()
-    n = 200000
+    n = 1 << 21 if cnode else 200000
     allk = gen.stratified_keys(n, 7)
     allv = gen.values(n, 8, 9)
     lo, hi = hbt.shard_plan(n, world, rank)
@@ -38,7 +41,10 @@ def main():
     if exchange == 0:
         t.set_param("exchange_chunks", chunks)
     if bucket == 1:
-        t.set_param("bucket_slice", 4096)
+        t.set_param("bucket_slice", 1 << 30 if cnode else 4096)
+    if cnode:
+        t.set_param("l2_levels_bytes", 4096)
+        t.set_param("item_cnode", 2)
     full = oracle.ITree.from_pairs(allk, allv, 16, 8)
     ok = True
     # batch sizes grow (window regrowth, a collective re-export) and shrink; several
